@@ -1,0 +1,384 @@
+"""bench.py — SEPO bulk insert-and-combine on B200 (BASELINE.json metric / configs).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--ratio 4] [--impl ours|reference]
+
+A step = one whole SEPO job (every SURVEY §8(a) row): reset the table, insert all records of the
+workload (input resident in HBM), re-probe + compact + evict + re-issue until nothing is
+postponed, and transfer the final generation to pinned host memory (P:L227 timing scope).
+Default workload: C2 (word count, 8 GiB Zipf(1.0) text = 1.1e9 words, V = 2^22) with the device
+budget capped at F/4, i.e. the table is 4x the budget (BASELINE.json configs[1]).
+
+Prints ONE JSON line (rank 0). `value` is input GB/s (CSR bytes the job consumes: key bytes +
+8 B offsets [+ values]) over the device-timed steps; `e2e` is the same job through sepo_run with
+pinned HOST buffers (H2D of the input + job + result assembly on the host). The oracle
+(oracle/, test infrastructure) is run only by the cpu_baseline leg and by --impl reference.
+"""
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+BASE = json.load(open(os.path.join(ROOT, "BASELINE.json")))
+METRIC = BASE["metric"]
+MiB, GiB = 1 << 20, 1 << 30
+
+CONFIG_TEXT = {
+    "C1": BASE["configs"][0], "C2": BASE["configs"][1], "C3": BASE["configs"][2], "C4": BASE["configs"][3],
+    "C5u": BASE["configs"][4] + " [uniform keys]", "C5z": BASE["configs"][4] + " [Zipf(1.2) keys]",
+}
+
+
+def next_pow2(x):
+    p = 1
+    while p < x:
+        p <<= 1
+    return p
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {"hbm_gbs": 6650.0, "_fallback": True}
+
+
+class Job:
+    """One workload at one budget ratio (table size / device budget)."""
+    _footprint_cache = {}
+
+    def __init__(self, cfg, ratio=4.0, page_bytes=None, scale=1.0):
+        import gen
+        self.cfg, self.ratio, self.scale = cfg, float(ratio), scale
+        self.stream = gen.config(cfg, scale=scale)
+        s = self.stream
+        self.page_bytes = page_bytes or (16384 if s.family != gen.GEN_URLS else 65536)
+        self.distinct = s.n_ranks
+        self.nb_full = max(1 << 16, next_pow2(self.distinct))
+        self._inputs = None
+        self.kw = {}
+        import paper_conf_ipps_mokhtaris17_b200 as sepo
+        self.sepo = sepo
+        if s.val == "u64":
+            self.kw = dict(mode=sepo.COMBINE, fixed_key_width=8, fixed_val_width=8)
+        elif s.val == "doc":
+            self.kw = dict(mode=sepo.GROUP, fixed_val_width=4)
+        else:
+            self.kw = dict(mode=sepo.COMBINE)
+
+    def inputs(self):
+        if self._inputs is None:
+            k, o, v = self.stream.device()
+            if self.stream.val == "u64":
+                o = None
+            self._inputs = (k, o, v)
+        return self._inputs
+
+    def csr_bytes(self):
+        k, o, v = self.inputs()
+        b = k.numel()
+        if o is not None:
+            b += 8 * (o.numel() - 1)
+        if v is not None:
+            b += v.numel()
+        return b
+
+    def footprint(self):
+        """F (SURVEY §8c reading 23): directory + pages an unconstrained run touches."""
+        key = (self.cfg, self.scale, self.page_bytes)
+        if key not in Job._footprint_cache:
+            sepo = self.sepo
+            t = sepo.Table(sepo.budget_for(self.nb_full, self.page_bytes, max(64, (self.csr_bytes() * 2) // self.page_bytes + 64)),
+                           self.nb_full, self.page_bytes, **self.kw)
+            k, o, v = self.inputs()
+            passes = t.run(k, o, v)
+            assert passes == 1
+            pages = t.stats()["pages_used_max"]
+            t.close()
+            Job._footprint_cache[key] = (pages, 4 * self.nb_full + pages * self.page_bytes)
+        return Job._footprint_cache[key]
+
+    def table_params(self):
+        pages_F, F = self.footprint()
+        if self.ratio <= 1.0:
+            nb = self.nb_full
+            pages = int(np.ceil(pages_F / self.ratio)) if self.ratio < 1 else pages_F + 8
+        else:
+            nb = max(1 << 16, next_pow2(int(self.distinct / self.ratio)))
+            pages = max(8, int((F / self.ratio - 4 * nb) // self.page_bytes))
+        return nb, pages, F
+
+    def table(self, **extra):
+        sepo = self.sepo
+        nb, pages, F = self.table_params()
+        kw = dict(self.kw)
+        kw.update(extra)
+        _, F = self.footprint()
+        arena = int(F * 1.25) + 64 * MiB
+        return sepo.Table(sepo.budget_for(nb, self.page_bytes, pages), nb, self.page_bytes, host_arena_bytes=arena, **kw)
+
+
+def make_job(cfg, ratio=4.0, **kw):
+    return Job(cfg, ratio, **kw)
+
+
+# ---------------------------------------------------------------- clocks during the timed region
+class ClockSampler:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index=0):
+        self.rows, self.proc = [], None
+        self.gpu = gpu_index
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.th = threading.Thread(target=self._read, daemon=True)
+            self.th.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+        sm = [float(r[1]) for r in self.rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) >= 9 and r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            if len(r) >= 9:
+                for nm, v in zip(names, r[5:9]):
+                    if v.strip().lower() == "active":
+                        reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ---------------------------------------------------------------- the CPU oracle legs
+def oracle_sample(job, max_records, budget_s=15.0):
+    """Time the oracle (as it stands) on the first records of the same stream. -> (GB/s, recs/s, desc)"""
+    import oracle
+    s = job.stream
+    chunk = min(max_records, 1 << 23)
+    done, t_ins, bytes_in = 0, 0.0, 0
+    h = oracle.Combine() if s.val != "doc" else oracle.Group()
+    while done < max_records and t_ins < budget_s:
+        cnt = min(chunk, s.n - done, max_records - done)
+        if cnt <= 0:
+            break
+        k, o, v = s.host(done, cnt)
+        t0 = time.perf_counter()
+        if s.val == "doc":
+            h.add(k, o, v, val_width=4)
+        elif s.val == "u64":
+            h.add(k, o, v, 8)
+        else:
+            h.add(k, o)
+        t_ins += time.perf_counter() - t0
+        bytes_in += len(k) + (8 * cnt if s.family != 2 else 0) + (len(v) if v is not None else 0)
+        done += cnt
+    return bytes_in / t_ins / 1e9, done / t_ins, done, t_ins
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    job = Job(args.config, args.ratio)
+    for _ in range(args.warmup):
+        oracle_sample(job, 1 << 20, budget_s=1.0)
+    vals, recs, times = [], [], []
+    for _ in range(args.steps):
+        gbs, rps, n, t = oracle_sample(job, args.ref_records, budget_s=args.ref_seconds)
+        vals.append(gbs); recs.append(n); times.append(t)
+    v = float(np.median(vals))
+    line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "GB/s", "n_gpus": args.gpus, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": float(np.median(times)) * 1e3, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+            "config": {"workload": CONFIG_TEXT[args.config], "ratio_table_over_budget": args.ratio},
+            "cpu_baseline": {"value": v, "unit": "GB/s", "cores": 1, "kind": "oracle",
+                             "sample": f"first {int(np.median(recs))} records of {args.config} per step (oracle/oracle.cpp "
+                                       f"std::unordered_map, single thread; generation excluded)"},
+            "e2e": {"value": v, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- our arm
+def timed_steps(job, t, steps, stream):
+    import torch
+    k, o, v = job.inputs()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ins_ms, launches, recs_ins, kb_ins, vb_ins = 0.0, 0, 0, 0, 0
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(steps):
+        t.reset()
+        t.run(k, o, v)
+        st = t.stats()
+        ins_ms += st["t_insert_ms"]
+        launches += st["kernel_launches"]
+        recs_ins += st["records_inserted"]
+        kb_ins += st["key_bytes_inserted"]
+        vb_ins += st["val_bytes_inserted"]
+    e1.record(stream)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1), dict(insert_ms=ins_ms, launches=launches, recs=recs_ins, kb=kb_ins, vb=vb_ins, last=st)
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    job = Job(args.config, args.ratio)
+    stream = torch.cuda.current_stream()
+    job.inputs()
+    nb, pages, F = job.table_params()
+    t = job.table()
+    k, o, v = job.inputs()
+    for _ in range(max(args.warmup, 3)):
+        t.reset()
+        t.run(k, o, v)
+    sampler = ClockSampler(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    sampler.start()
+    ms, info = timed_steps(job, t, args.steps, stream)
+    clocks = sampler.stop()
+    st = info["last"]
+    if world > 1:
+        tt = torch.tensor([ms], device="cuda")
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms = float(tt.item())
+    csr = job.csr_bytes()
+    n = job.stream.n
+    value = world * csr * args.steps / (ms / 1e3) / 1e9
+    recs_per_s = world * n * args.steps / (ms / 1e3)
+
+    # roofline of the dominant kernel (insert, a1..a7): algorithmic bytes = CSR bytes of every
+    # batch it was handed (key bytes + 8 B offset [+ value bytes]) over its CUDA-event time
+    pk = peaks()
+    alg = info["kb"] + (8 * info["recs"] if k is not None and o is not None else 0) + info["vb"]
+    achieved = alg / (info["insert_ms"] / 1e3) / 1e9
+    roof = {"bound": "hbm", "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
+            "frac": achieved / pk["hbm_gbs"], "traffic": args.traffic, "kernel": "sepo::insert_kernel<0>",
+            "insert_share_of_step": info["insert_ms"] / ms,
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if not pk.get("_fallback") else "fallback 6.65 TB/s"}
+
+    # end to end through sepo_run with pinned HOST buffers (H2D + job + host result assembly)
+    e2e = None
+    if args.e2e_steps > 0:
+        hk = torch.empty(k.numel(), dtype=torch.uint8, pin_memory=True); hk.copy_(k)
+        ho = torch.empty(o.numel(), dtype=torch.int64, pin_memory=True).copy_(o) if o is not None else None
+        hv = torch.empty(v.numel(), dtype=torch.uint8, pin_memory=True).copy_(v) if v is not None else None
+        # warm (staging buffers are allocated once)
+        t.reset(); t.run(hk, ho, hv); t.export(copy=False)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        d2h = 0
+        for _ in range(args.e2e_steps):
+            t.reset()
+            t.run(hk, ho, hv)
+            res = t.export(copy=False)
+            d2h += t.stats()["bytes_evicted"]
+        el = time.perf_counter() - t0
+        if world > 1:
+            tt = torch.tensor([el], device="cuda")
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            el = float(tt.item())
+        e2e = {"value": world * csr * args.e2e_steps / el / 1e9, "unit": "GB/s",
+               "h2d_bytes_per_step": csr, "d2h_bytes_per_step": d2h // args.e2e_steps,
+               "kv_inserts_per_s": world * n * args.e2e_steps / el,
+               "note": "sepo_run on pinned host buffers; includes H2D, all passes, page D2H, host result assembly"}
+
+    # slowdown curve (M3): job time at table/budget = 0.5 .. 4 relative to 0.5
+    curve = None
+    if args.curve and rank == 0:
+        curve = {}
+        base = None
+        for r in (0.5, 1.0, 2.0, 3.0, 4.0):
+            j2 = Job(args.config, r)
+            j2._inputs = job._inputs
+            t2 = j2.table()
+            for _ in range(2):
+                t2.reset(); t2.run(k, o, v)
+            m2, i2 = timed_steps(j2, t2, 2, stream)
+            ms2 = m2 / 2
+            if base is None:
+                base = ms2
+            curve[str(r)] = {"ms": ms2, "slowdown": ms2 / base, "passes": i2["last"]["passes"]}
+            t2.close()
+
+    cpu = None
+    if rank == 0 and args.cpu_baseline:
+        gbs, rps, nrec, tsec = oracle_sample(job, args.ref_records, budget_s=args.ref_seconds)
+        cpu = {"value": gbs, "unit": "GB/s", "cores": 1, "kind": "oracle",
+               "sample": f"first {nrec} records of {args.config} ({tsec:.1f} s, oracle/oracle.cpp std::unordered_map, "
+                         f"single thread pinned by construction; generation excluded)", "kv_inserts_per_s": rps}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+                "warmup": max(args.warmup, 3), "ms_per_step": ms / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+                "kv_inserts_per_s": recs_per_s,
+                "config": {"workload": CONFIG_TEXT[args.config], "records": n, "input_csr_bytes": csr,
+                           "distinct_keys": job.distinct, "ratio_table_over_budget": args.ratio,
+                           "table_footprint_bytes": F, "device_budget_bytes": job.sepo.budget_for(nb, job.page_bytes, pages),
+                           "n_buckets": nb, "page_bytes": job.page_bytes, "pool_pages": pages,
+                           "passes": st["passes"], "postponed_per_pass": st["postponed_per_pass"],
+                           "bytes_evicted": st["bytes_evicted"], "l2": "inputs (>= 15 GiB) far larger than L2 (126 MB)",
+                           "parallelism": f"replicas x{world}" if world > 1 else "1 GPU",
+                           "phase_ms": {kk: st[kk] for kk in ("t_insert_ms", "t_reprobe_ms", "t_compact_ms", "t_evict_ms")}},
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+                "gpu_launches": info["launches"], "slowdown_curve": curve}
+        print(json.dumps(line), flush=True)
+    t.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--ratio", type=float, default=4.0)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-curve", dest="curve", action="store_false")
+    ap.add_argument("--no-cpu", dest="cpu_baseline", action="store_false")
+    ap.add_argument("--ref-records", type=int, default=120_000_000)
+    ap.add_argument("--ref-seconds", type=float, default=15.0)
+    ap.add_argument("--traffic", type=float, default=None, help="dram bytes/launch from an ncu --set full capture")
+    args = ap.parse_args()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

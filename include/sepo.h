@@ -1,0 +1,190 @@
+/* sepo.h — C ABI of the B200-native SEPO hash table (Mokhtari & Stumm, IPDPS 2017).
+ *
+ * PAPER.md (= /root/reference/PAPER.md) is cited as P:L<line>. The calls follow the paper's
+ * statement of the problem:
+ *   * an insert either succeeds or returns POSTPONE, "like EAGAIN";
+ *   * the requestor tracks declined records in a bitmap with one bit per input record (P:L75,
+ *     P:L149) and re-issues only those later;
+ *   * at the end of each pass the table is told it no longer needs its resident pairs and copies
+ *     them to CPU memory, freeing the GPU heap;
+ *   * the final table is accessible from the CPU.
+ *
+ * Conventions for every call:
+ *   - "device" pointers are CUDA device memory (e.g. torch tensors' data_ptr()) and are
+ *     CALLER-OWNED: they must stay valid until the call returns; the library never frees them.
+ *   - Bitmap convention: bit (i & 31) of word (i >> 5) is 1 <=> record i was POSTPONED.
+ *     A bitmap for n records has ceil(n / 32) uint32 words.
+ *   - Key i of a batch is the byte string keys[ko[i] .. ko[i+1]) (ko = key_offsets, absolute
+ *     offsets into keys, ko[0] need not be 0); ko == NULL means fixed-width keys of
+ *     opts.fixed_key_width bytes (key i at keys + i * width).
+ *   - Errors: a negative return is an error code (sepo_status); sepo_last_error() describes the
+ *     last one on the calling thread. Argument errors leave the table unchanged. CUDA errors are
+ *     sticky: the table then only accepts sepo_stats / sepo_destroy.
+ *   - A table is bound to the CUDA device current at sepo_create and is NOT thread-safe.
+ *   - Every hot-path step runs in this library's sm_100a kernels; there is no CPU fallback.
+ */
+#ifndef SEPO_H
+#define SEPO_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct sepo_table sepo_table; /* opaque; one per GPU */
+
+enum sepo_status {
+    SEPO_OK = 0,
+    SEPO_E_INVAL = -1,    /* bad argument / unsupported combination */
+    SEPO_E_NOMEM = -2,    /* budget too small, or a host/device allocation failed */
+    SEPO_E_TOOLARGE = -3, /* a record's entry can never fit in one page (its bit is set) */
+    SEPO_E_CUDA = -4,     /* CUDA error (sticky) */
+    SEPO_E_STATE = -5,    /* call not allowed in the table's current state */
+    SEPO_E_NCCL = -6      /* NCCL error (sticky) */
+};
+
+/* Bucket organizations. BASIC is not implemented. */
+typedef enum {
+    SEPO_COMBINE_SUM_U64 = 0, /* "combining": one entry per key, value = u64 wrapping sum */
+    SEPO_GROUP = 1            /* "multi-valued": key entries + per-key value lists */
+} sepo_mode;
+
+typedef struct sepo_options {
+    int32_t mode;             /* sepo_mode; default SEPO_COMBINE_SUM_U64 */
+    uint32_t fixed_key_width; /* key bytes when key_offsets == NULL (1..page_bytes-32) */
+    uint32_t fixed_val_width; /* COMBINE: bytes of each LE unsigned value when vals != NULL
+                                 (1, 2, 4 or 8; default 8). GROUP: bytes per value when
+                                 val_offsets == NULL (1..256). */
+    uint32_t grid_ctas;       /* persistent CTAs = allocator slots (0 = 2 per SM) */
+    uint64_t hash_seed;       /* seed of the table's key hash (result is independent of it) */
+    uint32_t fail_alloc_ppm;  /* TEST ONLY: decline this many allocations per million */
+    uint32_t fail_mode;       /* 0: by hash(key, pass) (monotone per key); 1: by (record, pass) */
+    uint32_t fail_until_pass; /* injection is off from this pass on (default 16) */
+    uint32_t check_dups;      /* sepo_export merges + counts keys found in >1 generation */
+    void* stream;             /* cudaStream_t for all device work (NULL: a table-owned stream) */
+    uint64_t host_arena_bytes;/* pinned host memory to pre-allocate for evicted pages */
+} sepo_options;
+
+/* Host-side result, owned by the table (valid until the next sepo_reset / sepo_destroy).
+ * Order of keys is unspecified (canonicalise by sorting to compare). */
+typedef struct sepo_result {
+    uint64_t n_keys;
+    const uint8_t* keys;          /* key bytes, CSR */
+    const uint64_t* key_offsets;  /* n_keys + 1 */
+    const uint64_t* values;       /* COMBINE: n_keys u64 sums */
+    const uint64_t* list_offsets; /* GROUP: n_keys + 1, key k owns values [lo[k], lo[k+1]) */
+    uint64_t n_vals;              /* GROUP */
+    const uint8_t* vals;          /* GROUP: value bytes, CSR */
+    const uint64_t* val_offsets;  /* GROUP: n_vals + 1 */
+} sepo_result;
+
+#define SEPO_MAX_PASS_STATS 64
+typedef struct sepo_stats {
+    uint64_t passes;               /* evictions so far, the final one included (P:L237 counts) */
+    uint64_t insert_calls;
+    uint64_t records_inserted;     /* records handed to sepo_insert_batch (re-issues included) */
+    uint64_t postponed_per_pass[SEPO_MAX_PASS_STATS]; /* after re-probe, per pass */
+    uint64_t n_buckets, page_bytes, pool_pages, grid_ctas;
+    uint64_t pages_used_max;       /* most pages resident at once */
+    uint64_t bytes_evicted;        /* D2H bytes of evicted pages (final export included) */
+    uint64_t dead_bytes;           /* bytes of entries that lost a link race */
+    uint64_t cross_gen_dups;       /* keys merged across generations at export (check_dups) */
+    uint64_t forced_full_evictions;/* GROUP: passes that evicted retained key pages */
+    uint64_t toolarge;             /* records whose entry cannot fit a page */
+    uint64_t key_bytes_inserted;   /* key bytes handed to sepo_insert_batch */
+    uint64_t val_bytes_inserted;   /* value bytes handed to sepo_insert_batch */
+    uint64_t kernel_launches;      /* this library's kernels launched since create/reset */
+    double t_insert_ms, t_reprobe_ms, t_compact_ms, t_evict_ms, t_export_ms, t_h2d_ms;
+} sepo_stats;
+
+/* Create a table on the current CUDA device.
+ * device_budget_bytes: ONE device allocation of exactly this size holds the bucket directory
+ *   (4 B x n_buckets), the allocator state and the page pool ("a heap
+ *   pre-allocated in GPU memory ... partitioned into pages"). The paper sizes the heap as "the
+ *   remaining free space"; here the caller caps it, which is how tables larger than the
+ *   budget are produced. Must leave room for at least 4 pages; the pool is limited to 32 GiB.
+ * n_buckets: >= 1, <= 2^32 - 1.   page_bytes: power of two in [4096, 16 MiB].
+ * Returns NULL on error (sepo_last_error()). */
+sepo_table* sepo_create(size_t device_budget_bytes, uint64_t n_buckets, uint32_t page_bytes);
+
+/* Budget (bytes) that sepo_create needs so that the pool holds exactly `pool_pages` pages.
+ * Pure arithmetic on the host (no CUDA call). */
+size_t sepo_budget_for(uint64_t n_buckets, uint32_t page_bytes, uint64_t pool_pages);
+
+/* Set options (only before the first insert, or right after sepo_reset). */
+int sepo_configure(sepo_table* t, const sepo_options* opts);
+
+/* Insert n records (the SEPO "insert"). Each key is hashed to a bucket, the
+ * bucket chain is walked; a key already resident in this pass is combined/grouped in place
+ * (P:L77); a new key gets an entry allocated from the page pool and linked at the
+ * chain head. If allocation fails the record is POSTPONED: its bitmap bit is set.
+ * keys/key_offsets/vals/val_offsets: device; see conventions above.
+ *   COMBINE: vals == NULL => every value is 1 (Word Count / PVC); else fixed-width LE
+ *            unsigned values (opts.fixed_val_width bytes each); val_offsets must be NULL.
+ *   GROUP:   vals required; val_offsets != NULL => value i = vals[vo[i] .. vo[i+1]) (<= 256 B),
+ *            else opts.fixed_val_width bytes each.
+ * postponed_bitmap: device, ceil(n/32) words, fully written (bits >= n are 0).
+ * Returns the number of postponed records (>= 0; POSTPONE is not an error), or < 0.
+ * The count is an upper bound of what must be re-issued: a declined record whose key another
+ * thread linked concurrently is absorbed by sepo_reprobe at the end of the pass.
+ * Stream-ordered on the table's stream; synchronizes once to read the count. */
+int64_t sepo_insert_batch(sepo_table* t, const uint8_t* keys, const uint64_t* key_offsets, const uint8_t* vals,
+                          const uint64_t* val_offsets, uint64_t n, uint32_t* postponed_bitmap);
+
+/* End-of-pass re-probe (restores the residency guarantee P:L77, P:L79 under
+ * lock-free insertion). For every record whose bit is set, look its key up in the resident
+ * generation: if present, combine/append it now and clear the bit; in GROUP mode a resident key
+ * that still cannot take its value marks its key page as retained. Call after the last
+ * insert of a pass and before sepo_evict, with each batch of the pass.
+ * bitmap: device, updated in place. *key_bytes / *val_bytes (may be NULL) receive the bytes the
+ * remaining records occupy (to size sepo_compact's outputs). Returns the remaining count. */
+int64_t sepo_reprobe(sepo_table* t, const uint8_t* keys, const uint64_t* key_offsets, const uint8_t* vals,
+                     const uint64_t* val_offsets, uint64_t n, uint32_t* bitmap, uint64_t* key_bytes,
+                     uint64_t* val_bytes);
+
+/* Stream-compaction re-issue (a9; replaces the paper's restart "from the point where a request
+ * was postponed for the first time"): gather the records whose bit is set, in
+ * input order, into out_* (device, caller-owned, sized from sepo_reprobe's byte counts; out_ko
+ * and out_vo need m + 1 entries). Output offsets are rebased to 0. Fixed-width keys/values stay
+ * fixed-width (out_ko / out_vo unused then and may be NULL). Returns m. */
+int64_t sepo_compact(sepo_table* t, const uint8_t* keys, const uint64_t* key_offsets, const uint8_t* vals,
+                     const uint64_t* val_offsets, uint64_t n, const uint32_t* bitmap, uint8_t* out_keys,
+                     uint64_t* out_key_offsets, uint8_t* out_vals, uint64_t* out_val_offsets);
+
+/* Pass boundary (a10): copy the cold pages — COMBINE: every page of the generation;
+ * GROUP: value pages + key pages without pending keys — to pinned host memory and
+ * return them to the pool; reset the bucket directory. Returns bytes copied (>= 0) or < 0. */
+int64_t sepo_evict(sepo_table* t);
+
+/* Finish the job (a11): evict the resident generation, wait for all copies, and assemble the
+ * result on the host from every generation's page images. After this only
+ * sepo_stats / sepo_reset / sepo_destroy are allowed. */
+int sepo_export(sepo_table* t, sepo_result* out);
+
+/* The whole SEPO job in one call: insert all n records, then re-probe / compact / evict and
+ * re-issue until nothing is postponed, then evict the final generation (the table is then on the
+ * host; call sepo_export for the assembled result). keys/key_offsets/vals/val_offsets may be
+ * HOST or DEVICE memory (all four alike); host input is streamed to the device in chunks.
+ * Returns the number of passes (>= 1) or < 0. */
+int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* key_offsets, const uint8_t* vals,
+                 const uint64_t* val_offsets, uint64_t n);
+
+/* Drop all generations and results and start a new job with the same budget and options;
+ * pinned host memory and device scratch are kept for reuse. */
+int sepo_reset(sepo_table* t);
+
+int sepo_stats_get(const sepo_table* t, sepo_stats* out);
+
+/* Milliseconds of device time of the most recent sepo_insert_batch kernel(s), measured with CUDA
+ * events on the table's stream (bench roofline). */
+double sepo_last_insert_ms(const sepo_table* t);
+
+void sepo_destroy(sepo_table* t);
+const char* sepo_last_error(void);
+const char* sepo_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SEPO_H */

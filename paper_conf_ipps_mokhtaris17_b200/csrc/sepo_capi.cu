@@ -1,0 +1,902 @@
+// sepo_capi.cu — host engine + C ABI of the SEPO hash table (include/sepo.h).
+//
+// The engine owns: the device budget region (one cudaMalloc, carved into directory, allocator
+// state and page pool), a pinned host arena that receives evicted pages, the
+// generation images used to assemble the result, streams/events, and device scratch for
+// sepo_run's re-issue buffers. All record processing runs in sepo_kernels.cu; the host only
+// sequences kernels, copies pages and parses page images into the exported arrays.
+#include <cuda_runtime.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <chrono>
+#include <atomic>
+#include <string>
+#include <string_view>
+#include <thread>
+#include <unordered_map>
+#include <vector>
+
+#include "sepo.h"
+#include "sepo_dev.cuh"
+#include "sepo_kernels.h"
+
+using namespace sepo;
+
+namespace {
+thread_local std::string g_err;
+
+int fail(int code, const std::string& msg) {
+    g_err = msg;
+    return code;
+}
+
+struct PinChunk {
+    uint8_t* p = nullptr;
+    size_t cap = 0, used = 0;
+};
+
+struct Run {  // consecutive evicted pages [first, first+count) at host address p
+    uint32_t first, count;
+    uint8_t* p;
+};
+struct GenImage {
+    uint32_t gen;
+    std::vector<Run> runs;
+};
+
+struct DevBuf {
+    void* p = nullptr;
+    size_t cap = 0;
+    int grow(size_t bytes) {
+        if (bytes <= cap) return 0;
+        if (p) cudaFree(p);
+        p = nullptr;
+        cap = 0;
+        size_t want = std::max<size_t>(bytes, 1 << 20);
+        if (cudaMalloc(&p, want) != cudaSuccess) {
+            cudaGetLastError();
+            return -1;
+        }
+        cap = want;
+        return 0;
+    }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        cap = 0;
+    }
+};
+
+enum State { ST_ACTIVE = 0, ST_EXPORTED = 1, ST_BROKEN = 2 };
+}  // namespace
+
+struct sepo_table {
+    int device = 0;
+    size_t budget = 0;
+    uint64_t n_buckets = 0;
+    uint32_t page_bytes = 0, page_shift = 0, n_pages = 0;
+    int grid = 0, n_sms = 0;
+    uint8_t* region = nullptr;
+    Dev d{};
+    sepo_options opts{};
+    cudaStream_t stream = nullptr, copy_stream = nullptr;
+    bool own_stream = false;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev_copy = nullptr, ev_comp = nullptr;
+    Ctrl* h_ctrl = nullptr;        // pinned mirror of the device control block
+    uint32_t* h_evict = nullptr;   // pinned evict list
+    uint64_t* h_ko = nullptr;      // pinned: first/last key offset of the last insert batch
+    State state = ST_ACTIVE;
+    bool dirty = false;            // resident generation holds data not yet evicted
+    bool configured_once = false;
+    bool inserted = false;
+    uint32_t batch_seq = 0;
+    uint64_t pages_resident_retained = 0;
+    std::vector<PinChunk> arena;
+    std::vector<GenImage> gens;
+    sepo_stats st{};
+    double last_insert_ms = 0;
+    // scratch
+    DevBuf tile_counts, bm, buf[2][4];  // ping-pong: keys, key offsets, vals, val offsets
+    DevBuf in_stage[4];
+    // export storage
+    std::vector<uint8_t> x_keys, x_vals;
+    std::vector<uint64_t> x_koffs, x_values, x_loffs, x_voffs;
+    uint64_t x_nkeys = 0, x_nvals = 0;
+};
+
+namespace {
+int cuda_check(sepo_table* t, cudaError_t e, const char* what) {
+    if (e == cudaSuccess) return 0;
+    t->state = ST_BROKEN;
+    return fail(SEPO_E_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+#define CK(t, expr)                                              \
+    do {                                                         \
+        int _rc = cuda_check((t), (cudaError_t)(expr), #expr);   \
+        if (_rc) return _rc;                                     \
+    } while (0)
+
+uint8_t* arena_alloc(sepo_table* t, size_t bytes) {
+    for (auto& c : t->arena)
+        if (c.cap - c.used >= bytes) {
+            uint8_t* p = c.p + c.used;
+            c.used += (bytes + 255) & ~(size_t)255;
+            if (c.used > c.cap) c.used = c.cap;
+            return p;
+        }
+    PinChunk c;
+    c.cap = std::max<size_t>(bytes, (size_t)256 << 20);
+    if (cudaHostAlloc((void**)&c.p, c.cap, cudaHostAllocDefault) != cudaSuccess) {
+        cudaGetLastError();
+        return nullptr;
+    }
+    c.used = (bytes + 255) & ~(size_t)255;
+    if (c.used > c.cap) c.used = c.cap;
+    t->arena.push_back(c);
+    return c.p;
+}
+
+int check_active(sepo_table* t) {
+    if (!t) return fail(SEPO_E_INVAL, "null table");
+    if (t->state == ST_BROKEN) return fail(SEPO_E_CUDA, "table is broken by an earlier CUDA error");
+    if (t->state == ST_EXPORTED) return fail(SEPO_E_STATE, "table already exported (sepo_reset to reuse)");
+    return 0;
+}
+
+int make_batch(sepo_table* t, Batch& b, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
+               uint64_t n, uint32_t* bitmap) {
+    b.keys = keys;
+    b.ko = ko;
+    b.kw = t->opts.fixed_key_width;
+    b.vals = vals;
+    b.vo = vo;
+    b.vw = t->opts.fixed_val_width;
+    b.n = n;
+    b.bitmap = bitmap;
+    if (n == 0) return 0;
+    if (!keys && !(ko == nullptr && b.kw == 0)) return fail(SEPO_E_INVAL, "keys is NULL");
+    if (!ko && b.kw == 0) return fail(SEPO_E_INVAL, "key_offsets is NULL and fixed_key_width is 0");
+    if (t->opts.mode == SEPO_COMBINE_SUM_U64) {
+        if (vo) return fail(SEPO_E_INVAL, "COMBINE mode takes fixed-width values (val_offsets must be NULL)");
+        if (vals && !(b.vw == 1 || b.vw == 2 || b.vw == 4 || b.vw == 8))
+            return fail(SEPO_E_INVAL, "COMBINE fixed_val_width must be 1, 2, 4 or 8");
+        if (vals && ((uintptr_t)vals % b.vw)) return fail(SEPO_E_INVAL, "vals not aligned to fixed_val_width");
+    } else {
+        if (!vals) return fail(SEPO_E_INVAL, "GROUP mode needs values");
+        if (vo) return fail(SEPO_E_INVAL, "GROUP mode: variable-length values are not supported yet (use fixed_val_width)");
+        if (b.vw == 0 || b.vw > 256) return fail(SEPO_E_INVAL, "GROUP fixed_val_width must be in 1..256");
+    }
+    return 0;
+}
+
+void sync_dev(sepo_table* t) { t->d.batch_seq = t->batch_seq; }
+
+int read_ctrl(sepo_table* t) {
+    CK(t, cudaMemcpyAsync(t->h_ctrl, t->d.ctrl, sizeof(Ctrl), cudaMemcpyDeviceToHost, t->stream));
+    CK(t, cudaStreamSynchronize(t->stream));
+    return 0;
+}
+int zero_ctrl_counters(sepo_table* t) {
+    // postponed, toolarge, dead_bytes, kept_key_bytes, kept_val_bytes (fields 1..5)
+    CK(t, cudaMemsetAsync(&t->d.ctrl->postponed, 0, 5 * sizeof(unsigned long long), t->stream));
+    return 0;
+}
+
+double elapsed_ms(cudaEvent_t a, cudaEvent_t b) {
+    float ms = 0;
+    cudaEventElapsedTime(&ms, a, b);
+    return ms;
+}
+
+int init_device_state(sepo_table* t) {
+    CK(t, cudaMemsetAsync(t->d.dir, 0, t->n_buckets * 4, t->stream));
+    int rc = sepo_launch_init(t->d, (uint32_t)t->grid, t->stream);
+    if (rc) return cuda_check(t, (cudaError_t)rc, "init kernel");
+    t->st.kernel_launches += 1;
+    t->d.n_free = t->n_pages;
+    t->d.gen = 0;
+    CK(t, cudaStreamSynchronize(t->stream));
+    return 0;
+}
+}  // namespace
+
+// (exported functions get C linkage from their declarations in sepo.h)
+
+const char* sepo_last_error(void) { return g_err.c_str(); }
+const char* sepo_version(void) { return "sepo-b200 0.1 (sm_100a)"; }
+
+static size_t al256(size_t x) { return (x + 255) & ~(size_t)255; }
+static const size_t kMaxGrid = 1024;  // cursor slots reserved in the budget region
+static size_t fixed_bytes(uint64_t n_buckets) {
+    return al256(n_buckets * 4) + al256(sizeof(Ctrl)) + al256(kMaxGrid * 2 * 8);
+}
+static const size_t kPerPageMeta = 4 + 1 + 1 + 4;  // stack, page_state, retain, evict_list
+
+size_t sepo_budget_for(uint64_t n_buckets, uint32_t page_bytes, uint64_t pool_pages) {
+    return fixed_bytes(n_buckets) + 4 * 256 + (size_t)page_bytes + pool_pages * ((size_t)page_bytes + kPerPageMeta) + 4096;
+}
+
+sepo_table* sepo_create(size_t budget, uint64_t n_buckets, uint32_t page_bytes) {
+    if (n_buckets == 0 || n_buckets > 0xffffffffull) { fail(SEPO_E_INVAL, "n_buckets must be in [1, 2^32-1]"); return nullptr; }
+    if (page_bytes < 4096 || page_bytes > (4u << 20) || (page_bytes & (page_bytes - 1))) {
+        fail(SEPO_E_INVAL, "page_bytes must be a power of two in [4 KiB, 4 MiB]");
+        return nullptr;
+    }
+    auto* t = new sepo_table();
+    cudaGetDevice(&t->device);
+    cudaDeviceGetAttribute(&t->n_sms, cudaDevAttrMultiProcessorCount, t->device);
+    t->budget = budget;
+    t->n_buckets = n_buckets;
+    t->page_bytes = page_bytes;
+    t->page_shift = 0;
+    while ((1u << t->page_shift) < page_bytes) ++t->page_shift;
+    t->grid = 2 * t->n_sms;
+    t->opts.mode = SEPO_COMBINE_SUM_U64;
+    t->opts.fixed_val_width = 8;
+    t->opts.fail_until_pass = 16;
+    // carve: dir | ctrl | cursors | stack | page_state | retain | evict_list | (align) pool
+    auto al = al256;
+    const size_t max_grid = kMaxGrid;
+    size_t fixed = fixed_bytes(n_buckets);
+    if (budget <= fixed + 4 * (size_t)page_bytes) {
+        fail(SEPO_E_NOMEM, "device budget too small for the directory + 4 pages");
+        delete t;
+        return nullptr;
+    }
+    size_t per_page = (size_t)page_bytes + kPerPageMeta;
+    size_t np = (budget - fixed - 4 * 256 - page_bytes) / per_page;
+    if (np > ((size_t)32 << 30) / page_bytes) np = ((size_t)32 << 30) / page_bytes;  // 32 GiB pool limit (u32 refs)
+    if (np < 4) {
+        fail(SEPO_E_NOMEM, "device budget too small for 4 pages");
+        delete t;
+        return nullptr;
+    }
+    t->n_pages = (uint32_t)np;
+    if (cudaMalloc((void**)&t->region, budget) != cudaSuccess) {
+        cudaGetLastError();
+        fail(SEPO_E_NOMEM, "cudaMalloc of the device budget failed");
+        delete t;
+        return nullptr;
+    }
+    uint8_t* p = t->region;
+    Dev& d = t->d;
+    d.dir = (uint32_t*)p; p += al(n_buckets * 4);
+    d.ctrl = (Ctrl*)p; p += al(sizeof(Ctrl));
+    d.cursors = (unsigned long long*)p; p += al(max_grid * 2 * 8);
+    d.stack = (uint32_t*)p; p += al(np * 4);
+    d.page_state = p; p += al(np);
+    d.retain = p; p += al(np);
+    d.evict_list = (uint32_t*)p; p += al(np * 4);
+    uintptr_t pa = ((uintptr_t)p + page_bytes - 1) & ~(uintptr_t)(page_bytes - 1);
+    if (pa + np * (size_t)page_bytes > (uintptr_t)t->region + budget) {
+        // alignment ate a page
+        --np;
+        t->n_pages = (uint32_t)np;
+    }
+    d.pool = (uint8_t*)pa;
+    d.n_buckets = n_buckets;
+    d.page_bytes = page_bytes;
+    d.page_shift = t->page_shift;
+    d.n_pages = t->n_pages;
+    d.seed = 0x5e9053eedull;
+    d.fail_until = 16;
+    cudaStreamCreateWithFlags(&t->stream, cudaStreamNonBlocking);
+    t->own_stream = true;
+    cudaStreamCreateWithFlags(&t->copy_stream, cudaStreamNonBlocking);
+    cudaEventCreate(&t->ev0);
+    cudaEventCreate(&t->ev1);
+    cudaEventCreateWithFlags(&t->ev_copy, cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&t->ev_comp, cudaEventDisableTiming);
+    cudaHostAlloc((void**)&t->h_ctrl, sizeof(Ctrl), cudaHostAllocDefault);
+    cudaHostAlloc((void**)&t->h_evict, (size_t)t->n_pages * 4, cudaHostAllocDefault);
+    cudaHostAlloc((void**)&t->h_ko, 16, cudaHostAllocDefault);
+    if (cudaGetLastError() != cudaSuccess || !t->h_ctrl || !t->h_evict) {
+        fail(SEPO_E_CUDA, "stream/event/pinned allocation failed");
+        sepo_destroy(t);
+        return nullptr;
+    }
+    t->st.n_buckets = n_buckets;
+    t->st.page_bytes = page_bytes;
+    t->st.pool_pages = t->n_pages;
+    t->st.grid_ctas = t->grid;
+    if (init_device_state(t)) {
+        sepo_destroy(t);
+        return nullptr;
+    }
+    return t;
+}
+
+int sepo_configure(sepo_table* t, const sepo_options* o) {
+    int rc = check_active(t);
+    if (rc) return rc;
+    if (!o) return fail(SEPO_E_INVAL, "null options");
+    if (t->inserted) return fail(SEPO_E_STATE, "configure only before the first insert (or after sepo_reset)");
+    if (o->mode != SEPO_COMBINE_SUM_U64 && o->mode != SEPO_GROUP) return fail(SEPO_E_INVAL, "unknown mode");
+    if (o->fixed_key_width > 65535u - 64u) return fail(SEPO_E_INVAL, "fixed_key_width too large");
+    if (o->grid_ctas > 1024) return fail(SEPO_E_INVAL, "grid_ctas must be <= 1024");
+    sepo_options n = *o;
+    if (n.mode == SEPO_COMBINE_SUM_U64 && n.fixed_val_width == 0) n.fixed_val_width = 8;
+    if (n.fail_until_pass == 0) n.fail_until_pass = 16;
+    if (n.grid_ctas == 0) n.grid_ctas = 2 * t->n_sms;
+    t->grid = (int)n.grid_ctas;
+    t->st.grid_ctas = t->grid;
+    if (n.stream) {
+        if (t->own_stream && t->stream) cudaStreamDestroy(t->stream);
+        t->stream = (cudaStream_t)n.stream;
+        t->own_stream = false;
+    }
+    t->opts = n;
+    t->d.seed = n.hash_seed ^ 0x5e9053eedull;
+    t->d.fail_ppm = n.fail_alloc_ppm;
+    t->d.fail_mode = n.fail_mode;
+    t->d.fail_until = n.fail_until_pass;
+    if (n.host_arena_bytes) {
+        size_t have = 0;
+        for (auto& c : t->arena) have += c.cap;
+        if (have < n.host_arena_bytes) {
+            PinChunk c;
+            c.cap = n.host_arena_bytes - have;
+            if (cudaHostAlloc((void**)&c.p, c.cap, cudaHostAllocDefault) != cudaSuccess) {
+                cudaGetLastError();
+                return fail(SEPO_E_NOMEM, "pinned host arena allocation failed");
+            }
+            t->arena.push_back(c);
+        }
+    }
+    t->configured_once = true;
+    return 0;
+}
+
+int64_t sepo_insert_batch(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
+                          uint64_t n, uint32_t* bitmap) {
+    int rc = check_active(t);
+    if (rc) return rc;
+    Batch b;
+    rc = make_batch(t, b, keys, ko, vals, vo, n, bitmap);
+    if (rc) return rc;
+    if (n == 0) return 0;
+    if (!bitmap) return fail(SEPO_E_INVAL, "postponed_bitmap is NULL");
+    t->inserted = true;
+    t->dirty = true;
+    ++t->batch_seq;
+    sync_dev(t);
+    if ((rc = zero_ctrl_counters(t))) return rc;
+    CK(t, cudaEventRecord(t->ev0, t->stream));
+    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream);
+    if (rc) return cuda_check(t, (cudaError_t)rc, "insert kernel launch");
+    CK(t, cudaEventRecord(t->ev1, t->stream));
+    t->st.kernel_launches += 1;
+    if (ko) {
+        CK(t, cudaMemcpyAsync(&t->h_ko[0], ko, 8, cudaMemcpyDeviceToHost, t->stream));
+        CK(t, cudaMemcpyAsync(&t->h_ko[1], ko + n, 8, cudaMemcpyDeviceToHost, t->stream));
+    }
+    if ((rc = read_ctrl(t))) return rc;
+    t->last_insert_ms = elapsed_ms(t->ev0, t->ev1);
+    t->st.t_insert_ms += t->last_insert_ms;
+    t->st.insert_calls++;
+    t->st.records_inserted += n;
+    t->st.key_bytes_inserted += ko ? (t->h_ko[1] - t->h_ko[0]) : n * (uint64_t)t->opts.fixed_key_width;
+    t->st.val_bytes_inserted += vals ? n * (uint64_t)t->opts.fixed_val_width : 0;
+    t->st.dead_bytes += t->h_ctrl->dead_bytes;
+    const uint64_t used = std::min<uint64_t>(t->h_ctrl->pool_taken, t->d.n_free) + t->pages_resident_retained;
+    t->st.pages_used_max = std::max<uint64_t>(t->st.pages_used_max, used);
+    if (t->h_ctrl->toolarge) {
+        t->st.toolarge += t->h_ctrl->toolarge;
+        return fail(SEPO_E_TOOLARGE, std::to_string(t->h_ctrl->toolarge) + " record(s) cannot fit in one page");
+    }
+    return (int64_t)t->h_ctrl->postponed;
+}
+
+static int64_t count_or_probe(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
+                              uint64_t n, uint32_t* bitmap, int probe, uint64_t* kb, uint64_t* vb) {
+    Batch b;
+    int rc = make_batch(t, b, keys, ko, vals, vo, n, bitmap);
+    if (rc) return rc;
+    if (kb) *kb = 0;
+    if (vb) *vb = 0;
+    if (n == 0) return 0;
+    if (!bitmap) return fail(SEPO_E_INVAL, "bitmap is NULL");
+    const uint64_t nt = sepo_reprobe_tiles(n);
+    if (t->tile_counts.grow(nt * 3 * 8)) return fail(SEPO_E_NOMEM, "tile count scratch");
+    sync_dev(t);
+    if ((rc = zero_ctrl_counters(t))) return rc;
+    rc = sepo_launch_reprobe(t->d, b, t->opts.mode, probe, t->grid, (unsigned long long*)t->tile_counts.p, t->stream);
+    t->st.kernel_launches += 1;
+    if (rc) return cuda_check(t, (cudaError_t)rc, "reprobe kernel launch");
+    if ((rc = read_ctrl(t))) return rc;
+    if (kb) *kb = t->h_ctrl->kept_key_bytes;
+    if (vb) *vb = t->h_ctrl->kept_val_bytes;
+    return (int64_t)t->h_ctrl->postponed;
+}
+
+int64_t sepo_reprobe(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
+                     uint64_t n, uint32_t* bitmap, uint64_t* kb, uint64_t* vb) {
+    int rc = check_active(t);
+    if (rc) return rc;
+    CK(t, cudaEventRecord(t->ev0, t->stream));
+    int64_t r = count_or_probe(t, keys, ko, vals, vo, n, bitmap, 1, kb, vb);
+    if (r < 0) return r;
+    CK(t, cudaEventRecord(t->ev1, t->stream));
+    CK(t, cudaEventSynchronize(t->ev1));
+    t->st.t_reprobe_ms += elapsed_ms(t->ev0, t->ev1);
+    const uint64_t pass = t->st.passes;
+    if (pass < SEPO_MAX_PASS_STATS) t->st.postponed_per_pass[pass] += (uint64_t)r;
+    return r;
+}
+
+int64_t sepo_compact(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
+                     uint64_t n, const uint32_t* bitmap, uint8_t* ok, uint64_t* oko, uint8_t* ov, uint64_t* ovo) {
+    int rc = check_active(t);
+    if (rc) return rc;
+    CK(t, cudaEventRecord(t->ev0, t->stream));
+    uint64_t kb = 0, vb = 0;
+    int64_t m = count_or_probe(t, keys, ko, vals, vo, n, const_cast<uint32_t*>(bitmap), 0, &kb, &vb);
+    if (m < 0) return m;
+    Batch b;
+    make_batch(t, b, keys, ko, vals, vo, n, const_cast<uint32_t*>(bitmap));
+    if (m > 0 && (!ok || (ko && !oko) || (vals && !ov) || (vo && !ovo)))
+        return fail(SEPO_E_INVAL, "compaction output buffer is NULL");
+    rc = sepo_launch_compact(b, (unsigned long long*)t->tile_counts.p, ok, oko, ov, ovo, (uint64_t)m, kb, vb, t->grid,
+                             t->stream);
+    if (rc) return cuda_check(t, (cudaError_t)rc, "compact kernel launch");
+    t->st.kernel_launches += sepo_reprobe_tiles(n) ? 3 : 1;
+    CK(t, cudaEventRecord(t->ev1, t->stream));
+    CK(t, cudaEventSynchronize(t->ev1));
+    t->st.t_compact_ms += elapsed_ms(t->ev0, t->ev1);
+    return m;
+}
+
+// Pass boundary. honor_retain = 0 evicts every resident page (final export / forced).
+static int64_t evict_impl(sepo_table* t, int honor_retain) {
+    CK(t, cudaEventRecord(t->ev0, t->stream));
+    sync_dev(t);
+    int rc = sepo_launch_seal(t->d, (uint32_t)t->grid, t->stream);
+    if (rc) return cuda_check(t, (cudaError_t)rc, "seal kernel");
+    rc = sepo_launch_classify(t->d, honor_retain, t->stream);
+    if (rc) return cuda_check(t, (cudaError_t)rc, "classify kernel");
+    t->st.kernel_launches += 2;
+    if ((rc = read_ctrl(t))) return rc;
+    const uint64_t ne = t->h_ctrl->n_evict;
+    if (ne) {
+        CK(t, cudaMemcpyAsync(t->h_evict, t->d.evict_list, ne * 4, cudaMemcpyDeviceToHost, t->stream));
+        CK(t, cudaStreamSynchronize(t->stream));
+    }
+    // page copies on the copy stream, ordered after the compute stream (event)
+    CK(t, cudaEventRecord(t->ev_comp, t->stream));
+    CK(t, cudaStreamWaitEvent(t->copy_stream, t->ev_comp, 0));
+    GenImage img;
+    img.gen = t->d.gen;
+    uint64_t bytes = 0;
+    for (uint64_t i = 0; i < ne;) {
+        uint64_t j = i + 1;
+        while (j < ne && t->h_evict[j] == t->h_evict[j - 1] + 1) ++j;
+        const uint32_t first = t->h_evict[i], cnt = (uint32_t)(j - i);
+        const size_t nbytes = (size_t)cnt * t->page_bytes;
+        uint8_t* hp = arena_alloc(t, nbytes);
+        if (!hp) return fail(SEPO_E_NOMEM, "pinned host arena exhausted");
+        CK(t, cudaMemcpyAsync(hp, t->d.pool + ((size_t)first << t->page_shift), nbytes, cudaMemcpyDeviceToHost,
+                              t->copy_stream));
+        img.runs.push_back({first, cnt, hp});
+        bytes += nbytes;
+        i = j;
+    }
+    CK(t, cudaEventRecord(t->ev_copy, t->copy_stream));
+    // the freed pages are reused only after their copy finished
+    CK(t, cudaStreamWaitEvent(t->stream, t->ev_copy, 0));
+    CK(t, cudaMemsetAsync(t->d.dir, 0, t->n_buckets * 4, t->stream));
+    t->d.n_free = (uint32_t)t->h_ctrl->n_free;
+    t->pages_resident_retained = t->h_ctrl->n_resident;
+    t->d.gen += 1;
+    if (t->opts.mode == SEPO_GROUP && t->pages_resident_retained) {
+        rc = sepo_launch_relink(t->d, t->stream);
+        if (rc) return cuda_check(t, (cudaError_t)rc, "relink kernel");
+        t->st.kernel_launches += 1;
+    }
+    CK(t, cudaEventRecord(t->ev1, t->stream));
+    CK(t, cudaEventSynchronize(t->ev1));
+    t->st.t_evict_ms += elapsed_ms(t->ev0, t->ev1);
+    if (!img.runs.empty()) t->gens.push_back(std::move(img));
+    t->st.bytes_evicted += bytes;
+    t->st.passes += 1;
+    t->dirty = t->pages_resident_retained > 0;
+    return (int64_t)bytes;
+}
+
+int64_t sepo_evict(sepo_table* t) {
+    int rc = check_active(t);
+    if (rc) return rc;
+    return evict_impl(t, 1);
+}
+
+// ---------------------------------------------------------------- export (host assembly, a11)
+namespace {
+struct PageRef {
+    const uint8_t* p;
+    uint32_t page;
+    uint32_t gen;
+};
+
+void collect_pages(sepo_table* t, std::vector<PageRef>& pages) {
+    for (auto& g : t->gens)
+        for (auto& r : g.runs)
+            for (uint32_t k = 0; k < r.count; ++k) pages.push_back({r.p + (size_t)k * t->page_bytes, r.first + k, g.gen});
+}
+
+template <class F>
+void parallel_for(size_t n, F f) {
+    unsigned nt = std::max(1u, std::min(16u, std::thread::hardware_concurrency()));
+    if (n < 64) nt = 1;
+    std::vector<std::thread> th;
+    for (unsigned w = 0; w < nt; ++w)
+        th.emplace_back([&, w] {
+            size_t lo = n * w / nt, hi = n * (w + 1) / nt;
+            f(w, lo, hi);
+        });
+    for (auto& x : th) x.join();
+}
+
+int export_combine(sepo_table* t) {
+    std::vector<PageRef> pages;
+    collect_pages(t, pages);
+    const uint32_t PB = t->page_bytes;
+    const size_t np = pages.size();
+    std::vector<uint64_t> pk(np + 1, 0), pb(np + 1, 0);
+    std::atomic<int> bad{0};
+    parallel_for(np, [&](unsigned, size_t lo, size_t hi) {
+        for (size_t i = lo; i < hi; ++i) {
+            uint64_t k = 0, kb = 0;
+            uint32_t off = 0;
+            const uint8_t* base = pages[i].p;
+            while (off < PB) {
+                uint32_t hdr;
+                memcpy(&hdr, base + off, 4);
+                uint32_t sz = hdr & ~KIND_MASK;
+                if (sz == 0 || off + sz > PB) { bad = 1; break; }
+                if ((hdr & KIND_MASK) == K_COMBINE) {
+                    uint32_t klen;
+                    memcpy(&klen, base + off + 12, 4);
+                    ++k;
+                    kb += klen;
+                }
+                off += sz;
+            }
+            pk[i + 1] = k;
+            pb[i + 1] = kb;
+        }
+    });
+    if (bad) return fail(SEPO_E_STATE, "corrupt page image during export");
+    for (size_t i = 0; i < np; ++i) { pk[i + 1] += pk[i]; pb[i + 1] += pb[i]; }
+    const uint64_t nk = pk[np], nkb = pb[np];
+    t->x_keys.resize(nkb);
+    t->x_koffs.resize(nk + 1);
+    t->x_values.resize(nk);
+    parallel_for(np, [&](unsigned, size_t lo, size_t hi) {
+        for (size_t i = lo; i < hi; ++i) {
+            uint64_t k = pk[i], kb = pb[i];
+            uint32_t off = 0;
+            const uint8_t* base = pages[i].p;
+            while (off < PB) {
+                uint32_t hdr;
+                memcpy(&hdr, base + off, 4);
+                uint32_t sz = hdr & ~KIND_MASK;
+                if ((hdr & KIND_MASK) == K_COMBINE) {
+                    uint32_t klen;
+                    memcpy(&klen, base + off + 12, 4);
+                    t->x_koffs[k] = kb;
+                    memcpy(&t->x_values[k], base + off + 16, 8);
+                    memcpy(t->x_keys.data() + kb, base + off + CENTRY_HDR, klen);
+                    ++k;
+                    kb += klen;
+                }
+                off += sz;
+            }
+        }
+    });
+    t->x_koffs[nk] = nkb;
+    t->x_nkeys = nk;
+    // keys found in more than one generation (only possible under record-mode fault injection)
+    const bool merge = t->opts.check_dups || (t->opts.fail_alloc_ppm && t->opts.fail_mode == 1);
+    if (merge && nk) {
+        std::unordered_map<std::string_view, uint64_t> idx;
+        idx.reserve(nk * 2);
+        std::vector<uint8_t> keys2;
+        std::vector<uint64_t> offs2, vals2;
+        offs2.push_back(0);
+        uint64_t dups = 0;
+        std::vector<uint64_t> order;
+        for (uint64_t k = 0; k < nk; ++k) {
+            std::string_view sv((const char*)t->x_keys.data() + t->x_koffs[k], t->x_koffs[k + 1] - t->x_koffs[k]);
+            auto it = idx.find(sv);
+            if (it == idx.end()) {
+                idx.emplace(sv, vals2.size());
+                vals2.push_back(t->x_values[k]);
+                order.push_back(k);
+            } else {
+                ++dups;
+                vals2[it->second] += t->x_values[k];
+            }
+        }
+        if (dups) {
+            for (uint64_t k : order) {
+                keys2.insert(keys2.end(), t->x_keys.begin() + t->x_koffs[k], t->x_keys.begin() + t->x_koffs[k + 1]);
+                offs2.push_back(keys2.size());
+            }
+            t->x_keys.swap(keys2);
+            t->x_koffs.swap(offs2);
+            t->x_values.swap(vals2);
+            t->x_nkeys = t->x_values.size();
+        }
+        t->st.cross_gen_dups = dups;
+    }
+    return 0;
+}
+
+int export_group(sepo_table* t) {
+    std::vector<PageRef> pages;
+    collect_pages(t, pages);
+    const uint32_t PB = t->page_bytes;
+    const size_t np = pages.size();
+    // pass A: key entries (identity = birth gen << 40 | entry ref) and value chunks
+    struct KeyRec { const uint8_t* key; uint32_t len; uint64_t id; };
+    struct ChunkRec { const uint8_t* vals; uint32_t cnt; uint64_t owner; };
+    std::vector<std::vector<KeyRec>> tk(16);
+    std::vector<std::vector<ChunkRec>> tc(16);
+    std::atomic<int> bad{0};
+    uint32_t vw = t->opts.fixed_val_width;
+    parallel_for(np, [&](unsigned w, size_t lo, size_t hi) {
+        for (size_t i = lo; i < hi; ++i) {
+            uint32_t off = 0;
+            const uint8_t* base = pages[i].p;
+            while (off < PB) {
+                uint32_t hdr;
+                memcpy(&hdr, base + off, 4);
+                uint32_t sz = hdr & ~KIND_MASK;
+                if (sz == 0 || off + sz > PB) { bad = 1; break; }
+                uint32_t kind = hdr & KIND_MASK;
+                if (kind == K_GKEY) {
+                    uint32_t klen, birth;
+                    memcpy(&klen, base + off + 12, 4);
+                    memcpy(&birth, base + off + 24, 4);
+                    uint64_t poolo = ((uint64_t)pages[i].page << t->page_shift) + off;
+                    tk[w].push_back({base + off + GKEY_HDR, klen, ((uint64_t)birth << 40) | ((poolo >> 3) + 1)});
+                } else if (kind == K_VCHUNK) {
+                    uint32_t fill, cap;
+                    uint64_t owner;
+                    memcpy(&fill, base + off + 4, 4);
+                    memcpy(&owner, base + off + 8, 8);
+                    memcpy(&cap, base + off + 24, 4);
+                    tc[w].push_back({base + off + CHUNK_HDR, std::min(fill, cap), owner});
+                }
+                off += sz;
+            }
+        }
+    });
+    if (bad) return fail(SEPO_E_STATE, "corrupt page image during export");
+    // key index; keys that appear under several identities (forced full evictions / injection) merge
+    std::unordered_map<uint64_t, uint64_t> id2k;
+    std::unordered_map<std::string_view, uint64_t> name2k;
+    std::vector<const KeyRec*> keys;
+    uint64_t dups = 0;
+    size_t total = 0;
+    for (auto& v : tk) total += v.size();
+    id2k.reserve(total * 2);
+    name2k.reserve(total * 2);
+    for (auto& v : tk)
+        for (auto& kr : v) {
+            std::string_view sv((const char*)kr.key, kr.len);
+            auto it = name2k.find(sv);
+            uint64_t k;
+            if (it == name2k.end()) { k = keys.size(); name2k.emplace(sv, k); keys.push_back(&kr); }
+            else { k = it->second; ++dups; }
+            id2k[kr.id] = k;
+        }
+    t->st.cross_gen_dups = dups;
+    const uint64_t nk = keys.size();
+    std::vector<uint64_t> cnt(nk + 1, 0);
+    for (auto& v : tc)
+        for (auto& c : v) {
+            auto it = id2k.find(c.owner);
+            if (it == id2k.end()) return fail(SEPO_E_STATE, "value chunk with unknown owner");
+            cnt[it->second + 1] += c.cnt;
+        }
+    for (uint64_t k = 0; k < nk; ++k) cnt[k + 1] += cnt[k];
+    const uint64_t nv = cnt[nk];
+    t->x_loffs.assign(cnt.begin(), cnt.end());
+    t->x_vals.resize(nv * vw);
+    t->x_voffs.resize(nv + 1);
+    for (uint64_t i = 0; i <= nv; ++i) t->x_voffs[i] = i * vw;
+    std::vector<uint64_t> cur(cnt.begin(), cnt.end() - 1);
+    for (auto& v : tc)
+        for (auto& c : v) {
+            uint64_t k = id2k[c.owner];
+            memcpy(t->x_vals.data() + cur[k] * vw, c.vals, (size_t)c.cnt * vw);
+            cur[k] += c.cnt;
+        }
+    uint64_t kb = 0;
+    for (auto* kr : keys) kb += kr->len;
+    t->x_keys.resize(kb);
+    t->x_koffs.resize(nk + 1);
+    kb = 0;
+    for (uint64_t k = 0; k < nk; ++k) {
+        t->x_koffs[k] = kb;
+        memcpy(t->x_keys.data() + kb, keys[k]->key, keys[k]->len);
+        kb += keys[k]->len;
+    }
+    t->x_koffs[nk] = kb;
+    t->x_nkeys = nk;
+    t->x_nvals = nv;
+    return 0;
+}
+}  // namespace
+
+int sepo_export(sepo_table* t, sepo_result* out) {
+    int rc = check_active(t);
+    if (rc) return rc;
+    if (!out) return fail(SEPO_E_INVAL, "null result");
+    if (t->dirty) {
+        int64_t e = evict_impl(t, 0);
+        if (e < 0) return (int)e;
+    }
+    CK(t, cudaStreamSynchronize(t->copy_stream));
+    auto t0 = std::chrono::steady_clock::now();
+    rc = t->opts.mode == SEPO_COMBINE_SUM_U64 ? export_combine(t) : export_group(t);
+    if (rc) return rc;
+    t->st.t_export_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    memset(out, 0, sizeof(*out));
+    out->n_keys = t->x_nkeys;
+    out->keys = t->x_keys.data();
+    out->key_offsets = t->x_koffs.data();
+    if (t->opts.mode == SEPO_COMBINE_SUM_U64) {
+        out->values = t->x_values.data();
+    } else {
+        out->list_offsets = t->x_loffs.data();
+        out->n_vals = t->x_nvals;
+        out->vals = t->x_vals.data();
+        out->val_offsets = t->x_voffs.data();
+    }
+    t->state = ST_EXPORTED;
+    return 0;
+}
+
+// ---------------------------------------------------------------- the whole job
+static bool is_device_ptr(const void* p) {
+    if (!p) return true;
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
+                 uint64_t n) {
+    int rc = check_active(t);
+    if (rc) return rc;
+    const bool dev = is_device_ptr(keys) && is_device_ptr(ko) && is_device_ptr(vals) && is_device_ptr(vo);
+    const uint32_t kw = t->opts.fixed_key_width, vw = t->opts.fixed_val_width;
+    if (!dev && n) {
+        // host input: stage it in device memory (one H2D per array, P:L227 counts this transfer)
+        auto t0 = std::chrono::steady_clock::now();
+        uint64_t kbytes = 0, vbytes = 0;
+        uint64_t k0 = 0, v0 = 0;
+        if (ko) { k0 = ko[0]; kbytes = ko[n] - ko[0]; } else kbytes = n * (uint64_t)kw;
+        if (vals) { if (vo) { v0 = vo[0]; vbytes = vo[n] - vo[0]; } else vbytes = n * (uint64_t)vw; }
+        if (t->in_stage[0].grow(kbytes + 16) || (ko && t->in_stage[1].grow((n + 1) * 8)) ||
+            (vals && t->in_stage[2].grow(vbytes + 16)) || (vo && t->in_stage[3].grow((n + 1) * 8)))
+            return fail(SEPO_E_NOMEM, "device staging for host input");
+        CK(t, cudaMemcpyAsync(t->in_stage[0].p, keys + k0, kbytes, cudaMemcpyHostToDevice, t->stream));
+        if (ko) CK(t, cudaMemcpyAsync(t->in_stage[1].p, ko, (n + 1) * 8, cudaMemcpyHostToDevice, t->stream));
+        if (vals) CK(t, cudaMemcpyAsync(t->in_stage[2].p, vals + v0, vbytes, cudaMemcpyHostToDevice, t->stream));
+        if (vo) CK(t, cudaMemcpyAsync(t->in_stage[3].p, vo, (n + 1) * 8, cudaMemcpyHostToDevice, t->stream));
+        CK(t, cudaStreamSynchronize(t->stream));
+        t->st.t_h2d_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+        // offsets stay absolute: shift the key base so keys[ko[i]] addresses the staged copy
+        const uint8_t* kdev = (const uint8_t*)t->in_stage[0].p - k0;
+        const uint8_t* vdev = vals ? (const uint8_t*)t->in_stage[2].p - v0 : nullptr;
+        return sepo_run(t, kdev, ko ? (const uint64_t*)t->in_stage[1].p : nullptr, vdev,
+                        vo ? (const uint64_t*)t->in_stage[3].p : nullptr, n);
+    }
+    const uint8_t* ck = keys;
+    const uint64_t* cko = ko;
+    const uint8_t* cv = vals;
+    const uint64_t* cvo = vo;
+    uint64_t cn = n;
+    int side = 0;
+    int64_t passes_start = (int64_t)t->st.passes;
+    uint64_t prev = ~0ull;
+    while (cn > 0) {
+        if (t->bm.grow(((cn + 31) / 32) * 4)) return fail(SEPO_E_NOMEM, "bitmap scratch");
+        uint32_t* bmp = (uint32_t*)t->bm.p;
+        int64_t c = sepo_insert_batch(t, ck, cko, cv, cvo, cn, bmp);
+        if (c < 0) return c;
+        uint64_t kb = 0, vb = 0;
+        if (c > 0) c = sepo_reprobe(t, ck, cko, cv, cvo, cn, bmp, &kb, &vb);
+        if (c < 0) return c;
+        if (c == 0) break;
+        DevBuf* o = t->buf[side];
+        if (o[0].grow(kb + 16) || (cko && o[1].grow(((uint64_t)c + 1) * 8)) || (cv && o[2].grow(vb + 16)) ||
+            (cvo && o[3].grow(((uint64_t)c + 1) * 8)))
+            return fail(SEPO_E_NOMEM, "re-issue buffers");
+        int64_t m = sepo_compact(t, ck, cko, cv, cvo, cn, bmp, (uint8_t*)o[0].p, cko ? (uint64_t*)o[1].p : nullptr,
+                                 cv ? (uint8_t*)o[2].p : nullptr, cvo ? (uint64_t*)o[3].p : nullptr);
+        if (m < 0) return m;
+        // GROUP: a pass without progress (retained key pages starve the pool) evicts everything
+        // (the paper is silent; reading R14)
+        int honor = 1;
+        if (t->opts.mode == SEPO_GROUP && (uint64_t)m >= prev) {
+            honor = 0;
+            t->st.forced_full_evictions++;
+        }
+        prev = (uint64_t)m;
+        int64_t e = evict_impl(t, honor);
+        if (e < 0) return e;
+        ck = (const uint8_t*)o[0].p;
+        cko = cko ? (const uint64_t*)o[1].p : nullptr;
+        cv = cv ? (const uint8_t*)o[2].p : nullptr;
+        cvo = cvo ? (const uint64_t*)o[3].p : nullptr;
+        cn = (uint64_t)m;
+        side ^= 1;
+        if (t->st.passes - passes_start > 100000) return fail(SEPO_E_STATE, "no progress");
+    }
+    // final generation to host (P:L227 timing scope includes the table transfer)
+    if (t->dirty) {
+        int64_t e = evict_impl(t, 0);
+        if (e < 0) return e;
+    }
+    CK(t, cudaStreamSynchronize(t->copy_stream));
+    return (int64_t)t->st.passes - passes_start;
+}
+
+int sepo_reset(sepo_table* t) {
+    if (!t) return fail(SEPO_E_INVAL, "null table");
+    if (t->state == ST_BROKEN) return fail(SEPO_E_CUDA, "table is broken");
+    cudaStreamSynchronize(t->copy_stream);
+    for (auto& c : t->arena) c.used = 0;
+    t->gens.clear();
+    t->state = ST_ACTIVE;
+    t->dirty = false;
+    t->inserted = false;
+    t->batch_seq = 0;
+    t->pages_resident_retained = 0;
+    sepo_stats z{};
+    z.n_buckets = t->n_buckets;
+    z.page_bytes = t->page_bytes;
+    z.pool_pages = t->n_pages;
+    z.grid_ctas = t->grid;
+    t->st = z;
+    return init_device_state(t);
+}
+
+int sepo_stats_get(const sepo_table* t, sepo_stats* out) {
+    if (!t || !out) return fail(SEPO_E_INVAL, "null argument");
+    *out = t->st;
+    return 0;
+}
+
+double sepo_last_insert_ms(const sepo_table* t) { return t ? t->last_insert_ms : 0.0; }
+
+void sepo_destroy(sepo_table* t) {
+    if (!t) return;
+    if (t->stream) cudaStreamSynchronize(t->stream);
+    if (t->copy_stream) cudaStreamSynchronize(t->copy_stream);
+    t->tile_counts.release();
+    t->bm.release();
+    for (auto& s : t->buf)
+        for (auto& b : s) b.release();
+    for (auto& b : t->in_stage) b.release();
+    for (auto& c : t->arena) cudaFreeHost(c.p);
+    if (t->h_ctrl) cudaFreeHost(t->h_ctrl);
+    if (t->h_evict) cudaFreeHost(t->h_evict);
+    if (t->h_ko) cudaFreeHost(t->h_ko);
+    if (t->region) cudaFree(t->region);
+    if (t->ev0) cudaEventDestroy(t->ev0);
+    if (t->ev1) cudaEventDestroy(t->ev1);
+    if (t->ev_copy) cudaEventDestroy(t->ev_copy);
+    if (t->ev_comp) cudaEventDestroy(t->ev_comp);
+    if (t->own_stream && t->stream) cudaStreamDestroy(t->stream);
+    if (t->copy_stream) cudaStreamDestroy(t->copy_stream);
+    delete t;
+}

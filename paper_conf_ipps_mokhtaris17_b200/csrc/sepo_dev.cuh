@@ -1,0 +1,242 @@
+// sepo_dev.cuh — device data structures and primitives of the SEPO hash table (sm_100a).
+//
+// PAPER.md cited as P:L<line>. Layout of the budget region (one cudaMalloc, host side carves it):
+//   dir[n_buckets]      u32 entry refs, "a simple array of null pointers"
+//   ctrl                counters (pool_taken, postponed, dead bytes, ...)
+//   cursors[G][2]       per-CTA allocation cursors {page<<32 | offset} (key/combine, value)
+//   stack[P]            free-page stack (pages handed out by pool_taken)
+//   page_state[P]       0 free, 1 entry/key page, 2 value page
+//   retain[P]           GROUP: key page kept resident at the pass end
+//   evict_list[P]       pages evicted at the last pass boundary
+//   pool                P pages of page_bytes (the paper's heap)
+//
+// Entry refs are u32: ref = pool_offset/8 + 1 (0 = null). A value-list ref (GROUP) is u64:
+// generation << 40 | (pool_offset/8 + 1), so a list can point into an evicted generation — the
+// relocatable stand-in for the paper's "two pointers ... GPU ... and eventual location in CPU
+// memory". Device code never follows a value-list ref, it only CASes the list head.
+//
+// Every record in a page is 8-byte aligned and starts with a u32 header = size | kind, so an
+// evicted page image is parsed linearly on the host (a filler covers every unused tail):
+//   COMBINE entry       : hdr | next u32 | tag u32 | klen u32 | value u64 | key[pad8]
+//   GROUP key entry     : hdr | next u32 | tag u32 | klen u32 | list_head u64 |
+//                                      birth_gen u32 | pad u32 | key[pad8]
+//   GROUP value chunk: hdr | fill u32 | owner u64 | next u64 | cap u32 | vw u32 | values
+//   filler                            : hdr (size of the gap)
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace sepo {
+
+constexpr uint32_t FULLMASK = 0xffffffffu;
+enum : uint32_t { K_FREE = 0, K_COMBINE = 1, K_FILL = 2, K_DEAD = 3, K_GKEY = 4, K_VCHUNK = 5 };
+constexpr uint32_t KIND_MASK = 7u;
+constexpr uint32_t CENTRY_HDR = 24;  // combine entry header (incl. value)
+constexpr uint32_t GKEY_HDR = 32;    // group key entry header
+constexpr uint32_t CHUNK_HDR = 32;   // value chunk header
+constexpr uint32_t NOPAGE = 0xfffffffeu, FULLPAGE = 0xffffffffu;
+constexpr uint32_t PAGE_ENTRY = 1, PAGE_VALUE = 2;
+
+// result codes of a slot / record
+enum : uint32_t { R_OK = 0, R_POST = 1, R_TOOLARGE = 2 };
+
+struct Ctrl {
+    unsigned long long pool_taken;     // pages handed out from the free stack this generation
+    unsigned long long postponed;      // per-call accumulator
+    unsigned long long toolarge;
+    unsigned long long dead_bytes;
+    unsigned long long kept_key_bytes; // reprobe: bytes of the still-postponed records
+    unsigned long long kept_val_bytes;
+    unsigned long long n_evict;        // evict: pages in evict_list
+    unsigned long long n_free;         // evict: pages in the new free stack
+    unsigned long long n_resident;     // evict: pages that stay resident (retained)
+    unsigned long long pad[7];
+};
+
+struct Dev {
+    uint32_t* dir;
+    uint64_t n_buckets;
+    uint8_t* pool;
+    uint32_t page_bytes;
+    uint32_t page_shift;
+    uint32_t n_pages;
+    uint32_t n_free;          // pages available in `stack` this generation
+    uint32_t* stack;
+    uint8_t* page_state;
+    uint8_t* retain;
+    uint32_t* evict_list;
+    unsigned long long* cursors;  // [grid][2]
+    Ctrl* ctrl;
+    uint64_t seed;
+    uint32_t gen;             // generation (= pass index) of resident data
+    uint32_t fail_ppm, fail_mode, fail_until;
+    uint32_t batch_seq;
+};
+
+// ---------------------------------------------------------------- memory access helpers
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+// L2-coherent loads of published entry fields (never stale L1 lines)
+__device__ __forceinline__ uint64_t ldcg64(const void* p) { return __ldcg(reinterpret_cast<const unsigned long long*>(p)); }
+__device__ __forceinline__ uint32_t ldcg32(const void* p) { return __ldcg(reinterpret_cast<const unsigned int*>(p)); }
+
+// Bytes [p, p+nb) (1 <= nb <= 8) of immutable INPUT as a little-endian word, zero-extended.
+// Only the aligned words that contain requested bytes are read.
+__device__ __forceinline__ uint64_t load_in_word(const uint8_t* p, uint32_t nb) {
+    uintptr_t a = reinterpret_cast<uintptr_t>(p);
+    uint32_t sh = (uint32_t)(a & 7u);
+    const unsigned long long* q = reinterpret_cast<const unsigned long long*>(a - sh);
+    uint64_t v = __ldg(q) >> (8 * sh);
+    if (sh + nb > 8) v |= __ldg(q + 1) << (64 - 8 * sh);
+    if (nb < 8) v &= (1ull << (8 * nb)) - 1ull;
+    return v;
+}
+
+// ---------------------------------------------------------------- key hash (the paper leaves it open)
+__device__ __forceinline__ uint64_t fmix64(uint64_t k) {
+    k ^= k >> 33; k *= 0xff51afd7ed558ccdull;
+    k ^= k >> 33; k *= 0xc4ceb9fe1a85ec53ull;
+    k ^= k >> 33; return k;
+}
+__device__ __forceinline__ uint64_t hash_key(const uint8_t* p, uint32_t len, uint64_t seed) {
+    uint64_t h = seed ^ ((uint64_t)len * 0x87c37b91114253d5ull);
+    for (uint32_t o = 0; o < len; o += 8) {
+        uint32_t nb = len - o < 8 ? len - o : 8;
+        uint64_t w = load_in_word(p + o, nb);
+        h ^= w * 0x4cf5ad432745937full;
+        h = ((h << 29) | (h >> 35)) * 0x9e3779b97f4a7c15ull + 0x52dce729ull;
+    }
+    return fmix64(h);
+}
+__device__ __forceinline__ uint32_t bucket_of(uint64_t h, uint64_t n_buckets) {
+    return (uint32_t)(((h >> 32) * n_buckets) >> 32);
+}
+__device__ __forceinline__ uint32_t tag_of(uint64_t h) { return (uint32_t)h; }
+
+__device__ __forceinline__ uint32_t align8(uint32_t x) { return (x + 7u) & ~7u; }
+__device__ __forceinline__ uint8_t* ref_ptr(const Dev& d, uint32_t ref) { return d.pool + ((uint64_t)(ref - 1) << 3); }
+__device__ __forceinline__ uint32_t off_ref(uint64_t off) { return (uint32_t)(off >> 3) + 1u; }
+
+// Key equality: entry key at e + koff (8-aligned, zero padded) vs input key [p, p+len).
+__device__ __forceinline__ bool entry_key_eq(const uint8_t* ek, const uint8_t* p, uint32_t len) {
+    for (uint32_t o = 0; o < len; o += 8) {
+        uint32_t nb = len - o < 8 ? len - o : 8;
+        if (ldcg64(ek + o) != load_in_word(p + o, nb)) return false;
+    }
+    return true;
+}
+// Input-vs-input key equality (both immutable input bytes)
+__device__ __forceinline__ bool in_key_eq(const uint8_t* a, const uint8_t* b, uint32_t len) {
+    for (uint32_t o = 0; o < len; o += 8) {
+        uint32_t nb = len - o < 8 ? len - o : 8;
+        if (load_in_word(a + o, nb) != load_in_word(b + o, nb)) return false;
+    }
+    return true;
+}
+// Copy an input key into an entry (8-aligned destination, zero padded tail)
+__device__ __forceinline__ void store_key(uint8_t* ek, const uint8_t* p, uint32_t len) {
+    for (uint32_t o = 0; o < len; o += 8) {
+        uint32_t nb = len - o < 8 ? len - o : 8;
+        *reinterpret_cast<unsigned long long*>(ek + o) = load_in_word(p + o, nb);
+    }
+}
+
+// Walk the chain [ref .. stop) for an entry with (tag, len, key). koff = key offset in entry.
+// Only entries of the resident generation are reachable (head insertion; the directory
+// is reset at every pass boundary).
+__device__ __forceinline__ uint8_t* chain_find(const Dev& d, uint32_t ref, uint32_t stop, uint32_t tag, uint32_t len,
+                                               const uint8_t* key, uint32_t koff) {
+    while (ref != 0 && ref != stop) {
+        uint8_t* e = ref_ptr(d, ref);
+        uint64_t w0 = ldcg64(e);      // hdr | next
+        uint64_t w1 = ldcg64(e + 8);  // tag | klen
+        if ((uint32_t)w1 == tag && (uint32_t)(w1 >> 32) == len && entry_key_eq(e + koff, key, len)) return e;
+        ref = (uint32_t)(w0 >> 32);
+    }
+    return nullptr;
+}
+
+// ---------------------------------------------------------------- fault injection (tests only)
+__device__ __forceinline__ bool inject_fail(const Dev& d, uint64_t h, uint64_t rec) {
+    if (d.fail_ppm == 0 || d.gen >= d.fail_until) return false;
+    uint64_t x = d.fail_mode == 0 ? fmix64(h ^ (0x9e37ull * (d.gen + 1)))
+                                  : fmix64(rec * 0x100000001b3ull ^ ((uint64_t)d.batch_seq << 40) ^ (d.gen + 7));
+    return (x % 1000000ull) < d.fail_ppm;
+}
+
+// ---------------------------------------------------------------- page-pool allocator
+// Warp-collective bump allocation from this CTA's current page (cursor in shared memory, packed
+// {page << 32 | offset}). Lanes with `need` get `size` bytes (multiple of 8, <= page_bytes) and
+// the pool offset back, or ~0 when the page is full and the pool has no free page (POSTPONE).
+// The first lane whose range crosses the page end writes a filler over the tail, takes a page
+// from the free stack (one global atomic per page) and installs it; lanes of other warps that
+// overshot wait for the install and retry. Must be called by all 32 lanes.
+__device__ __forceinline__ uint64_t warp_alloc(const Dev& d, unsigned long long* scur, bool need, uint32_t size,
+                                               uint8_t page_kind) {
+    const uint32_t lane = threadIdx.x & 31u;
+    const uint32_t PB = d.page_bytes;
+    uint64_t result = ~0ull;
+    bool pending = need;
+    while (true) {
+        unsigned pm = __ballot_sync(FULLMASK, pending);
+        if (!pm) break;
+        uint32_t s = pending ? size : 0u;
+        uint32_t incl = s;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            uint32_t y = __shfl_up_sync(FULLMASK, incl, o);
+            if (lane >= (uint32_t)o) incl += y;
+        }
+        uint32_t total = __shfl_sync(FULLMASK, incl, 31);
+        uint32_t excl = incl - s;
+        unsigned long long cur = 0;
+        if (lane == 0) cur = atomicAdd(scur, (unsigned long long)total);
+        cur = __shfl_sync(FULLMASK, cur, 0);
+        const uint32_t page = (uint32_t)(cur >> 32);
+        const uint32_t off = (uint32_t)cur;
+        if (page == FULLPAGE) break;  // pool exhausted for this CTA: every pending lane POSTPONEs
+        bool again = false;
+        if (pending) {
+            uint64_t start = (uint64_t)off + excl;
+            if (page != NOPAGE && start + s <= PB) {
+                result = ((uint64_t)page << d.page_shift) + start;
+                pending = false;
+            } else {
+                if (start <= PB) {  // the unique crossing lane: seal the tail, install a new page
+                    if (page != NOPAGE && start < PB)
+                        *reinterpret_cast<uint32_t*>(d.pool + ((uint64_t)page << d.page_shift) + start) =
+                            (uint32_t)(PB - start) | K_FILL;
+                    unsigned long long q = atomicAdd(&d.ctrl->pool_taken, 1ull);
+                    unsigned long long nw;
+                    if (q < d.n_free) {
+                        uint32_t np = d.stack[q];
+                        d.page_state[np] = page_kind;
+                        nw = (unsigned long long)np << 32;
+                    } else {
+                        nw = (unsigned long long)FULLPAGE << 32;
+                    }
+                    __threadfence_block();
+                    atomicExch(scur, nw);
+                }
+                again = true;
+            }
+        }
+        if (__any_sync(FULLMASK, again)) {
+            if (lane == 0) {
+                while ((uint32_t)(*reinterpret_cast<volatile unsigned long long*>(scur) >> 32) == page) __nanosleep(20);
+            }
+            __syncwarp();
+        }
+    }
+    return result;
+}
+
+}  // namespace sepo

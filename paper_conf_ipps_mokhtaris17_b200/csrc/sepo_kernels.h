@@ -1,0 +1,32 @@
+// sepo_kernels.h — launcher interface between the host engine (sepo_capi.cu) and the kernels.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include "sepo_dev.cuh"
+
+namespace sepo {
+// One batch of records as passed to sepo_insert_batch / sepo_reprobe / sepo_compact.
+struct Batch {
+    const uint8_t* keys;
+    const uint64_t* ko;   // nullptr => fixed width kw
+    uint32_t kw;
+    uint32_t vw;          // COMBINE: value bytes (vals != nullptr); GROUP: fixed value bytes
+    const uint8_t* vals;  // COMBINE: nullptr => 1
+    const uint64_t* vo;   // GROUP variable-length values (not supported yet: must be nullptr)
+    uint64_t n;
+    uint32_t* bitmap;
+};
+}  // namespace sepo
+
+int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int grid, cudaStream_t s);
+size_t sepo_insert_smem(int mode);
+int sepo_insert_threads(int mode);
+int sepo_launch_reprobe(const sepo::Dev& d, const sepo::Batch& b, int mode, int probe, int grid,
+                        unsigned long long* tile_counts, cudaStream_t s);
+uint64_t sepo_reprobe_tiles(uint64_t n);
+int sepo_launch_compact(const sepo::Batch& b, unsigned long long* tile_counts, uint8_t* ok, uint64_t* oko, uint8_t* ov,
+                        uint64_t* ovo, uint64_t m, uint64_t kb, uint64_t vb, int grid, cudaStream_t s);
+int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);
+int sepo_launch_classify(const sepo::Dev& d, int honor_retain, cudaStream_t s);
+int sepo_launch_relink(const sepo::Dev& d, cudaStream_t s);
+int sepo_launch_init(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);

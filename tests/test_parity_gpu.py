@@ -1,0 +1,258 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle, element by element after
+canonical sorting (all aggregation is integer => bit-exact), plus the SEPO invariants the paper
+states: multi-pass result == single-pass result, no key in two generations,
+each pass makes progress, order/budget/postponement independence."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from tests.util import device_inputs, footprint_pages, oracle_expected, run_job
+
+pytestmark = pytest.mark.gpu
+
+
+def sepo():
+    import paper_conf_ipps_mokhtaris17_b200 as m
+    return m
+
+
+def assert_same(got, exp):
+    assert len(got) == len(exp), f"{len(got)} keys vs {len(exp)} expected"
+    bad = [k for k in exp if got.get(k) != exp[k]]
+    assert not bad, f"{len(bad)} mismatching keys, e.g. {bad[:3]}: got {[got.get(k) for k in bad[:3]]}, exp {[exp[k] for k in bad[:3]]}"
+
+
+def budget_pages(stream, k, n_buckets, page_bytes, inputs, **kw):
+    F = footprint_pages(stream, n_buckets, page_bytes, inputs=inputs, **kw)
+    return F, max(4, int(np.ceil(F / k)))
+
+
+# ------------------------------------------------------------------ in-budget (one pass)
+def test_c1_in_budget(cuda):
+    s = gen.config("C1")
+    exp = oracle_expected(s)
+    assert exp == s.expected_combine()  # oracle pinned to the closed form on this very input
+    got, passes, st = run_job(s, sepo().budget_for(1 << 16, 65536, 256), 1 << 16, 65536)
+    assert passes == 1  # P:L241 "Word Count will rarely need multiple iterations"
+    assert st["postponed_per_pass"][0] == 0
+    assert_same(got, exp)
+
+
+@pytest.mark.parametrize("ratio", [2, 4])
+def test_c1_over_budget(cuda, ratio):
+    s = gen.config("C1")
+    inp = device_inputs(s)
+    exp = oracle_expected(s)
+    F, P = budget_pages(s, ratio, 1 << 14, 4096, inp)
+    got, passes, st = run_job(s, sepo().budget_for(1 << 14, 4096, P), 1 << 14, 4096, inputs=inp, check_dups=True)
+    assert_same(got, exp)
+    assert passes >= 2
+    assert st["cross_gen_dups"] == 0  # no key is needed again after its eviction
+    post = st["postponed_per_pass"]
+    assert all(post[i] > post[i + 1] for i in range(len(post) - 1)) and post[-1] == 0, post
+
+
+@pytest.mark.parametrize("ppm,mode", [(10_000, 0), (500_000, 0), (500_000, 1)])
+def test_fault_injection(cuda, ppm, mode):
+    """postponement pattern does not change the result; key-mode failure is monotone per key"""
+    s = gen.config("C1", scale=0.3)
+    exp = oracle_expected(s)
+    got, passes, st = run_job(s, sepo().budget_for(1 << 14, 65536, 64), 1 << 14, 65536, fail_alloc_ppm=ppm,
+                              fail_mode=mode, check_dups=True)
+    assert_same(got, exp)
+    assert passes >= 2
+    if mode == 0:
+        assert st["cross_gen_dups"] == 0
+
+
+@pytest.mark.parametrize("page_bytes,n_buckets,grid,seed", [(4096, 1 << 10, 1, 1), (1 << 20, 1 << 20, 37, 2),
+                                                           (65536, 3, 296, 3), (16384, 12345, 148, 4)])
+def test_invariant_to_table_shape(cuda, page_bytes, n_buckets, grid, seed):
+    s = gen.config("C1", scale=0.2)
+    exp = oracle_expected(s)
+    got, _, _ = run_job(s, sepo().budget_for(n_buckets, page_bytes, max(8, (8 << 20) // page_bytes)), n_buckets,
+                        page_bytes, grid_ctas=grid, hash_seed=seed)
+    assert_same(got, exp)
+
+
+def test_permutation_and_batches(cuda):
+    """records in another order, inserted in several batches per pass"""
+    s = gen.config("C1", scale=0.1)
+    keys, offs, _ = s.host()
+    exp = oracle.combine(keys, offs).as_dict()
+    perm = np.random.default_rng(5).permutation(s.n)
+    kb = keys.tobytes()
+    words = [kb[offs[i]:offs[i + 1]] for i in perm]
+    lens = np.array([len(w) for w in words], dtype=np.int64)
+    o2 = np.zeros(s.n + 1, dtype=np.int64)
+    np.cumsum(lens, out=o2[1:])
+    k2 = torch.from_numpy(np.frombuffer(b"".join(words), dtype=np.uint8).copy()).cuda()
+    o2t = torch.from_numpy(o2).cuda()
+    t = sepo().Table(sepo().budget_for(1 << 12, 4096, 24), 1 << 12, 4096, check_dups=True)
+    # requestor-driven pass loop over 3 batches: insert, re-probe, compact, evict
+    cuts = [0, s.n // 3, 2 * s.n // 3, s.n]
+    batches = [(k2, o2t[cuts[i]:cuts[i + 1] + 1].clone(), cuts[i + 1] - cuts[i]) for i in range(3)]
+    passes = 0
+    while batches:
+        bms = []
+        for (k, o, n) in batches:
+            c, bm = t.insert_batch(k, o, n=n)
+            bms.append(bm)
+        nxt = []
+        for (k, o, n), bm in zip(batches, bms):
+            rem, kbytes, _ = t.reprobe(k, o, None, bm, n=n)
+            if rem:
+                # the compaction must equal the oracle's definition on this very bitmap
+                ok, oko, _, m = t.compact(k, o, None, bm, n=n)
+                hk = k.cpu().numpy(); ho = o.cpu().numpy().view(np.uint64)
+                bmh = bm.cpu().numpy().view(np.uint32)
+                ek, eo, _, _, em = oracle.compact(hk, ho - 0, bmh)
+                assert m == em == rem and int(oko[-1]) == kbytes
+                assert ok.cpu().numpy().tobytes() == ek.tobytes()
+                assert (oko.cpu().numpy().view(np.uint64) == eo).all()
+                nxt.append((ok, oko, m))
+        t.evict()
+        passes += 1
+        batches = nxt
+        assert passes < 200
+    got = sepo().result_dict(t.export())
+    assert_same(got, exp)
+    assert t.stats()["cross_gen_dups"] == 0
+    t.close()
+
+
+# ------------------------------------------------------------------ other workloads
+@pytest.mark.parametrize("name,ratio", [("C5u", 4), ("C5z", 4), ("C5u", 1)])
+def test_pairs_fixed_width(cuda, name, ratio):
+    s = gen.config(name, scale=2 ** -12)
+    exp = oracle_expected(s)
+    inp = device_inputs(s)
+    F, P = budget_pages(s, ratio, 1 << 16, 16384, inp)
+    got, passes, st = run_job(s, sepo().budget_for(1 << 16, 16384, P), 1 << 16, 16384, inputs=inp, check_dups=True)
+    assert_same(got, exp)
+    assert st["cross_gen_dups"] == 0
+    if ratio > 1:
+        assert passes >= 2
+
+
+def test_urls_c3(cuda):
+    s = gen.config("C3", scale=1 / 2000)
+    exp = oracle_expected(s)
+    inp = device_inputs(s)
+    F, P = budget_pages(s, 2, 1 << 16, 65536, inp)
+    got, passes, st = run_job(s, sepo().budget_for(1 << 16, 65536, P), 1 << 16, 65536, inputs=inp, check_dups=True)
+    assert_same(got, exp)
+    assert st["cross_gen_dups"] == 0
+
+
+@pytest.mark.parametrize("ratio", [1, 3])
+def test_group_c4(cuda, ratio):
+    s = gen.config("C4", scale=1 / 1000)
+    exp = oracle_expected(s)
+    inp = device_inputs(s)
+    F, P = budget_pages(s, ratio, 1 << 16, 16384, inp)
+    got, passes, st = run_job(s, sepo().budget_for(1 << 16, 16384, P + 2), 1 << 16, 16384, inputs=inp, check_dups=True)
+    assert_same(got, exp)
+    if ratio == 3:
+        assert passes >= 2
+
+
+# ------------------------------------------------------------------ edge cases
+def _tensors(keys):
+    offs = np.zeros(len(keys) + 1, dtype=np.int64)
+    offs[1:] = np.cumsum([len(k) for k in keys])
+    kb = np.frombuffer(b"".join(keys) + b"\0", dtype=np.uint8).copy()
+    return torch.from_numpy(kb).cuda(), torch.from_numpy(offs).cuda()
+
+
+@pytest.mark.parametrize("case", ["empty", "one", "ragged33", "hot", "zero_len", "long", "adversarial"])
+def test_edge_cases(cuda, case):
+    rng = np.random.default_rng(1)
+    if case == "empty":
+        keys = []
+    elif case == "one":
+        keys = [b"k"]
+    elif case == "ragged33":
+        keys = [bytes([65 + i % 7]) * (i % 5) for i in range(33)]
+    elif case == "hot":
+        keys = [b"the"] * 100_000 + [b"a"] * 3
+    elif case == "zero_len":
+        keys = [b""] * 40 + [b"x"] * 5 + [b""]
+    elif case == "long":
+        keys = [bytes(rng.integers(97, 100, size=int(L))) for L in rng.integers(200, 3000, size=500)] * 3
+    else:
+        pool = [b"", b"a", b"ab", b"a" * 256, b"a" * 255 + b"b", b"\0", b"\0\0", b"\xff" * 7, b"abcdefgh", b"abcdefgi"]
+        keys = [pool[i] for i in rng.integers(0, len(pool), size=5000)]
+    k, o = _tensors(keys)
+    t = sepo().Table(sepo().budget_for(1 << 10, 16384, 16), 1 << 10, 16384, check_dups=True)
+    passes = t.run(k, o)
+    got = sepo().result_dict(t.export())
+    exp = {}
+    for x in keys:
+        exp[x] = exp.get(x, 0) + 1
+    assert_same(got, exp)
+    assert t.stats()["cross_gen_dups"] == 0
+    t.close()
+
+
+def test_toolarge(cuda):
+    keys = [b"a", b"z" * 5000, b"b"]
+    k, o = _tensors(keys)
+    t = sepo().Table(sepo().budget_for(1 << 10, 4096, 16), 1 << 10, 4096)
+    with pytest.raises(sepo().SepoError) as e:
+        t.run(k, o)
+    assert e.value.code == sepo().E_TOOLARGE
+    t.close()
+
+
+def test_host_input_equals_device_input(cuda):
+    s = gen.config("C3", scale=1 / 4000)
+    exp = oracle_expected(s)
+    keys, offs, _ = s.host()
+    t = sepo().Table(sepo().budget_for(1 << 16, 65536, 64), 1 << 16, 65536)
+    t.run(keys, offs)  # numpy (host) arrays: staged by the library
+    assert_same(sepo().result_dict(t.export()), exp)
+    t.close()
+
+
+def test_reset_and_reuse(cuda):
+    s = gen.config("C1", scale=0.1)
+    exp = oracle_expected(s)
+    k, o, _ = device_inputs(s)
+    t = sepo().Table(sepo().budget_for(1 << 12, 4096, 32), 1 << 12, 4096)
+    for _ in range(3):
+        t.run(k, o)
+        assert_same(sepo().result_dict(t.export()), exp)
+        t.reset()
+    t.close()
+
+
+# ------------------------------------------------------------------ full size (bench launch config)
+def test_c2_full_size_sampled(cuda):
+    """C2 at BASELINE size (8 GiB text, 1.1e9 records) and budget F/4, as bench.py runs it:
+    every key's count equals the closed form c_r; totals: sum = n, #keys = V."""
+    import bench
+    s = gen.config("C2")
+    job = bench.make_job("C2", ratio=4.0)
+    k, o, v = job.inputs()
+    t = job.table()
+    passes = t.run(k, o, v)
+    res = t.export(copy=False)
+    assert passes >= 4
+    vals = res["values"]
+    assert res["n_keys"] == s.n_ranks
+    assert int(vals.sum(dtype=np.uint64)) == s.n
+    kb, ko = res["keys"], res["key_offsets"]
+    idx = np.random.default_rng(0).choice(res["n_keys"], 2000, replace=False)
+    spell2rank = None
+    for i in idx:
+        key = kb[ko[i]:ko[i + 1]].tobytes()
+        # rank from the spelling (base-26 digits) and its exact count c_r = floor(C/r)
+        r = 0
+        for ch in key:
+            r = r * 26 + (ch - 97)
+        assert s.spell(r) == key
+        assert int(vals[i]) == int(s.count_of_rank(r)), (key, r)
+    t.close()
