@@ -251,7 +251,7 @@ def run_ours(args):
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    job = Job(args.config, args.ratio)
+    job = Job(args.config, args.ratio, scale=args.scale)
     stream = torch.cuda.current_stream()
     job.inputs()
     nb, pages, F = job.table_params()
@@ -319,7 +319,7 @@ def run_ours(args):
         curve = {}
         base = None
         for r in (0.5, 1.0, 2.0, 3.0, 4.0):
-            j2 = Job(args.config, r)
+            j2 = Job(args.config, r, scale=args.scale)
             j2._inputs = job._inputs
             t2 = j2.table()
             for _ in range(2):
@@ -366,6 +366,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="C2")
     ap.add_argument("--ratio", type=float, default=4.0)
+    ap.add_argument("--scale", type=float, default=1.0, help="shrink the workload (profiling only; not a bench value)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-curve", dest="curve", action="store_false")
