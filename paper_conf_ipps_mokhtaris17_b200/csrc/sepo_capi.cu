@@ -70,6 +70,7 @@ struct DevBuf {
 };
 
 enum State { ST_ACTIVE = 0, ST_EXPORTED = 1, ST_BROKEN = 2 };
+const size_t kMaxGrid = 1024;  // cursor slots reserved in the budget region
 }  // namespace
 
 struct sepo_table {
@@ -93,6 +94,7 @@ struct sepo_table {
     bool inserted = false;
     uint32_t batch_seq = 0;
     uint64_t pages_resident_retained = 0;
+    uint64_t pending_idx_key_bytes = 0;  // key bytes of the next indexed re-issue batch (stats)
     std::vector<PinChunk> arena;
     std::vector<GenImage> gens;
     sepo_stats st{};
@@ -100,6 +102,9 @@ struct sepo_table {
     // scratch
     DevBuf tile_counts, bm, buf[2][4];  // ping-pong: keys, key offsets, vals, val offsets
     DevBuf in_stage[4];
+    DevBuf hot;  // hot-set discovery scratch (COMBINE)
+    DevBuf idxb[2];  // sepo_run re-issue index lists (ping-pong)
+
     // export storage
     std::vector<uint8_t> x_keys, x_vals;
     std::vector<uint64_t> x_koffs, x_values, x_loffs, x_voffs;
@@ -155,6 +160,7 @@ int make_batch(sepo_table* t, Batch& b, const uint8_t* keys, const uint64_t* ko,
     b.vw = t->opts.fixed_val_width;
     b.n = n;
     b.bitmap = bitmap;
+    b.idx = nullptr;
     if (n == 0) return 0;
     if (!keys && !(ko == nullptr && b.kw == 0)) return fail(SEPO_E_INVAL, "keys is NULL");
     if (!ko && b.kw == 0) return fail(SEPO_E_INVAL, "key_offsets is NULL and fixed_key_width is 0");
@@ -192,7 +198,7 @@ double elapsed_ms(cudaEvent_t a, cudaEvent_t b) {
 
 int init_device_state(sepo_table* t) {
     CK(t, cudaMemsetAsync(t->d.dir, 0, t->n_buckets * 4, t->stream));
-    int rc = sepo_launch_init(t->d, (uint32_t)t->grid, t->stream);
+    int rc = sepo_launch_init(t->d, (uint32_t)kMaxGrid, t->stream);  // every cursor slot, whatever the grid
     if (rc) return cuda_check(t, (cudaError_t)rc, "init kernel");
     t->st.kernel_launches += 1;
     t->d.n_free = t->n_pages;
@@ -208,7 +214,6 @@ const char* sepo_last_error(void) { return g_err.c_str(); }
 const char* sepo_version(void) { return "sepo-b200 0.1 (sm_100a)"; }
 
 static size_t al256(size_t x) { return (x + 255) & ~(size_t)255; }
-static const size_t kMaxGrid = 1024;  // cursor slots reserved in the budget region
 static size_t fixed_bytes(uint64_t n_buckets) {
     return al256(n_buckets * 4) + al256(sizeof(Ctrl)) + al256(kMaxGrid * 2 * 8);
 }
@@ -232,7 +237,7 @@ sepo_table* sepo_create(size_t budget, uint64_t n_buckets, uint32_t page_bytes) 
     t->page_bytes = page_bytes;
     t->page_shift = 0;
     while ((1u << t->page_shift) < page_bytes) ++t->page_shift;
-    t->grid = 2 * t->n_sms;
+    t->grid = sepo_default_grid(SEPO_COMBINE_SUM_U64, t->n_sms);
     t->opts.mode = SEPO_COMBINE_SUM_U64;
     t->opts.fixed_val_width = 8;
     t->opts.fail_until_pass = 16;
@@ -319,7 +324,7 @@ int sepo_configure(sepo_table* t, const sepo_options* o) {
     sepo_options n = *o;
     if (n.mode == SEPO_COMBINE_SUM_U64 && n.fixed_val_width == 0) n.fixed_val_width = 8;
     if (n.fail_until_pass == 0) n.fail_until_pass = 16;
-    if (n.grid_ctas == 0) n.grid_ctas = 2 * t->n_sms;
+    if (n.grid_ctas == 0) n.grid_ctas = (uint32_t)sepo_default_grid(n.mode, t->n_sms);
     t->grid = (int)n.grid_ctas;
     t->st.grid_ctas = t->grid;
     if (n.stream) {
@@ -349,36 +354,34 @@ int sepo_configure(sepo_table* t, const sepo_options* o) {
     return 0;
 }
 
-int64_t sepo_insert_batch(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
-                          uint64_t n, uint32_t* bitmap) {
-    int rc = check_active(t);
-    if (rc) return rc;
-    Batch b;
-    rc = make_batch(t, b, keys, ko, vals, vo, n, bitmap);
-    if (rc) return rc;
+static int64_t insert_impl(sepo_table* t, const Batch& b) {
+    int rc;
+    const uint64_t n = b.n;
     if (n == 0) return 0;
-    if (!bitmap) return fail(SEPO_E_INVAL, "postponed_bitmap is NULL");
+    if (!b.bitmap) return fail(SEPO_E_INVAL, "postponed_bitmap is NULL");
     t->inserted = true;
     t->dirty = true;
     ++t->batch_seq;
     sync_dev(t);
     if ((rc = zero_ctrl_counters(t))) return rc;
     CK(t, cudaEventRecord(t->ev0, t->stream));
-    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream);
+    if (t->opts.mode == SEPO_COMBINE_SUM_U64 && t->hot.grow(sepo_hot_scratch_bytes())) return fail(SEPO_E_NOMEM, "hot-set scratch");
+    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->opts.mode == SEPO_COMBINE_SUM_U64 ? t->hot.p : nullptr);
     if (rc) return cuda_check(t, (cudaError_t)rc, "insert kernel launch");
     CK(t, cudaEventRecord(t->ev1, t->stream));
-    t->st.kernel_launches += 1;
-    if (ko) {
-        CK(t, cudaMemcpyAsync(&t->h_ko[0], ko, 8, cudaMemcpyDeviceToHost, t->stream));
-        CK(t, cudaMemcpyAsync(&t->h_ko[1], ko + n, 8, cudaMemcpyDeviceToHost, t->stream));
+    t->st.kernel_launches += (t->opts.mode == SEPO_COMBINE_SUM_U64 && n >= (8ull << 18)) ? 4 : 1;
+    if (b.ko && !b.idx) {
+        CK(t, cudaMemcpyAsync(&t->h_ko[0], b.ko, 8, cudaMemcpyDeviceToHost, t->stream));
+        CK(t, cudaMemcpyAsync(&t->h_ko[1], b.ko + n, 8, cudaMemcpyDeviceToHost, t->stream));
     }
     if ((rc = read_ctrl(t))) return rc;
     t->last_insert_ms = elapsed_ms(t->ev0, t->ev1);
     t->st.t_insert_ms += t->last_insert_ms;
     t->st.insert_calls++;
     t->st.records_inserted += n;
-    t->st.key_bytes_inserted += ko ? (t->h_ko[1] - t->h_ko[0]) : n * (uint64_t)t->opts.fixed_key_width;
-    t->st.val_bytes_inserted += vals ? n * (uint64_t)t->opts.fixed_val_width : 0;
+    if (b.idx) t->st.key_bytes_inserted += t->pending_idx_key_bytes;
+    else t->st.key_bytes_inserted += b.ko ? (t->h_ko[1] - t->h_ko[0]) : n * (uint64_t)t->opts.fixed_key_width;
+    t->st.val_bytes_inserted += b.vals ? n * (uint64_t)t->opts.fixed_val_width : 0;
     t->st.dead_bytes += t->h_ctrl->dead_bytes;
     const uint64_t used = std::min<uint64_t>(t->h_ctrl->pool_taken, t->d.n_free) + t->pages_resident_retained;
     t->st.pages_used_max = std::max<uint64_t>(t->st.pages_used_max, used);
@@ -389,20 +392,31 @@ int64_t sepo_insert_batch(sepo_table* t, const uint8_t* keys, const uint64_t* ko
     return (int64_t)t->h_ctrl->postponed;
 }
 
-static int64_t count_or_probe(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
-                              uint64_t n, uint32_t* bitmap, int probe, uint64_t* kb, uint64_t* vb) {
-    Batch b;
-    int rc = make_batch(t, b, keys, ko, vals, vo, n, bitmap);
+int64_t sepo_insert_batch(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
+                          uint64_t n, uint32_t* bitmap) {
+    int rc = check_active(t);
     if (rc) return rc;
+    Batch b;
+    rc = make_batch(t, b, keys, ko, vals, vo, n, bitmap);
+    if (rc) return rc;
+    return insert_impl(t, b);
+}
+
+static int64_t count_or_probe(sepo_table* t, const Batch& b, int probe, uint64_t* kb, uint64_t* vb) {
+    int rc;
     if (kb) *kb = 0;
     if (vb) *vb = 0;
+    const uint64_t n = b.n;
     if (n == 0) return 0;
-    if (!bitmap) return fail(SEPO_E_INVAL, "bitmap is NULL");
+    if (!b.bitmap) return fail(SEPO_E_INVAL, "bitmap is NULL");
     const uint64_t nt = sepo_reprobe_tiles(n);
     if (t->tile_counts.grow(nt * 3 * 8)) return fail(SEPO_E_NOMEM, "tile count scratch");
     sync_dev(t);
     if ((rc = zero_ctrl_counters(t))) return rc;
-    rc = sepo_launch_reprobe(t->d, b, t->opts.mode, probe, t->grid, (unsigned long long*)t->tile_counts.p, t->stream);
+    // COMBINE re-probe and every count-only pass never allocate: use a full-occupancy grid.
+    // GROUP re-probe allocates value chunks, so it runs on the allocator slots (one per CTA).
+    const int rgrid = (probe && t->opts.mode == SEPO_GROUP) ? t->grid : 8 * t->n_sms;
+    rc = sepo_launch_reprobe(t->d, b, t->opts.mode, probe, rgrid, (unsigned long long*)t->tile_counts.p, t->stream);
     t->st.kernel_launches += 1;
     if (rc) return cuda_check(t, (cudaError_t)rc, "reprobe kernel launch");
     if ((rc = read_ctrl(t))) return rc;
@@ -411,12 +425,14 @@ static int64_t count_or_probe(sepo_table* t, const uint8_t* keys, const uint64_t
     return (int64_t)t->h_ctrl->postponed;
 }
 
-int64_t sepo_reprobe(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
-                     uint64_t n, uint32_t* bitmap, uint64_t* kb, uint64_t* vb) {
-    int rc = check_active(t);
-    if (rc) return rc;
+// a8 for one batch. COMBINE declines are certified inside the insert kernel (R15), so this is a
+// recount — except under record-mode fault injection, whose declines are not monotone per key.
+// GROUP re-probes every postponed record (its value may fit now; pending keys).
+static int64_t reprobe_impl(sepo_table* t, const Batch& b, uint64_t* kb, uint64_t* vb) {
     CK(t, cudaEventRecord(t->ev0, t->stream));
-    int64_t r = count_or_probe(t, keys, ko, vals, vo, n, bitmap, 1, kb, vb);
+    const bool record_injection = t->opts.fail_alloc_ppm && t->opts.fail_mode == 1;
+    const int probe = (t->opts.mode == SEPO_GROUP || record_injection) ? 1 : 0;
+    int64_t r = count_or_probe(t, b, probe, kb, vb);
     if (r < 0) return r;
     CK(t, cudaEventRecord(t->ev1, t->stream));
     CK(t, cudaEventSynchronize(t->ev1));
@@ -426,26 +442,50 @@ int64_t sepo_reprobe(sepo_table* t, const uint8_t* keys, const uint64_t* ko, con
     return r;
 }
 
+int64_t sepo_reprobe(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
+                     uint64_t n, uint32_t* bitmap, uint64_t* kb, uint64_t* vb) {
+    int rc = check_active(t);
+    if (rc) return rc;
+    Batch b;
+    rc = make_batch(t, b, keys, ko, vals, vo, n, bitmap);
+    if (rc) return rc;
+    return reprobe_impl(t, b, kb, vb);
+}
+
 int64_t sepo_compact(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
                      uint64_t n, const uint32_t* bitmap, uint8_t* ok, uint64_t* oko, uint8_t* ov, uint64_t* ovo) {
     int rc = check_active(t);
     if (rc) return rc;
+    Batch b;
+    rc = make_batch(t, b, keys, ko, vals, vo, n, const_cast<uint32_t*>(bitmap));
+    if (rc) return rc;
     CK(t, cudaEventRecord(t->ev0, t->stream));
     uint64_t kb = 0, vb = 0;
-    int64_t m = count_or_probe(t, keys, ko, vals, vo, n, const_cast<uint32_t*>(bitmap), 0, &kb, &vb);
+    int64_t m = count_or_probe(t, b, 0, &kb, &vb);
     if (m < 0) return m;
-    Batch b;
-    make_batch(t, b, keys, ko, vals, vo, n, const_cast<uint32_t*>(bitmap));
     if (m > 0 && (!ok || (ko && !oko) || (vals && !ov) || (vo && !ovo)))
         return fail(SEPO_E_INVAL, "compaction output buffer is NULL");
-    rc = sepo_launch_compact(b, (unsigned long long*)t->tile_counts.p, ok, oko, ov, ovo, (uint64_t)m, kb, vb, t->grid,
-                             t->stream);
+    rc = sepo_launch_compact(b, (unsigned long long*)t->tile_counts.p, ok, oko, ov, ovo, (uint64_t)m, kb, vb,
+                             8 * t->n_sms, t->stream);
     if (rc) return cuda_check(t, (cudaError_t)rc, "compact kernel launch");
     t->st.kernel_launches += sepo_reprobe_tiles(n) ? 3 : 1;
     CK(t, cudaEventRecord(t->ev1, t->stream));
     CK(t, cudaEventSynchronize(t->ev1));
     t->st.t_compact_ms += elapsed_ms(t->ev0, t->ev1);
     return m;
+}
+
+// a9 by index (sepo_run): the postponed records of batch b as indices into the original arrays
+static int64_t compact_index_impl(sepo_table* t, const Batch& b, uint64_t m, uint64_t* idx_out) {
+    int rc;
+    CK(t, cudaEventRecord(t->ev0, t->stream));
+    rc = sepo_launch_compact_index(b, (unsigned long long*)t->tile_counts.p, idx_out, 8 * t->n_sms, t->stream);
+    if (rc) return cuda_check(t, (cudaError_t)rc, "compact_index kernel launch");
+    t->st.kernel_launches += 2;
+    CK(t, cudaEventRecord(t->ev1, t->stream));
+    CK(t, cudaEventSynchronize(t->ev1));
+    t->st.t_compact_ms += elapsed_ms(t->ev0, t->ev1);
+    return (int64_t)m;
 }
 
 // Pass boundary. honor_retain = 0 evicts every resident page (final export / forced).
@@ -456,6 +496,7 @@ static int64_t evict_impl(sepo_table* t, int honor_retain) {
     if (rc) return cuda_check(t, (cudaError_t)rc, "seal kernel");
     rc = sepo_launch_classify(t->d, honor_retain, t->stream);
     if (rc) return cuda_check(t, (cudaError_t)rc, "classify kernel");
+    CK(t, cudaMemsetAsync(&t->d.ctrl->full, 0, 2 * sizeof(unsigned long long), t->stream));  // full, inflight
     t->st.kernel_launches += 2;
     if ((rc = read_ctrl(t))) return rc;
     const uint64_t ne = t->h_ctrl->n_evict;
@@ -585,8 +626,8 @@ int export_combine(sepo_table* t) {
                     uint32_t klen;
                     memcpy(&klen, base + off + 12, 4);
                     t->x_koffs[k] = kb;
-                    memcpy(&t->x_values[k], base + off + 16, 8);
-                    memcpy(t->x_keys.data() + kb, base + off + CENTRY_HDR, klen);
+                    memcpy(&t->x_values[k], base + off + KEY_OFF + ((klen + 7) & ~7u), 8);
+                    memcpy(t->x_keys.data() + kb, base + off + KEY_OFF, klen);
                     ++k;
                     kb += klen;
                 }
@@ -658,9 +699,9 @@ int export_group(sepo_table* t) {
                 if (kind == K_GKEY) {
                     uint32_t klen, birth;
                     memcpy(&klen, base + off + 12, 4);
-                    memcpy(&birth, base + off + 24, 4);
+                    memcpy(&birth, base + off + KEY_OFF + ((klen + 7) & ~7u) + 8, 4);
                     uint64_t poolo = ((uint64_t)pages[i].page << t->page_shift) + off;
-                    tk[w].push_back({base + off + GKEY_HDR, klen, ((uint64_t)birth << 40) | ((poolo >> 3) + 1)});
+                    tk[w].push_back({base + off + KEY_OFF, klen, ((uint64_t)birth << 40) | ((poolo >> 3) + 1)});
                 } else if (kind == K_VCHUNK) {
                     uint32_t fill, cap;
                     uint64_t owner;
@@ -799,29 +840,25 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
         return sepo_run(t, kdev, ko ? (const uint64_t*)t->in_stage[1].p : nullptr, vdev,
                         vo ? (const uint64_t*)t->in_stage[3].p : nullptr, n);
     }
-    const uint8_t* ck = keys;
-    const uint64_t* cko = ko;
-    const uint8_t* cv = vals;
-    const uint64_t* cvo = vo;
-    uint64_t cn = n;
+    Batch cur;
+    int rc2 = make_batch(t, cur, keys, ko, vals, vo, n, nullptr);
+    if (rc2) return rc2;
     int side = 0;
     int64_t passes_start = (int64_t)t->st.passes;
     uint64_t prev = ~0ull;
-    while (cn > 0) {
-        if (t->bm.grow(((cn + 31) / 32) * 4)) return fail(SEPO_E_NOMEM, "bitmap scratch");
-        uint32_t* bmp = (uint32_t*)t->bm.p;
-        int64_t c = sepo_insert_batch(t, ck, cko, cv, cvo, cn, bmp);
+    while (cur.n > 0) {
+        if (t->bm.grow(((cur.n + 31) / 32) * 4)) return fail(SEPO_E_NOMEM, "bitmap scratch");
+        cur.bitmap = (uint32_t*)t->bm.p;
+        int64_t c = insert_impl(t, cur);
         if (c < 0) return c;
         uint64_t kb = 0, vb = 0;
-        if (c > 0) c = sepo_reprobe(t, ck, cko, cv, cvo, cn, bmp, &kb, &vb);
+        if (c > 0) c = reprobe_impl(t, cur, &kb, &vb);
         if (c < 0) return c;
         if (c == 0) break;
-        DevBuf* o = t->buf[side];
-        if (o[0].grow(kb + 16) || (cko && o[1].grow(((uint64_t)c + 1) * 8)) || (cv && o[2].grow(vb + 16)) ||
-            (cvo && o[3].grow(((uint64_t)c + 1) * 8)))
-            return fail(SEPO_E_NOMEM, "re-issue buffers");
-        int64_t m = sepo_compact(t, ck, cko, cv, cvo, cn, bmp, (uint8_t*)o[0].p, cko ? (uint64_t*)o[1].p : nullptr,
-                                 cv ? (uint8_t*)o[2].p : nullptr, cvo ? (uint64_t*)o[3].p : nullptr);
+        // re-issue by index: the postponed records stay where they are in the caller's arrays
+        if (t->idxb[side].grow((uint64_t)c * 8)) return fail(SEPO_E_NOMEM, "re-issue index list");
+        uint64_t* nidx = (uint64_t*)t->idxb[side].p;
+        int64_t m = compact_index_impl(t, cur, (uint64_t)c, nidx);
         if (m < 0) return m;
         // GROUP: a pass without progress (retained key pages starve the pool) evicts everything
         // (the paper is silent; reading R14)
@@ -833,11 +870,9 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
         prev = (uint64_t)m;
         int64_t e = evict_impl(t, honor);
         if (e < 0) return e;
-        ck = (const uint8_t*)o[0].p;
-        cko = cko ? (const uint64_t*)o[1].p : nullptr;
-        cv = cv ? (const uint8_t*)o[2].p : nullptr;
-        cvo = cvo ? (const uint64_t*)o[3].p : nullptr;
-        cn = (uint64_t)m;
+        cur.idx = nidx;
+        cur.n = (uint64_t)m;
+        t->pending_idx_key_bytes = kb;
         side ^= 1;
         if (t->st.passes - passes_start > 100000) return fail(SEPO_E_STATE, "no progress");
     }
@@ -883,6 +918,9 @@ void sepo_destroy(sepo_table* t) {
     if (t->stream) cudaStreamSynchronize(t->stream);
     if (t->copy_stream) cudaStreamSynchronize(t->copy_stream);
     t->tile_counts.release();
+    t->hot.release();
+    t->idxb[0].release();
+    t->idxb[1].release();
     t->bm.release();
     for (auto& s : t->buf)
         for (auto& b : s) b.release();

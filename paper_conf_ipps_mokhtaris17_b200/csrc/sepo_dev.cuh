@@ -15,11 +15,12 @@
 // relocatable stand-in for the paper's "two pointers ... GPU ... and eventual location in CPU
 // memory". Device code never follows a value-list ref, it only CASes the list head.
 //
-// Every record in a page is 8-byte aligned and starts with a u32 header = size | kind, so an
-// evicted page image is parsed linearly on the host (a filler covers every unused tail):
-//   COMBINE entry       : hdr | next u32 | tag u32 | klen u32 | value u64 | key[pad8]
-//   GROUP key entry     : hdr | next u32 | tag u32 | klen u32 | list_head u64 |
-//                                      birth_gen u32 | pad u32 | key[pad8]
+// Every record in a page is 16-byte aligned and starts with a u32 header = size | kind, so an
+// evicted page image is parsed linearly on the host (a filler covers every unused tail). The
+// first 32 bytes of an entry (header + first 16 key bytes) are fetched with two 16-B vector loads:
+//   COMBINE entry       : hdr | next u32 | tag u32 | klen u32 | key[pad8] | value u64
+//   GROUP key entry     : hdr | next u32 | tag u32 | klen u32 | key[pad8] | list_head u64 |
+//                                      birth_gen u32 | pad u32
 //   GROUP value chunk: hdr | fill u32 | owner u64 | next u64 | cap u32 | vw u32 | values
 //   filler                            : hdr (size of the gap)
 #pragma once
@@ -31,8 +32,7 @@ namespace sepo {
 constexpr uint32_t FULLMASK = 0xffffffffu;
 enum : uint32_t { K_FREE = 0, K_COMBINE = 1, K_FILL = 2, K_DEAD = 3, K_GKEY = 4, K_VCHUNK = 5 };
 constexpr uint32_t KIND_MASK = 7u;
-constexpr uint32_t CENTRY_HDR = 24;  // combine entry header (incl. value)
-constexpr uint32_t GKEY_HDR = 32;    // group key entry header
+constexpr uint32_t KEY_OFF = 16;     // key bytes start here in combine and group key entries
 constexpr uint32_t CHUNK_HDR = 32;   // value chunk header
 constexpr uint32_t NOPAGE = 0xfffffffeu, FULLPAGE = 0xffffffffu;
 constexpr uint32_t PAGE_ENTRY = 1, PAGE_VALUE = 2;
@@ -50,7 +50,9 @@ struct Ctrl {
     unsigned long long n_evict;        // evict: pages in evict_list
     unsigned long long n_free;         // evict: pages in the new free stack
     unsigned long long n_resident;     // evict: pages that stay resident (retained)
-    unsigned long long pad[7];
+    unsigned long long full;           // 1 once the pool ran out this generation: every later allocation fails
+    unsigned long long inflight;       // warps between announcing an allocation and linking it
+    unsigned long long pad[5];
 };
 
 struct Dev {
@@ -84,6 +86,23 @@ __device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long
     asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
+// Publishing CAS / add with release semantics: the entry (or chunk) written before is visible to
+// any thread that reads the new link. Unlike __threadfence() (MEMBAR.SC + CCTL.IVALL on sm_100),
+// a release RMW does not invalidate L1, which holds the streamed input keys.
+__device__ __forceinline__ uint32_t cas_release(uint32_t* p, uint32_t cmp, uint32_t val) {
+    uint32_t old;
+    asm volatile("atom.release.gpu.global.cas.b32 %0, [%1], %2, %3;" : "=r"(old) : "l"(p), "r"(cmp), "r"(val) : "memory");
+    return old;
+}
+__device__ __forceinline__ unsigned long long cas_release64(unsigned long long* p, unsigned long long cmp,
+                                                            unsigned long long val) {
+    unsigned long long old;
+    asm volatile("atom.release.gpu.global.cas.b64 %0, [%1], %2, %3;" : "=l"(old) : "l"(p), "l"(cmp), "l"(val) : "memory");
+    return old;
+}
+__device__ __forceinline__ void add_release64(unsigned long long* p, unsigned long long v) {
+    asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 // L2-coherent loads of published entry fields (never stale L1 lines)
 __device__ __forceinline__ uint64_t ldcg64(const void* p) { return __ldcg(reinterpret_cast<const unsigned long long*>(p)); }
 __device__ __forceinline__ uint32_t ldcg32(const void* p) { return __ldcg(reinterpret_cast<const unsigned int*>(p)); }
@@ -106,13 +125,17 @@ __device__ __forceinline__ uint64_t fmix64(uint64_t k) {
     k ^= k >> 33; k *= 0xc4ceb9fe1a85ec53ull;
     k ^= k >> 33; return k;
 }
+// h = fmix64(fold over the key's 8-byte LE words (zero padded), seeded with the length)
+__device__ __forceinline__ uint64_t hash_init(uint32_t len, uint64_t seed) { return seed ^ ((uint64_t)len * 0x87c37b91114253d5ull); }
+__device__ __forceinline__ uint64_t hash_word(uint64_t h, uint64_t w) {
+    h ^= w * 0x4cf5ad432745937full;
+    return ((h << 29) | (h >> 35)) * 0x9e3779b97f4a7c15ull + 0x52dce729ull;
+}
 __device__ __forceinline__ uint64_t hash_key(const uint8_t* p, uint32_t len, uint64_t seed) {
-    uint64_t h = seed ^ ((uint64_t)len * 0x87c37b91114253d5ull);
+    uint64_t h = hash_init(len, seed);
     for (uint32_t o = 0; o < len; o += 8) {
         uint32_t nb = len - o < 8 ? len - o : 8;
-        uint64_t w = load_in_word(p + o, nb);
-        h ^= w * 0x4cf5ad432745937full;
-        h = ((h << 29) | (h >> 35)) * 0x9e3779b97f4a7c15ull + 0x52dce729ull;
+        h = hash_word(h, load_in_word(p + o, nb));
     }
     return fmix64(h);
 }
@@ -122,6 +145,12 @@ __device__ __forceinline__ uint32_t bucket_of(uint64_t h, uint64_t n_buckets) {
 __device__ __forceinline__ uint32_t tag_of(uint64_t h) { return (uint32_t)h; }
 
 __device__ __forceinline__ uint32_t align8(uint32_t x) { return (x + 7u) & ~7u; }
+__device__ __forceinline__ uint32_t align16(uint32_t x) { return (x + 15u) & ~15u; }
+// entry sizes (16-byte aligned records)
+__device__ __forceinline__ uint32_t centry_size(uint32_t klen) { return align16(KEY_OFF + align8(klen) + 8u); }
+__device__ __forceinline__ uint32_t gkey_size(uint32_t klen) { return align16(KEY_OFF + align8(klen) + 16u); }
+// value (COMBINE) / list head (GROUP) of an entry with key length klen
+__device__ __forceinline__ uint8_t* entry_val(uint8_t* e, uint32_t klen) { return e + KEY_OFF + align8(klen); }
 __device__ __forceinline__ uint8_t* ref_ptr(const Dev& d, uint32_t ref) { return d.pool + ((uint64_t)(ref - 1) << 3); }
 __device__ __forceinline__ uint32_t off_ref(uint64_t off) { return (uint32_t)(off >> 3) + 1u; }
 
@@ -149,19 +178,56 @@ __device__ __forceinline__ void store_key(uint8_t* ek, const uint8_t* p, uint32_
     }
 }
 
-// Walk the chain [ref .. stop) for an entry with (tag, len, key). koff = key offset in entry.
+__device__ __forceinline__ uint4 ldcg128(const void* p) { return __ldcg(reinterpret_cast<const uint4*>(p)); }
+__device__ __forceinline__ ulonglong2 ldcg128u(const void* p) { return __ldcg(reinterpret_cast<const ulonglong2*>(p)); }
+
+// Walk the chain [ref .. stop) for an entry with (tag, len, key) — key given by its INPUT bytes.
 // Only entries of the resident generation are reachable (head insertion; the directory
 // is reset at every pass boundary).
 __device__ __forceinline__ uint8_t* chain_find(const Dev& d, uint32_t ref, uint32_t stop, uint32_t tag, uint32_t len,
-                                               const uint8_t* key, uint32_t koff) {
+                                               const uint8_t* key) {
     while (ref != 0 && ref != stop) {
         uint8_t* e = ref_ptr(d, ref);
-        uint64_t w0 = ldcg64(e);      // hdr | next
-        uint64_t w1 = ldcg64(e + 8);  // tag | klen
-        if ((uint32_t)w1 == tag && (uint32_t)(w1 >> 32) == len && entry_key_eq(e + koff, key, len)) return e;
-        ref = (uint32_t)(w0 >> 32);
+        const uint4 hd = ldcg128(e);  // hdr | next | tag | klen
+        if (hd.z == tag && hd.w == len && entry_key_eq(e + KEY_OFF, key, len)) return e;
+        ref = hd.y;
     }
     return nullptr;
+}
+// Same, with the key's first 16 bytes in registers (w0, w1 zero padded); bytes >= 16 of a long
+// key are compared against `tail` (the input key + 16).
+__device__ __forceinline__ uint8_t* chain_find_w(const Dev& d, uint32_t ref, uint32_t stop, uint32_t tag, uint32_t len,
+                                                 uint64_t w0, uint64_t w1, const uint8_t* tail) {
+    while (ref != 0 && ref != stop) {
+        uint8_t* e = ref_ptr(d, ref);
+        const uint4 hd = ldcg128(e);
+        const ulonglong2 kw = ldcg128u(e + KEY_OFF);
+        if (hd.z == tag && hd.w == len && (len == 0 || kw.x == w0) && (len <= 8 || kw.y == w1) &&
+            (len <= 16 || entry_key_eq(e + KEY_OFF + 16, tail, len - 16)))
+            return e;
+        ref = hd.y;
+    }
+    return nullptr;
+}
+// First 16 bytes of an input key as two zero-padded LE words (at most 3 aligned loads).
+__device__ __forceinline__ void load_key16(const uint8_t* p, uint32_t len, uint64_t& w0, uint64_t& w1) {
+    w0 = 0; w1 = 0;
+    if (len == 0) return;
+    const uintptr_t a = reinterpret_cast<uintptr_t>(p);
+    const uint32_t sh = (uint32_t)(a & 7u);
+    const unsigned long long* q = reinterpret_cast<const unsigned long long*>(a - sh);
+    const uint32_t nb = len < 16 ? len : 16;
+    const uint32_t nw = (sh + nb + 7) >> 3;  // aligned words touched (1..3)
+    const uint64_t x0 = __ldg(q);
+    const uint64_t x1 = nw > 1 ? __ldg(q + 1) : 0ull;
+    const uint64_t x2 = nw > 2 ? __ldg(q + 2) : 0ull;
+    if (sh == 0) { w0 = x0; w1 = x1; }
+    else {
+        w0 = (x0 >> (8 * sh)) | (x1 << (64 - 8 * sh));
+        w1 = (x1 >> (8 * sh)) | (x2 << (64 - 8 * sh));
+    }
+    if (nb < 8) { w0 &= (1ull << (8 * nb)) - 1ull; w1 = 0; }
+    else if (nb < 16) w1 &= (1ull << (8 * (nb - 8))) - 1ull;
 }
 
 // ---------------------------------------------------------------- fault injection (tests only)
@@ -185,6 +251,12 @@ __device__ __forceinline__ uint64_t warp_alloc(const Dev& d, unsigned long long*
     const uint32_t PB = d.page_bytes;
     uint64_t result = ~0ull;
     bool pending = need;
+    // failure is monotone for the whole generation: once the pool ran out, nobody allocates
+    if (__any_sync(FULLMASK, pending)) {
+        unsigned long long full = 0;
+        if (lane == 0) full = ld_relaxed_u64(&d.ctrl->full);
+        if (__shfl_sync(FULLMASK, full, 0) != 0ull) return ~0ull;  // warp-uniform decision
+    }
     while (true) {
         unsigned pm = __ballot_sync(FULLMASK, pending);
         if (!pm) break;
@@ -222,6 +294,7 @@ __device__ __forceinline__ uint64_t warp_alloc(const Dev& d, unsigned long long*
                         nw = (unsigned long long)np << 32;
                     } else {
                         nw = (unsigned long long)FULLPAGE << 32;
+                        atomicExch(&d.ctrl->full, 1ull);
                     }
                     __threadfence_block();
                     atomicExch(scur, nw);

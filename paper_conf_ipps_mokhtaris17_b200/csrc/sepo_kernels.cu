@@ -15,13 +15,13 @@
 // table with one thread per key.
 #include "sepo_dev.cuh"
 #include "sepo_kernels.h"
+#include <algorithm>
 
 namespace sepo {
 
 constexpr uint32_t EMPTY = 0xffffffffu;
 
 template <int MODE> struct Cfg;
-template <> struct Cfg<0> { static constexpr int THREADS = 512, TILE = 2048, NSLOT = 4096; };  // COMBINE
 template <> struct Cfg<1> { static constexpr int THREADS = 512, TILE = 1024, NSLOT = 2048; };  // GROUP
 
 template <int MODE>
@@ -47,9 +47,12 @@ struct Smem {
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31u; }
 __device__ __forceinline__ uint32_t lanemask_lt() { return (1u << lane_id()) - 1u; }
 
+// record i of a batch -> its index in keys / key_offsets / vals (re-issue by index, a9)
+__device__ __forceinline__ uint64_t rec_index(const Batch& b, uint64_t i) { return b.idx ? __ldg(reinterpret_cast<const unsigned long long*>(b.idx) + i) : i; }
 // value of record i for COMBINE (vw bytes LE, or 1 when vals == nullptr)
 __device__ __forceinline__ uint64_t rec_value(const Batch& b, uint64_t i) {
     if (b.vals == nullptr) return 1ull;
+    i = rec_index(b, i);
     switch (b.vw) {
         case 8: return __ldg(reinterpret_cast<const unsigned long long*>(b.vals) + i);
         case 4: return __ldg(reinterpret_cast<const unsigned int*>(b.vals) + i);
@@ -58,6 +61,7 @@ __device__ __forceinline__ uint64_t rec_value(const Batch& b, uint64_t i) {
     }
 }
 __device__ __forceinline__ void rec_key(const Batch& b, uint64_t i, uint64_t& s, uint32_t& len) {
+    i = rec_index(b, i);
     if (b.ko) {
         s = __ldg(reinterpret_cast<const unsigned long long*>(b.ko) + i);
         len = (uint32_t)(__ldg(reinterpret_cast<const unsigned long long*>(b.ko) + i + 1) - s);
@@ -68,6 +72,7 @@ __device__ __forceinline__ void rec_key(const Batch& b, uint64_t i, uint64_t& s,
 }
 // GROUP value bytes of record i
 __device__ __forceinline__ void rec_val_span(const Batch& b, uint64_t i, uint64_t& s, uint32_t& len) {
+    i = rec_index(b, i);
     if (b.vo) {
         s = __ldg(reinterpret_cast<const unsigned long long*>(b.vo) + i);
         len = (uint32_t)(__ldg(reinterpret_cast<const unsigned long long*>(b.vo) + i + 1) - s);
@@ -86,14 +91,17 @@ __device__ __forceinline__ uint32_t chunk_cap(const Dev& d, uint32_t k, uint32_t
     c = max(c, k);
     return min(c, (d.page_bytes - CHUNK_HDR) / slot_bytes);
 }
-__device__ __forceinline__ uint32_t chunk_bytes(uint32_t cap, uint32_t slot_bytes) { return CHUNK_HDR + align8(cap * slot_bytes); }
+__device__ __forceinline__ uint32_t chunk_bytes(uint32_t cap, uint32_t slot_bytes) { return align16(CHUNK_HDR + cap * slot_bytes); }
 __device__ __forceinline__ uint64_t vref_of(const Dev& d, uint64_t off) { return ((uint64_t)d.gen << 40) | (uint64_t)off_ref(off); }
 __device__ __forceinline__ bool vref_resident(const Dev& d, uint64_t vref) { return vref != 0 && (uint32_t)(vref >> 40) == d.gen; }
 __device__ __forceinline__ uint8_t* vref_ptr(const Dev& d, uint64_t vref) { return ref_ptr(d, (uint32_t)vref); }
 // owner identity of a key entry: birth generation << 40 | entry ref
 __device__ __forceinline__ uint64_t owner_of(const Dev& d, uint8_t* e) {
-    uint32_t birth = ldcg32(e + 24);
+    uint32_t birth = ldcg32(entry_val(e, ldcg32(e + 12)) + 8);
     return ((uint64_t)birth << 40) | (uint64_t)off_ref((uint64_t)(e - d.pool));
+}
+__device__ __forceinline__ unsigned long long* list_head(uint8_t* e) {
+    return reinterpret_cast<unsigned long long*>(entry_val(e, ldcg32(e + 12)));
 }
 __device__ __forceinline__ void init_chunk(uint8_t* c, uint32_t cap, uint32_t vwslot, uint32_t fill, uint64_t owner,
                                            uint64_t next) {
@@ -106,11 +114,10 @@ __device__ __forceinline__ void init_chunk(uint8_t* c, uint32_t cap, uint32_t vw
 }
 // push chunk `cref` (already holding its values' slots) onto the list head of key entry e
 __device__ __forceinline__ void push_chunk(uint8_t* e, uint8_t* c, uint64_t cref, uint64_t observed) {
-    unsigned long long* head = reinterpret_cast<unsigned long long*>(e + 16);
+    unsigned long long* head = list_head(e);
     while (true) {
         *reinterpret_cast<unsigned long long*>(c + 16) = observed;
-        __threadfence();
-        unsigned long long old = atomicCAS(head, observed, cref);
+        unsigned long long old = cas_release64(head, observed, cref);
         if (old == observed) return;
         observed = old;
     }
@@ -119,7 +126,7 @@ __device__ __forceinline__ void push_chunk(uint8_t* e, uint8_t* c, uint64_t cref
 // the chunk ref in *cref and the first slot in *base; *head_out = observed head, *prev_cap.
 __device__ __forceinline__ uint32_t reserve_head(const Dev& d, uint8_t* e, uint32_t k, uint64_t* cref, uint32_t* base,
                                                  uint64_t* head_out, uint32_t* prev_cap) {
-    uint64_t h = ld_relaxed_u64(reinterpret_cast<const unsigned long long*>(e + 16));
+    uint64_t h = ld_relaxed_u64(list_head(e));
     *head_out = h;
     *prev_cap = 0;
     *cref = 0;
@@ -265,21 +272,20 @@ __global__ void __launch_bounds__(Cfg<MODE>::THREADS, 2) insert_kernel(Dev d, Ba
             const uint8_t* key = b.keys + s;
             const uint32_t bkt = act ? bucket_of(h, d.n_buckets) : 0;
             const uint32_t tag = tag_of(h);
-            const uint32_t koff = MODE == 0 ? CENTRY_HDR : GKEY_HDR;
             uint32_t head = 0;
             uint8_t* found = nullptr;
             if (act) {
                 head = ld_relaxed_u32(d.dir + bkt);
-                found = chain_find(d, head, 0, tag, len, key, koff);
+                found = chain_find(d, head, 0, tag, len, key);
             }
             uint32_t res = R_OK;
-            const uint32_t esize = koff + align8(len);
+            const uint32_t esize = MODE == 0 ? centry_size(len) : gkey_size(len);
             bool need = act && !found;
             if (need && (len > 65535u - 64u || esize > PB)) { need = false; res = R_TOOLARGE; }
             if (need && inject_fail(d, h, t0 + r)) { need = false; res = R_POST; }
 
             if (MODE == 0) {
-                if (act && found) atomicAdd(reinterpret_cast<unsigned long long*>(found + 16), (unsigned long long)sum);
+                if (act && found) atomicAdd(reinterpret_cast<unsigned long long*>(entry_val(found, len)), (unsigned long long)sum);
                 const uint64_t off = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
                 if (need) {
                     if (off == ~0ull) {
@@ -290,23 +296,21 @@ __global__ void __launch_bounds__(Cfg<MODE>::THREADS, 2) insert_kernel(Dev d, Ba
                         *reinterpret_cast<uint32_t*>(e + 4) = head;
                         *reinterpret_cast<uint32_t*>(e + 8) = tag;
                         *reinterpret_cast<uint32_t*>(e + 12) = len;
-                        *reinterpret_cast<unsigned long long*>(e + 16) = sum;
-                        store_key(e + CENTRY_HDR, key, len);
-                        __threadfence();
+                        store_key(e + KEY_OFF, key, len);
+                        *reinterpret_cast<unsigned long long*>(entry_val(e, len)) = sum;
                         const uint32_t me = off_ref(off);
                         while (true) {  // lock-free head insertion
-                            const uint32_t old = atomicCAS(d.dir + bkt, head, me);
+                            const uint32_t old = cas_release(d.dir + bkt, head, me);
                             if (old == head) break;
-                            uint8_t* w = chain_find(d, old, head, tag, len, key, CENTRY_HDR);
+                            uint8_t* w = chain_find(d, old, head, tag, len, key);
                             if (w) {  // the key was linked meanwhile: combine there, retire ours
-                                atomicAdd(reinterpret_cast<unsigned long long*>(w + 16), (unsigned long long)sum);
+                                atomicAdd(reinterpret_cast<unsigned long long*>(entry_val(w, len)), (unsigned long long)sum);
                                 *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
                                 atomicAdd(&S.dead, (unsigned long long)esize);
                                 break;
                             }
                             head = old;
                             *reinterpret_cast<uint32_t*>(e + 4) = head;
-                            __threadfence();
                         }
                     }
                 }
@@ -342,17 +346,16 @@ __global__ void __launch_bounds__(Cfg<MODE>::THREADS, 2) insert_kernel(Dev d, Ba
                     *reinterpret_cast<uint32_t*>(ne + 4) = head;
                     *reinterpret_cast<uint32_t*>(ne + 8) = tag;
                     *reinterpret_cast<uint32_t*>(ne + 12) = len;
-                    *reinterpret_cast<unsigned long long*>(ne + 16) = 0ull;
-                    *reinterpret_cast<uint32_t*>(ne + 24) = d.gen;
-                    *reinterpret_cast<uint32_t*>(ne + 28) = 0u;
-                    store_key(ne + GKEY_HDR, key, len);
-                    __threadfence();
-                    const uint32_t me = off_ref(koffp);
+                    store_key(ne + KEY_OFF, key, len);
+                    *reinterpret_cast<unsigned long long*>(entry_val(ne, len)) = 0ull;
+                    *reinterpret_cast<uint32_t*>(entry_val(ne, len) + 8) = d.gen;
+                    *reinterpret_cast<uint32_t*>(entry_val(ne, len) + 12) = 0u;
+                                        const uint32_t me = off_ref(koffp);
                     e = ne;
                     while (true) {
-                        const uint32_t old = atomicCAS(d.dir + bkt, head, me);
+                        const uint32_t old = cas_release(d.dir + bkt, head, me);
                         if (old == head) break;
-                        uint8_t* w = chain_find(d, old, head, tag, len, key, GKEY_HDR);
+                        uint8_t* w = chain_find(d, old, head, tag, len, key);
                         if (w) {
                             *reinterpret_cast<uint32_t*>(ne) = esize | K_DEAD;
                             atomicAdd(&S.dead, (unsigned long long)esize);
@@ -361,14 +364,13 @@ __global__ void __launch_bounds__(Cfg<MODE>::THREADS, 2) insert_kernel(Dev d, Ba
                         }
                         head = old;
                         *reinterpret_cast<uint32_t*>(ne + 4) = head;
-                        __threadfence();
                     }
                 }
                 if (want_chunk && coff != ~0ull) {
                     uint8_t* c = d.pool + coff;
                     const uint64_t cref = vref_of(d, coff);
                     init_chunk(c, ccap, vws, rest, owner_of(d, e), 0ull);
-                    push_chunk(e, c, cref, ld_relaxed_u64(reinterpret_cast<const unsigned long long*>(e + 16)));
+                    push_chunk(e, c, cref, ld_relaxed_u64(list_head(e)));
                     b_ref = cref;
                 } else if (want_chunk) {
                     b_ref = 0;  // rest of the values are postponed (key stays resident: pending)
@@ -437,6 +439,414 @@ __global__ void __launch_bounds__(Cfg<MODE>::THREADS, 2) insert_kernel(Dev d, Ba
     }
 }
 
+// ================================================================ COMBINE insert (a1..a7): hot set + streaming warps
+// Zipf inputs put most records on a few keys (C2: the top 2048 words are 52 % of all words), and
+// same-address global atomics serialise (the paper's Word Count contention).
+// So a COMBINE batch runs in two steps:
+//   (i)  hot-set discovery: a strided sample of the batch is counted in a scratch table; the
+//        keys whose sample count clears a threshold (at most HOT_K of them) are looked up or
+//        inserted in the table (value 0), giving their resident entry refs;
+//   (ii) insert_stream_kernel: one CTA per SM loads the hot set into shared memory (read-only
+//        for the whole launch) next to a pending-sum array; every warp then streams 32-record
+//        groups with no CTA barrier: key words + hash in registers, __match_any_sync folds equal
+//        keys of the warp, the leader adds to the hot key's pending sum in shared memory, or
+//        walks the global chain (red.add on a hit; allocate + CAS-link on a miss; POSTPONE if the
+//        pool is exhausted), and a __ballot_sync writes the bitmap word. Pending sums are added to
+//        the global entries when the CTA finishes (hot entries are resident for the whole
+//        generation, so each record's SUCCESS is final).
+namespace hot {
+constexpr int K = 2048;          // hot keys at most
+constexpr int NB = 1024;         // shared buckets of 4 slots (2-choice): constant-time probe
+constexpr int NH = 4 * NB;       // slots
+constexpr uint32_t EMPTY_LEN = 0xffffffffu;
+__device__ __forceinline__ uint32_t fp(uint64_t h) { return (uint32_t)(h >> 32) | 1u; }  // 0 = empty
+__device__ __forceinline__ uint32_t b1(uint64_t h) { return (uint32_t)(h >> 3) & (NB - 1); }
+__device__ __forceinline__ uint32_t b2(uint64_t h) { return (uint32_t)(h >> 13) & (NB - 1); }
+constexpr int SAMPLE_SLOTS = 1 << 20;  // global scratch table for the sample
+struct Entry {                   // one hot key (global list, built by hot_select / hot_resolve)
+    uint64_t h, w0, w1;
+    uint32_t len, ref;           // ref = resident entry (0: not usable)
+    uint64_t src;                // input byte offset of a representative record (tail bytes)
+};
+struct SampleSlot { unsigned long long h; unsigned int count, rec; };
+}  // namespace hot
+
+__device__ __forceinline__ void red_add_u64(unsigned long long* p, unsigned long long v) {
+    asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// hash + first 16 key bytes of record i
+__device__ __forceinline__ void rec_hash16(const Dev& d, const Batch& b, uint64_t i, uint64_t& s, uint32_t& len,
+                                           uint64_t& w0, uint64_t& w1, uint64_t& h) {
+    rec_key(b, i, s, len);
+    const uint8_t* p = b.keys + s;
+    load_key16(p, len, w0, w1);
+    uint64_t x = hash_init(len, d.seed);
+    if (len > 0) x = hash_word(x, w0);
+    if (len > 8) x = hash_word(x, w1);
+    for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(p + o, len - o < 8 ? len - o : 8));
+    h = fmix64(x);
+}
+
+// (i-a) count a strided sample of the batch: record i = j * stride
+__global__ void __launch_bounds__(256) hot_sample_kernel(Dev d, Batch b, uint64_t stride, uint64_t n_sample,
+                                                         hot::SampleSlot* tab) {
+    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < n_sample; j += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t i = j * stride;
+        uint64_t s, w0, w1, h; uint32_t len;
+        rec_hash16(d, b, i, s, len, w0, w1, h);
+        const unsigned long long key = h | 1ull;  // 0 marks an empty slot
+        uint32_t pos = (uint32_t)(h >> 20) & (hot::SAMPLE_SLOTS - 1);
+        for (int probe = 0; probe < 32; ++probe) {
+            const unsigned long long cur = atomicCAS(&tab[pos].h, 0ull, key);
+            if (cur == 0ull) { tab[pos].rec = (unsigned)(i & 0xffffffffu); atomicAdd(&tab[pos].count, 1u); break; }
+            if (cur == key) { atomicAdd(&tab[pos].count, 1u); break; }
+            pos = (pos + 1) & (hot::SAMPLE_SLOTS - 1);
+        }
+    }
+}
+
+// (i-b) one CTA: threshold = smallest count such that at most K keys reach it; emit those keys.
+// (Hash-identified: two keys with the same 64-bit hash would share a sample slot; the hot set is
+// only a cache, so a wrong pick costs speed, never correctness — entries are matched on bytes.)
+__global__ void __launch_bounds__(1024) hot_select_kernel(Dev d, Batch b, const hot::SampleSlot* tab, hot::Entry* out,
+                                                          unsigned int* n_out, uint32_t min_count) {
+    __shared__ unsigned int hist[4096];
+    __shared__ unsigned int s_thr, s_n;
+    for (int i = threadIdx.x; i < 4096; i += blockDim.x) hist[i] = 0;
+    if (threadIdx.x == 0) { s_n = 0; s_thr = 0xffffffffu; }
+    __syncthreads();
+    for (int i = threadIdx.x; i < hot::SAMPLE_SLOTS; i += blockDim.x) {
+        const unsigned c = tab[i].count;
+        if (tab[i].h != 0ull && c >= min_count) atomicAdd(&hist[min(c, 4095u)], 1u);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        unsigned acc = 0, thr = 0xffffffffu;
+        for (int c = 4095; c >= (int)min_count; --c) {
+            if (acc + hist[c] > (unsigned)hot::K) break;
+            acc += hist[c];
+            thr = c;
+        }
+        s_thr = thr;
+    }
+    __syncthreads();
+    const unsigned thr = s_thr;
+    for (int i = threadIdx.x; i < hot::SAMPLE_SLOTS; i += blockDim.x) {
+        const unsigned c = tab[i].count;
+        if (tab[i].h != 0ull && c >= thr && thr != 0xffffffffu) {
+            const unsigned j = atomicAdd(&s_n, 1u);
+            if (j < (unsigned)hot::K) {
+                uint64_t s, w0, w1, h; uint32_t len;
+                rec_hash16(d, b, tab[i].rec, s, len, w0, w1, h);
+                hot::Entry e;
+                e.h = h; e.w0 = w0; e.w1 = w1; e.len = len; e.ref = 0; e.src = s;
+                out[j] = e;
+            }
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) *n_out = min(s_n, (unsigned)hot::K);
+}
+
+// (i-c) one CTA on allocator slot 0: look up / insert (value 0) every hot key
+__global__ void __launch_bounds__(1024) hot_resolve_kernel(Dev d, Batch b, hot::Entry* list, const unsigned int* n_list) {
+    __shared__ unsigned long long s_cur;
+    __shared__ unsigned long long s_dead;
+    if (threadIdx.x == 0) { s_cur = d.cursors[0]; s_dead = 0; }
+    __syncthreads();
+    const unsigned n = *n_list;
+    for (unsigned j0 = 0; j0 < n; j0 += blockDim.x) {
+        const unsigned j = j0 + threadIdx.x;
+        const bool act = j < n;
+        hot::Entry e = act ? list[j] : hot::Entry{};
+        const uint8_t* tail = b.keys + e.src + 16;
+        const uint32_t bkt = act ? bucket_of(e.h, d.n_buckets) : 0;
+        const uint32_t tag = tag_of(e.h);
+        uint32_t head = 0;
+        uint8_t* found = nullptr;
+        if (act) {
+            head = ld_relaxed_u32(d.dir + bkt);
+            found = chain_find_w(d, head, 0, tag, e.len, e.w0, e.w1, tail);
+        }
+        const uint32_t esize = centry_size(e.len);
+        bool need = act && !found && e.len <= 65535u - 64u && esize <= d.page_bytes && !inject_fail(d, e.h, j);
+        uint32_t ref = found ? off_ref((uint64_t)(found - d.pool)) : 0u;
+        const uint64_t off = warp_alloc(d, &s_cur, need, esize, (uint8_t)PAGE_ENTRY);
+        if (need && off != ~0ull) {
+            uint8_t* ne = d.pool + off;
+            *reinterpret_cast<uint4*>(ne) = make_uint4(esize | K_COMBINE, head, tag, e.len);
+            if (e.len > 0) *reinterpret_cast<unsigned long long*>(ne + KEY_OFF) = e.w0;
+            if (e.len > 8) *reinterpret_cast<unsigned long long*>(ne + KEY_OFF + 8) = e.w1;
+            if (e.len > 16) store_key(ne + KEY_OFF + 16, tail, e.len - 16);
+            *reinterpret_cast<unsigned long long*>(entry_val(ne, e.len)) = 0ull;
+            ref = off_ref(off);
+            while (true) {
+                const uint32_t old = cas_release(d.dir + bkt, head, ref);
+                if (old == head) break;
+                uint8_t* w = chain_find_w(d, old, head, tag, e.len, e.w0, e.w1, tail);
+                if (w) {
+                    *reinterpret_cast<uint32_t*>(ne) = esize | K_DEAD;
+                    atomicAdd(&s_dead, (unsigned long long)esize);
+                    ref = off_ref((uint64_t)(w - d.pool));
+                    break;
+                }
+                head = old;
+                *reinterpret_cast<uint32_t*>(ne + 4) = head;
+            }
+        }
+        if (act) list[j].ref = ref;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        d.cursors[0] = s_cur;
+        if (s_dead) atomicAdd(&d.ctrl->dead_bytes, s_dead);
+    }
+}
+
+namespace stream {
+constexpr int THREADS = 1024;
+constexpr int SUB = 1;  // 32-record groups per warp step
+struct Smem {
+    uint4 tags[hot::NB];  // 4 fingerprints per bucket (one 16-B load per probed bucket)
+    uint64_t h[hot::NH], w0[hot::NH], w1[hot::NH];
+    uint32_t len[hot::NH], ref[hot::NH];
+    unsigned int plo[hot::NH], phi[hot::NH];  // pending sum = phi:plo (exact via carry)
+    unsigned long long cur[2];
+    unsigned long long post, toolarge, dead;
+};
+}  // namespace stream
+
+__device__ __forceinline__ void smem_add_u64(unsigned int* lo, unsigned int* hi, uint64_t v) {
+    const unsigned int vl = (unsigned int)v;
+    const unsigned int old = atomicAdd(lo, vl);
+    const unsigned int carry = (old + vl < old) ? 1u : 0u;
+    const unsigned int vh = (unsigned int)(v >> 32) + carry;
+    if (vh) atomicAdd(hi, vh);
+}
+
+template <bool VALS>
+__global__ void __launch_bounds__(stream::THREADS, 1) insert_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
+                                                                           const unsigned int* n_hot) {
+    using stream::THREADS;
+    using stream::SUB;
+    extern __shared__ __align__(16) uint8_t smem_raw[];
+    stream::Smem& S = *reinterpret_cast<stream::Smem*>(smem_raw);
+    const uint32_t tid = threadIdx.x, lane = lane_id();
+    const uint32_t PB = d.page_bytes;
+    for (int p = tid; p < hot::NH; p += THREADS) { S.len[p] = hot::EMPTY_LEN; S.plo[p] = 0; S.phi[p] = 0; }
+    for (int p = tid; p < hot::NB; p += THREADS) S.tags[p] = make_uint4(0, 0, 0, 0);
+    if (tid == 0) {
+        S.cur[0] = d.cursors[2 * blockIdx.x];
+        S.cur[1] = d.cursors[2 * blockIdx.x + 1];
+        S.post = 0; S.toolarge = 0; S.dead = 0;
+    }
+    __syncthreads();
+    // load the hot set (read-only during the main loop)
+    const unsigned nh = hl ? *n_hot : 0u;
+    for (unsigned j = tid; j < nh; j += THREADS) {
+        const hot::Entry e = hl[j];
+        if (e.ref == 0) continue;
+        // claim a free slot in bucket b1, else b2, else leave the key out (the set is only a cache)
+        const uint32_t f = hot::fp(e.h);
+        int pos = -1;
+        for (int c = 0; c < 2 && pos < 0; ++c) {
+            const uint32_t bk = c == 0 ? hot::b1(e.h) : hot::b2(e.h);
+            uint32_t* t = reinterpret_cast<uint32_t*>(&S.tags[bk]);
+            for (int w = 0; w < 4 && pos < 0; ++w)
+                if (atomicCAS(&t[w], 0u, f) == 0u) pos = (int)(bk * 4 + w);
+        }
+        if (pos < 0) continue;
+        S.h[pos] = e.h; S.w0[pos] = e.w0; S.w1[pos] = e.w1; S.ref[pos] = e.ref; S.len[pos] = e.len;
+    }
+    __syncthreads();
+    const bool have_hot = nh > 0;
+
+    const uint64_t ngroups = (b.n + 31) / 32;
+    const uint64_t gw = (uint64_t)blockIdx.x * (THREADS / 32) + (tid >> 5);
+    const uint64_t nw = (uint64_t)gridDim.x * (THREADS / 32);
+    unsigned long long c_post = 0, c_tl = 0, c_dead = 0;
+    bool w_full = false, w_quiet = false;  // warp-uniform: pool ran out / quiescence observed
+    for (uint64_t g0 = gw * SUB; g0 < ngroups; g0 += nw * SUB) {
+        uint64_t s[SUB], w0[SUB], w1[SUB], h[SUB], v[SUB];
+        uint32_t len[SUB];
+        bool valid[SUB];
+#pragma unroll
+        for (int q = 0; q < SUB; ++q) {
+            const uint64_t i = (g0 + q) * 32 + lane;
+            valid[q] = i < b.n;
+            s[q] = 0; len[q] = 0; w0[q] = 0; w1[q] = 0; h[q] = 0; v[q] = 0;
+            if (valid[q]) {
+                rec_hash16(d, b, i, s[q], len[q], w0[q], w1[q], h[q]);
+                if (VALS) v[q] = rec_value(b, i);
+            }
+        }
+#pragma unroll
+        for (int q = 0; q < SUB; ++q) {
+            const unsigned vm = __ballot_sync(FULLMASK, valid[q]);
+            if (vm == 0) continue;  // warp-uniform
+            // ---- fold equal keys of the warp (a2)
+            // fold on 32 hash bits; equal keys are then confirmed on bytes (collisions stay apart)
+            const unsigned hh = valid[q] ? (unsigned)h[q] : (0x80000000u | lane);
+            const unsigned grp = __match_any_sync(FULLMASK, hh) & vm;
+            const uint32_t leader = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
+            const uint64_t lw0 = __shfl_sync(FULLMASK, w0[q], leader);
+            const uint64_t lw1 = __shfl_sync(FULLMASK, w1[q], leader);
+            const uint32_t llen = __shfl_sync(FULLMASK, len[q], leader);
+            const uint64_t ls = __shfl_sync(FULLMASK, s[q], leader);
+            const bool eq = valid[q] && (lane == leader ||
+                                         (len[q] == llen && w0[q] == lw0 && w1[q] == lw1 &&
+                                          (len[q] <= 16 || in_key_eq(b.keys + s[q] + 16, b.keys + ls + 16, len[q] - 16))));
+            const unsigned joined = grp & __ballot_sync(FULLMASK, eq);
+            const bool ins = valid[q] && (lane == leader || !eq);
+            uint64_t contrib;
+            if (!VALS) {
+                contrib = (lane == leader) ? (uint64_t)__popc(joined) : 1ull;
+            } else {
+                uint64_t acc = v[q];
+                if (__any_sync(FULLMASK, __popc(joined) > 1)) {
+                    acc = 0;
+                    for (int x = 0; x < 32; ++x) {
+                        const uint64_t vx = __shfl_sync(FULLMASK, v[q], x);
+                        if ((joined >> x) & 1u) acc += vx;
+                    }
+                }
+                contrib = (lane == leader) ? acc : v[q];
+            }
+            // ---- hot set (shared memory, read-only keys)
+            bool done = !ins;
+            if (ins && have_hot) {
+                const uint32_t f = hot::fp(h[q]);
+                const uint32_t k1 = hot::b1(h[q]), k2 = hot::b2(h[q]);
+                const uint4 t1 = S.tags[k1], t2 = S.tags[k2];
+                int pos = -1;
+                if (t1.x == f) pos = 4 * k1; else if (t1.y == f) pos = 4 * k1 + 1;
+                else if (t1.z == f) pos = 4 * k1 + 2; else if (t1.w == f) pos = 4 * k1 + 3;
+                else if (t2.x == f) pos = 4 * k2; else if (t2.y == f) pos = 4 * k2 + 1;
+                else if (t2.z == f) pos = 4 * k2 + 2; else if (t2.w == f) pos = 4 * k2 + 3;
+                if (pos >= 0 && S.h[pos] == h[q] && S.len[pos] == len[q] && S.w0[pos] == w0[q] && S.w1[pos] == w1[q] &&
+                    (len[q] <= 16 || entry_key_eq(ref_ptr(d, S.ref[pos]) + KEY_OFF + 16, b.keys + s[q] + 16, len[q] - 16))) {
+                    if (!VALS) atomicAdd(&S.plo[pos], (unsigned int)contrib);
+                    else smem_add_u64(&S.plo[pos], &S.phi[pos], contrib);
+                    done = true;
+                }
+            }
+            // ---- global chain walk / combine / allocate + link (a3..a6)
+            const bool look = ins && !done;
+            const uint8_t* tail = b.keys + s[q] + 16;
+            const uint32_t bkt = look ? bucket_of(h[q], d.n_buckets) : 0;
+            const uint32_t tag = tag_of(h[q]);
+            uint32_t head = 0;
+            uint8_t* found = nullptr;
+            if (look) {
+                head = ld_relaxed_u32(d.dir + bkt);
+                found = chain_find_w(d, head, 0, tag, len[q], w0[q], w1[q], tail);
+                if (found) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found, len[q])), contrib);
+            }
+            uint32_t res = R_OK;
+            const uint32_t esize = centry_size(len[q]);
+            bool need = look && !found;
+            if (need && (len[q] > 65535u - 64u || esize > PB)) { need = false; res = R_TOOLARGE; }
+            if (need && inject_fail(d, h[q], (g0 + q) * 32 + lane)) { need = false; res = R_POST; }
+            // Certified declines (R15): allocation failure is monotone for the generation (the
+            // `full` flag), and a warp announces itself in `inflight` before it may reserve an
+            // entry and leaves after linking it. A warp that declines waits (once per launch)
+            // until no warp is between reserving and linking; every entry reserved before the
+            // pool ran out is then linked and no later one can exist, so one re-walk of the
+            // chain decides the record for good: the key is absorbed now or it is not resident
+            // in this generation (the residency guarantee of P:L77/P:L79).
+            const bool any_need = __any_sync(FULLMASK, need);
+            uint64_t off = ~0ull;
+            if (any_need && !w_full) {  // cheap check first: no announcement once the pool is known full
+                unsigned long long f0 = 0;
+                if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
+                if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
+            }
+            if (any_need && !w_full) {
+                if (lane == 0) atomicAdd(&d.ctrl->inflight, 1ull);
+                __syncwarp();
+                asm volatile("fence.sc.gpu;" ::: "memory");
+                unsigned long long f = 0;
+                if (lane == 0) f = ld_relaxed_u64(&d.ctrl->full);
+                f = __shfl_sync(FULLMASK, f, 0);
+                if (f) w_full = true;
+                else off = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
+                if (need && off != ~0ull) {
+                    uint8_t* e = d.pool + off;
+                    *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_COMBINE, head, tag, len[q]);
+                    if (len[q] > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0[q];
+                    if (len[q] > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1[q];
+                    if (len[q] > 16) store_key(e + KEY_OFF + 16, tail, len[q] - 16);
+                    *reinterpret_cast<unsigned long long*>(entry_val(e, len[q])) = contrib;
+                                        const uint32_t me = off_ref(off);
+                    while (true) {  // lock-free head insertion
+                        const uint32_t old = cas_release(d.dir + bkt, head, me);
+                        if (old == head) break;
+                        uint8_t* w = chain_find_w(d, old, head, tag, len[q], w0[q], w1[q], tail);
+                        if (w) {  // linked meanwhile by another warp: combine there, retire ours
+                            red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len[q])), contrib);
+                            *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
+                            c_dead += esize;
+                            break;
+                        }
+                        head = old;
+                        *reinterpret_cast<uint32_t*>(e + 4) = head;
+                    }
+                }
+                __syncwarp();
+                if (lane == 0) add_release64(&d.ctrl->inflight, ~0ull);  // -1, after every link above
+            }
+            const bool declined = need && off == ~0ull;
+            if (__any_sync(FULLMASK, declined)) {
+                w_full = true;
+                if (!w_quiet) {
+                    asm volatile("fence.sc.gpu;" ::: "memory");
+                    if (lane == 0)
+                        while (ld_relaxed_u64(&d.ctrl->inflight) != 0ull) __nanosleep(64);
+                    __syncwarp();
+                    if (declined) {
+                        uint8_t* w = chain_find_w(d, ld_relaxed_u32(d.dir + bkt), 0, tag, len[q], w0[q], w1[q], tail);
+                        if (w) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len[q])), contrib);
+                        else res = R_POST;
+                    }
+                    w_quiet = true;
+                } else if (declined) {
+                    res = R_POST;  // walked after quiescence: the miss is final
+                }
+            }
+            // ---- outcome of every record = outcome of its inserter (a7)
+            const uint32_t lres = __shfl_sync(FULLMASK, res, leader);
+            const uint32_t myres = (valid[q] && eq && lane != leader) ? lres : res;
+            const unsigned bits = __ballot_sync(FULLMASK, valid[q] && myres != R_OK);
+            const unsigned tl = __ballot_sync(FULLMASK, valid[q] && myres == R_TOOLARGE);
+            if (lane == 0) {
+                b.bitmap[g0 + q] = bits;
+                c_post += __popc(bits);
+                c_tl += __popc(tl);
+            }
+        }
+    }
+    if (lane == 0 && (c_post | c_tl)) {
+        if (c_post) atomicAdd(&S.post, c_post);
+        if (c_tl) atomicAdd(&S.toolarge, c_tl);
+    }
+    if (c_dead) atomicAdd(&S.dead, c_dead);
+    __syncthreads();
+    // flush the hot keys' pending sums into their resident entries
+    for (int p = tid; p < hot::NH; p += THREADS) {
+        if (S.len[p] == hot::EMPTY_LEN) continue;
+        const uint64_t sum = ((uint64_t)S.phi[p] << 32) | S.plo[p];
+        if (sum) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(ref_ptr(d, S.ref[p]), S.len[p])), sum);
+    }
+    if (tid == 0) {
+        d.cursors[2 * blockIdx.x] = S.cur[0];
+        d.cursors[2 * blockIdx.x + 1] = S.cur[1];
+        if (S.post) atomicAdd(&d.ctrl->postponed, S.post);
+        if (S.toolarge) atomicAdd(&d.ctrl->toolarge, S.toolarge);
+        if (S.dead) atomicAdd(&d.ctrl->dead_bytes, S.dead);
+    }
+}
+
 // ================================================================ re-probe (a8)
 // One warp per bitmap word. Declined records whose key is now resident are combined / appended
 // and their bit cleared; per tile of RP_TILE records the remaining count and bytes are written
@@ -476,11 +886,10 @@ __global__ void __launch_bounds__(RP_THREADS) reprobe_kernel(Dev d, Batch b, uns
                 uint32_t want_cap = 0;
                 if (mine) {
                     const uint64_t h = hash_key(b.keys + s, len, d.seed);
-                    const uint32_t koff = MODE == 0 ? CENTRY_HDR : GKEY_HDR;
                     const uint32_t head = ld_relaxed_u32(d.dir + bucket_of(h, d.n_buckets));
-                    e = chain_find(d, head, 0, tag_of(h), len, b.keys + s, koff);
+                    e = chain_find(d, head, 0, tag_of(h), len, b.keys + s);
                     if (MODE == 0 && e) {  // resident: combine now
-                        atomicAdd(reinterpret_cast<unsigned long long*>(e + 16), (unsigned long long)rec_value(b, i));
+                        atomicAdd(reinterpret_cast<unsigned long long*>(entry_val(e, len)), (unsigned long long)rec_value(b, i));
                         still = false;
                     }
                     if (MODE == 1 && e) {  // resident key: append the value if its head chunk has room
@@ -509,8 +918,7 @@ __global__ void __launch_bounds__(RP_THREADS) reprobe_kernel(Dev d, Batch b, uns
                             uint64_t vs; uint32_t vl;
                             rec_val_span(b, i, vs, vl);
                             for (uint32_t q = 0; q < vl; ++q) c[CHUNK_HDR + q] = __ldg(b.vals + vs + q);
-                            push_chunk(e, c, vref_of(d, coff),
-                                       ld_relaxed_u64(reinterpret_cast<const unsigned long long*>(e + 16)));
+                            push_chunk(e, c, vref_of(d, coff), ld_relaxed_u64(list_head(e)));
                             still = false;
                         } else {
                             // resident key with values still pending: keep its key page
@@ -651,7 +1059,7 @@ __global__ void __launch_bounds__(CP_THREADS) compact_kernel(Batch b, const unsi
             if (b.vals) {
                 uint64_t vs; uint32_t vl;
                 if (b.vo) { rec_val_span(b, i, vs, vl); ovo[pos[0]] = pos[2]; }
-                else { vs = i * (uint64_t)b.vw; vl = b.vw; }
+                else { vs = rec_index(b, i) * (uint64_t)b.vw; vl = b.vw; }
                 for (uint32_t x = 0; x < vl; ++x) ov[pos[2] + x] = __ldg(b.vals + vs + x);
                 pos[2] += vl;
             }
@@ -665,6 +1073,41 @@ __global__ void finish_offsets_kernel(uint64_t* oko, uint64_t m, uint64_t kb, ui
     if (threadIdx.x == 0 && blockIdx.x == 0) {
         if (oko) oko[m] = kb;
         if (ovo) ovo[m] = vb;
+    }
+}
+
+// index stream compaction (a9): positions of set bits, mapped through the batch's own index
+// list, written in order: out[k] = rec_index(b, i) for the k-th postponed record i.
+__global__ void __launch_bounds__(256) compact_index_kernel(Batch b, const unsigned long long* tile_base, uint64_t* out) {
+    __shared__ unsigned int s_w[8];
+    const uint32_t tid = threadIdx.x, lane = lane_id(), warp = tid >> 5;
+    const uint64_t ntiles = (b.n + RP_TILE - 1) / RP_TILE;
+    for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        // thread t owns bits [8t, 8t+8) of the tile = one byte of the tile's 64 bitmap words
+        const uint64_t i0 = tile * RP_TILE + (uint64_t)tid * 8;
+        uint32_t byte = 0;
+        if (i0 < b.n) {
+            byte = (b.bitmap[i0 >> 5] >> (i0 & 31)) & 0xffu;
+            const uint64_t rem = b.n - i0;
+            if (rem < 8) byte &= (1u << rem) - 1u;
+        }
+        const uint32_t c = __popc(byte);
+        uint32_t inc = c;
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(FULLMASK, inc, o);
+            if (lane >= (uint32_t)o) inc += y;
+        }
+        if (lane == 31) s_w[warp] = inc;
+        __syncthreads();
+        uint64_t pos = tile_base[3 * tile];
+        for (uint32_t w2 = 0; w2 < warp; ++w2) pos += s_w[w2];
+        pos += inc - c;
+        while (byte) {
+            const int q = __ffs(byte) - 1;
+            byte &= byte - 1;
+            out[pos++] = rec_index(b, i0 + q);
+        }
+        __syncthreads();
     }
 }
 
@@ -750,15 +1193,14 @@ __global__ void relink_kernel(Dev d) {
                 const uint32_t len = *reinterpret_cast<uint32_t*>(e + 12);
                 (void)len;
                 // recompute the bucket from the stored key
-                const uint64_t h = hash_key(e + GKEY_HDR, len, d.seed);
+                const uint64_t h = hash_key(e + KEY_OFF, len, d.seed);
                 (void)tag;
                 const uint32_t bkt = bucket_of(h, d.n_buckets);
                 const uint32_t me = off_ref((uint64_t)(e - d.pool));
                 uint32_t head = ld_relaxed_u32(d.dir + bkt);
                 while (true) {
                     *reinterpret_cast<uint32_t*>(e + 4) = head;
-                    __threadfence();
-                    const uint32_t old = atomicCAS(d.dir + bkt, head, me);
+                    const uint32_t old = cas_release(d.dir + bkt, head, me);
                     if (old == head) break;
                     head = old;
                 }
@@ -788,12 +1230,33 @@ __global__ void init_state_kernel(Dev d, uint32_t n_slots) {
 // ================================================================ launchers
 using namespace sepo;
 
-int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStream_t s) {
+int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch) {
     if (mode == 0) {
-        size_t sm = sizeof(Smem<0>);
-        static bool attr0 = false;
-        if (!attr0) { cudaFuncSetAttribute(insert_kernel<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm); attr0 = true; }
-        insert_kernel<0><<<grid, Cfg<0>::THREADS, sm, s>>>(d, b);
+        // hot-set discovery on a strided sample (skipped for small batches)
+        const hot::Entry* hl = nullptr;
+        const unsigned int* nh = nullptr;
+        const uint64_t n_sample = 1ull << 18;
+        if (hot_scratch && b.n >= 8 * n_sample) {
+            uint8_t* p = reinterpret_cast<uint8_t*>(hot_scratch);
+            hot::SampleSlot* tab = reinterpret_cast<hot::SampleSlot*>(p);
+            hot::Entry* list = reinterpret_cast<hot::Entry*>(p + sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS);
+            unsigned int* n_out = reinterpret_cast<unsigned int*>(list + hot::K);
+            cudaMemsetAsync(tab, 0, sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS, s);
+            hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, b.n / n_sample, n_sample, tab);
+            hot_select_kernel<<<1, 1024, 0, s>>>(d, b, tab, list, n_out, 4u);
+            hot_resolve_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
+            hl = list;
+            nh = n_out;
+        }
+        const size_t sm = sizeof(stream::Smem);
+        static bool attr = false;
+        if (!attr) {
+            cudaFuncSetAttribute(insert_stream_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            cudaFuncSetAttribute(insert_stream_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            attr = true;
+        }
+        if (b.vals) insert_stream_kernel<true><<<grid, stream::THREADS, sm, s>>>(d, b, hl, nh);
+        else insert_stream_kernel<false><<<grid, stream::THREADS, sm, s>>>(d, b, hl, nh);
     } else {
         size_t sm = sizeof(Smem<1>);
         static bool attr1 = false;
@@ -802,8 +1265,10 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
     }
     return cudaGetLastError();
 }
-size_t sepo_insert_smem(int mode) { return mode == 0 ? sizeof(Smem<0>) : sizeof(Smem<1>); }
-int sepo_insert_threads(int mode) { return mode == 0 ? Cfg<0>::THREADS : Cfg<1>::THREADS; }
+size_t sepo_hot_scratch_bytes() {
+    return sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS + sizeof(hot::Entry) * hot::K + 256;
+}
+int sepo_default_grid(int mode, int n_sms) { return mode == 0 ? n_sms : 2 * n_sms; }
 
 int sepo_launch_reprobe(const Dev& d, const Batch& b, int mode, int probe, int grid, unsigned long long* tile_counts,
                         cudaStream_t s) {
@@ -829,6 +1294,14 @@ int sepo_launch_compact(const Batch& b, unsigned long long* tile_counts, uint8_t
     return cudaGetLastError();
 }
 
+int sepo_launch_compact_index(const Batch& b, unsigned long long* tile_counts, uint64_t* idx_out, int grid, cudaStream_t s) {
+    const uint64_t nt = sepo_reprobe_tiles(b.n);
+    if (nt) {
+        scan_tiles_kernel<<<1, 1024, 0, s>>>(tile_counts, nt);
+        compact_index_kernel<<<grid, 256, 0, s>>>(b, tile_counts, idx_out);
+    }
+    return cudaGetLastError();
+}
 int sepo_launch_seal(const Dev& d, uint32_t n_slots, cudaStream_t s) {
     seal_kernel<<<(2 * n_slots + 255) / 256, 256, 0, s>>>(d, n_slots);
     return cudaGetLastError();

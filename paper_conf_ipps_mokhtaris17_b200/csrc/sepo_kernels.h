@@ -15,17 +15,20 @@ struct Batch {
     const uint64_t* vo;   // GROUP variable-length values (not supported yet: must be nullptr)
     uint64_t n;
     uint32_t* bitmap;
+    const uint64_t* idx;  // nullptr, or: record i of the batch is record idx[i] of keys/ko/vals (re-issue)
 };
 }  // namespace sepo
 
-int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int grid, cudaStream_t s);
-size_t sepo_insert_smem(int mode);
-int sepo_insert_threads(int mode);
+int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch);
+size_t sepo_hot_scratch_bytes();
+int sepo_default_grid(int mode, int n_sms);
 int sepo_launch_reprobe(const sepo::Dev& d, const sepo::Batch& b, int mode, int probe, int grid,
                         unsigned long long* tile_counts, cudaStream_t s);
 uint64_t sepo_reprobe_tiles(uint64_t n);
 int sepo_launch_compact(const sepo::Batch& b, unsigned long long* tile_counts, uint8_t* ok, uint64_t* oko, uint8_t* ov,
                         uint64_t* ovo, uint64_t m, uint64_t kb, uint64_t vb, int grid, cudaStream_t s);
+int sepo_launch_compact_index(const sepo::Batch& b, unsigned long long* tile_counts, uint64_t* idx_out, int grid,
+                              cudaStream_t s);
 int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);
 int sepo_launch_classify(const sepo::Dev& d, int honor_retain, cudaStream_t s);
 int sepo_launch_relink(const sepo::Dev& d, cudaStream_t s);
