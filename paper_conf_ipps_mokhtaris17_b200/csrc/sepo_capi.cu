@@ -198,6 +198,7 @@ double elapsed_ms(cudaEvent_t a, cudaEvent_t b) {
 
 int init_device_state(sepo_table* t) {
     CK(t, cudaMemsetAsync(t->d.dir, 0, t->n_buckets * 4, t->stream));
+    CK(t, cudaMemsetAsync(t->d.ann, 0, kMaxGrid * ANN_STRIDE * 8, t->stream));
     int rc = sepo_launch_init(t->d, (uint32_t)kMaxGrid, t->stream);  // every cursor slot, whatever the grid
     if (rc) return cuda_check(t, (cudaError_t)rc, "init kernel");
     t->st.kernel_launches += 1;
@@ -215,7 +216,7 @@ const char* sepo_version(void) { return "sepo-b200 0.1 (sm_100a)"; }
 
 static size_t al256(size_t x) { return (x + 255) & ~(size_t)255; }
 static size_t fixed_bytes(uint64_t n_buckets) {
-    return al256(n_buckets * 4) + al256(sizeof(Ctrl)) + al256(kMaxGrid * 2 * 8);
+    return al256(n_buckets * 4) + al256(sizeof(Ctrl)) + al256(kMaxGrid * 2 * 8) + al256(kMaxGrid * ANN_STRIDE * 8);
 }
 static const size_t kPerPageMeta = 4 + 1 + 1 + 4;  // stack, page_state, retain, evict_list
 
@@ -270,6 +271,7 @@ sepo_table* sepo_create(size_t budget, uint64_t n_buckets, uint32_t page_bytes) 
     d.dir = (uint32_t*)p; p += al(n_buckets * 4);
     d.ctrl = (Ctrl*)p; p += al(sizeof(Ctrl));
     d.cursors = (unsigned long long*)p; p += al(max_grid * 2 * 8);
+    d.ann = (unsigned long long*)p; p += al(max_grid * ANN_STRIDE * 8);
     d.stack = (uint32_t*)p; p += al(np * 4);
     d.page_state = p; p += al(np);
     d.retain = p; p += al(np);
@@ -281,6 +283,7 @@ sepo_table* sepo_create(size_t budget, uint64_t n_buckets, uint32_t page_bytes) 
         t->n_pages = (uint32_t)np;
     }
     d.pool = (uint8_t*)pa;
+    d.n_slots = (uint32_t)t->grid;
     d.n_buckets = n_buckets;
     d.page_bytes = page_bytes;
     d.page_shift = t->page_shift;
@@ -326,6 +329,7 @@ int sepo_configure(sepo_table* t, const sepo_options* o) {
     if (n.fail_until_pass == 0) n.fail_until_pass = 16;
     if (n.grid_ctas == 0) n.grid_ctas = (uint32_t)sepo_default_grid(n.mode, t->n_sms);
     t->grid = (int)n.grid_ctas;
+    t->d.n_slots = (uint32_t)t->grid;
     t->st.grid_ctas = t->grid;
     if (n.stream) {
         if (t->own_stream && t->stream) cudaStreamDestroy(t->stream);
@@ -496,7 +500,8 @@ static int64_t evict_impl(sepo_table* t, int honor_retain) {
     if (rc) return cuda_check(t, (cudaError_t)rc, "seal kernel");
     rc = sepo_launch_classify(t->d, honor_retain, t->stream);
     if (rc) return cuda_check(t, (cudaError_t)rc, "classify kernel");
-    CK(t, cudaMemsetAsync(&t->d.ctrl->full, 0, 2 * sizeof(unsigned long long), t->stream));  // full, inflight
+    CK(t, cudaMemsetAsync(&t->d.ctrl->full, 0, sizeof(unsigned long long), t->stream));
+    CK(t, cudaMemsetAsync(t->d.ann, 0, kMaxGrid * ANN_STRIDE * 8, t->stream));
     t->st.kernel_launches += 2;
     if ((rc = read_ctrl(t))) return rc;
     const uint64_t ne = t->h_ctrl->n_evict;

@@ -51,8 +51,7 @@ struct Ctrl {
     unsigned long long n_free;         // evict: pages in the new free stack
     unsigned long long n_resident;     // evict: pages that stay resident (retained)
     unsigned long long full;           // 1 once the pool ran out this generation: every later allocation fails
-    unsigned long long inflight;       // warps between announcing an allocation and linking it
-    unsigned long long pad[5];
+    unsigned long long pad[6];
 };
 
 struct Dev {
@@ -69,6 +68,10 @@ struct Dev {
     uint32_t* evict_list;
     unsigned long long* cursors;  // [grid][2]
     Ctrl* ctrl;
+    // per-allocator-slot announcement words (128 B apart): bit 63 = pool full, low bits = warps of
+    // that CTA between announcing an allocation and linking its entries (certified declines, R15)
+    unsigned long long* ann;
+    uint32_t n_slots;
     uint64_t seed;
     uint32_t gen;             // generation (= pass index) of resident data
     uint32_t fail_ppm, fail_mode, fail_until;
@@ -103,6 +106,13 @@ __device__ __forceinline__ unsigned long long cas_release64(unsigned long long* 
 __device__ __forceinline__ void add_release64(unsigned long long* p, unsigned long long v) {
     asm volatile("red.release.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+constexpr unsigned long long ANN_FULL = 1ull << 63;
+constexpr uint32_t ANN_STRIDE = 16;  // u64 words between announcement words (128 B)
 // L2-coherent loads of published entry fields (never stale L1 lines)
 __device__ __forceinline__ uint64_t ldcg64(const void* p) { return __ldcg(reinterpret_cast<const unsigned long long*>(p)); }
 __device__ __forceinline__ uint32_t ldcg32(const void* p) { return __ldcg(reinterpret_cast<const unsigned int*>(p)); }
@@ -125,11 +135,10 @@ __device__ __forceinline__ uint64_t fmix64(uint64_t k) {
     k ^= k >> 33; k *= 0xc4ceb9fe1a85ec53ull;
     k ^= k >> 33; return k;
 }
-// h = fmix64(fold over the key's 8-byte LE words (zero padded), seeded with the length)
+// h = fmix64(multiply-xor fold over the key's 8-byte LE words (zero padded), seeded with the length)
 __device__ __forceinline__ uint64_t hash_init(uint32_t len, uint64_t seed) { return seed ^ ((uint64_t)len * 0x87c37b91114253d5ull); }
 __device__ __forceinline__ uint64_t hash_word(uint64_t h, uint64_t w) {
-    h ^= w * 0x4cf5ad432745937full;
-    return ((h << 29) | (h >> 35)) * 0x9e3779b97f4a7c15ull + 0x52dce729ull;
+    return (h ^ w) * 0x9e3779b97f4a7c15ull;  // odd multiplier: a bijection per word
 }
 __device__ __forceinline__ uint64_t hash_key(const uint8_t* p, uint32_t len, uint64_t seed) {
     uint64_t h = hash_init(len, seed);
@@ -294,7 +303,11 @@ __device__ __forceinline__ uint64_t warp_alloc(const Dev& d, unsigned long long*
                         nw = (unsigned long long)np << 32;
                     } else {
                         nw = (unsigned long long)FULLPAGE << 32;
-                        atomicExch(&d.ctrl->full, 1ull);
+                        // the pool ran out: every later allocation of this generation fails. The
+                        // bit goes into every slot's announcement word (same-location RMWs order
+                        // it against each announcement; see the COMBINE insert kernel).
+                        if (atomicExch(&d.ctrl->full, 1ull) == 0ull)
+                            for (uint32_t c = 0; c < d.n_slots; ++c) atomicOr(&d.ann[(uint64_t)c * ANN_STRIDE], ANN_FULL);
                     }
                     __threadfence_block();
                     atomicExch(scur, nw);

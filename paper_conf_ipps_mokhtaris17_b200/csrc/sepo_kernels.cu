@@ -606,7 +606,6 @@ __global__ void __launch_bounds__(1024) hot_resolve_kernel(Dev d, Batch b, hot::
 
 namespace stream {
 constexpr int THREADS = 1024;
-constexpr int SUB = 1;  // 32-record groups per warp step
 struct Smem {
     uint4 tags[hot::NB];  // 4 fingerprints per bucket (one 16-B load per probed bucket)
     uint64_t h[hot::NH], w0[hot::NH], w1[hot::NH];
@@ -629,7 +628,6 @@ template <bool VALS>
 __global__ void __launch_bounds__(stream::THREADS, 1) insert_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
                                                                            const unsigned int* n_hot) {
     using stream::THREADS;
-    using stream::SUB;
     extern __shared__ __align__(16) uint8_t smem_raw[];
     stream::Smem& S = *reinterpret_cast<stream::Smem*>(smem_raw);
     const uint32_t tid = threadIdx.x, lane = lane_id();
@@ -661,169 +659,172 @@ __global__ void __launch_bounds__(stream::THREADS, 1) insert_stream_kernel(Dev d
     }
     __syncthreads();
     const bool have_hot = nh > 0;
+    const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
 
+    // Each warp streams 32-record groups. Order per group: hot probe first (shared memory), then
+    // the directory load for the misses is issued and overlaps the folding of the hits; the
+    // misses then walk their chains (one record per lane: tail keys rarely repeat in a warp).
     const uint64_t ngroups = (b.n + 31) / 32;
     const uint64_t gw = (uint64_t)blockIdx.x * (THREADS / 32) + (tid >> 5);
     const uint64_t nw = (uint64_t)gridDim.x * (THREADS / 32);
     unsigned long long c_post = 0, c_tl = 0, c_dead = 0;
     bool w_full = false, w_quiet = false;  // warp-uniform: pool ran out / quiescence observed
-    for (uint64_t g0 = gw * SUB; g0 < ngroups; g0 += nw * SUB) {
-        uint64_t s[SUB], w0[SUB], w1[SUB], h[SUB], v[SUB];
-        uint32_t len[SUB];
-        bool valid[SUB];
-#pragma unroll
-        for (int q = 0; q < SUB; ++q) {
-            const uint64_t i = (g0 + q) * 32 + lane;
-            valid[q] = i < b.n;
-            s[q] = 0; len[q] = 0; w0[q] = 0; w1[q] = 0; h[q] = 0; v[q] = 0;
-            if (valid[q]) {
-                rec_hash16(d, b, i, s[q], len[q], w0[q], w1[q], h[q]);
-                if (VALS) v[q] = rec_value(b, i);
-            }
+    // software pipeline: the next group's key offsets and first 16 key bytes are loaded while
+    // the current group's lookups are in flight
+    uint64_t ns = 0, nw0 = 0, nw1 = 0;
+    uint32_t nlen = 0;
+    if (gw < ngroups && gw * 32 + lane < b.n) {
+        rec_key(b, gw * 32 + lane, ns, nlen);
+        load_key16(b.keys + ns, nlen, nw0, nw1);
+    }
+    for (uint64_t g = gw; g < ngroups; g += nw) {
+        const uint64_t i = g * 32 + lane;
+        const bool valid = i < b.n;
+        const uint64_t s = ns, w0 = nw0, w1 = nw1;
+        const uint32_t len = nlen;
+        uint64_t h = 0, v = 1;
+        if (valid) {
+            uint64_t x = hash_init(len, d.seed);
+            if (len > 0) x = hash_word(x, w0);
+            if (len > 8) x = hash_word(x, w1);
+            for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(b.keys + s + o, len - o < 8 ? len - o : 8));
+            h = fmix64(x);
+            if (VALS) v = rec_value(b, i);
         }
-#pragma unroll
-        for (int q = 0; q < SUB; ++q) {
-            const unsigned vm = __ballot_sync(FULLMASK, valid[q]);
-            if (vm == 0) continue;  // warp-uniform
-            // ---- fold equal keys of the warp (a2)
-            // fold on 32 hash bits; equal keys are then confirmed on bytes (collisions stay apart)
-            const unsigned hh = valid[q] ? (unsigned)h[q] : (0x80000000u | lane);
-            const unsigned grp = __match_any_sync(FULLMASK, hh) & vm;
+        {   // issue the next group's offsets now; its key bytes at the end of this iteration
+            const uint64_t gn = g + nw;
+            ns = 0; nlen = 0;
+            if (gn < ngroups && gn * 32 + lane < b.n) rec_key(b, gn * 32 + lane, ns, nlen);
+        }
+        // ---- hot set: constant-time probe of two 4-way buckets, then a full-key check
+        int pos = -1;
+        if (valid && have_hot) {
+            const uint32_t f = hot::fp(h);
+            const uint32_t k1 = hot::b1(h), k2 = hot::b2(h);
+            const uint4 t1 = S.tags[k1];
+            if (t1.x == f) pos = 4 * k1; else if (t1.y == f) pos = 4 * k1 + 1;
+            else if (t1.z == f) pos = 4 * k1 + 2; else if (t1.w == f) pos = 4 * k1 + 3;
+            else {
+                const uint4 t2 = S.tags[k2];
+                if (t2.x == f) pos = 4 * k2; else if (t2.y == f) pos = 4 * k2 + 1;
+                else if (t2.z == f) pos = 4 * k2 + 2; else if (t2.w == f) pos = 4 * k2 + 3;
+            }
+            if (pos >= 0 && !(S.h[pos] == h && S.len[pos] == len && S.w0[pos] == w0 && S.w1[pos] == w1 &&
+                              (len <= 16 || entry_key_eq(ref_ptr(d, S.ref[pos]) + KEY_OFF + 16, b.keys + s + 16, len - 16))))
+                pos = -1;
+        }
+        const bool miss = valid && pos < 0;
+        const uint8_t* tail = b.keys + s + 16;
+        const uint32_t bkt = bucket_of(h, d.n_buckets);
+        const uint32_t tag = tag_of(h);
+        uint32_t head = 0;
+        if (miss) head = ld_relaxed_u32(d.dir + bkt);  // in flight while the hits are folded
+        // ---- fold the hits of the warp per hot slot (a2): one shared atomic per distinct key
+        const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
+        if (hm) {
+            const unsigned key = pos >= 0 ? (unsigned)pos : (0x10000u | lane);
+            const unsigned grp = __match_any_sync(FULLMASK, key) & hm;
             const uint32_t leader = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
-            const uint64_t lw0 = __shfl_sync(FULLMASK, w0[q], leader);
-            const uint64_t lw1 = __shfl_sync(FULLMASK, w1[q], leader);
-            const uint32_t llen = __shfl_sync(FULLMASK, len[q], leader);
-            const uint64_t ls = __shfl_sync(FULLMASK, s[q], leader);
-            const bool eq = valid[q] && (lane == leader ||
-                                         (len[q] == llen && w0[q] == lw0 && w1[q] == lw1 &&
-                                          (len[q] <= 16 || in_key_eq(b.keys + s[q] + 16, b.keys + ls + 16, len[q] - 16))));
-            const unsigned joined = grp & __ballot_sync(FULLMASK, eq);
-            const bool ins = valid[q] && (lane == leader || !eq);
-            uint64_t contrib;
             if (!VALS) {
-                contrib = (lane == leader) ? (uint64_t)__popc(joined) : 1ull;
+                if (pos >= 0 && lane == leader) atomicAdd(&S.plo[pos], (unsigned int)__popc(grp));
             } else {
-                uint64_t acc = v[q];
-                if (__any_sync(FULLMASK, __popc(joined) > 1)) {
+                uint64_t acc = v;
+                if (__any_sync(FULLMASK, __popc(grp) > 1)) {
                     acc = 0;
                     for (int x = 0; x < 32; ++x) {
-                        const uint64_t vx = __shfl_sync(FULLMASK, v[q], x);
-                        if ((joined >> x) & 1u) acc += vx;
+                        const uint64_t vx = __shfl_sync(FULLMASK, v, x);
+                        if ((grp >> x) & 1u) acc += vx;
                     }
                 }
-                contrib = (lane == leader) ? acc : v[q];
+                if (pos >= 0 && lane == leader) smem_add_u64(&S.plo[pos], &S.phi[pos], acc);
             }
-            // ---- hot set (shared memory, read-only keys)
-            bool done = !ins;
-            if (ins && have_hot) {
-                const uint32_t f = hot::fp(h[q]);
-                const uint32_t k1 = hot::b1(h[q]), k2 = hot::b2(h[q]);
-                const uint4 t1 = S.tags[k1], t2 = S.tags[k2];
-                int pos = -1;
-                if (t1.x == f) pos = 4 * k1; else if (t1.y == f) pos = 4 * k1 + 1;
-                else if (t1.z == f) pos = 4 * k1 + 2; else if (t1.w == f) pos = 4 * k1 + 3;
-                else if (t2.x == f) pos = 4 * k2; else if (t2.y == f) pos = 4 * k2 + 1;
-                else if (t2.z == f) pos = 4 * k2 + 2; else if (t2.w == f) pos = 4 * k2 + 3;
-                if (pos >= 0 && S.h[pos] == h[q] && S.len[pos] == len[q] && S.w0[pos] == w0[q] && S.w1[pos] == w1[q] &&
-                    (len[q] <= 16 || entry_key_eq(ref_ptr(d, S.ref[pos]) + KEY_OFF + 16, b.keys + s[q] + 16, len[q] - 16))) {
-                    if (!VALS) atomicAdd(&S.plo[pos], (unsigned int)contrib);
-                    else smem_add_u64(&S.plo[pos], &S.phi[pos], contrib);
-                    done = true;
+        }
+        // ---- misses: chain walk, combine in place, or allocate + link (a3..a6)
+        uint8_t* found = nullptr;
+        if (miss) {
+            found = chain_find_w(d, head, 0, tag, len, w0, w1, tail);
+            if (found) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found, len)), v);
+        }
+        uint32_t res = R_OK;
+        const uint32_t esize = centry_size(len);
+        bool need = miss && !found;
+        if (need && (len > 65535u - 64u || esize > PB)) { need = false; res = R_TOOLARGE; }
+        if (inj && need && inject_fail(d, h, i)) { need = false; res = R_POST; }
+        // Certified declines (R15). Allocation failure is monotone for the generation (`full`).
+        // A warp announces itself in its CTA's announcement word before it may reserve entries
+        // (one RMW; if the word already carries the FULL bit it backs off) and withdraws with a
+        // release-add after linking them. The FULL bit is OR-ed into every word when the pool runs
+        // out, so per word the RMW order decides: an announcement either precedes the bit (and is
+        // counted) or sees it. A declining warp waits (once per launch) until every word shows
+        // FULL with no announcement: every entry reserved before the pool ran out is then linked
+        // and none can follow, so one re-walk of the chain decides the record for good — absorbed
+        // now, or not resident in this generation (the residency guarantee of P:L77/P:L79).
+        const bool any_need = __any_sync(FULLMASK, need);
+        uint64_t off = ~0ull;
+        if (any_need && !w_full) {  // cheap check first: no announcement once the pool is known full
+            unsigned long long f0 = 0;
+            if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
+            if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
+        }
+        if (any_need && !w_full) {
+            unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
+            unsigned long long a = 0;
+            if (lane == 0) a = atomicAdd(my_ann, 1ull);
+            a = __shfl_sync(FULLMASK, a, 0);
+            if (a & ANN_FULL) w_full = true;
+            else off = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
+            if (need && off != ~0ull) {
+                uint8_t* e = d.pool + off;
+                *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_COMBINE, head, tag, len);
+                if (len > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0;
+                if (len > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1;
+                if (len > 16) store_key(e + KEY_OFF + 16, tail, len - 16);
+                *reinterpret_cast<unsigned long long*>(entry_val(e, len)) = v;
+                const uint32_t me = off_ref(off);
+                while (true) {  // lock-free head insertion
+                    const uint32_t old = cas_release(d.dir + bkt, head, me);
+                    if (old == head) break;
+                    uint8_t* w = chain_find_w(d, old, head, tag, len, w0, w1, tail);
+                    if (w) {  // linked meanwhile by another warp: combine there, retire ours
+                        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
+                        *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
+                        c_dead += esize;
+                        break;
+                    }
+                    head = old;
+                    *reinterpret_cast<uint32_t*>(e + 4) = head;
                 }
             }
-            // ---- global chain walk / combine / allocate + link (a3..a6)
-            const bool look = ins && !done;
-            const uint8_t* tail = b.keys + s[q] + 16;
-            const uint32_t bkt = look ? bucket_of(h[q], d.n_buckets) : 0;
-            const uint32_t tag = tag_of(h[q]);
-            uint32_t head = 0;
-            uint8_t* found = nullptr;
-            if (look) {
-                head = ld_relaxed_u32(d.dir + bkt);
-                found = chain_find_w(d, head, 0, tag, len[q], w0[q], w1[q], tail);
-                if (found) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found, len[q])), contrib);
-            }
-            uint32_t res = R_OK;
-            const uint32_t esize = centry_size(len[q]);
-            bool need = look && !found;
-            if (need && (len[q] > 65535u - 64u || esize > PB)) { need = false; res = R_TOOLARGE; }
-            if (need && inject_fail(d, h[q], (g0 + q) * 32 + lane)) { need = false; res = R_POST; }
-            // Certified declines (R15): allocation failure is monotone for the generation (the
-            // `full` flag), and a warp announces itself in `inflight` before it may reserve an
-            // entry and leaves after linking it. A warp that declines waits (once per launch)
-            // until no warp is between reserving and linking; every entry reserved before the
-            // pool ran out is then linked and no later one can exist, so one re-walk of the
-            // chain decides the record for good: the key is absorbed now or it is not resident
-            // in this generation (the residency guarantee of P:L77/P:L79).
-            const bool any_need = __any_sync(FULLMASK, need);
-            uint64_t off = ~0ull;
-            if (any_need && !w_full) {  // cheap check first: no announcement once the pool is known full
-                unsigned long long f0 = 0;
-                if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
-                if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
-            }
-            if (any_need && !w_full) {
-                if (lane == 0) atomicAdd(&d.ctrl->inflight, 1ull);
+            __syncwarp();
+            if (lane == 0) add_release64(my_ann, ~0ull);  // withdraw (-1), after every link above
+        }
+        const bool declined = need && off == ~0ull;
+        if (__any_sync(FULLMASK, declined)) {
+            w_full = true;
+            if (!w_quiet) {
+                if (lane == 0)
+                    for (uint32_t c = 0; c < d.n_slots; ++c)
+                        while (ld_acquire_u64(d.ann + (uint64_t)c * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
                 __syncwarp();
-                asm volatile("fence.sc.gpu;" ::: "memory");
-                unsigned long long f = 0;
-                if (lane == 0) f = ld_relaxed_u64(&d.ctrl->full);
-                f = __shfl_sync(FULLMASK, f, 0);
-                if (f) w_full = true;
-                else off = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
-                if (need && off != ~0ull) {
-                    uint8_t* e = d.pool + off;
-                    *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_COMBINE, head, tag, len[q]);
-                    if (len[q] > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0[q];
-                    if (len[q] > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1[q];
-                    if (len[q] > 16) store_key(e + KEY_OFF + 16, tail, len[q] - 16);
-                    *reinterpret_cast<unsigned long long*>(entry_val(e, len[q])) = contrib;
-                                        const uint32_t me = off_ref(off);
-                    while (true) {  // lock-free head insertion
-                        const uint32_t old = cas_release(d.dir + bkt, head, me);
-                        if (old == head) break;
-                        uint8_t* w = chain_find_w(d, old, head, tag, len[q], w0[q], w1[q], tail);
-                        if (w) {  // linked meanwhile by another warp: combine there, retire ours
-                            red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len[q])), contrib);
-                            *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
-                            c_dead += esize;
-                            break;
-                        }
-                        head = old;
-                        *reinterpret_cast<uint32_t*>(e + 4) = head;
-                    }
+                if (declined) {
+                    uint8_t* w = chain_find_w(d, ld_relaxed_u32(d.dir + bkt), 0, tag, len, w0, w1, tail);
+                    if (w) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
+                    else res = R_POST;
                 }
-                __syncwarp();
-                if (lane == 0) add_release64(&d.ctrl->inflight, ~0ull);  // -1, after every link above
+                w_quiet = true;
+            } else if (declined) {
+                res = R_POST;  // walked after quiescence: the miss is final
             }
-            const bool declined = need && off == ~0ull;
-            if (__any_sync(FULLMASK, declined)) {
-                w_full = true;
-                if (!w_quiet) {
-                    asm volatile("fence.sc.gpu;" ::: "memory");
-                    if (lane == 0)
-                        while (ld_relaxed_u64(&d.ctrl->inflight) != 0ull) __nanosleep(64);
-                    __syncwarp();
-                    if (declined) {
-                        uint8_t* w = chain_find_w(d, ld_relaxed_u32(d.dir + bkt), 0, tag, len[q], w0[q], w1[q], tail);
-                        if (w) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len[q])), contrib);
-                        else res = R_POST;
-                    }
-                    w_quiet = true;
-                } else if (declined) {
-                    res = R_POST;  // walked after quiescence: the miss is final
-                }
-            }
-            // ---- outcome of every record = outcome of its inserter (a7)
-            const uint32_t lres = __shfl_sync(FULLMASK, res, leader);
-            const uint32_t myres = (valid[q] && eq && lane != leader) ? lres : res;
-            const unsigned bits = __ballot_sync(FULLMASK, valid[q] && myres != R_OK);
-            const unsigned tl = __ballot_sync(FULLMASK, valid[q] && myres == R_TOOLARGE);
-            if (lane == 0) {
-                b.bitmap[g0 + q] = bits;
-                c_post += __popc(bits);
-                c_tl += __popc(tl);
-            }
+        }
+        nw0 = 0; nw1 = 0;
+        if (nlen) load_key16(b.keys + ns, nlen, nw0, nw1);
+        // ---- outcome -> bitmap word (a7)
+        const unsigned bits = __ballot_sync(FULLMASK, valid && res != R_OK);
+        const unsigned tl = __ballot_sync(FULLMASK, valid && res == R_TOOLARGE);
+        if (lane == 0 && g * 32 < b.n) {
+            b.bitmap[g] = bits;
+            c_post += __popc(bits);
+            c_tl += __popc(tl);
         }
     }
     if (lane == 0 && (c_post | c_tl)) {
