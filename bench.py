@@ -283,7 +283,7 @@ def run_ours(args):
     alg = info["kb"] + (8 * info["recs"] if k is not None and o is not None else 0) + info["vb"]
     achieved = alg / (info["insert_ms"] / 1e3) / 1e9
     roof = {"bound": "hbm", "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
-            "frac": achieved / pk["hbm_gbs"], "traffic": args.traffic, "kernel": "sepo::insert_kernel<0>",
+            "frac": achieved / pk["hbm_gbs"], "traffic": args.traffic, "kernel": "sepo::insert_stream_kernel (COMBINE) / sepo::insert_kernel<1> (GROUP)",
             "insert_share_of_step": info["insert_ms"] / ms,
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if not pk.get("_fallback") else "fallback 6.65 TB/s"}
 

@@ -373,7 +373,7 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
     rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->opts.mode == SEPO_COMBINE_SUM_U64 ? t->hot.p : nullptr);
     if (rc) return cuda_check(t, (cudaError_t)rc, "insert kernel launch");
     CK(t, cudaEventRecord(t->ev1, t->stream));
-    t->st.kernel_launches += (t->opts.mode == SEPO_COMBINE_SUM_U64 && n >= (8ull << 18)) ? 4 : 1;
+    t->st.kernel_launches += (t->opts.mode == SEPO_COMBINE_SUM_U64 && n >= (8ull << 18)) ? 7 : 1;
     if (b.ko && !b.idx) {
         CK(t, cudaMemcpyAsync(&t->h_ko[0], b.ko, 8, cudaMemcpyDeviceToHost, t->stream));
         CK(t, cudaMemcpyAsync(&t->h_ko[1], b.ko + n, 8, cudaMemcpyDeviceToHost, t->stream));
@@ -856,10 +856,20 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
         cur.bitmap = (uint32_t*)t->bm.p;
         int64_t c = insert_impl(t, cur);
         if (c < 0) return c;
-        uint64_t kb = 0, vb = 0;
-        if (c > 0) c = reprobe_impl(t, cur, &kb, &vb);
+        uint64_t kb = t->h_ctrl->kept_key_bytes, vb = 0;
+        const bool combine_exact = t->opts.mode == SEPO_COMBINE_SUM_U64 && !(t->opts.fail_alloc_ppm && t->opts.fail_mode == 1);
+        if (c > 0 && !combine_exact) c = reprobe_impl(t, cur, &kb, &vb);
         if (c < 0) return c;
         if (c == 0) break;
+        if (combine_exact) {
+            // the insert's count is exact (certified declines, R15): only the per-tile counts
+            const uint64_t pass = t->st.passes;
+            if (pass < SEPO_MAX_PASS_STATS) t->st.postponed_per_pass[pass] += (uint64_t)c;
+            if (t->tile_counts.grow(sepo_reprobe_tiles(cur.n) * 3 * 8)) return fail(SEPO_E_NOMEM, "tile count scratch");
+            int rc3 = sepo_launch_tile_popc(cur, (unsigned long long*)t->tile_counts.p, 8 * t->n_sms, t->stream);
+            if (rc3) return cuda_check(t, (cudaError_t)rc3, "tile_popc kernel");
+            t->st.kernel_launches += 1;
+        }
         // re-issue by index: the postponed records stay where they are in the caller's arrays
         if (t->idxb[side].grow((uint64_t)c * 8)) return fail(SEPO_E_NOMEM, "re-issue index list");
         uint64_t* nidx = (uint64_t*)t->idxb[side].p;

@@ -506,36 +506,34 @@ __global__ void __launch_bounds__(256) hot_sample_kernel(Dev d, Batch b, uint64_
     }
 }
 
-// (i-b) one CTA: threshold = smallest count such that at most K keys reach it; emit those keys.
+// (i-b) threshold = smallest count such that at most K keys reach it; emit those keys.
 // (Hash-identified: two keys with the same 64-bit hash would share a sample slot; the hot set is
 // only a cache, so a wrong pick costs speed, never correctness — entries are matched on bytes.)
-__global__ void __launch_bounds__(1024) hot_select_kernel(Dev d, Batch b, const hot::SampleSlot* tab, hot::Entry* out,
-                                                          unsigned int* n_out, uint32_t min_count) {
-    __shared__ unsigned int hist[4096];
-    __shared__ unsigned int s_thr, s_n;
-    for (int i = threadIdx.x; i < 4096; i += blockDim.x) hist[i] = 0;
-    if (threadIdx.x == 0) { s_n = 0; s_thr = 0xffffffffu; }
-    __syncthreads();
-    for (int i = threadIdx.x; i < hot::SAMPLE_SLOTS; i += blockDim.x) {
+constexpr int HOT_HIST = 4096;
+__global__ void __launch_bounds__(256) hot_hist_kernel(const hot::SampleSlot* tab, unsigned int* hist, uint32_t min_count) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < hot::SAMPLE_SLOTS; i += gridDim.x * blockDim.x) {
         const unsigned c = tab[i].count;
-        if (tab[i].h != 0ull && c >= min_count) atomicAdd(&hist[min(c, 4095u)], 1u);
+        if (tab[i].h != 0ull && c >= min_count) atomicAdd(&hist[min(c, (unsigned)HOT_HIST - 1)], 1u);
     }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        unsigned acc = 0, thr = 0xffffffffu;
-        for (int c = 4095; c >= (int)min_count; --c) {
-            if (acc + hist[c] > (unsigned)hot::K) break;
-            acc += hist[c];
-            thr = c;
-        }
-        s_thr = thr;
+}
+__global__ void __launch_bounds__(32) hot_threshold_kernel(unsigned int* hist, uint32_t min_count) {
+    if (threadIdx.x != 0) return;
+    unsigned acc = 0, thr = 0xffffffffu;
+    for (int c = HOT_HIST - 1; c >= (int)min_count; --c) {
+        if (acc + hist[c] > (unsigned)hot::K) break;
+        acc += hist[c];
+        thr = c;
     }
-    __syncthreads();
-    const unsigned thr = s_thr;
-    for (int i = threadIdx.x; i < hot::SAMPLE_SLOTS; i += blockDim.x) {
+    hist[HOT_HIST] = thr;  // threshold
+}
+__global__ void __launch_bounds__(256) hot_emit_kernel(Dev d, Batch b, const hot::SampleSlot* tab, const unsigned int* hist,
+                                                       hot::Entry* out, unsigned int* n_out) {
+    const unsigned thr = hist[HOT_HIST];
+    if (thr == 0xffffffffu) return;
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < hot::SAMPLE_SLOTS; i += gridDim.x * blockDim.x) {
         const unsigned c = tab[i].count;
-        if (tab[i].h != 0ull && c >= thr && thr != 0xffffffffu) {
-            const unsigned j = atomicAdd(&s_n, 1u);
+        if (tab[i].h != 0ull && c >= thr) {
+            const unsigned j = atomicAdd(n_out, 1u);
             if (j < (unsigned)hot::K) {
                 uint64_t s, w0, w1, h; uint32_t len;
                 rec_hash16(d, b, tab[i].rec, s, len, w0, w1, h);
@@ -545,9 +543,8 @@ __global__ void __launch_bounds__(1024) hot_select_kernel(Dev d, Batch b, const 
             }
         }
     }
-    __syncthreads();
-    if (threadIdx.x == 0) *n_out = min(s_n, (unsigned)hot::K);
 }
+__global__ void hot_clamp_kernel(unsigned int* n_out) { if (threadIdx.x == 0 && *n_out > (unsigned)hot::K) *n_out = hot::K; }
 
 // (i-c) one CTA on allocator slot 0: look up / insert (value 0) every hot key
 __global__ void __launch_bounds__(1024) hot_resolve_kernel(Dev d, Batch b, hot::Entry* list, const unsigned int* n_list) {
@@ -667,7 +664,7 @@ __global__ void __launch_bounds__(stream::THREADS, 1) insert_stream_kernel(Dev d
     const uint64_t ngroups = (b.n + 31) / 32;
     const uint64_t gw = (uint64_t)blockIdx.x * (THREADS / 32) + (tid >> 5);
     const uint64_t nw = (uint64_t)gridDim.x * (THREADS / 32);
-    unsigned long long c_post = 0, c_tl = 0, c_dead = 0;
+    unsigned long long c_post = 0, c_tl = 0, c_dead = 0, c_pkb = 0;
     bool w_full = false, w_quiet = false;  // warp-uniform: pool ran out / quiescence observed
     // software pipeline: the next group's key offsets and first 16 key bytes are loaded while
     // the current group's lookups are in flight
@@ -818,18 +815,21 @@ __global__ void __launch_bounds__(stream::THREADS, 1) insert_stream_kernel(Dev d
         }
         nw0 = 0; nw1 = 0;
         if (nlen) load_key16(b.keys + ns, nlen, nw0, nw1);
-        // ---- outcome -> bitmap word (a7)
+        // ---- outcome -> bitmap word (a7); key bytes of the declined records (re-issue sizing)
         const unsigned bits = __ballot_sync(FULLMASK, valid && res != R_OK);
         const unsigned tl = __ballot_sync(FULLMASK, valid && res == R_TOOLARGE);
+        const unsigned pkb = bits ? __reduce_add_sync(FULLMASK, (valid && res != R_OK) ? len : 0u) : 0u;
         if (lane == 0 && g * 32 < b.n) {
             b.bitmap[g] = bits;
             c_post += __popc(bits);
             c_tl += __popc(tl);
+            c_pkb += pkb;
         }
     }
     if (lane == 0 && (c_post | c_tl)) {
         if (c_post) atomicAdd(&S.post, c_post);
         if (c_tl) atomicAdd(&S.toolarge, c_tl);
+        if (c_pkb) atomicAdd(&d.ctrl->kept_key_bytes, c_pkb);
     }
     if (c_dead) atomicAdd(&S.dead, c_dead);
     __syncthreads();
@@ -1077,6 +1077,26 @@ __global__ void finish_offsets_kernel(uint64_t* oko, uint64_t m, uint64_t kb, ui
     }
 }
 
+// per-tile counts of set bits (COMBINE re-issue: the insert's count is exact, R15)
+__global__ void __launch_bounds__(64) tile_popc_kernel(Batch b, unsigned long long* tile_counts) {
+    const uint64_t ntiles = (b.n + RP_TILE - 1) / RP_TILE;
+    const uint64_t nwords = (b.n + 31) / 32;
+    for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        const uint64_t w = tile * (RP_TILE / 32) + threadIdx.x;
+        unsigned c = w < nwords ? __popc(b.bitmap[w]) : 0u;
+        c = __reduce_add_sync(FULLMASK, c);
+        __shared__ unsigned s2[2];
+        if ((threadIdx.x & 31) == 0) s2[threadIdx.x >> 5] = c;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            tile_counts[3 * tile] = s2[0] + s2[1];
+            tile_counts[3 * tile + 1] = 0;
+            tile_counts[3 * tile + 2] = 0;
+        }
+        __syncthreads();
+    }
+}
+
 // index stream compaction (a9): positions of set bits, mapped through the batch's own index
 // list, written in order: out[k] = rec_index(b, i) for the k-th postponed record i.
 __global__ void __launch_bounds__(256) compact_index_kernel(Batch b, const unsigned long long* tile_base, uint64_t* out) {
@@ -1244,7 +1264,12 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             unsigned int* n_out = reinterpret_cast<unsigned int*>(list + hot::K);
             cudaMemsetAsync(tab, 0, sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS, s);
             hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, b.n / n_sample, n_sample, tab);
-            hot_select_kernel<<<1, 1024, 0, s>>>(d, b, tab, list, n_out, 4u);
+            unsigned int* hist = n_out + 1;
+            cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
+            hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
+            hot_threshold_kernel<<<1, 32, 0, s>>>(hist, 4u);
+            hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out);
+            hot_clamp_kernel<<<1, 32, 0, s>>>(n_out);
             hot_resolve_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
             hl = list;
             nh = n_out;
@@ -1267,7 +1292,7 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
     return cudaGetLastError();
 }
 size_t sepo_hot_scratch_bytes() {
-    return sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS + sizeof(hot::Entry) * hot::K + 256;
+    return sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS + sizeof(hot::Entry) * hot::K + (HOT_HIST + 16) * 4;
 }
 int sepo_default_grid(int mode, int n_sms) { return mode == 0 ? n_sms : 2 * n_sms; }
 
@@ -1295,6 +1320,10 @@ int sepo_launch_compact(const Batch& b, unsigned long long* tile_counts, uint8_t
     return cudaGetLastError();
 }
 
+int sepo_launch_tile_popc(const Batch& b, unsigned long long* tile_counts, int grid, cudaStream_t s) {
+    if (b.n) tile_popc_kernel<<<grid, 64, 0, s>>>(b, tile_counts);
+    return cudaGetLastError();
+}
 int sepo_launch_compact_index(const Batch& b, unsigned long long* tile_counts, uint64_t* idx_out, int grid, cudaStream_t s) {
     const uint64_t nt = sepo_reprobe_tiles(b.n);
     if (nt) {

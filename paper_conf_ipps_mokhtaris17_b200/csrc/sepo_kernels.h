@@ -27,6 +27,7 @@ int sepo_launch_reprobe(const sepo::Dev& d, const sepo::Batch& b, int mode, int 
 uint64_t sepo_reprobe_tiles(uint64_t n);
 int sepo_launch_compact(const sepo::Batch& b, unsigned long long* tile_counts, uint8_t* ok, uint64_t* oko, uint8_t* ov,
                         uint64_t* ovo, uint64_t m, uint64_t kb, uint64_t vb, int grid, cudaStream_t s);
+int sepo_launch_tile_popc(const sepo::Batch& b, unsigned long long* tile_counts, int grid, cudaStream_t s);
 int sepo_launch_compact_index(const sepo::Batch& b, unsigned long long* tile_counts, uint64_t* idx_out, int grid,
                               cudaStream_t s);
 int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);
