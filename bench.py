@@ -221,7 +221,7 @@ def run_reference(args):
 
 
 # ---------------------------------------------------------------- our arm
-def timed_steps(job, t, steps, stream):
+def timed_steps(job, t, steps, stream, route_fn=None):
     import torch
     k, o, v = job.inputs()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -229,6 +229,9 @@ def timed_steps(job, t, steps, stream):
     torch.cuda.synchronize()
     e0.record(stream)
     for _ in range(steps):
+        if route_fn is not None:  # sharded: route this rank's slice by key owner every step
+            k, o, v = route_fn()
+            launches += 2
         t.reset()
         t.run(k, o, v)
         st = t.stats()
@@ -251,8 +254,35 @@ def run_ours(args):
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if args.route and world == 1 and not dist.is_initialized():
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29511")
+        dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", local))
     job = Job(args.config, args.ratio, scale=args.scale)
     stream = torch.cuda.current_stream()
+    routed = world > 1 or args.route
+    fixed = job.stream.family == 2
+    route_fn = None
+    if routed:
+        # strong scaling: rank r holds records [r*n/W, (r+1)*n/W) of the SAME global stream; each
+        # step routes them by key hash (sepo_partition + NCCL all-to-all) and runs
+        # the SEPO job on the records this rank owns
+        from paper_conf_ipps_mokhtaris17_b200 import shard
+        if not dist.is_initialized():
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        n_all = job.stream.n
+        j0, j1 = rank * n_all // world, (rank + 1) * n_all // world
+        sk, so, sv = job.stream.device(j0, j1 - j0)
+        if fixed:
+            so = None
+
+        def route_fn():
+            return shard.route(sk, so, sv, route_seed=0x5eed, fixed_key_width=8 if fixed else 0,
+                               fixed_val_width=job.stream.val_width if sv is not None else 0)
+        job.distinct = max(1, job.distinct // world)  # keys per rank (sizes the directory)
+        job._inputs = route_fn()
+        job.slice_bytes = sk.numel() + (8 * (so.numel() - 1) if so is not None else 0) + (sv.numel() if sv is not None else 0)
+        job.slice_records = j1 - j0
     job.inputs()
     nb, pages, F = job.table_params()
     t = job.table()
@@ -265,17 +295,26 @@ def run_ours(args):
         dist.barrier()
     torch.cuda.synchronize()
     sampler.start()
-    ms, info = timed_steps(job, t, args.steps, stream)
+    ms, info = timed_steps(job, t, args.steps, stream, route_fn)
     clocks = sampler.stop()
     st = info["last"]
     if world > 1:
         tt = torch.tensor([ms], device="cuda")
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         ms = float(tt.item())
-    csr = job.csr_bytes()
-    n = job.stream.n
-    value = world * csr * args.steps / (ms / 1e3) / 1e9
-    recs_per_s = world * n * args.steps / (ms / 1e3)
+    if routed:  # strong scaling: the whole stream is split over the ranks
+        csr_all = job.slice_bytes
+        tt = torch.tensor([csr_all], device="cuda", dtype=torch.float64)
+        if world > 1:
+            dist.all_reduce(tt)
+        csr, n = float(tt.item()), job.stream.n
+        value = csr * args.steps / (ms / 1e3) / 1e9
+        recs_per_s = n * args.steps / (ms / 1e3)
+    else:
+        csr = job.csr_bytes()
+        n = job.stream.n
+        value = world * csr * args.steps / (ms / 1e3) / 1e9
+        recs_per_s = world * n * args.steps / (ms / 1e3)
 
     # roofline of the dominant kernel (insert, a1..a7): algorithmic bytes = CSR bytes of every
     # batch it was handed (key bytes + 8 B offset [+ value bytes]) over its CUDA-event time
@@ -289,7 +328,7 @@ def run_ours(args):
 
     # end to end through sepo_run with pinned HOST buffers (H2D + job + host result assembly)
     e2e = None
-    if args.e2e_steps > 0:
+    if args.e2e_steps > 0 and not routed:
         hk = torch.empty(k.numel(), dtype=torch.uint8, pin_memory=True); hk.copy_(k)
         ho = torch.empty(o.numel(), dtype=torch.int64, pin_memory=True).copy_(o) if o is not None else None
         hv = torch.empty(v.numel(), dtype=torch.uint8, pin_memory=True).copy_(v) if v is not None else None
@@ -315,7 +354,7 @@ def run_ours(args):
 
     # slowdown curve (M3): job time at table/budget = 0.5 .. 4 relative to 0.5
     curve = None
-    if args.curve and rank == 0:
+    if args.curve and rank == 0 and not routed:
         curve = {}
         base = None
         for r in (0.5, 1.0, 2.0, 3.0, 4.0):
@@ -341,7 +380,7 @@ def run_ours(args):
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
                 "warmup": max(args.warmup, 3), "ms_per_step": ms / args.steps, "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+                "scaling": "strong" if routed else "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
                 "kv_inserts_per_s": recs_per_s,
                 "config": {"workload": CONFIG_TEXT[args.config], "records": n, "input_csr_bytes": csr,
                            "distinct_keys": job.distinct, "ratio_table_over_budget": args.ratio,
@@ -349,13 +388,14 @@ def run_ours(args):
                            "n_buckets": nb, "page_bytes": job.page_bytes, "pool_pages": pages,
                            "passes": st["passes"], "postponed_per_pass": st["postponed_per_pass"],
                            "bytes_evicted": st["bytes_evicted"], "l2": "inputs (>= 15 GiB) far larger than L2 (126 MB)",
-                           "parallelism": f"replicas x{world}" if world > 1 else "1 GPU",
+                           "parallelism": (f"key-hash sharded x{world} (sepo_partition + NCCL all-to-all)" if routed
+                                           else "1 GPU"),
                            "phase_ms": {kk: st[kk] for kk in ("t_insert_ms", "t_reprobe_ms", "t_compact_ms", "t_evict_ms")}},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "gpu_launches": info["launches"], "slowdown_curve": curve}
         print(json.dumps(line), flush=True)
     t.close()
-    if world > 1:
+    if dist.is_initialized():
         dist.destroy_process_group()
 
 
@@ -373,6 +413,7 @@ def main():
     ap.add_argument("--no-cpu", dest="cpu_baseline", action="store_false")
     ap.add_argument("--ref-records", type=int, default=120_000_000)
     ap.add_argument("--ref-seconds", type=float, default=15.0)
+    ap.add_argument("--route", action="store_true", help="run the sharded (router) path even at N=1")
     ap.add_argument("--traffic", type=float, default=None, help="dram bytes/launch from an ncu --set full capture")
     args = ap.parse_args()
     if args.impl == "reference":

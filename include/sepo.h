@@ -181,6 +181,34 @@ int sepo_stats_get(const sepo_table* t, sepo_stats* out);
 double sepo_last_insert_ms(const sepo_table* t);
 
 void sepo_destroy(sepo_table* t);
+
+/* ---------------------------------------------------------------- multi-GPU key-hash router (a12)
+ * The method shards naturally: a key's result depends only on its own records, so the table is
+ * split across GPUs by owner(k) = hi32(H(route_seed, k)) * n_parts >> 32 (H = the table's key hash
+ * with another seed, so owner and bucket are independent). Each rank partitions its slice of the
+ * input, exchanges the parts with an all-to-all (NCCL over NVLink, driven by the caller's process
+ * group), then runs its own SEPO job; the union of the ranks' exports is the result (no merge). */
+
+/* Device scratch bytes sepo_partition needs for n records and n_parts parts. */
+size_t sepo_partition_scratch(uint64_t n, uint32_t n_parts);
+
+/* Stable partition of n records by owner (1 <= n_parts <= 32). Inputs as in sepo_insert_batch
+ * (key_offsets == NULL => fixed_key_width; vals == NULL => no values, else fixed_val_width bytes
+ * each). Outputs (device, caller-owned, same sizes as the inputs): out_keys, out_key_offsets
+ * (n entries: record j's offset relative to the first byte of ITS part; NULL for fixed-width
+ * keys), out_vals. part_starts (HOST, 3 * (n_parts + 1) u64): for part p, (first record, first key
+ * byte, first value byte) in the outputs; entry n_parts holds the totals. Records keep their input
+ * order within a part. Synchronizes the stream. */
+int sepo_partition(const uint8_t* keys, const uint64_t* key_offsets, uint32_t fixed_key_width, const uint8_t* vals,
+                   uint32_t fixed_val_width, uint64_t n, uint32_t n_parts, uint64_t route_seed, uint8_t* out_keys,
+                   uint64_t* out_key_offsets, uint8_t* out_vals, uint64_t* part_starts, void* scratch,
+                   size_t scratch_bytes, void* stream);
+
+/* After an exchange, key_offsets[0..n) holds n_segs received segments whose offsets are relative
+ * to their own key bytes. Adds seg_byte_base[s] to segment s (records [seg_rec_start[s],
+ * seg_rec_start[s+1]); device arrays of n_segs entries) and writes key_offsets[n] = total_bytes. */
+int sepo_shift_offsets(uint64_t* key_offsets, uint64_t n, const uint64_t* seg_rec_start, const uint64_t* seg_byte_base,
+                       uint32_t n_segs, uint64_t total_bytes, void* stream);
 const char* sepo_last_error(void);
 const char* sepo_version(void);
 

@@ -60,7 +60,8 @@ E_INVAL, E_NOMEM, E_TOOLARGE, E_CUDA, E_STATE, E_NCCL = -1, -2, -3, -4, -5, -6
 # every entry point declared in include/sepo.h
 EXPORTS = ["sepo_create", "sepo_configure", "sepo_insert_batch", "sepo_reprobe", "sepo_compact", "sepo_evict",
            "sepo_export", "sepo_run", "sepo_reset", "sepo_stats_get", "sepo_last_insert_ms", "sepo_destroy",
-           "sepo_last_error", "sepo_version", "sepo_budget_for"]
+           "sepo_last_error", "sepo_version", "sepo_budget_for", "sepo_partition_scratch", "sepo_partition",
+           "sepo_shift_offsets"]
 
 
 def budget_for(n_buckets, page_bytes, pool_pages):

@@ -953,3 +953,50 @@ void sepo_destroy(sepo_table* t) {
     if (t->copy_stream) cudaStreamDestroy(t->copy_stream);
     delete t;
 }
+
+// ---------------------------------------------------------------- key-hash router (a12)
+size_t sepo_partition_scratch(uint64_t n, uint32_t n_parts) {
+    return (size_t)sepo_partition_tiles(n) * n_parts * 3 * 8 + 256;
+}
+
+int sepo_partition(const uint8_t* keys, const uint64_t* ko, uint32_t kw, const uint8_t* vals, uint32_t vw, uint64_t n,
+                   uint32_t P, uint64_t route_seed, uint8_t* ok, uint64_t* oko, uint8_t* ov, uint64_t* part_starts,
+                   void* scratch, size_t scratch_bytes, void* stream) {
+    if (P < 1 || P > 32) return fail(SEPO_E_INVAL, "n_parts must be in [1, 32]");
+    if (!part_starts) return fail(SEPO_E_INVAL, "part_starts is NULL");
+    if (!ko && kw == 0) return fail(SEPO_E_INVAL, "key_offsets is NULL and fixed_key_width is 0");
+    if (vals && vw == 0) return fail(SEPO_E_INVAL, "fixed_val_width is 0");
+    if (scratch_bytes < sepo_partition_scratch(n, P)) return fail(SEPO_E_INVAL, "partition scratch too small");
+    if (n && (!keys || !ok || (ko && !oko) || (vals && !ov))) return fail(SEPO_E_INVAL, "NULL buffer");
+    Batch b;
+    b.keys = keys; b.ko = ko; b.kw = kw; b.vals = vals; b.vo = nullptr; b.vw = vw; b.n = n; b.bitmap = nullptr; b.idx = nullptr;
+    cudaStream_t s = (cudaStream_t)stream;
+    std::vector<unsigned long long> h(3 * P, 0);
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    int rc = sepo_launch_partition(b, P, route_seed ^ 0x6a09e667f3bcc909ull, (unsigned long long*)scratch, ok, oko, ov,
+                                   h.data(), sms, s);
+    if (rc) return fail(SEPO_E_CUDA, std::string("partition: ") + cudaGetErrorString((cudaError_t)rc));
+    cudaError_t e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return fail(SEPO_E_CUDA, std::string("partition: ") + cudaGetErrorString(e));
+    for (uint32_t p = 0; p < 3 * P; ++p) part_starts[p] = h[p];
+    part_starts[3 * P] = n;
+    part_starts[3 * P + 1] = ko ? 0 : n * (uint64_t)kw;
+    part_starts[3 * P + 2] = vals ? n * (uint64_t)vw : 0;
+    if (ko && n) {
+        uint64_t first = 0, last = 0;
+        cudaMemcpy(&first, ko, 8, cudaMemcpyDeviceToHost);
+        cudaMemcpy(&last, ko + n, 8, cudaMemcpyDeviceToHost);
+        part_starts[3 * P + 1] = last - first;
+    }
+    return 0;
+}
+
+int sepo_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const uint64_t* seg_base, uint32_t n_segs,
+                       uint64_t total, void* stream) {
+    if (!ko || (n && (!seg_rec || !seg_base || n_segs == 0))) return fail(SEPO_E_INVAL, "NULL argument");
+    int rc = sepo_launch_shift_offsets(ko, n, seg_rec, seg_base, n_segs, total, (cudaStream_t)stream);
+    if (rc) return fail(SEPO_E_CUDA, std::string("shift_offsets: ") + cudaGetErrorString((cudaError_t)rc));
+    return 0;
+}

@@ -16,6 +16,7 @@
 #include "sepo_dev.cuh"
 #include "sepo_kernels.h"
 #include <algorithm>
+#include <cstring>
 
 namespace sepo {
 
@@ -1132,6 +1133,126 @@ __global__ void __launch_bounds__(256) compact_index_kernel(Batch b, const unsig
     }
 }
 
+// ================================================================ key-hash router (a12, multi-GPU)
+// owner(k) = hi32(H(route_seed, k)) * P >> 32 — a hash independent of the table's bucket hash
+// (different seed), so a rank's keys spread over all of its buckets. A stable partition of the
+// batch by owner: per tile per part counts -> one exclusive scan in part-major order -> scatter,
+// so part p's records are contiguous, in input order, with offsets rebased to the part.
+constexpr int PT_THREADS = 1024, PT_TILE = 2048, PT_MAXP = 32;
+
+__device__ __forceinline__ uint32_t route_owner(const Batch& b, uint64_t i, uint64_t seed, uint32_t P, uint64_t& s,
+                                                uint32_t& len) {
+    rec_key(b, i, s, len);
+    const uint64_t h = hash_key(b.keys + s, len, seed);
+    return (uint32_t)(((h >> 32) * (uint64_t)P) >> 32);
+}
+
+__global__ void __launch_bounds__(PT_THREADS) part_count_kernel(Batch b, uint32_t P, uint64_t seed,
+                                                                unsigned long long* counts, uint64_t ntiles) {
+    __shared__ unsigned long long c[PT_MAXP][3];
+    for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        for (int x = threadIdx.x; x < PT_MAXP * 3; x += blockDim.x) (&c[0][0])[x] = 0;
+        __syncthreads();
+        for (int k = 0; k < PT_TILE / PT_THREADS; ++k) {
+            const uint64_t i = tile * PT_TILE + k * PT_THREADS + threadIdx.x;
+            if (i < b.n) {
+                uint64_t s; uint32_t len;
+                const uint32_t o = route_owner(b, i, seed, P, s, len);
+                atomicAdd(&c[o][0], 1ull);
+                atomicAdd(&c[o][1], (unsigned long long)len);
+                if (b.vals) atomicAdd(&c[o][2], (unsigned long long)b.vw);
+            }
+        }
+        __syncthreads();
+        for (uint32_t x = threadIdx.x; x < P * 3; x += blockDim.x)
+            counts[((uint64_t)(x / 3) * ntiles + tile) * 3 + (x % 3)] = c[x / 3][x % 3];
+        __syncthreads();
+    }
+}
+
+__global__ void __launch_bounds__(PT_THREADS) part_scatter_kernel(Batch b, uint32_t P, uint64_t seed,
+                                                                  const unsigned long long* base, uint64_t ntiles,
+                                                                  uint8_t* ok, uint64_t* oko, uint8_t* ov) {
+    constexpr int R = PT_TILE / PT_THREADS, NW = PT_THREADS / 32;
+    __shared__ unsigned int wrec[R][NW][PT_MAXP];
+    __shared__ unsigned long long wbytes[R][NW][PT_MAXP];
+    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        uint32_t own[R], rank[R], len[R];
+        uint64_t src[R], boff[R];
+        for (int k = 0; k < R; ++k) {
+            const uint64_t i = tile * PT_TILE + k * PT_THREADS + threadIdx.x;
+            const bool valid = i < b.n;
+            own[k] = 0xffu; len[k] = 0; src[k] = 0;
+            if (valid) own[k] = route_owner(b, i, seed, P, src[k], len[k]);
+            // per part present in the warp: exclusive rank and byte offset among its members
+            for (uint32_t p = lane; p < P; p += 32) { wrec[k][warp][p] = 0; wbytes[k][warp][p] = 0; }
+            __syncwarp();
+            unsigned todo = __ballot_sync(FULLMASK, valid);
+            rank[k] = 0; boff[k] = 0;
+            while (todo) {
+                const uint32_t p = __shfl_sync(FULLMASK, own[k], __ffs(todo) - 1);
+                const bool mem = valid && own[k] == p;
+                const unsigned mm = __ballot_sync(FULLMASK, mem);
+                todo &= ~mm;
+                const unsigned long long x = mem ? len[k] : 0ull;
+                unsigned long long incl = x;
+                for (int o = 1; o < 32; o <<= 1) {
+                    const unsigned long long y = __shfl_up_sync(FULLMASK, incl, o);
+                    if (lane >= (uint32_t)o) incl += y;
+                }
+                if (mem) { rank[k] = __popc(mm & ((1u << lane) - 1u)); boff[k] = incl - x; }
+                if (lane == 31) { wrec[k][warp][p] = __popc(mm); wbytes[k][warp][p] = incl; }
+                __syncwarp();
+            }
+        }
+        __syncthreads();
+        // exclusive prefix per part over the (k, warp) order, one thread per part
+        if (threadIdx.x < P) {
+            const uint32_t p = threadIdx.x;
+            unsigned int r = 0;
+            unsigned long long by = 0;
+            for (int k = 0; k < R; ++k)
+                for (int w = 0; w < NW; ++w) {
+                    const unsigned int r0 = wrec[k][w][p];
+                    const unsigned long long b0 = wbytes[k][w][p];
+                    wrec[k][w][p] = r; wbytes[k][w][p] = by;
+                    r += r0; by += b0;
+                }
+        }
+        __syncthreads();
+        for (int k = 0; k < R; ++k) {
+            const uint64_t i = tile * PT_TILE + k * PT_THREADS + threadIdx.x;
+            if (i >= b.n) continue;
+            const uint32_t p = own[k];
+            const unsigned long long rb = wrec[k][warp][p], bb = wbytes[k][warp][p];
+            const unsigned long long* bp = base + ((uint64_t)p * ntiles + tile) * 3;
+            const unsigned long long* b0 = base + ((uint64_t)p * ntiles) * 3;  // start of part p
+            const uint64_t orec = bp[0] + rb + rank[k];
+            const uint64_t obyte = bp[1] + bb + boff[k];
+            if (oko) oko[orec] = obyte - b0[1];  // rebased to the part's segment
+            for (uint32_t x = 0; x < len[k]; ++x) ok[obyte + x] = __ldg(b.keys + src[k] + x);
+            if (b.vals) {
+                const uint64_t vs = rec_index(b, i) * (uint64_t)b.vw;
+                for (uint32_t x = 0; x < b.vw; ++x) ov[orec * b.vw + x] = __ldg(b.vals + vs + x);
+            }
+        }
+        __syncthreads();
+    }
+}
+
+// received segments: offsets of segment s are relative to its own bytes; shift them by the bytes
+// of the segments before it and close the CSR with the total
+__global__ void shift_offsets_kernel(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const uint64_t* seg_base,
+                                     uint32_t n_segs, uint64_t total) {
+    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < n; j += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t sgi = 0;
+        while (sgi + 1 < n_segs && seg_rec[sgi + 1] <= j) ++sgi;
+        ko[j] += seg_base[sgi];
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) ko[n] = total;
+}
+
 // ================================================================ pass boundary (a10)
 // Seal every open page (filler over its unused tail) and reset the CTA cursors.
 __global__ void seal_kernel(Dev d, uint32_t n_slots) {
@@ -1330,6 +1451,27 @@ int sepo_launch_compact_index(const Batch& b, unsigned long long* tile_counts, u
         scan_tiles_kernel<<<1, 1024, 0, s>>>(tile_counts, nt);
         compact_index_kernel<<<grid, 256, 0, s>>>(b, tile_counts, idx_out);
     }
+    return cudaGetLastError();
+}
+int sepo_launch_partition(const Batch& b, uint32_t P, uint64_t seed, unsigned long long* counts, uint8_t* ok,
+                          uint64_t* oko, uint8_t* ov, unsigned long long* h_counts, int grid, cudaStream_t s) {
+    const uint64_t ntiles = (b.n + PT_TILE - 1) / PT_TILE;
+    if (ntiles == 0) { memset(h_counts, 0, sizeof(unsigned long long) * 3 * P); return 0; }
+    part_count_kernel<<<grid, PT_THREADS, 0, s>>>(b, P, seed, counts, ntiles);
+    // per-part totals (before the scan turns counts into bases): copy the last base later instead
+    scan_tiles_kernel<<<1, 1024, 0, s>>>(counts, (uint64_t)P * ntiles);
+    part_scatter_kernel<<<grid, PT_THREADS, 0, s>>>(b, P, seed, counts, ntiles, ok, oko, ov);
+    // part starts (the bases of tile 0 of every part) to the host: totals follow by difference
+    for (uint32_t p = 0; p < P; ++p)
+        cudaMemcpyAsync(h_counts + 3 * p, counts + (uint64_t)p * ntiles * 3, 3 * sizeof(unsigned long long),
+                        cudaMemcpyDeviceToHost, s);
+    return cudaGetLastError();
+}
+uint64_t sepo_partition_tiles(uint64_t n) { return (n + PT_TILE - 1) / PT_TILE; }
+int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const uint64_t* seg_base, uint32_t n_segs,
+                              uint64_t total, cudaStream_t s) {
+    shift_offsets_kernel<<<(unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n + 255) / 256, 4096)), 256, 0, s>>>(
+        ko, n, seg_rec, seg_base, n_segs, total);
     return cudaGetLastError();
 }
 int sepo_launch_seal(const Dev& d, uint32_t n_slots, cudaStream_t s) {

@@ -30,6 +30,11 @@ int sepo_launch_compact(const sepo::Batch& b, unsigned long long* tile_counts, u
 int sepo_launch_tile_popc(const sepo::Batch& b, unsigned long long* tile_counts, int grid, cudaStream_t s);
 int sepo_launch_compact_index(const sepo::Batch& b, unsigned long long* tile_counts, uint64_t* idx_out, int grid,
                               cudaStream_t s);
+int sepo_launch_partition(const sepo::Batch& b, uint32_t P, uint64_t seed, unsigned long long* counts, uint8_t* ok,
+                          uint64_t* oko, uint8_t* ov, unsigned long long* h_counts, int grid, cudaStream_t s);
+uint64_t sepo_partition_tiles(uint64_t n);
+int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const uint64_t* seg_base, uint32_t n_segs,
+                              uint64_t total, cudaStream_t s);
 int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);
 int sepo_launch_classify(const sepo::Dev& d, int honor_retain, cudaStream_t s);
 int sepo_launch_relink(const sepo::Dev& d, cudaStream_t s);

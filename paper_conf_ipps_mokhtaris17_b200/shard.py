@@ -1,0 +1,102 @@
+"""Multi-GPU key-hash sharding: partition -> all-to-all -> local SEPO job.
+
+One process per GPU. `torch.distributed` (backend "nccl" on GPUs, "gloo" in CPU tests) carries the
+all-to-all; the partition and the offset rebasing run in libsepo's kernels (sepo_partition,
+sepo_shift_offsets). A key's records all land on its owner rank, so every rank's export is final
+and the union over ranks is the result (no merge).
+"""
+import ctypes
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+from . import _err, _ptr, lib
+
+_bound = False
+
+
+def _bind():
+    global _bound
+    if _bound:
+        return
+    L = lib()
+    vp, u64, u32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32
+    L.sepo_partition_scratch.argtypes = [u64, u32]
+    L.sepo_partition_scratch.restype = ctypes.c_size_t
+    L.sepo_partition.argtypes = [vp, vp, u32, vp, u32, u64, u32, u64, vp, vp, vp, vp, vp, ctypes.c_size_t, vp]
+    L.sepo_partition.restype = ctypes.c_int
+    L.sepo_shift_offsets.argtypes = [vp, u64, vp, vp, u32, u64, vp]
+    L.sepo_shift_offsets.restype = ctypes.c_int
+    _bound = True
+
+
+def partition(keys, key_offsets, vals, n_parts, route_seed=0, fixed_key_width=0, fixed_val_width=0):
+    """Stable partition of a device batch by key owner. -> (keys, key_offsets or None, vals or None,
+    starts) where starts[p] = (first record, first key byte, first value byte) of part p and
+    starts[n_parts] = totals (numpy uint64 [n_parts + 1, 3]). Offsets are relative to each part."""
+    _bind()
+    L = lib()
+    n = (key_offsets.numel() - 1) if key_offsets is not None else keys.numel() // fixed_key_width
+    ok = torch.empty_like(keys)
+    oko = torch.empty(max(n, 1), dtype=torch.int64, device=keys.device) if key_offsets is not None else None
+    ov = torch.empty_like(vals) if vals is not None else None
+    scratch = torch.empty(int(L.sepo_partition_scratch(n, n_parts)), dtype=torch.uint8, device=keys.device)
+    starts = np.zeros(3 * (n_parts + 1), dtype=np.uint64)
+    stream = torch.cuda.current_stream(keys.device).cuda_stream
+    rc = L.sepo_partition(_ptr(keys), _ptr(key_offsets), fixed_key_width, _ptr(vals), fixed_val_width, n, n_parts,
+                          route_seed, _ptr(ok), _ptr(oko), _ptr(ov), starts.ctypes.data, scratch.data_ptr(),
+                          scratch.numel(), ctypes.c_void_p(stream))
+    if rc:
+        _err(rc)
+    return ok, (oko[:n] if oko is not None else None), ov, starts.reshape(n_parts + 1, 3)
+
+
+def shift_offsets_cuda(ko, seg_rec, seg_base, total):
+    """ko[j] += seg_base[s] for records of segment s; ko[n] = total (libsepo kernel)."""
+    _bind()
+    n = ko.numel() - 1
+    dev = ko.device
+    sr = torch.as_tensor(np.asarray(seg_rec, dtype=np.int64), device=dev)
+    sb = torch.as_tensor(np.asarray(seg_base, dtype=np.int64), device=dev)
+    rc = lib().sepo_shift_offsets(ko.data_ptr(), n, sr.data_ptr(), sb.data_ptr(), len(seg_rec), int(total),
+                                  ctypes.c_void_p(torch.cuda.current_stream(dev).cuda_stream))
+    if rc:
+        _err(rc)
+    return ko
+
+
+def exchange(ok, oko, ov, starts, group=None, shift_fn=shift_offsets_cuda):
+    """All-to-all of the parts (part p -> rank p). -> (keys, key_offsets [n+1] or None, vals or None)
+    for the records this rank owns, in sender-rank order (sender's input order within a sender)."""
+    world = dist.get_world_size(group)
+    starts = np.asarray(starts, dtype=np.int64)
+    send = np.diff(starts, axis=0)  # [world, 3]: records, key bytes, value bytes per destination
+    dev = ok.device
+    send_t = torch.as_tensor(send.reshape(-1), dtype=torch.int64, device=dev)
+    recv_t = torch.empty_like(send_t)
+    dist.all_to_all_single(recv_t, send_t, group=group)
+    recv = recv_t.cpu().numpy().reshape(world, 3)
+    nrec, nkb, nvb = (int(x) for x in recv.sum(axis=0))
+    rk = torch.empty(max(nkb, 1), dtype=torch.uint8, device=dev)
+    dist.all_to_all_single(rk[:nkb], ok, recv[:, 1].tolist(), send[:, 1].tolist(), group=group)
+    rko = None
+    if oko is not None:
+        rko = torch.empty(nrec + 1, dtype=torch.int64, device=dev)
+        dist.all_to_all_single(rko[:nrec], oko, recv[:, 0].tolist(), send[:, 0].tolist(), group=group)
+        seg_rec = np.concatenate([[0], np.cumsum(recv[:, 0])[:-1]])
+        seg_base = np.concatenate([[0], np.cumsum(recv[:, 1])[:-1]])
+        shift_fn(rko, seg_rec, seg_base, nkb)
+    rv = None
+    if ov is not None:
+        rv = torch.empty(max(nvb, 1), dtype=torch.uint8, device=dev)
+        dist.all_to_all_single(rv[:nvb], ov, recv[:, 2].tolist(), send[:, 2].tolist(), group=group)
+        rv = rv[:nvb]
+    return rk[:nkb], rko, rv
+
+
+def route(keys, key_offsets, vals, group=None, route_seed=0, fixed_key_width=0, fixed_val_width=0):
+    """partition + exchange: the records of this rank's keys."""
+    world = dist.get_world_size(group)
+    ok, oko, ov, starts = partition(keys, key_offsets, vals, world, route_seed, fixed_key_width, fixed_val_width)
+    return exchange(ok, oko, ov, starts, group)

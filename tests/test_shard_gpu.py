@@ -1,0 +1,109 @@
+"""GPU checks of the key-hash router (row a12) on one device: the partition kernel's properties
+and a P-way sharded SEPO job run as P loopback "ranks" (one table each) against the oracle."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from tests.util import oracle_expected
+
+pytestmark = pytest.mark.gpu
+
+
+def sepo():
+    import paper_conf_ipps_mokhtaris17_b200 as m
+    return m
+
+
+def segment(ok, oko, starts, p):
+    r0, r1 = int(starts[p][0]), int(starts[p + 1][0])
+    b0, b1 = int(starts[p][1]), int(starts[p + 1][1])
+    ko = torch.empty(r1 - r0 + 1, dtype=torch.int64, device=ok.device)
+    ko[:-1] = oko[r0:r1]
+    ko[-1] = b1 - b0
+    return ok[b0:b1], ko
+
+
+@pytest.mark.parametrize("P", [1, 2, 5, 8])
+def test_partition_properties(cuda, P):
+    from paper_conf_ipps_mokhtaris17_b200 import shard
+    s = gen.config("C3", scale=1 / 4000)
+    k, o, _ = s.device()
+    ok, oko, _, starts = shard.partition(k, o, None, P, route_seed=7)
+    assert int(starts[P][0]) == s.n and int(starts[P][1]) == k.numel()
+    keysets, all_counts = [], oracle.Combine()
+    for p in range(P):
+        sk, so = segment(ok, oko, starts, p)
+        # purity: partitioning a part again keeps every record in the same part
+        _, _, _, st2 = shard.partition(sk, so, None, P, route_seed=7)
+        n_p = so.numel() - 1
+        assert int(st2[p + 1][0] - st2[p][0]) == n_p
+        hk, ho = sk.cpu().numpy(), so.cpu().numpy().view(np.uint64)
+        d = oracle.combine(hk, ho).as_dict()
+        keysets.append(set(d))
+        all_counts.add(hk, ho)
+    # disjoint key sets, and the records are a permutation of the input
+    for a in range(P):
+        for b in range(a + 1, P):
+            assert not (keysets[a] & keysets[b])
+    assert all_counts.as_dict() == oracle_expected(s)
+
+
+def test_partition_is_stable_and_carries_values(cuda):
+    from paper_conf_ipps_mokhtaris17_b200 import shard
+    s = gen.config("C5u", scale=2 ** -14)  # fixed 8-byte keys, 8-byte values
+    k, _, v = s.device()
+    P = 4
+    ok, oko, ov, starts = shard.partition(k, None, v, P, route_seed=3, fixed_key_width=8, fixed_val_width=8)
+    assert oko is None
+    hk = k.cpu().numpy().view(np.uint64)
+    hv = v.cpu().numpy().view(np.uint64)
+    pk = ok.cpu().numpy().view(np.uint64)
+    pv = ov.cpu().numpy().view(np.uint64)
+    pos = 0
+    seen = np.zeros(s.n, dtype=bool)
+    for p in range(P):
+        r0, r1 = int(starts[p][0]), int(starts[p + 1][0])
+        # records of part p appear in input order: their (key, value) pairs are a subsequence
+        idx = []
+        j = 0
+        for x in range(r0, r1):
+            while not (hk[j] == pk[x] and hv[j] == pv[x] and not seen[j]):
+                j += 1
+            seen[j] = True
+            idx.append(j)
+        assert idx == sorted(idx)
+    assert seen.all()
+
+
+@pytest.mark.parametrize("name,P", [("C3", 4), ("C5z", 3), ("C2", 8)])
+def test_sharded_job_loopback(cuda, name, P):
+    """P loopback ranks: partition, one SEPO table per part (budget 2x over), union == oracle."""
+    from paper_conf_ipps_mokhtaris17_b200 import shard
+    scale = {"C3": 1 / 4000, "C5z": 2 ** -12, "C2": 1 / 512}[name]
+    s = gen.config(name, scale=scale)
+    exp = oracle_expected(s)
+    k, o, v = s.device()
+    fixed = s.family == gen.GEN_PAIRS
+    ok, oko, ov, starts = shard.partition(k, None if fixed else o, v, P, route_seed=11,
+                                          fixed_key_width=8 if fixed else 0, fixed_val_width=8 if v is not None else 0)
+    got = {}
+    for p in range(P):
+        r0, r1 = int(starts[p][0]), int(starts[p + 1][0])
+        kw = dict(mode=sepo().COMBINE)
+        if fixed:
+            sk, so = ok[int(starts[p][1]):int(starts[p + 1][1])], None
+            sv = ov[int(starts[p][2]):int(starts[p + 1][2])]
+            kw.update(fixed_key_width=8, fixed_val_width=8)
+        else:
+            sk, so = segment(ok, oko, starts, p)
+            sv = None
+        t = sepo().Table(sepo().budget_for(1 << 14, 16384, 64), 1 << 14, 16384, check_dups=True, **kw)
+        t.run(sk, so, sv, n=r1 - r0)
+        part = sepo().result_dict(t.export())
+        assert t.stats()["cross_gen_dups"] == 0
+        t.close()
+        assert not (set(part) & set(got))  # shards own disjoint keys
+        got.update(part)
+    assert got == exp
