@@ -95,6 +95,8 @@ typedef struct sepo_stats {
     uint64_t key_bytes_inserted;   /* key bytes handed to sepo_insert_batch */
     uint64_t val_bytes_inserted;   /* value bytes handed to sepo_insert_batch */
     uint64_t kernel_launches;      /* this library's kernels launched since create/reset */
+    uint64_t value_chunks;         /* GROUP export: value chunks parsed */
+    uint64_t value_slots;          /* GROUP export: value slots in those chunks (capacity) */
     double t_insert_ms, t_reprobe_ms, t_compact_ms, t_evict_ms, t_export_ms, t_h2d_ms;
 } sepo_stats;
 

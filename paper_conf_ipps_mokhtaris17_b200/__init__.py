@@ -13,7 +13,7 @@ import numpy as np
 __all__ = ["Table", "SepoError", "lib", "COMBINE", "GROUP", "Stats"]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "lib", "libsepo.so")
+LIB_PATH = os.environ.get("SEPO_LIB") or os.path.join(_HERE, "lib", "libsepo.so")
 COMBINE, GROUP = 0, 1
 _LIB = None
 
@@ -39,7 +39,7 @@ class Stats(ctypes.Structure):
                 ("n_buckets", u64), ("page_bytes", u64), ("pool_pages", u64), ("grid_ctas", u64),
                 ("pages_used_max", u64), ("bytes_evicted", u64), ("dead_bytes", u64), ("cross_gen_dups", u64),
                 ("forced_full_evictions", u64), ("toolarge", u64),
-                ("key_bytes_inserted", u64), ("val_bytes_inserted", u64), ("kernel_launches", u64), ("t_insert_ms", ctypes.c_double),
+                ("key_bytes_inserted", u64), ("val_bytes_inserted", u64), ("kernel_launches", u64), ("value_chunks", u64), ("value_slots", u64), ("t_insert_ms", ctypes.c_double),
                 ("t_reprobe_ms", ctypes.c_double), ("t_compact_ms", ctypes.c_double), ("t_evict_ms", ctypes.c_double),
                 ("t_export_ms", ctypes.c_double), ("t_h2d_ms", ctypes.c_double)]
 

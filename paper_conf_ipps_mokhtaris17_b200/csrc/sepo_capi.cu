@@ -11,6 +11,7 @@
 
 #include <algorithm>
 #include <chrono>
+#include <functional>
 #include <atomic>
 #include <string>
 #include <string_view>
@@ -84,7 +85,7 @@ struct sepo_table {
     sepo_options opts{};
     cudaStream_t stream = nullptr, copy_stream = nullptr;
     bool own_stream = false;
-    cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev_copy = nullptr, ev_comp = nullptr;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev_copy = nullptr, ev_comp = nullptr, evc0 = nullptr, evc1 = nullptr;
     Ctrl* h_ctrl = nullptr;        // pinned mirror of the device control block
     uint32_t* h_evict = nullptr;   // pinned evict list
     uint64_t* h_ko = nullptr;      // pinned: first/last key offset of the last insert batch
@@ -295,6 +296,8 @@ sepo_table* sepo_create(size_t budget, uint64_t n_buckets, uint32_t page_bytes) 
     cudaStreamCreateWithFlags(&t->copy_stream, cudaStreamNonBlocking);
     cudaEventCreate(&t->ev0);
     cudaEventCreate(&t->ev1);
+    cudaEventCreate(&t->evc0);
+    cudaEventCreate(&t->evc1);
     cudaEventCreateWithFlags(&t->ev_copy, cudaEventDisableTiming);
     cudaEventCreateWithFlags(&t->ev_comp, cudaEventDisableTiming);
     cudaHostAlloc((void**)&t->h_ctrl, sizeof(Ctrl), cudaHostAllocDefault);
@@ -482,18 +485,20 @@ int64_t sepo_compact(sepo_table* t, const uint8_t* keys, const uint64_t* ko, con
 // a9 by index (sepo_run): the postponed records of batch b as indices into the original arrays
 static int64_t compact_index_impl(sepo_table* t, const Batch& b, uint64_t m, uint64_t* idx_out) {
     int rc;
-    CK(t, cudaEventRecord(t->ev0, t->stream));
+    CK(t, cudaEventRecord(t->evc0, t->stream));
     rc = sepo_launch_compact_index(b, (unsigned long long*)t->tile_counts.p, idx_out, 8 * t->n_sms, t->stream);
     if (rc) return cuda_check(t, (cudaError_t)rc, "compact_index kernel launch");
     t->st.kernel_launches += 2;
-    CK(t, cudaEventRecord(t->ev1, t->stream));
-    CK(t, cudaEventSynchronize(t->ev1));
-    t->st.t_compact_ms += elapsed_ms(t->ev0, t->ev1);
+    CK(t, cudaEventRecord(t->evc1, t->stream));
+    CK(t, cudaEventSynchronize(t->evc1));
+    t->st.t_compact_ms += elapsed_ms(t->evc0, t->evc1);
     return (int64_t)m;
 }
 
 // Pass boundary. honor_retain = 0 evicts every resident page (final export / forced).
-static int64_t evict_impl(sepo_table* t, int honor_retain) {
+// `overlap` (optional) enqueues compute-stream work that does not touch the pool (the re-issue
+// compaction): it runs while the evicted pages stream to host memory on the copy stream (a10).
+static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<int()>& overlap = nullptr) {
     CK(t, cudaEventRecord(t->ev0, t->stream));
     sync_dev(t);
     int rc = sepo_launch_seal(t->d, (uint32_t)t->grid, t->stream);
@@ -529,6 +534,10 @@ static int64_t evict_impl(sepo_table* t, int honor_retain) {
         i = j;
     }
     CK(t, cudaEventRecord(t->ev_copy, t->copy_stream));
+    if (overlap) {
+        int orc = overlap();
+        if (orc) return orc;
+    }
     // the freed pages are reused only after their copy finished
     CK(t, cudaStreamWaitEvent(t->stream, t->ev_copy, 0));
     CK(t, cudaMemsetAsync(t->d.dir, 0, t->n_buckets * 4, t->stream));
@@ -687,6 +696,7 @@ int export_group(sepo_table* t) {
     // pass A: key entries (identity = birth gen << 40 | entry ref) and value chunks
     struct KeyRec { const uint8_t* key; uint32_t len; uint64_t id; };
     struct ChunkRec { const uint8_t* vals; uint32_t cnt; uint64_t owner; };
+    std::vector<uint64_t> slots(16, 0);
     std::vector<std::vector<KeyRec>> tk(16);
     std::vector<std::vector<ChunkRec>> tc(16);
     std::atomic<int> bad{0};
@@ -714,6 +724,7 @@ int export_group(sepo_table* t) {
                     memcpy(&owner, base + off + 8, 8);
                     memcpy(&cap, base + off + 24, 4);
                     tc[w].push_back({base + off + CHUNK_HDR, std::min(fill, cap), owner});
+                    slots[w] += cap;
                 }
                 off += sz;
             }
@@ -739,6 +750,10 @@ int export_group(sepo_table* t) {
             id2k[kr.id] = k;
         }
     t->st.cross_gen_dups = dups;
+    t->st.value_chunks = 0;
+    t->st.value_slots = 0;
+    for (auto& v : tc) t->st.value_chunks += v.size();
+    for (auto x : slots) t->st.value_slots += x;
     const uint64_t nk = keys.size();
     std::vector<uint64_t> cnt(nk + 1, 0);
     for (auto& v : tc)
@@ -873,8 +888,7 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
         // re-issue by index: the postponed records stay where they are in the caller's arrays
         if (t->idxb[side].grow((uint64_t)c * 8)) return fail(SEPO_E_NOMEM, "re-issue index list");
         uint64_t* nidx = (uint64_t*)t->idxb[side].p;
-        int64_t m = compact_index_impl(t, cur, (uint64_t)c, nidx);
-        if (m < 0) return m;
+        const int64_t m = c;
         // GROUP: a pass without progress (retained key pages starve the pool) evicts everything
         // (the paper is silent; reading R14)
         int honor = 1;
@@ -883,7 +897,11 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
             t->st.forced_full_evictions++;
         }
         prev = (uint64_t)m;
-        int64_t e = evict_impl(t, honor);
+        // the compaction only reads the bitmap: it overlaps the eviction's D2H copies
+        int64_t e = evict_impl(t, honor, [&]() -> int {
+            const int64_t mm = compact_index_impl(t, cur, (uint64_t)c, nidx);
+            return mm < 0 ? (int)mm : 0;
+        });
         if (e < 0) return e;
         cur.idx = nidx;
         cur.n = (uint64_t)m;
@@ -947,6 +965,8 @@ void sepo_destroy(sepo_table* t) {
     if (t->region) cudaFree(t->region);
     if (t->ev0) cudaEventDestroy(t->ev0);
     if (t->ev1) cudaEventDestroy(t->ev1);
+    if (t->evc0) cudaEventDestroy(t->evc0);
+    if (t->evc1) cudaEventDestroy(t->evc1);
     if (t->ev_copy) cudaEventDestroy(t->ev_copy);
     if (t->ev_comp) cudaEventDestroy(t->ev_comp);
     if (t->own_stream && t->stream) cudaStreamDestroy(t->stream);

@@ -84,12 +84,15 @@ __device__ __forceinline__ void rec_val_span(const Batch& b, uint64_t i, uint64_
 }
 
 // ---------------------------------------------------------------- GROUP value-list helpers
-// Value chunk capacity for k values when the key's head chunk has capacity `prev` (0: none in
-// this generation): geometric growth so a hot key's list is a few large chunks.
+// Value chunk capacity for k values about to be appended: twice the demand (at least 8 slots).
+// Sized by the demand rather than grown from the previous chunk: many CTAs may find a hot key's
+// head chunk full at once and each installs a chunk, so large geometric chunks would mostly stay
+// empty (measured: 8x slot over-allocation on C4 with doubling).
 __device__ __forceinline__ uint32_t chunk_cap(const Dev& d, uint32_t k, uint32_t prev, uint32_t slot_bytes) {
-    uint32_t maxcap = (d.page_bytes / 4 - CHUNK_HDR) / slot_bytes;
-    uint32_t c = prev ? min(prev * 2u, maxcap) : 4u;
-    c = max(c, k);
+    (void)prev;
+    const uint32_t maxcap = (d.page_bytes / 4 - CHUNK_HDR) / slot_bytes;
+    uint32_t c = max(8u, 2u * k);
+    c = min(c, max(maxcap, k));
     return min(c, (d.page_bytes - CHUNK_HDR) / slot_bytes);
 }
 __device__ __forceinline__ uint32_t chunk_bytes(uint32_t cap, uint32_t slot_bytes) { return align16(CHUNK_HDR + cap * slot_bytes); }
@@ -603,7 +606,12 @@ __global__ void __launch_bounds__(1024) hot_resolve_kernel(Dev d, Batch b, hot::
 }
 
 namespace stream {
-constexpr int THREADS = 1024;
+#ifndef SEPO_STREAM_THREADS
+#define SEPO_STREAM_THREADS 1024  // measured best (profiles/r01_summary.md): 32 warps x 1 group
+#define SEPO_STREAM_SUB 1
+#endif
+constexpr int THREADS = SEPO_STREAM_THREADS;  // warps x groups in flight per warp: see DESIGN.md §6
+constexpr int SUB = SEPO_STREAM_SUB;
 struct Smem {
     uint4 tags[hot::NB];  // 4 fingerprints per bucket (one 16-B load per probed bucket)
     uint64_t h[hot::NH], w0[hot::NH], w1[hot::NH];
@@ -622,10 +630,9 @@ __device__ __forceinline__ void smem_add_u64(unsigned int* lo, unsigned int* hi,
     if (vh) atomicAdd(hi, vh);
 }
 
-template <bool VALS>
-__global__ void __launch_bounds__(stream::THREADS, 1) insert_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
-                                                                           const unsigned int* n_hot) {
-    using stream::THREADS;
+template <bool VALS, int THREADS, int SUB>
+__global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
+                                                                   const unsigned int* n_hot) {
     extern __shared__ __align__(16) uint8_t smem_raw[];
     stream::Smem& S = *reinterpret_cast<stream::Smem*>(smem_raw);
     const uint32_t tid = threadIdx.x, lane = lane_id();
@@ -659,172 +666,190 @@ __global__ void __launch_bounds__(stream::THREADS, 1) insert_stream_kernel(Dev d
     const bool have_hot = nh > 0;
     const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
 
-    // Each warp streams 32-record groups. Order per group: hot probe first (shared memory), then
-    // the directory load for the misses is issued and overlaps the folding of the hits; the
-    // misses then walk their chains (one record per lane: tail keys rarely repeat in a warp).
+    // Each warp streams SUB 32-record groups per step, stage by stage, so the loads of the SUB
+    // groups are in flight together (memory-level parallelism without more warps): input words
+    // and hashes; hot-set probe (shared memory); directory loads of the misses; folding of the
+    // hits; chain walks of the misses (one record per lane: tail keys rarely repeat in a warp).
     const uint64_t ngroups = (b.n + 31) / 32;
     const uint64_t gw = (uint64_t)blockIdx.x * (THREADS / 32) + (tid >> 5);
     const uint64_t nw = (uint64_t)gridDim.x * (THREADS / 32);
     unsigned long long c_post = 0, c_tl = 0, c_dead = 0, c_pkb = 0;
     bool w_full = false, w_quiet = false;  // warp-uniform: pool ran out / quiescence observed
-    // software pipeline: the next group's key offsets and first 16 key bytes are loaded while
-    // the current group's lookups are in flight
-    uint64_t ns = 0, nw0 = 0, nw1 = 0;
-    uint32_t nlen = 0;
-    if (gw < ngroups && gw * 32 + lane < b.n) {
-        rec_key(b, gw * 32 + lane, ns, nlen);
-        load_key16(b.keys + ns, nlen, nw0, nw1);
-    }
-    for (uint64_t g = gw; g < ngroups; g += nw) {
-        const uint64_t i = g * 32 + lane;
-        const bool valid = i < b.n;
-        const uint64_t s = ns, w0 = nw0, w1 = nw1;
-        const uint32_t len = nlen;
-        uint64_t h = 0, v = 1;
-        if (valid) {
-            uint64_t x = hash_init(len, d.seed);
-            if (len > 0) x = hash_word(x, w0);
-            if (len > 8) x = hash_word(x, w1);
-            for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(b.keys + s + o, len - o < 8 ? len - o : 8));
-            h = fmix64(x);
-            if (VALS) v = rec_value(b, i);
+    for (uint64_t g0 = gw * SUB; g0 < ngroups; g0 += nw * SUB) {
+        uint64_t s[SUB], w0[SUB], w1[SUB], h[SUB], v[SUB];
+        uint32_t len[SUB];
+        bool valid[SUB];
+#pragma unroll
+        for (int q = 0; q < SUB; ++q) {
+            const uint64_t i = (g0 + q) * 32 + lane;
+            valid[q] = i < b.n;
+            s[q] = 0; len[q] = 0; w0[q] = 0; w1[q] = 0; v[q] = 1;
+            if (valid[q]) {
+                rec_key(b, i, s[q], len[q]);
+                load_key16(b.keys + s[q], len[q], w0[q], w1[q]);
+                if (VALS) v[q] = rec_value(b, i);
+            }
         }
-        {   // issue the next group's offsets now; its key bytes at the end of this iteration
-            const uint64_t gn = g + nw;
-            ns = 0; nlen = 0;
-            if (gn < ngroups && gn * 32 + lane < b.n) rec_key(b, gn * 32 + lane, ns, nlen);
+#pragma unroll
+        for (int q = 0; q < SUB; ++q) {
+            uint64_t x = hash_init(len[q], d.seed);
+            if (len[q] > 0) x = hash_word(x, w0[q]);
+            if (len[q] > 8) x = hash_word(x, w1[q]);
+            for (uint32_t o = 16; o < len[q]; o += 8)
+                x = hash_word(x, load_in_word(b.keys + s[q] + o, len[q] - o < 8 ? len[q] - o : 8));
+            h[q] = fmix64(x);
         }
         // ---- hot set: constant-time probe of two 4-way buckets, then a full-key check
-        int pos = -1;
-        if (valid && have_hot) {
-            const uint32_t f = hot::fp(h);
-            const uint32_t k1 = hot::b1(h), k2 = hot::b2(h);
-            const uint4 t1 = S.tags[k1];
-            if (t1.x == f) pos = 4 * k1; else if (t1.y == f) pos = 4 * k1 + 1;
-            else if (t1.z == f) pos = 4 * k1 + 2; else if (t1.w == f) pos = 4 * k1 + 3;
-            else {
-                const uint4 t2 = S.tags[k2];
-                if (t2.x == f) pos = 4 * k2; else if (t2.y == f) pos = 4 * k2 + 1;
-                else if (t2.z == f) pos = 4 * k2 + 2; else if (t2.w == f) pos = 4 * k2 + 3;
+        int pos[SUB];
+#pragma unroll
+        for (int q = 0; q < SUB; ++q) {
+            pos[q] = -1;
+            if (valid[q] && have_hot) {
+                const uint32_t f = hot::fp(h[q]);
+                const uint32_t k1 = hot::b1(h[q]), k2 = hot::b2(h[q]);
+                const uint4 t1 = S.tags[k1];
+                int p = -1;
+                if (t1.x == f) p = 4 * k1; else if (t1.y == f) p = 4 * k1 + 1;
+                else if (t1.z == f) p = 4 * k1 + 2; else if (t1.w == f) p = 4 * k1 + 3;
+                else {
+                    const uint4 t2 = S.tags[k2];
+                    if (t2.x == f) p = 4 * k2; else if (t2.y == f) p = 4 * k2 + 1;
+                    else if (t2.z == f) p = 4 * k2 + 2; else if (t2.w == f) p = 4 * k2 + 3;
+                }
+                if (p >= 0 && S.h[p] == h[q] && S.len[p] == len[q] && S.w0[p] == w0[q] && S.w1[p] == w1[q] &&
+                    (len[q] <= 16 || entry_key_eq(ref_ptr(d, S.ref[p]) + KEY_OFF + 16, b.keys + s[q] + 16, len[q] - 16)))
+                    pos[q] = p;
             }
-            if (pos >= 0 && !(S.h[pos] == h && S.len[pos] == len && S.w0[pos] == w0 && S.w1[pos] == w1 &&
-                              (len <= 16 || entry_key_eq(ref_ptr(d, S.ref[pos]) + KEY_OFF + 16, b.keys + s + 16, len - 16))))
-                pos = -1;
         }
-        const bool miss = valid && pos < 0;
-        const uint8_t* tail = b.keys + s + 16;
-        const uint32_t bkt = bucket_of(h, d.n_buckets);
-        const uint32_t tag = tag_of(h);
-        uint32_t head = 0;
-        if (miss) head = ld_relaxed_u32(d.dir + bkt);  // in flight while the hits are folded
+        // ---- directory loads of the misses: in flight while the hits are folded
+        uint32_t head[SUB];
+#pragma unroll
+        for (int q = 0; q < SUB; ++q) {
+            head[q] = 0;
+            if (valid[q] && pos[q] < 0) head[q] = ld_relaxed_u32(d.dir + bucket_of(h[q], d.n_buckets));
+        }
         // ---- fold the hits of the warp per hot slot (a2): one shared atomic per distinct key
-        const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
-        if (hm) {
-            const unsigned key = pos >= 0 ? (unsigned)pos : (0x10000u | lane);
+#pragma unroll
+        for (int q = 0; q < SUB; ++q) {
+            const unsigned hm = __ballot_sync(FULLMASK, pos[q] >= 0);
+            if (!hm) continue;
+            const unsigned key = pos[q] >= 0 ? (unsigned)pos[q] : (0x10000u | lane);
             const unsigned grp = __match_any_sync(FULLMASK, key) & hm;
             const uint32_t leader = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
             if (!VALS) {
-                if (pos >= 0 && lane == leader) atomicAdd(&S.plo[pos], (unsigned int)__popc(grp));
+                if (pos[q] >= 0 && lane == leader) atomicAdd(&S.plo[pos[q]], (unsigned int)__popc(grp));
             } else {
-                uint64_t acc = v;
+                uint64_t acc = v[q];
                 if (__any_sync(FULLMASK, __popc(grp) > 1)) {
                     acc = 0;
                     for (int x = 0; x < 32; ++x) {
-                        const uint64_t vx = __shfl_sync(FULLMASK, v, x);
+                        const uint64_t vx = __shfl_sync(FULLMASK, v[q], x);
                         if ((grp >> x) & 1u) acc += vx;
                     }
                 }
-                if (pos >= 0 && lane == leader) smem_add_u64(&S.plo[pos], &S.phi[pos], acc);
+                if (pos[q] >= 0 && lane == leader) smem_add_u64(&S.plo[pos[q]], &S.phi[pos[q]], acc);
             }
         }
-        // ---- misses: chain walk, combine in place, or allocate + link (a3..a6)
-        uint8_t* found = nullptr;
-        if (miss) {
-            found = chain_find_w(d, head, 0, tag, len, w0, w1, tail);
-            if (found) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found, len)), v);
+        // ---- misses: chain walk, combine in place (a3, a4)
+        uint8_t* found[SUB];
+#pragma unroll
+        for (int q = 0; q < SUB; ++q) {
+            found[q] = nullptr;
+            if (valid[q] && pos[q] < 0) {
+                found[q] = chain_find_w(d, head[q], 0, tag_of(h[q]), len[q], w0[q], w1[q], b.keys + s[q] + 16);
+                if (found[q]) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found[q], len[q])), v[q]);
+            }
         }
-        uint32_t res = R_OK;
-        const uint32_t esize = centry_size(len);
-        bool need = miss && !found;
-        if (need && (len > 65535u - 64u || esize > PB)) { need = false; res = R_TOOLARGE; }
-        if (inj && need && inject_fail(d, h, i)) { need = false; res = R_POST; }
-        // Certified declines (R15). Allocation failure is monotone for the generation (`full`).
-        // A warp announces itself in its CTA's announcement word before it may reserve entries
-        // (one RMW; if the word already carries the FULL bit it backs off) and withdraws with a
-        // release-add after linking them. The FULL bit is OR-ed into every word when the pool runs
-        // out, so per word the RMW order decides: an announcement either precedes the bit (and is
-        // counted) or sees it. A declining warp waits (once per launch) until every word shows
-        // FULL with no announcement: every entry reserved before the pool ran out is then linked
-        // and none can follow, so one re-walk of the chain decides the record for good — absorbed
-        // now, or not resident in this generation (the residency guarantee of P:L77/P:L79).
-        const bool any_need = __any_sync(FULLMASK, need);
-        uint64_t off = ~0ull;
-        if (any_need && !w_full) {  // cheap check first: no announcement once the pool is known full
-            unsigned long long f0 = 0;
-            if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
-            if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
-        }
-        if (any_need && !w_full) {
-            unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
-            unsigned long long a = 0;
-            if (lane == 0) a = atomicAdd(my_ann, 1ull);
-            a = __shfl_sync(FULLMASK, a, 0);
-            if (a & ANN_FULL) w_full = true;
-            else off = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
-            if (need && off != ~0ull) {
-                uint8_t* e = d.pool + off;
-                *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_COMBINE, head, tag, len);
-                if (len > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0;
-                if (len > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1;
-                if (len > 16) store_key(e + KEY_OFF + 16, tail, len - 16);
-                *reinterpret_cast<unsigned long long*>(entry_val(e, len)) = v;
-                const uint32_t me = off_ref(off);
-                while (true) {  // lock-free head insertion
-                    const uint32_t old = cas_release(d.dir + bkt, head, me);
-                    if (old == head) break;
-                    uint8_t* w = chain_find_w(d, old, head, tag, len, w0, w1, tail);
-                    if (w) {  // linked meanwhile by another warp: combine there, retire ours
-                        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
-                        *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
-                        c_dead += esize;
-                        break;
+        // ---- new keys: allocate + link (a5, a6), decline (a7)
+#pragma unroll
+        for (int q = 0; q < SUB; ++q) {
+            const uint64_t i = (g0 + q) * 32 + lane;
+            const bool miss = valid[q] && pos[q] < 0;
+            const uint8_t* tail = b.keys + s[q] + 16;
+            const uint32_t bkt = bucket_of(h[q], d.n_buckets);
+            const uint32_t tag = tag_of(h[q]);
+            const uint32_t ln = len[q];
+            const uint64_t vq = v[q];
+            uint32_t hd = head[q];
+            uint32_t res = R_OK;
+            const uint32_t esize = centry_size(ln);
+            bool need = miss && !found[q];
+            if (need && (ln > 65535u - 64u || esize > PB)) { need = false; res = R_TOOLARGE; }
+            if (inj && need && inject_fail(d, h[q], i)) { need = false; res = R_POST; }
+            // Certified declines (R15). Allocation failure is monotone for the generation (`full`).
+            // A warp announces itself in its CTA's announcement word before it may reserve entries
+            // (one RMW; if the word already carries the FULL bit it backs off) and withdraws with a
+            // release-add after linking them. The FULL bit is OR-ed into every word when the pool runs
+            // out, so per word the RMW order decides: an announcement either precedes the bit (and is
+            // counted) or sees it. A declining warp waits (once per launch) until every word shows
+            // FULL with no announcement: every entry reserved before the pool ran out is then linked
+            // and none can follow, so one re-walk of the chain decides the record for good — absorbed
+            // now, or not resident in this generation (the residency guarantee of P:L77/P:L79).
+            const bool any_need = __any_sync(FULLMASK, need);
+            uint64_t off = ~0ull;
+            if (any_need && !w_full) {  // cheap check first: no announcement once the pool is known full
+                unsigned long long f0 = 0;
+                if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
+                if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
+            }
+            if (any_need && !w_full) {
+                unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
+                unsigned long long a = 0;
+                if (lane == 0) a = atomicAdd(my_ann, 1ull);
+                a = __shfl_sync(FULLMASK, a, 0);
+                if (a & ANN_FULL) w_full = true;
+                else off = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
+                if (need && off != ~0ull) {
+                    uint8_t* e = d.pool + off;
+                    *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_COMBINE, hd, tag, ln);
+                    if (ln > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0[q];
+                    if (ln > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1[q];
+                    if (ln > 16) store_key(e + KEY_OFF + 16, tail, ln - 16);
+                    *reinterpret_cast<unsigned long long*>(entry_val(e, ln)) = vq;
+                    const uint32_t me = off_ref(off);
+                    while (true) {  // lock-free head insertion
+                        const uint32_t old = cas_release(d.dir + bkt, hd, me);
+                        if (old == hd) break;
+                        uint8_t* w = chain_find_w(d, old, hd, tag, ln, w0[q], w1[q], tail);
+                        if (w) {  // linked meanwhile by another warp: combine there, retire ours
+                            red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, ln)), vq);
+                            *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
+                            c_dead += esize;
+                            break;
+                        }
+                        hd = old;
+                        *reinterpret_cast<uint32_t*>(e + 4) = hd;
                     }
-                    head = old;
-                    *reinterpret_cast<uint32_t*>(e + 4) = head;
                 }
-            }
-            __syncwarp();
-            if (lane == 0) add_release64(my_ann, ~0ull);  // withdraw (-1), after every link above
-        }
-        const bool declined = need && off == ~0ull;
-        if (__any_sync(FULLMASK, declined)) {
-            w_full = true;
-            if (!w_quiet) {
-                if (lane == 0)
-                    for (uint32_t c = 0; c < d.n_slots; ++c)
-                        while (ld_acquire_u64(d.ann + (uint64_t)c * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
                 __syncwarp();
-                if (declined) {
-                    uint8_t* w = chain_find_w(d, ld_relaxed_u32(d.dir + bkt), 0, tag, len, w0, w1, tail);
-                    if (w) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
-                    else res = R_POST;
-                }
-                w_quiet = true;
-            } else if (declined) {
-                res = R_POST;  // walked after quiescence: the miss is final
+                if (lane == 0) add_release64(my_ann, ~0ull);  // withdraw (-1), after every link above
             }
-        }
-        nw0 = 0; nw1 = 0;
-        if (nlen) load_key16(b.keys + ns, nlen, nw0, nw1);
-        // ---- outcome -> bitmap word (a7); key bytes of the declined records (re-issue sizing)
-        const unsigned bits = __ballot_sync(FULLMASK, valid && res != R_OK);
-        const unsigned tl = __ballot_sync(FULLMASK, valid && res == R_TOOLARGE);
-        const unsigned pkb = bits ? __reduce_add_sync(FULLMASK, (valid && res != R_OK) ? len : 0u) : 0u;
-        if (lane == 0 && g * 32 < b.n) {
-            b.bitmap[g] = bits;
-            c_post += __popc(bits);
-            c_tl += __popc(tl);
-            c_pkb += pkb;
+            const bool declined = need && off == ~0ull;
+            if (__any_sync(FULLMASK, declined)) {
+                w_full = true;
+                if (!w_quiet) {
+                    if (lane == 0)
+                        for (uint32_t c = 0; c < d.n_slots; ++c)
+                            while (ld_acquire_u64(d.ann + (uint64_t)c * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
+                    __syncwarp();
+                    if (declined) {
+                        uint8_t* w = chain_find_w(d, ld_relaxed_u32(d.dir + bkt), 0, tag, ln, w0[q], w1[q], tail);
+                        if (w) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, ln)), vq);
+                        else res = R_POST;
+                    }
+                    w_quiet = true;
+                } else if (declined) {
+                    res = R_POST;  // walked after quiescence: the miss is final
+                }
+            }
+            // ---- outcome -> bitmap word (a7); key bytes of the declined records (re-issue sizing)
+            const unsigned bits = __ballot_sync(FULLMASK, valid[q] && res != R_OK);
+            if (bits) {
+                const unsigned tl = __ballot_sync(FULLMASK, valid[q] && res == R_TOOLARGE);
+                const unsigned pkb = __reduce_add_sync(FULLMASK, (valid[q] && res != R_OK) ? ln : 0u);
+                if (lane == 0) { c_post += __popc(bits); c_tl += __popc(tl); c_pkb += pkb; }
+            }
+            if (lane == 0 && (g0 + q) < ngroups) b.bitmap[g0 + q] = bits;
         }
     }
     if (lane == 0 && (c_post | c_tl)) {
@@ -1396,14 +1421,15 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             nh = n_out;
         }
         const size_t sm = sizeof(stream::Smem);
+        constexpr int T = stream::THREADS, SUB = stream::SUB;
         static bool attr = false;
         if (!attr) {
-            cudaFuncSetAttribute(insert_stream_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-            cudaFuncSetAttribute(insert_stream_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            cudaFuncSetAttribute(insert_stream_kernel<false, T, SUB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            cudaFuncSetAttribute(insert_stream_kernel<true, T, SUB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
             attr = true;
         }
-        if (b.vals) insert_stream_kernel<true><<<grid, stream::THREADS, sm, s>>>(d, b, hl, nh);
-        else insert_stream_kernel<false><<<grid, stream::THREADS, sm, s>>>(d, b, hl, nh);
+        if (b.vals) insert_stream_kernel<true, T, SUB><<<grid, T, sm, s>>>(d, b, hl, nh);
+        else insert_stream_kernel<false, T, SUB><<<grid, T, sm, s>>>(d, b, hl, nh);
     } else {
         size_t sm = sizeof(Smem<1>);
         static bool attr1 = false;

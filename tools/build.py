@@ -65,9 +65,9 @@ def build_oracle(force=False):
     return tgt
 
 
-def build_sepo(force=False):
+def build_sepo(force=False, target=None, extra=()):
     os.makedirs(os.path.join(PKG, "lib"), exist_ok=True)
-    tgt = os.path.join(PKG, "lib", "libsepo.so")
+    tgt = target or os.path.join(PKG, "lib", "libsepo.so")
     csrc = os.path.join(PKG, "csrc")
     deps = _files(csrc, {".h", ".cuh", ".cu", ".cpp"}) + _files(os.path.join(ROOT, "include"), {".h"})
     if not force and not _stale(tgt, deps):
@@ -79,7 +79,7 @@ def build_sepo(force=False):
            "-Iinclude", "-I" + os.path.relpath(csrc, ROOT)]
     if inc:
         cmd += ["-I" + inc, "-DSEPO_WITH_NCCL=1", "-L" + lib, "-l:libnccl.so.2", "-Xlinker", "-rpath=" + lib]
-    cmd += srcs + ["-o", tgt]
+    cmd += list(extra) + srcs + ["-o", tgt]
     _run(cmd)
     return tgt
 
