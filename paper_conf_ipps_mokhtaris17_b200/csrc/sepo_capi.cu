@@ -55,7 +55,11 @@ struct DevBuf {
         if (p) cudaFree(p);
         p = nullptr;
         cap = 0;
-        size_t want = std::max<size_t>(bytes, 1 << 20);
+        // 25 % headroom, 2 MiB granules: re-issue sizes fluctuate from run to run (the order in
+        // which warps race for the last pages), and a cudaFree + cudaMalloc of a GiB-sized buffer
+        // inside a job costs tens of milliseconds
+        size_t want = std::max<size_t>(bytes + bytes / 4, 1 << 20);
+        want = (want + (2u << 20) - 1) & ~(size_t)((2u << 20) - 1);
         if (cudaMalloc(&p, want) != cudaSuccess) {
             cudaGetLastError();
             return -1;

@@ -606,6 +606,9 @@ __global__ void __launch_bounds__(1024) hot_resolve_kernel(Dev d, Batch b, hot::
 }
 
 namespace stream {
+#ifndef SEPO_DIR_ALL
+#define SEPO_DIR_ALL 1  // issue every record's directory load before the hot-set probe
+#endif
 #ifndef SEPO_STREAM_THREADS
 #define SEPO_STREAM_THREADS 1024  // measured best (profiles/r01_summary.md): 32 warps x 1 group
 #define SEPO_STREAM_SUB 1
@@ -628,6 +631,60 @@ __device__ __forceinline__ void smem_add_u64(unsigned int* lo, unsigned int* hi,
     const unsigned int carry = (old + vl < old) ? 1u : 0u;
     const unsigned int vh = (unsigned int)(v >> 32) + carry;
     if (vh) atomicAdd(hi, vh);
+}
+
+// Warp-cooperative load of 32 consecutive records (group g): each lane loads one key offset
+// (the next lane's offset is its end), then the warp's contiguous key bytes are read as 16-B
+// chunks — lane L loads chunk L with one coalesced 128-bit load — and every lane assembles its
+// first 16 key bytes from the two chunks that hold them (__shfl_sync + funnel shifts). Falls back
+// to per-lane loads when the group's key bytes exceed 512 B (long keys) or the batch is indexed.
+__device__ __forceinline__ void warp_load_group(const Batch& b, uint64_t g, uint32_t lane, bool valid, uint64_t& s,
+                                                uint32_t& len, uint64_t& w0, uint64_t& w1) {
+    const uint64_t i = g * 32 + lane;
+    if (b.idx) {  // re-issued records are not contiguous (warp-uniform branch)
+        s = 0; len = 0; w0 = 0; w1 = 0;
+        if (valid) { rec_key(b, i, s, len); load_key16(b.keys + s, len, w0, w1); }
+        return;
+    }
+    uint64_t e;
+    if (b.ko) {
+        s = valid ? __ldg(reinterpret_cast<const unsigned long long*>(b.ko) + i) : 0ull;
+        e = __shfl_down_sync(FULLMASK, s, 1);
+        const bool last = valid && (lane == 31 || i + 1 >= b.n);
+        if (last) e = __ldg(reinterpret_cast<const unsigned long long*>(b.ko) + i + 1);
+    } else {
+        s = i * (uint64_t)b.kw;
+        e = s + b.kw;
+    }
+    len = valid ? (uint32_t)(e - s) : 0u;
+    const uint64_t base = __shfl_sync(FULLMASK, s, 0);
+    const unsigned vm = __ballot_sync(FULLMASK, valid);
+    const uint32_t lastl = 31 - __clz(vm | 1u);
+    const uint64_t end = __shfl_sync(FULLMASK, e, lastl);
+    const uint64_t base_al = base & ~15ull;
+    const uintptr_t kaddr = reinterpret_cast<uintptr_t>(b.keys);
+    if (end - base_al > 512 || (kaddr & 15)) {  // warp-uniform fallback
+        w0 = 0; w1 = 0;
+        if (valid) load_key16(b.keys + s, len, w0, w1);
+        return;
+    }
+    uint4 ch = make_uint4(0, 0, 0, 0);
+    if (base_al + 16ull * lane < end) ch = __ldg(reinterpret_cast<const uint4*>(b.keys + base_al) + lane);
+    const uint32_t off = (uint32_t)(s - base_al);
+    const uint32_t c0 = valid ? (off >> 4) : 0u, c1 = min(c0 + 1u, 31u);
+    const uint32_t x0 = __shfl_sync(FULLMASK, ch.x, c0), x1 = __shfl_sync(FULLMASK, ch.y, c0);
+    const uint32_t x2 = __shfl_sync(FULLMASK, ch.z, c0), x3 = __shfl_sync(FULLMASK, ch.w, c0);
+    const uint32_t y0 = __shfl_sync(FULLMASK, ch.x, c1), y1 = __shfl_sync(FULLMASK, ch.y, c1);
+    const uint32_t y2 = __shfl_sync(FULLMASK, ch.z, c1), y3 = __shfl_sync(FULLMASK, ch.w, c1);
+    const uint64_t X0 = ((uint64_t)x1 << 32) | x0, X1 = ((uint64_t)x3 << 32) | x2;
+    const uint64_t Y0 = ((uint64_t)y1 << 32) | y0, Y1 = ((uint64_t)y3 << 32) | y2;
+    const uint32_t r = off & 15u, sh = 8u * (r & 7u);
+    const uint64_t q0 = r < 8 ? X0 : X1, q1 = r < 8 ? X1 : Y0, q2 = r < 8 ? Y0 : Y1;
+    w0 = sh ? (q0 >> sh) | (q1 << (64 - sh)) : q0;
+    w1 = sh ? (q1 >> sh) | (q2 << (64 - sh)) : q1;
+    if (!valid || len == 0) { w0 = 0; w1 = 0; }
+    else if (len < 8) { w0 &= (1ull << (8 * len)) - 1ull; w1 = 0; }
+    else if (len < 16) w1 &= (1ull << (8 * (len - 8))) - 1ull;
 }
 
 template <bool VALS, int THREADS, int SUB>
@@ -683,12 +740,9 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         for (int q = 0; q < SUB; ++q) {
             const uint64_t i = (g0 + q) * 32 + lane;
             valid[q] = i < b.n;
-            s[q] = 0; len[q] = 0; w0[q] = 0; w1[q] = 0; v[q] = 1;
-            if (valid[q]) {
-                rec_key(b, i, s[q], len[q]);
-                load_key16(b.keys + s[q], len[q], w0[q], w1[q]);
-                if (VALS) v[q] = rec_value(b, i);
-            }
+            v[q] = 1;
+            warp_load_group(b, g0 + q, lane, valid[q], s[q], len[q], w0[q], w1[q]);
+            if (VALS && valid[q]) v[q] = rec_value(b, i);
         }
 #pragma unroll
         for (int q = 0; q < SUB; ++q) {
@@ -699,6 +753,13 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
                 x = hash_word(x, load_in_word(b.keys + s[q] + o, len[q] - o < 8 ? len[q] - o : 8));
             h[q] = fmix64(x);
         }
+        // ---- directory load for every record, issued before the hot-set probe so that its latency
+        // (and the first chain entry's, below) overlaps the shared-memory work of the hits
+        uint32_t head[SUB];
+#if SEPO_DIR_ALL
+#pragma unroll
+        for (int q = 0; q < SUB; ++q) head[q] = valid[q] ? ld_relaxed_u32(d.dir + bucket_of(h[q], d.n_buckets)) : 0u;
+#endif
         // ---- hot set: constant-time probe of two 4-way buckets, then a full-key check
         int pos[SUB];
 #pragma unroll
@@ -721,12 +782,23 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
                     pos[q] = p;
             }
         }
-        // ---- directory loads of the misses: in flight while the hits are folded
-        uint32_t head[SUB];
+#if !SEPO_DIR_ALL
+#pragma unroll
+        for (int q = 0; q < SUB; ++q)
+            head[q] = (valid[q] && pos[q] < 0) ? ld_relaxed_u32(d.dir + bucket_of(h[q], d.n_buckets)) : 0u;
+#endif
+        // ---- misses: the chain head entry (header + first 16 key bytes) is fetched now
+        uint4 e_hd[SUB];
+        ulonglong2 e_kw[SUB];
 #pragma unroll
         for (int q = 0; q < SUB; ++q) {
-            head[q] = 0;
-            if (valid[q] && pos[q] < 0) head[q] = ld_relaxed_u32(d.dir + bucket_of(h[q], d.n_buckets));
+            e_hd[q] = make_uint4(0, 0, 0, 0);
+            e_kw[q] = make_ulonglong2(0, 0);
+            if (valid[q] && pos[q] < 0 && head[q]) {
+                const uint8_t* e = ref_ptr(d, head[q]);
+                e_hd[q] = ldcg128(e);
+                e_kw[q] = ldcg128u(e + KEY_OFF);
+            }
         }
         // ---- fold the hits of the warp per hot slot (a2): one shared atomic per distinct key
 #pragma unroll
@@ -750,14 +822,20 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
                 if (pos[q] >= 0 && lane == leader) smem_add_u64(&S.plo[pos[q]], &S.phi[pos[q]], acc);
             }
         }
-        // ---- misses: chain walk, combine in place (a3, a4)
+        // ---- misses: compare the prefetched head entry, then walk the rest of the chain (a3, a4)
         uint8_t* found[SUB];
 #pragma unroll
         for (int q = 0; q < SUB; ++q) {
             found[q] = nullptr;
-            if (valid[q] && pos[q] < 0) {
-                found[q] = chain_find_w(d, head[q], 0, tag_of(h[q]), len[q], w0[q], w1[q], b.keys + s[q] + 16);
-                if (found[q]) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found[q], len[q])), v[q]);
+            if (valid[q] && pos[q] < 0 && head[q]) {
+                const uint32_t tag = tag_of(h[q]), ln = len[q];
+                const uint8_t* tail = b.keys + s[q] + 16;
+                if (e_hd[q].z == tag && e_hd[q].w == ln && (ln == 0 || e_kw[q].x == w0[q]) && (ln <= 8 || e_kw[q].y == w1[q]) &&
+                    (ln <= 16 || entry_key_eq(ref_ptr(d, head[q]) + KEY_OFF + 16, tail, ln - 16)))
+                    found[q] = ref_ptr(d, head[q]);
+                else
+                    found[q] = chain_find_w(d, e_hd[q].y, 0, tag, ln, w0[q], w1[q], tail);
+                if (found[q]) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found[q], ln)), v[q]);
             }
         }
         // ---- new keys: allocate + link (a5, a6), decline (a7)
