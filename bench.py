@@ -321,8 +321,15 @@ def run_ours(args):
     pk = peaks()
     alg = info["kb"] + (8 * info["recs"] if k is not None and o is not None else 0) + info["vb"]
     achieved = alg / (info["insert_ms"] / 1e3) / 1e9
+    traffic, traffic_note = args.traffic, None
+    tj = os.path.join(ROOT, "profiles", "r01_traffic.json")
+    if traffic is None and os.path.exists(tj) and args.config == "C2" and args.scale == 1.0:
+        tr = json.load(open(tj))
+        traffic = tr["dram_read_bytes"] + tr["dram_write_bytes"]
+        traffic_note = (f"dram read+write of one launch ({tr['launch']}); that launch's algorithmic bytes: "
+                        f"{tr['alg_bytes']}")
     roof = {"bound": "hbm", "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
-            "frac": achieved / pk["hbm_gbs"], "traffic": args.traffic, "kernel": "sepo::insert_stream_kernel (COMBINE) / sepo::insert_kernel<1> (GROUP)",
+            "frac": achieved / pk["hbm_gbs"], "traffic": traffic, "traffic_note": traffic_note, "kernel": "sepo::insert_stream_kernel (COMBINE) / sepo::insert_kernel<1> (GROUP)",
             "insert_share_of_step": info["insert_ms"] / ms,
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if not pk.get("_fallback") else "fallback 6.65 TB/s"}
 
