@@ -376,11 +376,11 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
     sync_dev(t);
     if ((rc = zero_ctrl_counters(t))) return rc;
     CK(t, cudaEventRecord(t->ev0, t->stream));
-    if (t->opts.mode == SEPO_COMBINE_SUM_U64 && t->hot.grow(sepo_hot_scratch_bytes())) return fail(SEPO_E_NOMEM, "hot-set scratch");
-    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->opts.mode == SEPO_COMBINE_SUM_U64 ? t->hot.p : nullptr);
+    if (t->hot.grow(sepo_hot_scratch_bytes())) return fail(SEPO_E_NOMEM, "hot-set scratch");
+    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p);
     if (rc) return cuda_check(t, (cudaError_t)rc, "insert kernel launch");
     CK(t, cudaEventRecord(t->ev1, t->stream));
-    t->st.kernel_launches += (t->opts.mode == SEPO_COMBINE_SUM_U64 && n >= (8ull << 18)) ? 7 : 1;
+    t->st.kernel_launches += (n >= (8ull << 18)) ? 7 : 1;
     if (b.ko && !b.idx) {
         CK(t, cudaMemcpyAsync(&t->h_ko[0], b.ko, 8, cudaMemcpyDeviceToHost, t->stream));
         CK(t, cudaMemcpyAsync(&t->h_ko[1], b.ko + n, 8, cudaMemcpyDeviceToHost, t->stream));
@@ -727,6 +727,7 @@ int export_group(sepo_table* t) {
                     memcpy(&fill, base + off + 4, 4);
                     memcpy(&owner, base + off + 8, 8);
                     memcpy(&cap, base + off + 24, 4);
+                    cap &= ~CHUNK_PRIVATE;
                     tc[w].push_back({base + off + CHUNK_HDR, std::min(fill, cap), owner});
                     slots[w] += cap;
                 }
@@ -876,7 +877,9 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
         int64_t c = insert_impl(t, cur);
         if (c < 0) return c;
         uint64_t kb = t->h_ctrl->kept_key_bytes, vb = 0;
-        const bool combine_exact = t->opts.mode == SEPO_COMBINE_SUM_U64 && !(t->opts.fail_alloc_ppm && t->opts.fail_mode == 1);
+        // both streaming kernels certify their declines (R15) and mark pending GROUP keys'
+        // pages themselves, so the insert's count is exact — except under record-mode injection
+        const bool combine_exact = !(t->opts.fail_alloc_ppm && t->opts.fail_mode == 1);
         if (c > 0 && !combine_exact) c = reprobe_impl(t, cur, &kb, &vb);
         if (c < 0) return c;
         if (c == 0) break;

@@ -34,6 +34,7 @@ enum : uint32_t { K_FREE = 0, K_COMBINE = 1, K_FILL = 2, K_DEAD = 3, K_GKEY = 4,
 constexpr uint32_t KIND_MASK = 7u;
 constexpr uint32_t KEY_OFF = 16;     // key bytes start here in combine and group key entries
 constexpr uint32_t CHUNK_HDR = 32;   // value chunk header
+constexpr uint32_t CHUNK_PRIVATE = 0x80000000u;  // cap flag: slots handed out by one CTA (hot key)
 constexpr uint32_t NOPAGE = 0xfffffffeu, FULLPAGE = 0xffffffffu;
 constexpr uint32_t PAGE_ENTRY = 1, PAGE_VALUE = 2;
 

@@ -116,15 +116,16 @@ __device__ __forceinline__ void init_chunk(uint8_t* c, uint32_t cap, uint32_t vw
     *reinterpret_cast<uint32_t*>(c + 24) = cap;
     *reinterpret_cast<uint32_t*>(c + 28) = vwslot;
 }
-// push chunk `cref` (already holding its values' slots) onto the list head of key entry e
+// push chunk `cref` (header already written) onto the list head of key entry e: one release-
+// exchange, then the chunk's `next` takes the previous head. Device code never follows `next`
+// (only the host export does, after the kernel), so a CAS retry loop — which serialises badly when
+// many CTAs push onto a hot key at once — is not needed.
 __device__ __forceinline__ void push_chunk(uint8_t* e, uint8_t* c, uint64_t cref, uint64_t observed) {
+    (void)observed;
     unsigned long long* head = list_head(e);
-    while (true) {
-        *reinterpret_cast<unsigned long long*>(c + 16) = observed;
-        unsigned long long old = cas_release64(head, observed, cref);
-        if (old == observed) return;
-        observed = old;
-    }
+    unsigned long long old;
+    asm volatile("atom.release.gpu.global.exch.b64 %0, [%1], %2;" : "=l"(old) : "l"(head), "l"(cref) : "memory");
+    *reinterpret_cast<unsigned long long*>(c + 16) = old;
 }
 // Reserve k slots in the resident head chunk of key entry e. Returns granted count (0..k),
 // the chunk ref in *cref and the first slot in *base; *head_out = observed head, *prev_cap.
@@ -137,6 +138,7 @@ __device__ __forceinline__ uint32_t reserve_head(const Dev& d, uint8_t* e, uint3
     if (!vref_resident(d, h)) return 0;
     uint8_t* c = vref_ptr(d, h);
     uint32_t cap = ldcg32(c + 24);
+    if (cap & CHUNK_PRIVATE) return 0;  // a CTA's private chunk: slots are handed out in its smem
     *prev_cap = cap;
     if (ldcg32(c + 4) >= cap) return 0;
     uint32_t old = atomicAdd(reinterpret_cast<unsigned int*>(c + 4), k);
@@ -520,25 +522,25 @@ __global__ void __launch_bounds__(256) hot_hist_kernel(const hot::SampleSlot* ta
         if (tab[i].h != 0ull && c >= min_count) atomicAdd(&hist[min(c, (unsigned)HOT_HIST - 1)], 1u);
     }
 }
-__global__ void __launch_bounds__(32) hot_threshold_kernel(unsigned int* hist, uint32_t min_count) {
+__global__ void __launch_bounds__(32) hot_threshold_kernel(unsigned int* hist, uint32_t min_count, uint32_t kmax) {
     if (threadIdx.x != 0) return;
     unsigned acc = 0, thr = 0xffffffffu;
     for (int c = HOT_HIST - 1; c >= (int)min_count; --c) {
-        if (acc + hist[c] > (unsigned)hot::K) break;
+        if (acc + hist[c] > kmax) break;
         acc += hist[c];
         thr = c;
     }
     hist[HOT_HIST] = thr;  // threshold
 }
 __global__ void __launch_bounds__(256) hot_emit_kernel(Dev d, Batch b, const hot::SampleSlot* tab, const unsigned int* hist,
-                                                       hot::Entry* out, unsigned int* n_out) {
+                                                       hot::Entry* out, unsigned int* n_out, uint32_t kmax) {
     const unsigned thr = hist[HOT_HIST];
     if (thr == 0xffffffffu) return;
     for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < hot::SAMPLE_SLOTS; i += gridDim.x * blockDim.x) {
         const unsigned c = tab[i].count;
         if (tab[i].h != 0ull && c >= thr) {
             const unsigned j = atomicAdd(n_out, 1u);
-            if (j < (unsigned)hot::K) {
+            if (j < kmax) {
                 uint64_t s, w0, w1, h; uint32_t len;
                 rec_hash16(d, b, tab[i].rec, s, len, w0, w1, h);
                 hot::Entry e;
@@ -548,7 +550,7 @@ __global__ void __launch_bounds__(256) hot_emit_kernel(Dev d, Batch b, const hot
         }
     }
 }
-__global__ void hot_clamp_kernel(unsigned int* n_out) { if (threadIdx.x == 0 && *n_out > (unsigned)hot::K) *n_out = hot::K; }
+__global__ void hot_clamp_kernel(unsigned int* n_out, uint32_t kmax) { if (threadIdx.x == 0 && *n_out > kmax) *n_out = kmax; }
 
 // (i-c) one CTA on allocator slot 0: look up / insert (value 0) every hot key
 __global__ void __launch_bounds__(1024) hot_resolve_kernel(Dev d, Batch b, hot::Entry* list, const unsigned int* n_list) {
@@ -942,6 +944,352 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         if (S.len[p] == hot::EMPTY_LEN) continue;
         const uint64_t sum = ((uint64_t)S.phi[p] << 32) | S.plo[p];
         if (sum) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(ref_ptr(d, S.ref[p]), S.len[p])), sum);
+    }
+    if (tid == 0) {
+        d.cursors[2 * blockIdx.x] = S.cur[0];
+        d.cursors[2 * blockIdx.x + 1] = S.cur[1];
+        if (S.post) atomicAdd(&d.ctrl->postponed, S.post);
+        if (S.toolarge) atomicAdd(&d.ctrl->toolarge, S.toolarge);
+        if (S.dead) atomicAdd(&d.ctrl->dead_bytes, S.dead);
+    }
+}
+
+// ================================================================ GROUP insert (a1..a7): hot set + streaming warps
+// Multi-valued method. Same structure as the COMBINE kernel: a sampled hot set lives
+// in shared memory; each hot key also owns a CTA-PRIVATE value chunk whose slots are handed out by
+// a shared-memory word {chunk ref, fill} (a whole warp's values of that key reserved with one
+// shared atomic); when it fills, the warp that crosses the end installs the next private chunk.
+// Other keys append through the key's shared head chunk (one global atomic per record) or a new
+// demand-sized chunk pushed onto the list head (release-CAS). A record whose value cannot get a
+// slot while its key is resident is postponed and marks the key's page retained (pending key,
+// P:L165); new-key declines are certified as in the COMBINE kernel (R15), so a GROUP pass needs no
+// separate re-probe.
+namespace gst {
+constexpr int THREADS = 1024;
+constexpr int NB = 512, NH = 4 * NB;  // hot slots (2-choice 4-way buckets)
+constexpr int K = 1024;               // hot keys at most
+constexpr uint32_t PC_CAP = 256;      // slots of a private chunk
+struct Smem {
+    uint4 tags[NB];
+    uint64_t h[NH], w0[NH], w1[NH];
+    uint32_t len[NH], ref[NH];
+    unsigned long long pw[NH];  // private chunk word: chunk ref << 32 | fill (ref 0: none)
+    unsigned long long cur[2];
+    unsigned long long post, toolarge, dead;
+};
+__device__ __forceinline__ uint32_t b1(uint64_t h) { return (uint32_t)(h >> 3) & (NB - 1); }
+__device__ __forceinline__ uint32_t b2(uint64_t h) { return (uint32_t)(h >> 13) & (NB - 1); }
+}  // namespace gst
+
+// write record i's value (vw bytes) into slot `slot` of chunk c
+__device__ __forceinline__ void put_value(const Batch& b, uint64_t i, uint8_t* c, uint32_t slot) {
+    const uint64_t src = rec_index(b, i) * (uint64_t)b.vw;
+    uint8_t* dst = c + CHUNK_HDR + (uint64_t)slot * b.vw;
+    if (b.vw == 4) *reinterpret_cast<uint32_t*>(dst) = __ldg(reinterpret_cast<const unsigned int*>(b.vals + src));
+    else if (b.vw == 8) *reinterpret_cast<unsigned long long*>(dst) = __ldg(reinterpret_cast<const unsigned long long*>(b.vals + src));
+    else for (uint32_t x = 0; x < b.vw; ++x) dst[x] = __ldg(b.vals + src + x);
+}
+
+// GROUP hot keys: look up / insert the key entry (empty list) on allocator slot 0
+__global__ void __launch_bounds__(1024) hot_resolve_group_kernel(Dev d, Batch b, hot::Entry* list, const unsigned int* n_list) {
+    __shared__ unsigned long long s_cur;
+    if (threadIdx.x == 0) s_cur = d.cursors[0];
+    __syncthreads();
+    const unsigned n = *n_list;
+    for (unsigned j0 = 0; j0 < n; j0 += blockDim.x) {
+        const unsigned j = j0 + threadIdx.x;
+        const bool act = j < n;
+        hot::Entry e = act ? list[j] : hot::Entry{};
+        const uint8_t* tail = b.keys + e.src + 16;
+        const uint32_t bkt = act ? bucket_of(e.h, d.n_buckets) : 0;
+        const uint32_t tag = tag_of(e.h);
+        uint32_t head = 0;
+        uint8_t* found = nullptr;
+        if (act) {
+            head = ld_relaxed_u32(d.dir + bkt);
+            found = chain_find_w(d, head, 0, tag, e.len, e.w0, e.w1, tail);
+        }
+        const uint32_t esize = gkey_size(e.len);
+        bool need = act && !found && e.len <= 65535u - 64u && esize <= d.page_bytes && !inject_fail(d, e.h, j);
+        uint32_t ref = found ? off_ref((uint64_t)(found - d.pool)) : 0u;
+        const uint64_t off = warp_alloc(d, &s_cur, need, esize, (uint8_t)PAGE_ENTRY);
+        if (need && off != ~0ull) {
+            uint8_t* ne = d.pool + off;
+            *reinterpret_cast<uint4*>(ne) = make_uint4(esize | K_GKEY, head, tag, e.len);
+            if (e.len > 0) *reinterpret_cast<unsigned long long*>(ne + KEY_OFF) = e.w0;
+            if (e.len > 8) *reinterpret_cast<unsigned long long*>(ne + KEY_OFF + 8) = e.w1;
+            if (e.len > 16) store_key(ne + KEY_OFF + 16, tail, e.len - 16);
+            *reinterpret_cast<unsigned long long*>(entry_val(ne, e.len)) = 0ull;
+            *reinterpret_cast<uint32_t*>(entry_val(ne, e.len) + 8) = d.gen;
+            *reinterpret_cast<uint32_t*>(entry_val(ne, e.len) + 12) = 0u;
+            ref = off_ref(off);
+            while (true) {
+                const uint32_t old = cas_release(d.dir + bkt, head, ref);
+                if (old == head) break;
+                uint8_t* w = chain_find_w(d, old, head, tag, e.len, e.w0, e.w1, tail);
+                if (w) {
+                    *reinterpret_cast<uint32_t*>(ne) = esize | K_DEAD;
+                    ref = off_ref((uint64_t)(w - d.pool));
+                    break;
+                }
+                head = old;
+                *reinterpret_cast<uint32_t*>(ne + 4) = head;
+            }
+        }
+        if (act) list[j].ref = ref;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) d.cursors[0] = s_cur;
+}
+
+__global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
+                                                                              const unsigned int* n_hot) {
+    using gst::THREADS; using gst::NB; using gst::NH; using gst::PC_CAP; using gst::b1; using gst::b2;
+    extern __shared__ __align__(16) uint8_t smem_raw[];
+    gst::Smem& S = *reinterpret_cast<gst::Smem*>(smem_raw);
+    const uint32_t tid = threadIdx.x, lane = lane_id();
+    const uint32_t PB = d.page_bytes;
+    const uint32_t vw = b.vw;
+    for (int p = tid; p < NH; p += THREADS) { S.len[p] = hot::EMPTY_LEN; S.pw[p] = PC_CAP; }
+    for (int p = tid; p < NB; p += THREADS) S.tags[p] = make_uint4(0, 0, 0, 0);
+    if (tid == 0) {
+        S.cur[0] = d.cursors[2 * blockIdx.x];
+        S.cur[1] = d.cursors[2 * blockIdx.x + 1];
+        S.post = 0; S.toolarge = 0; S.dead = 0;
+    }
+    __syncthreads();
+    const unsigned nh = hl ? *n_hot : 0u;
+    for (unsigned j = tid; j < nh; j += THREADS) {
+        const hot::Entry e = hl[j];
+        if (e.ref == 0) continue;
+        const uint32_t f = hot::fp(e.h);
+        int pos = -1;
+        for (int c = 0; c < 2 && pos < 0; ++c) {
+            const uint32_t bk = c == 0 ? b1(e.h) : b2(e.h);
+            uint32_t* t = reinterpret_cast<uint32_t*>(&S.tags[bk]);
+            for (int w = 0; w < 4 && pos < 0; ++w)
+                if (atomicCAS(&t[w], 0u, f) == 0u) pos = (int)(bk * 4 + w);
+        }
+        if (pos < 0) continue;
+        S.h[pos] = e.h; S.w0[pos] = e.w0; S.w1[pos] = e.w1; S.ref[pos] = e.ref; S.len[pos] = e.len;
+    }
+    __syncthreads();
+    const bool have_hot = nh > 0;
+    const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
+    const uint32_t pc_bytes = chunk_bytes(PC_CAP, vw);
+
+    const uint64_t ngroups = (b.n + 31) / 32;
+    const uint64_t gw = (uint64_t)blockIdx.x * (THREADS / 32) + (tid >> 5);
+    const uint64_t nw = (uint64_t)gridDim.x * (THREADS / 32);
+    unsigned long long c_post = 0, c_tl = 0, c_dead = 0, c_pkb = 0;
+    bool w_full = false, w_quiet = false;
+    for (uint64_t g = gw; g < ngroups; g += nw) {
+        const uint64_t i = g * 32 + lane;
+        const bool valid = i < b.n;
+        uint64_t s, w0, w1;
+        uint32_t len;
+        warp_load_group(b, g, lane, valid, s, len, w0, w1);
+        uint64_t x = hash_init(len, d.seed);
+        if (len > 0) x = hash_word(x, w0);
+        if (len > 8) x = hash_word(x, w1);
+        for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(b.keys + s + o, len - o < 8 ? len - o : 8));
+        const uint64_t h = fmix64(x);
+        const uint8_t* tail = b.keys + s + 16;
+        const uint32_t tag = tag_of(h), bkt = bucket_of(h, d.n_buckets);
+        // ---- hot set probe
+        int pos = -1;
+        if (valid && have_hot) {
+            const uint32_t f = hot::fp(h);
+            const uint32_t k1 = b1(h), k2 = b2(h);
+            const uint4 t1 = S.tags[k1];
+            int p = -1;
+            if (t1.x == f) p = 4 * k1; else if (t1.y == f) p = 4 * k1 + 1;
+            else if (t1.z == f) p = 4 * k1 + 2; else if (t1.w == f) p = 4 * k1 + 3;
+            else {
+                const uint4 t2 = S.tags[k2];
+                if (t2.x == f) p = 4 * k2; else if (t2.y == f) p = 4 * k2 + 1;
+                else if (t2.z == f) p = 4 * k2 + 2; else if (t2.w == f) p = 4 * k2 + 3;
+            }
+            if (p >= 0 && S.h[p] == h && S.len[p] == len && S.w0[p] == w0 && S.w1[p] == w1 &&
+                (len <= 16 || entry_key_eq(ref_ptr(d, S.ref[p]) + KEY_OFF + 16, tail, len - 16)))
+                pos = p;
+        }
+        uint32_t head = 0;
+        if (valid && pos < 0) head = ld_relaxed_u32(d.dir + bkt);
+        // ---- hot keys: reserve the warp's values of a key in its private chunk (one shared atomic)
+        bool done = false;
+        uint8_t* e = nullptr;  // resident key entry for the global path
+        {
+            const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
+            if (hm) {
+                const unsigned key = pos >= 0 ? (unsigned)pos : (0x10000u | lane);
+                const unsigned grp = __match_any_sync(FULLMASK, key) & hm;
+                const uint32_t leader = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
+                const uint32_t k = __popc(grp), rank = __popc(grp & ((1u << lane) - 1u));
+                unsigned long long old = 0;
+                if (pos >= 0 && lane == leader) old = atomicAdd(&S.pw[pos], (unsigned long long)k);
+                old = __shfl_sync(FULLMASK, old, leader);
+                const uint32_t cref = (uint32_t)(old >> 32), f0 = (uint32_t)old;
+                // the warp that crosses the end of the private chunk installs the next one
+                const bool cross = pos >= 0 && f0 <= PC_CAP && f0 + k > PC_CAP;
+                const bool want = cross && lane == leader && !w_full;
+                unsigned long long ann = 0;
+                const bool anyw = __any_sync(FULLMASK, want);
+                uint64_t coff = ~0ull;
+                if (anyw) {  // announcement protocol (R15) around the allocation
+                    if (lane == 0) ann = atomicAdd(d.ann + (uint64_t)blockIdx.x * ANN_STRIDE, 1ull);
+                    ann = __shfl_sync(FULLMASK, ann, 0);
+                    if (ann & ANN_FULL) w_full = true;
+                    else coff = warp_alloc(d, &S.cur[1], want, pc_bytes, (uint8_t)PAGE_VALUE);
+                }
+                uint32_t nref = 0;
+                if (want) {
+                    if (cref) *reinterpret_cast<uint32_t*>(ref_ptr(d, cref) + 4) = PC_CAP;  // old chunk is full
+                    if (coff != ~0ull) {
+                        uint8_t* c = d.pool + coff;
+                        uint8_t* ke = ref_ptr(d, S.ref[pos]);
+                        init_chunk(c, PC_CAP, vw, 0, owner_of(d, ke), 0ull);
+                        *reinterpret_cast<uint32_t*>(c + 24) = PC_CAP | CHUNK_PRIVATE;
+                        push_chunk(ke, c, vref_of(d, coff), ld_relaxed_u64(list_head(ke)));
+                        nref = off_ref(coff);
+                        const uint32_t rest = f0 + k - PC_CAP;
+                        atomicExch(&S.pw[pos], ((unsigned long long)nref << 32) | rest);
+                    } else {
+                        atomicExch(&S.pw[pos], (unsigned long long)PC_CAP << 1);  // no chunk: hits go global
+                    }
+                }
+                if (anyw) {
+                    __syncwarp();
+                    if (lane == 0) add_release64(d.ann + (uint64_t)blockIdx.x * ANN_STRIDE, ~0ull);
+                }
+                nref = __shfl_sync(FULLMASK, nref, leader);
+                if (pos >= 0) {
+                    const uint32_t slot = f0 + rank;
+                    if (cref && slot < PC_CAP) { put_value(b, i, ref_ptr(d, cref), slot); done = true; }
+                    else if (cross && nref) { put_value(b, i, ref_ptr(d, nref), slot - PC_CAP); done = true; }
+                    else e = ref_ptr(d, S.ref[pos]);  // overflow: this record takes the global path
+                }
+            }
+        }
+        // ---- global path: chain walk (non-hot), reserve one slot in the key's shared head chunk
+        if (valid && !done && pos < 0) e = chain_find_w(d, head, 0, tag, len, w0, w1, tail);
+        bool need_key = valid && !done && e == nullptr;
+        bool need_chunk = valid && !done;
+        if (valid && !done && e) {
+            uint64_t cr = 0, lh = 0;
+            uint32_t base = 0, pc = 0;
+            if (reserve_head(d, e, 1, &cr, &base, &lh, &pc)) {
+                put_value(b, i, vref_ptr(d, cr), base);
+                done = true;
+                need_chunk = false;
+            }
+        }
+        uint32_t res = R_OK;
+        const uint32_t ksize = gkey_size(len);
+        const uint32_t ccap = chunk_cap(d, 1, 0, vw);
+        const uint32_t csize = chunk_bytes(ccap, vw);
+        if (need_key && (len > 65535u - 64u || ksize > PB)) { need_key = false; need_chunk = false; res = R_TOOLARGE; }
+        if (inj && need_key && inject_fail(d, h, i)) { need_key = false; need_chunk = false; res = R_POST; }
+        const bool any_need = __any_sync(FULLMASK, need_chunk);
+        uint64_t koff = ~0ull, coff = ~0ull;
+        if (any_need && !w_full) {
+            unsigned long long f0 = 0;
+            if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
+            if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
+        }
+        if (any_need && !w_full) {
+            unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
+            unsigned long long a = 0;
+            if (lane == 0) a = atomicAdd(my_ann, 1ull);
+            a = __shfl_sync(FULLMASK, a, 0);
+            if (a & ANN_FULL) w_full = true;
+            else {
+                koff = warp_alloc(d, &S.cur[0], need_key, ksize, (uint8_t)PAGE_ENTRY);
+                const bool wc = need_chunk && (!need_key || koff != ~0ull);
+                coff = warp_alloc(d, &S.cur[1], wc, csize, (uint8_t)PAGE_VALUE);
+            }
+            if (need_key && koff != ~0ull) {  // new key entry, linked even if its chunk failed (pending)
+                uint8_t* ne = d.pool + koff;
+                *reinterpret_cast<uint4*>(ne) = make_uint4(ksize | K_GKEY, head, tag, len);
+                if (len > 0) *reinterpret_cast<unsigned long long*>(ne + KEY_OFF) = w0;
+                if (len > 8) *reinterpret_cast<unsigned long long*>(ne + KEY_OFF + 8) = w1;
+                if (len > 16) store_key(ne + KEY_OFF + 16, tail, len - 16);
+                *reinterpret_cast<unsigned long long*>(entry_val(ne, len)) = 0ull;
+                *reinterpret_cast<uint32_t*>(entry_val(ne, len) + 8) = d.gen;
+                *reinterpret_cast<uint32_t*>(entry_val(ne, len) + 12) = 0u;
+                const uint32_t me = off_ref(koff);
+                e = ne;
+                uint32_t hd = head;
+                while (true) {
+                    const uint32_t old = cas_release(d.dir + bkt, hd, me);
+                    if (old == hd) break;
+                    uint8_t* w = chain_find_w(d, old, hd, tag, len, w0, w1, tail);
+                    if (w) {
+                        *reinterpret_cast<uint32_t*>(ne) = ksize | K_DEAD;
+                        c_dead += ksize;
+                        e = w;
+                        break;
+                    }
+                    hd = old;
+                    *reinterpret_cast<uint32_t*>(ne + 4) = hd;
+                }
+            }
+            if (need_chunk && coff != ~0ull && e) {
+                uint8_t* c = d.pool + coff;
+                init_chunk(c, ccap, vw, 1, owner_of(d, e), 0ull);
+                put_value(b, i, c, 0);
+                push_chunk(e, c, vref_of(d, coff), ld_relaxed_u64(list_head(e)));
+                done = true;
+            }
+            __syncwarp();
+            if (lane == 0) add_release64(my_ann, ~0ull);
+        }
+        // ---- declines: certified for new keys; a resident key with a value left over is pending
+        const bool declined = valid && !done && res == R_OK;
+        if (__any_sync(FULLMASK, declined)) {
+            w_full = true;
+            if (!w_quiet) {
+                if (lane == 0)
+                    for (uint32_t c = 0; c < d.n_slots; ++c)
+                        while (ld_acquire_u64(d.ann + (uint64_t)c * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
+                __syncwarp();
+                w_quiet = true;
+                if (declined && !e) e = chain_find_w(d, ld_relaxed_u32(d.dir + bkt), 0, tag, len, w0, w1, tail);
+            }
+            if (declined) {
+                res = R_POST;
+                if (e) {  // resident key: its value may still fit a shared head chunk
+                    uint64_t cr = 0, lh = 0;
+                    uint32_t base = 0, pc = 0;
+                    if (reserve_head(d, e, 1, &cr, &base, &lh, &pc)) {
+                        put_value(b, i, vref_ptr(d, cr), base);
+                        res = R_OK;
+                    } else {
+                        d.retain[(uint32_t)((uint64_t)(e - d.pool) >> d.page_shift)] = 1;  // pending key
+                    }
+                }
+            }
+        }
+        const unsigned bits = __ballot_sync(FULLMASK, valid && res != R_OK);
+        if (bits) {
+            const unsigned tl = __ballot_sync(FULLMASK, valid && res == R_TOOLARGE);
+            const unsigned pkb = __reduce_add_sync(FULLMASK, (valid && res != R_OK) ? len : 0u);
+            if (lane == 0) { c_post += __popc(bits); c_tl += __popc(tl); c_pkb += pkb; }
+        }
+        if (lane == 0) b.bitmap[g] = bits;
+    }
+    if (lane == 0) {
+        if (c_post) atomicAdd(&S.post, c_post);
+        if (c_tl) atomicAdd(&S.toolarge, c_tl);
+        if (c_pkb) atomicAdd(&d.ctrl->kept_key_bytes, c_pkb);
+    }
+    if (c_dead) atomicAdd(&S.dead, c_dead);
+    __syncthreads();
+    // final fill of every private chunk still open
+    for (int p = tid; p < NH; p += THREADS) {
+        const unsigned long long w = S.pw[p];
+        const uint32_t cref = (uint32_t)(w >> 32);
+        if (cref) *reinterpret_cast<uint32_t*>(ref_ptr(d, cref) + 4) = min((uint32_t)w, PC_CAP);
     }
     if (tid == 0) {
         d.cursors[2 * blockIdx.x] = S.cur[0];
@@ -1491,9 +1839,9 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             unsigned int* hist = n_out + 1;
             cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
             hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
-            hot_threshold_kernel<<<1, 32, 0, s>>>(hist, 4u);
-            hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out);
-            hot_clamp_kernel<<<1, 32, 0, s>>>(n_out);
+            hot_threshold_kernel<<<1, 32, 0, s>>>(hist, 4u, (uint32_t)hot::K);
+            hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)hot::K);
+            hot_clamp_kernel<<<1, 32, 0, s>>>(n_out, (uint32_t)hot::K);
             hot_resolve_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
             hl = list;
             nh = n_out;
@@ -1509,17 +1857,40 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
         if (b.vals) insert_stream_kernel<true, T, SUB><<<grid, T, sm, s>>>(d, b, hl, nh);
         else insert_stream_kernel<false, T, SUB><<<grid, T, sm, s>>>(d, b, hl, nh);
     } else {
-        size_t sm = sizeof(Smem<1>);
-        static bool attr1 = false;
-        if (!attr1) { cudaFuncSetAttribute(insert_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm); attr1 = true; }
-        insert_kernel<1><<<grid, Cfg<1>::THREADS, sm, s>>>(d, b);
+        const hot::Entry* hl = nullptr;
+        const unsigned int* nh = nullptr;
+        const uint64_t n_sample = 1ull << 18;
+        if (hot_scratch && b.n >= 8 * n_sample) {
+            uint8_t* p = reinterpret_cast<uint8_t*>(hot_scratch);
+            hot::SampleSlot* tab = reinterpret_cast<hot::SampleSlot*>(p);
+            hot::Entry* list = reinterpret_cast<hot::Entry*>(p + sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS);
+            unsigned int* n_out = reinterpret_cast<unsigned int*>(list + hot::K);
+            unsigned int* hist = n_out + 1;
+            cudaMemsetAsync(tab, 0, sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS, s);
+            cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
+            hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, b.n / n_sample, n_sample, tab);
+            hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
+            hot_threshold_kernel<<<1, 32, 0, s>>>(hist, 4u, (uint32_t)gst::K);
+            hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)gst::K);
+            hot_clamp_kernel<<<1, 32, 0, s>>>(n_out, (uint32_t)gst::K);
+            hot_resolve_group_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
+            hl = list;
+            nh = n_out;
+        }
+        const size_t sm = sizeof(gst::Smem);
+        static bool attrg = false;
+        if (!attrg) {
+            cudaFuncSetAttribute(insert_group_stream_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            attrg = true;
+        }
+        insert_group_stream_kernel<<<grid, gst::THREADS, sm, s>>>(d, b, hl, nh);
     }
     return cudaGetLastError();
 }
 size_t sepo_hot_scratch_bytes() {
     return sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS + sizeof(hot::Entry) * hot::K + (HOT_HIST + 16) * 4;
 }
-int sepo_default_grid(int mode, int n_sms) { return mode == 0 ? n_sms : 2 * n_sms; }
+int sepo_default_grid(int mode, int n_sms) { (void)mode; return n_sms; }
 
 int sepo_launch_reprobe(const Dev& d, const Batch& b, int mode, int probe, int grid, unsigned long long* tile_counts,
                         cudaStream_t s) {
