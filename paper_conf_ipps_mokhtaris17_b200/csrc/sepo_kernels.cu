@@ -1,18 +1,16 @@
 // sepo_kernels.cu — the SEPO hot path on sm_100a (PAPER.md cited as P:L<line>).
 //
-//   insert_kernel   a1..a7  record ingest + hash, tile pre-aggregation of equal keys, chain walk,
+//   insert_stream_kernel / insert_group_stream_kernel
+//                   a1..a7  record ingest + hash, hot-key folding in shared memory, chain walk,
 //                           combine / group in place, page-pool allocation, lock-free head link,
-//                           decline -> postpone bitmap + count
+//                           certified decline -> postpone bitmap + count
 //   reprobe_kernel  a8      end-of-pass re-probe of declined records
 //   compact_*       a9      stream compaction of the postponed records (re-issue)
 //   seal/classify/relink a10 pass boundary: seal open pages, pick cold pages, rebuild the free
 //                           stack and (GROUP) re-link retained key pages
 //
-// The insert kernel is persistent: gridDim.x CTAs (the allocator slots) stride over tiles of TILE
-// records; per tile it stages offsets/hashes in shared memory, folds equal keys into one slot of
-// a shared open-addressing table (warp __match_any_sync first, so a hot Zipf key costs one shared
-// atomic per warp and one global op per tile), then resolves each distinct key against the global
-// table with one thread per key.
+// The insert kernels are persistent (one CTA of 1024 threads per SM = one allocator slot); every
+// warp streams 32-record groups without CTA barriers (see the kernel comments below).
 #include "sepo_dev.cuh"
 #include "sepo_kernels.h"
 #include <algorithm>
@@ -20,30 +18,6 @@
 
 namespace sepo {
 
-constexpr uint32_t EMPTY = 0xffffffffu;
-
-template <int MODE> struct Cfg;
-template <> struct Cfg<1> { static constexpr int THREADS = 512, TILE = 1024, NSLOT = 2048; };  // GROUP
-
-template <int MODE>
-struct Smem {
-    static constexpr int TILE = Cfg<MODE>::TILE, NSLOT = Cfg<MODE>::NSLOT;
-    uint64_t rec_off[TILE];
-    uint64_t rec_hash[TILE];
-    uint32_t rec_len[TILE];
-    uint32_t slot_rep[NSLOT];
-    unsigned long long slot_sum[NSLOT];  // COMBINE: value sum; GROUP: record count (rank source)
-    uint16_t dlist[NSLOT];
-    uint8_t slot_res[NSLOT];
-    // GROUP: where the slot's values go: chunk A (base slot a, `granted` values), then chunk B
-    uint64_t g_a[MODE == 1 ? NSLOT : 1];
-    uint64_t g_b[MODE == 1 ? NSLOT : 1];
-    uint32_t g_abase[MODE == 1 ? NSLOT : 1];
-    uint32_t g_granted[MODE == 1 ? NSLOT : 1];
-    unsigned long long cur[2];  // allocation cursors (entry/key pages, value pages)
-    uint32_t ndist;
-    unsigned long long post, toolarge, dead;
-};
 
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31u; }
 __device__ __forceinline__ uint32_t lanemask_lt() { return (1u << lane_id()) - 1u; }
@@ -146,303 +120,6 @@ __device__ __forceinline__ uint32_t reserve_head(const Dev& d, uint8_t* e, uint3
     *cref = h;
     *base = old;
     return min(k, cap - old);
-}
-
-// ================================================================ insert kernel (a1..a7)
-template <int MODE>
-__global__ void __launch_bounds__(Cfg<MODE>::THREADS, 2) insert_kernel(Dev d, Batch b) {
-    constexpr int THREADS = Cfg<MODE>::THREADS, TILE = Cfg<MODE>::TILE, NSLOT = Cfg<MODE>::NSLOT;
-    constexpr int R = TILE / THREADS;
-    extern __shared__ __align__(16) uint8_t smem_raw[];
-    Smem<MODE>& S = *reinterpret_cast<Smem<MODE>*>(smem_raw);
-    const uint32_t tid = threadIdx.x, lane = lane_id(), warp = tid >> 5;
-    const uint32_t PB = d.page_bytes;
-
-    for (int p = tid; p < NSLOT; p += THREADS) { S.slot_rep[p] = EMPTY; S.slot_sum[p] = 0; }
-    if (tid == 0) {
-        S.cur[0] = d.cursors[2 * blockIdx.x];
-        S.cur[1] = d.cursors[2 * blockIdx.x + 1];
-        S.post = 0; S.toolarge = 0; S.dead = 0;
-    }
-    __syncthreads();
-
-    const uint64_t ntiles = (b.n + TILE - 1) / TILE;
-    for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        const uint64_t t0 = tile * TILE;
-        // ---- phase 1: ingest + hash (a1)
-        uint64_t my_s[R], my_h[R];
-        uint32_t my_len[R];
-#pragma unroll
-        for (int k = 0; k < R; ++k) {
-            const uint32_t r = k * THREADS + tid;
-            const uint64_t i = t0 + r;
-            my_len[k] = 0; my_s[k] = 0; my_h[k] = 0;
-            if (i < b.n) {
-                rec_key(b, i, my_s[k], my_len[k]);
-                my_h[k] = hash_key(b.keys + my_s[k], my_len[k], d.seed);
-                S.rec_off[r] = my_s[k];
-                S.rec_len[r] = my_len[k];
-                S.rec_hash[r] = my_h[k];
-            }
-        }
-        if (tid == 0) S.ndist = 0;
-        __syncthreads();
-        // ---- phase 2: fold equal keys of the tile into shared slots (a2)
-        uint32_t my_slot[R], my_rank[R];
-#pragma unroll
-        for (int k = 0; k < R; ++k) {
-            const uint32_t r = k * THREADS + tid;
-            const bool valid = t0 + r < b.n;
-            const unsigned vm = __ballot_sync(FULLMASK, valid);
-            const unsigned long long hh = valid ? my_h[k] : (0xffffffff00000000ull | lane);
-            unsigned grp = __match_any_sync(FULLMASK, hh) & vm;
-            const uint32_t leader = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
-            const uint64_t ls = __shfl_sync(FULLMASK, my_s[k], leader);
-            const uint32_t llen = __shfl_sync(FULLMASK, my_len[k], leader);
-            bool eq = valid && (lane == leader || (llen == my_len[k] && in_key_eq(b.keys + my_s[k], b.keys + ls, llen)));
-            const unsigned eqm = __ballot_sync(FULLMASK, eq);
-            const unsigned joined = grp & eqm;           // lanes folded into the leader
-            const bool inserter = valid && (lane == leader || !eq);
-            uint64_t contrib = 0;
-            if (MODE == 0) {
-                const uint64_t v = valid ? rec_value(b, t0 + r) : 0;
-                if (b.vals == nullptr) {
-                    contrib = (lane == leader) ? (uint64_t)__popc(joined) : 1ull;
-                } else {
-                    uint64_t acc = 0;
-                    if (__any_sync(FULLMASK, __popc(joined) > 1)) {
-                        for (int q = 0; q < 32; ++q) {
-                            uint64_t vq = __shfl_sync(FULLMASK, v, q);
-                            if ((joined >> q) & 1u) acc += vq;
-                        }
-                    } else {
-                        acc = v;
-                    }
-                    contrib = (lane == leader) ? acc : v;
-                }
-            } else {
-                contrib = (lane == leader) ? (uint64_t)__popc(joined) : 1ull;
-            }
-            uint32_t pos = EMPTY, rank0 = 0;
-            if (inserter) {
-                pos = (uint32_t)(my_h[k] >> 7) & (NSLOT - 1);
-                while (true) {
-                    uint32_t cur = *reinterpret_cast<volatile uint32_t*>(&S.slot_rep[pos]);
-                    if (cur == EMPTY) {
-                        cur = atomicCAS(&S.slot_rep[pos], EMPTY, r);
-                        if (cur == EMPTY) break;
-                    }
-                    if (S.rec_hash[cur] == my_h[k] && S.rec_len[cur] == my_len[k] &&
-                        in_key_eq(b.keys + S.rec_off[cur], b.keys + my_s[k], my_len[k]))
-                        break;
-                    pos = (pos + 1) & (NSLOT - 1);
-                }
-                rank0 = (uint32_t)atomicAdd(&S.slot_sum[pos], (unsigned long long)contrib);
-            }
-            // followers take the leader's slot; rank of a record among its key's records in the tile
-            const uint32_t lpos = __shfl_sync(FULLMASK, pos, leader);
-            const uint32_t lrank = __shfl_sync(FULLMASK, rank0, leader);
-            if (valid && eq && lane != leader) {
-                my_slot[k] = lpos;
-                my_rank[k] = lrank + __popc(joined & lanemask_lt());
-            } else {
-                my_slot[k] = pos;
-                my_rank[k] = rank0;
-            }
-        }
-        __syncthreads();
-        // ---- phase 3: dense list of the tile's distinct keys
-        for (int p0 = 0; p0 < NSLOT; p0 += THREADS) {
-            const int p = p0 + tid;
-            const bool occ = S.slot_rep[p] != EMPTY;
-            const unsigned bal = __ballot_sync(FULLMASK, occ);
-            uint32_t base = 0;
-            if (lane == 0 && bal) base = atomicAdd(&S.ndist, (uint32_t)__popc(bal));
-            base = __shfl_sync(FULLMASK, base, 0);
-            if (occ) S.dlist[base + __popc(bal & lanemask_lt())] = (uint16_t)p;
-        }
-        __syncthreads();
-        // ---- phase 4: one thread per distinct key against the global table (a3..a6)
-        const uint32_t nd = S.ndist;
-        for (uint32_t j0 = 0; j0 < nd; j0 += THREADS) {
-            const uint32_t j = j0 + tid;
-            const bool act = j < nd;
-            uint32_t pos = 0, r = 0, len = 0;
-            uint64_t s = 0, h = 0, sum = 0;
-            if (act) {
-                pos = S.dlist[j];
-                r = S.slot_rep[pos];
-                s = S.rec_off[r]; len = S.rec_len[r]; h = S.rec_hash[r];
-                sum = S.slot_sum[pos];
-            }
-            const uint8_t* key = b.keys + s;
-            const uint32_t bkt = act ? bucket_of(h, d.n_buckets) : 0;
-            const uint32_t tag = tag_of(h);
-            uint32_t head = 0;
-            uint8_t* found = nullptr;
-            if (act) {
-                head = ld_relaxed_u32(d.dir + bkt);
-                found = chain_find(d, head, 0, tag, len, key);
-            }
-            uint32_t res = R_OK;
-            const uint32_t esize = MODE == 0 ? centry_size(len) : gkey_size(len);
-            bool need = act && !found;
-            if (need && (len > 65535u - 64u || esize > PB)) { need = false; res = R_TOOLARGE; }
-            if (need && inject_fail(d, h, t0 + r)) { need = false; res = R_POST; }
-
-            if (MODE == 0) {
-                if (act && found) atomicAdd(reinterpret_cast<unsigned long long*>(entry_val(found, len)), (unsigned long long)sum);
-                const uint64_t off = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
-                if (need) {
-                    if (off == ~0ull) {
-                        res = R_POST;
-                    } else {
-                        uint8_t* e = d.pool + off;
-                        *reinterpret_cast<uint32_t*>(e) = esize | K_COMBINE;
-                        *reinterpret_cast<uint32_t*>(e + 4) = head;
-                        *reinterpret_cast<uint32_t*>(e + 8) = tag;
-                        *reinterpret_cast<uint32_t*>(e + 12) = len;
-                        store_key(e + KEY_OFF, key, len);
-                        *reinterpret_cast<unsigned long long*>(entry_val(e, len)) = sum;
-                        const uint32_t me = off_ref(off);
-                        while (true) {  // lock-free head insertion
-                            const uint32_t old = cas_release(d.dir + bkt, head, me);
-                            if (old == head) break;
-                            uint8_t* w = chain_find(d, old, head, tag, len, key);
-                            if (w) {  // the key was linked meanwhile: combine there, retire ours
-                                atomicAdd(reinterpret_cast<unsigned long long*>(entry_val(w, len)), (unsigned long long)sum);
-                                *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
-                                atomicAdd(&S.dead, (unsigned long long)esize);
-                                break;
-                            }
-                            head = old;
-                            *reinterpret_cast<uint32_t*>(e + 4) = head;
-                        }
-                    }
-                }
-                if (act) {
-                    S.slot_res[pos] = (uint8_t)res;
-                    S.slot_rep[pos] = EMPTY;
-                    S.slot_sum[pos] = 0;
-                }
-            } else {
-                // ---------------- GROUP (multi-valued): key entry + value chunks
-                const uint32_t k = (uint32_t)sum;
-                const uint32_t vws = b.vo ? 0u : b.vw;  // fixed-width slot bytes (variable: see host)
-                uint64_t a_ref = 0, b_ref = 0;
-                uint32_t abase = 0, granted = 0, prev_cap = 0;
-                uint64_t lhead = 0;
-                if (act && found) granted = reserve_head(d, found, k, &a_ref, &abase, &lhead, &prev_cap);
-                // values that still need a chunk
-                const bool need_chunk = act && res == R_OK && granted < k;
-                const uint32_t rest = k - granted;
-                const uint32_t ccap = need_chunk ? chunk_cap(d, rest, prev_cap, vws) : 0;
-                const uint32_t csize = chunk_bytes(ccap, vws);
-                // allocate the key entry (new keys), then the chunk (value pages)
-                const uint64_t koffp = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
-                if (need && koffp == ~0ull) res = R_POST;
-                const bool want_chunk = need_chunk && res == R_OK;
-                const uint64_t coff = warp_alloc(d, &S.cur[1], want_chunk, csize, (uint8_t)PAGE_VALUE);
-                uint8_t* e = found;
-                if (need && res == R_OK) {
-                    // new key entry; linked even if its chunk allocation failed (then all its
-                    // values are pending and its page is retained at the pass end)
-                    uint8_t* ne = d.pool + koffp;
-                    *reinterpret_cast<uint32_t*>(ne) = esize | K_GKEY;
-                    *reinterpret_cast<uint32_t*>(ne + 4) = head;
-                    *reinterpret_cast<uint32_t*>(ne + 8) = tag;
-                    *reinterpret_cast<uint32_t*>(ne + 12) = len;
-                    store_key(ne + KEY_OFF, key, len);
-                    *reinterpret_cast<unsigned long long*>(entry_val(ne, len)) = 0ull;
-                    *reinterpret_cast<uint32_t*>(entry_val(ne, len) + 8) = d.gen;
-                    *reinterpret_cast<uint32_t*>(entry_val(ne, len) + 12) = 0u;
-                                        const uint32_t me = off_ref(koffp);
-                    e = ne;
-                    while (true) {
-                        const uint32_t old = cas_release(d.dir + bkt, head, me);
-                        if (old == head) break;
-                        uint8_t* w = chain_find(d, old, head, tag, len, key);
-                        if (w) {
-                            *reinterpret_cast<uint32_t*>(ne) = esize | K_DEAD;
-                            atomicAdd(&S.dead, (unsigned long long)esize);
-                            e = w;
-                            break;
-                        }
-                        head = old;
-                        *reinterpret_cast<uint32_t*>(ne + 4) = head;
-                    }
-                }
-                if (want_chunk && coff != ~0ull) {
-                    uint8_t* c = d.pool + coff;
-                    const uint64_t cref = vref_of(d, coff);
-                    init_chunk(c, ccap, vws, rest, owner_of(d, e), 0ull);
-                    push_chunk(e, c, cref, ld_relaxed_u64(list_head(e)));
-                    b_ref = cref;
-                } else if (want_chunk) {
-                    b_ref = 0;  // rest of the values are postponed (key stays resident: pending)
-                }
-                if (act) {
-                    if (res == R_OK && granted == 0 && b_ref == 0) res = R_POST;
-                    S.slot_res[pos] = (uint8_t)res;
-                    S.g_a[pos] = a_ref;
-                    S.g_b[pos] = b_ref;
-                    S.g_abase[pos] = abase;
-                    S.g_granted[pos] = granted;
-                    S.slot_rep[pos] = EMPTY;
-                    S.slot_sum[pos] = 0;
-                }
-            }
-        }
-        __syncthreads();
-        // ---- phase 5: per-record outcome -> bitmap word (a7); GROUP: write values into slots
-#pragma unroll
-        for (int k = 0; k < R; ++k) {
-            const uint32_t r = k * THREADS + tid;
-            const uint64_t i = t0 + r;
-            const bool valid = i < b.n;
-            bool post = false;
-            if (valid) {
-                const uint32_t res = S.slot_res[my_slot[k]];
-                if (MODE == 0) {
-                    post = res != R_OK;
-                } else {
-                    post = res != R_OK;
-                    if (!post) {
-                        const uint32_t g = S.g_granted[my_slot[k]];
-                        const uint32_t rk = my_rank[k];
-                        uint8_t* c = nullptr;
-                        uint32_t slot = 0;
-                        if (rk < g) { c = vref_ptr(d, S.g_a[my_slot[k]]); slot = S.g_abase[my_slot[k]] + rk; }
-                        else if (S.g_b[my_slot[k]]) { c = vref_ptr(d, S.g_b[my_slot[k]]); slot = rk - g; }
-                        else post = true;
-                        if (c) {
-                            uint64_t vs; uint32_t vl;
-                            rec_val_span(b, i, vs, vl);
-                            uint8_t* dst = c + CHUNK_HDR + (uint64_t)slot * vl;
-                            for (uint32_t q = 0; q < vl; ++q) dst[q] = __ldg(b.vals + vs + q);
-                        }
-                    }
-                }
-            }
-            const unsigned bits = __ballot_sync(FULLMASK, post);
-            const unsigned tl = __ballot_sync(FULLMASK, valid && S.slot_res[valid ? my_slot[k] : 0] == R_TOOLARGE);
-            const uint64_t wstart = t0 + k * THREADS + warp * 32;
-            if (lane == 0 && wstart < b.n) {
-                b.bitmap[wstart >> 5] = bits;
-                if (bits) atomicAdd(&S.post, (unsigned long long)__popc(bits));
-                if (tl) atomicAdd(&S.toolarge, (unsigned long long)__popc(tl));
-            }
-        }
-        __syncthreads();
-    }
-    __syncthreads();
-    if (tid == 0) {
-        d.cursors[2 * blockIdx.x] = S.cur[0];
-        d.cursors[2 * blockIdx.x + 1] = S.cur[1];
-        if (S.post) atomicAdd(&d.ctrl->postponed, S.post);
-        if (S.toolarge) atomicAdd(&d.ctrl->toolarge, S.toolarge);
-        if (S.dead) atomicAdd(&d.ctrl->dead_bytes, S.dead);
-    }
 }
 
 // ================================================================ COMBINE insert (a1..a7): hot set + streaming warps
