@@ -124,8 +124,9 @@ int sepo_configure(sepo_table* t, const sepo_options* opts);
  * keys/key_offsets/vals/val_offsets: device; see conventions above.
  *   COMBINE: vals == NULL => every value is 1 (Word Count / PVC); else fixed-width LE
  *            unsigned values (opts.fixed_val_width bytes each); val_offsets must be NULL.
- *   GROUP:   vals required; val_offsets != NULL => value i = vals[vo[i] .. vo[i+1]) (<= 256 B),
- *            else opts.fixed_val_width bytes each.
+ *   GROUP:   vals required; val_offsets != NULL => value i = vals[vo[i] .. vo[i+1]) (variable
+ *            length, stored as {u32 length, bytes} items; at most page_bytes - 40 bytes), else
+ *            opts.fixed_val_width bytes each (1..256).
  * postponed_bitmap: device, ceil(n/32) words, fully written (bits >= n are 0).
  * Returns the number of postponed records (>= 0; POSTPONE is not an error), or < 0.
  * The count is an upper bound of what must be re-issued: a declined record whose key another

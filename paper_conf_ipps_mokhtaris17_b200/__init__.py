@@ -145,12 +145,13 @@ class Table:
     __del__ = close
 
     # ---- the fine-grained SEPO calls (the requestor drives the pass loop)
-    def insert_batch(self, keys, key_offsets, vals=None, bitmap=None, n=None):
+    def insert_batch(self, keys, key_offsets, vals=None, bitmap=None, n=None, val_offsets=None):
         n = self._n(key_offsets, keys, n)
         if bitmap is None:
             import torch
             bitmap = torch.empty(max((n + 31) // 32, 1), dtype=torch.int32, device="cuda")
-        rc = self._L.sepo_insert_batch(self.h, _ptr(keys), _ptr(key_offsets), _ptr(vals), None, n, _ptr(bitmap))
+        rc = self._L.sepo_insert_batch(self.h, _ptr(keys), _ptr(key_offsets), _ptr(vals), _ptr(val_offsets), n,
+                                       _ptr(bitmap))
         if rc < 0:
             _err(rc)
         return int(rc), bitmap
@@ -195,9 +196,9 @@ class Table:
         return int(rc)
 
     # ---- the whole job
-    def run(self, keys, key_offsets, vals=None, n=None):
+    def run(self, keys, key_offsets, vals=None, n=None, val_offsets=None):
         n = self._n(key_offsets, keys, n)
-        rc = self._L.sepo_run(self.h, _ptr(keys), _ptr(key_offsets), _ptr(vals), None, n)
+        rc = self._L.sepo_run(self.h, _ptr(keys), _ptr(key_offsets), _ptr(vals), _ptr(val_offsets), n)
         if rc < 0:
             _err(rc)
         return int(rc)

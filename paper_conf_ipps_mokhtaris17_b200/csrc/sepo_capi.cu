@@ -176,8 +176,7 @@ int make_batch(sepo_table* t, Batch& b, const uint8_t* keys, const uint64_t* ko,
         if (vals && ((uintptr_t)vals % b.vw)) return fail(SEPO_E_INVAL, "vals not aligned to fixed_val_width");
     } else {
         if (!vals) return fail(SEPO_E_INVAL, "GROUP mode needs values");
-        if (vo) return fail(SEPO_E_INVAL, "GROUP mode: variable-length values are not supported yet (use fixed_val_width)");
-        if (b.vw == 0 || b.vw > 256) return fail(SEPO_E_INVAL, "GROUP fixed_val_width must be in 1..256");
+        if (!vo && (b.vw == 0 || b.vw > 256)) return fail(SEPO_E_INVAL, "GROUP fixed_val_width must be in 1..256");
     }
     return 0;
 }
@@ -699,12 +698,12 @@ int export_group(sepo_table* t) {
     const size_t np = pages.size();
     // pass A: key entries (identity = birth gen << 40 | entry ref) and value chunks
     struct KeyRec { const uint8_t* key; uint32_t len; uint64_t id; };
-    struct ChunkRec { const uint8_t* vals; uint32_t cnt; uint64_t owner; };
+    // units = used slots (fixed-width values, vw > 0) or used bytes (variable items, vw == 0)
+    struct ChunkRec { const uint8_t* vals; uint32_t units; uint64_t owner; uint32_t vw; uint32_t nitems; uint64_t nbytes; };
     std::vector<uint64_t> slots(16, 0);
     std::vector<std::vector<KeyRec>> tk(16);
     std::vector<std::vector<ChunkRec>> tc(16);
     std::atomic<int> bad{0};
-    uint32_t vw = t->opts.fixed_val_width;
     parallel_for(np, [&](unsigned w, size_t lo, size_t hi) {
         for (size_t i = lo; i < hi; ++i) {
             uint32_t off = 0;
@@ -722,13 +721,29 @@ int export_group(sepo_table* t) {
                     uint64_t poolo = ((uint64_t)pages[i].page << t->page_shift) + off;
                     tk[w].push_back({base + off + KEY_OFF, klen, ((uint64_t)birth << 40) | ((poolo >> 3) + 1)});
                 } else if (kind == K_VCHUNK) {
-                    uint32_t fill, cap;
+                    uint32_t fill, cap, cvw;
                     uint64_t owner;
                     memcpy(&fill, base + off + 4, 4);
                     memcpy(&owner, base + off + 8, 8);
                     memcpy(&cap, base + off + 24, 4);
+                    memcpy(&cvw, base + off + 28, 4);
                     cap &= ~CHUNK_PRIVATE;
-                    tc[w].push_back({base + off + CHUNK_HDR, std::min(fill, cap), owner});
+                    ChunkRec cr{base + off + CHUNK_HDR, std::min(fill, cap), owner, cvw, 0, 0};
+                    if (cvw) {
+                        cr.nitems = cr.units;
+                        cr.nbytes = (uint64_t)cr.units * cvw;
+                    } else {  // variable items {u32 len, bytes, pad4} up to the fill or an end mark
+                        uint32_t o = 0;
+                        while (o + 4 <= cr.units) {
+                            uint32_t l;
+                            memcpy(&l, cr.vals + o, 4);
+                            if (l == 0xffffffffu || o + 4 + l > cr.units) break;
+                            ++cr.nitems;
+                            cr.nbytes += l;
+                            o += (4 + l + 3) & ~3u;
+                        }
+                    }
+                    tc[w].push_back(cr);
                     slots[w] += cap;
                 }
                 off += sz;
@@ -760,25 +775,40 @@ int export_group(sepo_table* t) {
     for (auto& v : tc) t->st.value_chunks += v.size();
     for (auto x : slots) t->st.value_slots += x;
     const uint64_t nk = keys.size();
-    std::vector<uint64_t> cnt(nk + 1, 0);
+    std::vector<uint64_t> cnt(nk + 1, 0), byt(nk + 1, 0);
     for (auto& v : tc)
         for (auto& c : v) {
             auto it = id2k.find(c.owner);
             if (it == id2k.end()) return fail(SEPO_E_STATE, "value chunk with unknown owner");
-            cnt[it->second + 1] += c.cnt;
+            cnt[it->second + 1] += c.nitems;
+            byt[it->second + 1] += c.nbytes;
         }
-    for (uint64_t k = 0; k < nk; ++k) cnt[k + 1] += cnt[k];
+    for (uint64_t k = 0; k < nk; ++k) { cnt[k + 1] += cnt[k]; byt[k + 1] += byt[k]; }
     const uint64_t nv = cnt[nk];
     t->x_loffs.assign(cnt.begin(), cnt.end());
-    t->x_vals.resize(nv * vw);
+    t->x_vals.resize(byt[nk]);
     t->x_voffs.resize(nv + 1);
-    for (uint64_t i = 0; i <= nv; ++i) t->x_voffs[i] = i * vw;
-    std::vector<uint64_t> cur(cnt.begin(), cnt.end() - 1);
+    t->x_voffs[nv] = byt[nk];
+    std::vector<uint64_t> cur(cnt.begin(), cnt.end() - 1), curb(byt.begin(), byt.end() - 1);
     for (auto& v : tc)
         for (auto& c : v) {
-            uint64_t k = id2k[c.owner];
-            memcpy(t->x_vals.data() + cur[k] * vw, c.vals, (size_t)c.cnt * vw);
-            cur[k] += c.cnt;
+            const uint64_t k = id2k[c.owner];
+            if (c.vw) {
+                memcpy(t->x_vals.data() + curb[k], c.vals, (size_t)c.nbytes);
+                for (uint32_t j = 0; j < c.nitems; ++j) t->x_voffs[cur[k] + j] = curb[k] + (uint64_t)j * c.vw;
+                cur[k] += c.nitems;
+                curb[k] += c.nbytes;
+            } else {
+                uint32_t o = 0;
+                for (uint32_t j = 0; j < c.nitems; ++j) {
+                    uint32_t l;
+                    memcpy(&l, c.vals + o, 4);
+                    t->x_voffs[cur[k]++] = curb[k];
+                    memcpy(t->x_vals.data() + curb[k], c.vals + o + 4, l);
+                    curb[k] += l;
+                    o += (4 + l + 3) & ~3u;
+                }
+            }
         }
     uint64_t kb = 0;
     for (auto* kr : keys) kb += kr->len;

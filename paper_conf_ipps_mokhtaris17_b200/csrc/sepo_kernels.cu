@@ -58,18 +58,24 @@ __device__ __forceinline__ void rec_val_span(const Batch& b, uint64_t i, uint64_
 }
 
 // ---------------------------------------------------------------- GROUP value-list helpers
-// Value chunk capacity for k values about to be appended: twice the demand (at least 8 slots).
-// Sized by the demand rather than grown from the previous chunk: many CTAs may find a hot key's
-// head chunk full at once and each installs a chunk, so large geometric chunks would mostly stay
-// empty (measured: 8x slot over-allocation on C4 with doubling).
-__device__ __forceinline__ uint32_t chunk_cap(const Dev& d, uint32_t k, uint32_t prev, uint32_t slot_bytes) {
+// Value chunks hold fixed-width values (vw > 0: capacity and fill count slots) or variable-length
+// values (vw == 0: items {u32 length, bytes, pad to 4}; capacity and fill count bytes; an unused
+// tail after a reservation that did not fit is closed by a 0xffffffff length).
+constexpr uint32_t ITEM_END = 0xffffffffu;
+__device__ __forceinline__ uint32_t item_units(uint32_t vw, uint32_t vlen) { return vw ? 1u : ((4u + vlen + 3u) & ~3u); }
+// Capacity for `need` units about to be appended: twice the demand (at least 8 slots / 64 bytes).
+// Sized by the demand rather than grown from the previous chunk: many CTAs may find a key's head
+// chunk full at once and each installs a chunk, so large geometric chunks would mostly stay empty
+// (measured: 8x slot over-allocation on C4 with doubling).
+__device__ __forceinline__ uint32_t chunk_cap(const Dev& d, uint32_t need, uint32_t prev, uint32_t vw) {
     (void)prev;
-    const uint32_t maxcap = (d.page_bytes / 4 - CHUNK_HDR) / slot_bytes;
-    uint32_t c = max(8u, 2u * k);
-    c = min(c, max(maxcap, k));
-    return min(c, (d.page_bytes - CHUNK_HDR) / slot_bytes);
+    const uint32_t unit = vw ? vw : 1u;
+    const uint32_t maxcap = (d.page_bytes / 4 - CHUNK_HDR) / unit;
+    uint32_t c = max(vw ? 8u : 64u, 2u * need);
+    c = min(c, max(maxcap, need));
+    return min(c, (d.page_bytes - CHUNK_HDR) / unit);
 }
-__device__ __forceinline__ uint32_t chunk_bytes(uint32_t cap, uint32_t slot_bytes) { return align16(CHUNK_HDR + cap * slot_bytes); }
+__device__ __forceinline__ uint32_t chunk_bytes(uint32_t cap, uint32_t vw) { return align16(CHUNK_HDR + cap * (vw ? vw : 1u)); }
 __device__ __forceinline__ uint64_t vref_of(const Dev& d, uint64_t off) { return ((uint64_t)d.gen << 40) | (uint64_t)off_ref(off); }
 __device__ __forceinline__ bool vref_resident(const Dev& d, uint64_t vref) { return vref != 0 && (uint32_t)(vref >> 40) == d.gen; }
 __device__ __forceinline__ uint8_t* vref_ptr(const Dev& d, uint64_t vref) { return ref_ptr(d, (uint32_t)vref); }
@@ -101,9 +107,10 @@ __device__ __forceinline__ void push_chunk(uint8_t* e, uint8_t* c, uint64_t cref
     asm volatile("atom.release.gpu.global.exch.b64 %0, [%1], %2;" : "=l"(old) : "l"(head), "l"(cref) : "memory");
     *reinterpret_cast<unsigned long long*>(c + 16) = old;
 }
-// Reserve k slots in the resident head chunk of key entry e. Returns granted count (0..k),
-// the chunk ref in *cref and the first slot in *base; *head_out = observed head, *prev_cap.
-__device__ __forceinline__ uint32_t reserve_head(const Dev& d, uint8_t* e, uint32_t k, uint64_t* cref, uint32_t* base,
+// Reserve `units` (1 slot, or an item's bytes) in the resident head chunk of key entry e.
+// Returns 1 and the first unit in *base if the whole reservation fits, else 0. A reservation that
+// crosses the end of a variable-value chunk closes the chunk's tail with ITEM_END.
+__device__ __forceinline__ uint32_t reserve_head(const Dev& d, uint8_t* e, uint32_t units, uint64_t* cref, uint32_t* base,
                                                  uint64_t* head_out, uint32_t* prev_cap) {
     uint64_t h = ld_relaxed_u64(list_head(e));
     *head_out = h;
@@ -112,14 +119,17 @@ __device__ __forceinline__ uint32_t reserve_head(const Dev& d, uint8_t* e, uint3
     if (!vref_resident(d, h)) return 0;
     uint8_t* c = vref_ptr(d, h);
     uint32_t cap = ldcg32(c + 24);
-    if (cap & CHUNK_PRIVATE) return 0;  // a CTA's private chunk: slots are handed out in its smem
+    if (cap & CHUNK_PRIVATE) return 0;  // a CTA's private chunk: its units are handed out in smem
     *prev_cap = cap;
     if (ldcg32(c + 4) >= cap) return 0;
-    uint32_t old = atomicAdd(reinterpret_cast<unsigned int*>(c + 4), k);
-    if (old >= cap) return 0;
+    uint32_t old = atomicAdd(reinterpret_cast<unsigned int*>(c + 4), units);
+    if (old + units > cap) {
+        if (old + 4 <= cap && ldcg32(c + 28) == 0) *reinterpret_cast<uint32_t*>(c + CHUNK_HDR + old) = ITEM_END;
+        return 0;
+    }
     *cref = h;
     *base = old;
-    return min(k, cap - old);
+    return 1;
 }
 
 // ================================================================ COMBINE insert (a1..a7): hot set + streaming warps
@@ -658,13 +668,21 @@ __device__ __forceinline__ uint32_t b1(uint64_t h) { return (uint32_t)(h >> 3) &
 __device__ __forceinline__ uint32_t b2(uint64_t h) { return (uint32_t)(h >> 13) & (NB - 1); }
 }  // namespace gst
 
-// write record i's value (vw bytes) into slot `slot` of chunk c
-__device__ __forceinline__ void put_value(const Batch& b, uint64_t i, uint8_t* c, uint32_t slot) {
-    const uint64_t src = rec_index(b, i) * (uint64_t)b.vw;
-    uint8_t* dst = c + CHUNK_HDR + (uint64_t)slot * b.vw;
-    if (b.vw == 4) *reinterpret_cast<uint32_t*>(dst) = __ldg(reinterpret_cast<const unsigned int*>(b.vals + src));
-    else if (b.vw == 8) *reinterpret_cast<unsigned long long*>(dst) = __ldg(reinterpret_cast<const unsigned long long*>(b.vals + src));
-    else for (uint32_t x = 0; x < b.vw; ++x) dst[x] = __ldg(b.vals + src + x);
+// write record i's value into chunk c at unit `at` (slot index, or byte offset of the item)
+__device__ __forceinline__ void put_value(const Batch& b, uint64_t i, uint8_t* c, uint32_t at) {
+    if (b.vo == nullptr) {
+        const uint64_t src = rec_index(b, i) * (uint64_t)b.vw;
+        uint8_t* dst = c + CHUNK_HDR + (uint64_t)at * b.vw;
+        if (b.vw == 4) *reinterpret_cast<uint32_t*>(dst) = __ldg(reinterpret_cast<const unsigned int*>(b.vals + src));
+        else if (b.vw == 8) *reinterpret_cast<unsigned long long*>(dst) = __ldg(reinterpret_cast<const unsigned long long*>(b.vals + src));
+        else for (uint32_t x = 0; x < b.vw; ++x) dst[x] = __ldg(b.vals + src + x);
+    } else {
+        uint64_t vs; uint32_t vl;
+        rec_val_span(b, i, vs, vl);
+        uint8_t* dst = c + CHUNK_HDR + at;
+        *reinterpret_cast<uint32_t*>(dst) = vl;
+        for (uint32_t x = 0; x < vl; ++x) dst[4 + x] = __ldg(b.vals + vs + x);
+    }
 }
 
 // GROUP hot keys: look up / insert the key entry (empty list) on allocator slot 0
@@ -721,12 +739,13 @@ __global__ void __launch_bounds__(1024) hot_resolve_group_kernel(Dev d, Batch b,
 
 __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
                                                                               const unsigned int* n_hot) {
-    using gst::THREADS; using gst::NB; using gst::NH; using gst::PC_CAP; using gst::b1; using gst::b2;
+    using gst::THREADS; using gst::NB; using gst::NH; using gst::b1; using gst::b2;
     extern __shared__ __align__(16) uint8_t smem_raw[];
     gst::Smem& S = *reinterpret_cast<gst::Smem*>(smem_raw);
     const uint32_t tid = threadIdx.x, lane = lane_id();
     const uint32_t PB = d.page_bytes;
-    const uint32_t vw = b.vw;
+    const uint32_t vw = b.vo ? 0u : b.vw;  // chunk format: fixed slots, or variable items (vw 0)
+    const uint32_t PC_CAP = vw ? gst::PC_CAP : 2048u;  // private chunk capacity (slots / bytes)
     for (int p = tid; p < NH; p += THREADS) { S.len[p] = hot::EMPTY_LEN; S.pw[p] = PC_CAP; }
     for (int p = tid; p < NB; p += THREADS) S.tags[p] = make_uint4(0, 0, 0, 0);
     if (tid == 0) {
@@ -771,6 +790,12 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
         if (len > 8) x = hash_word(x, w1);
         for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(b.keys + s + o, len - o < 8 ? len - o : 8));
         const uint64_t h = fmix64(x);
+        uint32_t units = 0;  // this record's value size in chunk units
+        if (valid) {
+            uint32_t vlen = vw;
+            if (b.vo) { uint64_t vs; rec_val_span(b, i, vs, vlen); }
+            units = item_units(vw, vlen);
+        }
         const uint8_t* tail = b.keys + s + 16;
         const uint32_t tag = tag_of(h), bkt = bucket_of(h, d.n_buckets);
         // ---- hot set probe
@@ -802,13 +827,29 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
                 const unsigned key = pos >= 0 ? (unsigned)pos : (0x10000u | lane);
                 const unsigned grp = __match_any_sync(FULLMASK, key) & hm;
                 const uint32_t leader = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
-                const uint32_t k = __popc(grp), rank = __popc(grp & ((1u << lane) - 1u));
+                // units of the group before this lane (excl) and in total (tot)
+                uint32_t excl = __popc(grp & ((1u << lane) - 1u)), tot = __popc(grp);
+                if (!vw && __any_sync(FULLMASK, pos >= 0)) {
+                    excl = 0; tot = 0;
+                    for (int x2 = 0; x2 < 32; ++x2) {
+                        const uint32_t ux = __shfl_sync(FULLMASK, units, x2);
+                        if ((grp >> x2) & 1u) { tot += ux; if ((uint32_t)x2 < lane) excl += ux; }
+                    }
+                }
                 unsigned long long old = 0;
-                if (pos >= 0 && lane == leader) old = atomicAdd(&S.pw[pos], (unsigned long long)k);
+                if (pos >= 0 && lane == leader) old = atomicAdd(&S.pw[pos], (unsigned long long)tot);
                 old = __shfl_sync(FULLMASK, old, leader);
                 const uint32_t cref = (uint32_t)(old >> 32), f0 = (uint32_t)old;
                 // the warp that crosses the end of the private chunk installs the next one
-                const bool cross = pos >= 0 && f0 <= PC_CAP && f0 + k > PC_CAP;
+                const bool cross = pos >= 0 && f0 <= PC_CAP && f0 + tot > PC_CAP;
+                const bool fits_old = pos >= 0 && cref && f0 + excl + units <= PC_CAP;
+                // variable items: the old chunk's used extent = the prefix of the group that fits
+                uint32_t used = PC_CAP;
+                if (!vw) {
+                    const unsigned fm = __ballot_sync(FULLMASK, fits_old) & grp;
+                    const uint32_t fu = __reduce_add_sync(FULLMASK, ((fm >> lane) & 1u) ? units : 0u);
+                    used = f0 + fu;
+                }
                 const bool want = cross && lane == leader && !w_full;
                 unsigned long long ann = 0;
                 const bool anyw = __any_sync(FULLMASK, want);
@@ -821,7 +862,7 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
                 }
                 uint32_t nref = 0;
                 if (want) {
-                    if (cref) *reinterpret_cast<uint32_t*>(ref_ptr(d, cref) + 4) = PC_CAP;  // old chunk is full
+                    if (cref) *reinterpret_cast<uint32_t*>(ref_ptr(d, cref) + 4) = used;  // old chunk is closed
                     if (coff != ~0ull) {
                         uint8_t* c = d.pool + coff;
                         uint8_t* ke = ref_ptr(d, S.ref[pos]);
@@ -829,7 +870,7 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
                         *reinterpret_cast<uint32_t*>(c + 24) = PC_CAP | CHUNK_PRIVATE;
                         push_chunk(ke, c, vref_of(d, coff), ld_relaxed_u64(list_head(ke)));
                         nref = off_ref(coff);
-                        const uint32_t rest = f0 + k - PC_CAP;
+                        const uint32_t rest = vw ? f0 + tot - PC_CAP : 0u;  // fixed: the overflow goes here
                         atomicExch(&S.pw[pos], ((unsigned long long)nref << 32) | rest);
                     } else {
                         atomicExch(&S.pw[pos], (unsigned long long)PC_CAP << 1);  // no chunk: hits go global
@@ -841,9 +882,9 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
                 }
                 nref = __shfl_sync(FULLMASK, nref, leader);
                 if (pos >= 0) {
-                    const uint32_t slot = f0 + rank;
-                    if (cref && slot < PC_CAP) { put_value(b, i, ref_ptr(d, cref), slot); done = true; }
-                    else if (cross && nref) { put_value(b, i, ref_ptr(d, nref), slot - PC_CAP); done = true; }
+                    const uint32_t at = f0 + excl;
+                    if (fits_old) { put_value(b, i, ref_ptr(d, cref), at); done = true; }
+                    else if (vw && cross && nref) { put_value(b, i, ref_ptr(d, nref), at - PC_CAP); done = true; }
                     else e = ref_ptr(d, S.ref[pos]);  // overflow: this record takes the global path
                 }
             }
@@ -855,7 +896,7 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
         if (valid && !done && e) {
             uint64_t cr = 0, lh = 0;
             uint32_t base = 0, pc = 0;
-            if (reserve_head(d, e, 1, &cr, &base, &lh, &pc)) {
+            if (reserve_head(d, e, units, &cr, &base, &lh, &pc)) {
                 put_value(b, i, vref_ptr(d, cr), base);
                 done = true;
                 need_chunk = false;
@@ -863,9 +904,11 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
         }
         uint32_t res = R_OK;
         const uint32_t ksize = gkey_size(len);
-        const uint32_t ccap = chunk_cap(d, 1, 0, vw);
+        const uint32_t ccap = chunk_cap(d, units, 0, vw);
         const uint32_t csize = chunk_bytes(ccap, vw);
-        if (need_key && (len > 65535u - 64u || ksize > PB)) { need_key = false; need_chunk = false; res = R_TOOLARGE; }
+        if ((need_key && (len > 65535u - 64u || ksize > PB)) || (need_chunk && CHUNK_HDR + units * (vw ? vw : 1u) > PB)) {
+            need_key = false; need_chunk = false; res = R_TOOLARGE;
+        }
         if (inj && need_key && inject_fail(d, h, i)) { need_key = false; need_chunk = false; res = R_POST; }
         const bool any_need = __any_sync(FULLMASK, need_chunk);
         uint64_t koff = ~0ull, coff = ~0ull;
@@ -913,7 +956,7 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
             }
             if (need_chunk && coff != ~0ull && e) {
                 uint8_t* c = d.pool + coff;
-                init_chunk(c, ccap, vw, 1, owner_of(d, e), 0ull);
+                init_chunk(c, ccap, vw, units, owner_of(d, e), 0ull);
                 put_value(b, i, c, 0);
                 push_chunk(e, c, vref_of(d, coff), ld_relaxed_u64(list_head(e)));
                 done = true;
@@ -938,7 +981,7 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
                 if (e) {  // resident key: its value may still fit a shared head chunk
                     uint64_t cr = 0, lh = 0;
                     uint32_t base = 0, pc = 0;
-                    if (reserve_head(d, e, 1, &cr, &base, &lh, &pc)) {
+                    if (reserve_head(d, e, units, &cr, &base, &lh, &pc)) {
                         put_value(b, i, vref_ptr(d, cr), base);
                         res = R_OK;
                     } else {
@@ -1013,7 +1056,7 @@ __global__ void __launch_bounds__(RP_THREADS) reprobe_kernel(Dev d, Batch b, uns
             if (mine) rec_key(b, i, s, len);
             if (PROBE) {
                 uint8_t* e = nullptr;
-                uint32_t want_cap = 0;
+                uint32_t want_cap = 0, units = 0;
                 if (mine) {
                     const uint64_t h = hash_key(b.keys + s, len, d.seed);
                     const uint32_t head = ld_relaxed_u32(d.dir + bucket_of(h, d.n_buckets));
@@ -1023,31 +1066,30 @@ __global__ void __launch_bounds__(RP_THREADS) reprobe_kernel(Dev d, Batch b, uns
                         still = false;
                     }
                     if (MODE == 1 && e) {  // resident key: append the value if its head chunk has room
+                        uint64_t vs; uint32_t vl;
+                        rec_val_span(b, i, vs, vl);
+                        const uint32_t cvw = b.vo ? 0u : b.vw;
+                        units = item_units(cvw, vl);
                         uint64_t cref = 0, lhead = 0;
                         uint32_t base = 0, pcap = 0;
-                        const uint32_t g = reserve_head(d, e, 1, &cref, &base, &lhead, &pcap);
-                        if (g) {
-                            uint64_t vs; uint32_t vl;
-                            rec_val_span(b, i, vs, vl);
-                            uint8_t* dst = vref_ptr(d, cref) + CHUNK_HDR + (uint64_t)base * vl;
-                            for (uint32_t q = 0; q < vl; ++q) dst[q] = __ldg(b.vals + vs + q);
+                        if (reserve_head(d, e, units, &cref, &base, &lhead, &pcap)) {
+                            put_value(b, i, vref_ptr(d, cref), base);
                             still = false;
                         } else {
-                            want_cap = chunk_cap(d, 1, pcap, b.vw);
+                            want_cap = chunk_cap(d, units, pcap, cvw);
                         }
                     }
                 }
                 if (MODE == 1) {
+                    const uint32_t cvw = b.vo ? 0u : b.vw;
                     const bool want = mine && still && e != nullptr;
-                    const uint64_t coff = warp_alloc(d, &s_cur[1], want, chunk_bytes(want ? want_cap : 0, b.vw),
+                    const uint64_t coff = warp_alloc(d, &s_cur[1], want, chunk_bytes(want ? want_cap : 0, cvw),
                                                      (uint8_t)PAGE_VALUE);
                     if (want) {
                         if (coff != ~0ull) {
                             uint8_t* c = d.pool + coff;
-                            init_chunk(c, want_cap, b.vw, 1, owner_of(d, e), 0ull);
-                            uint64_t vs; uint32_t vl;
-                            rec_val_span(b, i, vs, vl);
-                            for (uint32_t q = 0; q < vl; ++q) c[CHUNK_HDR + q] = __ldg(b.vals + vs + q);
+                            init_chunk(c, want_cap, cvw, units, owner_of(d, e), 0ull);
+                            put_value(b, i, c, 0);
                             push_chunk(e, c, vref_of(d, coff), ld_relaxed_u64(list_head(e)));
                             still = false;
                         } else {

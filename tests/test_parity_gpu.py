@@ -257,3 +257,52 @@ def test_c2_full_size_sampled(cuda):
         assert s.spell(r) == key
         assert int(vals[i]) == int(s.count_of_rank(r)), (key, r)
     t.close()
+
+
+# ------------------------------------------------------------------ variable-length GROUP values
+def _csr_t(items):
+    offs = np.zeros(len(items) + 1, dtype=np.int64)
+    offs[1:] = np.cumsum([len(x) for x in items])
+    data = np.frombuffer(b"".join(items) + b"\0" * 16, dtype=np.uint8).copy()
+    return torch.from_numpy(data).cuda(), torch.from_numpy(offs).cuda()
+
+
+def test_group_paper_example_variable_values(cuda):
+    """P:L133: http://google.com found in a.html, c.html and d.html -> one key, three paths."""
+    keys = [b"http://google.com", b"http://other.org", b"http://google.com", b"http://google.com"]
+    vals = [b"a.html", b"b.html", b"c.html", b"d.html"]
+    k, ko = _csr_t(keys)
+    v, vo = _csr_t(vals)
+    t = sepo().Table(sepo().budget_for(1 << 10, 4096, 16), 1 << 10, 4096, mode=sepo().GROUP)
+    t.run(k, ko, v, val_offsets=vo)
+    got = sepo().result_dict(t.export(), sepo().GROUP)
+    assert got == {b"http://google.com": [b"a.html", b"c.html", b"d.html"], b"http://other.org": [b"b.html"]}
+    t.close()
+
+
+@pytest.mark.parametrize("ratio", [1, 3])
+def test_group_variable_values_vs_oracle(cuda, ratio):
+    """Inverted index with variable-length page paths as values, over budget."""
+    s = gen.config("C1", scale=0.02)
+    hk, ho, _ = s.host()
+    kb = hk.tobytes()
+    words = [kb[ho[i]:ho[i + 1]] for i in range(s.n)]
+    rng = np.random.default_rng(3)
+    paths = [b"/site/%d/page%d.html" % (int(x) % 97, int(x)) for x in rng.integers(0, 5000, size=s.n)]
+    exp = oracle.group(*[np.frombuffer(b"".join(words), dtype=np.uint8), ho],
+                       np.frombuffer(b"".join(paths), dtype=np.uint8),
+                       val_offs=np.concatenate([[0], np.cumsum([len(p) for p in paths])]).astype(np.uint64)).as_dict()
+    k, ko = _csr_t(words)
+    v, vo = _csr_t(paths)
+    t = sepo().Table(sepo().budget_for(1 << 12, 4096, 4096), 1 << 12, 4096, mode=sepo().GROUP)
+    t.run(k, ko, v, val_offsets=vo)
+    pages = t.stats()["pages_used_max"]
+    t.close()
+    t = sepo().Table(sepo().budget_for(1 << 12, 4096, max(8, pages // ratio + 2)), 1 << 12, 4096, mode=sepo().GROUP,
+                     check_dups=True)
+    passes = t.run(k, ko, v, val_offsets=vo)
+    got = sepo().result_dict(t.export(), sepo().GROUP)
+    t.close()
+    assert_same(got, exp)
+    if ratio > 1:
+        assert passes >= 2
