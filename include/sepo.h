@@ -98,6 +98,7 @@ typedef struct sepo_stats {
     uint64_t value_chunks;         /* GROUP export: value chunks parsed */
     uint64_t value_slots;          /* GROUP export: value slots in those chunks (capacity) */
     double t_insert_ms, t_reprobe_ms, t_compact_ms, t_evict_ms, t_export_ms, t_h2d_ms;
+    double t_insert_ms_per_pass[SEPO_MAX_PASS_STATS]; /* insert-kernel time of each pass */
 } sepo_stats;
 
 /* Create a table on the current CUDA device.

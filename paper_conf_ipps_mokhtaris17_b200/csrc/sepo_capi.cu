@@ -387,6 +387,7 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
     if ((rc = read_ctrl(t))) return rc;
     t->last_insert_ms = elapsed_ms(t->ev0, t->ev1);
     t->st.t_insert_ms += t->last_insert_ms;
+    if (t->st.passes < SEPO_MAX_PASS_STATS) t->st.t_insert_ms_per_pass[t->st.passes] += t->last_insert_ms;
     t->st.insert_calls++;
     t->st.records_inserted += n;
     if (b.idx) t->st.key_bytes_inserted += t->pending_idx_key_bytes;

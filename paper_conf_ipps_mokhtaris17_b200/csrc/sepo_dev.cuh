@@ -114,6 +114,76 @@ __device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long
 }
 constexpr unsigned long long ANN_FULL = 1ull << 63;
 constexpr uint32_t ANN_STRIDE = 16;  // u64 words between announcement words (128 B)
+// ---------------------------------------------------------------- L2 residency policy
+// The streamed input (16 GB for C2) would otherwise push table lines out of L2: on B200 a 55 MB
+// table next to an evict_normal input stream missed L2 on 58 % of its sectors (ncu, pass 1 of the
+// C2 4x job: 71 GB DRAM read for 16 GB of input). Input loads therefore carry an L2 evict_first
+// policy (and skip L1 allocation); table accesses keep the default (or evict_last, SEPO_TAB_POLICY).
+// createpolicy with a constant fraction folds into the load's memory descriptor (no extra SASS).
+#ifndef SEPO_IN_POLICY
+#define SEPO_IN_POLICY 1
+#endif
+#ifndef SEPO_TAB_POLICY
+#define SEPO_TAB_POLICY 0
+#endif
+__device__ __forceinline__ uint64_t pol_in() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint64_t pol_tab() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+// immutable input (keys, offsets, values, re-issue indices): read-only path, L2 evict_first
+__device__ __forceinline__ uint64_t ld_in64(const void* p) {
+#if SEPO_IN_POLICY
+    uint64_t v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol_in()));
+    return v;
+#else
+    return __ldg(reinterpret_cast<const unsigned long long*>(p));
+#endif
+}
+__device__ __forceinline__ uint32_t ld_in32(const void* p) {
+#if SEPO_IN_POLICY
+    uint32_t v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol_in()));
+    return v;
+#else
+    return __ldg(reinterpret_cast<const unsigned int*>(p));
+#endif
+}
+__device__ __forceinline__ uint32_t ld_in16(const void* p) {
+#if SEPO_IN_POLICY
+    unsigned short v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u16 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol_in()));
+    return v;
+#else
+    return __ldg(reinterpret_cast<const unsigned short*>(p));
+#endif
+}
+__device__ __forceinline__ uint32_t ld_in8(const void* p) {
+#if SEPO_IN_POLICY
+    unsigned short v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol_in()));
+    return v & 0xffu;
+#else
+    return __ldg(reinterpret_cast<const unsigned char*>(p));
+#endif
+}
+__device__ __forceinline__ uint4 ld_in128(const void* p) {
+#if SEPO_IN_POLICY
+    uint4 v;
+    asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+        : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol_in()));
+    return v;
+#else
+    return __ldg(reinterpret_cast<const uint4*>(p));
+#endif
+}
+
 // L2-coherent loads of published entry fields (never stale L1 lines)
 __device__ __forceinline__ uint64_t ldcg64(const void* p) { return __ldcg(reinterpret_cast<const unsigned long long*>(p)); }
 __device__ __forceinline__ uint32_t ldcg32(const void* p) { return __ldcg(reinterpret_cast<const unsigned int*>(p)); }
@@ -124,8 +194,8 @@ __device__ __forceinline__ uint64_t load_in_word(const uint8_t* p, uint32_t nb) 
     uintptr_t a = reinterpret_cast<uintptr_t>(p);
     uint32_t sh = (uint32_t)(a & 7u);
     const unsigned long long* q = reinterpret_cast<const unsigned long long*>(a - sh);
-    uint64_t v = __ldg(q) >> (8 * sh);
-    if (sh + nb > 8) v |= __ldg(q + 1) << (64 - 8 * sh);
+    uint64_t v = ld_in64(q) >> (8 * sh);
+    if (sh + nb > 8) v |= ld_in64(q + 1) << (64 - 8 * sh);
     if (nb < 8) v &= (1ull << (8 * nb)) - 1ull;
     return v;
 }
@@ -188,8 +258,28 @@ __device__ __forceinline__ void store_key(uint8_t* ek, const uint8_t* p, uint32_
     }
 }
 
+#if SEPO_TAB_POLICY
+__device__ __forceinline__ uint4 ldcg128(const void* p) {
+    uint4 v;
+    asm volatile("ld.global.cg.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol_tab()));
+    return v;
+}
+__device__ __forceinline__ ulonglong2 ldcg128u(const void* p) {
+    ulonglong2 v;
+    asm volatile("ld.global.cg.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;" : "=l"(v.x), "=l"(v.y) : "l"(p), "l"(pol_tab()));
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_dir(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.relaxed.gpu.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol_tab()) : "memory");
+    return v;
+}
+#else
 __device__ __forceinline__ uint4 ldcg128(const void* p) { return __ldcg(reinterpret_cast<const uint4*>(p)); }
 __device__ __forceinline__ ulonglong2 ldcg128u(const void* p) { return __ldcg(reinterpret_cast<const ulonglong2*>(p)); }
+__device__ __forceinline__ uint32_t ld_dir(const uint32_t* p) { return ld_relaxed_u32(p); }
+#endif
 
 // Walk the chain [ref .. stop) for an entry with (tag, len, key) — key given by its INPUT bytes.
 // Only entries of the resident generation are reachable (head insertion; the directory
@@ -228,9 +318,9 @@ __device__ __forceinline__ void load_key16(const uint8_t* p, uint32_t len, uint6
     const unsigned long long* q = reinterpret_cast<const unsigned long long*>(a - sh);
     const uint32_t nb = len < 16 ? len : 16;
     const uint32_t nw = (sh + nb + 7) >> 3;  // aligned words touched (1..3)
-    const uint64_t x0 = __ldg(q);
-    const uint64_t x1 = nw > 1 ? __ldg(q + 1) : 0ull;
-    const uint64_t x2 = nw > 2 ? __ldg(q + 2) : 0ull;
+    const uint64_t x0 = ld_in64(q);
+    const uint64_t x1 = nw > 1 ? ld_in64(q + 1) : 0ull;
+    const uint64_t x2 = nw > 2 ? ld_in64(q + 2) : 0ull;
     if (sh == 0) { w0 = x0; w1 = x1; }
     else {
         w0 = (x0 >> (8 * sh)) | (x1 << (64 - 8 * sh));

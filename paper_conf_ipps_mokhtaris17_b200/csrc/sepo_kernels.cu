@@ -23,23 +23,23 @@ __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31u; }
 __device__ __forceinline__ uint32_t lanemask_lt() { return (1u << lane_id()) - 1u; }
 
 // record i of a batch -> its index in keys / key_offsets / vals (re-issue by index, a9)
-__device__ __forceinline__ uint64_t rec_index(const Batch& b, uint64_t i) { return b.idx ? __ldg(reinterpret_cast<const unsigned long long*>(b.idx) + i) : i; }
+__device__ __forceinline__ uint64_t rec_index(const Batch& b, uint64_t i) { return b.idx ? ld_in64(b.idx + i) : i; }
 // value of record i for COMBINE (vw bytes LE, or 1 when vals == nullptr)
 __device__ __forceinline__ uint64_t rec_value(const Batch& b, uint64_t i) {
     if (b.vals == nullptr) return 1ull;
     i = rec_index(b, i);
     switch (b.vw) {
-        case 8: return __ldg(reinterpret_cast<const unsigned long long*>(b.vals) + i);
-        case 4: return __ldg(reinterpret_cast<const unsigned int*>(b.vals) + i);
-        case 2: return __ldg(reinterpret_cast<const unsigned short*>(b.vals) + i);
-        default: return b.vals[i];
+        case 8: return ld_in64(reinterpret_cast<const unsigned long long*>(b.vals) + i);
+        case 4: return ld_in32(reinterpret_cast<const unsigned int*>(b.vals) + i);
+        case 2: return ld_in16(reinterpret_cast<const unsigned short*>(b.vals) + i);
+        default: return ld_in8(b.vals + i);
     }
 }
 __device__ __forceinline__ void rec_key(const Batch& b, uint64_t i, uint64_t& s, uint32_t& len) {
     i = rec_index(b, i);
     if (b.ko) {
-        s = __ldg(reinterpret_cast<const unsigned long long*>(b.ko) + i);
-        len = (uint32_t)(__ldg(reinterpret_cast<const unsigned long long*>(b.ko) + i + 1) - s);
+        s = ld_in64(b.ko + i);
+        len = (uint32_t)(ld_in64(b.ko + i + 1) - s);
     } else {
         s = i * (uint64_t)b.kw;
         len = b.kw;
@@ -49,8 +49,8 @@ __device__ __forceinline__ void rec_key(const Batch& b, uint64_t i, uint64_t& s,
 __device__ __forceinline__ void rec_val_span(const Batch& b, uint64_t i, uint64_t& s, uint32_t& len) {
     i = rec_index(b, i);
     if (b.vo) {
-        s = __ldg(reinterpret_cast<const unsigned long long*>(b.vo) + i);
-        len = (uint32_t)(__ldg(reinterpret_cast<const unsigned long long*>(b.vo) + i + 1) - s);
+        s = ld_in64(b.vo + i);
+        len = (uint32_t)(ld_in64(b.vo + i + 1) - s);
     } else {
         s = i * (uint64_t)b.vw;
         len = b.vw;
@@ -165,7 +165,11 @@ struct SampleSlot { unsigned long long h; unsigned int count, rec; };
 }  // namespace hot
 
 __device__ __forceinline__ void red_add_u64(unsigned long long* p, unsigned long long v) {
+#if SEPO_TAB_POLICY
+    asm volatile("red.relaxed.gpu.global.add.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(pol_tab()) : "memory");
+#else
     asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+#endif
 }
 
 // hash + first 16 key bytes of record i
@@ -256,7 +260,7 @@ __global__ void __launch_bounds__(1024) hot_resolve_kernel(Dev d, Batch b, hot::
         uint32_t head = 0;
         uint8_t* found = nullptr;
         if (act) {
-            head = ld_relaxed_u32(d.dir + bkt);
+            head = ld_dir(d.dir + bkt);
             found = chain_find_w(d, head, 0, tag, e.len, e.w0, e.w1, tail);
         }
         const uint32_t esize = centry_size(e.len);
@@ -299,19 +303,34 @@ namespace stream {
 #define SEPO_DIR_ALL 1  // issue every record's directory load before the hot-set probe
 #endif
 #ifndef SEPO_STREAM_THREADS
-#define SEPO_STREAM_THREADS 1024  // measured best (profiles/r01_summary.md): 32 warps x 1 group
-#define SEPO_STREAM_SUB 1
+#define SEPO_STREAM_THREADS 1024  // one persistent CTA per SM (register-bound: 64 regs x 1024)
 #endif
-constexpr int THREADS = SEPO_STREAM_THREADS;  // warps x groups in flight per warp: see DESIGN.md §6
-constexpr int SUB = SEPO_STREAM_SUB;
+#ifndef SEPO_CHUNK_GROUPS
+#define SEPO_CHUNK_GROUPS 32      // consecutive 32-record groups a warp streams before it strides
+#endif
+#ifndef SEPO_FOLD
+#define SEPO_FOLD 1               // fold equal hot keys of a warp before the shared atomic
+#endif
+constexpr int THREADS = SEPO_STREAM_THREADS;
+constexpr uint64_t CH = SEPO_CHUNK_GROUPS;
 struct Smem {
-    uint4 tags[hot::NB];  // 4 fingerprints per bucket (one 16-B load per probed bucket)
-    uint64_t h[hot::NH], w0[hot::NH], w1[hot::NH];
+    uint4 tags[hot::NB];          // 4 fingerprints per bucket (one 16-B load per probed bucket)
+    ulonglong2 kw[hot::NH];       // first 16 key bytes, zero padded (one 16-B load per candidate)
     uint32_t len[hot::NH], ref[hot::NH];
     unsigned int plo[hot::NH], phi[hot::NH];  // pending sum = phi:plo (exact via carry)
     unsigned long long cur[2];
-    unsigned long long post, toolarge, dead;
+    unsigned long long post, toolarge, dead, pkb;
 };
+// Fingerprint of a hot slot: 23 hash bits, bit 8 always set (0 marks an empty slot) and the key
+// length (saturated at 255) in the low byte, so a fingerprint match also fixes the length of
+// keys shorter than 255 bytes and the full-key check is one 16-byte compare.
+__device__ __forceinline__ uint32_t fpl(uint64_t h, uint32_t len) {
+    return ((uint32_t)(h >> 32) & 0xfffffe00u) | 0x100u | min(len, 255u);
+}
+// A warp streams chunks of CH consecutive groups; chunk c belongs to warp c mod nw.
+__device__ __forceinline__ uint64_t next_group(uint64_t g, uint64_t nw) {
+    return ((g + 1) % CH) ? g + 1 : g + 1 + (nw - 1) * CH;
+}
 }  // namespace stream
 
 __device__ __forceinline__ void smem_add_u64(unsigned int* lo, unsigned int* hi, uint64_t v) {
@@ -337,10 +356,10 @@ __device__ __forceinline__ void warp_load_group(const Batch& b, uint64_t g, uint
     }
     uint64_t e;
     if (b.ko) {
-        s = valid ? __ldg(reinterpret_cast<const unsigned long long*>(b.ko) + i) : 0ull;
+        s = valid ? ld_in64(b.ko + i) : 0ull;
         e = __shfl_down_sync(FULLMASK, s, 1);
         const bool last = valid && (lane == 31 || i + 1 >= b.n);
-        if (last) e = __ldg(reinterpret_cast<const unsigned long long*>(b.ko) + i + 1);
+        if (last) e = ld_in64(b.ko + i + 1);
     } else {
         s = i * (uint64_t)b.kw;
         e = s + b.kw;
@@ -358,7 +377,7 @@ __device__ __forceinline__ void warp_load_group(const Batch& b, uint64_t g, uint
         return;
     }
     uint4 ch = make_uint4(0, 0, 0, 0);
-    if (base_al + 16ull * lane < end) ch = __ldg(reinterpret_cast<const uint4*>(b.keys + base_al) + lane);
+    if (base_al + 16ull * lane < end) ch = ld_in128(b.keys + base_al + 16ull * lane);
     const uint32_t off = (uint32_t)(s - base_al);
     const uint32_t c0 = valid ? (off >> 4) : 0u, c1 = min(c0 + 1u, 31u);
     const uint32_t x0 = __shfl_sync(FULLMASK, ch.x, c0), x1 = __shfl_sync(FULLMASK, ch.y, c0);
@@ -376,7 +395,97 @@ __device__ __forceinline__ void warp_load_group(const Batch& b, uint64_t g, uint
     else if (len < 16) w1 &= (1ull << (8 * (len - 8))) - 1ull;
 }
 
-template <bool VALS, int THREADS, int SUB>
+// ---- software-pipelined input of the COMBINE stream (contiguous batches)
+// Stage 1 (two groups ahead): the lanes' key offsets (and fixed-width values), plain loads.
+// Stage 2 (one group ahead): the group's key bytes as 16-B chunks, chunk `lane` per lane, over the
+//   window [start of record 0, start of record 31 + 16) — the first 16 bytes of every key —
+//   clamped to the batch's key end. Only the starts are needed, so it is issued as soon as stage 1
+//   of that group landed. Groups whose window exceeds 512 B (long keys) load per lane instead.
+// Stage 3 (the group itself): ends by shuffle (lane 31: the next group's first start, or one
+//   load at a chunk boundary), first 16 key bytes assembled from the chunks (shuffles + funnel).
+// Indexed batches (re-issue lists) skip the pipeline and load per lane.
+struct InCtx {
+    uint64_t ngroups, nw, kend;  // kend: key bytes end of the batch (ko[n] or n*kw)
+};
+template <bool VALS>
+__device__ __forceinline__ void in_stage1(const Batch& b, uint64_t g, uint32_t lane, uint64_t& s, uint64_t& v) {
+    const uint64_t i = g * 32 + lane;
+    s = 0;
+    v = 1;
+    if (b.idx || i >= b.n) return;
+    if (b.ko) s = ld_in64(b.ko + i);
+    if (VALS) v = rec_value(b, i);
+}
+__device__ __forceinline__ uint4 in_stage2(const Batch& b, const InCtx& c, uint64_t g, uint32_t lane, uint64_t s) {
+    uint4 ch = make_uint4(0, 0, 0, 0);
+    if (b.idx || g >= c.ngroups) return ch;
+    const uint64_t cnt = min((uint64_t)32, b.n - g * 32);
+    uint64_t base, last;
+    if (b.ko) {
+        base = __shfl_sync(FULLMASK, s, 0);
+        last = __shfl_sync(FULLMASK, s, (int)cnt - 1);
+    } else {
+        base = g * 32 * (uint64_t)b.kw;
+        last = base + (cnt - 1) * b.kw;
+    }
+    const uint64_t wend = min(last + 16, c.kend);
+    const uint64_t base_al = base & ~15ull;
+    if (wend - base_al > 512 || (reinterpret_cast<uintptr_t>(b.keys) & 15)) return ch;  // per-lane path
+    if (base_al + 16ull * lane < wend) ch = ld_in128(b.keys + base_al + 16ull * lane);
+    return ch;
+}
+// stage 3: s (in: start from stage 1; out: start), len, first 16 key bytes
+__device__ __forceinline__ void in_stage3(const Batch& b, const InCtx& c, uint64_t g, uint64_t gn, uint32_t lane,
+                                          uint64_t s_next, uint4 ch, uint64_t& s, uint32_t& len, uint64_t& w0,
+                                          uint64_t& w1) {
+    const uint64_t i = g * 32 + lane;
+    const bool valid = i < b.n;
+    w0 = 0; w1 = 0; len = 0;
+    if (b.idx) {
+        s = 0;
+        if (valid) { rec_key(b, i, s, len); load_key16(b.keys + s, len, w0, w1); }
+        return;
+    }
+    const uint64_t cnt = min((uint64_t)32, b.n - g * 32);
+    uint64_t e;
+    if (b.ko) {
+        e = __shfl_down_sync(FULLMASK, s, 1);
+        const uint64_t first_next = __shfl_sync(FULLMASK, s_next, 0);
+        if (i + 1 == b.n) e = c.kend;
+        else if (lane == 31 && valid) e = (gn == g + 1) ? first_next : ld_in64(b.ko + i + 1);
+    } else {
+        s = i * (uint64_t)b.kw;
+        e = s + b.kw;
+    }
+    len = valid ? (uint32_t)(e - s) : 0u;
+    const uint64_t base = b.ko ? __shfl_sync(FULLMASK, s, 0) : g * 32 * (uint64_t)b.kw;
+    const uint64_t last = b.ko ? __shfl_sync(FULLMASK, s, (int)cnt - 1) : base + (cnt - 1) * b.kw;
+    const uint64_t base_al = base & ~15ull;
+    const bool perlane = min(last + 16, c.kend) - base_al > 512 || (reinterpret_cast<uintptr_t>(b.keys) & 15);
+    if (perlane) {  // warp-uniform
+        if (valid) load_key16(b.keys + s, len, w0, w1);
+        return;
+    }
+    // every lane takes part in the shuffles (a chunk may sit in a lane past the last record)
+    const uint32_t off = valid ? (uint32_t)(s - base_al) : 0u;
+    const uint32_t c0 = off >> 4, c1 = min(c0 + 1u, 31u);
+    const uint32_t x0 = __shfl_sync(FULLMASK, ch.x, c0), x1 = __shfl_sync(FULLMASK, ch.y, c0);
+    const uint32_t x2 = __shfl_sync(FULLMASK, ch.z, c0), x3 = __shfl_sync(FULLMASK, ch.w, c0);
+    const uint32_t y0 = __shfl_sync(FULLMASK, ch.x, c1), y1 = __shfl_sync(FULLMASK, ch.y, c1);
+    const uint32_t y2 = __shfl_sync(FULLMASK, ch.z, c1), y3 = __shfl_sync(FULLMASK, ch.w, c1);
+    if (!valid) return;
+    const uint64_t X0 = ((uint64_t)x1 << 32) | x0, X1 = ((uint64_t)x3 << 32) | x2;
+    const uint64_t Y0 = ((uint64_t)y1 << 32) | y0, Y1 = ((uint64_t)y3 << 32) | y2;
+    const uint32_t r = off & 15u, sh = 8u * (r & 7u);
+    const uint64_t q0 = r < 8 ? X0 : X1, q1 = r < 8 ? X1 : Y0, q2 = r < 8 ? Y0 : Y1;
+    w0 = sh ? (q0 >> sh) | (q1 << (64 - sh)) : q0;
+    w1 = sh ? (q1 >> sh) | (q2 << (64 - sh)) : q1;
+    if (len == 0) { w0 = 0; w1 = 0; }
+    else if (len < 8) { w0 &= (1ull << (8 * len)) - 1ull; w1 = 0; }
+    else if (len < 16) w1 &= (1ull << (8 * (len - 8))) - 1ull;
+}
+
+template <bool VALS, int THREADS>
 __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
                                                                    const unsigned int* n_hot) {
     extern __shared__ __align__(16) uint8_t smem_raw[];
@@ -388,7 +497,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     if (tid == 0) {
         S.cur[0] = d.cursors[2 * blockIdx.x];
         S.cur[1] = d.cursors[2 * blockIdx.x + 1];
-        S.post = 0; S.toolarge = 0; S.dead = 0;
+        S.post = 0; S.toolarge = 0; S.dead = 0; S.pkb = 0;
     }
     __syncthreads();
     // load the hot set (read-only during the main loop)
@@ -397,7 +506,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         const hot::Entry e = hl[j];
         if (e.ref == 0) continue;
         // claim a free slot in bucket b1, else b2, else leave the key out (the set is only a cache)
-        const uint32_t f = hot::fp(e.h);
+        const uint32_t f = stream::fpl(e.h, e.len);
         int pos = -1;
         for (int c = 0; c < 2 && pos < 0; ++c) {
             const uint32_t bk = c == 0 ? hot::b1(e.h) : hot::b2(e.h);
@@ -406,225 +515,220 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
                 if (atomicCAS(&t[w], 0u, f) == 0u) pos = (int)(bk * 4 + w);
         }
         if (pos < 0) continue;
-        S.h[pos] = e.h; S.w0[pos] = e.w0; S.w1[pos] = e.w1; S.ref[pos] = e.ref; S.len[pos] = e.len;
+        S.kw[pos] = make_ulonglong2(e.w0, e.w1); S.ref[pos] = e.ref; S.len[pos] = e.len;
     }
     __syncthreads();
     const bool have_hot = nh > 0;
     const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
 
-    // Each warp streams SUB 32-record groups per step, stage by stage, so the loads of the SUB
-    // groups are in flight together (memory-level parallelism without more warps): input words
-    // and hashes; hot-set probe (shared memory); directory loads of the misses; folding of the
-    // hits; chain walks of the misses (one record per lane: tail keys rarely repeat in a warp).
-    const uint64_t ngroups = (b.n + 31) / 32;
-    const uint64_t gw = (uint64_t)blockIdx.x * (THREADS / 32) + (tid >> 5);
-    const uint64_t nw = (uint64_t)gridDim.x * (THREADS / 32);
-    unsigned long long c_post = 0, c_tl = 0, c_dead = 0, c_pkb = 0;
+    InCtx c;
+    c.ngroups = (b.n + 31) / 32;
+    c.nw = (uint64_t)gridDim.x * (THREADS / 32);
+    c.kend = b.idx ? 0ull : (b.ko ? ld_in64(b.ko + b.n) : b.n * (uint64_t)b.kw);
     bool w_full = false, w_quiet = false;  // warp-uniform: pool ran out / quiescence observed
-    for (uint64_t g0 = gw * SUB; g0 < ngroups; g0 += nw * SUB) {
-        uint64_t s[SUB], w0[SUB], w1[SUB], h[SUB], v[SUB];
-        uint32_t len[SUB];
-        bool valid[SUB];
-#pragma unroll
-        for (int q = 0; q < SUB; ++q) {
-            const uint64_t i = (g0 + q) * 32 + lane;
-            valid[q] = i < b.n;
-            v[q] = 1;
-            warp_load_group(b, g0 + q, lane, valid[q], s[q], len[q], w0[q], w1[q]);
-            if (VALS && valid[q]) v[q] = rec_value(b, i);
-        }
-#pragma unroll
-        for (int q = 0; q < SUB; ++q) {
-            uint64_t x = hash_init(len[q], d.seed);
-            if (len[q] > 0) x = hash_word(x, w0[q]);
-            if (len[q] > 8) x = hash_word(x, w1[q]);
-            for (uint32_t o = 16; o < len[q]; o += 8)
-                x = hash_word(x, load_in_word(b.keys + s[q] + o, len[q] - o < 8 ? len[q] - o : 8));
-            h[q] = fmix64(x);
-        }
-        // ---- directory load for every record, issued before the hot-set probe so that its latency
-        // (and the first chain entry's, below) overlaps the shared-memory work of the hits
-        uint32_t head[SUB];
+
+    // pipeline prologue: group g (stages 1+2 done), group gn (stage 1 in flight)
+    uint64_t g = ((uint64_t)blockIdx.x * (THREADS / 32) + (tid >> 5)) * stream::CH;
+    uint64_t s_c = 0, v_c = 1, s_n = 0, v_n = 1;
+    uint4 ch_c = make_uint4(0, 0, 0, 0);
+    if (g < c.ngroups) {
+        in_stage1<VALS>(b, g, lane, s_c, v_c);
+        ch_c = in_stage2(b, c, g, lane, s_c);
+    }
+    uint64_t gn = stream::next_group(g, c.nw);
+    if (gn < c.ngroups) in_stage1<VALS>(b, gn, lane, s_n, v_n);
+
+    while (g < c.ngroups) {
+        // ---- issue ahead: key chunks of gn, offsets (values) of the group after it
+        const uint4 ch_n = in_stage2(b, c, gn, lane, s_n);
+        const uint64_t gnn = stream::next_group(gn, c.nw);
+        uint64_t s_nn = 0, v_nn = 1;
+        if (gnn < c.ngroups) in_stage1<VALS>(b, gnn, lane, s_nn, v_nn);
+
+        // ---- group g: key words + hash (a1)
+        const uint64_t i = g * 32 + lane;
+        const bool valid = i < b.n;
+        uint64_t s = s_c, w0, w1;
+        uint32_t len;
+        in_stage3(b, c, g, gn, lane, s_n, ch_c, s, len, w0, w1);
+        const uint64_t v = VALS ? (b.idx ? (valid ? rec_value(b, i) : 0ull) : v_c) : 1ull;
+        uint64_t x = hash_init(len, d.seed);
+        if (len > 0) x = hash_word(x, w0);
+        if (len > 8) x = hash_word(x, w1);
+        for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(b.keys + s + o, len - o < 8 ? len - o : 8));
+        const uint64_t h = fmix64(x);
+        const uint32_t bkt = bucket_of(h, d.n_buckets);
+        // ---- directory word, issued before the hot-set probe so its latency overlaps it
+        uint32_t head = 0;
 #if SEPO_DIR_ALL
-#pragma unroll
-        for (int q = 0; q < SUB; ++q) head[q] = valid[q] ? ld_relaxed_u32(d.dir + bucket_of(h[q], d.n_buckets)) : 0u;
+        if (valid) head = ld_dir(d.dir + bkt);
 #endif
-        // ---- hot set: constant-time probe of two 4-way buckets, then a full-key check
-        int pos[SUB];
-#pragma unroll
-        for (int q = 0; q < SUB; ++q) {
-            pos[q] = -1;
-            if (valid[q] && have_hot) {
-                const uint32_t f = hot::fp(h[q]);
-                const uint32_t k1 = hot::b1(h[q]), k2 = hot::b2(h[q]);
-                const uint4 t1 = S.tags[k1];
-                int p = -1;
-                if (t1.x == f) p = 4 * k1; else if (t1.y == f) p = 4 * k1 + 1;
-                else if (t1.z == f) p = 4 * k1 + 2; else if (t1.w == f) p = 4 * k1 + 3;
-                else {
-                    const uint4 t2 = S.tags[k2];
-                    if (t2.x == f) p = 4 * k2; else if (t2.y == f) p = 4 * k2 + 1;
-                    else if (t2.z == f) p = 4 * k2 + 2; else if (t2.w == f) p = 4 * k2 + 3;
-                }
-                if (p >= 0 && S.h[p] == h[q] && S.len[p] == len[q] && S.w0[p] == w0[q] && S.w1[p] == w1[q] &&
-                    (len[q] <= 16 || entry_key_eq(ref_ptr(d, S.ref[p]) + KEY_OFF + 16, b.keys + s[q] + 16, len[q] - 16)))
-                    pos[q] = p;
+        // ---- hot set (a2): two 4-way buckets of fingerprints, then one 16-byte key compare
+        int pos = -1;
+        if (valid && have_hot) {
+            const uint32_t f = stream::fpl(h, len);
+            const uint32_t k1 = hot::b1(h), k2 = hot::b2(h);
+            const uint4 t1 = S.tags[k1];
+            int p = -1;
+            if (t1.x == f) p = 4 * k1; else if (t1.y == f) p = 4 * k1 + 1;
+            else if (t1.z == f) p = 4 * k1 + 2; else if (t1.w == f) p = 4 * k1 + 3;
+            else {
+                const uint4 t2 = S.tags[k2];
+                if (t2.x == f) p = 4 * k2; else if (t2.y == f) p = 4 * k2 + 1;
+                else if (t2.z == f) p = 4 * k2 + 2; else if (t2.w == f) p = 4 * k2 + 3;
+            }
+            if (p >= 0) {
+                const ulonglong2 k = S.kw[p];
+                if (k.x == w0 && k.y == w1 &&
+                    (len <= 16 || ((len < 255 || S.len[p] == len) &&
+                                   entry_key_eq(ref_ptr(d, S.ref[p]) + KEY_OFF + 16, b.keys + s + 16, len - 16))))
+                    pos = p;
             }
         }
 #if !SEPO_DIR_ALL
-#pragma unroll
-        for (int q = 0; q < SUB; ++q)
-            head[q] = (valid[q] && pos[q] < 0) ? ld_relaxed_u32(d.dir + bucket_of(h[q], d.n_buckets)) : 0u;
+        if (valid && pos < 0) head = ld_dir(d.dir + bkt);
 #endif
         // ---- misses: the chain head entry (header + first 16 key bytes) is fetched now
-        uint4 e_hd[SUB];
-        ulonglong2 e_kw[SUB];
-#pragma unroll
-        for (int q = 0; q < SUB; ++q) {
-            e_hd[q] = make_uint4(0, 0, 0, 0);
-            e_kw[q] = make_ulonglong2(0, 0);
-            if (valid[q] && pos[q] < 0 && head[q]) {
-                const uint8_t* e = ref_ptr(d, head[q]);
-                e_hd[q] = ldcg128(e);
-                e_kw[q] = ldcg128u(e + KEY_OFF);
-            }
+        uint4 e_hd = make_uint4(0, 0, 0, 0);
+        ulonglong2 e_kw = make_ulonglong2(0, 0);
+        if (valid && pos < 0 && head) {
+            const uint8_t* e = ref_ptr(d, head);
+            e_hd = ldcg128(e);
+            e_kw = ldcg128u(e + KEY_OFF);
         }
         // ---- fold the hits of the warp per hot slot (a2): one shared atomic per distinct key
-#pragma unroll
-        for (int q = 0; q < SUB; ++q) {
-            const unsigned hm = __ballot_sync(FULLMASK, pos[q] >= 0);
-            if (!hm) continue;
-            const unsigned key = pos[q] >= 0 ? (unsigned)pos[q] : (0x10000u | lane);
-            const unsigned grp = __match_any_sync(FULLMASK, key) & hm;
-            const uint32_t leader = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
-            if (!VALS) {
-                if (pos[q] >= 0 && lane == leader) atomicAdd(&S.plo[pos[q]], (unsigned int)__popc(grp));
-            } else {
-                uint64_t acc = v[q];
-                if (__any_sync(FULLMASK, __popc(grp) > 1)) {
-                    acc = 0;
-                    for (int x = 0; x < 32; ++x) {
-                        const uint64_t vx = __shfl_sync(FULLMASK, v[q], x);
-                        if ((grp >> x) & 1u) acc += vx;
+        {
+            const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
+            if (hm) {
+#if SEPO_FOLD
+                const unsigned key = pos >= 0 ? (unsigned)pos : (0x10000u | lane);
+                const unsigned grp = __match_any_sync(FULLMASK, key) & hm;
+                const uint32_t leader = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
+                if (!VALS) {
+                    if (pos >= 0 && lane == leader) {
+                        const unsigned add = (unsigned)__popc(grp);
+                        const unsigned old = atomicAdd(&S.plo[pos], add);
+                        if (old + add < old) atomicAdd(&S.phi[pos], 1u);
                     }
+                } else {
+                    uint64_t acc = v;
+                    if (__any_sync(FULLMASK, __popc(grp) > 1)) {
+                        acc = 0;
+                        for (int xl = 0; xl < 32; ++xl) {
+                            const uint64_t vx = __shfl_sync(FULLMASK, v, xl);
+                            if ((grp >> xl) & 1u) acc += vx;
+                        }
+                    }
+                    if (pos >= 0 && lane == leader) smem_add_u64(&S.plo[pos], &S.phi[pos], acc);
                 }
-                if (pos[q] >= 0 && lane == leader) smem_add_u64(&S.plo[pos[q]], &S.phi[pos[q]], acc);
+#else
+                if (pos >= 0) smem_add_u64(&S.plo[pos], &S.phi[pos], v);
+#endif
             }
         }
         // ---- misses: compare the prefetched head entry, then walk the rest of the chain (a3, a4)
-        uint8_t* found[SUB];
-#pragma unroll
-        for (int q = 0; q < SUB; ++q) {
-            found[q] = nullptr;
-            if (valid[q] && pos[q] < 0 && head[q]) {
-                const uint32_t tag = tag_of(h[q]), ln = len[q];
-                const uint8_t* tail = b.keys + s[q] + 16;
-                if (e_hd[q].z == tag && e_hd[q].w == ln && (ln == 0 || e_kw[q].x == w0[q]) && (ln <= 8 || e_kw[q].y == w1[q]) &&
-                    (ln <= 16 || entry_key_eq(ref_ptr(d, head[q]) + KEY_OFF + 16, tail, ln - 16)))
-                    found[q] = ref_ptr(d, head[q]);
-                else
-                    found[q] = chain_find_w(d, e_hd[q].y, 0, tag, ln, w0[q], w1[q], tail);
-                if (found[q]) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found[q], ln)), v[q]);
-            }
+        const uint8_t* tail = b.keys + s + 16;
+        const uint32_t tag = tag_of(h);
+        uint8_t* found = nullptr;
+        if (valid && pos < 0 && head) {
+            if (e_hd.z == tag && e_hd.w == len && (len == 0 || e_kw.x == w0) && (len <= 8 || e_kw.y == w1) &&
+                (len <= 16 || entry_key_eq(ref_ptr(d, head) + KEY_OFF + 16, tail, len - 16)))
+                found = ref_ptr(d, head);
+            else
+                found = chain_find_w(d, e_hd.y, 0, tag, len, w0, w1, tail);
+            if (found) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found, len)), v);
         }
         // ---- new keys: allocate + link (a5, a6), decline (a7)
-#pragma unroll
-        for (int q = 0; q < SUB; ++q) {
-            const uint64_t i = (g0 + q) * 32 + lane;
-            const bool miss = valid[q] && pos[q] < 0;
-            const uint8_t* tail = b.keys + s[q] + 16;
-            const uint32_t bkt = bucket_of(h[q], d.n_buckets);
-            const uint32_t tag = tag_of(h[q]);
-            const uint32_t ln = len[q];
-            const uint64_t vq = v[q];
-            uint32_t hd = head[q];
-            uint32_t res = R_OK;
-            const uint32_t esize = centry_size(ln);
-            bool need = miss && !found[q];
-            if (need && (ln > 65535u - 64u || esize > PB)) { need = false; res = R_TOOLARGE; }
-            if (inj && need && inject_fail(d, h[q], i)) { need = false; res = R_POST; }
-            // Certified declines (R15). Allocation failure is monotone for the generation (`full`).
-            // A warp announces itself in its CTA's announcement word before it may reserve entries
-            // (one RMW; if the word already carries the FULL bit it backs off) and withdraws with a
-            // release-add after linking them. The FULL bit is OR-ed into every word when the pool runs
-            // out, so per word the RMW order decides: an announcement either precedes the bit (and is
-            // counted) or sees it. A declining warp waits (once per launch) until every word shows
-            // FULL with no announcement: every entry reserved before the pool ran out is then linked
-            // and none can follow, so one re-walk of the chain decides the record for good — absorbed
-            // now, or not resident in this generation (the residency guarantee of P:L77/P:L79).
-            const bool any_need = __any_sync(FULLMASK, need);
-            uint64_t off = ~0ull;
-            if (any_need && !w_full) {  // cheap check first: no announcement once the pool is known full
-                unsigned long long f0 = 0;
-                if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
-                if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
-            }
-            if (any_need && !w_full) {
-                unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
-                unsigned long long a = 0;
-                if (lane == 0) a = atomicAdd(my_ann, 1ull);
-                a = __shfl_sync(FULLMASK, a, 0);
-                if (a & ANN_FULL) w_full = true;
-                else off = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
-                if (need && off != ~0ull) {
-                    uint8_t* e = d.pool + off;
-                    *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_COMBINE, hd, tag, ln);
-                    if (ln > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0[q];
-                    if (ln > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1[q];
-                    if (ln > 16) store_key(e + KEY_OFF + 16, tail, ln - 16);
-                    *reinterpret_cast<unsigned long long*>(entry_val(e, ln)) = vq;
-                    const uint32_t me = off_ref(off);
-                    while (true) {  // lock-free head insertion
-                        const uint32_t old = cas_release(d.dir + bkt, hd, me);
-                        if (old == hd) break;
-                        uint8_t* w = chain_find_w(d, old, hd, tag, ln, w0[q], w1[q], tail);
-                        if (w) {  // linked meanwhile by another warp: combine there, retire ours
-                            red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, ln)), vq);
-                            *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
-                            c_dead += esize;
-                            break;
-                        }
-                        hd = old;
-                        *reinterpret_cast<uint32_t*>(e + 4) = hd;
-                    }
-                }
-                __syncwarp();
-                if (lane == 0) add_release64(my_ann, ~0ull);  // withdraw (-1), after every link above
-            }
-            const bool declined = need && off == ~0ull;
-            if (__any_sync(FULLMASK, declined)) {
-                w_full = true;
-                if (!w_quiet) {
-                    if (lane == 0)
-                        for (uint32_t c = 0; c < d.n_slots; ++c)
-                            while (ld_acquire_u64(d.ann + (uint64_t)c * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
-                    __syncwarp();
-                    if (declined) {
-                        uint8_t* w = chain_find_w(d, ld_relaxed_u32(d.dir + bkt), 0, tag, ln, w0[q], w1[q], tail);
-                        if (w) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, ln)), vq);
-                        else res = R_POST;
-                    }
-                    w_quiet = true;
-                } else if (declined) {
-                    res = R_POST;  // walked after quiescence: the miss is final
-                }
-            }
-            // ---- outcome -> bitmap word (a7); key bytes of the declined records (re-issue sizing)
-            const unsigned bits = __ballot_sync(FULLMASK, valid[q] && res != R_OK);
-            if (bits) {
-                const unsigned tl = __ballot_sync(FULLMASK, valid[q] && res == R_TOOLARGE);
-                const unsigned pkb = __reduce_add_sync(FULLMASK, (valid[q] && res != R_OK) ? ln : 0u);
-                if (lane == 0) { c_post += __popc(bits); c_tl += __popc(tl); c_pkb += pkb; }
-            }
-            if (lane == 0 && (g0 + q) < ngroups) b.bitmap[g0 + q] = bits;
+        uint32_t res = R_OK;
+        const uint32_t esize = centry_size(len);
+        bool need = valid && pos < 0 && !found;
+        if (need && (len > 65535u - 64u || esize > PB)) { need = false; res = R_TOOLARGE; }
+        if (inj && need && inject_fail(d, h, i)) { need = false; res = R_POST; }
+        // Certified declines (R15). Allocation failure is monotone for the generation (`full`).
+        // A warp announces itself in its CTA's announcement word before it may reserve entries
+        // (one RMW; if the word already carries the FULL bit it backs off) and withdraws with a
+        // release-add after linking them. The FULL bit is OR-ed into every word when the pool runs
+        // out, so per word the RMW order decides: an announcement either precedes the bit (and is
+        // counted) or sees it. A declining warp waits (once per launch) until every word shows
+        // FULL with no announcement: every entry reserved before the pool ran out is then linked
+        // and none can follow, so one re-walk of the chain decides the record for good — absorbed
+        // now, or not resident in this generation (the residency guarantee of P:L77/P:L79).
+        const bool any_need = __any_sync(FULLMASK, need);
+        uint64_t off = ~0ull;
+        if (any_need && !w_full) {  // cheap check first: no announcement once the pool is known full
+            unsigned long long f0 = 0;
+            if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
+            if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
         }
+        if (any_need && !w_full) {
+            unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
+            unsigned long long a = 0;
+            if (lane == 0) a = atomicAdd(my_ann, 1ull);
+            a = __shfl_sync(FULLMASK, a, 0);
+            if (a & ANN_FULL) w_full = true;
+            else off = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
+            if (need && off != ~0ull) {
+                uint8_t* e = d.pool + off;
+                uint32_t hd = head;
+                *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_COMBINE, hd, tag, len);
+                if (len > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0;
+                if (len > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1;
+                if (len > 16) store_key(e + KEY_OFF + 16, tail, len - 16);
+                *reinterpret_cast<unsigned long long*>(entry_val(e, len)) = v;
+                const uint32_t me = off_ref(off);
+                while (true) {  // lock-free head insertion
+                    const uint32_t old = cas_release(d.dir + bkt, hd, me);
+                    if (old == hd) break;
+                    uint8_t* w = chain_find_w(d, old, hd, tag, len, w0, w1, tail);
+                    if (w) {  // linked meanwhile by another warp: combine there, retire ours
+                        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
+                        *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
+                        atomicAdd(&S.dead, (unsigned long long)esize);
+                        break;
+                    }
+                    hd = old;
+                    *reinterpret_cast<uint32_t*>(e + 4) = hd;
+                }
+            }
+            __syncwarp();
+            if (lane == 0) add_release64(my_ann, ~0ull);  // withdraw (-1), after every link above
+        }
+        const bool declined = need && off == ~0ull;
+        if (__any_sync(FULLMASK, declined)) {
+            w_full = true;
+            if (!w_quiet) {
+                if (lane == 0)
+                    for (uint32_t cs = 0; cs < d.n_slots; ++cs)
+                        while (ld_acquire_u64(d.ann + (uint64_t)cs * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
+                __syncwarp();
+                if (declined) {
+                    uint8_t* w = chain_find_w(d, ld_dir(d.dir + bkt), 0, tag, len, w0, w1, tail);
+                    if (w) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
+                    else res = R_POST;
+                }
+                w_quiet = true;
+            } else if (declined) {
+                res = R_POST;  // walked after quiescence: the miss is final
+            }
+        }
+        // ---- outcome -> bitmap word (a7); key bytes of the declined records (re-issue sizing)
+        const unsigned bits = __ballot_sync(FULLMASK, valid && res != R_OK);
+        if (bits) {
+            const unsigned tl = __ballot_sync(FULLMASK, valid && res == R_TOOLARGE);
+            const unsigned pkb = __reduce_add_sync(FULLMASK, (valid && res != R_OK) ? len : 0u);
+            if (lane == 0) {
+                atomicAdd(&S.post, (unsigned long long)__popc(bits));
+                if (tl) atomicAdd(&S.toolarge, (unsigned long long)__popc(tl));
+                atomicAdd(&S.pkb, (unsigned long long)pkb);
+            }
+        }
+        if (lane == 0) b.bitmap[g] = bits;
+
+        // ---- rotate the pipeline
+        g = gn; gn = gnn;
+        s_c = s_n; v_c = v_n; ch_c = ch_n;
+        s_n = s_nn; v_n = v_nn;
     }
-    if (lane == 0 && (c_post | c_tl)) {
-        if (c_post) atomicAdd(&S.post, c_post);
-        if (c_tl) atomicAdd(&S.toolarge, c_tl);
-        if (c_pkb) atomicAdd(&d.ctrl->kept_key_bytes, c_pkb);
-    }
-    if (c_dead) atomicAdd(&S.dead, c_dead);
     __syncthreads();
     // flush the hot keys' pending sums into their resident entries
     for (int p = tid; p < hot::NH; p += THREADS) {
@@ -638,6 +742,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         if (S.post) atomicAdd(&d.ctrl->postponed, S.post);
         if (S.toolarge) atomicAdd(&d.ctrl->toolarge, S.toolarge);
         if (S.dead) atomicAdd(&d.ctrl->dead_bytes, S.dead);
+        if (S.pkb) atomicAdd(&d.ctrl->kept_key_bytes, S.pkb);
     }
 }
 
@@ -673,15 +778,15 @@ __device__ __forceinline__ void put_value(const Batch& b, uint64_t i, uint8_t* c
     if (b.vo == nullptr) {
         const uint64_t src = rec_index(b, i) * (uint64_t)b.vw;
         uint8_t* dst = c + CHUNK_HDR + (uint64_t)at * b.vw;
-        if (b.vw == 4) *reinterpret_cast<uint32_t*>(dst) = __ldg(reinterpret_cast<const unsigned int*>(b.vals + src));
-        else if (b.vw == 8) *reinterpret_cast<unsigned long long*>(dst) = __ldg(reinterpret_cast<const unsigned long long*>(b.vals + src));
-        else for (uint32_t x = 0; x < b.vw; ++x) dst[x] = __ldg(b.vals + src + x);
+        if (b.vw == 4) *reinterpret_cast<uint32_t*>(dst) = ld_in32(b.vals + src);
+        else if (b.vw == 8) *reinterpret_cast<unsigned long long*>(dst) = ld_in64(b.vals + src);
+        else for (uint32_t x = 0; x < b.vw; ++x) dst[x] = (uint8_t)ld_in8(b.vals + src + x);
     } else {
         uint64_t vs; uint32_t vl;
         rec_val_span(b, i, vs, vl);
         uint8_t* dst = c + CHUNK_HDR + at;
         *reinterpret_cast<uint32_t*>(dst) = vl;
-        for (uint32_t x = 0; x < vl; ++x) dst[4 + x] = __ldg(b.vals + vs + x);
+        for (uint32_t x = 0; x < vl; ++x) dst[4 + x] = (uint8_t)ld_in8(b.vals + vs + x);
     }
 }
 
@@ -701,7 +806,7 @@ __global__ void __launch_bounds__(1024) hot_resolve_group_kernel(Dev d, Batch b,
         uint32_t head = 0;
         uint8_t* found = nullptr;
         if (act) {
-            head = ld_relaxed_u32(d.dir + bkt);
+            head = ld_dir(d.dir + bkt);
             found = chain_find_w(d, head, 0, tag, e.len, e.w0, e.w1, tail);
         }
         const uint32_t esize = gkey_size(e.len);
@@ -817,7 +922,7 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
                 pos = p;
         }
         uint32_t head = 0;
-        if (valid && pos < 0) head = ld_relaxed_u32(d.dir + bkt);
+        if (valid && pos < 0) head = ld_dir(d.dir + bkt);
         // ---- hot keys: reserve the warp's values of a key in its private chunk (one shared atomic)
         bool done = false;
         uint8_t* e = nullptr;  // resident key entry for the global path
@@ -974,7 +1079,7 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
                         while (ld_acquire_u64(d.ann + (uint64_t)c * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
                 __syncwarp();
                 w_quiet = true;
-                if (declined && !e) e = chain_find_w(d, ld_relaxed_u32(d.dir + bkt), 0, tag, len, w0, w1, tail);
+                if (declined && !e) e = chain_find_w(d, ld_dir(d.dir + bkt), 0, tag, len, w0, w1, tail);
             }
             if (declined) {
                 res = R_POST;
@@ -1059,7 +1164,7 @@ __global__ void __launch_bounds__(RP_THREADS) reprobe_kernel(Dev d, Batch b, uns
                 uint32_t want_cap = 0, units = 0;
                 if (mine) {
                     const uint64_t h = hash_key(b.keys + s, len, d.seed);
-                    const uint32_t head = ld_relaxed_u32(d.dir + bucket_of(h, d.n_buckets));
+                    const uint32_t head = ld_dir(d.dir + bucket_of(h, d.n_buckets));
                     e = chain_find(d, head, 0, tag_of(h), len, b.keys + s);
                     if (MODE == 0 && e) {  // resident: combine now
                         atomicAdd(reinterpret_cast<unsigned long long*>(entry_val(e, len)), (unsigned long long)rec_value(b, i));
@@ -1509,7 +1614,7 @@ __global__ void relink_kernel(Dev d) {
                 (void)tag;
                 const uint32_t bkt = bucket_of(h, d.n_buckets);
                 const uint32_t me = off_ref((uint64_t)(e - d.pool));
-                uint32_t head = ld_relaxed_u32(d.dir + bkt);
+                uint32_t head = ld_dir(d.dir + bkt);
                 while (true) {
                     *reinterpret_cast<uint32_t*>(e + 4) = head;
                     const uint32_t old = cas_release(d.dir + bkt, head, me);
@@ -1566,15 +1671,15 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             nh = n_out;
         }
         const size_t sm = sizeof(stream::Smem);
-        constexpr int T = stream::THREADS, SUB = stream::SUB;
+        constexpr int T = stream::THREADS;
         static bool attr = false;
         if (!attr) {
-            cudaFuncSetAttribute(insert_stream_kernel<false, T, SUB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-            cudaFuncSetAttribute(insert_stream_kernel<true, T, SUB>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            cudaFuncSetAttribute(insert_stream_kernel<false, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            cudaFuncSetAttribute(insert_stream_kernel<true, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
             attr = true;
         }
-        if (b.vals) insert_stream_kernel<true, T, SUB><<<grid, T, sm, s>>>(d, b, hl, nh);
-        else insert_stream_kernel<false, T, SUB><<<grid, T, sm, s>>>(d, b, hl, nh);
+        if (b.vals) insert_stream_kernel<true, T><<<grid, T, sm, s>>>(d, b, hl, nh);
+        else insert_stream_kernel<false, T><<<grid, T, sm, s>>>(d, b, hl, nh);
     } else {
         const hot::Entry* hl = nullptr;
         const unsigned int* nh = nullptr;
