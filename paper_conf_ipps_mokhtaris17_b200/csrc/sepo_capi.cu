@@ -167,6 +167,7 @@ int make_batch(sepo_table* t, Batch& b, const uint8_t* keys, const uint64_t* ko,
     b.bitmap = bitmap;
     b.idx = nullptr;
     if (n == 0) return 0;
+    if (n > (1ull << 36)) return fail(SEPO_E_INVAL, "more than 2^36 records in one batch");
     if (!keys && !(ko == nullptr && b.kw == 0)) return fail(SEPO_E_INVAL, "keys is NULL");
     if (!ko && b.kw == 0) return fail(SEPO_E_INVAL, "key_offsets is NULL and fixed_key_width is 0");
     if (t->opts.mode == SEPO_COMBINE_SUM_U64) {

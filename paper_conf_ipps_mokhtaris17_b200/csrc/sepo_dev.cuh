@@ -206,18 +206,29 @@ __device__ __forceinline__ uint64_t fmix64(uint64_t k) {
     k ^= k >> 33; k *= 0xc4ceb9fe1a85ec53ull;
     k ^= k >> 33; return k;
 }
-// h = fmix64(multiply-xor fold over the key's 8-byte LE words (zero padded), seeded with the length)
+// h = fmix64(multiply-xor fold over the key's 8-byte LE words, zero padded, seeded with the length).
+// Every key folds at least two words (w0, w1), so keys of up to 16 bytes hash without branches.
 __device__ __forceinline__ uint64_t hash_init(uint32_t len, uint64_t seed) { return seed ^ ((uint64_t)len * 0x87c37b91114253d5ull); }
 __device__ __forceinline__ uint64_t hash_word(uint64_t h, uint64_t w) {
     return (h ^ w) * 0x9e3779b97f4a7c15ull;  // odd multiplier: a bijection per word
 }
+// hash of a key given its first 16 bytes (w0, w1) and, for longer keys, its bytes at p
+__device__ __forceinline__ uint64_t hash_key16(uint32_t len, uint64_t seed, uint64_t w0, uint64_t w1, const uint8_t* p) {
+#ifdef SEPO_HASH_V5
+    uint64_t x = hash_init(len, seed);
+    if (len > 0) x = hash_word(x, w0);
+    if (len > 8) x = hash_word(x, w1);
+#else
+    uint64_t x = hash_word(hash_word(hash_init(len, seed), w0), w1);
+#endif
+    for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(p + o, len - o < 8 ? len - o : 8));
+    return fmix64(x);
+}
+__device__ __forceinline__ void load_key16(const uint8_t* p, uint32_t len, uint64_t& w0, uint64_t& w1);
 __device__ __forceinline__ uint64_t hash_key(const uint8_t* p, uint32_t len, uint64_t seed) {
-    uint64_t h = hash_init(len, seed);
-    for (uint32_t o = 0; o < len; o += 8) {
-        uint32_t nb = len - o < 8 ? len - o : 8;
-        h = hash_word(h, load_in_word(p + o, nb));
-    }
-    return fmix64(h);
+    uint64_t w0, w1;
+    load_key16(p, len, w0, w1);
+    return hash_key16(len, seed, w0, w1, p);
 }
 __device__ __forceinline__ uint32_t bucket_of(uint64_t h, uint64_t n_buckets) {
     return (uint32_t)(((h >> 32) * n_buckets) >> 32);
@@ -298,13 +309,14 @@ __device__ __forceinline__ uint8_t* chain_find(const Dev& d, uint32_t ref, uint3
 // key are compared against `tail` (the input key + 16).
 __device__ __forceinline__ uint8_t* chain_find_w(const Dev& d, uint32_t ref, uint32_t stop, uint32_t tag, uint32_t len,
                                                  uint64_t w0, uint64_t w1, const uint8_t* tail) {
+    const uint64_t m0 = len ? ~0ull : 0ull, m1 = len > 8 ? ~0ull : 0ull;  // words that hold key bytes
     while (ref != 0 && ref != stop) {
         uint8_t* e = ref_ptr(d, ref);
         const uint4 hd = ldcg128(e);
         const ulonglong2 kw = ldcg128u(e + KEY_OFF);
-        if (hd.z == tag && hd.w == len && (len == 0 || kw.x == w0) && (len <= 8 || kw.y == w1) &&
-            (len <= 16 || entry_key_eq(e + KEY_OFF + 16, tail, len - 16)))
-            return e;
+        bool eq = hd.z == tag && hd.w == len && !((kw.x ^ w0) & m0) && !((kw.y ^ w1) & m1);
+        if (len > 16) eq = eq && entry_key_eq(e + KEY_OFF + 16, tail, len - 16);
+        if (eq) return e;
         ref = hd.y;
     }
     return nullptr;

@@ -14,6 +14,7 @@
 #include "sepo_dev.cuh"
 #include "sepo_kernels.h"
 #include <algorithm>
+#include <type_traits>
 #include <cstring>
 
 namespace sepo {
@@ -160,7 +161,12 @@ struct Entry {                   // one hot key (global list, built by hot_selec
     uint64_t h, w0, w1;
     uint32_t len, ref;           // ref = resident entry (0: not usable)
     uint64_t src;                // input byte offset of a representative record (tail bytes)
+    uint32_t count, pad;         // sample count (placement priority)
 };
+// Keys claim hot slots in rounds of decreasing sample count (log2 classes): when both of a key's
+// buckets are full, the key left out is one of the least frequent ones, never a Zipf head
+// (losing a head key sends a few % of all records to one global address).
+__device__ __forceinline__ int count_class(uint32_t c) { return 31 - __clz(c | 1u); }
 struct SampleSlot { unsigned long long h; unsigned int count, rec; };
 }  // namespace hot
 
@@ -178,11 +184,7 @@ __device__ __forceinline__ void rec_hash16(const Dev& d, const Batch& b, uint64_
     rec_key(b, i, s, len);
     const uint8_t* p = b.keys + s;
     load_key16(p, len, w0, w1);
-    uint64_t x = hash_init(len, d.seed);
-    if (len > 0) x = hash_word(x, w0);
-    if (len > 8) x = hash_word(x, w1);
-    for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(p + o, len - o < 8 ? len - o : 8));
-    h = fmix64(x);
+    h = hash_key16(len, d.seed, w0, w1, p);
 }
 
 // (i-a) count a strided sample of the batch: record i = j * stride
@@ -235,7 +237,7 @@ __global__ void __launch_bounds__(256) hot_emit_kernel(Dev d, Batch b, const hot
                 uint64_t s, w0, w1, h; uint32_t len;
                 rec_hash16(d, b, tab[i].rec, s, len, w0, w1, h);
                 hot::Entry e;
-                e.h = h; e.w0 = w0; e.w1 = w1; e.len = len; e.ref = 0; e.src = s;
+                e.h = h; e.w0 = w0; e.w1 = w1; e.len = len; e.ref = 0; e.src = s; e.count = c; e.pad = 0;
                 out[j] = e;
             }
         }
@@ -313,11 +315,21 @@ namespace stream {
 #endif
 constexpr int THREADS = SEPO_STREAM_THREADS;
 constexpr uint64_t CH = SEPO_CHUNK_GROUPS;
+constexpr int QCAP = 64;          // per-warp miss queue (slots): < 32 waiting + one group's 32
+// Shared memory of the COMBINE stream kernel: the hot set (read-only keys + per-CTA pending sums)
+// and one miss queue per warp (records that missed the hot set, resolved 32 at a time).
+template <bool VALS, int WARPS>
 struct Smem {
     uint4 tags[hot::NB];          // 4 fingerprints per bucket (one 16-B load per probed bucket)
     ulonglong2 kw[hot::NH];       // first 16 key bytes, zero padded (one 16-B load per candidate)
-    uint32_t len[hot::NH], ref[hot::NH];
-    unsigned int plo[hot::NH], phi[hot::NH];  // pending sum = phi:plo (exact via carry)
+    uint32_t ref[hot::NH];        // resident entry (0: empty slot)
+    typename std::conditional<VALS, unsigned long long, unsigned int>::type sum[hot::NH];  // pending sums
+    struct Queue {                // structure of arrays, QCAP slots, ring indexed by a warp counter
+        unsigned long long w0[QCAP], w1[QCAP], h[QCAP], s[QCAP];
+        typename std::conditional<VALS, unsigned long long, unsigned char>::type v[VALS ? QCAP : 1];
+        uint32_t g[QCAP];         // group of the record
+        uint32_t ll[QCAP];        // key length << 5 | lane of the record in its group
+    } q[WARPS];
     unsigned long long cur[2];
     unsigned long long post, toolarge, dead, pkb;
 };
@@ -328,8 +340,8 @@ __device__ __forceinline__ uint32_t fpl(uint64_t h, uint32_t len) {
     return ((uint32_t)(h >> 32) & 0xfffffe00u) | 0x100u | min(len, 255u);
 }
 // A warp streams chunks of CH consecutive groups; chunk c belongs to warp c mod nw.
-__device__ __forceinline__ uint64_t next_group(uint64_t g, uint64_t nw) {
-    return ((g + 1) % CH) ? g + 1 : g + 1 + (nw - 1) * CH;
+__device__ __forceinline__ uint32_t next_group(uint32_t g, uint32_t nw) {
+    return ((g + 1) % (uint32_t)CH) ? g + 1 : g + 1 + (nw - 1) * (uint32_t)CH;
 }
 }  // namespace stream
 
@@ -405,64 +417,73 @@ __device__ __forceinline__ void warp_load_group(const Batch& b, uint64_t g, uint
 //   load at a chunk boundary), first 16 key bytes assembled from the chunks (shuffles + funnel).
 // Indexed batches (re-issue lists) skip the pipeline and load per lane.
 struct InCtx {
-    uint64_t ngroups, nw, kend;  // kend: key bytes end of the batch (ko[n] or n*kw)
+    uint32_t ngroups, nw, tail;  // groups, warps in the grid, records in the last group (1..32)
+    uint64_t kend;               // key bytes end of the batch (ko[n] or n*kw)
 };
+// records in group g (1..32); g < ngroups
+__device__ __forceinline__ uint32_t group_cnt(const InCtx& c, uint32_t g) { return g + 1 == c.ngroups ? c.tail : 32u; }
 template <bool VALS>
-__device__ __forceinline__ void in_stage1(const Batch& b, uint64_t g, uint32_t lane, uint64_t& s, uint64_t& v) {
-    const uint64_t i = g * 32 + lane;
+__device__ __forceinline__ void in_stage1(const Batch& b, const InCtx& c, uint32_t g, uint32_t lane, uint64_t& s,
+                                          uint64_t& v) {
     s = 0;
     v = 1;
-    if (b.idx || i >= b.n) return;
+    if (b.idx || g >= c.ngroups || lane >= group_cnt(c, g)) return;
+    const uint64_t i = (uint64_t)g * 32 + lane;
     if (b.ko) s = ld_in64(b.ko + i);
     if (VALS) v = rec_value(b, i);
 }
-__device__ __forceinline__ uint4 in_stage2(const Batch& b, const InCtx& c, uint64_t g, uint32_t lane, uint64_t s) {
-    uint4 ch = make_uint4(0, 0, 0, 0);
-    if (b.idx || g >= c.ngroups) return ch;
-    const uint64_t cnt = min((uint64_t)32, b.n - g * 32);
+// the group's key-byte window: [base & ~15, min(start of its last record + 16, kend)) — the
+// first 16 bytes of every key; `fast` = contiguous batch and the window fits 32 x 16 B
+__device__ __forceinline__ void in_window(const Batch& b, const InCtx& c, uint32_t g, uint64_t s, uint64_t& base_al,
+                                          uint64_t& wend, bool& fast) {
+    const uint32_t cnt = group_cnt(c, g);
     uint64_t base, last;
     if (b.ko) {
         base = __shfl_sync(FULLMASK, s, 0);
         last = __shfl_sync(FULLMASK, s, (int)cnt - 1);
     } else {
-        base = g * 32 * (uint64_t)b.kw;
-        last = base + (cnt - 1) * b.kw;
+        base = (uint64_t)g * 32 * b.kw;
+        last = base + (uint64_t)(cnt - 1) * b.kw;
     }
-    const uint64_t wend = min(last + 16, c.kend);
-    const uint64_t base_al = base & ~15ull;
-    if (wend - base_al > 512 || (reinterpret_cast<uintptr_t>(b.keys) & 15)) return ch;  // per-lane path
-    if (base_al + 16ull * lane < wend) ch = ld_in128(b.keys + base_al + 16ull * lane);
+    base_al = base & ~15ull;
+    wend = min(last + 16, c.kend);
+    fast = wend - base_al <= 512 && !(reinterpret_cast<uintptr_t>(b.keys) & 15);
+}
+__device__ __forceinline__ uint4 in_stage2(const Batch& b, const InCtx& c, uint32_t g, uint32_t lane, uint64_t s) {
+    uint4 ch = make_uint4(0, 0, 0, 0);
+    if (b.idx || g >= c.ngroups) return ch;
+    uint64_t base_al, wend;
+    bool fast;
+    in_window(b, c, g, s, base_al, wend, fast);
+    if (fast && base_al + 16ull * lane < wend) ch = ld_in128(b.keys + base_al + 16ull * lane);
     return ch;
 }
-// stage 3: s (in: start from stage 1; out: start), len, first 16 key bytes
-__device__ __forceinline__ void in_stage3(const Batch& b, const InCtx& c, uint64_t g, uint64_t gn, uint32_t lane,
-                                          uint64_t s_next, uint4 ch, uint64_t& s, uint32_t& len, uint64_t& w0,
-                                          uint64_t& w1) {
-    const uint64_t i = g * 32 + lane;
-    const bool valid = i < b.n;
+// stage 3: s (in: start from stage 1; out: start), len, first 16 key bytes (zero padded)
+__device__ __forceinline__ void in_stage3(const Batch& b, const InCtx& c, uint32_t g, uint32_t gn, uint32_t lane,
+                                          bool valid, uint64_t s_next, uint4 ch, uint64_t& s, uint32_t& len,
+                                          uint64_t& w0, uint64_t& w1) {
     w0 = 0; w1 = 0; len = 0;
     if (b.idx) {
         s = 0;
-        if (valid) { rec_key(b, i, s, len); load_key16(b.keys + s, len, w0, w1); }
+        if (valid) { rec_key(b, (uint64_t)g * 32 + lane, s, len); load_key16(b.keys + s, len, w0, w1); }
         return;
     }
-    const uint64_t cnt = min((uint64_t)32, b.n - g * 32);
     uint64_t e;
     if (b.ko) {
         e = __shfl_down_sync(FULLMASK, s, 1);
         const uint64_t first_next = __shfl_sync(FULLMASK, s_next, 0);
-        if (i + 1 == b.n) e = c.kend;
-        else if (lane == 31 && valid) e = (gn == g + 1) ? first_next : ld_in64(b.ko + i + 1);
+        const uint32_t cnt = group_cnt(c, g);
+        if (lane + 1 == cnt && g + 1 == c.ngroups) e = c.kend;
+        else if (lane == 31) e = (gn == g + 1) ? first_next : ld_in64(b.ko + (uint64_t)g * 32 + 32);
     } else {
-        s = i * (uint64_t)b.kw;
+        s = ((uint64_t)g * 32 + lane) * b.kw;
         e = s + b.kw;
     }
     len = valid ? (uint32_t)(e - s) : 0u;
-    const uint64_t base = b.ko ? __shfl_sync(FULLMASK, s, 0) : g * 32 * (uint64_t)b.kw;
-    const uint64_t last = b.ko ? __shfl_sync(FULLMASK, s, (int)cnt - 1) : base + (cnt - 1) * b.kw;
-    const uint64_t base_al = base & ~15ull;
-    const bool perlane = min(last + 16, c.kend) - base_al > 512 || (reinterpret_cast<uintptr_t>(b.keys) & 15);
-    if (perlane) {  // warp-uniform
+    uint64_t base_al, wend;
+    bool fast;
+    in_window(b, c, g, s, base_al, wend, fast);
+    if (!fast) {  // warp-uniform
         if (valid) load_key16(b.keys + s, len, w0, w1);
         return;
     }
@@ -473,26 +494,160 @@ __device__ __forceinline__ void in_stage3(const Batch& b, const InCtx& c, uint64
     const uint32_t x2 = __shfl_sync(FULLMASK, ch.z, c0), x3 = __shfl_sync(FULLMASK, ch.w, c0);
     const uint32_t y0 = __shfl_sync(FULLMASK, ch.x, c1), y1 = __shfl_sync(FULLMASK, ch.y, c1);
     const uint32_t y2 = __shfl_sync(FULLMASK, ch.z, c1), y3 = __shfl_sync(FULLMASK, ch.w, c1);
-    if (!valid) return;
     const uint64_t X0 = ((uint64_t)x1 << 32) | x0, X1 = ((uint64_t)x3 << 32) | x2;
     const uint64_t Y0 = ((uint64_t)y1 << 32) | y0, Y1 = ((uint64_t)y3 << 32) | y2;
     const uint32_t r = off & 15u, sh = 8u * (r & 7u);
     const uint64_t q0 = r < 8 ? X0 : X1, q1 = r < 8 ? X1 : Y0, q2 = r < 8 ? Y0 : Y1;
-    w0 = sh ? (q0 >> sh) | (q1 << (64 - sh)) : q0;
-    w1 = sh ? (q1 >> sh) | (q2 << (64 - sh)) : q1;
-    if (len == 0) { w0 = 0; w1 = 0; }
-    else if (len < 8) { w0 &= (1ull << (8 * len)) - 1ull; w1 = 0; }
-    else if (len < 16) w1 &= (1ull << (8 * (len - 8))) - 1ull;
+    const uint64_t lo = sh ? (q0 >> sh) | (q1 << (64 - sh)) : q0;
+    const uint64_t hi = sh ? (q1 >> sh) | (q2 << (64 - sh)) : q1;
+    // zero the bytes past the key (len < 16)
+    const uint32_t nb = min(len, 16u);
+    const uint64_t mlo = nb >= 8 ? ~0ull : ((1ull << (8 * nb)) - 1ull);
+    const uint64_t mhi = nb <= 8 ? 0ull : (nb >= 16 ? ~0ull : ((1ull << (8 * (nb - 8))) - 1ull));
+    w0 = lo & mlo;
+    w1 = hi & mhi;
+}
+
+// Resolve up to 32 queued misses (a3..a7), one per lane: directory word, chain head entry
+// (header + first 16 key bytes), rest of the chain; red.add on a match; otherwise allocate + link a
+// new entry, or decline (certified, R15). Declines are OR-ed into their groups' bitmap words (the
+// words were stored as 0 when the groups were streamed, by this warp, before a __syncwarp).
+template <bool VALS, int WARPS>
+__device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, stream::Smem<VALS, WARPS>& S,
+                                               typename stream::Smem<VALS, WARPS>::Queue& Q, uint32_t qhead,
+                                               uint32_t cnt, bool inj, bool& w_full, bool& w_quiet) {
+    const uint32_t lane = lane_id();
+    const bool act = lane < cnt;
+    const uint32_t k = (qhead + lane) & (stream::QCAP - 1);
+    uint64_t w0 = 0, w1 = 0, h = 0, s = 0, v = 1;
+    uint32_t g = 0, len = 0, gl = 0;
+    if (act) {
+        w0 = Q.w0[k]; w1 = Q.w1[k]; h = Q.h[k]; s = Q.s[k];
+        if (VALS) v = Q.v[k];
+        g = Q.g[k];
+        const uint32_t ll = Q.ll[k];
+        len = ll >> 5; gl = ll & 31u;
+    }
+    const uint32_t bkt = bucket_of(h, d.n_buckets);
+    const uint32_t tag = tag_of(h);
+    const uint8_t* tail = b.keys + s + 16;
+    uint32_t head = act ? ld_dir(d.dir + bkt) : 0u;
+    uint8_t* found = nullptr;
+    if (head) {
+        const uint8_t* e = ref_ptr(d, head);
+        const uint4 e_hd = ldcg128(e);
+        const ulonglong2 e_kw = ldcg128u(e + KEY_OFF);
+        // entry key words are zero padded to 8 bytes and followed by the value: a key of at most 8
+        // bytes compares one word, an empty key none
+        const uint64_t m0 = len ? ~0ull : 0ull, m1 = len > 8 ? ~0ull : 0ull;
+        bool eq = e_hd.z == tag && e_hd.w == len && !((e_kw.x ^ w0) & m0) && !((e_kw.y ^ w1) & m1);
+        if (len > 16) eq = eq && entry_key_eq(e + KEY_OFF + 16, tail, len - 16);
+        found = eq ? const_cast<uint8_t*>(e) : chain_find_w(d, e_hd.y, 0, tag, len, w0, w1, tail);
+        if (found) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found, len)), v);
+    }
+    // ---- new keys: allocate + link (a5, a6), decline (a7)
+    uint32_t res = R_OK;
+    const uint32_t esize = centry_size(len);
+    bool need = act && !found;
+    if (need && (len > 65535u - 64u || esize > d.page_bytes)) { need = false; res = R_TOOLARGE; }
+    if (inj && need && inject_fail(d, h, (uint64_t)g * 32 + gl)) { need = false; res = R_POST; }
+    // Certified declines (R15). Allocation failure is monotone for the generation (`full`).
+    // A warp announces itself in its CTA's announcement word before it may reserve entries
+    // (one RMW; if the word already carries the FULL bit it backs off) and withdraws with a
+    // release-add after linking them. The FULL bit is OR-ed into every word when the pool runs
+    // out, so per word the RMW order decides: an announcement either precedes the bit (and is
+    // counted) or sees it. A declining warp waits (once per launch) until every word shows
+    // FULL with no announcement: every entry reserved before the pool ran out is then linked
+    // and none can follow, so one re-walk of the chain decides the record for good — absorbed
+    // now, or not resident in this generation (the residency guarantee of P:L77/P:L79).
+    const bool any_need = __any_sync(FULLMASK, need);
+    uint64_t off = ~0ull;
+    if (any_need && !w_full) {  // cheap check first: no announcement once the pool is known full
+        unsigned long long f0 = 0;
+        if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
+        if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
+    }
+    if (any_need && !w_full) {
+        unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
+        unsigned long long a = 0;
+        if (lane == 0) a = atomicAdd(my_ann, 1ull);
+        a = __shfl_sync(FULLMASK, a, 0);
+        if (a & ANN_FULL) w_full = true;
+        else off = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
+        if (need && off != ~0ull) {
+            uint8_t* e = d.pool + off;
+            uint32_t hd = head;
+            *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_COMBINE, hd, tag, len);
+            if (len > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0;
+            if (len > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1;
+            if (len > 16) store_key(e + KEY_OFF + 16, tail, len - 16);
+            *reinterpret_cast<unsigned long long*>(entry_val(e, len)) = v;
+            const uint32_t me = off_ref(off);
+            while (true) {  // lock-free head insertion
+                const uint32_t old = cas_release(d.dir + bkt, hd, me);
+                if (old == hd) break;
+                uint8_t* w = chain_find_w(d, old, hd, tag, len, w0, w1, tail);
+                if (w) {  // linked meanwhile by another warp: combine there, retire ours
+                    red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
+                    *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
+                    atomicAdd(&S.dead, (unsigned long long)esize);
+                    break;
+                }
+                hd = old;
+                *reinterpret_cast<uint32_t*>(e + 4) = hd;
+            }
+        }
+        __syncwarp();
+        if (lane == 0) add_release64(my_ann, ~0ull);  // withdraw (-1), after every link above
+    }
+    const bool declined = need && off == ~0ull;
+    if (__any_sync(FULLMASK, declined)) {
+        w_full = true;
+        if (!w_quiet) {
+            if (lane == 0)
+                for (uint32_t cs = 0; cs < d.n_slots; ++cs)
+                    while (ld_acquire_u64(d.ann + (uint64_t)cs * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
+            __syncwarp();
+            if (declined) {
+                uint8_t* w = chain_find_w(d, ld_dir(d.dir + bkt), 0, tag, len, w0, w1, tail);
+                if (w) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
+                else res = R_POST;
+            }
+            w_quiet = true;
+        } else if (declined) {
+            res = R_POST;  // walked after quiescence: the miss is final
+        }
+    }
+    // ---- outcomes -> bitmap bits (a7), one atomicOr per group word; counts for the host
+    const bool out = act && res != R_OK;
+    unsigned pend = __ballot_sync(FULLMASK, out);
+    if (pend) {
+        const unsigned tl = __ballot_sync(FULLMASK, act && res == R_TOOLARGE);
+        const unsigned pkb = __reduce_add_sync(FULLMASK, out ? len : 0u);
+        if (lane == 0) {
+            atomicAdd(&S.post, (unsigned long long)__popc(pend));
+            if (tl) atomicAdd(&S.toolarge, (unsigned long long)__popc(tl));
+            atomicAdd(&S.pkb, (unsigned long long)pkb);
+        }
+        while (pend) {  // group by bitmap word (a batch spans a few groups)
+            const uint32_t lg = __shfl_sync(FULLMASK, g, __ffs(pend) - 1);
+            const bool mine = out && g == lg;
+            const unsigned bits = __reduce_or_sync(FULLMASK, mine ? (1u << gl) : 0u);
+            if (lane == (uint32_t)(__ffs(pend) - 1)) atomicOr(b.bitmap + lg, bits);
+            pend &= ~__ballot_sync(FULLMASK, mine);
+        }
+    }
 }
 
 template <bool VALS, int THREADS>
 __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
                                                                    const unsigned int* n_hot) {
+    constexpr int WARPS = THREADS / 32;
+    using SM = stream::Smem<VALS, WARPS>;
     extern __shared__ __align__(16) uint8_t smem_raw[];
-    stream::Smem& S = *reinterpret_cast<stream::Smem*>(smem_raw);
+    SM& S = *reinterpret_cast<SM*>(smem_raw);
     const uint32_t tid = threadIdx.x, lane = lane_id();
-    const uint32_t PB = d.page_bytes;
-    for (int p = tid; p < hot::NH; p += THREADS) { S.len[p] = hot::EMPTY_LEN; S.plo[p] = 0; S.phi[p] = 0; }
+    for (int p = tid; p < hot::NH; p += THREADS) { S.ref[p] = 0; S.sum[p] = 0; }
     for (int p = tid; p < hot::NB; p += THREADS) S.tags[p] = make_uint4(0, 0, 0, 0);
     if (tid == 0) {
         S.cur[0] = d.cursors[2 * blockIdx.x];
@@ -502,239 +657,134 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     __syncthreads();
     // load the hot set (read-only during the main loop)
     const unsigned nh = hl ? *n_hot : 0u;
-    for (unsigned j = tid; j < nh; j += THREADS) {
-        const hot::Entry e = hl[j];
-        if (e.ref == 0) continue;
-        // claim a free slot in bucket b1, else b2, else leave the key out (the set is only a cache)
-        const uint32_t f = stream::fpl(e.h, e.len);
-        int pos = -1;
-        for (int c = 0; c < 2 && pos < 0; ++c) {
-            const uint32_t bk = c == 0 ? hot::b1(e.h) : hot::b2(e.h);
-            uint32_t* t = reinterpret_cast<uint32_t*>(&S.tags[bk]);
-            for (int w = 0; w < 4 && pos < 0; ++w)
-                if (atomicCAS(&t[w], 0u, f) == 0u) pos = (int)(bk * 4 + w);
+    for (int cls = 31; cls >= 0 && nh; --cls) {
+        for (unsigned j = tid; j < nh; j += THREADS) {
+            const hot::Entry e = hl[j];
+            if (e.ref == 0 || hot::count_class(e.count) != cls) continue;
+            // claim a free slot in bucket b1, else b2, else leave the key out (the set is only a cache)
+            const uint32_t f = stream::fpl(e.h, e.len);
+            int pos = -1;
+            for (int c = 0; c < 2 && pos < 0; ++c) {
+                const uint32_t bk = c == 0 ? hot::b1(e.h) : hot::b2(e.h);
+                uint32_t* t = reinterpret_cast<uint32_t*>(&S.tags[bk]);
+                for (int w = 0; w < 4 && pos < 0; ++w)
+                    if (atomicCAS(&t[w], 0u, f) == 0u) pos = (int)(bk * 4 + w);
+            }
+            if (pos < 0) continue;
+            S.kw[pos] = make_ulonglong2(e.w0, e.w1); S.ref[pos] = e.ref;
         }
-        if (pos < 0) continue;
-        S.kw[pos] = make_ulonglong2(e.w0, e.w1); S.ref[pos] = e.ref; S.len[pos] = e.len;
+        __syncthreads();
     }
     __syncthreads();
     const bool have_hot = nh > 0;
     const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
+    typename SM::Queue& Q = S.q[tid >> 5];
+    uint32_t qhead = 0, qtail = 0;  // warp-uniform ring counters
 
     InCtx c;
-    c.ngroups = (b.n + 31) / 32;
-    c.nw = (uint64_t)gridDim.x * (THREADS / 32);
+    c.ngroups = (uint32_t)((b.n + 31) / 32);
+    c.tail = (uint32_t)(b.n - (uint64_t)(c.ngroups ? c.ngroups - 1 : 0) * 32);
+    c.nw = gridDim.x * WARPS;
     c.kend = b.idx ? 0ull : (b.ko ? ld_in64(b.ko + b.n) : b.n * (uint64_t)b.kw);
     bool w_full = false, w_quiet = false;  // warp-uniform: pool ran out / quiescence observed
 
     // pipeline prologue: group g (stages 1+2 done), group gn (stage 1 in flight)
-    uint64_t g = ((uint64_t)blockIdx.x * (THREADS / 32) + (tid >> 5)) * stream::CH;
+    uint32_t g = (blockIdx.x * WARPS + (tid >> 5)) * (uint32_t)stream::CH;
     uint64_t s_c = 0, v_c = 1, s_n = 0, v_n = 1;
     uint4 ch_c = make_uint4(0, 0, 0, 0);
-    if (g < c.ngroups) {
-        in_stage1<VALS>(b, g, lane, s_c, v_c);
-        ch_c = in_stage2(b, c, g, lane, s_c);
-    }
-    uint64_t gn = stream::next_group(g, c.nw);
-    if (gn < c.ngroups) in_stage1<VALS>(b, gn, lane, s_n, v_n);
+    in_stage1<VALS>(b, c, g, lane, s_c, v_c);
+    ch_c = in_stage2(b, c, g, lane, s_c);
+    uint32_t gn = stream::next_group(g, c.nw);
+    in_stage1<VALS>(b, c, gn, lane, s_n, v_n);
 
     while (g < c.ngroups) {
         // ---- issue ahead: key chunks of gn, offsets (values) of the group after it
         const uint4 ch_n = in_stage2(b, c, gn, lane, s_n);
-        const uint64_t gnn = stream::next_group(gn, c.nw);
-        uint64_t s_nn = 0, v_nn = 1;
-        if (gnn < c.ngroups) in_stage1<VALS>(b, gnn, lane, s_nn, v_nn);
+        const uint32_t gnn = stream::next_group(gn, c.nw);
+        uint64_t s_nn, v_nn;
+        in_stage1<VALS>(b, c, gnn, lane, s_nn, v_nn);
 
         // ---- group g: key words + hash (a1)
-        const uint64_t i = g * 32 + lane;
-        const bool valid = i < b.n;
+        const bool valid = lane < group_cnt(c, g);
         uint64_t s = s_c, w0, w1;
         uint32_t len;
-        in_stage3(b, c, g, gn, lane, s_n, ch_c, s, len, w0, w1);
-        const uint64_t v = VALS ? (b.idx ? (valid ? rec_value(b, i) : 0ull) : v_c) : 1ull;
-        uint64_t x = hash_init(len, d.seed);
-        if (len > 0) x = hash_word(x, w0);
-        if (len > 8) x = hash_word(x, w1);
-        for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(b.keys + s + o, len - o < 8 ? len - o : 8));
-        const uint64_t h = fmix64(x);
-        const uint32_t bkt = bucket_of(h, d.n_buckets);
-        // ---- directory word, issued before the hot-set probe so its latency overlaps it
-        uint32_t head = 0;
-#if SEPO_DIR_ALL
-        if (valid) head = ld_dir(d.dir + bkt);
-#endif
-        // ---- hot set (a2): two 4-way buckets of fingerprints, then one 16-byte key compare
+        in_stage3(b, c, g, gn, lane, valid, s_n, ch_c, s, len, w0, w1);
+        const uint64_t v = VALS ? (b.idx ? (valid ? rec_value(b, (uint64_t)g * 32 + lane) : 0ull) : v_c) : 1ull;
+        const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
+        // ---- hot set (a2): both 4-way fingerprint buckets, then one 16-byte key compare
         int pos = -1;
-        if (valid && have_hot) {
+        if (have_hot) {
             const uint32_t f = stream::fpl(h, len);
             const uint32_t k1 = hot::b1(h), k2 = hot::b2(h);
-            const uint4 t1 = S.tags[k1];
-            int p = -1;
-            if (t1.x == f) p = 4 * k1; else if (t1.y == f) p = 4 * k1 + 1;
-            else if (t1.z == f) p = 4 * k1 + 2; else if (t1.w == f) p = 4 * k1 + 3;
-            else {
-                const uint4 t2 = S.tags[k2];
-                if (t2.x == f) p = 4 * k2; else if (t2.y == f) p = 4 * k2 + 1;
-                else if (t2.z == f) p = 4 * k2 + 2; else if (t2.w == f) p = 4 * k2 + 3;
+            const uint4 t1 = S.tags[k1], t2 = S.tags[k2];
+            const uint32_t m1 = (t1.x == f) | ((t1.y == f) << 1) | ((t1.z == f) << 2) | ((t1.w == f) << 3);
+            const uint32_t m2 = (t2.x == f) | ((t2.y == f) << 1) | ((t2.z == f) << 2) | ((t2.w == f) << 3);
+            const int p = m1 ? (int)(4 * k1 + __ffs(m1) - 1) : (int)(4 * k2 + __ffs(m2) - 1);
+            if (valid && (m1 | m2)) {
+                const ulonglong2 kk = S.kw[p];
+                bool eq = kk.x == w0 && kk.y == w1;
+                if (len > 16) {  // long key: exact length (the fingerprint saturates at 255) + tail bytes
+                    const uint8_t* e = ref_ptr(d, S.ref[p]);
+                    eq = eq && ldcg32(e + 12) == len && entry_key_eq(e + KEY_OFF + 16, b.keys + s + 16, len - 16);
+                }
+                if (eq) pos = p;
             }
-            if (p >= 0) {
-                const ulonglong2 k = S.kw[p];
-                if (k.x == w0 && k.y == w1 &&
-                    (len <= 16 || ((len < 255 || S.len[p] == len) &&
-                                   entry_key_eq(ref_ptr(d, S.ref[p]) + KEY_OFF + 16, b.keys + s + 16, len - 16))))
-                    pos = p;
-            }
-        }
-#if !SEPO_DIR_ALL
-        if (valid && pos < 0) head = ld_dir(d.dir + bkt);
-#endif
-        // ---- misses: the chain head entry (header + first 16 key bytes) is fetched now
-        uint4 e_hd = make_uint4(0, 0, 0, 0);
-        ulonglong2 e_kw = make_ulonglong2(0, 0);
-        if (valid && pos < 0 && head) {
-            const uint8_t* e = ref_ptr(d, head);
-            e_hd = ldcg128(e);
-            e_kw = ldcg128u(e + KEY_OFF);
         }
         // ---- fold the hits of the warp per hot slot (a2): one shared atomic per distinct key
-        {
-            const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
-            if (hm) {
-#if SEPO_FOLD
-                const unsigned key = pos >= 0 ? (unsigned)pos : (0x10000u | lane);
-                const unsigned grp = __match_any_sync(FULLMASK, key) & hm;
-                const uint32_t leader = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
-                if (!VALS) {
-                    if (pos >= 0 && lane == leader) {
-                        const unsigned add = (unsigned)__popc(grp);
-                        const unsigned old = atomicAdd(&S.plo[pos], add);
-                        if (old + add < old) atomicAdd(&S.phi[pos], 1u);
-                    }
-                } else {
-                    uint64_t acc = v;
-                    if (__any_sync(FULLMASK, __popc(grp) > 1)) {
-                        acc = 0;
-                        for (int xl = 0; xl < 32; ++xl) {
-                            const uint64_t vx = __shfl_sync(FULLMASK, v, xl);
-                            if ((grp >> xl) & 1u) acc += vx;
-                        }
-                    }
-                    if (pos >= 0 && lane == leader) smem_add_u64(&S.plo[pos], &S.phi[pos], acc);
+        const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
+        if (hm) {
+            const unsigned grp = __match_any_sync(FULLMASK, pos >= 0 ? (unsigned)pos : (0x10000u | lane)) & hm;
+            const bool leader = pos >= 0 && lane == (uint32_t)(__ffs(grp) - 1);
+            if (!VALS) {
+                if (leader) {
+                    const unsigned add = (unsigned)__popc(grp);
+                    const unsigned old = atomicAdd(reinterpret_cast<unsigned int*>(&S.sum[pos]), add);
+                    if (old + add < old)  // 2^32 wrap of the CTA-local count: carry into the entry
+                        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(ref_ptr(d, S.ref[pos]), len)), 1ull << 32);
                 }
-#else
-                if (pos >= 0) smem_add_u64(&S.plo[pos], &S.phi[pos], v);
-#endif
+            } else {
+                uint64_t acc = v;
+                if (__any_sync(FULLMASK, __popc(grp) > 1)) {
+                    acc = 0;
+                    for (int xl = 0; xl < 32; ++xl) {
+                        const uint64_t vx = __shfl_sync(FULLMASK, v, xl);
+                        if ((grp >> xl) & 1u) acc += vx;
+                    }
+                }
+                if (leader) atomicAdd(reinterpret_cast<unsigned long long*>(&S.sum[pos]), (unsigned long long)acc);
             }
         }
-        // ---- misses: compare the prefetched head entry, then walk the rest of the chain (a3, a4)
-        const uint8_t* tail = b.keys + s + 16;
-        const uint32_t tag = tag_of(h);
-        uint8_t* found = nullptr;
-        if (valid && pos < 0 && head) {
-            if (e_hd.z == tag && e_hd.w == len && (len == 0 || e_kw.x == w0) && (len <= 8 || e_kw.y == w1) &&
-                (len <= 16 || entry_key_eq(ref_ptr(d, head) + KEY_OFF + 16, tail, len - 16)))
-                found = ref_ptr(d, head);
-            else
-                found = chain_find_w(d, e_hd.y, 0, tag, len, w0, w1, tail);
-            if (found) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found, len)), v);
+        // ---- misses: queue them (resolved 32 at a time); the group's bitmap word starts at 0
+        const bool miss = valid && pos < 0;
+        const unsigned mm = __ballot_sync(FULLMASK, miss);
+        if (lane == 0) b.bitmap[g] = 0u;
+        if (miss) {
+            const uint32_t k = (qtail + __popc(mm & lanemask_lt())) & (stream::QCAP - 1);
+            Q.w0[k] = w0; Q.w1[k] = w1; Q.h[k] = h; Q.s[k] = s;
+            if (VALS) Q.v[k] = v;
+            Q.g[k] = g;
+            Q.ll[k] = (len << 5) | lane;
         }
-        // ---- new keys: allocate + link (a5, a6), decline (a7)
-        uint32_t res = R_OK;
-        const uint32_t esize = centry_size(len);
-        bool need = valid && pos < 0 && !found;
-        if (need && (len > 65535u - 64u || esize > PB)) { need = false; res = R_TOOLARGE; }
-        if (inj && need && inject_fail(d, h, i)) { need = false; res = R_POST; }
-        // Certified declines (R15). Allocation failure is monotone for the generation (`full`).
-        // A warp announces itself in its CTA's announcement word before it may reserve entries
-        // (one RMW; if the word already carries the FULL bit it backs off) and withdraws with a
-        // release-add after linking them. The FULL bit is OR-ed into every word when the pool runs
-        // out, so per word the RMW order decides: an announcement either precedes the bit (and is
-        // counted) or sees it. A declining warp waits (once per launch) until every word shows
-        // FULL with no announcement: every entry reserved before the pool ran out is then linked
-        // and none can follow, so one re-walk of the chain decides the record for good — absorbed
-        // now, or not resident in this generation (the residency guarantee of P:L77/P:L79).
-        const bool any_need = __any_sync(FULLMASK, need);
-        uint64_t off = ~0ull;
-        if (any_need && !w_full) {  // cheap check first: no announcement once the pool is known full
-            unsigned long long f0 = 0;
-            if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
-            if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
-        }
-        if (any_need && !w_full) {
-            unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
-            unsigned long long a = 0;
-            if (lane == 0) a = atomicAdd(my_ann, 1ull);
-            a = __shfl_sync(FULLMASK, a, 0);
-            if (a & ANN_FULL) w_full = true;
-            else off = warp_alloc(d, &S.cur[0], need, esize, (uint8_t)PAGE_ENTRY);
-            if (need && off != ~0ull) {
-                uint8_t* e = d.pool + off;
-                uint32_t hd = head;
-                *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_COMBINE, hd, tag, len);
-                if (len > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0;
-                if (len > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1;
-                if (len > 16) store_key(e + KEY_OFF + 16, tail, len - 16);
-                *reinterpret_cast<unsigned long long*>(entry_val(e, len)) = v;
-                const uint32_t me = off_ref(off);
-                while (true) {  // lock-free head insertion
-                    const uint32_t old = cas_release(d.dir + bkt, hd, me);
-                    if (old == hd) break;
-                    uint8_t* w = chain_find_w(d, old, hd, tag, len, w0, w1, tail);
-                    if (w) {  // linked meanwhile by another warp: combine there, retire ours
-                        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
-                        *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
-                        atomicAdd(&S.dead, (unsigned long long)esize);
-                        break;
-                    }
-                    hd = old;
-                    *reinterpret_cast<uint32_t*>(e + 4) = hd;
-                }
-            }
+        qtail += __popc(mm);
+        __syncwarp();
+        if (qtail - qhead >= 32) {
+            resolve_misses<VALS, WARPS>(d, b, S, Q, qhead, 32, inj, w_full, w_quiet);
+            qhead += 32;
             __syncwarp();
-            if (lane == 0) add_release64(my_ann, ~0ull);  // withdraw (-1), after every link above
         }
-        const bool declined = need && off == ~0ull;
-        if (__any_sync(FULLMASK, declined)) {
-            w_full = true;
-            if (!w_quiet) {
-                if (lane == 0)
-                    for (uint32_t cs = 0; cs < d.n_slots; ++cs)
-                        while (ld_acquire_u64(d.ann + (uint64_t)cs * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
-                __syncwarp();
-                if (declined) {
-                    uint8_t* w = chain_find_w(d, ld_dir(d.dir + bkt), 0, tag, len, w0, w1, tail);
-                    if (w) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
-                    else res = R_POST;
-                }
-                w_quiet = true;
-            } else if (declined) {
-                res = R_POST;  // walked after quiescence: the miss is final
-            }
-        }
-        // ---- outcome -> bitmap word (a7); key bytes of the declined records (re-issue sizing)
-        const unsigned bits = __ballot_sync(FULLMASK, valid && res != R_OK);
-        if (bits) {
-            const unsigned tl = __ballot_sync(FULLMASK, valid && res == R_TOOLARGE);
-            const unsigned pkb = __reduce_add_sync(FULLMASK, (valid && res != R_OK) ? len : 0u);
-            if (lane == 0) {
-                atomicAdd(&S.post, (unsigned long long)__popc(bits));
-                if (tl) atomicAdd(&S.toolarge, (unsigned long long)__popc(tl));
-                atomicAdd(&S.pkb, (unsigned long long)pkb);
-            }
-        }
-        if (lane == 0) b.bitmap[g] = bits;
 
         // ---- rotate the pipeline
         g = gn; gn = gnn;
         s_c = s_n; v_c = v_n; ch_c = ch_n;
         s_n = s_nn; v_n = v_nn;
     }
+    if (qtail != qhead) resolve_misses<VALS, WARPS>(d, b, S, Q, qhead, qtail - qhead, inj, w_full, w_quiet);
     __syncthreads();
     // flush the hot keys' pending sums into their resident entries
     for (int p = tid; p < hot::NH; p += THREADS) {
-        if (S.len[p] == hot::EMPTY_LEN) continue;
-        const uint64_t sum = ((uint64_t)S.phi[p] << 32) | S.plo[p];
-        if (sum) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(ref_ptr(d, S.ref[p]), S.len[p])), sum);
+        if (S.ref[p] == 0 || S.sum[p] == 0) continue;
+        uint8_t* e = ref_ptr(d, S.ref[p]);
+        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(e, ldcg32(e + 12))), (unsigned long long)S.sum[p]);
     }
     if (tid == 0) {
         d.cursors[2 * blockIdx.x] = S.cur[0];
@@ -860,19 +910,22 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
     }
     __syncthreads();
     const unsigned nh = hl ? *n_hot : 0u;
-    for (unsigned j = tid; j < nh; j += THREADS) {
-        const hot::Entry e = hl[j];
-        if (e.ref == 0) continue;
-        const uint32_t f = hot::fp(e.h);
-        int pos = -1;
-        for (int c = 0; c < 2 && pos < 0; ++c) {
-            const uint32_t bk = c == 0 ? b1(e.h) : b2(e.h);
-            uint32_t* t = reinterpret_cast<uint32_t*>(&S.tags[bk]);
-            for (int w = 0; w < 4 && pos < 0; ++w)
-                if (atomicCAS(&t[w], 0u, f) == 0u) pos = (int)(bk * 4 + w);
+    for (int cls = 31; cls >= 0 && nh; --cls) {
+        for (unsigned j = tid; j < nh; j += THREADS) {
+            const hot::Entry e = hl[j];
+            if (e.ref == 0 || hot::count_class(e.count) != cls) continue;
+            const uint32_t f = hot::fp(e.h);
+            int pos = -1;
+            for (int c = 0; c < 2 && pos < 0; ++c) {
+                const uint32_t bk = c == 0 ? b1(e.h) : b2(e.h);
+                uint32_t* t = reinterpret_cast<uint32_t*>(&S.tags[bk]);
+                for (int w = 0; w < 4 && pos < 0; ++w)
+                    if (atomicCAS(&t[w], 0u, f) == 0u) pos = (int)(bk * 4 + w);
+            }
+            if (pos < 0) continue;
+            S.h[pos] = e.h; S.w0[pos] = e.w0; S.w1[pos] = e.w1; S.ref[pos] = e.ref; S.len[pos] = e.len;
         }
-        if (pos < 0) continue;
-        S.h[pos] = e.h; S.w0[pos] = e.w0; S.w1[pos] = e.w1; S.ref[pos] = e.ref; S.len[pos] = e.len;
+        __syncthreads();
     }
     __syncthreads();
     const bool have_hot = nh > 0;
@@ -890,11 +943,7 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
         uint64_t s, w0, w1;
         uint32_t len;
         warp_load_group(b, g, lane, valid, s, len, w0, w1);
-        uint64_t x = hash_init(len, d.seed);
-        if (len > 0) x = hash_word(x, w0);
-        if (len > 8) x = hash_word(x, w1);
-        for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(b.keys + s + o, len - o < 8 ? len - o : 8));
-        const uint64_t h = fmix64(x);
+        const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
         uint32_t units = 0;  // this record's value size in chunk units
         if (valid) {
             uint32_t vlen = vw;
@@ -1670,12 +1719,14 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             hl = list;
             nh = n_out;
         }
-        const size_t sm = sizeof(stream::Smem);
         constexpr int T = stream::THREADS;
+        const size_t sm = b.vals ? sizeof(stream::Smem<true, T / 32>) : sizeof(stream::Smem<false, T / 32>);
         static bool attr = false;
         if (!attr) {
-            cudaFuncSetAttribute(insert_stream_kernel<false, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
-            cudaFuncSetAttribute(insert_stream_kernel<true, T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sm);
+            cudaFuncSetAttribute(insert_stream_kernel<false, T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)sizeof(stream::Smem<false, T / 32>));
+            cudaFuncSetAttribute(insert_stream_kernel<true, T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)sizeof(stream::Smem<true, T / 32>));
             attr = true;
         }
         if (b.vals) insert_stream_kernel<true, T><<<grid, T, sm, s>>>(d, b, hl, nh);
