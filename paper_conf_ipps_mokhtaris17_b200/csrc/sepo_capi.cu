@@ -7,6 +7,7 @@
 // sequences kernels, copies pages and parses page images into the exported arrays.
 #include <cuda_runtime.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -76,6 +77,7 @@ struct DevBuf {
 
 enum State { ST_ACTIVE = 0, ST_EXPORTED = 1, ST_BROKEN = 2 };
 const size_t kMaxGrid = 1024;  // cursor slots reserved in the budget region
+const uint64_t kPrepChunk = 256;  // = PREP_CHUNK (sepo_kernels.cu): prepared slots a warp reserves at once
 }  // namespace
 
 struct sepo_table {
@@ -109,6 +111,8 @@ struct sepo_table {
     DevBuf in_stage[4];
     DevBuf hot;  // hot-set discovery scratch (COMBINE)
     DevBuf idxb[2];  // sepo_run re-issue index lists (ping-pong)
+    DevBuf prep[2];  // sepo_run COMBINE: prepared re-issue records (ping-pong)
+    DevBuf prep_n;   // their device counters
 
     // export storage
     std::vector<uint8_t> x_keys, x_vals;
@@ -401,6 +405,33 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
         t->st.toolarge += t->h_ctrl->toolarge;
         return fail(SEPO_E_TOOLARGE, std::to_string(t->h_ctrl->toolarge) + " record(s) cannot fit in one page");
     }
+    return (int64_t)t->h_ctrl->postponed;
+}
+
+// A reinsert pass of sepo_run (COMBINE): the prepared records of the previous pass (a9).
+static int64_t reinsert_impl(sepo_table* t, const Batch& b, uint64_t key_bytes, uint64_t records) {
+    int rc;
+    if (b.n == 0) return 0;
+    t->inserted = true;
+    t->dirty = true;
+    ++t->batch_seq;
+    sync_dev(t);
+    if ((rc = zero_ctrl_counters(t))) return rc;
+    CK(t, cudaEventRecord(t->ev0, t->stream));
+    rc = sepo_launch_reinsert(t->d, b, t->grid, t->stream);
+    if (rc) return cuda_check(t, (cudaError_t)rc, "reinsert kernel launch");
+    CK(t, cudaEventRecord(t->ev1, t->stream));
+    t->st.kernel_launches += 1;
+    if ((rc = read_ctrl(t))) return rc;
+    t->last_insert_ms = elapsed_ms(t->ev0, t->ev1);
+    t->st.t_insert_ms += t->last_insert_ms;
+    if (t->st.passes < SEPO_MAX_PASS_STATS) t->st.t_insert_ms_per_pass[t->st.passes] += t->last_insert_ms;
+    t->st.insert_calls++;
+    t->st.records_inserted += records;
+    t->st.key_bytes_inserted += key_bytes;
+    t->st.dead_bytes += t->h_ctrl->dead_bytes;
+    const uint64_t used = std::min<uint64_t>(t->h_ctrl->pool_taken, t->d.n_free) + t->pages_resident_retained;
+    t->st.pages_used_max = std::max<uint64_t>(t->st.pages_used_max, used);
     return (int64_t)t->h_ctrl->postponed;
 }
 
@@ -903,18 +934,76 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
     int side = 0;
     int64_t passes_start = (int64_t)t->st.passes;
     uint64_t prev = ~0ull;
+    // both streaming kernels certify their declines (R15) and mark pending GROUP keys' pages
+    // themselves, so the insert's count is exact — except under record-mode injection
+    const bool combine_exact = !(t->opts.fail_alloc_ppm && t->opts.fail_mode == 1);
+    // COMBINE re-issue in prepared form (a9): the first pass appends each declined record as
+    // {hash, first 16 key bytes, key offset, value, length}; later passes read those records
+    // densely (no gather through an index list, no re-hash). The first pass's list is sized
+    // n/4 (SEPO_PREP_CAP overrides); on overflow the job continues on the index path.
+    const char* no_prep = getenv("SEPO_NO_PREP");
+    bool use_prep = t->opts.mode == SEPO_COMBINE_SUM_U64 && combine_exact && !(no_prep && no_prep[0] == '1') && n > 0;
+    if (use_prep) {
+        uint64_t cap = std::max<uint64_t>(1ull << 16, n / 4);
+        if (const char* pc = getenv("SEPO_PREP_CAP")) cap = strtoull(pc, nullptr, 10);
+        size_t fr = 0, tot = 0;
+        if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) cap = std::min<uint64_t>(cap, fr / 3 / sizeof(PRec));
+        if (t->prep_n.grow(64) || t->prep[0].grow(std::max<uint64_t>(cap, 1) * sizeof(PRec))) {
+            use_prep = false;
+        } else {
+            CK(t, cudaMemsetAsync(t->prep_n.p, 0, 16, t->stream));
+            cur.out = (PRec*)t->prep[0].p;
+            cur.out_n = (unsigned long long*)t->prep_n.p;
+            cur.out_cap = cap;
+        }
+    }
     while (cur.n > 0) {
         if (t->bm.grow(((cur.n + 31) / 32) * 4)) return fail(SEPO_E_NOMEM, "bitmap scratch");
         cur.bitmap = (uint32_t*)t->bm.p;
         int64_t c = insert_impl(t, cur);
         if (c < 0) return c;
         uint64_t kb = t->h_ctrl->kept_key_bytes, vb = 0;
-        // both streaming kernels certify their declines (R15) and mark pending GROUP keys'
-        // pages themselves, so the insert's count is exact — except under record-mode injection
-        const bool combine_exact = !(t->opts.fail_alloc_ppm && t->opts.fail_mode == 1);
         if (c > 0 && !combine_exact) c = reprobe_impl(t, cur, &kb, &vb);
         if (c < 0) return c;
         if (c == 0) break;
+        uint64_t reserved = 0;  // prepared slots the pass reserved (records + closed holes)
+        if (cur.out) {
+            CK(t, cudaMemcpy(&reserved, cur.out_n, 8, cudaMemcpyDeviceToHost));
+        }
+        if (cur.out && reserved <= cur.out_cap) {
+            // prepared re-issue: reinsert passes until nothing is postponed
+            int ps = 0;
+            uint64_t m = (uint64_t)c;
+            const uint64_t slack = (uint64_t)t->grid * 32 * kPrepChunk;  // holes: < one chunk per warp
+            while (m > 0) {
+                const uint64_t pass = t->st.passes;
+                if (pass < SEPO_MAX_PASS_STATS) t->st.postponed_per_pass[pass] += m;
+                const uint64_t ocap = reserved + slack;  // every record may decline again
+                if (t->prep[ps ^ 1].grow(ocap * sizeof(PRec))) return fail(SEPO_E_NOMEM, "prepared re-issue list");
+                int64_t e = evict_impl(t, 1);
+                if (e < 0) return e;
+                Batch pb = cur;
+                pb.keys = cur.keys; pb.ko = nullptr; pb.vals = nullptr; pb.vo = nullptr; pb.idx = nullptr;
+                pb.bitmap = nullptr;
+                pb.prep = (const PRec*)t->prep[ps].p;
+                pb.n = reserved;
+                pb.out = (PRec*)t->prep[ps ^ 1].p;
+                pb.out_n = (unsigned long long*)t->prep_n.p + (ps ^ 1);
+                pb.out_cap = ocap;
+                CK(t, cudaMemsetAsync(pb.out_n, 0, 8, t->stream));
+                const int64_t m2 = reinsert_impl(t, pb, kb, m);
+                if (m2 < 0) return m2;
+                if (t->h_ctrl->toolarge) return fail(SEPO_E_TOOLARGE, "record cannot fit in one page");
+                kb = t->h_ctrl->kept_key_bytes;
+                m = (uint64_t)m2;
+                if (m) CK(t, cudaMemcpy(&reserved, pb.out_n, 8, cudaMemcpyDeviceToHost));
+                if (reserved > ocap) return fail(SEPO_E_STATE, "prepared re-issue list overflow");
+                ps ^= 1;
+                if (t->st.passes - passes_start > 100000) return fail(SEPO_E_STATE, "no progress");
+            }
+            break;
+        }
+        cur.out = nullptr;  // index re-issue from here on
         if (combine_exact) {
             // the insert's count is exact (certified declines, R15): only the per-tile counts
             const uint64_t pass = t->st.passes;
@@ -993,6 +1082,9 @@ void sepo_destroy(sepo_table* t) {
     t->hot.release();
     t->idxb[0].release();
     t->idxb[1].release();
+    t->prep[0].release();
+    t->prep[1].release();
+    t->prep_n.release();
     t->bm.release();
     for (auto& s : t->buf)
         for (auto& b : s) b.release();

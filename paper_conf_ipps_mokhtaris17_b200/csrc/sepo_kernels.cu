@@ -316,6 +316,10 @@ namespace stream {
 constexpr int THREADS = SEPO_STREAM_THREADS;
 constexpr uint64_t CH = SEPO_CHUNK_GROUPS;
 constexpr int QCAP = 64;          // per-warp miss queue (slots): < 32 waiting + one group's 32
+struct CtaState {                 // allocator slot (the CTA's active pages) + per-launch counters
+    unsigned long long cur[2];
+    unsigned long long post, toolarge, dead, pkb;
+};
 // Shared memory of the COMBINE stream kernel: the hot set (read-only keys + per-CTA pending sums)
 // and one miss queue per warp (records that missed the hot set, resolved 32 at a time).
 template <bool VALS, int WARPS>
@@ -330,8 +334,7 @@ struct Smem {
         uint32_t g[QCAP];         // group of the record
         uint32_t ll[QCAP];        // key length << 5 | lane of the record in its group
     } q[WARPS];
-    unsigned long long cur[2];
-    unsigned long long post, toolarge, dead, pkb;
+    CtaState cs;
 };
 // Fingerprint of a hot slot: 23 hash bits, bit 8 always set (0 marks an empty slot) and the key
 // length (saturated at 255) in the low byte, so a fingerprint match also fixes the length of
@@ -508,26 +511,33 @@ __device__ __forceinline__ void in_stage3(const Batch& b, const InCtx& c, uint32
     w1 = hi & mhi;
 }
 
-// Resolve up to 32 queued misses (a3..a7), one per lane: directory word, chain head entry
-// (header + first 16 key bytes), rest of the chain; red.add on a match; otherwise allocate + link a
-// new entry, or decline (certified, R15). Declines are OR-ed into their groups' bitmap words (the
-// words were stored as 0 when the groups were streamed, by this warp, before a __syncwarp).
-template <bool VALS, int WARPS>
-__device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, stream::Smem<VALS, WARPS>& S,
-                                               typename stream::Smem<VALS, WARPS>::Queue& Q, uint32_t qhead,
-                                               uint32_t cnt, bool inj, bool& w_full, bool& w_quiet) {
+// Resolve one record per lane (a3..a7) — a lane with act = false only takes part in the warp
+// collectives: directory word, chain head entry (header + first 16 key bytes), rest of the chain;
+// red.add on a match; otherwise allocate + link a new entry, or decline (certified, R15).
+// Declines are OR-ed into their groups' bitmap words (stored as 0 by this warp when the groups
+// were streamed, before a __syncwarp) and, in sepo_run, appended to the prepared re-issue list.
+// Prepared re-issue list: a warp reserves PREP_CHUNK slots at a time from the global counter (one
+// atomic per chunk, not per batch: a single counter hit by every warp serialises in L2); slots a
+// warp leaves unused are closed with a sentinel length when it finishes (the reinsert pass skips them).
+constexpr uint32_t PREP_CHUNK = 256;
+constexpr uint32_t PREP_HOLE = 0xffffffffu;
+struct PrepCursor {
+    unsigned long long base = 0;  // first slot of the warp's chunk
+    uint32_t used = PREP_CHUNK;   // slots used in it (PREP_CHUNK: no chunk)
+};
+__device__ __forceinline__ void prep_close(const Batch& b, const PrepCursor& pc) {
     const uint32_t lane = lane_id();
-    const bool act = lane < cnt;
-    const uint32_t k = (qhead + lane) & (stream::QCAP - 1);
-    uint64_t w0 = 0, w1 = 0, h = 0, s = 0, v = 1;
-    uint32_t g = 0, len = 0, gl = 0;
-    if (act) {
-        w0 = Q.w0[k]; w1 = Q.w1[k]; h = Q.h[k]; s = Q.s[k];
-        if (VALS) v = Q.v[k];
-        g = Q.g[k];
-        const uint32_t ll = Q.ll[k];
-        len = ll >> 5; gl = ll & 31u;
+    for (uint32_t k = pc.used + lane; k < PREP_CHUNK; k += 32) {
+        const unsigned long long slot = pc.base + k;
+        if (slot < b.out_cap)
+            reinterpret_cast<ulonglong2*>(b.out + slot)[2] = make_ulonglong2(0ull, (unsigned long long)PREP_HOLE);
     }
+}
+
+__device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, stream::CtaState& S, bool act, uint64_t w0,
+                                             uint64_t w1, uint64_t h, uint64_t s, uint64_t v, uint32_t len, uint32_t g,
+                                             uint32_t gl, bool inj, bool& w_full, bool& w_quiet, PrepCursor& pc) {
+    const uint32_t lane = lane_id();
     const uint32_t bkt = bucket_of(h, d.n_buckets);
     const uint32_t tag = tag_of(h);
     const uint8_t* tail = b.keys + s + 16;
@@ -621,6 +631,25 @@ __device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, str
     // ---- outcomes -> bitmap bits (a7), one atomicOr per group word; counts for the host
     const bool out = act && res != R_OK;
     unsigned pend = __ballot_sync(FULLMASK, out);
+    if (pend && b.out) {  // prepared re-issue records (sepo_run), from the warp's reserved chunk
+        const unsigned pm = __ballot_sync(FULLMASK, act && res == R_POST);
+        const uint32_t k = __popc(pm);
+        if (pc.used + k > PREP_CHUNK) {
+            prep_close(b, pc);
+            unsigned long long nb = 0;
+            if (lane == 0) nb = atomicAdd(b.out_n, (unsigned long long)PREP_CHUNK);
+            pc.base = __shfl_sync(FULLMASK, nb, 0);
+            pc.used = 0;
+        }
+        const unsigned long long base = pc.base + pc.used + __popc(pm & lanemask_lt());
+        pc.used += k;
+        if (act && res == R_POST && base < b.out_cap) {
+            ulonglong2* o = reinterpret_cast<ulonglong2*>(b.out + base);
+            o[0] = make_ulonglong2(w0, w1);
+            o[1] = make_ulonglong2(h, s);
+            o[2] = make_ulonglong2(v, (unsigned long long)len);
+        }
+    }
     if (pend) {
         const unsigned tl = __ballot_sync(FULLMASK, act && res == R_TOOLARGE);
         const unsigned pkb = __reduce_add_sync(FULLMASK, out ? len : 0u);
@@ -629,13 +658,71 @@ __device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, str
             if (tl) atomicAdd(&S.toolarge, (unsigned long long)__popc(tl));
             atomicAdd(&S.pkb, (unsigned long long)pkb);
         }
-        while (pend) {  // group by bitmap word (a batch spans a few groups)
+        while (pend && b.bitmap) {  // group by bitmap word (a batch spans a few groups)
             const uint32_t lg = __shfl_sync(FULLMASK, g, __ffs(pend) - 1);
             const bool mine = out && g == lg;
             const unsigned bits = __reduce_or_sync(FULLMASK, mine ? (1u << gl) : 0u);
             if (lane == (uint32_t)(__ffs(pend) - 1)) atomicOr(b.bitmap + lg, bits);
             pend &= ~__ballot_sync(FULLMASK, mine);
         }
+    }
+}
+
+// Resolve up to 32 queued misses of the stream kernel, one per lane.
+template <bool VALS, int WARPS>
+__device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, stream::Smem<VALS, WARPS>& S,
+                                               typename stream::Smem<VALS, WARPS>::Queue& Q, uint32_t qhead,
+                                               uint32_t cnt, bool inj, bool& w_full, bool& w_quiet, PrepCursor& pc) {
+    const uint32_t lane = lane_id();
+    const bool act = lane < cnt;
+    const uint32_t k = (qhead + lane) & (stream::QCAP - 1);
+    uint64_t w0 = 0, w1 = 0, h = 0, s = 0, v = 1;
+    uint32_t g = 0, len = 0, gl = 0;
+    if (act) {
+        w0 = Q.w0[k]; w1 = Q.w1[k]; h = Q.h[k]; s = Q.s[k];
+        if (VALS) v = Q.v[k];
+        g = Q.g[k];
+        const uint32_t ll = Q.ll[k];
+        len = ll >> 5; gl = ll & 31u;
+    }
+    resolve_core(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
+}
+
+// Reinsert pass of sepo_run (a9 re-issue): the prepared records of the previous pass, 32 per warp
+// step, straight into resolve_core (keys of these passes are the Zipf tail: no hot set).
+__global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
+    __shared__ stream::CtaState S;
+    const uint32_t tid = threadIdx.x, lane = lane_id();
+    if (tid == 0) {
+        S.cur[0] = d.cursors[2 * blockIdx.x];
+        S.cur[1] = d.cursors[2 * blockIdx.x + 1];
+        S.post = 0; S.toolarge = 0; S.dead = 0; S.pkb = 0;
+    }
+    __syncthreads();
+    const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
+    bool w_full = false, w_quiet = false;
+    PrepCursor pc;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    for (uint64_t base = ((uint64_t)blockIdx.x * (blockDim.x / 32) + (tid >> 5)) * 32; base < b.n; base += nw * 32) {
+        const uint64_t i = base + lane;
+        ulonglong2 r0 = make_ulonglong2(0, 0), r1 = make_ulonglong2(0, 0), r2 = make_ulonglong2(1, 0);
+        if (i < b.n) {
+            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(b.prep + i);
+            r0 = __ldcs(p); r1 = __ldcs(p + 1); r2 = __ldcs(p + 2);
+        }
+        const bool act = i < b.n && (uint32_t)r2.y != PREP_HOLE;
+        resolve_core(d, b, S, act, r0.x, r0.y, r1.x, r1.y, r2.x, act ? (uint32_t)r2.y : 0u, (uint32_t)(i >> 5),
+                     (uint32_t)(i & 31), inj, w_full, w_quiet, pc);
+    }
+    if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
+    __syncthreads();
+    if (tid == 0) {
+        d.cursors[2 * blockIdx.x] = S.cur[0];
+        d.cursors[2 * blockIdx.x + 1] = S.cur[1];
+        if (S.post) atomicAdd(&d.ctrl->postponed, S.post);
+        if (S.toolarge) atomicAdd(&d.ctrl->toolarge, S.toolarge);
+        if (S.dead) atomicAdd(&d.ctrl->dead_bytes, S.dead);
+        if (S.pkb) atomicAdd(&d.ctrl->kept_key_bytes, S.pkb);
     }
 }
 
@@ -650,9 +737,9 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     for (int p = tid; p < hot::NH; p += THREADS) { S.ref[p] = 0; S.sum[p] = 0; }
     for (int p = tid; p < hot::NB; p += THREADS) S.tags[p] = make_uint4(0, 0, 0, 0);
     if (tid == 0) {
-        S.cur[0] = d.cursors[2 * blockIdx.x];
-        S.cur[1] = d.cursors[2 * blockIdx.x + 1];
-        S.post = 0; S.toolarge = 0; S.dead = 0; S.pkb = 0;
+        S.cs.cur[0] = d.cursors[2 * blockIdx.x];
+        S.cs.cur[1] = d.cursors[2 * blockIdx.x + 1];
+        S.cs.post = 0; S.cs.toolarge = 0; S.cs.dead = 0; S.cs.pkb = 0;
     }
     __syncthreads();
     // load the hot set (read-only during the main loop)
@@ -680,6 +767,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
     typename SM::Queue& Q = S.q[tid >> 5];
     uint32_t qhead = 0, qtail = 0;  // warp-uniform ring counters
+    PrepCursor pc;
 
     InCtx c;
     c.ngroups = (uint32_t)((b.n + 31) / 32);
@@ -768,7 +856,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         qtail += __popc(mm);
         __syncwarp();
         if (qtail - qhead >= 32) {
-            resolve_misses<VALS, WARPS>(d, b, S, Q, qhead, 32, inj, w_full, w_quiet);
+            resolve_misses<VALS, WARPS>(d, b, S, Q, qhead, 32, inj, w_full, w_quiet, pc);
             qhead += 32;
             __syncwarp();
         }
@@ -778,7 +866,8 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         s_c = s_n; v_c = v_n; ch_c = ch_n;
         s_n = s_nn; v_n = v_nn;
     }
-    if (qtail != qhead) resolve_misses<VALS, WARPS>(d, b, S, Q, qhead, qtail - qhead, inj, w_full, w_quiet);
+    if (qtail != qhead) resolve_misses<VALS, WARPS>(d, b, S, Q, qhead, qtail - qhead, inj, w_full, w_quiet, pc);
+    if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
     __syncthreads();
     // flush the hot keys' pending sums into their resident entries
     for (int p = tid; p < hot::NH; p += THREADS) {
@@ -787,12 +876,12 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(e, ldcg32(e + 12))), (unsigned long long)S.sum[p]);
     }
     if (tid == 0) {
-        d.cursors[2 * blockIdx.x] = S.cur[0];
-        d.cursors[2 * blockIdx.x + 1] = S.cur[1];
-        if (S.post) atomicAdd(&d.ctrl->postponed, S.post);
-        if (S.toolarge) atomicAdd(&d.ctrl->toolarge, S.toolarge);
-        if (S.dead) atomicAdd(&d.ctrl->dead_bytes, S.dead);
-        if (S.pkb) atomicAdd(&d.ctrl->kept_key_bytes, S.pkb);
+        d.cursors[2 * blockIdx.x] = S.cs.cur[0];
+        d.cursors[2 * blockIdx.x + 1] = S.cs.cur[1];
+        if (S.cs.post) atomicAdd(&d.ctrl->postponed, S.cs.post);
+        if (S.cs.toolarge) atomicAdd(&d.ctrl->toolarge, S.cs.toolarge);
+        if (S.cs.dead) atomicAdd(&d.ctrl->dead_bytes, S.cs.dead);
+        if (S.cs.pkb) atomicAdd(&d.ctrl->kept_key_bytes, S.cs.pkb);
     }
 }
 
@@ -1760,6 +1849,10 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
         }
         insert_group_stream_kernel<<<grid, gst::THREADS, sm, s>>>(d, b, hl, nh);
     }
+    return cudaGetLastError();
+}
+int sepo_launch_reinsert(const Dev& d, const Batch& b, int grid, cudaStream_t s) {
+    if (b.n) reinsert_kernel<<<grid, 1024, 0, s>>>(d, b);
     return cudaGetLastError();
 }
 size_t sepo_hot_scratch_bytes() {

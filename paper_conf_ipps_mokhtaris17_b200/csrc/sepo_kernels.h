@@ -5,6 +5,14 @@
 #include "sepo_dev.cuh"
 
 namespace sepo {
+// A postponed COMBINE record, re-issued by sepo_run in "prepared" form (a9): its hash, first 16
+// key bytes (zero padded), key offset in the caller's key bytes (tail of keys longer than 16 B),
+// value and key length — the next pass needs neither the input gather nor the hash again.
+struct PRec {
+    uint64_t w0, w1, h, s, v;
+    uint32_t len, pad;
+};
+static_assert(sizeof(PRec) == 48, "PRec layout");
 // One batch of records as passed to sepo_insert_batch / sepo_reprobe / sepo_compact.
 struct Batch {
     const uint8_t* keys;
@@ -16,10 +24,18 @@ struct Batch {
     uint64_t n;
     uint32_t* bitmap;
     const uint64_t* idx;  // nullptr, or: record i of the batch is record idx[i] of keys/ko/vals (re-issue)
+    // COMBINE, sepo_run only: declined records are also appended to out[] (capacity out_cap; the
+    // counter *out_n may exceed it, then the host falls back to the bitmap), and a prepared batch
+    // (prep != nullptr) replaces keys/ko/vals as the input of reinsert passes.
+    PRec* out = nullptr;
+    unsigned long long* out_n = nullptr;
+    uint64_t out_cap = 0;
+    const PRec* prep = nullptr;
 };
 }  // namespace sepo
 
 int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch);
+int sepo_launch_reinsert(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s);
 size_t sepo_hot_scratch_bytes();
 int sepo_default_grid(int mode, int n_sms);
 int sepo_launch_reprobe(const sepo::Dev& d, const sepo::Batch& b, int mode, int probe, int grid,

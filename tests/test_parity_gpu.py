@@ -55,6 +55,28 @@ def test_c1_over_budget(cuda, ratio):
     assert all(post[i] > post[i + 1] for i in range(len(post) - 1)) and post[-1] == 0, post
 
 
+@pytest.mark.parametrize("reissue", ["prepared", "prepared_overflow", "index"])
+def test_reissue_paths(cuda, monkeypatch, reissue):
+    """sepo_run re-issues postponed COMBINE records as prepared records (hash + key prefix +
+    offset), falls back to index lists when the first pass's prepared list overflows, or uses
+    index lists only (SEPO_NO_PREP=1): same result, same per-pass postponement invariants"""
+    if reissue == "prepared_overflow":
+        monkeypatch.setenv("SEPO_PREP_CAP", "1000")
+    if reissue == "index":
+        monkeypatch.setenv("SEPO_NO_PREP", "1")
+    s = gen.config("C3", scale=0.004)  # URLs: keys longer than 16 B take the tail path
+    inp = device_inputs(s)
+    exp = oracle_expected(s)
+    F, P = budget_pages(s, 3, 1 << 14, 16384, inp)
+    got, passes, st = run_job(s, sepo().budget_for(1 << 14, 16384, P), 1 << 14, 16384, inputs=inp, check_dups=True)
+    assert_same(got, exp)
+    assert passes >= 3
+    assert st["cross_gen_dups"] == 0
+    post = st["postponed_per_pass"]
+    assert all(post[i] > post[i + 1] for i in range(len(post) - 1)) and post[-1] == 0, post
+    assert st["records_inserted"] == s.n + sum(post[:-1])
+
+
 @pytest.mark.parametrize("ppm,mode", [(10_000, 0), (500_000, 0), (500_000, 1)])
 def test_fault_injection(cuda, ppm, mode):
     """postponement pattern does not change the result; key-mode failure is monotone per key"""

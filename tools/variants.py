@@ -24,8 +24,11 @@ def build(specs):
 
 def run(jobs, names):
     for name in names:
-        lib = os.path.join(ROOT, "exp", f"lib_{name}.so")
+        # NAME or NAME+VAR=VALUE[+VAR=VALUE]: library exp/lib_NAME.so with extra environment
+        base, *envs = name.split("+")
+        lib = os.path.join(ROOT, "exp", f"lib_{base}.so")
         env = dict(os.environ, SEPO_LIB=lib)
+        env.update(dict(e.split("=", 1) for e in envs))
         for j in jobs:
             parts = j.split(":")
             cmd = [sys.executable, os.path.join(ROOT, "tools", "time_job.py")] + parts
