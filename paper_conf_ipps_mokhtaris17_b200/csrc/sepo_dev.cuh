@@ -52,7 +52,10 @@ struct Ctrl {
     unsigned long long n_free;         // evict: pages in the new free stack
     unsigned long long n_resident;     // evict: pages that stay resident (retained)
     unsigned long long full;           // 1 once the pool ran out this generation: every later allocation fails
-    unsigned long long pad[6];
+    unsigned long long n_safe;         // evict: free pages that need no copy (never used last generation)
+    unsigned int copied;               // evicted pages whose D2H copy finished (written by the copy stream)
+    unsigned int pad0;
+    unsigned long long pad[4];
 };
 
 struct Dev {
@@ -63,6 +66,9 @@ struct Dev {
     uint32_t page_shift;
     uint32_t n_pages;
     uint32_t n_free;          // pages available in `stack` this generation
+    // Eviction overlapped with the next pass (a10): stack[0, n_safe) are pages the last generation
+    // did not use; stack[n_safe + j] is the j-th evicted page, reusable once ctrl->copied > j.
+    uint32_t n_safe;
     uint32_t* stack;
     uint8_t* page_state;
     uint8_t* retain;
@@ -423,6 +429,15 @@ __device__ __forceinline__ uint64_t warp_alloc(const Dev& d, unsigned long long*
                     unsigned long long q = atomicAdd(&d.ctrl->pool_taken, 1ull);
                     unsigned long long nw;
                     if (q < d.n_free) {
+                        if (q >= d.n_safe) {  // an evicted page: wait until its copy to the host is done
+                            const unsigned int need_copied = (unsigned int)(q - d.n_safe) + 1u;
+                            while (true) {
+                                unsigned int cp;
+                                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(cp) : "l"(&d.ctrl->copied) : "memory");
+                                if (cp >= need_copied) break;
+                                __nanosleep(256);
+                            }
+                        }
                         uint32_t np = d.stack[q];
                         d.page_state[np] = page_kind;
                         nw = (unsigned long long)np << 32;

@@ -1700,6 +1700,8 @@ __global__ void __launch_bounds__(1024) classify_kernel(Dev d, int honor_retain)
             if (!keep) d.page_state[p] = 0;
             d.retain[p] = 0;
         }
+        // free pages that need no copy first (stack order), the evicted ones follow in copy order
+        fr = fr && !ev;
         uint32_t ie = ev, ifr = fr;
         for (int o = 1; o < 32; o <<= 1) {
             uint32_t y0 = __shfl_up_sync(FULLMASK, ie, o), y1 = __shfl_up_sync(FULLMASK, ifr, o);
@@ -1723,9 +1725,13 @@ __global__ void __launch_bounds__(1024) classify_kernel(Dev d, int honor_retain)
     __syncthreads();
     if (lane == 0) atomicAdd(&s_res, n_res);
     __syncthreads();
+    // evicted pages go back to the stack behind the safe ones, in evict-list (= copy) order
+    const uint32_t n_ev = s_base[0], n_sf = s_base[1];
+    for (uint32_t j = tid; j < n_ev; j += blockDim.x) d.stack[n_sf + j] = d.evict_list[j];
     if (tid == 0) {
-        d.ctrl->n_evict = s_base[0];
-        d.ctrl->n_free = s_base[1];
+        d.ctrl->n_evict = n_ev;
+        d.ctrl->n_free = n_sf + n_ev;
+        d.ctrl->n_safe = n_sf;
         d.ctrl->n_resident = s_res;
         d.ctrl->pool_taken = 0;
     }

@@ -55,6 +55,21 @@ def test_c1_over_budget(cuda, ratio):
     assert all(post[i] > post[i + 1] for i in range(len(post) - 1)) and post[-1] == 0, post
 
 
+@pytest.mark.parametrize("overlap", ["1", "0"])
+def test_evict_overlap(cuda, monkeypatch, overlap):
+    """eviction copies overlapped with the next pass (SEPO_EVICT_OVERLAP=1: the allocator waits per
+    evicted page) or waited for as a whole (default): identical results, no key in two generations"""
+    monkeypatch.setenv("SEPO_EVICT_OVERLAP", overlap)
+    s = gen.config("C1")
+    inp = device_inputs(s)
+    exp = oracle_expected(s)
+    F, P = budget_pages(s, 4, 1 << 14, 4096, inp)
+    for _ in range(2):  # the second job reuses the table's pages while nothing is in flight
+        got, passes, st = run_job(s, sepo().budget_for(1 << 14, 4096, P), 1 << 14, 4096, inputs=inp, check_dups=True)
+        assert_same(got, exp)
+        assert passes >= 4 and st["cross_gen_dups"] == 0
+
+
 @pytest.mark.parametrize("reissue", ["prepared", "prepared_overflow", "index"])
 def test_reissue_paths(cuda, monkeypatch, reissue):
     """sepo_run re-issues postponed COMBINE records as prepared records (hash + key prefix +
