@@ -43,6 +43,13 @@ def next_pow2(x):
     return p
 
 
+def prev_pow2(x):
+    p = 1
+    while p * 2 <= x:
+        p *= 2
+    return p
+
+
 def peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -110,8 +117,9 @@ class Job:
         if self.ratio <= 1.0:
             nb = self.nb_full
             pages = int(np.ceil(pages_F / self.ratio)) if self.ratio < 1 else pages_F + 8
-        else:
-            nb = max(1 << 16, next_pow2(int(self.distinct / self.ratio)))
+        else:  # directory: the largest power of two <= 2x the keys of one generation (load <= ~1)
+            mult = float(os.environ.get("SEPO_BENCH_NB_MULT", "2"))
+            nb = max(1 << 16, prev_pow2(int(self.distinct * mult / self.ratio)))
             pages = max(8, int((F / self.ratio - 4 * nb) // self.page_bytes))
         return nb, pages, F
 
@@ -225,7 +233,7 @@ def timed_steps(job, t, steps, stream, route_fn=None):
     import torch
     k, o, v = job.inputs()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    ins_ms, launches, recs_ins, kb_ins, vb_ins = 0.0, 0, 0, 0, 0
+    ins_ms, launches, recs_ins, kb_ins, vb_ins, p1_ms = 0.0, 0, 0, 0, 0, 0.0
     torch.cuda.synchronize()
     e0.record(stream)
     for _ in range(steps):
@@ -236,13 +244,15 @@ def timed_steps(job, t, steps, stream, route_fn=None):
         t.run(k, o, v)
         st = t.stats()
         ins_ms += st["t_insert_ms"]
+        p1_ms += st["t_insert_ms_per_pass"][0]
         launches += st["kernel_launches"]
         recs_ins += st["records_inserted"]
         kb_ins += st["key_bytes_inserted"]
         vb_ins += st["val_bytes_inserted"]
     e1.record(stream)
     torch.cuda.synchronize()
-    return e0.elapsed_time(e1), dict(insert_ms=ins_ms, launches=launches, recs=recs_ins, kb=kb_ins, vb=vb_ins, last=st)
+    return e0.elapsed_time(e1), dict(insert_ms=ins_ms, p1_ms=p1_ms, launches=launches, recs=recs_ins, kb=kb_ins, vb=vb_ins,
+                                     last=st)
 
 
 def run_ours(args):
@@ -316,11 +326,13 @@ def run_ours(args):
         value = world * csr * args.steps / (ms / 1e3) / 1e9
         recs_per_s = world * n * args.steps / (ms / 1e3)
 
-    # roofline of the dominant kernel (insert, a1..a7): algorithmic bytes = CSR bytes of every
-    # batch it was handed (key bytes + 8 B offset [+ value bytes]) over its CUDA-event time
+    # roofline of the dominant kernel: the pass-1 insert (insert_stream_kernel, rows a1..a7, plus
+    # its hot-set sampling kernels) handed every record of the step. Algorithmic bytes = the
+    # step's CSR input (key bytes + 8 B offset [+ value bytes] per record) over the
+    # CUDA-event time of that insert call (on the table's stream), summed over the timed steps.
     pk = peaks()
-    alg = info["kb"] + (8 * info["recs"] if k is not None and o is not None else 0) + info["vb"]
-    achieved = alg / (info["insert_ms"] / 1e3) / 1e9
+    alg = job.csr_bytes() if not routed else job.slice_bytes
+    achieved = alg * args.steps / (info["p1_ms"] / 1e3) / 1e9
     traffic, traffic_note = args.traffic, None
     tj = os.path.join(ROOT, "profiles", "r01_traffic.json")
     if traffic is None and os.path.exists(tj) and args.config == "C2" and args.scale == 1.0:
@@ -329,8 +341,10 @@ def run_ours(args):
         traffic_note = (f"dram read+write of one launch ({tr['launch']}); that launch's algorithmic bytes: "
                         f"{tr['alg_bytes']}")
     roof = {"bound": "hbm", "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
-            "frac": achieved / pk["hbm_gbs"], "traffic": traffic, "traffic_note": traffic_note, "kernel": "sepo::insert_stream_kernel (COMBINE) / sepo::insert_kernel<1> (GROUP)",
-            "insert_share_of_step": info["insert_ms"] / ms,
+            "frac": achieved / pk["hbm_gbs"], "traffic": traffic, "traffic_note": traffic_note,
+            "kernel": "sepo::insert_stream_kernel (COMBINE, pass 1) / sepo::insert_group_stream_kernel (GROUP)",
+            "alg_bytes_per_launch": alg, "launch_ms": info["p1_ms"] / args.steps,
+            "share_of_step": info["p1_ms"] / ms, "all_insert_passes_share_of_step": info["insert_ms"] / ms,
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if not pk.get("_fallback") else "fallback 6.65 TB/s"}
 
     # end to end through sepo_run with pinned HOST buffers (H2D + job + host result assembly)

@@ -1006,8 +1006,10 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
     if (use_prep) {
         uint64_t cap = std::max<uint64_t>(1ull << 16, n / 4);
         if (const char* pc = getenv("SEPO_PREP_CAP")) cap = strtoull(pc, nullptr, 10);
-        size_t fr = 0, tot = 0;
-        if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) cap = std::min<uint64_t>(cap, fr / 3 / sizeof(PRec));
+        if ((uint64_t)t->prep[0].cap < cap * sizeof(PRec)) {  // first use / larger input: bound by free memory
+            size_t fr = 0, tot = 0;
+            if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) cap = std::min<uint64_t>(cap, (fr + t->prep[0].cap) / 3 / sizeof(PRec));
+        }
         if (t->prep_n.grow(64) || t->prep[0].grow(std::max<uint64_t>(cap, 1) * sizeof(PRec))) {
             use_prep = false;
         } else {

@@ -215,15 +215,40 @@ __global__ void __launch_bounds__(256) hot_hist_kernel(const hot::SampleSlot* ta
         if (tab[i].h != 0ull && c >= min_count) atomicAdd(&hist[min(c, (unsigned)HOT_HIST - 1)], 1u);
     }
 }
-__global__ void __launch_bounds__(32) hot_threshold_kernel(unsigned int* hist, uint32_t min_count, uint32_t kmax) {
-    if (threadIdx.x != 0) return;
-    unsigned acc = 0, thr = 0xffffffffu;
-    for (int c = HOT_HIST - 1; c >= (int)min_count; --c) {
-        if (acc + hist[c] > kmax) break;
-        acc += hist[c];
-        thr = c;
+// threshold = min { c >= min_count : S(c) <= kmax }, S(c) = keys whose sample count is >= c
+// (a suffix sum over the histogram; one CTA, 4 bins per thread)
+__global__ void __launch_bounds__(1024) hot_threshold_kernel(unsigned int* hist, uint32_t min_count, uint32_t kmax) {
+    __shared__ unsigned int warp_sum[32];
+    __shared__ unsigned int s_thr;
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, warp = tid >> 5;
+    constexpr int PER = HOT_HIST / 1024;
+    // thread t owns bins [HOT_HIST - PER*(t+1), HOT_HIST - PER*t): thread 0 holds the top bins
+    unsigned int v[PER], tot = 0;
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+        const int c = HOT_HIST - 1 - (int)(PER * tid) - k;
+        v[k] = c >= (int)min_count ? hist[c] : 0u;
+        tot += v[k];
     }
-    hist[HOT_HIST] = thr;  // threshold
+    unsigned int incl = tot;  // inclusive prefix over threads (top bins first)
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned int y = __shfl_up_sync(FULLMASK, incl, o);
+        if (lane >= (uint32_t)o) incl += y;
+    }
+    if (lane == 31) warp_sum[warp] = incl;
+    if (tid == 0) s_thr = 0xffffffffu;
+    __syncthreads();
+    unsigned int before = 0;
+    for (uint32_t w = 0; w < warp; ++w) before += warp_sum[w];
+    unsigned int acc = before + incl - tot;  // S of the bin just above this thread's range
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+        const int c = HOT_HIST - 1 - (int)(PER * tid) - k;
+        acc += v[k];
+        if (c >= (int)min_count && acc <= kmax) atomicMin(&s_thr, (unsigned int)c);
+    }
+    __syncthreads();
+    if (tid == 0) hist[HOT_HIST] = s_thr;
 }
 __global__ void __launch_bounds__(256) hot_emit_kernel(Dev d, Batch b, const hot::SampleSlot* tab, const unsigned int* hist,
                                                        hot::Entry* out, unsigned int* n_out, uint32_t kmax) {
@@ -1807,7 +1832,7 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             unsigned int* hist = n_out + 1;
             cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
             hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
-            hot_threshold_kernel<<<1, 32, 0, s>>>(hist, 4u, (uint32_t)hot::K);
+            hot_threshold_kernel<<<1, 1024, 0, s>>>(hist, 4u, (uint32_t)hot::K);
             hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)hot::K);
             hot_clamp_kernel<<<1, 32, 0, s>>>(n_out, (uint32_t)hot::K);
             hot_resolve_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
@@ -1840,7 +1865,7 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
             hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, b.n / n_sample, n_sample, tab);
             hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
-            hot_threshold_kernel<<<1, 32, 0, s>>>(hist, 4u, (uint32_t)gst::K);
+            hot_threshold_kernel<<<1, 1024, 0, s>>>(hist, 4u, (uint32_t)gst::K);
             hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)gst::K);
             hot_clamp_kernel<<<1, 32, 0, s>>>(n_out, (uint32_t)gst::K);
             hot_resolve_group_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
