@@ -9,7 +9,7 @@ rows = list(csv.reader(io.StringIO(out)))
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 src = {}
 for fn in ["paper_conf_ipps_mokhtaris17_b200/csrc/sepo_kernels.cu", "paper_conf_ipps_mokhtaris17_b200/csrc/sepo_dev.cuh"]:
-    src[os.path.basename(fn)] = open(os.path.join(ROOT, fn)).read().split('\n')
+    src[os.path.basename(fn)] = open(os.path.join(os.environ.get("SRC_DIR", ""), os.path.basename(fn)) if os.environ.get("SRC_DIR") else os.path.join(ROOT, fn)).read().split('\n')
 fname = hdr = None
 lines = []
 for r in rows:
