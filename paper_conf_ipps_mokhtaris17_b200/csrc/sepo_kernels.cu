@@ -447,76 +447,76 @@ __device__ __forceinline__ void warp_load_group(const Batch& b, uint64_t g, uint
 struct InCtx {
     uint32_t ngroups, nw, tail;  // groups, warps in the grid, records in the last group (1..32)
     uint64_t kend;               // key bytes end of the batch (ko[n] or n*kw)
+    bool kal;                    // key bytes 16-byte aligned (chunked loads allowed)
 };
+// input forms of a batch (template parameter of the stream kernel): contiguous CSR keys, fixed-
+// width keys, or a re-issue index list into the caller's arrays
+enum { IN_CSR = 0, IN_FIXED = 1, IN_IDX = 2 };
 // records in group g (1..32); g < ngroups
 __device__ __forceinline__ uint32_t group_cnt(const InCtx& c, uint32_t g) { return g + 1 == c.ngroups ? c.tail : 32u; }
-template <bool VALS>
+template <int IN, bool VALS>
 __device__ __forceinline__ void in_stage1(const Batch& b, const InCtx& c, uint32_t g, uint32_t lane, uint64_t& s,
                                           uint64_t& v) {
     s = 0;
     v = 1;
-    if (b.idx || g >= c.ngroups || lane >= group_cnt(c, g)) return;
+    if (IN == IN_IDX || g >= c.ngroups || lane >= group_cnt(c, g)) return;
     const uint64_t i = (uint64_t)g * 32 + lane;
-    if (b.ko) s = ld_in64(b.ko + i);
+    if (IN == IN_CSR) s = ld_in64(b.ko + i);
     if (VALS) v = rec_value(b, i);
 }
-// the group's key-byte window: [base & ~15, min(start of its last record + 16, kend)) — the
-// first 16 bytes of every key; `fast` = contiguous batch and the window fits 32 x 16 B
-__device__ __forceinline__ void in_window(const Batch& b, const InCtx& c, uint32_t g, uint64_t s, uint64_t& base_al,
-                                          uint64_t& wend, bool& fast) {
+// Stage 2: the group's key-byte window [base & ~15, min(start of its last record + 16, kend)) —
+// the first 16 bytes of every key — as 16-B chunks, chunk `lane` per lane. `win` returns the low
+// 32 bits of the aligned window base with bit 0 = the window was loaded (fits 32 x 16 B).
+template <int IN>
+__device__ __forceinline__ uint4 in_stage2(const Batch& b, const InCtx& c, uint32_t g, uint32_t lane, uint64_t s,
+                                           uint32_t& win) {
+    uint4 ch = make_uint4(0, 0, 0, 0);
+    win = 0;
+    if (IN == IN_IDX || g >= c.ngroups) return ch;
     const uint32_t cnt = group_cnt(c, g);
     uint64_t base, last;
-    if (b.ko) {
+    if (IN == IN_CSR) {
         base = __shfl_sync(FULLMASK, s, 0);
         last = __shfl_sync(FULLMASK, s, (int)cnt - 1);
     } else {
         base = (uint64_t)g * 32 * b.kw;
         last = base + (uint64_t)(cnt - 1) * b.kw;
     }
-    base_al = base & ~15ull;
-    wend = min(last + 16, c.kend);
-    fast = wend - base_al <= 512 && !(reinterpret_cast<uintptr_t>(b.keys) & 15);
-}
-__device__ __forceinline__ uint4 in_stage2(const Batch& b, const InCtx& c, uint32_t g, uint32_t lane, uint64_t s) {
-    uint4 ch = make_uint4(0, 0, 0, 0);
-    if (b.idx || g >= c.ngroups) return ch;
-    uint64_t base_al, wend;
-    bool fast;
-    in_window(b, c, g, s, base_al, wend, fast);
+    const uint64_t base_al = base & ~15ull;
+    const uint64_t wend = min(last + 16, c.kend);
+    const bool fast = c.kal && wend - base_al <= 512;
+    win = (uint32_t)base_al | (fast ? 1u : 0u);
     if (fast && base_al + 16ull * lane < wend) ch = ld_in128(b.keys + base_al + 16ull * lane);
     return ch;
 }
-// stage 3: s (in: start from stage 1; out: start), len, first 16 key bytes (zero padded)
+// Stage 3: s (in: start from stage 1; out: start), len, first 16 key bytes (zero padded)
+template <int IN>
 __device__ __forceinline__ void in_stage3(const Batch& b, const InCtx& c, uint32_t g, uint32_t gn, uint32_t lane,
-                                          bool valid, uint64_t s_next, uint4 ch, uint64_t& s, uint32_t& len,
-                                          uint64_t& w0, uint64_t& w1) {
+                                          bool valid, uint64_t s_next, uint4 ch, uint32_t win, uint64_t& s,
+                                          uint32_t& len, uint64_t& w0, uint64_t& w1) {
     w0 = 0; w1 = 0; len = 0;
-    if (b.idx) {
+    if (IN == IN_IDX) {
         s = 0;
         if (valid) { rec_key(b, (uint64_t)g * 32 + lane, s, len); load_key16(b.keys + s, len, w0, w1); }
         return;
     }
-    uint64_t e;
-    if (b.ko) {
-        e = __shfl_down_sync(FULLMASK, s, 1);
-        const uint64_t first_next = __shfl_sync(FULLMASK, s_next, 0);
-        const uint32_t cnt = group_cnt(c, g);
-        if (lane + 1 == cnt && g + 1 == c.ngroups) e = c.kend;
-        else if (lane == 31) e = (gn == g + 1) ? first_next : ld_in64(b.ko + (uint64_t)g * 32 + 32);
+    if (IN == IN_CSR) {
+        // lengths from the low 32 bits of the offsets (a key is shorter than 2^32 bytes)
+        uint32_t e = __shfl_down_sync(FULLMASK, (uint32_t)s, 1);
+        const uint32_t first_next = __shfl_sync(FULLMASK, (uint32_t)s_next, 0);
+        if (g + 1 == c.ngroups && lane + 1 == c.tail) e = (uint32_t)c.kend;
+        else if (lane == 31) e = (gn == g + 1) ? first_next : (uint32_t)ld_in64(b.ko + (uint64_t)g * 32 + 32);
+        len = valid ? e - (uint32_t)s : 0u;
     } else {
         s = ((uint64_t)g * 32 + lane) * b.kw;
-        e = s + b.kw;
+        len = valid ? b.kw : 0u;
     }
-    len = valid ? (uint32_t)(e - s) : 0u;
-    uint64_t base_al, wend;
-    bool fast;
-    in_window(b, c, g, s, base_al, wend, fast);
-    if (!fast) {  // warp-uniform
+    if (!(win & 1u)) {  // warp-uniform: window not loaded (long keys / unaligned key bytes)
         if (valid) load_key16(b.keys + s, len, w0, w1);
         return;
     }
     // every lane takes part in the shuffles (a chunk may sit in a lane past the last record)
-    const uint32_t off = valid ? (uint32_t)(s - base_al) : 0u;
+    const uint32_t off = valid ? (uint32_t)s - (win & ~1u) : 0u;
     const uint32_t c0 = off >> 4, c1 = min(c0 + 1u, 31u);
     const uint32_t x0 = __shfl_sync(FULLMASK, ch.x, c0), x1 = __shfl_sync(FULLMASK, ch.y, c0);
     const uint32_t x2 = __shfl_sync(FULLMASK, ch.z, c0), x3 = __shfl_sync(FULLMASK, ch.w, c0);
@@ -751,7 +751,7 @@ __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
     }
 }
 
-template <bool VALS, int THREADS>
+template <bool VALS, int THREADS, int IN>
 __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
                                                                    const unsigned int* n_hot) {
     constexpr int WARPS = THREADS / 32;
@@ -798,31 +798,33 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     c.ngroups = (uint32_t)((b.n + 31) / 32);
     c.tail = (uint32_t)(b.n - (uint64_t)(c.ngroups ? c.ngroups - 1 : 0) * 32);
     c.nw = gridDim.x * WARPS;
-    c.kend = b.idx ? 0ull : (b.ko ? ld_in64(b.ko + b.n) : b.n * (uint64_t)b.kw);
+    c.kend = IN == IN_IDX ? 0ull : (IN == IN_CSR ? ld_in64(b.ko + b.n) : b.n * (uint64_t)b.kw);
+    c.kal = !(reinterpret_cast<uintptr_t>(b.keys) & 15);
     bool w_full = false, w_quiet = false;  // warp-uniform: pool ran out / quiescence observed
 
     // pipeline prologue: group g (stages 1+2 done), group gn (stage 1 in flight)
     uint32_t g = (blockIdx.x * WARPS + (tid >> 5)) * (uint32_t)stream::CH;
     uint64_t s_c = 0, v_c = 1, s_n = 0, v_n = 1;
-    uint4 ch_c = make_uint4(0, 0, 0, 0);
-    in_stage1<VALS>(b, c, g, lane, s_c, v_c);
-    ch_c = in_stage2(b, c, g, lane, s_c);
+    uint32_t win_c;
+    in_stage1<IN, VALS>(b, c, g, lane, s_c, v_c);
+    uint4 ch_c = in_stage2<IN>(b, c, g, lane, s_c, win_c);
     uint32_t gn = stream::next_group(g, c.nw);
-    in_stage1<VALS>(b, c, gn, lane, s_n, v_n);
+    in_stage1<IN, VALS>(b, c, gn, lane, s_n, v_n);
 
     while (g < c.ngroups) {
         // ---- issue ahead: key chunks of gn, offsets (values) of the group after it
-        const uint4 ch_n = in_stage2(b, c, gn, lane, s_n);
+        uint32_t win_n;
+        const uint4 ch_n = in_stage2<IN>(b, c, gn, lane, s_n, win_n);
         const uint32_t gnn = stream::next_group(gn, c.nw);
         uint64_t s_nn, v_nn;
-        in_stage1<VALS>(b, c, gnn, lane, s_nn, v_nn);
+        in_stage1<IN, VALS>(b, c, gnn, lane, s_nn, v_nn);
 
         // ---- group g: key words + hash (a1)
         const bool valid = lane < group_cnt(c, g);
         uint64_t s = s_c, w0, w1;
         uint32_t len;
-        in_stage3(b, c, g, gn, lane, valid, s_n, ch_c, s, len, w0, w1);
-        const uint64_t v = VALS ? (b.idx ? (valid ? rec_value(b, (uint64_t)g * 32 + lane) : 0ull) : v_c) : 1ull;
+        in_stage3<IN>(b, c, g, gn, lane, valid, s_n, ch_c, win_c, s, len, w0, w1);
+        const uint64_t v = VALS ? (IN == IN_IDX ? (valid ? rec_value(b, (uint64_t)g * 32 + lane) : 0ull) : v_c) : 1ull;
         const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
         // ---- hot set (a2): both 4-way fingerprint buckets, then one 16-byte key compare
         int pos = -1;
@@ -888,7 +890,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
 
         // ---- rotate the pipeline
         g = gn; gn = gnn;
-        s_c = s_n; v_c = v_n; ch_c = ch_n;
+        s_c = s_n; v_c = v_n; ch_c = ch_n; win_c = win_n;
         s_n = s_nn; v_n = v_nn;
     }
     if (qtail != qhead) resolve_misses<VALS, WARPS>(d, b, S, Q, qhead, qtail - qhead, inj, w_full, w_quiet, pc);
@@ -1843,14 +1845,25 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
         const size_t sm = b.vals ? sizeof(stream::Smem<true, T / 32>) : sizeof(stream::Smem<false, T / 32>);
         static bool attr = false;
         if (!attr) {
-            cudaFuncSetAttribute(insert_stream_kernel<false, T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)sizeof(stream::Smem<false, T / 32>));
-            cudaFuncSetAttribute(insert_stream_kernel<true, T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)sizeof(stream::Smem<true, T / 32>));
+            const int s0 = (int)sizeof(stream::Smem<false, T / 32>), s1 = (int)sizeof(stream::Smem<true, T / 32>);
+            cudaFuncSetAttribute(insert_stream_kernel<false, T, IN_CSR>, cudaFuncAttributeMaxDynamicSharedMemorySize, s0);
+            cudaFuncSetAttribute(insert_stream_kernel<false, T, IN_FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, s0);
+            cudaFuncSetAttribute(insert_stream_kernel<false, T, IN_IDX>, cudaFuncAttributeMaxDynamicSharedMemorySize, s0);
+            cudaFuncSetAttribute(insert_stream_kernel<true, T, IN_CSR>, cudaFuncAttributeMaxDynamicSharedMemorySize, s1);
+            cudaFuncSetAttribute(insert_stream_kernel<true, T, IN_FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, s1);
+            cudaFuncSetAttribute(insert_stream_kernel<true, T, IN_IDX>, cudaFuncAttributeMaxDynamicSharedMemorySize, s1);
             attr = true;
         }
-        if (b.vals) insert_stream_kernel<true, T><<<grid, T, sm, s>>>(d, b, hl, nh);
-        else insert_stream_kernel<false, T><<<grid, T, sm, s>>>(d, b, hl, nh);
+        const int in = b.idx ? IN_IDX : (b.ko ? IN_CSR : IN_FIXED);
+        if (b.vals) {
+            if (in == IN_CSR) insert_stream_kernel<true, T, IN_CSR><<<grid, T, sm, s>>>(d, b, hl, nh);
+            else if (in == IN_FIXED) insert_stream_kernel<true, T, IN_FIXED><<<grid, T, sm, s>>>(d, b, hl, nh);
+            else insert_stream_kernel<true, T, IN_IDX><<<grid, T, sm, s>>>(d, b, hl, nh);
+        } else {
+            if (in == IN_CSR) insert_stream_kernel<false, T, IN_CSR><<<grid, T, sm, s>>>(d, b, hl, nh);
+            else if (in == IN_FIXED) insert_stream_kernel<false, T, IN_FIXED><<<grid, T, sm, s>>>(d, b, hl, nh);
+            else insert_stream_kernel<false, T, IN_IDX><<<grid, T, sm, s>>>(d, b, hl, nh);
+        }
     } else {
         const hot::Entry* hl = nullptr;
         const unsigned int* nh = nullptr;
