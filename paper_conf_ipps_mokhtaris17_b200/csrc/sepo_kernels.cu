@@ -338,6 +338,9 @@ namespace stream {
 #ifndef SEPO_FOLD
 #define SEPO_FOLD 1               // fold equal hot keys of a warp before the shared atomic
 #endif
+#ifndef SEPO_DIR_PREFETCH
+#define SEPO_DIR_PREFETCH 0       // L2 prefetch of a queued miss's directory word (in budget -1.5 %, 4x +1.3 %)
+#endif
 constexpr int THREADS = SEPO_STREAM_THREADS;
 constexpr uint64_t CH = SEPO_CHUNK_GROUPS;
 constexpr int QCAP = 64;          // per-warp miss queue (slots): < 32 waiting + one group's 32
@@ -789,6 +792,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     }
     __syncthreads();
     const bool have_hot = nh > 0;
+    const bool big = b.n >= (1ull << 32);
     const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
     typename SM::Queue& Q = S.q[tid >> 5];
     uint32_t qhead = 0, qtail = 0;  // warp-uniform ring counters
@@ -853,9 +857,14 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
             if (!VALS) {
                 if (leader) {
                     const unsigned add = (unsigned)__popc(grp);
-                    const unsigned old = atomicAdd(reinterpret_cast<unsigned int*>(&S.sum[pos]), add);
-                    if (old + add < old)  // 2^32 wrap of the CTA-local count: carry into the entry
-                        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(ref_ptr(d, S.ref[pos]), len)), 1ull << 32);
+                    if (!big) {  // fewer than 2^32 records: a CTA-local count cannot wrap
+                        atomicAdd(reinterpret_cast<unsigned int*>(&S.sum[pos]), add);
+                    } else {
+                        const unsigned old = atomicAdd(reinterpret_cast<unsigned int*>(&S.sum[pos]), add);
+                        if (old + add < old)  // 2^32 wrap of the CTA-local count: carry into the entry
+                            red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(ref_ptr(d, S.ref[pos]), len)),
+                                        1ull << 32);
+                    }
                 }
             } else {
                 uint64_t acc = v;
@@ -874,6 +883,11 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         const unsigned mm = __ballot_sync(FULLMASK, miss);
         if (lane == 0) b.bitmap[g] = 0u;
         if (miss) {
+#if SEPO_DIR_PREFETCH
+            // the directory word is read when the queue is resolved (a few groups later): start
+            // bringing its line into L2 now
+            asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(d.dir + bucket_of(h, d.n_buckets)));
+#endif
             const uint32_t k = (qtail + __popc(mm & lanemask_lt())) & (stream::QCAP - 1);
             Q.w0[k] = w0; Q.w1[k] = w1; Q.h[k] = h; Q.s[k] = s;
             if (VALS) Q.v[k] = v;
