@@ -962,6 +962,7 @@ static bool is_device_ptr(const void* p) {
 
 int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
                  uint64_t n) {
+    trace("run begin", n);
     int rc = check_active(t);
     if (rc) return rc;
     const bool dev = is_device_ptr(keys) && is_device_ptr(ko) && is_device_ptr(vals) && is_device_ptr(vo);
@@ -988,6 +989,7 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
         return sepo_run(t, kdev, ko ? (const uint64_t*)t->in_stage[1].p : nullptr, vdev,
                         vo ? (const uint64_t*)t->in_stage[3].p : nullptr, n);
     }
+    trace("run: inputs on device");
     Batch cur;
     int rc2 = make_batch(t, cur, keys, ko, vals, vo, n, nullptr);
     if (rc2) return rc2;
@@ -1127,6 +1129,7 @@ int sepo_reset(sepo_table* t) {
     t->inserted = false;
     t->batch_seq = 0;
     t->pages_resident_retained = 0;
+    trace("reset: copy stream idle");
     sepo_stats z{};
     z.n_buckets = t->n_buckets;
     z.page_bytes = t->page_bytes;

@@ -338,6 +338,9 @@ namespace stream {
 #ifndef SEPO_FOLD
 #define SEPO_FOLD 1               // fold equal hot keys of a warp before the shared atomic
 #endif
+#ifndef SEPO_IN_PREFETCH
+#define SEPO_IN_PREFETCH 0        // L2 prefetch of the input this many groups ahead (0: off)
+#endif
 #ifndef SEPO_DIR_PREFETCH
 #define SEPO_DIR_PREFETCH 0       // L2 prefetch of a queued miss's directory word (in budget -1.5 %, 4x +1.3 %)
 #endif
@@ -823,6 +826,24 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         uint64_t s_nn, v_nn;
         in_stage1<IN, VALS>(b, c, gnn, lane, s_nn, v_nn);
 
+#if SEPO_IN_PREFETCH
+        // L2 prefetch SEPO_IN_PREFETCH groups further ahead in the warp's chunk: the 2 lines of key
+        // offsets and ~4 lines of key bytes (extrapolated from this group's window)
+        if (IN == IN_CSR && (g % (uint32_t)stream::CH) + SEPO_IN_PREFETCH < (uint32_t)stream::CH &&
+            g + SEPO_IN_PREFETCH < c.ngroups && lane < 6) {
+            const uint32_t gp = g + SEPO_IN_PREFETCH;
+            const uint8_t* a;
+            if (lane < 2) {
+                a = reinterpret_cast<const uint8_t*>(b.ko + (uint64_t)gp * 32) + 128 * lane;
+            } else {
+                const uint64_t base_al = (win_c & ~1u) | (s_c & ~0xffffffffull);
+                const uint64_t span = (uint64_t)(uint32_t)((uint32_t)s_n - (win_c & ~1u));  // this group's bytes
+                a = b.keys + base_al + span * SEPO_IN_PREFETCH + 128 * (lane - 2);
+                if (a >= b.keys + c.kend) a = b.keys;
+            }
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(a));
+        }
+#endif
         // ---- group g: key words + hash (a1)
         const bool valid = lane < group_cnt(c, g);
         uint64_t s = s_c, w0, w1;
