@@ -139,14 +139,50 @@ def make_job(cfg, ratio=4.0, **kw):
 
 # ---------------------------------------------------------------- clocks during the timed region
 class ClockSampler:
+    """SM clock + throttle reasons sampled DURING the timed region: NVML in a thread every 5 ms
+    (a bench step is ~40 ms, far shorter than nvidia-smi's start-up), nvidia-smi -lms as fallback.
+    One sample is taken synchronously at start() so a short region still has one."""
     Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
 
     def __init__(self, gpu_index=0):
         self.rows, self.proc = [], None
         self.gpu = gpu_index
+        self.nv = None
+
+    def _nvml_sample(self):
+        nv, h = self.nv, self.handle
+        sm = nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM)
+        mx = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+        r = nv.nvmlDeviceGetCurrentClocksEventReasons(h)
+        bits = [nv.nvmlClocksEventReasonHwSlowdown, nv.nvmlClocksEventReasonHwThermalSlowdown,
+                nv.nvmlClocksEventReasonSwThermalSlowdown, nv.nvmlClocksEventReasonSwPowerCap]
+        self.rows.append([str(self.gpu), str(sm), str(mx), "", ""] + ["Active" if r & b else "Not Active" for b in bits])
+
+    def _nvml_loop(self):
+        while not self.done.is_set():
+            try:
+                self._nvml_sample()
+            except Exception:
+                pass
+            self.done.wait(0.005)
 
     def start(self):
+        try:
+            import pynvml as nv
+            nv.nvmlInit()
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES", "")
+            idx = int(vis.split(",")[self.gpu]) if vis and vis.split(",")[0].isdigit() else self.gpu
+            self.handle = nv.nvmlDeviceGetHandleByIndex(idx)
+            self.nv = nv
+            self._nvml_sample()
+            self.done = threading.Event()
+            self.th = threading.Thread(target=self._nvml_loop, daemon=True)
+            self.th.start()
+            return
+        except Exception:
+            self.nv = None
         try:
             self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
                                           "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
@@ -160,6 +196,13 @@ class ClockSampler:
             self.rows.append([x.strip() for x in line.split(",")])
 
     def stop(self):
+        if self.nv is not None:
+            self.done.set()
+            self.th.join(timeout=2)
+            try:
+                self._nvml_sample()
+            except Exception:
+                pass
         if self.proc:
             self.proc.terminate()
             try:

@@ -206,6 +206,13 @@ __device__ __forceinline__ uint64_t load_in_word(const uint8_t* p, uint32_t nb) 
     return v;
 }
 
+// x << n with the PTX semantics for n >= 64 (result 0), unlike C++ where it is undefined
+__device__ __forceinline__ uint64_t shl64_clamp(uint64_t x, uint32_t n) {
+    uint64_t r;
+    asm("shl.b64 %0, %1, %2;" : "=l"(r) : "l"(x), "r"(n));
+    return r;
+}
+
 // ---------------------------------------------------------------- key hash (the paper leaves it open)
 __device__ __forceinline__ uint64_t fmix64(uint64_t k) {
     k ^= k >> 33; k *= 0xff51afd7ed558ccdull;

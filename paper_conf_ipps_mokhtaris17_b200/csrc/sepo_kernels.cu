@@ -350,6 +350,7 @@ constexpr int QCAP = 64;          // per-warp miss queue (slots): < 32 waiting +
 struct CtaState {                 // allocator slot (the CTA's active pages) + per-launch counters
     unsigned long long cur[2];
     unsigned long long post, toolarge, dead, pkb;
+    unsigned long long wpost[32], wpkb[32];  // per-warp postponed records / key bytes (lane 0 only, no atomics)
 };
 // Shared memory of the COMBINE stream kernel: the hot set (read-only keys + per-CTA pending sums)
 // and one miss queue per warp (records that missed the hot set, resolved 32 at a time).
@@ -535,11 +536,10 @@ __device__ __forceinline__ void in_stage3(const Batch& b, const InCtx& c, uint32
     const uint64_t lo = sh ? (q0 >> sh) | (q1 << (64 - sh)) : q0;
     const uint64_t hi = sh ? (q1 >> sh) | (q2 << (64 - sh)) : q1;
     // zero the bytes past the key (len < 16)
-    const uint32_t nb = min(len, 16u);
-    const uint64_t mlo = nb >= 8 ? ~0ull : ((1ull << (8 * nb)) - 1ull);
-    const uint64_t mhi = nb <= 8 ? 0ull : (nb >= 16 ? ~0ull : ((1ull << (8 * (nb - 8))) - 1ull));
-    w0 = lo & mlo;
-    w1 = hi & mhi;
+    // (PTX shl clamps the shift count at 64: ~(~0 << 64) = all ones)
+    const uint32_t nb8 = 8u * min(len, 16u);
+    w0 = lo & ~shl64_clamp(~0ull, nb8);
+    w1 = hi & ~shl64_clamp(~0ull, nb8 > 64u ? nb8 - 64u : 0u);
 }
 
 // Resolve one record per lane (a3..a7) — a lane with act = false only takes part in the warp
@@ -684,18 +684,15 @@ __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, strea
     if (pend) {
         const unsigned tl = __ballot_sync(FULLMASK, act && res == R_TOOLARGE);
         const unsigned pkb = __reduce_add_sync(FULLMASK, out ? len : 0u);
-        if (lane == 0) {
-            atomicAdd(&S.post, (unsigned long long)__popc(pend));
+        if (lane == 0) {  // the warp's own counter slots: plain read-modify-write, no shared atomics
+            const uint32_t w = (threadIdx.x >> 5) & 31u;
+            S.wpost[w] += (unsigned long long)__popc(pend);
+            S.wpkb[w] += (unsigned long long)pkb;
             if (tl) atomicAdd(&S.toolarge, (unsigned long long)__popc(tl));
-            atomicAdd(&S.pkb, (unsigned long long)pkb);
         }
-        while (pend && b.bitmap) {  // group by bitmap word (a batch spans a few groups)
-            const uint32_t lg = __shfl_sync(FULLMASK, g, __ffs(pend) - 1);
-            const bool mine = out && g == lg;
-            const unsigned bits = __reduce_or_sync(FULLMASK, mine ? (1u << gl) : 0u);
-            if (lane == (uint32_t)(__ffs(pend) - 1)) atomicOr(b.bitmap + lg, bits);
-            pend &= ~__ballot_sync(FULLMASK, mine);
-        }
+        // one fire-and-forget red.or per postponed record into its group's bitmap word (the
+        // word was stored as 0 when the group was streamed, before a __syncwarp)
+        if (out && b.bitmap) atomicOr(b.bitmap + g, 1u << gl);
     }
 }
 
@@ -729,6 +726,7 @@ __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
         S.cur[1] = d.cursors[2 * blockIdx.x + 1];
         S.post = 0; S.toolarge = 0; S.dead = 0; S.pkb = 0;
     }
+    if (tid < 32) { S.wpost[tid] = 0; S.wpkb[tid] = 0; }
     __syncthreads();
     const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
     bool w_full = false, w_quiet = false;
@@ -750,6 +748,7 @@ __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
     if (tid == 0) {
         d.cursors[2 * blockIdx.x] = S.cur[0];
         d.cursors[2 * blockIdx.x + 1] = S.cur[1];
+        for (uint32_t w = 0; w < blockDim.x / 32; ++w) { S.post += S.wpost[w]; S.pkb += S.wpkb[w]; }
         if (S.post) atomicAdd(&d.ctrl->postponed, S.post);
         if (S.toolarge) atomicAdd(&d.ctrl->toolarge, S.toolarge);
         if (S.dead) atomicAdd(&d.ctrl->dead_bytes, S.dead);
@@ -772,6 +771,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         S.cs.cur[1] = d.cursors[2 * blockIdx.x + 1];
         S.cs.post = 0; S.cs.toolarge = 0; S.cs.dead = 0; S.cs.pkb = 0;
     }
+    if (tid < 32) { S.cs.wpost[tid] = 0; S.cs.wpkb[tid] = 0; }
     __syncthreads();
     // load the hot set (read-only during the main loop)
     const unsigned nh = hl ? *n_hot : 0u;
@@ -940,6 +940,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     if (tid == 0) {
         d.cursors[2 * blockIdx.x] = S.cs.cur[0];
         d.cursors[2 * blockIdx.x + 1] = S.cs.cur[1];
+        for (uint32_t w = 0; w < (uint32_t)WARPS; ++w) { S.cs.post += S.cs.wpost[w]; S.cs.pkb += S.cs.wpkb[w]; }
         if (S.cs.post) atomicAdd(&d.ctrl->postponed, S.cs.post);
         if (S.cs.toolarge) atomicAdd(&d.ctrl->toolarge, S.cs.toolarge);
         if (S.cs.dead) atomicAdd(&d.ctrl->dead_bytes, S.cs.dead);
