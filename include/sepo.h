@@ -111,6 +111,20 @@ typedef struct sepo_stats {
  * Returns NULL on error (sepo_last_error()). */
 sepo_table* sepo_create(size_t device_budget_bytes, uint64_t n_buckets, uint32_t page_bytes);
 
+/* Residency ablations: the same table and kernels with the
+ * page pool placed elsewhere. Directory, control words and page metadata stay in device memory
+ * (the paper's pinned experiment keeps "everything else" on the GPU); `device_budget_bytes`
+ * still fixes the pool size (pool pages as for sepo_create), but only the directory + metadata part
+ * is allocated on the device.
+ *   SEPO_POOL_DEVICE      = sepo_create (the SEPO table: the pool is the device budget)
+ *   SEPO_POOL_HOST_PINNED = pool in pinned host memory mapped into the device address space: every
+ *                           entry read, combine atomic and allocation touches host memory over the link
+ *   SEPO_POOL_MANAGED     = pool in cudaMallocManaged memory: pages migrate on demand (hardware paging);
+ *                           sepo_reset prefetches the pool back to host memory, so every job pays it
+ * Returns NULL on error (sepo_last_error): unknown placement -> INVAL; allocation failure -> NOMEM. */
+enum { SEPO_POOL_DEVICE = 0, SEPO_POOL_HOST_PINNED = 1, SEPO_POOL_MANAGED = 2 };
+sepo_table* sepo_create_placed(size_t device_budget_bytes, uint64_t n_buckets, uint32_t page_bytes, int placement);
+
 /* Budget (bytes) that sepo_create needs so that the pool holds exactly `pool_pages` pages.
  * Pure arithmetic on the host (no CUDA call). */
 size_t sepo_budget_for(uint64_t n_buckets, uint32_t page_bytes, uint64_t pool_pages);

@@ -58,9 +58,10 @@ class SepoError(RuntimeError):
 
 
 E_INVAL, E_NOMEM, E_TOOLARGE, E_CUDA, E_STATE, E_NCCL = -1, -2, -3, -4, -5, -6
+POOL_DEVICE, POOL_HOST_PINNED, POOL_MANAGED = 0, 1, 2  # sepo_create_placed (include/sepo.h)
 
 # every entry point declared in include/sepo.h
-EXPORTS = ["sepo_create", "sepo_configure", "sepo_insert_batch", "sepo_reprobe", "sepo_compact", "sepo_evict",
+EXPORTS = ["sepo_create", "sepo_create_placed", "sepo_configure", "sepo_insert_batch", "sepo_reprobe", "sepo_compact", "sepo_evict",
            "sepo_export", "sepo_run", "sepo_reset", "sepo_stats_get", "sepo_last_insert_ms", "sepo_destroy",
            "sepo_last_error", "sepo_version", "sepo_budget_for", "sepo_partition_scratch", "sepo_partition",
            "sepo_shift_offsets"]
@@ -79,6 +80,7 @@ def lib():
             raise ImportError(f"{LIB_PATH} not built: run `python tools/build.py` (no CPU fallback exists)")
         L = ctypes.CDLL(LIB_PATH)
         L.sepo_create.argtypes = [ctypes.c_size_t, u64, u32]; L.sepo_create.restype = vp
+        L.sepo_create_placed.argtypes = [ctypes.c_size_t, u64, u32, ctypes.c_int]; L.sepo_create_placed.restype = vp
         L.sepo_configure.argtypes = [vp, ctypes.POINTER(Options)]; L.sepo_configure.restype = ctypes.c_int
         L.sepo_insert_batch.argtypes = [vp, vp, vp, vp, vp, u64, vp]; L.sepo_insert_batch.restype = i64
         L.sepo_reprobe.argtypes = [vp, vp, vp, vp, vp, u64, vp, vp, vp]; L.sepo_reprobe.restype = i64
@@ -117,13 +119,16 @@ class Table:
 
     def __init__(self, budget_bytes, n_buckets, page_bytes=65536, mode=COMBINE, fixed_key_width=0,
                  fixed_val_width=0, grid_ctas=0, hash_seed=0, fail_alloc_ppm=0, fail_mode=0, fail_until_pass=0,
-                 check_dups=False, stream=None, host_arena_bytes=0):
+                 check_dups=False, stream=None, host_arena_bytes=0, placement=0):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("paper_conf_ipps_mokhtaris17_b200 needs a CUDA device (no CPU fallback)")
         L = lib()
         self._L = L
-        self.h = L.sepo_create(int(budget_bytes), int(n_buckets), int(page_bytes))
+        if placement == POOL_DEVICE:
+            self.h = L.sepo_create(int(budget_bytes), int(n_buckets), int(page_bytes))
+        else:  # residency ablations (NEXT-1): pool in pinned host / managed memory
+            self.h = L.sepo_create_placed(int(budget_bytes), int(n_buckets), int(page_bytes), int(placement))
         if not self.h:
             raise SepoError(E_NOMEM, L.sepo_last_error().decode())
         if stream is None:

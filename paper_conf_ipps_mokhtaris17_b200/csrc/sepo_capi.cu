@@ -87,6 +87,9 @@ struct sepo_table {
     uint32_t page_bytes = 0, page_shift = 0, n_pages = 0;
     int grid = 0, n_sms = 0;
     uint8_t* region = nullptr;
+    int placement = SEPO_POOL_DEVICE;  // where the page pool lives (residency ablations, NEXT-1)
+    uint8_t* pool_alloc = nullptr;     // non-device pool: the host pinned / managed allocation
+    uint8_t* pool_dev = nullptr;       // its device-visible address
     Dev d{};
     sepo_options opts{};
     cudaStream_t stream = nullptr, copy_stream = nullptr;
@@ -238,6 +241,14 @@ size_t sepo_budget_for(uint64_t n_buckets, uint32_t page_bytes, uint64_t pool_pa
 }
 
 sepo_table* sepo_create(size_t budget, uint64_t n_buckets, uint32_t page_bytes) {
+    return sepo_create_placed(budget, n_buckets, page_bytes, SEPO_POOL_DEVICE);
+}
+
+sepo_table* sepo_create_placed(size_t budget, uint64_t n_buckets, uint32_t page_bytes, int placement) {
+    if (placement != SEPO_POOL_DEVICE && placement != SEPO_POOL_HOST_PINNED && placement != SEPO_POOL_MANAGED) {
+        fail(SEPO_E_INVAL, "unknown pool placement");
+        return nullptr;
+    }
     if (n_buckets == 0 || n_buckets > 0xffffffffull) { fail(SEPO_E_INVAL, "n_buckets must be in [1, 2^32-1]"); return nullptr; }
     if (page_bytes < 4096 || page_bytes > (4u << 20) || (page_bytes & (page_bytes - 1))) {
         fail(SEPO_E_INVAL, "page_bytes must be a power of two in [4 KiB, 4 MiB]");
@@ -273,11 +284,40 @@ sepo_table* sepo_create(size_t budget, uint64_t n_buckets, uint32_t page_bytes) 
         return nullptr;
     }
     t->n_pages = (uint32_t)np;
-    if (cudaMalloc((void**)&t->region, budget) != cudaSuccess) {
+    t->placement = placement;
+    // DEVICE: one allocation of exactly the budget. HOST_PINNED / MANAGED (residency ablations,
+    // P:L263-303): directory, control words and page metadata stay in HBM (the paper keeps "everything
+    // else" on the GPU); only the page pool moves to pinned host memory mapped into the
+    // device address space (every table access crosses the host link) or to managed memory
+    // (pages migrate on demand by the hardware paging mechanism).
+    const size_t meta_end = fixed + al256(np * 4) + 2 * al256(np) + al256(np * 4) + 4 * 256;
+    const size_t dev_bytes = placement == SEPO_POOL_DEVICE ? budget : meta_end;
+    if (cudaMalloc((void**)&t->region, dev_bytes) != cudaSuccess) {
         cudaGetLastError();
         fail(SEPO_E_NOMEM, "cudaMalloc of the device budget failed");
         delete t;
         return nullptr;
+    }
+    uint8_t* pool_base = nullptr;  // non-device pool: page_bytes-aligned start inside t->pool_alloc
+    if (placement != SEPO_POOL_DEVICE) {
+        const size_t pool_bytes = np * (size_t)page_bytes + page_bytes;
+        cudaError_t e;
+        if (placement == SEPO_POOL_HOST_PINNED) {
+            e = cudaHostAlloc((void**)&t->pool_alloc, pool_bytes, cudaHostAllocMapped);
+            uint8_t* dp = nullptr;
+            if (e == cudaSuccess) e = cudaHostGetDevicePointer((void**)&dp, t->pool_alloc, 0);
+            if (e == cudaSuccess) t->pool_dev = dp;
+        } else {
+            e = cudaMallocManaged((void**)&t->pool_alloc, pool_bytes, cudaMemAttachGlobal);
+            t->pool_dev = t->pool_alloc;
+        }
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            fail(SEPO_E_NOMEM, "pool allocation (host pinned / managed) failed");
+            sepo_destroy(t);
+            return nullptr;
+        }
+        pool_base = (uint8_t*)(((uintptr_t)t->pool_dev + page_bytes - 1) & ~(uintptr_t)(page_bytes - 1));
     }
     uint8_t* p = t->region;
     Dev& d = t->d;
@@ -290,7 +330,8 @@ sepo_table* sepo_create(size_t budget, uint64_t n_buckets, uint32_t page_bytes) 
     d.retain = p; p += al(np);
     d.evict_list = (uint32_t*)p; p += al(np * 4);
     uintptr_t pa = ((uintptr_t)p + page_bytes - 1) & ~(uintptr_t)(page_bytes - 1);
-    if (pa + np * (size_t)page_bytes > (uintptr_t)t->region + budget) {
+    if (pool_base) pa = (uintptr_t)pool_base;
+    else if (pa + np * (size_t)page_bytes > (uintptr_t)t->region + budget) {
         // alignment ate a page
         --np;
         t->n_pages = (uint32_t)np;
@@ -612,7 +653,7 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
         for (uint64_t c0 = 0; c0 < cnt; c0 += chunk_pages) {
             const uint64_t cc = std::min<uint64_t>(chunk_pages, cnt - c0);
             CK(t, cudaMemcpyAsync(hp + (c0 << t->page_shift), t->d.pool + ((size_t)(first + c0) << t->page_shift),
-                                  (size_t)cc << t->page_shift, cudaMemcpyDeviceToHost, t->copy_stream));
+                                  (size_t)cc << t->page_shift, cudaMemcpyDefault, t->copy_stream));
             done += cc;
             if (overlapped) {
                 const int wr = t->write_value32(t->copy_stream, (unsigned long long)(uintptr_t)&t->d.ctrl->copied,
@@ -1136,6 +1177,12 @@ int sepo_reset(sepo_table* t) {
     z.pool_pages = t->n_pages;
     z.grid_ctas = t->grid;
     t->st = z;
+    if (t->placement == SEPO_POOL_MANAGED) {
+        // residency ablation: between jobs a managed pool's pages go back to host memory, so every
+        // job pays the hardware demand paging of its table
+        CK(t, cudaMemPrefetchAsync(t->pool_alloc, (size_t)t->n_pages * t->page_bytes + t->page_bytes, cudaCpuDeviceId,
+                                   t->stream));
+    }
     return init_device_state(t);
 }
 
@@ -1167,6 +1214,10 @@ void sepo_destroy(sepo_table* t) {
     if (t->h_evict) cudaFreeHost(t->h_evict);
     if (t->h_ko) cudaFreeHost(t->h_ko);
     if (t->region) cudaFree(t->region);
+    if (t->pool_alloc) {
+        if (t->placement == SEPO_POOL_HOST_PINNED) cudaFreeHost(t->pool_alloc);
+        else cudaFree(t->pool_alloc);
+    }
     if (t->ev0) cudaEventDestroy(t->ev0);
     if (t->ev1) cudaEventDestroy(t->ev1);
     if (t->evc0) cudaEventDestroy(t->evc0);
