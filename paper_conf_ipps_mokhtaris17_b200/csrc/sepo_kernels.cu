@@ -461,14 +461,20 @@ struct InCtx {
 enum { IN_CSR = 0, IN_FIXED = 1, IN_IDX = 2 };
 // records in group g (1..32); g < ngroups
 __device__ __forceinline__ uint32_t group_cnt(const InCtx& c, uint32_t g) { return g + 1 == c.ngroups ? c.tail : 32u; }
+// (CSR: at the last group of a warp's chunk, lane 31 also loads the end of its key — the start of the
+// next group, which this warp does not stream — here, two groups ahead, as the low 32 bits in
+// `eo`; loaded in stage 3 instead it shared a scoreboard with the loads in flight and stalled)
 template <int IN, bool VALS>
 __device__ __forceinline__ void in_stage1(const Batch& b, const InCtx& c, uint32_t g, uint32_t lane, uint64_t& s,
-                                          uint64_t& v) {
+                                          uint64_t& v, uint32_t& eo) {
     s = 0;
     v = 1;
     if (IN == IN_IDX || g >= c.ngroups || lane >= group_cnt(c, g)) return;
     const uint64_t i = (uint64_t)g * 32 + lane;
-    if (IN == IN_CSR) s = ld_in64(b.ko + i);
+    if (IN == IN_CSR) {
+        s = ld_in64(b.ko + i);
+        if (lane == 31 && (g + 1) % (uint32_t)stream::CH == 0) eo = ld_in32(b.ko + i + 1);
+    }
     if (VALS) v = rec_value(b, i);
 }
 // Stage 2: the group's key-byte window [base & ~15, min(start of its last record + 16, kend)) —
@@ -499,7 +505,7 @@ __device__ __forceinline__ uint4 in_stage2(const Batch& b, const InCtx& c, uint3
 // Stage 3: s (in: start from stage 1; out: start), len, first 16 key bytes (zero padded)
 template <int IN>
 __device__ __forceinline__ void in_stage3(const Batch& b, const InCtx& c, uint32_t g, uint32_t gn, uint32_t lane,
-                                          bool valid, uint64_t s_next, uint4 ch, uint32_t win, uint64_t& s,
+                                          bool valid, uint64_t s_next, uint32_t eo, uint4 ch, uint32_t win, uint64_t& s,
                                           uint32_t& len, uint64_t& w0, uint64_t& w1) {
     w0 = 0; w1 = 0; len = 0;
     if (IN == IN_IDX) {
@@ -512,7 +518,7 @@ __device__ __forceinline__ void in_stage3(const Batch& b, const InCtx& c, uint32
         uint32_t e = __shfl_down_sync(FULLMASK, (uint32_t)s, 1);
         const uint32_t first_next = __shfl_sync(FULLMASK, (uint32_t)s_next, 0);
         if (g + 1 == c.ngroups && lane + 1 == c.tail) e = (uint32_t)c.kend;
-        else if (lane == 31) e = (gn == g + 1) ? first_next : (uint32_t)ld_in64(b.ko + (uint64_t)g * 32 + 32);
+        else if (lane == 31) e = (gn == g + 1) ? first_next : eo;
         len = valid ? e - (uint32_t)s : 0u;
     } else {
         s = ((uint64_t)g * 32 + lane) * b.kw;
@@ -812,11 +818,11 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     // pipeline prologue: group g (stages 1+2 done), group gn (stage 1 in flight)
     uint32_t g = (blockIdx.x * WARPS + (tid >> 5)) * (uint32_t)stream::CH;
     uint64_t s_c = 0, v_c = 1, s_n = 0, v_n = 1;
-    uint32_t win_c;
-    in_stage1<IN, VALS>(b, c, g, lane, s_c, v_c);
+    uint32_t win_c, eo_c = 0, eo_n = 0;
+    in_stage1<IN, VALS>(b, c, g, lane, s_c, v_c, eo_c);
     uint4 ch_c = in_stage2<IN>(b, c, g, lane, s_c, win_c);
     uint32_t gn = stream::next_group(g, c.nw);
-    in_stage1<IN, VALS>(b, c, gn, lane, s_n, v_n);
+    in_stage1<IN, VALS>(b, c, gn, lane, s_n, v_n, eo_n);
 
     while (g < c.ngroups) {
         // ---- issue ahead: key chunks of gn, offsets (values) of the group after it
@@ -824,7 +830,8 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         const uint4 ch_n = in_stage2<IN>(b, c, gn, lane, s_n, win_n);
         const uint32_t gnn = stream::next_group(gn, c.nw);
         uint64_t s_nn, v_nn;
-        in_stage1<IN, VALS>(b, c, gnn, lane, s_nn, v_nn);
+        uint32_t eo_nn = 0;
+        in_stage1<IN, VALS>(b, c, gnn, lane, s_nn, v_nn, eo_nn);
 
 #if SEPO_IN_PREFETCH
         // L2 prefetch SEPO_IN_PREFETCH groups further ahead in the warp's chunk: the 2 lines of key
@@ -848,7 +855,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         const bool valid = lane < group_cnt(c, g);
         uint64_t s = s_c, w0, w1;
         uint32_t len;
-        in_stage3<IN>(b, c, g, gn, lane, valid, s_n, ch_c, win_c, s, len, w0, w1);
+        in_stage3<IN>(b, c, g, gn, lane, valid, s_n, eo_c, ch_c, win_c, s, len, w0, w1);
         const uint64_t v = VALS ? (IN == IN_IDX ? (valid ? rec_value(b, (uint64_t)g * 32 + lane) : 0ull) : v_c) : 1ull;
         const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
         // ---- hot set (a2): both 4-way fingerprint buckets, then one 16-byte key compare
@@ -927,6 +934,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         g = gn; gn = gnn;
         s_c = s_n; v_c = v_n; ch_c = ch_n; win_c = win_n;
         s_n = s_nn; v_n = v_nn;
+        eo_c = eo_n; eo_n = eo_nn;
     }
     if (qtail != qhead) resolve_misses<VALS, WARPS>(d, b, S, Q, qhead, qtail - qhead, inj, w_full, w_quiet, pc);
     if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
