@@ -47,7 +47,10 @@ enum sepo_status {
 /* Bucket organizations. BASIC is not implemented. */
 typedef enum {
     SEPO_COMBINE_SUM_U64 = 0, /* "combining": one entry per key, value = u64 wrapping sum */
-    SEPO_GROUP = 1            /* "multi-valued": key entries + per-key value lists */
+    SEPO_GROUP = 1,           /* "multi-valued": key entries + per-key value lists */
+    SEPO_BASIC = 2            /* "basic": every pair its own entry, duplicates kept;
+                                 a pass halts once basic_halt_pct % of the allocator slots failed
+                                 (P:L153-161). Values as COMBINE (fixed width <= 8 B LE, or 1). */
 } sepo_mode;
 
 typedef struct sepo_options {
@@ -64,6 +67,9 @@ typedef struct sepo_options {
     uint32_t check_dups;      /* sepo_export merges + counts keys found in >1 generation */
     void* stream;             /* cudaStream_t for all device work (NULL: a table-owned stream) */
     uint64_t host_arena_bytes;/* pinned host memory to pre-allocate for evicted pages */
+    uint32_t basic_halt_pct;  /* BASIC: halt the pass once this % of allocator slots (the paper's
+                                 bucket groups) failed to allocate (1..100; 0 = 50) */
+    uint32_t pad_;
 } sepo_options;
 
 /* Host-side result, owned by the table (valid until the next sepo_reset / sepo_destroy).

@@ -138,6 +138,25 @@ def group(keys, offs, vals, val_offs=None, val_width=0):
     return Group().add(keys, offs, vals, val_offs, val_width)
 
 
+def basic(keys, offs, vals=None, val_width=0):
+    """Basic organization ("Two KV pairs with the same key are stored as two separate
+    entries"): the table holds exactly the input multiset of (key, value) pairs. Canonical form:
+    {key bytes: sorted list of values}. Values as the combining method reads them: width 0 -> 1
+    (P:L73), else val_width little-endian bytes per record. Plain loop (small inputs only)."""
+    keys = _u8(keys).tobytes()
+    offs = np.asarray(offs, dtype=np.uint64)
+    n = len(offs) - 1
+    if val_width:
+        v = np.frombuffer(_u8(vals).tobytes()[: n * val_width], dtype=np.uint8).reshape(n, val_width)
+        vv = [int.from_bytes(v[i].tobytes(), "little") for i in range(n)]
+    else:
+        vv = [1] * n
+    out = {}
+    for i in range(n):
+        out.setdefault(keys[int(offs[i]):int(offs[i + 1])], []).append(vv[i])
+    return {k: sorted(x) for k, x in out.items()}
+
+
 def compact(keys, offs, bitmap, vals=None, val_offs=None, val_width=0):
     """Gather the records whose bitmap bit is 1 -> (keys, offs, vals, val_offs, m)."""
     keys, offs = _u8(keys), np.ascontiguousarray(offs, dtype=np.uint64)

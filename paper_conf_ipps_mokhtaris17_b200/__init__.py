@@ -14,7 +14,7 @@ __all__ = ["Table", "SepoError", "lib", "COMBINE", "GROUP", "Stats"]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.environ.get("SEPO_LIB") or os.path.join(_HERE, "lib", "libsepo.so")
-COMBINE, GROUP = 0, 1
+COMBINE, GROUP, BASIC = 0, 1, 2  # sepo_mode (include/sepo.h)
 _LIB = None
 
 vp, u64, u32, i64 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int64
@@ -23,7 +23,8 @@ vp, u64, u32, i64 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_
 class Options(ctypes.Structure):
     _fields_ = [("mode", ctypes.c_int32), ("fixed_key_width", u32), ("fixed_val_width", u32), ("grid_ctas", u32),
                 ("hash_seed", u64), ("fail_alloc_ppm", u32), ("fail_mode", u32), ("fail_until_pass", u32),
-                ("check_dups", u32), ("stream", vp), ("host_arena_bytes", u64)]
+                ("check_dups", u32), ("stream", vp), ("host_arena_bytes", u64), ("basic_halt_pct", u32),
+                ("pad_", u32)]
 
 
 class Result(ctypes.Structure):
@@ -119,7 +120,7 @@ class Table:
 
     def __init__(self, budget_bytes, n_buckets, page_bytes=65536, mode=COMBINE, fixed_key_width=0,
                  fixed_val_width=0, grid_ctas=0, hash_seed=0, fail_alloc_ppm=0, fail_mode=0, fail_until_pass=0,
-                 check_dups=False, stream=None, host_arena_bytes=0, placement=0):
+                 check_dups=False, stream=None, host_arena_bytes=0, placement=0, basic_halt_pct=0):
         import torch
         if not torch.cuda.is_available():
             raise RuntimeError("paper_conf_ipps_mokhtaris17_b200 needs a CUDA device (no CPU fallback)")
@@ -134,9 +135,9 @@ class Table:
         if stream is None:
             stream = torch.cuda.current_stream()
         self.mode = mode
-        self.opts = Options(mode, fixed_key_width, fixed_val_width or (8 if mode == COMBINE else 0), grid_ctas,
+        self.opts = Options(mode, fixed_key_width, fixed_val_width or (8 if mode != GROUP else 0), grid_ctas,
                             hash_seed, fail_alloc_ppm, fail_mode, fail_until_pass, int(bool(check_dups)),
-                            ctypes.c_void_p(stream.cuda_stream), int(host_arena_bytes))
+                            ctypes.c_void_p(stream.cuda_stream), int(host_arena_bytes), int(basic_halt_pct), 0)
         rc = L.sepo_configure(self.h, ctypes.byref(self.opts))
         if rc:
             L.sepo_destroy(self.h)
@@ -226,7 +227,7 @@ class Table:
 
         ko = arr(r.key_offsets, k + 1, np.uint64)
         out = {"n_keys": k, "key_offsets": ko, "keys": arr(r.keys, int(ko[-1]) if k else 0, np.uint8)}
-        if self.mode == COMBINE:
+        if self.mode in (COMBINE, BASIC):  # BASIC: one (key, value) row per stored pair
             out["values"] = arr(r.values, k, np.uint64)
         else:
             lo = arr(r.list_offsets, k + 1, np.uint64)
@@ -259,9 +260,16 @@ class Table:
 
 
 def result_dict(res, mode=COMBINE):
-    """Exported arrays -> {key bytes: value} (COMBINE) or {key: sorted list of value bytes}."""
+    """Exported arrays -> {key bytes: value} (COMBINE), {key: sorted list of value bytes} (GROUP) or
+    {key: sorted list of u64 values} (BASIC: the multiset of stored pairs)."""
     kb = res["keys"].tobytes()
     ko = res["key_offsets"]
+    if mode == BASIC:
+        v = res["values"]
+        out = {}
+        for i in range(res["n_keys"]):
+            out.setdefault(kb[ko[i]:ko[i + 1]], []).append(int(v[i]))
+        return {k: sorted(x) for k, x in out.items()}
     if mode == COMBINE:
         v = res["values"]
         return {kb[ko[i]:ko[i + 1]]: int(v[i]) for i in range(res["n_keys"])}

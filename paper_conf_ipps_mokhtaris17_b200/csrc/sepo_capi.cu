@@ -180,8 +180,8 @@ int make_batch(sepo_table* t, Batch& b, const uint8_t* keys, const uint64_t* ko,
     if (n > (1ull << 36)) return fail(SEPO_E_INVAL, "more than 2^36 records in one batch");
     if (!keys && !(ko == nullptr && b.kw == 0)) return fail(SEPO_E_INVAL, "keys is NULL");
     if (!ko && b.kw == 0) return fail(SEPO_E_INVAL, "key_offsets is NULL and fixed_key_width is 0");
-    if (t->opts.mode == SEPO_COMBINE_SUM_U64) {
-        if (vo) return fail(SEPO_E_INVAL, "COMBINE mode takes fixed-width values (val_offsets must be NULL)");
+    if (t->opts.mode != SEPO_GROUP) {
+        if (vo) return fail(SEPO_E_INVAL, "COMBINE/BASIC mode takes fixed-width values (val_offsets must be NULL)");
         if (vals && !(b.vw == 1 || b.vw == 2 || b.vw == 4 || b.vw == 8))
             return fail(SEPO_E_INVAL, "COMBINE fixed_val_width must be 1, 2, 4 or 8");
         if (vals && ((uintptr_t)vals % b.vw)) return fail(SEPO_E_INVAL, "vals not aligned to fixed_val_width");
@@ -395,11 +395,14 @@ int sepo_configure(sepo_table* t, const sepo_options* o) {
     if (rc) return rc;
     if (!o) return fail(SEPO_E_INVAL, "null options");
     if (t->inserted) return fail(SEPO_E_STATE, "configure only before the first insert (or after sepo_reset)");
-    if (o->mode != SEPO_COMBINE_SUM_U64 && o->mode != SEPO_GROUP) return fail(SEPO_E_INVAL, "unknown mode");
+    if (o->mode != SEPO_COMBINE_SUM_U64 && o->mode != SEPO_GROUP && o->mode != SEPO_BASIC)
+        return fail(SEPO_E_INVAL, "unknown mode");
+    if (o->basic_halt_pct > 100) return fail(SEPO_E_INVAL, "basic_halt_pct must be <= 100");
     if (o->fixed_key_width > 65535u - 64u) return fail(SEPO_E_INVAL, "fixed_key_width too large");
     if (o->grid_ctas > 1024) return fail(SEPO_E_INVAL, "grid_ctas must be <= 1024");
     sepo_options n = *o;
-    if (n.mode == SEPO_COMBINE_SUM_U64 && n.fixed_val_width == 0) n.fixed_val_width = 8;
+    if (n.mode != SEPO_GROUP && n.fixed_val_width == 0) n.fixed_val_width = 8;
+    if (n.basic_halt_pct == 0) n.basic_halt_pct = 50;
     if (n.fail_until_pass == 0) n.fail_until_pass = 16;
     if (n.grid_ctas == 0) n.grid_ctas = (uint32_t)sepo_default_grid(n.mode, t->n_sms);
     t->grid = (int)n.grid_ctas;
@@ -454,7 +457,9 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
     if ((rc = zero_ctrl_counters(t))) return rc;
     CK(t, cudaEventRecord(t->ev0, t->stream));
     if (t->hot.grow(sepo_hot_scratch_bytes())) return fail(SEPO_E_NOMEM, "hot-set scratch");
-    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p);
+    // BASIC halt rule: the pass stops once this many allocator slots failed
+    const uint32_t halt_slots = (uint32_t)std::max<uint64_t>(1, ((uint64_t)t->grid * t->opts.basic_halt_pct + 99) / 100);
+    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p, halt_slots);
     if (rc) return cuda_check(t, (cudaError_t)rc, "insert kernel launch");
     CK(t, cudaEventRecord(t->ev1, t->stream));
     t->st.kernel_launches += (n >= (8ull << 18)) ? 7 : 1;
@@ -535,7 +540,10 @@ static int64_t count_or_probe(sepo_table* t, const Batch& b, int probe, uint64_t
     // COMBINE re-probe and every count-only pass never allocate: use a full-occupancy grid.
     // GROUP re-probe allocates value chunks, so it runs on the allocator slots (one per CTA).
     const int rgrid = (probe && t->opts.mode == SEPO_GROUP) ? t->grid : 8 * t->n_sms;
-    rc = sepo_launch_reprobe(t->d, b, t->opts.mode, probe, rgrid, (unsigned long long*)t->tile_counts.p, t->stream);
+    // BASIC: nothing to re-probe (a postponed pair left nothing in the table): count only
+    rc = sepo_launch_reprobe(t->d, b, t->opts.mode == SEPO_BASIC ? SEPO_COMBINE_SUM_U64 : t->opts.mode,
+                             t->opts.mode == SEPO_BASIC ? 0 : probe, rgrid, (unsigned long long*)t->tile_counts.p,
+                             t->stream);
     t->st.kernel_launches += 1;
     if (rc) return cuda_check(t, (cudaError_t)rc, "reprobe kernel launch");
     if ((rc = read_ctrl(t))) return rc;
@@ -619,6 +627,7 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
     rc = sepo_launch_classify(t->d, honor_retain, t->stream);
     if (rc) return cuda_check(t, (cudaError_t)rc, "classify kernel");
     CK(t, cudaMemsetAsync(&t->d.ctrl->full, 0, sizeof(unsigned long long), t->stream));
+    CK(t, cudaMemsetAsync(&t->d.ctrl->failed_slots, 0, sizeof(unsigned int), t->stream));
     CK(t, cudaMemsetAsync(t->d.ann, 0, kMaxGrid * ANN_STRIDE * 8, t->stream));
     t->st.kernel_launches += 2;
     // the previous eviction's copies (and its writes of ctrl->copied) are done before the reset
@@ -729,7 +738,10 @@ void parallel_for(size_t n, F f) {
     for (auto& x : th) x.join();
 }
 
+// COMBINE: one entry per key (merge of cross-generation duplicates as a backstop); BASIC: one
+// entry per pair (K_BASIC), duplicates are the result, never merged
 int export_combine(sepo_table* t) {
+    const uint32_t kind = t->opts.mode == SEPO_BASIC ? K_BASIC : K_COMBINE;
     std::vector<PageRef> pages;
     collect_pages(t, pages);
     const uint32_t PB = t->page_bytes;
@@ -746,7 +758,7 @@ int export_combine(sepo_table* t) {
                 memcpy(&hdr, base + off, 4);
                 uint32_t sz = hdr & ~KIND_MASK;
                 if (sz == 0 || off + sz > PB) { bad = 1; break; }
-                if ((hdr & KIND_MASK) == K_COMBINE) {
+                if ((hdr & KIND_MASK) == kind) {
                     uint32_t klen;
                     memcpy(&klen, base + off + 12, 4);
                     ++k;
@@ -773,7 +785,7 @@ int export_combine(sepo_table* t) {
                 uint32_t hdr;
                 memcpy(&hdr, base + off, 4);
                 uint32_t sz = hdr & ~KIND_MASK;
-                if ((hdr & KIND_MASK) == K_COMBINE) {
+                if ((hdr & KIND_MASK) == kind) {
                     uint32_t klen;
                     memcpy(&klen, base + off + 12, 4);
                     t->x_koffs[k] = kb;
@@ -789,7 +801,7 @@ int export_combine(sepo_table* t) {
     t->x_koffs[nk] = nkb;
     t->x_nkeys = nk;
     // keys found in more than one generation (only possible under record-mode fault injection)
-    const bool merge = t->opts.check_dups || (t->opts.fail_alloc_ppm && t->opts.fail_mode == 1);
+    const bool merge = kind == K_COMBINE && (t->opts.check_dups || (t->opts.fail_alloc_ppm && t->opts.fail_mode == 1));
     if (merge && nk) {
         std::unordered_map<std::string_view, uint64_t> idx;
         idx.reserve(nk * 2);
@@ -971,14 +983,14 @@ int sepo_export(sepo_table* t, sepo_result* out) {
     }
     CK(t, cudaStreamSynchronize(t->copy_stream));
     auto t0 = std::chrono::steady_clock::now();
-    rc = t->opts.mode == SEPO_COMBINE_SUM_U64 ? export_combine(t) : export_group(t);
+    rc = t->opts.mode == SEPO_GROUP ? export_group(t) : export_combine(t);
     if (rc) return rc;
     t->st.t_export_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     memset(out, 0, sizeof(*out));
     out->n_keys = t->x_nkeys;
     out->keys = t->x_keys.data();
     out->key_offsets = t->x_koffs.data();
-    if (t->opts.mode == SEPO_COMBINE_SUM_U64) {
+    if (t->opts.mode != SEPO_GROUP) {  // COMBINE: one (key, sum) per key; BASIC: one (key, value) per pair
         out->values = t->x_values.data();
     } else {
         out->list_offsets = t->x_loffs.data();
@@ -1039,7 +1051,7 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
     uint64_t prev = ~0ull;
     // both streaming kernels certify their declines (R15) and mark pending GROUP keys' pages
     // themselves, so the insert's count is exact — except under record-mode injection
-    const bool combine_exact = !(t->opts.fail_alloc_ppm && t->opts.fail_mode == 1);
+    const bool combine_exact = t->opts.mode == SEPO_BASIC || !(t->opts.fail_alloc_ppm && t->opts.fail_mode == 1);
     // COMBINE re-issue in prepared form (a9): the first pass appends each declined record as
     // {hash, first 16 key bytes, key offset, value, length}; later passes read those records
     // densely (no gather through an index list, no re-hash). The first pass's list is sized

@@ -30,7 +30,7 @@
 namespace sepo {
 
 constexpr uint32_t FULLMASK = 0xffffffffu;
-enum : uint32_t { K_FREE = 0, K_COMBINE = 1, K_FILL = 2, K_DEAD = 3, K_GKEY = 4, K_VCHUNK = 5 };
+enum : uint32_t { K_FREE = 0, K_COMBINE = 1, K_FILL = 2, K_DEAD = 3, K_GKEY = 4, K_VCHUNK = 5, K_BASIC = 6 };
 constexpr uint32_t KIND_MASK = 7u;
 constexpr uint32_t KEY_OFF = 16;     // key bytes start here in combine and group key entries
 constexpr uint32_t CHUNK_HDR = 32;   // value chunk header
@@ -54,7 +54,7 @@ struct Ctrl {
     unsigned long long full;           // 1 once the pool ran out this generation: every later allocation fails
     unsigned long long n_safe;         // evict: free pages that need no copy (never used last generation)
     unsigned int copied;               // evicted pages whose D2H copy finished (written by the copy stream)
-    unsigned int pad0;
+    unsigned int failed_slots;         // BASIC: allocator slots whose allocation failed this generation
     unsigned long long pad[4];
 };
 
@@ -393,13 +393,14 @@ __device__ __forceinline__ bool inject_fail(const Dev& d, uint64_t h, uint64_t r
 // from the free stack (one global atomic per page) and installs it; lanes of other warps that
 // overshot wait for the install and retry. Must be called by all 32 lanes.
 __device__ __forceinline__ uint64_t warp_alloc(const Dev& d, unsigned long long* scur, bool need, uint32_t size,
-                                               uint8_t page_kind) {
+                                               uint8_t page_kind, bool monotone = true) {
     const uint32_t lane = threadIdx.x & 31u;
     const uint32_t PB = d.page_bytes;
     uint64_t result = ~0ull;
     bool pending = need;
     // failure is monotone for the whole generation: once the pool ran out, nobody allocates
-    if (__any_sync(FULLMASK, pending)) {
+    // (BASIC passes monotone = false: a slot keeps filling its open page)
+    if (monotone && __any_sync(FULLMASK, pending)) {
         unsigned long long full = 0;
         if (lane == 0) full = ld_relaxed_u64(&d.ctrl->full);
         if (__shfl_sync(FULLMASK, full, 0) != 0ull) return ~0ull;  // warp-uniform decision

@@ -335,6 +335,9 @@ namespace stream {
 #ifndef SEPO_CHUNK_GROUPS
 #define SEPO_CHUNK_GROUPS 32      // consecutive 32-record groups a warp streams before it strides
 #endif
+#ifndef SEPO_S1_AHEAD
+#define SEPO_S1_AHEAD 2           // groups ahead the key offsets are loaded (2 or 3)
+#endif
 #ifndef SEPO_FOLD
 #define SEPO_FOLD 1               // fold equal hot keys of a warp before the shared atomic
 #endif
@@ -354,12 +357,34 @@ struct CtaState {                 // allocator slot (the CTA's active pages) + p
 };
 // Shared memory of the COMBINE stream kernel: the hot set (read-only keys + per-CTA pending sums)
 // and one miss queue per warp (records that missed the hot set, resolved 32 at a time).
+#ifndef SEPO_HOT_DIRECT
+#define SEPO_HOT_DIRECT 1  // direct-indexed hot set (C2 4x pass 1 22.2 -> 21.3 ms); 0: 4-way bucket fingerprints
+#endif
+#if SEPO_HOT_DIRECT
+// Direct-indexed hot set: DS one-word slots (2-choice, one slot per choice); a slot holds the key's
+// fingerprint and its index into the dense key arrays, so a probe is two 4-byte loads, two
+// compares and one 16-byte key load.
+constexpr int DS = 16384;                 // slots (hot keys <= hot::K = 2048: load <= 1/8)
+constexpr int NKEY = hot::K;
+__device__ __forceinline__ uint32_t ds1(uint64_t h) { return (uint32_t)(h >> 3) & (DS - 1); }
+__device__ __forceinline__ uint32_t ds2(uint64_t h) { return (uint32_t)(h >> 17) & (DS - 1); }
+// slot word: fingerprint (12 hash bits + the key length saturated at 255) | 1 | key index (11 bits)
+__device__ __forceinline__ uint32_t dfp(uint64_t h, uint32_t len) {
+    return ((((uint32_t)(h >> 52) << 8) | min(len, 255u)) << 12) | 0x800u;
+}
+#else
+constexpr int NKEY = hot::NH;
+#endif
 template <bool VALS, int WARPS>
 struct Smem {
+#if SEPO_HOT_DIRECT
+    uint32_t tags[DS];            // slot words (0: empty)
+#else
     uint4 tags[hot::NB];          // 4 fingerprints per bucket (one 16-B load per probed bucket)
-    ulonglong2 kw[hot::NH];       // first 16 key bytes, zero padded (one 16-B load per candidate)
-    uint32_t ref[hot::NH];        // resident entry (0: empty slot)
-    typename std::conditional<VALS, unsigned long long, unsigned int>::type sum[hot::NH];  // pending sums
+#endif
+    ulonglong2 kw[NKEY];          // first 16 key bytes, zero padded (one 16-B load per candidate)
+    uint32_t ref[NKEY];           // resident entry (0: empty slot)
+    typename std::conditional<VALS, unsigned long long, unsigned int>::type sum[NKEY];  // pending sums
     struct Queue {                // structure of arrays, QCAP slots, ring indexed by a warp counter
         unsigned long long w0[QCAP], w1[QCAP], h[QCAP], s[QCAP];
         typename std::conditional<VALS, unsigned long long, unsigned char>::type v[VALS ? QCAP : 1];
@@ -762,6 +787,95 @@ __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
     }
 }
 
+// ================================================================ BASIC insert (NEXT-3)
+// The paper's basic organization: every pair is its own entry — no key compare, no
+// combining; duplicates stay separate entries of the bucket's chain. A pair is POSTPONED when its
+// allocator slot's open page is full and the pool has no free page (the slots play the
+// paper's bucket groups, R7, and fail independently here: warp_alloc non-monotone). The pass HALTS
+// once `halt_slots` slots have failed (50 % of the bucket groups): every later record of the
+// pass is postponed without an attempt, and the host evicts the whole heap and restarts from the
+// postponed records (R11). No race needs certifying: a postponed pair leaves nothing
+// in the table, and a key may legitimately appear in several generations.
+__global__ void __launch_bounds__(1024, 1) insert_basic_kernel(Dev d, Batch b, uint32_t halt_slots) {
+    __shared__ unsigned long long s_cur;
+    __shared__ int s_failed;
+    __shared__ unsigned long long s_post[32], s_pkb[32];
+    const uint32_t tid = threadIdx.x, lane = lane_id(), warp = tid >> 5;
+    if (tid == 0) { s_cur = d.cursors[2 * blockIdx.x]; s_failed = 0; }
+    if (tid < 32) { s_post[tid] = 0; s_pkb[tid] = 0; }
+    __syncthreads();
+    const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
+    const uint64_t ngroups = (b.n + 31) / 32;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    bool halted = false;  // warp-uniform
+    for (uint64_t g = (uint64_t)blockIdx.x * (blockDim.x / 32) + warp; g < ngroups; g += nw) {
+        const uint64_t i = g * 32 + lane;
+        const bool valid = i < b.n;
+        if (!halted) {
+            unsigned int fs = 0;
+            if (lane == 0) fs = ld_relaxed_u32(&d.ctrl->failed_slots);
+            halted = __shfl_sync(FULLMASK, fs, 0) >= halt_slots;
+        }
+        uint64_t s = 0;
+        uint32_t len = 0, res = R_POST;
+        if (valid) rec_key(b, i, s, len);
+        if (!halted) {
+            uint64_t w0 = 0, w1 = 0;
+            if (valid) load_key16(b.keys + s, len, w0, w1);
+            const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
+            const uint64_t v = valid ? rec_value(b, i) : 0ull;
+            const uint32_t esize = centry_size(len);
+            bool need = valid;
+            res = R_OK;
+            if (need && (len > 65535u - 64u || esize > d.page_bytes)) { need = false; res = R_TOOLARGE; }
+            if (inj && need && inject_fail(d, h, i)) { need = false; res = R_POST; }
+            const uint64_t off = warp_alloc(d, &s_cur, need, esize, (uint8_t)PAGE_ENTRY, false);
+            const bool declined = need && off == ~0ull;
+            if (declined) res = R_POST;
+            if (__any_sync(FULLMASK, declined) && lane == 0 && atomicExch(&s_failed, 1) == 0)
+                atomicAdd(&d.ctrl->failed_slots, 1u);  // this slot (bucket group) failed
+            if (need && off != ~0ull) {
+                uint8_t* e = d.pool + off;
+                const uint32_t bkt = bucket_of(h, d.n_buckets);
+                uint32_t head = ld_dir(d.dir + bkt);
+                *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_BASIC, head, tag_of(h), len);
+                if (len > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0;
+                if (len > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1;
+                if (len > 16) store_key(e + KEY_OFF + 16, b.keys + s + 16, len - 16);
+                *reinterpret_cast<unsigned long long*>(entry_val(e, len)) = v;
+                const uint32_t me = off_ref(off);
+                while (true) {  // lock-free head insertion; duplicates are allowed
+                    const uint32_t old = cas_release(d.dir + bkt, head, me);
+                    if (old == head) break;
+                    head = old;
+                    *reinterpret_cast<uint32_t*>(e + 4) = head;
+                }
+            }
+        }
+        // outcomes -> the group's bitmap word (this warp owns it) + counts (a7)
+        const bool out = valid && res != R_OK;
+        const unsigned pm = __ballot_sync(FULLMASK, out);
+        if (lane == 0 && b.bitmap) b.bitmap[g] = pm;
+        if (pm) {
+            const unsigned tl = __ballot_sync(FULLMASK, valid && res == R_TOOLARGE);
+            const unsigned pkb = __reduce_add_sync(FULLMASK, out ? len : 0u);
+            if (lane == 0) {
+                s_post[warp] += __popc(pm);
+                s_pkb[warp] += pkb;
+                if (tl) atomicAdd(&d.ctrl->toolarge, (unsigned long long)__popc(tl));
+            }
+        }
+    }
+    __syncthreads();
+    if (tid == 0) {
+        d.cursors[2 * blockIdx.x] = s_cur;
+        unsigned long long post = 0, pkb = 0;
+        for (uint32_t w = 0; w < blockDim.x / 32; ++w) { post += s_post[w]; pkb += s_pkb[w]; }
+        if (post) atomicAdd(&d.ctrl->postponed, post);
+        if (pkb) atomicAdd(&d.ctrl->kept_key_bytes, pkb);
+    }
+}
+
 template <bool VALS, int THREADS, int IN>
 __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
                                                                    const unsigned int* n_hot) {
@@ -770,8 +884,12 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     extern __shared__ __align__(16) uint8_t smem_raw[];
     SM& S = *reinterpret_cast<SM*>(smem_raw);
     const uint32_t tid = threadIdx.x, lane = lane_id();
-    for (int p = tid; p < hot::NH; p += THREADS) { S.ref[p] = 0; S.sum[p] = 0; }
+    for (int p = tid; p < stream::NKEY; p += THREADS) { S.ref[p] = 0; S.sum[p] = 0; }
+#if SEPO_HOT_DIRECT
+    for (int p = tid; p < stream::DS; p += THREADS) S.tags[p] = 0u;
+#else
     for (int p = tid; p < hot::NB; p += THREADS) S.tags[p] = make_uint4(0, 0, 0, 0);
+#endif
     if (tid == 0) {
         S.cs.cur[0] = d.cursors[2 * blockIdx.x];
         S.cs.cur[1] = d.cursors[2 * blockIdx.x + 1];
@@ -785,6 +903,16 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         for (unsigned j = tid; j < nh; j += THREADS) {
             const hot::Entry e = hl[j];
             if (e.ref == 0 || hot::count_class(e.count) != cls) continue;
+#if SEPO_HOT_DIRECT
+            if (j < (unsigned)stream::NKEY) {  // claim slot ds1, else ds2, else leave the key out
+                const uint32_t f = stream::dfp(e.h, e.len) | j;
+                if (atomicCAS(&S.tags[stream::ds1(e.h)], 0u, f) == 0u || atomicCAS(&S.tags[stream::ds2(e.h)], 0u, f) == 0u) {
+                    S.kw[j] = make_ulonglong2(e.w0, e.w1);
+                    S.ref[j] = e.ref;
+                }
+            }
+            continue;
+#endif
             // claim a free slot in bucket b1, else b2, else leave the key out (the set is only a cache)
             const uint32_t f = stream::fpl(e.h, e.len);
             int pos = -1;
@@ -823,15 +951,30 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     uint4 ch_c = in_stage2<IN>(b, c, g, lane, s_c, win_c);
     uint32_t gn = stream::next_group(g, c.nw);
     in_stage1<IN, VALS>(b, c, gn, lane, s_n, v_n, eo_n);
+#if SEPO_S1_AHEAD == 3
+    // offsets three groups ahead: group gx (stage 1 in flight one iteration longer)
+    uint32_t gx = stream::next_group(gn, c.nw);
+    uint64_t s_x = 0, v_x = 1;
+    uint32_t eo_x = 0;
+    in_stage1<IN, VALS>(b, c, gx, lane, s_x, v_x, eo_x);
+#endif
 
     while (g < c.ngroups) {
         // ---- issue ahead: key chunks of gn, offsets (values) of the group after it
         uint32_t win_n;
         const uint4 ch_n = in_stage2<IN>(b, c, gn, lane, s_n, win_n);
+#if SEPO_S1_AHEAD == 3
+        const uint32_t gnn = gx;
+        uint64_t s_nn = s_x, v_nn = v_x;
+        uint32_t eo_nn = eo_x;
+        gx = stream::next_group(gx, c.nw);
+        in_stage1<IN, VALS>(b, c, gx, lane, s_x, v_x, eo_x);
+#else
         const uint32_t gnn = stream::next_group(gn, c.nw);
         uint64_t s_nn, v_nn;
         uint32_t eo_nn = 0;
         in_stage1<IN, VALS>(b, c, gnn, lane, s_nn, v_nn, eo_nn);
+#endif
 
 #if SEPO_IN_PREFETCH
         // L2 prefetch SEPO_IN_PREFETCH groups further ahead in the warp's chunk: the 2 lines of key
@@ -860,6 +1003,23 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
         // ---- hot set (a2): both 4-way fingerprint buckets, then one 16-byte key compare
         int pos = -1;
+#if SEPO_HOT_DIRECT
+        if (have_hot) {
+            const uint32_t f = stream::dfp(h, len);
+            const uint32_t t1 = S.tags[stream::ds1(h)], t2 = S.tags[stream::ds2(h)];
+            const bool m1 = (t1 & 0xfffff800u) == f, m2 = (t2 & 0xfffff800u) == f;
+            const uint32_t p = (m1 ? t1 : t2) & 0x7ffu;
+            if (valid && (m1 || m2)) {
+                const ulonglong2 kk = S.kw[p];
+                bool eq = kk.x == w0 && kk.y == w1;
+                if (len > 16) {  // long key: exact length (the fingerprint saturates at 255) + tail bytes
+                    const uint8_t* e = ref_ptr(d, S.ref[p]);
+                    eq = eq && ldcg32(e + 12) == len && entry_key_eq(e + KEY_OFF + 16, b.keys + s + 16, len - 16);
+                }
+                if (eq) pos = (int)p;
+            }
+        }
+#else
         if (have_hot) {
             const uint32_t f = stream::fpl(h, len);
             const uint32_t k1 = hot::b1(h), k2 = hot::b2(h);
@@ -877,6 +1037,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
                 if (eq) pos = p;
             }
         }
+#endif
         // ---- fold the hits of the warp per hot slot (a2): one shared atomic per distinct key
         const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
         if (hm) {
@@ -940,7 +1101,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
     __syncthreads();
     // flush the hot keys' pending sums into their resident entries
-    for (int p = tid; p < hot::NH; p += THREADS) {
+    for (int p = tid; p < stream::NKEY; p += THREADS) {
         if (S.ref[p] == 0 || S.sum[p] == 0) continue;
         uint8_t* e = ref_ptr(d, S.ref[p]);
         red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(e, ldcg32(e + 12))), (unsigned long long)S.sum[p]);
@@ -1862,7 +2023,12 @@ __global__ void init_state_kernel(Dev d, uint32_t n_slots) {
 // ================================================================ launchers
 using namespace sepo;
 
-int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch) {
+int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
+                       uint32_t halt_slots) {
+    if (mode == 2) {
+        insert_basic_kernel<<<grid, 1024, 0, s>>>(d, b, halt_slots);
+        return cudaGetLastError();
+    }
     if (mode == 0) {
         // hot-set discovery on a strided sample (skipped for small batches)
         const hot::Entry* hl = nullptr;

@@ -34,7 +34,8 @@ struct Batch {
 };
 }  // namespace sepo
 
-int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch);
+int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
+                       uint32_t halt_slots = 0);
 int sepo_launch_reinsert(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s);
 size_t sepo_hot_scratch_bytes();
 int sepo_default_grid(int mode, int n_sms);

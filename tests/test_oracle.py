@@ -251,3 +251,47 @@ def test_sepo_sim_group_exact(ratio):
     passes, post, out, forced = oracle.sepo_sim_group(keys, offs, vals, int(F / ratio), val_width=4, val_overhead=0)
     assert out.as_dict() == ref
     assert passes >= 1 if ratio == 1.0 else passes >= 3
+
+
+# ------------------------------------------------------------------ basic organization (NEXT-3)
+def test_basic_closed_form_pairs():
+    """basic stores every pair: per key, the multiset of its records' values. Pinned to
+    the generator's closed form (records of rank r = perm^-1 of its multiset block, their values),
+    which never looks at the input bytes the oracle reads."""
+    for name in ("C5u", "C5z"):
+        s = gen.config(name, scale=2e-5)
+        keys, offs, vals = s.host()
+        got = oracle.basic(keys, offs, vals, 8)
+        assert sum(len(v) for v in got.values()) == s.n
+        for r in [1, 2, 3, s.n_ranks // 2, s.n_ranks]:
+            assert got[s.spell(r)] == s.expected_group(r)
+
+
+def test_basic_vs_combine_and_counts():
+    """per key: count = the closed-form c_r (implicit-1 values), and the u64 sum of the stored
+    values = the (independent, C++) combining oracle's value"""
+    s = gen.config("C1", scale=0.02)
+    keys, offs, _ = s.host()
+    got = oracle.basic(keys, offs)
+    comb = oracle.combine(keys, offs).as_dict()
+    assert got.keys() == comb.keys()
+    for r in range(1, s.n_ranks + 1, 97):
+        k = s.spell(r)
+        if int(s.count_of_rank(r)):
+            assert len(got[k]) == int(s.count_of_rank(r)) and set(got[k]) == {1}
+    s = gen.config("C5z", scale=2e-5)
+    keys, offs, vals = s.host()
+    got = oracle.basic(keys, offs, vals, 8)
+    comb = oracle.combine(keys, offs, vals, 8).as_dict()
+    assert {k: sum(v) % (1 << 64) for k, v in got.items()} == comb
+
+
+def test_basic_tiny_adversarial():
+    """duplicates, empty keys, prefixes: every record is one pair of the result"""
+    ks = [b"", b"a", b"a", b"ab", b"", b"b\x00", b"b", b"a"]
+    vs = [5, 1, 1, 7, 0, 3, 3, 2]
+    keys = np.frombuffer(b"".join(ks), dtype=np.uint8)
+    offs = np.cumsum([0] + [len(k) for k in ks]).astype(np.uint64)
+    vals = np.array(vs, dtype=np.uint64).view(np.uint8)
+    got = oracle.basic(keys, offs, vals, 8)
+    assert got == {b"": [0, 5], b"a": [1, 1, 2], b"ab": [7], b"b\x00": [3], b"b": [3]}
