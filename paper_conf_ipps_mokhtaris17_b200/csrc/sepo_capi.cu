@@ -652,7 +652,33 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
     uint64_t bytes = 0, done = 0;
     const uint64_t chunk_pages = overlapped ? std::max<uint64_t>(std::max<uint64_t>(1, (1u << 20) >> t->page_shift), ne / 48)
                                             : ~0ull;  // progress granularity (overlap only)
-    for (uint64_t i = 0; i < ne;) {
+    // Fragmented evict lists (many short runs of consecutive pages, e.g. GROUP generations with
+    // retained key pages) go through one gather-copy kernel into a contiguous host region; long
+    // runs through cudaMemcpyAsync (copy engine). SEPO_EVICT_KERNEL=0/1 forces either.
+    uint64_t n_runs = 0;
+    for (uint64_t i = 0; i < ne; ++i) n_runs += (i == 0 || t->h_evict[i] != t->h_evict[i - 1] + 1);
+    const char* eks = getenv("SEPO_EVICT_KERNEL");
+    const int ek = eks ? atoi(eks) : -1;
+    const bool use_kernel = !overlapped && ne > 0 && (ek == 1 || (ek < 0 && n_runs * 64 > ne));
+    if (use_kernel) {
+        const size_t nbytes = (size_t)ne << t->page_shift;
+        uint8_t* hp = arena_alloc(t, nbytes);
+        if (!hp) return fail(SEPO_E_NOMEM, "pinned host arena exhausted");
+        uint8_t* dp = nullptr;
+        CK(t, cudaHostGetDevicePointer((void**)&dp, hp, 0));
+        rc = sepo_launch_evict_copy(t->d, (uint32_t)ne, dp, 2 * t->n_sms, t->copy_stream);
+        if (rc) return cuda_check(t, (cudaError_t)rc, "evict copy kernel");
+        t->st.kernel_launches += 1;
+        for (uint64_t i = 0; i < ne;) {
+            uint64_t j = i + 1;
+            while (j < ne && t->h_evict[j] == t->h_evict[j - 1] + 1) ++j;
+            img.runs.push_back({t->h_evict[i], (uint32_t)(j - i), hp + (i << t->page_shift)});
+            i = j;
+        }
+        bytes = nbytes;
+        done = ne;
+    }
+    for (uint64_t i = use_kernel ? ne : 0; i < ne;) {
         uint64_t j = i + 1;
         while (j < ne && t->h_evict[j] == t->h_evict[j - 1] + 1) ++j;
         const uint32_t first = t->h_evict[i], cnt = (uint32_t)(j - i);
@@ -1058,14 +1084,16 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
     // n/4 (SEPO_PREP_CAP overrides); on overflow the job continues on the index path.
     const char* no_prep = getenv("SEPO_NO_PREP");
     bool use_prep = t->opts.mode == SEPO_COMBINE_SUM_U64 && combine_exact && !(no_prep && no_prep[0] == '1') && n > 0;
+    const uint64_t prb = vals ? sizeof(PRec) : 32;  // prepared record bytes (implicit value 1: 32)
+    cur.prep_rb = (uint32_t)prb;
     if (use_prep) {
         uint64_t cap = std::max<uint64_t>(1ull << 16, n / 4);
         if (const char* pc = getenv("SEPO_PREP_CAP")) cap = strtoull(pc, nullptr, 10);
-        if ((uint64_t)t->prep[0].cap < cap * sizeof(PRec)) {  // first use / larger input: bound by free memory
+        if ((uint64_t)t->prep[0].cap < cap * prb) {  // first use / larger input: bound by free memory
             size_t fr = 0, tot = 0;
-            if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) cap = std::min<uint64_t>(cap, (fr + t->prep[0].cap) / 3 / sizeof(PRec));
+            if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) cap = std::min<uint64_t>(cap, (fr + t->prep[0].cap) / 3 / prb);
         }
-        if (t->prep_n.grow(64) || t->prep[0].grow(std::max<uint64_t>(cap, 1) * sizeof(PRec))) {
+        if (t->prep_n.grow(64) || t->prep[0].grow(std::max<uint64_t>(cap, 1) * prb)) {
             use_prep = false;
         } else {
             CK(t, cudaMemsetAsync(t->prep_n.p, 0, 16, t->stream));
@@ -1098,7 +1126,7 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
                 const uint64_t pass = t->st.passes;
                 if (pass < SEPO_MAX_PASS_STATS) t->st.postponed_per_pass[pass] += m;
                 const uint64_t ocap = reserved + slack;  // every record may decline again
-                if (t->prep[ps ^ 1].grow(ocap * sizeof(PRec))) return fail(SEPO_E_NOMEM, "prepared re-issue list");
+                if (t->prep[ps ^ 1].grow(ocap * prb)) return fail(SEPO_E_NOMEM, "prepared re-issue list");
                 int64_t e = evict_impl(t, 1);
                 if (e < 0) return e;
                 Batch pb = cur;

@@ -583,6 +583,7 @@ __device__ __forceinline__ void in_stage3(const Batch& b, const InCtx& c, uint32
 // warp leaves unused are closed with a sentinel length when it finishes (the reinsert pass skips them).
 constexpr uint32_t PREP_CHUNK = 256;
 constexpr uint32_t PREP_HOLE = 0xffffffffu;
+constexpr unsigned long long PREP_HOLE32 = 0xffffull;  // 32-B records: length field of a hole
 struct PrepCursor {
     unsigned long long base = 0;  // first slot of the warp's chunk
     uint32_t used = PREP_CHUNK;   // slots used in it (PREP_CHUNK: no chunk)
@@ -591,11 +592,16 @@ __device__ __forceinline__ void prep_close(const Batch& b, const PrepCursor& pc)
     const uint32_t lane = lane_id();
     for (uint32_t k = pc.used + lane; k < PREP_CHUNK; k += 32) {
         const unsigned long long slot = pc.base + k;
-        if (slot < b.out_cap)
-            reinterpret_cast<ulonglong2*>(b.out + slot)[2] = make_ulonglong2(0ull, (unsigned long long)PREP_HOLE);
+        if (slot < b.out_cap) {
+            ulonglong2* o = reinterpret_cast<ulonglong2*>(reinterpret_cast<uint8_t*>(b.out) + slot * b.prep_rb);
+            if (b.prep_rb == 32) o[1] = make_ulonglong2(0ull, PREP_HOLE32 << 48);
+            else o[2] = make_ulonglong2(0ull, (unsigned long long)PREP_HOLE);
+        }
     }
 }
 
+// RB: bytes of a prepared re-issue record written for a declined record (32: implicit value 1)
+template <int RB>
 __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, stream::CtaState& S, bool act, uint64_t w0,
                                              uint64_t w1, uint64_t h, uint64_t s, uint64_t v, uint32_t len, uint32_t g,
                                              uint32_t gl, bool inj, bool& w_full, bool& w_quiet, PrepCursor& pc) {
@@ -706,10 +712,14 @@ __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, strea
         const unsigned long long base = pc.base + pc.used + __popc(pm & lanemask_lt());
         pc.used += k;
         if (act && res == R_POST && base < b.out_cap) {
-            ulonglong2* o = reinterpret_cast<ulonglong2*>(b.out + base);
+            ulonglong2* o = reinterpret_cast<ulonglong2*>(reinterpret_cast<uint8_t*>(b.out) + base * RB);
             o[0] = make_ulonglong2(w0, w1);
-            o[1] = make_ulonglong2(h, s);
-            o[2] = make_ulonglong2(v, (unsigned long long)len);
+            if (RB == 32) {  // implicit value 1: {key words, hash, offset | length << 48}
+                o[1] = make_ulonglong2(h, s | ((unsigned long long)len << 48));
+            } else {
+                o[1] = make_ulonglong2(h, s);
+                o[2] = make_ulonglong2(v, (unsigned long long)len);
+            }
         }
     }
     if (pend) {
@@ -744,11 +754,12 @@ __device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, str
         const uint32_t ll = Q.ll[k];
         len = ll >> 5; gl = ll & 31u;
     }
-    resolve_core(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
+    resolve_core<VALS ? 48 : 32>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
 }
 
 // Reinsert pass of sepo_run (a9 re-issue): the prepared records of the previous pass, 32 per warp
 // step, straight into resolve_core (keys of these passes are the Zipf tail: no hot set).
+template <int RB>
 __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
     __shared__ stream::CtaState S;
     const uint32_t tid = threadIdx.x, lane = lane_id();
@@ -767,12 +778,23 @@ __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
         const uint64_t i = base + lane;
         ulonglong2 r0 = make_ulonglong2(0, 0), r1 = make_ulonglong2(0, 0), r2 = make_ulonglong2(1, 0);
         if (i < b.n) {
-            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(b.prep + i);
-            r0 = __ldcs(p); r1 = __ldcs(p + 1); r2 = __ldcs(p + 2);
+            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(reinterpret_cast<const uint8_t*>(b.prep) + i * RB);
+            r0 = __ldcs(p); r1 = __ldcs(p + 1);
+            if (RB == 48) r2 = __ldcs(p + 2);
         }
-        const bool act = i < b.n && (uint32_t)r2.y != PREP_HOLE;
-        resolve_core(d, b, S, act, r0.x, r0.y, r1.x, r1.y, r2.x, act ? (uint32_t)r2.y : 0u, (uint32_t)(i >> 5),
-                     (uint32_t)(i & 31), inj, w_full, w_quiet, pc);
+        uint64_t s = r1.y, v = r2.x;
+        uint32_t len = (uint32_t)r2.y;
+        bool act;
+        if (RB == 32) {  // {w0, w1, h, s | len << 48}, value 1
+            len = (uint32_t)(r1.y >> 48);
+            s = r1.y & 0xffffffffffffull;
+            v = 1;
+            act = i < b.n && len != (uint32_t)PREP_HOLE32;
+        } else {
+            act = i < b.n && len != PREP_HOLE;
+        }
+        resolve_core<RB>(d, b, S, act, r0.x, r0.y, r1.x, s, v, act ? len : 0u, (uint32_t)(i >> 5), (uint32_t)(i & 31), inj,
+                     w_full, w_quiet, pc);
     }
     if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
     __syncthreads();
@@ -2018,10 +2040,37 @@ __global__ void init_state_kernel(Dev d, uint32_t n_slots) {
     }
 }
 
+// Eviction gather copy (a10): evicted pages -> one contiguous pinned host region, page k of the
+// evict list at dst + k * page_bytes. The host arena is page-locked and mapped (UVA), so SM stores
+// cross the host link directly: one launch per eviction however fragmented the evict list is (a
+// cudaMemcpyAsync per run of consecutive pages costs microseconds per run: GROUP generations with
+// retained key pages evict 10^5 short runs). A warp copies a page with 16-byte loads/stores.
+__global__ void __launch_bounds__(512) evict_copy_kernel(const uint8_t* __restrict__ pool, const uint32_t* __restrict__ list,
+                                                      uint32_t n, uint8_t* __restrict__ dst, uint32_t page_shift) {
+    const uint32_t lane = lane_id();
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    const uint32_t per_page = (1u << page_shift) / 16;  // 16-byte units
+    for (uint64_t k = (uint64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); k < n; k += nw) {
+        const uint4* src = reinterpret_cast<const uint4*>(pool + ((uint64_t)list[k] << page_shift));
+        uint4* out = reinterpret_cast<uint4*>(dst + (k << page_shift));
+        uint32_t u = lane;
+        for (; u + 96 < per_page; u += 128) {
+            const uint4 a = __ldcg(src + u), b = __ldcg(src + u + 32), c = __ldcg(src + u + 64), e = __ldcg(src + u + 96);
+            __stcs(out + u, a); __stcs(out + u + 32, b); __stcs(out + u + 64, c); __stcs(out + u + 96, e);
+        }
+        for (; u < per_page; u += 32) __stcs(out + u, __ldcg(src + u));
+    }
+}
+
 }  // namespace sepo
 
 // ================================================================ launchers
 using namespace sepo;
+
+int sepo_launch_evict_copy(const Dev& d, uint32_t n, uint8_t* dst, int grid, cudaStream_t s) {
+    if (n) evict_copy_kernel<<<grid, 512, 0, s>>>(d.pool, d.evict_list, n, dst, d.page_shift);
+    return cudaGetLastError();
+}
 
 int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
                        uint32_t halt_slots) {
@@ -2106,7 +2155,9 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
     return cudaGetLastError();
 }
 int sepo_launch_reinsert(const Dev& d, const Batch& b, int grid, cudaStream_t s) {
-    if (b.n) reinsert_kernel<<<grid, 1024, 0, s>>>(d, b);
+    if (b.n == 0) return cudaGetLastError();
+    if (b.prep_rb == 32) reinsert_kernel<32><<<grid, 1024, 0, s>>>(d, b);
+    else reinsert_kernel<48><<<grid, 1024, 0, s>>>(d, b);
     return cudaGetLastError();
 }
 size_t sepo_hot_scratch_bytes() {

@@ -31,6 +31,8 @@ struct Batch {
     unsigned long long* out_n = nullptr;
     uint64_t out_cap = 0;
     const PRec* prep = nullptr;
+    uint32_t prep_rb = 48;  // bytes per prepared record: 48 (PRec), or 32 when every value is 1:
+                            // {w0, w1, h, s | len << 48} (a third less re-issue traffic)
 };
 }  // namespace sepo
 
@@ -53,6 +55,7 @@ uint64_t sepo_partition_tiles(uint64_t n);
 int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const uint64_t* seg_base, uint32_t n_segs,
                               uint64_t total, cudaStream_t s);
 int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);
+int sepo_launch_evict_copy(const sepo::Dev& d, uint32_t n, uint8_t* dst, int grid, cudaStream_t s);
 int sepo_launch_classify(const sepo::Dev& d, int honor_retain, cudaStream_t s);
 int sepo_launch_relink(const sepo::Dev& d, cudaStream_t s);
 int sepo_launch_init(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);

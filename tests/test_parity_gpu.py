@@ -343,3 +343,19 @@ def test_group_variable_values_vs_oracle(cuda, ratio):
     assert_same(got, exp)
     if ratio > 1:
         assert passes >= 2
+
+
+@pytest.mark.parametrize("cfg", ["C1", "C4"])
+@pytest.mark.parametrize("evk", ["0", "1"])
+def test_evict_copy_paths(cuda, monkeypatch, cfg, evk):
+    """evicted pages leave through cudaMemcpyAsync per run of consecutive pages (0) or through the
+    gather-copy kernel into one contiguous pinned region (1): identical page images, results"""
+    monkeypatch.setenv("SEPO_EVICT_KERNEL", evk)
+    s = gen.config(cfg, scale=0.25 if cfg == "C1" else 2e-4)
+    inp = device_inputs(s)
+    exp = oracle_expected(s)
+    kw = {} if cfg == "C1" else dict(mode=sepo().GROUP, fixed_val_width=4)
+    F, P = budget_pages(s, 3, 1 << 14, 4096, inp, **kw)
+    got, passes, st = run_job(s, sepo().budget_for(1 << 14, 4096, P), 1 << 14, 4096, inputs=inp, check_dups=True, **kw)
+    assert_same(got, exp)
+    assert passes >= 3
