@@ -55,6 +55,8 @@ def lib():
         L.gen_offsets_dev.argtypes = [P, u64, u64, vp, vp, u64, vp]; L.gen_offsets_dev.restype = ctypes.c_int64
         L.gen_keys_dev.argtypes = [P, u64, u64, vp, vp, vp, vp]; L.gen_keys_dev.restype = ctypes.c_int
         L.gen_ranks_dev.argtypes = [P, u64, u64, vp, vp]; L.gen_ranks_dev.restype = ctypes.c_int
+        L.gen_text_dev.argtypes = [P, u64, u64, vp, vp, vp, vp]; L.gen_text_dev.restype = ctypes.c_int
+        L.gen_text_host.argtypes = [P, u64, u64, vp, vp, vp]
         _LIB = L
     return _LIB
 
@@ -159,6 +161,28 @@ class Stream:
                             vals.data_ptr() if vals is not None else None, ctypes.c_void_p(s.cuda_stream))
         assert rc == 0, rc
         return keys[:total], offs, vals
+
+    def text_host(self, j0=0, cnt=None):
+        """Raw text of a word/URL stream: each key followed by one separator (' ' or '\n')."""
+        keys, offs, _ = self.host(j0, cnt)
+        n = len(offs) - 1
+        text = np.empty(len(keys) + n, dtype=np.uint8)
+        lib().gen_text_host(ctypes.byref(self.params()), j0, n, _ptr(np.ascontiguousarray(offs, dtype=np.uint64)),
+                            _ptr(keys), _ptr(text))
+        return text
+
+    def text_device(self, j0=0, cnt=None, device="cuda"):
+        """Raw text on the device (16-byte aligned torch allocation), same bytes as text_host."""
+        import torch
+        keys, offs, _ = self.device(j0, cnt, device)
+        n = offs.numel() - 1
+        text = torch.empty(keys.numel() + n, dtype=torch.uint8, device=device)
+        s = torch.cuda.current_stream(device)
+        rc = lib().gen_text_dev(ctypes.byref(self.params(device)), j0, n, offs.data_ptr(), keys.data_ptr(),
+                                text.data_ptr(), ctypes.c_void_p(s.cuda_stream))
+        assert rc == 0, rc
+        del keys, offs
+        return text
 
     def ranks_host(self, j0=0, cnt=None):
         if cnt is None:

@@ -147,6 +147,12 @@ GEN_HD void gen_url_spell(const gen_params* p, uint64_t r, uint32_t L, uint8_t* 
     for (; q < L; ++q) out[q] = (uint8_t)b36[gen_mix64(h ^ (uint64_t)q) % 36];
 }
 
+/* ---- raw text (word streams): the separator written after word j — '\n' with p = 1/10, else
+ * ' ' (SURVEY §8(d) C1 recipe) — so record j's word starts at text byte offs[j] + j ---- */
+GEN_HD uint8_t gen_text_sep(const gen_params* p, uint64_t j) {
+    return (gen_rnd(p->seed, 0x7e47ULL, j) % 10 == 0) ? (uint8_t)'\n' : (uint8_t)' ';
+}
+
 /* ---- PAIRS: key = splitmix64 finalizer of rank (bijective on u64), value = lo32 random ---- */
 GEN_HD uint64_t gen_pair_key(uint64_t r) { return gen_mix64(r); }
 GEN_HD uint64_t gen_pair_val(const gen_params* p, uint64_t j) { return gen_rnd(p->seed, GEN_S_VAL, j) & 0xffffffffULL; }

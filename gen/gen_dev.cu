@@ -31,6 +31,14 @@ __global__ void k_ranks(gen_params p, uint64_t j0, uint64_t cnt, uint64_t* ranks
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < cnt; i += (uint64_t)gridDim.x * blockDim.x)
         ranks[i] = gen_rank(&p, j0 + i);
 }
+// raw text of records [j0, j0+cnt): word j (CSR keys/offs) at text[offs[i] - offs[0] + i], then its separator
+__global__ void k_text(gen_params p, uint64_t j0, uint64_t cnt, const uint64_t* offs, const uint8_t* keys, uint8_t* text) {
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < cnt; i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t o = offs[i] - offs[0], e = offs[i + 1] - offs[0];
+        for (uint64_t q = o; q < e; ++q) text[q + i] = keys[q];
+        text[e + i] = gen_text_sep(&p, j0 + i);
+    }
+}
 int grid_for(uint64_t cnt) {
     uint64_t g = (cnt + 255) / 256;
     return (int)(g < 148 * 64 ? (g ? g : 1) : 148 * 64);
@@ -54,6 +62,12 @@ int64_t gen_offsets_dev(const gen_params* p, uint64_t j0, uint64_t cnt, uint64_t
 int gen_keys_dev(const gen_params* p, uint64_t j0, uint64_t cnt, const uint64_t* offs, uint8_t* keys, uint8_t* vals, void* stream) {
     if (cnt == 0) return 0;
     k_keys<<<grid_for(cnt), 256, 0, (cudaStream_t)stream>>>(*p, j0, cnt, offs, keys, vals);
+    return cudaGetLastError() == cudaSuccess ? 0 : -2;
+}
+int gen_text_dev(const gen_params* p, uint64_t j0, uint64_t cnt, const uint64_t* offs, const uint8_t* keys, uint8_t* text,
+                 void* stream) {
+    if (cnt == 0) return 0;
+    k_text<<<grid_for(cnt), 256, 0, (cudaStream_t)stream>>>(*p, j0, cnt, offs, keys, text);
     return cudaGetLastError() == cudaSuccess ? 0 : -2;
 }
 int gen_ranks_dev(const gen_params* p, uint64_t j0, uint64_t cnt, uint64_t* ranks, void* stream) {

@@ -69,6 +69,16 @@ void gen_keys_host(const gen_params* p, uint64_t j0, uint64_t cnt, const uint64_
 int gen_num_threads(void) { return omp_get_max_threads(); }
 }
 
+// raw text of records [j0, j0+cnt) from their CSR (see gen_text_sep)
+extern "C" void gen_text_host(const gen_params* p, uint64_t j0, uint64_t cnt, const uint64_t* offs, const uint8_t* keys,
+                              uint8_t* text) {
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < (int64_t)cnt; ++i) {
+        const uint64_t o = offs[i] - offs[0], e = offs[i + 1] - offs[0];
+        for (uint64_t q = o; q < e; ++q) text[q + (uint64_t)i] = keys[q];
+        text[e + (uint64_t)i] = gen_text_sep(p, j0 + (uint64_t)i);
+    }
+}
 extern "C" void gen_doc_lens_host(uint64_t seed, uint64_t d0, uint64_t cnt, uint64_t* out) {
 #pragma omp parallel for schedule(static)
     for (int64_t i = 0; i < (int64_t)cnt; ++i) out[i] = gen_doc_len(seed, d0 + (uint64_t)i);

@@ -194,6 +194,16 @@ int sepo_export(sepo_table* t, sepo_result* out);
 int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* key_offsets, const uint8_t* vals,
                  const uint64_t* val_offsets, uint64_t n);
 
+/* Word count on RAW TEXT (the paper's WC): the whole SEPO job like
+ * sepo_run, with the tokenizer fused into the insert kernel (text is read once; no CSR). A word is
+ * a maximal run of bytes other than ' ', '\n', '\t', '\r' (reading R20); every word is a record
+ * with value 1, combined by u64 sum (COMBINE mode only, else SEPO_E_INVAL). `text` is device
+ * memory (16-byte aligned, else SEPO_E_INVAL) or host memory (staged to the device first).
+ * Returns the number of passes (evictions, the final one included) or < 0; stats.records_inserted
+ * counts the words of pass 1 plus every re-issue. A word longer than page_bytes - 32 fails the job
+ * with SEPO_E_TOOLARGE. */
+int64_t sepo_run_text(sepo_table* t, const uint8_t* text, uint64_t n_bytes);
+
 /* Drop all generations and results and start a new job with the same budget and options;
  * pinned host memory and device scratch are kept for reuse. */
 int sepo_reset(sepo_table* t);

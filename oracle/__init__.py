@@ -27,6 +27,7 @@ def lib():
         L.oracle_combine_new.restype = vp
         L.oracle_combine_free.argtypes = [vp]
         L.oracle_combine_add.argtypes = [vp, vp, vp, vp, u32, u64]
+        L.oracle_combine_add_text.argtypes = [vp, vp, u64]
         L.oracle_combine_size.argtypes = [vp, vp]; L.oracle_combine_size.restype = u64
         L.oracle_combine_result.argtypes = [vp, vp, vp, vp]
         L.oracle_combine_get.argtypes = [vp, vp, u64, vp]; L.oracle_combine_get.restype = u64
@@ -71,6 +72,12 @@ class Combine:
         n = len(offs) - 1
         v = _u8(vals) if vals is not None else None
         lib().oracle_combine_add(self.h, _p(keys), _p(offs), _p(v), val_width if v is not None else 0, n)
+        return self
+
+    def add_text(self, text):
+        """raw text: every word (maximal run of bytes other than ' ', '\n', '\t', '\r') adds 1"""
+        t = _u8(text)
+        lib().oracle_combine_add_text(self.h, _p(t), len(t))
         return self
 
     def result(self):
@@ -132,6 +139,11 @@ class Group:
 
 def combine(keys, offs, vals=None, val_width=0):
     return Combine().add(keys, offs, vals, val_width)
+
+
+def word_count_text(text):
+    """{word bytes: occurrences} of raw text (combining method, reading R20)."""
+    return Combine().add_text(text).as_dict()
 
 
 def group(keys, offs, vals, val_offs=None, val_width=0):

@@ -66,6 +66,17 @@ void oracle_combine_add(void* h, const uint8_t* keys, const uint64_t* offs, cons
     for (uint64_t i = 0; i < n; ++i) c->m[key_of(keys, offs, i)] += value_u64(vals, vw, i);
 }
 /* number of distinct keys; *key_bytes = total bytes of the distinct keys */
+/* Word count on raw text (the paper's WC; reading R20): a word is a maximal run of bytes
+ * other than ' ', '\n', '\t', '\r'; each occurrence adds 1 to its word. */
+void oracle_combine_add_text(void* h, const uint8_t* text, uint64_t n) {
+    CombineMap& m = ((Combine*)h)->m;
+    std::string word;
+    for (uint64_t i = 0; i <= n; ++i) {
+        const bool sep = i == n || text[i] == ' ' || text[i] == '\n' || text[i] == '\t' || text[i] == '\r';
+        if (!sep) { word.push_back((char)text[i]); continue; }
+        if (!word.empty()) { m[word] += 1; word.clear(); }
+    }
+}
 uint64_t oracle_combine_size(void* h, uint64_t* key_bytes) {
     Combine* c = (Combine*)h;
     c->sorted.clear();

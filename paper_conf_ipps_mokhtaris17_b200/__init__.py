@@ -62,7 +62,7 @@ E_INVAL, E_NOMEM, E_TOOLARGE, E_CUDA, E_STATE, E_NCCL = -1, -2, -3, -4, -5, -6
 POOL_DEVICE, POOL_HOST_PINNED, POOL_MANAGED = 0, 1, 2  # sepo_create_placed (include/sepo.h)
 
 # every entry point declared in include/sepo.h
-EXPORTS = ["sepo_create", "sepo_create_placed", "sepo_configure", "sepo_insert_batch", "sepo_reprobe", "sepo_compact", "sepo_evict",
+EXPORTS = ["sepo_create", "sepo_create_placed", "sepo_configure", "sepo_run_text", "sepo_insert_batch", "sepo_reprobe", "sepo_compact", "sepo_evict",
            "sepo_export", "sepo_run", "sepo_reset", "sepo_stats_get", "sepo_last_insert_ms", "sepo_destroy",
            "sepo_last_error", "sepo_version", "sepo_budget_for", "sepo_partition_scratch", "sepo_partition",
            "sepo_shift_offsets"]
@@ -89,6 +89,7 @@ def lib():
         L.sepo_evict.argtypes = [vp]; L.sepo_evict.restype = i64
         L.sepo_export.argtypes = [vp, ctypes.POINTER(Result)]; L.sepo_export.restype = ctypes.c_int
         L.sepo_run.argtypes = [vp, vp, vp, vp, vp, u64]; L.sepo_run.restype = i64
+        L.sepo_run_text.argtypes = [vp, vp, u64]; L.sepo_run_text.restype = i64
         L.sepo_reset.argtypes = [vp]; L.sepo_reset.restype = ctypes.c_int
         L.sepo_stats_get.argtypes = [vp, ctypes.POINTER(Stats)]; L.sepo_stats_get.restype = ctypes.c_int
         L.sepo_last_insert_ms.argtypes = [vp]; L.sepo_last_insert_ms.restype = ctypes.c_double
@@ -207,6 +208,14 @@ class Table:
     def run(self, keys, key_offsets, vals=None, n=None, val_offsets=None):
         n = self._n(key_offsets, keys, n)
         rc = self._L.sepo_run(self.h, _ptr(keys), _ptr(key_offsets), _ptr(vals), _ptr(val_offsets), n)
+        if rc < 0:
+            _err(rc)
+        return int(rc)
+
+    def run_text(self, text, n=None):
+        """Word count on raw text (sepo_run_text): tokenizer fused into the insert kernel."""
+        n = int(n) if n is not None else (text.numel() if hasattr(text, "numel") else len(text))
+        rc = self._L.sepo_run_text(self.h, _ptr(text), n)
         if rc < 0:
             _err(rc)
         return int(rc)

@@ -116,6 +116,7 @@ struct sepo_table {
     DevBuf idxb[2];  // sepo_run re-issue index lists (ping-pong)
     DevBuf prep[2];  // sepo_run COMBINE: prepared re-issue records (ping-pong)
     DevBuf prep_n;   // their device counters
+    DevBuf tbm;      // sepo_run_text: start bits of declined words that did not fit the prepared list
     // cuStreamWriteValue32 (driver entry point): the copy stream publishes eviction progress
     int (*write_value32)(cudaStream_t, unsigned long long, unsigned int, unsigned int) = nullptr;
     bool no_overlap = true;  // SEPO_EVICT_OVERLAP=1: the next pass starts while the copy drains
@@ -1039,6 +1040,45 @@ static bool is_device_ptr(const void* p) {
     return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
 }
 
+// Prepared re-issue passes (a9) of a COMBINE job: evict, then reinsert the `reserved` slots of
+// prep[ps] (m postponed records, kb key bytes) until nothing is postponed. <0 on error.
+static int64_t prep_passes(sepo_table* t, const Batch& cur, int ps, uint64_t reserved, uint64_t m, uint64_t kb,
+                           uint64_t prb, int64_t passes_start) {
+    const uint64_t slack = (uint64_t)t->grid * 32 * kPrepChunk;  // holes: < one chunk per warp
+    while (m > 0) {
+        const uint64_t pass = t->st.passes;
+        if (pass < SEPO_MAX_PASS_STATS) t->st.postponed_per_pass[pass] += m;
+        const uint64_t ocap = reserved + slack;  // every record may decline again
+        if (t->prep[ps ^ 1].grow(ocap * prb)) return fail(SEPO_E_NOMEM, "prepared re-issue list");
+        int64_t e = evict_impl(t, 1);
+        if (e < 0) return e;
+        Batch pb = cur;
+        pb.keys = cur.keys; pb.ko = nullptr; pb.vals = nullptr; pb.vo = nullptr; pb.idx = nullptr;
+        pb.bitmap = nullptr;
+        pb.text = 0; pb.tbm = nullptr;
+        pb.prep = (const PRec*)t->prep[ps].p;
+        pb.n = reserved;
+        pb.out = (PRec*)t->prep[ps ^ 1].p;
+        pb.out_n = (unsigned long long*)t->prep_n.p + (ps ^ 1);
+        pb.out_cap = ocap;
+        CK(t, cudaMemsetAsync(pb.out_n, 0, 8, t->stream));
+        const int64_t m2 = reinsert_impl(t, pb, kb, m);
+        if (m2 < 0) return m2;
+        if (t->h_ctrl->toolarge) return fail(SEPO_E_TOOLARGE, "record cannot fit in one page");
+        kb = t->h_ctrl->kept_key_bytes;
+        m = (uint64_t)m2;
+        if (m) {
+            CK(t, cudaMemcpyAsync(&t->h_ko[0], pb.out_n, 8, cudaMemcpyDeviceToHost, t->stream));
+            CK(t, cudaStreamSynchronize(t->stream));
+            reserved = t->h_ko[0];
+        }
+        if (reserved > ocap) return fail(SEPO_E_STATE, "prepared re-issue list overflow");
+        ps ^= 1;
+        if (t->st.passes - passes_start > 100000) return fail(SEPO_E_STATE, "no progress");
+    }
+    return 0;
+}
+
 int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
                  uint64_t n) {
     trace("run begin", n);
@@ -1119,39 +1159,8 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
         }
         if (cur.out && reserved <= cur.out_cap) {
             // prepared re-issue: reinsert passes until nothing is postponed
-            int ps = 0;
-            uint64_t m = (uint64_t)c;
-            const uint64_t slack = (uint64_t)t->grid * 32 * kPrepChunk;  // holes: < one chunk per warp
-            while (m > 0) {
-                const uint64_t pass = t->st.passes;
-                if (pass < SEPO_MAX_PASS_STATS) t->st.postponed_per_pass[pass] += m;
-                const uint64_t ocap = reserved + slack;  // every record may decline again
-                if (t->prep[ps ^ 1].grow(ocap * prb)) return fail(SEPO_E_NOMEM, "prepared re-issue list");
-                int64_t e = evict_impl(t, 1);
-                if (e < 0) return e;
-                Batch pb = cur;
-                pb.keys = cur.keys; pb.ko = nullptr; pb.vals = nullptr; pb.vo = nullptr; pb.idx = nullptr;
-                pb.bitmap = nullptr;
-                pb.prep = (const PRec*)t->prep[ps].p;
-                pb.n = reserved;
-                pb.out = (PRec*)t->prep[ps ^ 1].p;
-                pb.out_n = (unsigned long long*)t->prep_n.p + (ps ^ 1);
-                pb.out_cap = ocap;
-                CK(t, cudaMemsetAsync(pb.out_n, 0, 8, t->stream));
-                const int64_t m2 = reinsert_impl(t, pb, kb, m);
-                if (m2 < 0) return m2;
-                if (t->h_ctrl->toolarge) return fail(SEPO_E_TOOLARGE, "record cannot fit in one page");
-                kb = t->h_ctrl->kept_key_bytes;
-                m = (uint64_t)m2;
-                if (m) {
-                    CK(t, cudaMemcpyAsync(&t->h_ko[0], pb.out_n, 8, cudaMemcpyDeviceToHost, t->stream));
-                    CK(t, cudaStreamSynchronize(t->stream));
-                    reserved = t->h_ko[0];
-                }
-                if (reserved > ocap) return fail(SEPO_E_STATE, "prepared re-issue list overflow");
-                ps ^= 1;
-                if (t->st.passes - passes_start > 100000) return fail(SEPO_E_STATE, "no progress");
-            }
+            const int64_t r = prep_passes(t, cur, 0, reserved, (uint64_t)c, kb, prb, passes_start);
+            if (r < 0) return r;
             break;
         }
         cur.out = nullptr;  // index re-issue from here on
@@ -1195,6 +1204,117 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
     }
     CK(t, cudaStreamSynchronize(t->copy_stream));
     trace("run end", t->st.passes - passes_start);
+    return (int64_t)t->st.passes - passes_start;
+}
+
+// ---------------------------------------------------------------- raw-text word count (NEXT-2)
+// The whole SEPO job on raw text (COMBINE, value 1 per word): pass 1 tokenizes and inserts in one
+// kernel (insert_text_kernel); declined words become prepared records (their text offsets); later
+// passes are the ordinary reinsert passes. Words declined after the prepared list filled up set
+// their start bit in a text bitmap and are converted to prepared records after pass 1.
+int64_t sepo_run_text(sepo_table* t, const uint8_t* text, uint64_t n_bytes) {
+    trace("run_text begin", n_bytes);
+    int rc = check_active(t);
+    if (rc) return rc;
+    if (t->opts.mode != SEPO_COMBINE_SUM_U64) return fail(SEPO_E_INVAL, "sepo_run_text needs COMBINE mode");
+    if (n_bytes && !text) return fail(SEPO_E_INVAL, "text is NULL");
+    if (n_bytes == 0) {
+        if (t->dirty) { int64_t e = evict_impl(t, 0); if (e < 0) return e; }
+        return 0;
+    }
+    if (!is_device_ptr(text)) {  // host text: one staged H2D (P:L227 counts this transfer)
+        auto t0 = std::chrono::steady_clock::now();
+        if (t->in_stage[0].grow(n_bytes + 16)) return fail(SEPO_E_NOMEM, "device staging for host text");
+        CK(t, cudaMemcpyAsync(t->in_stage[0].p, text, n_bytes, cudaMemcpyHostToDevice, t->stream));
+        CK(t, cudaStreamSynchronize(t->stream));
+        t->st.t_h2d_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+        return sepo_run_text(t, (const uint8_t*)t->in_stage[0].p, n_bytes);
+    }
+    if ((uintptr_t)text & 15) return fail(SEPO_E_INVAL, "device text must be 16-byte aligned");
+    const int64_t passes_start = (int64_t)t->st.passes;
+    Batch cur{};
+    cur.keys = text;
+    cur.n = n_bytes;
+    cur.text = 1;
+    cur.prep_rb = 32;
+    // prepared list for pass 1 (a word is >= 2 bytes with its separator; ~n/32 slots = a quarter of
+    // 8-byte words), the overflow bitmap over the text bytes (zero between uses)
+    uint64_t cap = std::max<uint64_t>(1ull << 16, n_bytes / 32);
+    if (const char* pc = getenv("SEPO_PREP_CAP")) cap = strtoull(pc, nullptr, 10);
+    const uint64_t tbm_bytes = ((n_bytes + 31) / 32) * 4;
+    if (t->prep_n.grow(64) || t->prep[0].grow(std::max<uint64_t>(cap, 1) * 32)) return fail(SEPO_E_NOMEM, "prepared list");
+    if ((size_t)t->tbm.cap < tbm_bytes) {
+        if (t->tbm.grow(tbm_bytes)) return fail(SEPO_E_NOMEM, "text overflow bitmap");
+        CK(t, cudaMemsetAsync(t->tbm.p, 0, t->tbm.cap, t->stream));
+    }
+    CK(t, cudaMemsetAsync(t->prep_n.p, 0, 16, t->stream));
+    cur.out = (PRec*)t->prep[0].p;
+    cur.out_n = (unsigned long long*)t->prep_n.p;
+    cur.out_cap = cap;
+    cur.tbm = (uint32_t*)t->tbm.p;
+    // ---- pass 1: fused tokenize + insert
+    t->inserted = true;
+    t->dirty = true;
+    ++t->batch_seq;
+    sync_dev(t);
+    if ((rc = zero_ctrl_counters(t))) return rc;
+    CK(t, cudaMemsetAsync(&t->d.ctrl->text_words, 0, 8, t->stream));
+    CK(t, cudaEventRecord(t->ev0, t->stream));
+    if (t->hot.grow(sepo_hot_scratch_bytes())) return fail(SEPO_E_NOMEM, "hot-set scratch");
+    rc = sepo_launch_insert_text(t->d, cur, t->grid, t->stream, t->hot.p);
+    if (rc) return cuda_check(t, (cudaError_t)rc, "text insert kernel launch");
+    CK(t, cudaEventRecord(t->ev1, t->stream));
+    t->st.kernel_launches += (n_bytes >= (64ull << 18)) ? 7 : 1;
+    CK(t, cudaMemcpyAsync(&t->h_ko[0], cur.out_n, 8, cudaMemcpyDeviceToHost, t->stream));
+    if ((rc = read_ctrl(t))) return rc;
+    t->last_insert_ms = elapsed_ms(t->ev0, t->ev1);
+    t->st.t_insert_ms += t->last_insert_ms;
+    if (t->st.passes < SEPO_MAX_PASS_STATS) t->st.t_insert_ms_per_pass[t->st.passes] += t->last_insert_ms;
+    t->st.insert_calls++;
+    t->st.records_inserted += t->h_ctrl->text_words;
+    t->st.key_bytes_inserted += n_bytes;
+    t->st.dead_bytes += t->h_ctrl->dead_bytes;
+    {
+        const uint64_t used = std::min<uint64_t>(t->h_ctrl->pool_taken, t->d.n_free) + t->pages_resident_retained;
+        t->st.pages_used_max = std::max<uint64_t>(t->st.pages_used_max, used);
+    }
+    if (t->h_ctrl->toolarge) {
+        t->st.toolarge += t->h_ctrl->toolarge;
+        return fail(SEPO_E_TOOLARGE, std::to_string(t->h_ctrl->toolarge) + " word(s) cannot fit in one page");
+    }
+    const uint64_t c = t->h_ctrl->postponed;
+    uint64_t kb = t->h_ctrl->kept_key_bytes;
+    uint64_t reserved = t->h_ko[0];
+    int ps = 0;
+    if (c > 0 && reserved > cap) {
+        // overflow: the first `cap` slots hold prepared records, the other declined words are
+        // bits of tbm -> copy the list to prep[1] and append one record per bit behind it
+        const uint64_t slack = (uint64_t)t->grid * 32 * kPrepChunk;
+        if (t->prep[1].grow((cap + c + slack) * 32)) return fail(SEPO_E_NOMEM, "prepared list (overflow)");
+        CK(t, cudaMemcpyAsync(t->prep[1].p, t->prep[0].p, cap * 32, cudaMemcpyDeviceToDevice, t->stream));
+        unsigned long long* counter = (unsigned long long*)t->prep_n.p + 2;
+        t->h_ko[0] = cap;
+        CK(t, cudaMemcpyAsync(counter, &t->h_ko[0], 8, cudaMemcpyHostToDevice, t->stream));
+        Batch bb = cur;
+        bb.out = (PRec*)t->prep[1].p;
+        rc = sepo_launch_text_bits(t->d, bb, counter, t->stream);
+        if (rc) return cuda_check(t, (cudaError_t)rc, "text bits kernel");
+        t->st.kernel_launches += 1;
+        CK(t, cudaMemcpyAsync(&t->h_ko[0], counter, 8, cudaMemcpyDeviceToHost, t->stream));
+        CK(t, cudaStreamSynchronize(t->stream));
+        reserved = t->h_ko[0];
+        ps = 1;
+    }
+    if (c > 0) {
+        const int64_t r = prep_passes(t, cur, ps, reserved, c, kb, 32, passes_start);
+        if (r < 0) return r;
+    }
+    if (t->dirty) {
+        int64_t e = evict_impl(t, 0);
+        if (e < 0) return e;
+    }
+    CK(t, cudaStreamSynchronize(t->copy_stream));
+    trace("run_text end", t->st.passes - passes_start);
     return (int64_t)t->st.passes - passes_start;
 }
 
@@ -1245,6 +1365,7 @@ void sepo_destroy(sepo_table* t) {
     t->prep[0].release();
     t->prep[1].release();
     t->prep_n.release();
+    t->tbm.release();
     t->bm.release();
     for (auto& s : t->buf)
         for (auto& b : s) b.release();

@@ -55,7 +55,8 @@ struct Ctrl {
     unsigned long long n_safe;         // evict: free pages that need no copy (never used last generation)
     unsigned int copied;               // evicted pages whose D2H copy finished (written by the copy stream)
     unsigned int failed_slots;         // BASIC: allocator slots whose allocation failed this generation
-    unsigned long long pad[4];
+    unsigned long long text_words;     // sepo_run_text: words tokenized by the last insert call
+    unsigned long long pad[3];
 };
 
 struct Dev {

@@ -36,7 +36,24 @@ __device__ __forceinline__ uint64_t rec_value(const Batch& b, uint64_t i) {
         default: return ld_in8(b.vals + i);
     }
 }
+// ---- raw text (NEXT-2, reading R20): a word is a maximal run of bytes other than ' ', '\n', '\t',
+// '\r'; in text batches record i is the word starting at byte i.
+__device__ __forceinline__ bool is_sep(uint32_t c) { return c == 0x20u || c == 0x0au || c == 0x09u || c == 0x0du; }
+__device__ __forceinline__ uint32_t text_word_len(const uint8_t* t, uint64_t n, uint64_t s) {
+    uint64_t e = s;
+    while (e < n && !is_sep(ld_in8(t + e))) ++e;
+    const uint64_t L = e - s;
+    return L > 0xffffffffull ? 0xffffffffu : (uint32_t)L;
+}
+// first word start at or after byte i (n if none)
+__device__ __forceinline__ uint64_t text_next_word(const uint8_t* t, uint64_t n, uint64_t i) {
+    if (i > 0 && i < n && !is_sep(ld_in8(t + i - 1)))  // inside a word: skip to its end
+        while (i < n && !is_sep(ld_in8(t + i))) ++i;
+    while (i < n && is_sep(ld_in8(t + i))) ++i;
+    return i;
+}
 __device__ __forceinline__ void rec_key(const Batch& b, uint64_t i, uint64_t& s, uint32_t& len) {
+    if (b.text) { s = i; len = text_word_len(b.keys, b.n, i); return; }
     i = rec_index(b, i);
     if (b.ko) {
         s = ld_in64(b.ko + i);
@@ -167,7 +184,7 @@ struct Entry {                   // one hot key (global list, built by hot_selec
 // buckets are full, the key left out is one of the least frequent ones, never a Zipf head
 // (losing a head key sends a few % of all records to one global address).
 __device__ __forceinline__ int count_class(uint32_t c) { return 31 - __clz(c | 1u); }
-struct SampleSlot { unsigned long long h; unsigned int count, rec; };
+struct SampleSlot { unsigned long long h; unsigned int count, pad; unsigned long long rec; };
 }  // namespace hot
 
 __device__ __forceinline__ void red_add_u64(unsigned long long* p, unsigned long long v) {
@@ -191,14 +208,18 @@ __device__ __forceinline__ void rec_hash16(const Dev& d, const Batch& b, uint64_
 __global__ void __launch_bounds__(256) hot_sample_kernel(Dev d, Batch b, uint64_t stride, uint64_t n_sample,
                                                          hot::SampleSlot* tab) {
     for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < n_sample; j += (uint64_t)gridDim.x * blockDim.x) {
-        const uint64_t i = j * stride;
+        uint64_t i = j * stride;
+        if (b.text) {  // the first word starting at or after the sampled byte
+            i = text_next_word(b.keys, b.n, i);
+            if (i >= b.n) continue;
+        }
         uint64_t s, w0, w1, h; uint32_t len;
         rec_hash16(d, b, i, s, len, w0, w1, h);
         const unsigned long long key = h | 1ull;  // 0 marks an empty slot
         uint32_t pos = (uint32_t)(h >> 20) & (hot::SAMPLE_SLOTS - 1);
         for (int probe = 0; probe < 32; ++probe) {
             const unsigned long long cur = atomicCAS(&tab[pos].h, 0ull, key);
-            if (cur == 0ull) { tab[pos].rec = (unsigned)(i & 0xffffffffu); atomicAdd(&tab[pos].count, 1u); break; }
+            if (cur == 0ull) { tab[pos].rec = i; atomicAdd(&tab[pos].count, 1u); break; }
             if (cur == key) { atomicAdd(&tab[pos].count, 1u); break; }
             pos = (pos + 1) & (hot::SAMPLE_SLOTS - 1);
         }
@@ -711,6 +732,8 @@ __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, strea
         }
         const unsigned long long base = pc.base + pc.used + __popc(pm & lanemask_lt());
         pc.used += k;
+        if (act && res == R_POST && base >= b.out_cap && b.tbm)  // text: the list is full, mark the word
+            atomicOr(b.tbm + (s >> 5), 1u << (s & 31));
         if (act && res == R_POST && base < b.out_cap) {
             ulonglong2* o = reinterpret_cast<ulonglong2*>(reinterpret_cast<uint8_t*>(b.out) + base * RB);
             o[0] = make_ulonglong2(w0, w1);
@@ -856,22 +879,34 @@ __global__ void __launch_bounds__(1024, 1) insert_basic_kernel(Dev d, Batch b, u
             if (declined) res = R_POST;
             if (__any_sync(FULLMASK, declined) && lane == 0 && atomicExch(&s_failed, 1) == 0)
                 atomicAdd(&d.ctrl->failed_slots, 1u);  // this slot (bucket group) failed
-            if (need && off != ~0ull) {
-                uint8_t* e = d.pool + off;
-                const uint32_t bkt = bucket_of(h, d.n_buckets);
-                uint32_t head = ld_dir(d.dir + bkt);
-                *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_BASIC, head, tag_of(h), len);
+            // link: the warp's new entries of one bucket form a sub-chain (lane order) that one
+            // CAS puts at the head — duplicates of a Zipf head key would otherwise serialise on
+            // one directory word, one CAS each
+            const bool linking = need && off != ~0ull;
+            const uint32_t bkt = bucket_of(h, d.n_buckets);
+            const unsigned grp = __match_any_sync(FULLMASK, linking ? (unsigned long long)bkt : (1ull << 32) | lane);
+            uint8_t* e = d.pool + (linking ? off : 0ull);
+            const uint32_t me = linking ? off_ref(off) : 0u;
+            const unsigned above = grp & ~((2u << lane) - 1u);           // group lanes after me
+            const uint32_t nxt_lane = above ? (uint32_t)(__ffs(above) - 1) : lane;
+            const uint32_t nxt_ref = __shfl_sync(FULLMASK, me, nxt_lane);
+            const uint32_t leader = (uint32_t)(__ffs(grp) - 1), tail_lane = 31u - __clz(grp);
+            if (linking) {
+                *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_BASIC, above ? nxt_ref : 0u, tag_of(h), len);
                 if (len > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0;
                 if (len > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1;
                 if (len > 16) store_key(e + KEY_OFF + 16, b.keys + s + 16, len - 16);
                 *reinterpret_cast<unsigned long long*>(entry_val(e, len)) = v;
-                const uint32_t me = off_ref(off);
-                while (true) {  // lock-free head insertion; duplicates are allowed
-                    const uint32_t old = cas_release(d.dir + bkt, head, me);
-                    if (old == head) break;
-                    head = old;
-                    *reinterpret_cast<uint32_t*>(e + 4) = head;
-                }
+                __threadfence();
+            }
+            const unsigned long long tail_e = __shfl_sync(FULLMASK, (unsigned long long)(uintptr_t)e, tail_lane);
+            __syncwarp();
+            if (linking && lane == leader) {
+                // head insertion by exchange: nothing reads a BASIC chain while the batch
+                // is inserted (no key is looked up; export parses pages), so the tail's link may
+                // follow the exchange — one atomic per sub-chain, no CAS retries on a hot bucket
+                const uint32_t old = atomicExch(d.dir + bkt, me);
+                *reinterpret_cast<uint32_t*>((uint8_t*)(uintptr_t)tail_e + 4) = old;
             }
         }
         // outcomes -> the group's bitmap word (this warp owns it) + counts (a7)
@@ -2040,6 +2075,278 @@ __global__ void init_state_kernel(Dev d, uint32_t n_slots) {
     }
 }
 
+// ================================================================ fused tokenizer + COMBINE insert (NEXT-2)
+// Word count on raw text (reading R20): the text is read once, in 512-byte
+// windows (a 16-byte chunk per lane), instead of text -> CSR -> insert. Per window a warp computes the
+// separator bits of its bytes, the word starts (a non-separator byte after a separator), their
+// warp-wide prefix count and a list of start offsets in shared memory; then it takes the window's
+// words 32 at a time, one per lane: the end is the first separator bit at or after the start in
+// the [window | next window] bitmap, the first 16 key bytes come from the two-window text ring in
+// shared memory, and from there on the word is a record of the COMBINE stream kernel (hash, hot
+// set, warp fold, miss queue, resolve_core with value 1). A word belongs to the window it starts
+// in; one that runs past the next window (> 512 B) is measured in global memory. Declined words
+// go to the prepared re-issue list (key offset = the word's text offset), or — if the list is
+// full — set their start bit in b.tbm for the host to convert into prepared records.
+namespace textk {
+constexpr int THREADS = 1024, WARPS = THREADS / 32;
+constexpr int WB = 512;    // window bytes: 32 lanes x 16 B
+constexpr int CHW = 64;    // consecutive windows a warp streams before it strides
+constexpr int DSZ = 8192;  // hot slots (the text ring takes the room of half the CSR kernel's slots)
+__device__ __forceinline__ uint32_t ds1(uint64_t h) { return (uint32_t)(h >> 3) & (DSZ - 1); }
+__device__ __forceinline__ uint32_t ds2(uint64_t h) { return (uint32_t)(h >> 17) & (DSZ - 1); }
+struct WarpText {
+    uint4 t[2][32];         // text ring: two consecutive windows
+    uint32_t sep[2][16];    // separator bits, bit j of word k = byte 32k + j of the window
+    uint16_t wp[WB / 2];    // word start offsets of the current window
+};
+struct Smem {
+    uint32_t tags[DSZ];
+    ulonglong2 kw[hot::K];
+    uint32_t ref[hot::K];
+    unsigned int sum[hot::K];
+    stream::Smem<false, WARPS>::Queue q[WARPS];
+    WarpText w[WARPS];
+    stream::CtaState cs;
+};
+// 16 separator bits of a 16-byte chunk (bytes past `valid` count as separators)
+__device__ __forceinline__ uint32_t sep16(uint4 c, uint32_t valid) {
+    const uint32_t wv[4] = {c.x, c.y, c.z, c.w};
+    uint32_t out = 0;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const uint32_t w = wv[k];
+        uint32_t m = __vcmpeq4(w, 0x20202020u) | __vcmpeq4(w, 0x0a0a0a0au) | __vcmpeq4(w, 0x09090909u) |
+                     __vcmpeq4(w, 0x0d0d0d0du);
+        m &= 0x01010101u;
+        out |= ((m * 0x10204080u) >> 28) << (4 * k);  // byte k -> bit k (distinct partial products)
+    }
+    if (valid < 16) out |= (0xffffu << valid) & 0xffffu;
+    return out;
+}
+// the lane's 16-byte chunk of window `win` (zeros past the end of the text)
+__device__ __forceinline__ uint4 load_chunk(const uint8_t* T, uint64_t n, uint64_t win, uint32_t lane, uint32_t& valid) {
+    const uint64_t a = win * WB + 16ull * lane;
+    if (a + 16 <= n) { valid = 16; return ld_in128(T + a); }
+    valid = a < n ? (uint32_t)(n - a) : 0u;
+    uint32_t by[16];
+#pragma unroll
+    for (int j = 0; j < 16; ++j) by[j] = (uint32_t)j < valid ? ld_in8(T + a + j) : 0u;
+    return make_uint4(by[0] | by[1] << 8 | by[2] << 16 | by[3] << 24, by[4] | by[5] << 8 | by[6] << 16 | by[7] << 24,
+                      by[8] | by[9] << 8 | by[10] << 16 | by[11] << 24, by[12] | by[13] << 8 | by[14] << 16 | by[15] << 24);
+}
+// stage a chunk into ring slot `slot`: text bytes + the window's separator bits
+__device__ __forceinline__ void stage(WarpText& W, uint32_t slot, uint32_t lane, uint4 ch, uint32_t valid) {
+    W.t[slot][lane] = ch;
+    const uint32_t sp = sep16(ch, valid);
+    const uint32_t other = __shfl_down_sync(FULLMASK, sp, 1);
+    if (!(lane & 1)) W.sep[slot][lane >> 1] = sp | (other << 16);
+}
+}  // namespace textk
+
+__global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, Batch b, const hot::Entry* hl,
+                                                                         const unsigned int* n_hot) {
+    using namespace textk;
+    extern __shared__ __align__(16) uint8_t smem_raw[];
+    textk::Smem& S = *reinterpret_cast<textk::Smem*>(smem_raw);
+    const uint32_t tid = threadIdx.x, lane = lane_id(), wid = tid >> 5;
+    for (int p = tid; p < hot::K; p += THREADS) { S.ref[p] = 0; S.sum[p] = 0; }
+    for (int p = tid; p < DSZ; p += THREADS) S.tags[p] = 0u;
+    if (tid == 0) {
+        S.cs.cur[0] = d.cursors[2 * blockIdx.x];
+        S.cs.cur[1] = d.cursors[2 * blockIdx.x + 1];
+        S.cs.post = 0; S.cs.toolarge = 0; S.cs.dead = 0; S.cs.pkb = 0;
+    }
+    if (tid < 32) { S.cs.wpost[tid] = 0; S.cs.wpkb[tid] = 0; }
+    __syncthreads();
+    const unsigned nh = hl ? *n_hot : 0u;
+    for (int cls = 31; cls >= 0 && nh; --cls) {  // hot set, most frequent keys first (as the CSR kernel)
+        for (unsigned j = tid; j < nh && j < (unsigned)hot::K; j += THREADS) {
+            const hot::Entry e = hl[j];
+            if (e.ref == 0 || hot::count_class(e.count) != cls) continue;
+            const uint32_t f = stream::dfp(e.h, e.len) | j;
+            if (atomicCAS(&S.tags[ds1(e.h)], 0u, f) == 0u || atomicCAS(&S.tags[ds2(e.h)], 0u, f) == 0u) {
+                S.kw[j] = make_ulonglong2(e.w0, e.w1);
+                S.ref[j] = e.ref;
+            }
+        }
+        __syncthreads();
+    }
+    __syncthreads();
+    const bool have_hot = nh > 0;
+    const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
+    const uint8_t* T = b.keys;
+    const uint64_t n = b.n;
+    const uint64_t nwin = (n + WB - 1) / WB;
+    const bool big = n / 2 >= (1ull << 32);  // words < 2^32: a CTA-local count cannot wrap
+    WarpText& W = S.w[wid];
+    auto& Q = S.q[wid];
+    uint32_t qhead = 0, qtail = 0;
+    PrepCursor pc;
+    bool w_full = false, w_quiet = false;
+    unsigned long long words = 0;  // lane 0
+    const uint8_t* ring = reinterpret_cast<const uint8_t*>(&W.t[0][0]);
+    const uint64_t nwarps = (uint64_t)gridDim.x * WARPS;
+    for (uint64_t c0 = ((uint64_t)blockIdx.x * WARPS + wid) * CHW; c0 < nwin; c0 += nwarps * CHW) {
+        const uint64_t c1 = (c0 + CHW < nwin) ? c0 + CHW : nwin;
+        uint32_t prev = 1u;  // is the byte before the window a separator (text start: yes)
+        if (c0 > 0) prev = is_sep(ld_in8(T + c0 * WB - 1)) ? 1u : 0u;
+        uint32_t vl;
+        uint4 ch = load_chunk(T, n, c0, lane, vl);
+        stage(W, 0, lane, ch, vl);
+        uint32_t vl_n;
+        uint4 ch_n = load_chunk(T, n, c0 + 1, lane, vl_n);
+        uint32_t slot = 0;
+        for (uint64_t w = c0; w < c1; ++w) {
+            // window w+1 into the other slot (the words of w may run into it); load w+2 if ours
+            stage(W, slot ^ 1u, lane, ch_n, vl_n);
+            if (w + 2 < c1 + 1) ch_n = load_chunk(T, n, w + 2, lane, vl_n);
+            __syncwarp();
+            // ---- word starts of window w (a1): separator bits -> starts -> offsets in smem
+            const uint32_t sw = W.sep[slot][lane >> 1];
+            const uint32_t sp = (lane & 1) ? (sw >> 16) : (sw & 0xffffu);
+            const uint32_t up = __shfl_up_sync(FULLMASK, sp, 1);
+            const uint32_t pbit = lane == 0 ? prev : ((up >> 15) & 1u);
+            const uint32_t st = ~sp & ((sp << 1) | pbit) & 0xffffu;
+            prev = (__shfl_sync(FULLMASK, sp, 31) >> 15) & 1u;
+            const uint32_t cnt = __popc(st);
+            uint32_t incl = cnt;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(FULLMASK, incl, o);
+                if (lane >= (uint32_t)o) incl += y;
+            }
+            const uint32_t total = __shfl_sync(FULLMASK, incl, 31);
+            for (uint32_t m = st, k = incl - cnt; m; m &= m - 1) W.wp[k++] = (uint16_t)(lane * 16 + __ffs(m) - 1);
+            words += total;
+            __syncwarp();
+            for (uint32_t r = 0; r < total; r += 32) {
+                const uint32_t k = r + lane;
+                const bool valid = k < total;
+                const uint32_t p = valid ? W.wp[k] : 0u;
+                const uint64_t s = w * WB + p;
+                uint32_t len = 0;
+                uint64_t w0 = 0, w1 = 0;
+                if (valid) {
+                    // end: the first separator at or after p in [window w | window w+1]
+                    uint32_t wi = p >> 5;
+                    uint32_t m2 = W.sep[slot][wi] & (~0u << (p & 31));
+                    while (m2 == 0 && wi < 31) {
+                        ++wi;
+                        m2 = wi < 16 ? W.sep[slot][wi] : W.sep[slot ^ 1u][wi - 16];
+                    }
+                    len = m2 ? wi * 32 + __ffs(m2) - 1 - p : text_word_len(T, n, s);
+                    // first 16 key bytes from the ring (aligned 8-byte words, wrapping at 1 KB)
+                    const uint32_t base = slot * WB + p;
+                    const uint32_t a0 = (base & ~7u) & 1023u;
+                    const uint64_t x0 = *reinterpret_cast<const uint64_t*>(ring + a0);
+                    const uint64_t x1 = *reinterpret_cast<const uint64_t*>(ring + ((a0 + 8) & 1023u));
+                    const uint64_t x2 = *reinterpret_cast<const uint64_t*>(ring + ((a0 + 16) & 1023u));
+                    const uint32_t sh = 8u * (base & 7u);
+                    const uint64_t lo = sh ? (x0 >> sh) | (x1 << (64 - sh)) : x0;
+                    const uint64_t hi = sh ? (x1 >> sh) | (x2 << (64 - sh)) : x1;
+                    const uint32_t nb8 = 8u * min(len, 16u);
+                    w0 = lo & ~shl64_clamp(~0ull, nb8);
+                    w1 = hi & ~shl64_clamp(~0ull, nb8 > 64u ? nb8 - 64u : 0u);
+                }
+                const uint64_t h = hash_key16(len, d.seed, w0, w1, T + s);
+                // ---- hot set (a2)
+                int pos = -1;
+                if (have_hot) {
+                    const uint32_t f = stream::dfp(h, len);
+                    const uint32_t t1 = S.tags[ds1(h)], t2 = S.tags[ds2(h)];
+                    const bool m1 = (t1 & 0xfffff800u) == f, m2 = (t2 & 0xfffff800u) == f;
+                    const uint32_t q = (m1 ? t1 : t2) & 0x7ffu;
+                    if (valid && (m1 || m2)) {
+                        const ulonglong2 kk = S.kw[q];
+                        bool eq = kk.x == w0 && kk.y == w1;
+                        if (len > 16) {
+                            const uint8_t* e = ref_ptr(d, S.ref[q]);
+                            eq = eq && ldcg32(e + 12) == len && entry_key_eq(e + KEY_OFF + 16, T + s + 16, len - 16);
+                        }
+                        if (eq) pos = (int)q;
+                    }
+                }
+                const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
+                if (hm) {
+                    const unsigned grp = __match_any_sync(FULLMASK, pos >= 0 ? (unsigned)pos : (0x10000u | lane)) & hm;
+                    if (pos >= 0 && lane == (uint32_t)(__ffs(grp) - 1)) {
+                        const unsigned add = (unsigned)__popc(grp);
+                        const unsigned old = atomicAdd(&S.sum[pos], add);
+                        if (big && old + add < old)
+                            red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(ref_ptr(d, S.ref[pos]), len)), 1ull << 32);
+                    }
+                }
+                // ---- misses: the warp's queue, resolved 32 at a time (a3..a7)
+                const bool miss = valid && pos < 0;
+                const unsigned mm = __ballot_sync(FULLMASK, miss);
+                if (miss) {
+                    const uint32_t kq = (qtail + __popc(mm & lanemask_lt())) & (stream::QCAP - 1);
+                    Q.w0[kq] = w0; Q.w1[kq] = w1; Q.h[kq] = h; Q.s[kq] = s;
+                    Q.g[kq] = 0;
+                    Q.ll[kq] = (min(len, 1u << 26) << 5) | lane;
+                }
+                qtail += __popc(mm);
+                __syncwarp();
+                if (qtail - qhead >= 32) {
+                    const uint32_t kq = (qhead + lane) & (stream::QCAP - 1);
+                    const uint32_t ll = Q.ll[kq];
+                    resolve_core<32>(d, b, S.cs, true, Q.w0[kq], Q.w1[kq], Q.h[kq], Q.s[kq], 1ull, ll >> 5, 0u, ll & 31u,
+                                     inj, w_full, w_quiet, pc);
+                    qhead += 32;
+                    __syncwarp();
+                }
+            }
+            slot ^= 1u;
+        }
+    }
+    if (qtail != qhead) {
+        const bool act = lane < qtail - qhead;
+        const uint32_t kq = (qhead + lane) & (stream::QCAP - 1);
+        const uint32_t ll = act ? Q.ll[kq] : 0u;
+        resolve_core<32>(d, b, S.cs, act, act ? Q.w0[kq] : 0ull, act ? Q.w1[kq] : 0ull, act ? Q.h[kq] : 0ull,
+                         act ? Q.s[kq] : 0ull, 1ull, ll >> 5, 0u, ll & 31u, inj, w_full, w_quiet, pc);
+    }
+    if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
+    if (lane == 0 && words) atomicAdd(&d.ctrl->text_words, words);
+    __syncthreads();
+    for (int p = tid; p < hot::K; p += THREADS) {
+        if (S.ref[p] == 0 || S.sum[p] == 0) continue;
+        uint8_t* e = ref_ptr(d, S.ref[p]);
+        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(e, ldcg32(e + 12))), (unsigned long long)S.sum[p]);
+    }
+    if (tid == 0) {
+        d.cursors[2 * blockIdx.x] = S.cs.cur[0];
+        d.cursors[2 * blockIdx.x + 1] = S.cs.cur[1];
+        for (uint32_t w = 0; w < (uint32_t)WARPS; ++w) { S.cs.post += S.cs.wpost[w]; S.cs.pkb += S.cs.wpkb[w]; }
+        if (S.cs.post) atomicAdd(&d.ctrl->postponed, S.cs.post);
+        if (S.cs.toolarge) atomicAdd(&d.ctrl->toolarge, S.cs.toolarge);
+        if (S.cs.dead) atomicAdd(&d.ctrl->dead_bytes, S.cs.dead);
+        if (S.cs.pkb) atomicAdd(&d.ctrl->kept_key_bytes, S.cs.pkb);
+    }
+}
+
+// Words whose start bit is set in b.tbm (declined when the prepared list was full) -> 32-byte
+// prepared records appended at out[*counter++]; the bits are cleared for the next use.
+__global__ void __launch_bounds__(256) text_bits_kernel(Dev d, Batch b, unsigned long long* counter) {
+    const uint64_t nw = (b.n + 31) / 32;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < nw; i += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t bits = b.tbm[i];
+        if (!bits) continue;
+        b.tbm[i] = 0u;
+        for (; bits; bits &= bits - 1) {
+            const uint64_t s = i * 32 + __ffs(bits) - 1;
+            const uint32_t len = text_word_len(b.keys, b.n, s);
+            uint64_t w0, w1;
+            load_key16(b.keys + s, len, w0, w1);
+            const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
+            const unsigned long long k = atomicAdd(counter, 1ull);
+            ulonglong2* o = reinterpret_cast<ulonglong2*>(reinterpret_cast<uint8_t*>(b.out) + k * 32);
+            o[0] = make_ulonglong2(w0, w1);
+            o[1] = make_ulonglong2(h, s | ((unsigned long long)min(len, 0xfffeu) << 48));
+        }
+    }
+}
+
 // Eviction gather copy (a10): evicted pages -> one contiguous pinned host region, page k of the
 // evict list at dst + k * page_bytes. The host arena is page-locked and mapped (UVA), so SM stores
 // cross the host link directly: one launch per eviction however fragmented the evict list is (a
@@ -2066,6 +2373,40 @@ __global__ void __launch_bounds__(512) evict_copy_kernel(const uint8_t* __restri
 
 // ================================================================ launchers
 using namespace sepo;
+
+int sepo_launch_insert_text(const Dev& d, const Batch& b, int grid, cudaStream_t s, void* hot_scratch) {
+    const hot::Entry* hl = nullptr;
+    const unsigned int* nh = nullptr;
+    const uint64_t n_sample = 1ull << 18;
+    if (hot_scratch && b.n >= 64 * n_sample) {  // hot-set discovery on words at sampled byte offsets
+        uint8_t* p = reinterpret_cast<uint8_t*>(hot_scratch);
+        hot::SampleSlot* tab = reinterpret_cast<hot::SampleSlot*>(p);
+        hot::Entry* list = reinterpret_cast<hot::Entry*>(p + sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS);
+        unsigned int* n_out = reinterpret_cast<unsigned int*>(list + hot::K);
+        unsigned int* hist = n_out + 1;
+        cudaMemsetAsync(tab, 0, sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS, s);
+        cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
+        hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, b.n / n_sample, n_sample, tab);
+        hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
+        hot_threshold_kernel<<<1, 1024, 0, s>>>(hist, 4u, (uint32_t)hot::K);
+        hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)hot::K);
+        hot_clamp_kernel<<<1, 32, 0, s>>>(n_out, (uint32_t)hot::K);
+        hot_resolve_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
+        hl = list;
+        nh = n_out;
+    }
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(insert_text_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(textk::Smem));
+        attr = true;
+    }
+    insert_text_kernel<<<grid, textk::THREADS, sizeof(textk::Smem), s>>>(d, b, hl, nh);
+    return cudaGetLastError();
+}
+int sepo_launch_text_bits(const Dev& d, const Batch& b, unsigned long long* counter, cudaStream_t s) {
+    text_bits_kernel<<<4 * 148, 256, 0, s>>>(d, b, counter);
+    return cudaGetLastError();
+}
 
 int sepo_launch_evict_copy(const Dev& d, uint32_t n, uint8_t* dst, int grid, cudaStream_t s) {
     if (n) evict_copy_kernel<<<grid, 512, 0, s>>>(d.pool, d.evict_list, n, dst, d.page_shift);

@@ -33,6 +33,11 @@ struct Batch {
     const PRec* prep = nullptr;
     uint32_t prep_rb = 48;  // bytes per prepared record: 48 (PRec), or 32 when every value is 1:
                             // {w0, w1, h, s | len << 48} (a third less re-issue traffic)
+    // raw-text input (sepo_run_text, NEXT-2): keys = text bytes, n = text bytes; records are the
+    // words (maximal runs of non-separator bytes), identified by their start offset. Declined
+    // words that do not fit the prepared list set bit (start) in tbm (u32 words over the text).
+    uint32_t text = 0;
+    uint32_t* tbm = nullptr;
 };
 }  // namespace sepo
 
@@ -56,6 +61,8 @@ int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec,
                               uint64_t total, cudaStream_t s);
 int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);
 int sepo_launch_evict_copy(const sepo::Dev& d, uint32_t n, uint8_t* dst, int grid, cudaStream_t s);
+int sepo_launch_insert_text(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s, void* hot_scratch);
+int sepo_launch_text_bits(const sepo::Dev& d, const sepo::Batch& b, unsigned long long* counter, cudaStream_t s);
 int sepo_launch_classify(const sepo::Dev& d, int honor_retain, cudaStream_t s);
 int sepo_launch_relink(const sepo::Dev& d, cudaStream_t s);
 int sepo_launch_init(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);

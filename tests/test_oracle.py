@@ -295,3 +295,32 @@ def test_basic_tiny_adversarial():
     vals = np.array(vs, dtype=np.uint64).view(np.uint8)
     got = oracle.basic(keys, offs, vals, 8)
     assert got == {b"": [0, 5], b"a": [1, 1, 2], b"ab": [7], b"b\x00": [3], b"b": [3]}
+
+
+# ------------------------------------------------------------------ raw text word count (NEXT-2)
+def test_word_count_text_closed_form():
+    """the raw text of a word stream (each word + one separator) counts exactly the generator's
+    closed-form c_r per word — independent of the oracle's own tokenizer"""
+    for name, scale in (("C1", 0.05), ("C2", 2e-5)):
+        s = gen.config(name, scale=scale)
+        assert oracle.word_count_text(s.text_host()) == s.expected_combine()
+
+
+def test_word_count_text_tokenizer_rules():
+    """R20: separators are exactly ' ', '\\n', '\\t', '\\r'; runs of them, leading/trailing ones and
+    an empty text yield no empty words; other bytes (\\x0b, \\x00, 0xff) belong to words"""
+    t = b"  ab\tab\r\n\nc \x0bx\x0b ab\x00 \xff\xff  c"
+    exp = {b"ab": 2, b"c": 2, b"\x0bx\x0b": 1, b"ab\x00": 1, b"\xff\xff": 1}
+    assert oracle.word_count_text(np.frombuffer(t, dtype=np.uint8)) == exp
+    assert oracle.word_count_text(np.zeros(0, dtype=np.uint8)) == {}
+    assert oracle.word_count_text(np.frombuffer(b" \n\t\r", dtype=np.uint8)) == {}
+    # brute force: Python's regex split on the same separator set
+    import re
+    rng = random.Random(7)
+    for _ in range(20):
+        t = bytes(rng.choice(b"ab \n\t\rc\x0b") for _ in range(rng.randrange(0, 300)))
+        ref = {}
+        for w in re.split(rb"[ \n\t\r]+", t):
+            if w:
+                ref[w] = ref.get(w, 0) + 1
+        assert oracle.word_count_text(np.frombuffer(t, dtype=np.uint8)) == ref

@@ -1,0 +1,95 @@
+"""GPU parity of the fused tokenizer + insert path (sepo_run_text): raw
+text in, word counts out, exactly the oracle's (tokenizer reading R20) — in one pass and over
+budget, with and without the sampled hot set, through the prepared-list overflow path, from host
+memory, and on adversarial texts (separator runs, words across 512-byte windows and longer than
+two windows, a text not ending in a separator)."""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from tests.util import footprint_pages
+
+pytestmark = pytest.mark.gpu
+
+
+def sepo():
+    import paper_conf_ipps_mokhtaris17_b200 as m
+    return m
+
+
+def run_text(text, budget_pages, nb=1 << 14, pb=4096, **kw):
+    S = sepo()
+    t = S.Table(S.budget_for(nb, pb, budget_pages), nb, pb, check_dups=True, **kw)
+    passes = t.run_text(text)
+    got = S.result_dict(t.export())
+    st = t.stats()
+    t.close()
+    return got, passes, st
+
+
+@pytest.mark.parametrize("cfg,scale,ratio", [("C1", 0.25, 0.5), ("C1", 0.25, 4), ("C2", 0.004, 0.5), ("C2", 0.004, 3)])
+def test_text_parity(cuda, cfg, scale, ratio):
+    s = gen.config(cfg, scale=scale)
+    text = s.text_device()
+    exp = s.expected_combine()
+    assert oracle.word_count_text(s.text_host()) == exp
+    pb = 4096 if cfg == "C1" else 16384
+    F = footprint_pages(s, 1 << 14, pb)
+    P = int(np.ceil(F / ratio)) + (600 if ratio < 1 else 0)
+    got, passes, st = run_text(text, P, pb=pb)
+    assert got == exp
+    assert st["records_inserted"] >= s.n and st["cross_gen_dups"] == 0
+    if ratio > 1:
+        assert passes >= 2
+        post = st["postponed_per_pass"]
+        assert all(post[i] > post[i + 1] for i in range(len(post) - 1)) and post[-1] == 0, post
+    else:
+        assert passes == 1 and st["records_inserted"] == s.n
+
+
+def test_text_prepared_overflow(cuda, monkeypatch):
+    """declined words beyond the prepared list's capacity go through the text bitmap"""
+    monkeypatch.setenv("SEPO_PREP_CAP", "1000")
+    s = gen.config("C1", scale=0.25)
+    F = footprint_pages(s, 1 << 14, 4096)
+    got, passes, st = run_text(s.text_device(), max(8, F // 4))
+    assert got == s.expected_combine() and passes >= 3
+
+
+def test_text_from_host(cuda):
+    s = gen.config("C1", scale=0.1)
+    got, passes, _ = run_text(s.text_host(), 4096)
+    assert got == s.expected_combine() and passes == 1
+
+
+def _dev(b):
+    t = torch.empty(len(b) + 64, dtype=torch.uint8, device="cuda")[:len(b)]
+    if len(b):
+        t.copy_(torch.frombuffer(bytearray(b), dtype=torch.uint8))
+    return t
+
+
+def test_text_adversarial(cuda):
+    rng = np.random.default_rng(5)
+    parts = [b"  ", b"a" * 15, b" ", b"b" * 17, b"\n", b"x" * 700, b"\t\r", b"\x0bq\x0b", b" "]
+    parts += [b"w%d " % i for i in range(200)]
+    parts += [b"L" * 1500, b" ", b"y" * 511, b"\n", b"z" * 513, b" end"]  # no final separator
+    t = b"".join(parts)
+    for shift in (0, 1, 7, 16, 495, 511):  # move every word across the 16- and 512-byte boundaries
+        tt = b"\r" * shift + t
+        exp = oracle.word_count_text(np.frombuffer(tt, dtype=np.uint8))
+        got, passes, _ = run_text(_dev(tt), 256, pb=8192)
+        assert got == exp, shift
+    # random texts over a small alphabet, many windows, over budget
+    for seed in range(3):
+        r = np.random.default_rng(seed)
+        tt = bytes(r.choice(np.frombuffer(b"abcd  \n\t", dtype=np.uint8), size=200_000))
+        exp = oracle.word_count_text(np.frombuffer(tt, dtype=np.uint8))
+        got, passes, _ = run_text(_dev(tt), 8, pb=4096, grid_ctas=8)
+        assert got == exp
+    got, passes, _ = run_text(_dev(b""), 16)
+    assert got == {}
+    got, passes, _ = run_text(_dev(b" \n \t"), 16)
+    assert got == {}
