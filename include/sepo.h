@@ -204,6 +204,20 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* key_offsets
  * with SEPO_E_TOOLARGE. */
 int64_t sepo_run_text(sepo_table* t, const uint8_t* text, uint64_t n_bytes);
 
+/* SEPO LOOKUPS on the larger-than-memory table ("The SEPO model can also
+ * be used for lookup operations on larger-than-memory hash tables"). COMBINE tables only (else
+ * SEPO_E_INVAL). keys/key_offsets (CSR, or fixed_key_width when key_offsets is NULL), values_out
+ * (n u64) and found_bitmap (ceil(n/32) u32) are DEVICE arrays (else SEPO_E_INVAL). The resident
+ * generation is evicted first; then every generation's page images go back into the device pool
+ * (each page to the slot it left, so entry refs stay valid), the directory is rebuilt from them
+ * and every query not yet found is probed — a query whose key is not in this generation is
+ * postponed to the next one. Query i: bit (i&31) of found_bitmap[i>>5] = 1 and values_out[i] =
+ * the key's value if the key is in the table, else bit 0 and value 0. Returns the number found
+ * (or < 0). Allowed before or after sepo_export; afterwards only sepo_lookup, sepo_export,
+ * sepo_stats, sepo_reset and sepo_destroy (inserts: SEPO_E_STATE until sepo_reset). */
+int64_t sepo_lookup(sepo_table* t, const uint8_t* keys, const uint64_t* key_offsets, uint64_t n, uint64_t* values_out,
+                    uint32_t* found_bitmap);
+
 /* Drop all generations and results and start a new job with the same budget and options;
  * pinned host memory and device scratch are kept for reuse. */
 int sepo_reset(sepo_table* t);

@@ -62,7 +62,7 @@ E_INVAL, E_NOMEM, E_TOOLARGE, E_CUDA, E_STATE, E_NCCL = -1, -2, -3, -4, -5, -6
 POOL_DEVICE, POOL_HOST_PINNED, POOL_MANAGED = 0, 1, 2  # sepo_create_placed (include/sepo.h)
 
 # every entry point declared in include/sepo.h
-EXPORTS = ["sepo_create", "sepo_create_placed", "sepo_configure", "sepo_run_text", "sepo_insert_batch", "sepo_reprobe", "sepo_compact", "sepo_evict",
+EXPORTS = ["sepo_create", "sepo_create_placed", "sepo_configure", "sepo_run_text", "sepo_lookup", "sepo_insert_batch", "sepo_reprobe", "sepo_compact", "sepo_evict",
            "sepo_export", "sepo_run", "sepo_reset", "sepo_stats_get", "sepo_last_insert_ms", "sepo_destroy",
            "sepo_last_error", "sepo_version", "sepo_budget_for", "sepo_partition_scratch", "sepo_partition",
            "sepo_shift_offsets"]
@@ -90,6 +90,7 @@ def lib():
         L.sepo_export.argtypes = [vp, ctypes.POINTER(Result)]; L.sepo_export.restype = ctypes.c_int
         L.sepo_run.argtypes = [vp, vp, vp, vp, vp, u64]; L.sepo_run.restype = i64
         L.sepo_run_text.argtypes = [vp, vp, u64]; L.sepo_run_text.restype = i64
+        L.sepo_lookup.argtypes = [vp, vp, vp, u64, vp, vp]; L.sepo_lookup.restype = i64
         L.sepo_reset.argtypes = [vp]; L.sepo_reset.restype = ctypes.c_int
         L.sepo_stats_get.argtypes = [vp, ctypes.POINTER(Stats)]; L.sepo_stats_get.restype = ctypes.c_int
         L.sepo_last_insert_ms.argtypes = [vp]; L.sepo_last_insert_ms.restype = ctypes.c_double
@@ -219,6 +220,18 @@ class Table:
         if rc < 0:
             _err(rc)
         return int(rc)
+
+    def lookup(self, keys, key_offsets, n=None):
+        """SEPO lookups over every generation (sepo_lookup) -> (found count, values u64 tensor,
+        found bitmap int32 tensor), device tensors."""
+        import torch
+        n = self._n(key_offsets, keys, n)
+        vals = torch.empty(max(n, 1), dtype=torch.int64, device="cuda")
+        bm = torch.empty(max((n + 31) // 32, 1), dtype=torch.int32, device="cuda")
+        rc = self._L.sepo_lookup(self.h, _ptr(keys), _ptr(key_offsets), n, _ptr(vals), _ptr(bm))
+        if rc < 0:
+            _err(rc)
+        return int(rc), vals[:n], bm
 
     def export(self, copy=True):
         """-> dict of numpy arrays (copies unless copy=False: views of table-owned memory)."""

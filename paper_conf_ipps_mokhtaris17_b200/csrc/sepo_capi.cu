@@ -116,6 +116,8 @@ struct sepo_table {
     DevBuf idxb[2];  // sepo_run re-issue index lists (ping-pong)
     DevBuf prep[2];  // sepo_run COMBINE: prepared re-issue records (ping-pong)
     DevBuf prep_n;   // their device counters
+    DevBuf lk_pages; // sepo_lookup: page ids of the generation being probed
+    bool lookup_done = false;  // sepo_lookup restored old generations into the pool: no inserts until reset
     DevBuf tbm;      // sepo_run_text: start bits of declined words that did not fit the prepared list
     // cuStreamWriteValue32 (driver entry point): the copy stream publishes eviction progress
     int (*write_value32)(cudaStream_t, unsigned long long, unsigned int, unsigned int) = nullptr;
@@ -163,6 +165,7 @@ int check_active(sepo_table* t) {
     if (!t) return fail(SEPO_E_INVAL, "null table");
     if (t->state == ST_BROKEN) return fail(SEPO_E_CUDA, "table is broken by an earlier CUDA error");
     if (t->state == ST_EXPORTED) return fail(SEPO_E_STATE, "table already exported (sepo_reset to reuse)");
+    if (t->lookup_done) return fail(SEPO_E_STATE, "table was probed by sepo_lookup (sepo_reset to insert again)");
     return 0;
 }
 
@@ -1001,8 +1004,10 @@ int export_group(sepo_table* t) {
 }  // namespace
 
 int sepo_export(sepo_table* t, sepo_result* out) {
-    int rc = check_active(t);
-    if (rc) return rc;
+    if (!t) return fail(SEPO_E_INVAL, "null table");
+    if (t->state == ST_BROKEN) return fail(SEPO_E_CUDA, "table is broken by an earlier CUDA error");
+    if (t->state == ST_EXPORTED) return fail(SEPO_E_STATE, "table already exported (sepo_reset to reuse)");
+    int rc = 0;  // (allowed after sepo_lookup: export reads the host page images)
     if (!out) return fail(SEPO_E_INVAL, "null result");
     if (t->dirty) {
         int64_t e = evict_impl(t, 0);
@@ -1318,6 +1323,52 @@ int64_t sepo_run_text(sepo_table* t, const uint8_t* text, uint64_t n_bytes) {
     return (int64_t)t->st.passes - passes_start;
 }
 
+// ---------------------------------------------------------------- SEPO lookups (NEXT-4)
+int64_t sepo_lookup(sepo_table* t, const uint8_t* keys, const uint64_t* ko, uint64_t n, uint64_t* values_out,
+                    uint32_t* found_bitmap) {
+    if (!t) return fail(SEPO_E_INVAL, "null table");
+    if (t->state == ST_BROKEN) return fail(SEPO_E_CUDA, "table is broken by an earlier CUDA error");
+    if (t->opts.mode != SEPO_COMBINE_SUM_U64) return fail(SEPO_E_INVAL, "sepo_lookup supports COMBINE tables");
+    if (n == 0) return 0;
+    if (!values_out || !found_bitmap) return fail(SEPO_E_INVAL, "values_out / found_bitmap is NULL");
+    if (!is_device_ptr(keys) || !is_device_ptr(ko) || !is_device_ptr(values_out) || !is_device_ptr(found_bitmap))
+        return fail(SEPO_E_INVAL, "sepo_lookup takes device arrays");
+    Batch b;
+    int rc = make_batch(t, b, keys, ko, nullptr, nullptr, n, nullptr);
+    if (rc) return rc;
+    if (t->state == ST_ACTIVE && t->dirty) {  // the resident generation joins the host images first
+        int64_t e = evict_impl(t, 0);
+        if (e < 0) return e;
+    }
+    CK(t, cudaStreamSynchronize(t->copy_stream));
+    CK(t, cudaMemsetAsync(found_bitmap, 0, ((n + 31) / 32) * 4, t->stream));
+    CK(t, cudaMemsetAsync(values_out, 0, n * 8, t->stream));
+    t->lookup_done = true;  // the pool now holds restored images: inserts need sepo_reset
+    uint64_t found = 0;
+    std::vector<uint32_t> ids;
+    for (auto& g : t->gens) {
+        // restore the generation's pages to their slots (one H2D per run), then link + probe
+        ids.clear();
+        for (auto& r : g.runs) {
+            CK(t, cudaMemcpyAsync(t->d.pool + ((size_t)r.first << t->page_shift), r.p, (size_t)r.count << t->page_shift,
+                                  cudaMemcpyDefault, t->stream));
+            for (uint32_t k = 0; k < r.count; ++k) ids.push_back(r.first + k);
+        }
+        if (t->lk_pages.grow(ids.size() * 4 + 4)) return fail(SEPO_E_NOMEM, "lookup page list");
+        CK(t, cudaMemcpyAsync(t->lk_pages.p, ids.data(), ids.size() * 4, cudaMemcpyHostToDevice, t->stream));
+        CK(t, cudaMemsetAsync(t->d.dir, 0, t->n_buckets * 4, t->stream));
+        if ((rc = zero_ctrl_counters(t))) return rc;
+        rc = sepo_launch_lookup_gen(t->d, b, (const uint32_t*)t->lk_pages.p, (uint32_t)ids.size(),
+                                    (unsigned long long*)values_out, found_bitmap, t->stream);
+        if (rc) return cuda_check(t, (cudaError_t)rc, "lookup kernels");
+        t->st.kernel_launches += 2;
+        if ((rc = read_ctrl(t))) return rc;  // (also orders the host vector reuse after the copy)
+        found += t->h_ctrl->postponed;
+        if (found == n) break;  // every query resolved: later generations are not needed
+    }
+    return (int64_t)found;
+}
+
 int sepo_reset(sepo_table* t) {
     trace("reset");
     if (!t) return fail(SEPO_E_INVAL, "null table");
@@ -1330,6 +1381,7 @@ int sepo_reset(sepo_table* t) {
     t->inserted = false;
     t->batch_seq = 0;
     t->pages_resident_retained = 0;
+    t->lookup_done = false;
     trace("reset: copy stream idle");
     sepo_stats z{};
     z.n_buckets = t->n_buckets;
@@ -1366,6 +1418,7 @@ void sepo_destroy(sepo_table* t) {
     t->prep[1].release();
     t->prep_n.release();
     t->tbm.release();
+    t->lk_pages.release();
     t->bm.release();
     for (auto& s : t->buf)
         for (auto& b : s) b.release();

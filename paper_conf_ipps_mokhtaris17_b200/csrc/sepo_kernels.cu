@@ -85,11 +85,18 @@ __device__ __forceinline__ uint32_t item_units(uint32_t vw, uint32_t vlen) { ret
 // Sized by the demand rather than grown from the previous chunk: many CTAs may find a key's head
 // chunk full at once and each installs a chunk, so large geometric chunks would mostly stay empty
 // (measured: 8x slot over-allocation on C4 with doubling).
+#ifndef SEPO_CHUNK_GROW
+#define SEPO_CHUNK_GROW 0   // > 0: a key's next shared chunk gets min(2 x the full one's capacity, this many slots)
+#endif
 __device__ __forceinline__ uint32_t chunk_cap(const Dev& d, uint32_t need, uint32_t prev, uint32_t vw) {
-    (void)prev;
     const uint32_t unit = vw ? vw : 1u;
     const uint32_t maxcap = (d.page_bytes / 4 - CHUNK_HDR) / unit;
     uint32_t c = max(vw ? 8u : 64u, 2u * need);
+#if SEPO_CHUNK_GROW
+    if (vw) c = max(c, min(2u * (prev & ~CHUNK_PRIVATE), (uint32_t)SEPO_CHUNK_GROW));
+#else
+    (void)prev;
+#endif
     c = min(c, max(maxcap, need));
     return min(c, (d.page_bytes - CHUNK_HDR) / unit);
 }
@@ -378,6 +385,9 @@ struct CtaState {                 // allocator slot (the CTA's active pages) + p
 };
 // Shared memory of the COMBINE stream kernel: the hot set (read-only keys + per-CTA pending sums)
 // and one miss queue per warp (records that missed the hot set, resolved 32 at a time).
+#ifndef SEPO_BRANCHLESS
+#define SEPO_BRANCHLESS 0
+#endif
 #ifndef SEPO_HOT_DIRECT
 #define SEPO_HOT_DIRECT 1  // direct-indexed hot set (C2 4x pass 1 22.2 -> 21.3 ms); 0: 4-way bucket fingerprints
 #endif
@@ -1066,6 +1076,20 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
             const uint32_t t1 = S.tags[stream::ds1(h)], t2 = S.tags[stream::ds2(h)];
             const bool m1 = (t1 & 0xfffff800u) == f, m2 = (t2 & 0xfffff800u) == f;
             const uint32_t p = (m1 ? t1 : t2) & 0x7ffu;
+#if SEPO_BRANCHLESS
+            // branch-free common case: the candidate's 16 key bytes are loaded for every lane (p is
+            // always a valid index); keys longer than 16 bytes take a warp-uniform slow path
+            const bool cand = valid && (m1 || m2);
+            const ulonglong2 kk = S.kw[p];
+            bool eq = cand && kk.x == w0 && kk.y == w1;
+            if (__any_sync(FULLMASK, eq && len > 16)) {
+                if (eq && len > 16) {
+                    const uint8_t* e = ref_ptr(d, S.ref[p]);
+                    eq = ldcg32(e + 12) == len && entry_key_eq(e + KEY_OFF + 16, b.keys + s + 16, len - 16);
+                }
+            }
+            pos = eq ? (int)p : -1;
+#else
             if (valid && (m1 || m2)) {
                 const ulonglong2 kk = S.kw[p];
                 bool eq = kk.x == w0 && kk.y == w1;
@@ -1075,6 +1099,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
                 }
                 if (eq) pos = (int)p;
             }
+#endif
         }
 #else
         if (have_hot) {
@@ -1425,6 +1450,7 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
         if (valid && !done && pos < 0) e = chain_find_w(d, head, 0, tag, len, w0, w1, tail);
         bool need_key = valid && !done && e == nullptr;
         bool need_chunk = valid && !done;
+        uint32_t prev_cap = 0;
         if (valid && !done && e) {
             uint64_t cr = 0, lh = 0;
             uint32_t base = 0, pc = 0;
@@ -1433,10 +1459,11 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
                 done = true;
                 need_chunk = false;
             }
+            prev_cap = pc;
         }
         uint32_t res = R_OK;
         const uint32_t ksize = gkey_size(len);
-        const uint32_t ccap = chunk_cap(d, units, 0, vw);
+        const uint32_t ccap = chunk_cap(d, units, prev_cap, vw);
         const uint32_t csize = chunk_bytes(ccap, vw);
         if ((need_key && (len > 65535u - 64u || ksize > PB)) || (need_chunk && CHUNK_HDR + units * (vw ? vw : 1u) > PB)) {
             need_key = false; need_chunk = false; res = R_TOOLARGE;
@@ -2347,6 +2374,56 @@ __global__ void __launch_bounds__(256) text_bits_kernel(Dev d, Batch b, unsigned
     }
 }
 
+// ================================================================ SEPO lookups (NEXT-4)
+// Lookups on the larger-than-memory table ("The SEPO model can also be used for lookup
+// operations on larger-than-memory hash tables"): the host streams the evicted generations back
+// through the device pool one at a time (each page to the slot it was evicted from, so refs stay
+// valid); the directory is rebuilt from the restored pages and every still-unresolved query is
+// probed; queries whose key is not in this generation are POSTPONED to the next one.
+__global__ void lookup_link_kernel(Dev d, const uint32_t* pages, uint32_t np) {
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < np; i += gridDim.x * blockDim.x) {
+        uint8_t* base = d.pool + ((uint64_t)pages[i] << d.page_shift);
+        for (uint32_t off = 0; off < d.page_bytes;) {
+            const uint32_t hdr = *reinterpret_cast<uint32_t*>(base + off);
+            const uint32_t size = hdr & ~KIND_MASK;
+            if (size == 0) break;
+            if ((hdr & KIND_MASK) == K_COMBINE) {
+                uint8_t* e = base + off;
+                const uint32_t len = *reinterpret_cast<uint32_t*>(e + 12);
+                const uint32_t bkt = bucket_of(hash_key(e + KEY_OFF, len, d.seed), d.n_buckets);
+                const uint32_t me = off_ref((uint64_t)(e - d.pool));
+                uint32_t head = ld_dir(d.dir + bkt);
+                while (true) {
+                    *reinterpret_cast<uint32_t*>(e + 4) = head;
+                    const uint32_t old = cas_release(d.dir + bkt, head, me);
+                    if (old == head) break;
+                    head = old;
+                }
+            }
+            off += size;
+        }
+    }
+}
+// one query per thread: skip the ones already found; probe the restored generation
+__global__ void __launch_bounds__(256) lookup_kernel(Dev d, Batch b, unsigned long long* vals_out, uint32_t* found) {
+    unsigned long long hits = 0;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < b.n; i += (uint64_t)gridDim.x * blockDim.x) {
+        if ((found[i >> 5] >> (i & 31)) & 1u) continue;
+        uint64_t s, w0, w1, h;
+        uint32_t len;
+        rec_hash16(d, b, i, s, len, w0, w1, h);
+        const uint8_t* e = chain_find_w(d, ld_dir(d.dir + bucket_of(h, d.n_buckets)), 0, tag_of(h), len, w0, w1,
+                                        b.keys + s + 16);
+        if (e) {
+            vals_out[i] = ldcg64(entry_val(const_cast<uint8_t*>(e), len));
+            atomicOr(found + (i >> 5), 1u << (i & 31));
+            ++hits;
+        }
+    }
+    for (int o = 16; o; o >>= 1) hits += __shfl_xor_sync(FULLMASK, hits, o);
+    if ((threadIdx.x & 31) == 0 && hits) atomicAdd(&d.ctrl->postponed, hits);
+}
+
 // Eviction gather copy (a10): evicted pages -> one contiguous pinned host region, page k of the
 // evict list at dst + k * page_bytes. The host arena is page-locked and mapped (UVA), so SM stores
 // cross the host link directly: one launch per eviction however fragmented the evict list is (a
@@ -2401,6 +2478,12 @@ int sepo_launch_insert_text(const Dev& d, const Batch& b, int grid, cudaStream_t
         attr = true;
     }
     insert_text_kernel<<<grid, textk::THREADS, sizeof(textk::Smem), s>>>(d, b, hl, nh);
+    return cudaGetLastError();
+}
+int sepo_launch_lookup_gen(const Dev& d, const Batch& b, const uint32_t* pages, uint32_t np, unsigned long long* vals,
+                           uint32_t* found, cudaStream_t s) {
+    if (np) lookup_link_kernel<<<(np + 127) / 128, 128, 0, s>>>(d, pages, np);
+    if (b.n) lookup_kernel<<<8 * 148, 256, 0, s>>>(d, b, vals, found);
     return cudaGetLastError();
 }
 int sepo_launch_text_bits(const Dev& d, const Batch& b, unsigned long long* counter, cudaStream_t s) {

@@ -62,6 +62,8 @@ int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec,
 int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);
 int sepo_launch_evict_copy(const sepo::Dev& d, uint32_t n, uint8_t* dst, int grid, cudaStream_t s);
 int sepo_launch_insert_text(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s, void* hot_scratch);
+int sepo_launch_lookup_gen(const sepo::Dev& d, const sepo::Batch& b, const uint32_t* pages, uint32_t np,
+                           unsigned long long* vals, uint32_t* found, cudaStream_t s);
 int sepo_launch_text_bits(const sepo::Dev& d, const sepo::Batch& b, unsigned long long* counter, cudaStream_t s);
 int sepo_launch_classify(const sepo::Dev& d, int honor_retain, cudaStream_t s);
 int sepo_launch_relink(const sepo::Dev& d, cudaStream_t s);
