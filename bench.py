@@ -376,19 +376,29 @@ def run_ours(args):
     pk = peaks()
     alg = job.csr_bytes() if not routed else job.slice_bytes
     achieved = alg * args.steps / (info["p1_ms"] / 1e3) / 1e9
-    traffic, traffic_note = args.traffic, None
+    traffic, traffic_note, issue = args.traffic, None, None
     tj = os.path.join(ROOT, "profiles", "r01_traffic.json")
     if traffic is None and os.path.exists(tj) and args.config == "C2" and args.scale == 1.0:
         tr = json.load(open(tj))
         traffic = tr["dram_read_bytes"] + tr["dram_write_bytes"]
         traffic_note = (f"dram read+write of one launch ({tr['launch']}); that launch's algorithmic bytes: "
                         f"{tr['alg_bytes']}")
+        if "warp_instructions" in tr:
+            # the kernel is issue-bound, not HBM-bound: its instruction roofline from the same capture
+            # (peak = 148 SMs x 4 schedulers x 1 warp instruction / cycle at the sampled SM clock)
+            peak_wi = 148 * 4 * (clocks.get("sm_mhz") or 1965.0) * 1e6
+            wi_per_s = tr["warp_instructions"] / (info["p1_ms"] / args.steps / 1e3)
+            issue = {"warp_instructions_per_launch": tr["warp_instructions"],
+                     "warp_instructions_per_record": tr["warp_instructions"] / n,
+                     "achieved_warp_instr_per_s": wi_per_s, "peak_warp_instr_per_s": peak_wi,
+                     "frac": wi_per_s / peak_wi, "ncu_issue_active": tr.get("issue_active_pct", 0) / 100.0}
     roof = {"bound": "hbm", "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
             "frac": achieved / pk["hbm_gbs"], "traffic": traffic, "traffic_note": traffic_note,
             "kernel": "sepo::insert_stream_kernel (COMBINE, pass 1) / sepo::insert_group_stream_kernel (GROUP)",
             "alg_bytes_per_launch": alg, "launch_ms": info["p1_ms"] / args.steps,
             "share_of_step": info["p1_ms"] / ms, "all_insert_passes_share_of_step": info["insert_ms"] / ms,
-            "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if not pk.get("_fallback") else "fallback 6.65 TB/s"}
+            "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if not pk.get("_fallback") else "fallback 6.65 TB/s",
+            "issue": issue}
 
     # end to end through sepo_run with pinned HOST buffers (H2D + job + host result assembly)
     e2e = None
@@ -434,6 +444,47 @@ def run_ours(args):
             curve[str(r)] = {"ms": ms2, "slowdown": ms2 / base, "passes": i2["last"]["passes"]}
             t2.close()
 
+    # raw-text job (NEXT-2 (i), sepo_run_text): the same word stream as the 8 GB text the config
+    # names (each word + one separator), tokenized inside the insert kernel; device-resident
+    # input timed like the main line, plus e2e from pinned host text (H2D inside the timed region)
+    raw_text = None
+    if args.text and rank == 0 and not routed and job.stream.family == 0 and job.stream.val == "one":
+        text = job.stream.text_device()
+        tb = text.numel()
+        for _ in range(2):
+            t.reset(); t.run_text(text)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            t.reset(); t.run_text(text)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        tms = e0.elapsed_time(e1) / args.steps
+        stt = t.stats()
+        raw_text = {"text_bytes": tb, "ms_per_step": tms, "value": tb / tms / 1e6, "unit": "GB/s of raw text",
+                    "words_per_s": n / tms * 1e3, "passes": stt["passes"],
+                    "pass1_ms": stt["t_insert_ms_per_pass"][0]}
+        if args.e2e_steps > 0:
+            ht = torch.empty(tb, dtype=torch.uint8, pin_memory=True)
+            ht.copy_(text)
+            del text
+            t.reset(); t.run_text(ht); t.export(copy=False)
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            d2h = 0
+            for _ in range(args.e2e_steps):
+                t.reset(); t.run_text(ht); t.export(copy=False)
+                d2h += t.stats()["bytes_evicted"]
+            el = (time.perf_counter() - t0) / args.e2e_steps
+            raw_text["e2e"] = {"value": tb / el / 1e9, "unit": "GB/s of raw text", "words_per_s": n / el,
+                               "h2d_bytes_per_step": tb, "d2h_bytes_per_step": d2h // args.e2e_steps,
+                               "note": "sepo_run_text on pinned host text; includes H2D, all passes, page D2H, host result assembly"}
+            del ht
+        else:
+            del text
+        torch.cuda.empty_cache()
+
     cpu = None
     if rank == 0 and args.cpu_baseline:
         gbs, rps, nrec, tsec = oracle_sample(job, args.ref_records, budget_s=args.ref_seconds)
@@ -456,7 +507,7 @@ def run_ours(args):
                                            else "1 GPU"),
                            "phase_ms": {kk: st[kk] for kk in ("t_insert_ms", "t_reprobe_ms", "t_compact_ms", "t_evict_ms")}},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
-                "gpu_launches": info["launches"], "slowdown_curve": curve}
+                "gpu_launches": info["launches"], "slowdown_curve": curve, "raw_text": raw_text}
         print(json.dumps(line), flush=True)
     t.close()
     if dist.is_initialized():
@@ -475,6 +526,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-curve", dest="curve", action="store_false")
     ap.add_argument("--no-cpu", dest="cpu_baseline", action="store_false")
+    ap.add_argument("--no-text", dest="text", action="store_false", help="skip the raw-text (fused tokenizer) line")
     ap.add_argument("--ref-records", type=int, default=120_000_000)
     ap.add_argument("--ref-seconds", type=float, default=15.0)
     ap.add_argument("--route", action="store_true", help="run the sharded (router) path even at N=1")

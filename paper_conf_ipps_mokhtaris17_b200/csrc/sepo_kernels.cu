@@ -2404,24 +2404,35 @@ __global__ void lookup_link_kernel(Dev d, const uint32_t* pages, uint32_t np) {
         }
     }
 }
-// one query per thread: skip the ones already found; probe the restored generation
+// a warp per 32 consecutive queries: the group's found word decides which lanes still probe; keys
+// are read with the warp-cooperative 16-byte loads of the insert path; the found word is rewritten
+// once per group (this warp owns it)
 __global__ void __launch_bounds__(256) lookup_kernel(Dev d, Batch b, unsigned long long* vals_out, uint32_t* found) {
+    const uint32_t lane = lane_id();
+    const uint64_t ngroups = (b.n + 31) / 32;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
     unsigned long long hits = 0;
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < b.n; i += (uint64_t)gridDim.x * blockDim.x) {
-        if ((found[i >> 5] >> (i & 31)) & 1u) continue;
-        uint64_t s, w0, w1, h;
+    for (uint64_t g = (uint64_t)blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5); g < ngroups; g += nw) {
+        const uint32_t fw = found[g];
+        const uint64_t i = g * 32 + lane;
+        const bool valid = i < b.n;
+        const bool todo = valid && !((fw >> lane) & 1u);
+        if (!__any_sync(FULLMASK, todo)) continue;
+        uint64_t s, w0, w1;
         uint32_t len;
-        rec_hash16(d, b, i, s, len, w0, w1, h);
-        const uint8_t* e = chain_find_w(d, ld_dir(d.dir + bucket_of(h, d.n_buckets)), 0, tag_of(h), len, w0, w1,
-                                        b.keys + s + 16);
-        if (e) {
-            vals_out[i] = ldcg64(entry_val(const_cast<uint8_t*>(e), len));
-            atomicOr(found + (i >> 5), 1u << (i & 31));
-            ++hits;
+        warp_load_group(b, g, lane, valid, s, len, w0, w1);
+        const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
+        const uint8_t* e = nullptr;
+        if (todo)
+            e = chain_find_w(d, ld_dir(d.dir + bucket_of(h, d.n_buckets)), 0, tag_of(h), len, w0, w1, b.keys + s + 16);
+        if (e) vals_out[i] = ldcg64(entry_val(const_cast<uint8_t*>(e), len));
+        const unsigned hm = __ballot_sync(FULLMASK, e != nullptr);
+        if (lane == 0 && hm) {
+            found[g] = fw | hm;
+            hits += __popc(hm);
         }
     }
-    for (int o = 16; o; o >>= 1) hits += __shfl_xor_sync(FULLMASK, hits, o);
-    if ((threadIdx.x & 31) == 0 && hits) atomicAdd(&d.ctrl->postponed, hits);
+    if (lane == 0 && hits) atomicAdd(&d.ctrl->postponed, hits);
 }
 
 // Eviction gather copy (a10): evicted pages -> one contiguous pinned host region, page k of the
