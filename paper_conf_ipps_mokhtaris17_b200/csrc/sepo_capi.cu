@@ -463,7 +463,13 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
     if (t->hot.grow(sepo_hot_scratch_bytes())) return fail(SEPO_E_NOMEM, "hot-set scratch");
     // BASIC halt rule: the pass stops once this many allocator slots failed
     const uint32_t halt_slots = (uint32_t)std::max<uint64_t>(1, ((uint64_t)t->grid * t->opts.basic_halt_pct + 99) / 100);
-    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p, halt_slots);
+    uint64_t key_end = 0;
+    if (b.ko && !b.idx) {  // the end of the batch's key bytes, a kernel parameter (see the kernel)
+        CK(t, cudaMemcpyAsync(&t->h_ko[1], b.ko + n, 8, cudaMemcpyDeviceToHost, t->stream));
+        CK(t, cudaStreamSynchronize(t->stream));
+        key_end = t->h_ko[1];
+    }
+    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p, halt_slots, key_end);
     if (rc) return cuda_check(t, (cudaError_t)rc, "insert kernel launch");
     CK(t, cudaEventRecord(t->ev1, t->stream));
     t->st.kernel_launches += (n >= (8ull << 18)) ? 7 : 1;

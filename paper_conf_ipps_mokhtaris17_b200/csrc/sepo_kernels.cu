@@ -20,7 +20,12 @@
 namespace sepo {
 
 
-__device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31u; }
+// %laneid: one S2R when the compiler rematerialises it (threadIdx.x & 31 costs two)
+__device__ __forceinline__ uint32_t lane_id() {
+    uint32_t l;
+    asm("mov.u32 %0, %%laneid;" : "=r"(l));
+    return l;
+}
 __device__ __forceinline__ uint32_t lanemask_lt() { return (1u << lane_id()) - 1u; }
 
 // record i of a batch -> its index in keys / key_offsets / vals (re-issue by index, a9)
@@ -943,9 +948,13 @@ __global__ void __launch_bounds__(1024, 1) insert_basic_kernel(Dev d, Batch b, u
     }
 }
 
+// The input context (groups, last group's size, warps, key bytes end, alignment) comes from the
+// host as a kernel parameter: in the constant bank a loop-invariant costs one load when the
+// register-bound loop (64 registers x 1024 threads) rematerialises it, not its whole computation
+// (measured ~30 warp instructions per group before).
 template <bool VALS, int THREADS, int IN>
 __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
-                                                                   const unsigned int* n_hot) {
+                                                                   const unsigned int* n_hot, const InCtx c) {
     constexpr int WARPS = THREADS / 32;
     using SM = stream::Smem<VALS, WARPS>;
     extern __shared__ __align__(16) uint8_t smem_raw[];
@@ -1002,12 +1011,6 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     uint32_t qhead = 0, qtail = 0;  // warp-uniform ring counters
     PrepCursor pc;
 
-    InCtx c;
-    c.ngroups = (uint32_t)((b.n + 31) / 32);
-    c.tail = (uint32_t)(b.n - (uint64_t)(c.ngroups ? c.ngroups - 1 : 0) * 32);
-    c.nw = gridDim.x * WARPS;
-    c.kend = IN == IN_IDX ? 0ull : (IN == IN_CSR ? ld_in64(b.ko + b.n) : b.n * (uint64_t)b.kw);
-    c.kal = !(reinterpret_cast<uintptr_t>(b.keys) & 15);
     bool w_full = false, w_quiet = false;  // warp-uniform: pool ran out / quiescence observed
 
     // pipeline prologue: group g (stages 1+2 done), group gn (stage 1 in flight)
@@ -2508,7 +2511,7 @@ int sepo_launch_evict_copy(const Dev& d, uint32_t n, uint8_t* dst, int grid, cud
 }
 
 int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
-                       uint32_t halt_slots) {
+                       uint32_t halt_slots, uint64_t key_end) {
     if (mode == 2) {
         insert_basic_kernel<<<grid, 1024, 0, s>>>(d, b, halt_slots);
         return cudaGetLastError();
@@ -2549,14 +2552,20 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             attr = true;
         }
         const int in = b.idx ? IN_IDX : (b.ko ? IN_CSR : IN_FIXED);
+        InCtx c;
+        c.ngroups = (uint32_t)((b.n + 31) / 32);
+        c.tail = (uint32_t)(b.n - (uint64_t)(c.ngroups ? c.ngroups - 1 : 0) * 32);
+        c.nw = (uint32_t)grid * (T / 32);
+        c.kend = in == IN_IDX ? 0ull : (in == IN_CSR ? key_end : b.n * (uint64_t)b.kw);
+        c.kal = !(reinterpret_cast<uintptr_t>(b.keys) & 15);
         if (b.vals) {
-            if (in == IN_CSR) insert_stream_kernel<true, T, IN_CSR><<<grid, T, sm, s>>>(d, b, hl, nh);
-            else if (in == IN_FIXED) insert_stream_kernel<true, T, IN_FIXED><<<grid, T, sm, s>>>(d, b, hl, nh);
-            else insert_stream_kernel<true, T, IN_IDX><<<grid, T, sm, s>>>(d, b, hl, nh);
+            if (in == IN_CSR) insert_stream_kernel<true, T, IN_CSR><<<grid, T, sm, s>>>(d, b, hl, nh, c);
+            else if (in == IN_FIXED) insert_stream_kernel<true, T, IN_FIXED><<<grid, T, sm, s>>>(d, b, hl, nh, c);
+            else insert_stream_kernel<true, T, IN_IDX><<<grid, T, sm, s>>>(d, b, hl, nh, c);
         } else {
-            if (in == IN_CSR) insert_stream_kernel<false, T, IN_CSR><<<grid, T, sm, s>>>(d, b, hl, nh);
-            else if (in == IN_FIXED) insert_stream_kernel<false, T, IN_FIXED><<<grid, T, sm, s>>>(d, b, hl, nh);
-            else insert_stream_kernel<false, T, IN_IDX><<<grid, T, sm, s>>>(d, b, hl, nh);
+            if (in == IN_CSR) insert_stream_kernel<false, T, IN_CSR><<<grid, T, sm, s>>>(d, b, hl, nh, c);
+            else if (in == IN_FIXED) insert_stream_kernel<false, T, IN_FIXED><<<grid, T, sm, s>>>(d, b, hl, nh, c);
+            else insert_stream_kernel<false, T, IN_IDX><<<grid, T, sm, s>>>(d, b, hl, nh, c);
         }
     } else {
         const hot::Entry* hl = nullptr;
