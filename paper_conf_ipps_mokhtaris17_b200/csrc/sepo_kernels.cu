@@ -178,7 +178,10 @@ __device__ __forceinline__ uint32_t reserve_head(const Dev& d, uint8_t* e, uint3
 //        the global entries when the CTA finishes (hot entries are resident for the whole
 //        generation, so each record's SUCCESS is final).
 namespace hot {
-constexpr int K = 2048;          // hot keys at most
+#ifndef SEPO_HOT_K
+#define SEPO_HOT_K 2048
+#endif
+constexpr int K = SEPO_HOT_K;    // hot keys at most (a power of two)
 constexpr int NB = 1024;         // shared buckets of 4 slots (2-choice): constant-time probe
 constexpr int NH = 4 * NB;       // slots
 constexpr uint32_t EMPTY_LEN = 0xffffffffu;
@@ -396,17 +399,27 @@ struct CtaState {                 // allocator slot (the CTA's active pages) + p
 #ifndef SEPO_HOT_DIRECT
 #define SEPO_HOT_DIRECT 1  // direct-indexed hot set (C2 4x pass 1 22.2 -> 21.3 ms); 0: 4-way bucket fingerprints
 #endif
+// slot word of the direct-indexed hot sets: fingerprint (hash bits + the key length saturated at
+// 255) | 1 | key index (B bits); 0 marks an empty slot
+template <int B>
+__device__ __forceinline__ uint32_t dfp_b(uint64_t h, uint32_t len) {
+    return ((((uint32_t)(h >> (64 - (23 - B))) << 8) | min(len, 255u)) << (B + 1)) | (1u << B);
+}
 #if SEPO_HOT_DIRECT
 // Direct-indexed hot set: DS one-word slots (2-choice, one slot per choice); a slot holds the key's
 // fingerprint and its index into the dense key arrays, so a probe is two 4-byte loads, two
 // compares and one 16-byte key load.
-constexpr int DS = 16384;                 // slots (hot keys <= hot::K = 2048: load <= 1/8)
+#ifndef SEPO_HOT_DS
+#define SEPO_HOT_DS 16384
+#endif
+constexpr int DS = SEPO_HOT_DS;           // slots (2048 hot keys in 16384: load <= 1/8)
 constexpr int NKEY = hot::K;
+constexpr int IDXB = NKEY <= 2048 ? 11 : (NKEY <= 4096 ? 12 : 13);  // key-index bits of a slot word
 __device__ __forceinline__ uint32_t ds1(uint64_t h) { return (uint32_t)(h >> 3) & (DS - 1); }
 __device__ __forceinline__ uint32_t ds2(uint64_t h) { return (uint32_t)(h >> 17) & (DS - 1); }
 // slot word: fingerprint (12 hash bits + the key length saturated at 255) | 1 | key index (11 bits)
 __device__ __forceinline__ uint32_t dfp(uint64_t h, uint32_t len) {
-    return ((((uint32_t)(h >> 52) << 8) | min(len, 255u)) << 12) | 0x800u;
+    return dfp_b<IDXB>(h, len);
 }
 #else
 constexpr int NKEY = hot::NH;
@@ -429,6 +442,10 @@ struct Smem {
     } q[WARPS];
     CtaState cs;
 };
+#if SEPO_HOT_K == 2048  // (experiments with more hot keys only fit the implicit-value kernel)
+static_assert(sizeof(Smem<true, SEPO_STREAM_THREADS / 32>) <= 232448, "stream kernel shared memory > 227 KB");
+#endif
+static_assert(sizeof(Smem<false, SEPO_STREAM_THREADS / 32>) <= 232448, "stream kernel shared memory > 227 KB");
 // Fingerprint of a hot slot: 23 hash bits, bit 8 always set (0 marks an empty slot) and the key
 // length (saturated at 255) in the low byte, so a fingerprint match also fixes the length of
 // keys shorter than 255 bytes and the full-key check is one 16-byte compare.
@@ -1077,8 +1094,9 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         if (have_hot) {
             const uint32_t f = stream::dfp(h, len);
             const uint32_t t1 = S.tags[stream::ds1(h)], t2 = S.tags[stream::ds2(h)];
-            const bool m1 = (t1 & 0xfffff800u) == f, m2 = (t2 & 0xfffff800u) == f;
-            const uint32_t p = (m1 ? t1 : t2) & 0x7ffu;
+            constexpr uint32_t IM = (1u << stream::IDXB) - 1u;
+            const bool m1 = (t1 & ~IM) == f, m2 = (t2 & ~IM) == f;
+            const uint32_t p = (m1 ? t1 : t2) & IM;
 #if SEPO_BRANCHLESS
             // branch-free common case: the candidate's 16 key bytes are loaded for every lane (p is
             // always a valid index); keys longer than 16 bytes take a warp-uniform slow path
@@ -2138,6 +2156,7 @@ constexpr int THREADS = 1024, WARPS = THREADS / 32;
 constexpr int WB = 512;    // window bytes: 32 lanes x 16 B
 constexpr int CHW = 64;    // consecutive windows a warp streams before it strides
 constexpr int DSZ = 8192;  // hot slots (the text ring takes the room of half the CSR kernel's slots)
+constexpr int TK = 2048;   // hot keys at most
 __device__ __forceinline__ uint32_t ds1(uint64_t h) { return (uint32_t)(h >> 3) & (DSZ - 1); }
 __device__ __forceinline__ uint32_t ds2(uint64_t h) { return (uint32_t)(h >> 17) & (DSZ - 1); }
 struct WarpText {
@@ -2147,9 +2166,9 @@ struct WarpText {
 };
 struct Smem {
     uint32_t tags[DSZ];
-    ulonglong2 kw[hot::K];
-    uint32_t ref[hot::K];
-    unsigned int sum[hot::K];
+    ulonglong2 kw[TK];
+    uint32_t ref[TK];
+    unsigned int sum[TK];
     stream::Smem<false, WARPS>::Queue q[WARPS];
     WarpText w[WARPS];
     stream::CtaState cs;
@@ -2195,7 +2214,7 @@ __global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, B
     extern __shared__ __align__(16) uint8_t smem_raw[];
     textk::Smem& S = *reinterpret_cast<textk::Smem*>(smem_raw);
     const uint32_t tid = threadIdx.x, lane = lane_id(), wid = tid >> 5;
-    for (int p = tid; p < hot::K; p += THREADS) { S.ref[p] = 0; S.sum[p] = 0; }
+    for (int p = tid; p < TK; p += THREADS) { S.ref[p] = 0; S.sum[p] = 0; }
     for (int p = tid; p < DSZ; p += THREADS) S.tags[p] = 0u;
     if (tid == 0) {
         S.cs.cur[0] = d.cursors[2 * blockIdx.x];
@@ -2206,10 +2225,10 @@ __global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, B
     __syncthreads();
     const unsigned nh = hl ? *n_hot : 0u;
     for (int cls = 31; cls >= 0 && nh; --cls) {  // hot set, most frequent keys first (as the CSR kernel)
-        for (unsigned j = tid; j < nh && j < (unsigned)hot::K; j += THREADS) {
+        for (unsigned j = tid; j < nh && j < (unsigned)TK; j += THREADS) {
             const hot::Entry e = hl[j];
             if (e.ref == 0 || hot::count_class(e.count) != cls) continue;
-            const uint32_t f = stream::dfp(e.h, e.len) | j;
+            const uint32_t f = stream::dfp_b<11>(e.h, e.len) | j;
             if (atomicCAS(&S.tags[ds1(e.h)], 0u, f) == 0u || atomicCAS(&S.tags[ds2(e.h)], 0u, f) == 0u) {
                 S.kw[j] = make_ulonglong2(e.w0, e.w1);
                 S.ref[j] = e.ref;
@@ -2298,7 +2317,7 @@ __global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, B
                 // ---- hot set (a2)
                 int pos = -1;
                 if (have_hot) {
-                    const uint32_t f = stream::dfp(h, len);
+                    const uint32_t f = stream::dfp_b<11>(h, len);
                     const uint32_t t1 = S.tags[ds1(h)], t2 = S.tags[ds2(h)];
                     const bool m1 = (t1 & 0xfffff800u) == f, m2 = (t2 & 0xfffff800u) == f;
                     const uint32_t q = (m1 ? t1 : t2) & 0x7ffu;
@@ -2355,7 +2374,7 @@ __global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, B
     if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
     if (lane == 0 && words) atomicAdd(&d.ctrl->text_words, words);
     __syncthreads();
-    for (int p = tid; p < hot::K; p += THREADS) {
+    for (int p = tid; p < TK; p += THREADS) {
         if (S.ref[p] == 0 || S.sum[p] == 0) continue;
         uint8_t* e = ref_ptr(d, S.ref[p]);
         red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(e, ldcg32(e + 12))), (unsigned long long)S.sum[p]);
@@ -2495,9 +2514,9 @@ int sepo_launch_insert_text(const Dev& d, const Batch& b, int grid, cudaStream_t
         cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
         hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, b.n / n_sample, n_sample, tab);
         hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
-        hot_threshold_kernel<<<1, 1024, 0, s>>>(hist, 4u, (uint32_t)hot::K);
-        hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)hot::K);
-        hot_clamp_kernel<<<1, 32, 0, s>>>(n_out, (uint32_t)hot::K);
+        hot_threshold_kernel<<<1, 1024, 0, s>>>(hist, 4u, (uint32_t)textk::TK);
+        hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)textk::TK);
+        hot_clamp_kernel<<<1, 32, 0, s>>>(n_out, (uint32_t)textk::TK);
         hot_resolve_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
         hl = list;
         nh = n_out;
