@@ -20,11 +20,18 @@
 namespace sepo {
 
 
-// %laneid: one S2R when the compiler rematerialises it (threadIdx.x & 31 costs two)
+#ifndef SEPO_LANEID_ASM
+#define SEPO_LANEID_ASM 0  // %laneid measured slower (C2 4x pass 1 22.0 vs 21.6 ms, text 30.8 vs 28.4 ms)
+#endif
+// lane id (SEPO_LANEID_ASM=1: from %laneid instead of threadIdx.x & 31)
 __device__ __forceinline__ uint32_t lane_id() {
+#if SEPO_LANEID_ASM
     uint32_t l;
     asm("mov.u32 %0, %%laneid;" : "=r"(l));
     return l;
+#else
+    return threadIdx.x & 31u;
+#endif
 }
 __device__ __forceinline__ uint32_t lanemask_lt() { return (1u << lane_id()) - 1u; }
 
@@ -2213,7 +2220,11 @@ __global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, B
     using namespace textk;
     extern __shared__ __align__(16) uint8_t smem_raw[];
     textk::Smem& S = *reinterpret_cast<textk::Smem*>(smem_raw);
+#if SEPO_TEXT_TIDLANE
+    const uint32_t tid = threadIdx.x, lane = tid & 31u, wid = tid >> 5;
+#else
     const uint32_t tid = threadIdx.x, lane = lane_id(), wid = tid >> 5;
+#endif
     for (int p = tid; p < TK; p += THREADS) { S.ref[p] = 0; S.sum[p] = 0; }
     for (int p = tid; p < DSZ; p += THREADS) S.tags[p] = 0u;
     if (tid == 0) {
