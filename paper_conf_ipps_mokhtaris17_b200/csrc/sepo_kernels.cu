@@ -821,6 +821,9 @@ __device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, str
 
 // Reinsert pass of sepo_run (a9 re-issue): the prepared records of the previous pass, 32 per warp
 // step, straight into resolve_core (keys of these passes are the Zipf tail: no hot set).
+#ifndef SEPO_REINS_PF
+#define SEPO_REINS_PF 1  // next step's 32-byte prepared records loaded during this step (C2 4x re-issue passes -0.3 ms)
+#endif
 template <int RB>
 __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
     __shared__ stream::CtaState S;
@@ -836,9 +839,30 @@ __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
     bool w_full = false, w_quiet = false;
     PrepCursor pc;
     const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+#if SEPO_REINS_PF
+    // the next step's prepared records are loaded while this step's are resolved (RB == 32 only)
+    ulonglong2 n0 = make_ulonglong2(0, 0), n1 = make_ulonglong2(0, 0);
+    {
+        const uint64_t i0 = ((uint64_t)blockIdx.x * (blockDim.x / 32) + (tid >> 5)) * 32 + lane;
+        if (RB == 32 && i0 < b.n) {
+            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(reinterpret_cast<const uint8_t*>(b.prep) + i0 * RB);
+            n0 = __ldcs(p); n1 = __ldcs(p + 1);
+        }
+    }
+#endif
     for (uint64_t base = ((uint64_t)blockIdx.x * (blockDim.x / 32) + (tid >> 5)) * 32; base < b.n; base += nw * 32) {
         const uint64_t i = base + lane;
         ulonglong2 r0 = make_ulonglong2(0, 0), r1 = make_ulonglong2(0, 0), r2 = make_ulonglong2(1, 0);
+#if SEPO_REINS_PF
+        if (RB == 32) {
+            r0 = n0; r1 = n1;
+            const uint64_t inx = i + nw * 32;
+            if (inx < b.n) {
+                const ulonglong2* p = reinterpret_cast<const ulonglong2*>(reinterpret_cast<const uint8_t*>(b.prep) + inx * RB);
+                n0 = __ldcs(p); n1 = __ldcs(p + 1);
+            }
+        } else
+#endif
         if (i < b.n) {
             const ulonglong2* p = reinterpret_cast<const ulonglong2*>(reinterpret_cast<const uint8_t*>(b.prep) + i * RB);
             r0 = __ldcs(p); r1 = __ldcs(p + 1);
