@@ -195,14 +195,32 @@ __device__ __forceinline__ uint4 ld_in128(const void* p) {
 __device__ __forceinline__ uint64_t ldcg64(const void* p) { return __ldcg(reinterpret_cast<const unsigned long long*>(p)); }
 __device__ __forceinline__ uint32_t ldcg32(const void* p) { return __ldcg(reinterpret_cast<const unsigned int*>(p)); }
 
+#ifndef SEPO_TAIL_L1
+#define SEPO_TAIL_L1 1   // C3 pass 1 55.2 -> 50.4 ms
+#endif
+#ifndef SEPO_HEAD_L1
+#define SEPO_HEAD_L1 0   // the per-lane first-16-byte loads (long-key groups, index re-issue) L1-allocating too
+#endif
+// input words read lane by lane (key tails beyond the first 16 bytes): L1-allocating, so the
+// group's neighbouring keys (one 128-byte line holds two 64-byte URLs) are read from L1 after the
+// first lane's miss (L1::no_allocate sent every 8-byte tail load to L2: C3 pass 1 load-bound)
+__device__ __forceinline__ uint64_t ld_tail64(const void* p) {
+#if SEPO_TAIL_L1
+    uint64_t v;
+    asm("ld.global.nc.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol_in()));
+    return v;
+#else
+    return ld_in64(p);
+#endif
+}
 // Bytes [p, p+nb) (1 <= nb <= 8) of immutable INPUT as a little-endian word, zero-extended.
 // Only the aligned words that contain requested bytes are read.
 __device__ __forceinline__ uint64_t load_in_word(const uint8_t* p, uint32_t nb) {
     uintptr_t a = reinterpret_cast<uintptr_t>(p);
     uint32_t sh = (uint32_t)(a & 7u);
     const unsigned long long* q = reinterpret_cast<const unsigned long long*>(a - sh);
-    uint64_t v = ld_in64(q) >> (8 * sh);
-    if (sh + nb > 8) v |= ld_in64(q + 1) << (64 - 8 * sh);
+    uint64_t v = ld_tail64(q) >> (8 * sh);
+    if (sh + nb > 8) v |= ld_tail64(q + 1) << (64 - 8 * sh);
     if (nb < 8) v &= (1ull << (8 * nb)) - 1ull;
     return v;
 }
@@ -344,9 +362,15 @@ __device__ __forceinline__ void load_key16(const uint8_t* p, uint32_t len, uint6
     const unsigned long long* q = reinterpret_cast<const unsigned long long*>(a - sh);
     const uint32_t nb = len < 16 ? len : 16;
     const uint32_t nw = (sh + nb + 7) >> 3;  // aligned words touched (1..3)
+#if SEPO_HEAD_L1
+    const uint64_t x0 = ld_tail64(q);
+    const uint64_t x1 = nw > 1 ? ld_tail64(q + 1) : 0ull;
+    const uint64_t x2 = nw > 2 ? ld_tail64(q + 2) : 0ull;
+#else
     const uint64_t x0 = ld_in64(q);
     const uint64_t x1 = nw > 1 ? ld_in64(q + 1) : 0ull;
     const uint64_t x2 = nw > 2 ? ld_in64(q + 2) : 0ull;
+#endif
     if (sh == 0) { w0 = x0; w1 = x1; }
     else {
         w0 = (x0 >> (8 * sh)) | (x1 << (64 - 8 * sh));
