@@ -400,6 +400,21 @@ def run_ours(args):
             "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if not pk.get("_fallback") else "fallback 6.65 TB/s",
             "issue": issue}
 
+    # host link: page bytes evicted (intermediate generations + the final one)
+    # over the eviction phase time, against the measured pinned D2H bandwidth (PEAKS_EXTRA.json)
+    host_link = None
+    try:
+        d2h_peak = json.load(open(os.path.join(ROOT, "PEAKS_EXTRA.json"))).get("d2h_GBps")
+    except Exception:
+        d2h_peak = None
+    if st["t_evict_ms"] > 0:
+        gbs = st["bytes_evicted"] / (st["t_evict_ms"] / 1e3) / 1e9
+        host_link = {"bytes_evicted_per_step": st["bytes_evicted"], "evict_ms_per_step": st["t_evict_ms"],
+                     "achieved": gbs, "unit": "GB/s", "peak": d2h_peak,
+                     "frac": (gbs / d2h_peak) if d2h_peak else None,
+                     "note": "evict phase includes seal/classify kernels and the directory reset; peak = "
+                             "measured pinned D2H (PEAKS_EXTRA.json)"}
+
     # end to end through sepo_run with pinned HOST buffers (H2D + job + host result assembly)
     e2e = None
     if args.e2e_steps > 0 and not routed:
@@ -506,7 +521,7 @@ def run_ours(args):
                            "parallelism": (f"key-hash sharded x{world} (sepo_partition + NCCL all-to-all)" if routed
                                            else "1 GPU"),
                            "phase_ms": {kk: st[kk] for kk in ("t_insert_ms", "t_reprobe_ms", "t_compact_ms", "t_evict_ms")}},
-                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+                "roofline": roof, "host_link": host_link, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
                 "gpu_launches": info["launches"], "slowdown_curve": curve, "raw_text": raw_text}
         print(json.dumps(line), flush=True)
     t.close()
