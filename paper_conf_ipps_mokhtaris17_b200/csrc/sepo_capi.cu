@@ -117,7 +117,9 @@ struct sepo_table {
     DevBuf prep[2];  // sepo_run COMBINE: prepared re-issue records (ping-pong)
     DevBuf prep_n;   // their device counters
     DevBuf lk_pages; // sepo_lookup: page ids of the generation being probed
-    bool lookup_done = false;  // sepo_lookup restored old generations into the pool: no inserts until reset
+    bool lookup_done = false;
+    std::vector<cudaEvent_t>* h2d_chunks = nullptr;  // sepo_run on host input: copy events of pass-1 chunks
+    uint64_t h2d_chunk_records = 0;  // sepo_lookup restored old generations into the pool: no inserts until reset
     DevBuf tbm;      // sepo_run_text: start bits of declined words that did not fit the prepared list
     // cuStreamWriteValue32 (driver entry point): the copy stream publishes eviction progress
     int (*write_value32)(cudaStream_t, unsigned long long, unsigned int, unsigned int) = nullptr;
@@ -1097,6 +1099,54 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
     if (rc) return rc;
     const bool dev = is_device_ptr(keys) && is_device_ptr(ko) && is_device_ptr(vals) && is_device_ptr(vo);
     const uint32_t kw = t->opts.fixed_key_width, vw = t->opts.fixed_val_width;
+    // (tests shrink the thresholds: SEPO_H2D_PIPE_MIN records, SEPO_H2D_CHUNK records per chunk)
+    const char* pmin = getenv("SEPO_H2D_PIPE_MIN");
+    const uint64_t pipe_min = pmin ? strtoull(pmin, nullptr, 10) : (64ull << 20);
+    if (!dev && n && t->opts.mode == SEPO_COMBINE_SUM_U64 && ko && !vo && n >= pipe_min && !getenv("SEPO_NO_H2D_PIPE")) {
+        // host input, COMBINE: the H2D copy (P:L227 counts this transfer) is pipelined with pass 1 —
+        // chunks of records go over the host link on the copy stream while the previous chunk is
+        // inserted; the staged copy keeps the caller's absolute offsets
+        uint64_t kbytes = 0, vbytes = 0, k0 = 0;
+        if (ko) { k0 = ko[0]; kbytes = ko[n] - ko[0]; } else kbytes = n * (uint64_t)kw;
+        if (vals) vbytes = n * (uint64_t)vw;
+        if (t->in_stage[0].grow(kbytes + 16) || (ko && t->in_stage[1].grow((n + 1) * 8)) ||
+            (vals && t->in_stage[2].grow(vbytes + 16)))
+            return fail(SEPO_E_NOMEM, "device staging for host input");
+        const char* pch = getenv("SEPO_H2D_CHUNK");
+        uint64_t per = pch ? strtoull(pch, nullptr, 10) : (32ull << 20);  // records per chunk
+        per = std::max<uint64_t>(32, per & ~31ull);                       // a multiple of 32: bitmap words
+        const uint64_t nch = (n + per - 1) / per;
+        std::vector<cudaEvent_t> evs(nch);
+        for (auto& e : evs) cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+        cudaEvent_t h0, h1;
+        cudaEventCreate(&h0);
+        cudaEventCreate(&h1);
+        CK(t, cudaEventRecord(h0, t->copy_stream));
+        uint8_t* kst = (uint8_t*)t->in_stage[0].p;
+        uint64_t* ost = (uint64_t*)t->in_stage[1].p;
+        for (uint64_t c = 0; c < nch; ++c) {
+            const uint64_t r0 = c * per, r1 = std::min(n, r0 + per);
+            const uint64_t b0 = ko ? ko[r0] - k0 : r0 * kw, b1 = ko ? ko[r1] - k0 : r1 * kw;
+            CK(t, cudaMemcpyAsync(kst + b0, keys + k0 + b0, b1 - b0, cudaMemcpyHostToDevice, t->copy_stream));
+            // r1 - r0 + 1 offsets: the chunk's last key ends at ko[r1] (the next chunk copies it again)
+            if (ko) CK(t, cudaMemcpyAsync(ost + r0, ko + r0, (r1 - r0 + 1) * 8, cudaMemcpyHostToDevice, t->copy_stream));
+            if (vals) CK(t, cudaMemcpyAsync((uint8_t*)t->in_stage[2].p + r0 * vw, vals + r0 * vw, (r1 - r0) * vw,
+                                            cudaMemcpyHostToDevice, t->copy_stream));
+            CK(t, cudaEventRecord(evs[c], t->copy_stream));
+        }
+        CK(t, cudaEventRecord(h1, t->copy_stream));
+        t->h2d_chunks = &evs;
+        t->h2d_chunk_records = per;
+        const int64_t r = sepo_run(t, kst - k0, ko ? ost : nullptr, vals ? (const uint8_t*)t->in_stage[2].p : nullptr,
+                                   nullptr, n);
+        t->h2d_chunks = nullptr;
+        cudaEventSynchronize(h1);
+        t->st.t_h2d_ms += elapsed_ms(h0, h1);
+        for (auto& e : evs) cudaEventDestroy(e);
+        cudaEventDestroy(h0);
+        cudaEventDestroy(h1);
+        return r;
+    }
     if (!dev && n) {
         // host input: stage it in device memory (one H2D per array, P:L227 counts this transfer)
         auto t0 = std::chrono::steady_clock::now();
@@ -1153,12 +1203,35 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
             cur.out_cap = cap;
         }
     }
+    std::vector<cudaEvent_t>* chunks = t->h2d_chunks;  // pass 1 of pipelined host input
+    t->h2d_chunks = nullptr;
     while (cur.n > 0) {
         if (t->bm.grow(((cur.n + 31) / 32) * 4)) return fail(SEPO_E_NOMEM, "bitmap scratch");
         cur.bitmap = (uint32_t*)t->bm.p;
-        int64_t c = insert_impl(t, cur);
-        if (c < 0) return c;
-        uint64_t kb = t->h_ctrl->kept_key_bytes, vb = 0;
+        int64_t c = 0;
+        uint64_t kb = 0, vb = 0;
+        if (chunks) {  // insert each chunk as soon as its copy landed
+            const uint64_t per = t->h2d_chunk_records;
+            for (size_t k = 0; k < chunks->size(); ++k) {
+                CK(t, cudaStreamWaitEvent(t->stream, (*chunks)[k], 0));
+                Batch bc = cur;
+                const uint64_t r0 = k * per, r1 = std::min(cur.n, r0 + per);
+                if (cur.ko) bc.ko = cur.ko + r0;
+                else bc.keys = cur.keys + r0 * (uint64_t)cur.kw;
+                if (cur.vals) bc.vals = cur.vals + r0 * (uint64_t)cur.vw;
+                bc.n = r1 - r0;
+                bc.bitmap = cur.bitmap + r0 / 32;
+                const int64_t cc = insert_impl(t, bc);
+                if (cc < 0) return cc;
+                c += cc;
+                kb += t->h_ctrl->kept_key_bytes;
+            }
+            chunks = nullptr;
+        } else {
+            c = insert_impl(t, cur);
+            if (c < 0) return c;
+            kb = t->h_ctrl->kept_key_bytes;
+        }
         if (c > 0 && !combine_exact) c = reprobe_impl(t, cur, &kb, &vb);
         if (c < 0) return c;
         if (c == 0) break;

@@ -359,3 +359,25 @@ def test_evict_copy_paths(cuda, monkeypatch, cfg, evk):
     got, passes, st = run_job(s, sepo().budget_for(1 << 14, 4096, P), 1 << 14, 4096, inputs=inp, check_dups=True, **kw)
     assert_same(got, exp)
     assert passes >= 3
+
+
+@pytest.mark.parametrize("ratio", [0.5, 4])
+def test_host_input_pipelined(cuda, monkeypatch, ratio):
+    """host (pinned numpy) input with the H2D copy pipelined with pass 1 in chunks of records
+    (thresholds shrunk for the test): same result as the oracle, in and over budget"""
+    monkeypatch.setenv("SEPO_H2D_PIPE_MIN", "1000")
+    monkeypatch.setenv("SEPO_H2D_CHUNK", "40000")
+    s = gen.config("C1")
+    hk, ho, _ = s.host()
+    exp = oracle_expected(s)
+    inp = device_inputs(s)
+    F, P = budget_pages(s, ratio if ratio > 1 else 1, 1 << 14, 4096, inp)
+    P = P + 600 if ratio < 1 else P
+    t = sepo().Table(sepo().budget_for(1 << 14, 4096, P), 1 << 14, 4096, check_dups=True)
+    passes = t.run(hk, ho.astype(np.uint64))
+    got = sepo().result_dict(t.export())
+    st = t.stats()
+    t.close()
+    assert_same(got, exp)
+    assert st["records_inserted"] >= s.n and st["cross_gen_dups"] == 0
+    assert (passes == 1) if ratio < 1 else (passes >= 2)
