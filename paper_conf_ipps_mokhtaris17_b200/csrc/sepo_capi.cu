@@ -1306,14 +1306,47 @@ int64_t sepo_run_text(sepo_table* t, const uint8_t* text, uint64_t n_bytes) {
         if (t->dirty) { int64_t e = evict_impl(t, 0); if (e < 0) return e; }
         return 0;
     }
-    if (!is_device_ptr(text)) {  // host text: one staged H2D (P:L227 counts this transfer)
-        auto t0 = std::chrono::steady_clock::now();
+    if (!is_device_ptr(text)) {
+        // host text: the H2D copy (P:L227 counts this transfer) is pipelined with pass 1 — 1 GiB
+        // chunks (whole 512-byte windows) go over the host link on the copy stream, each with
+        // max(64 KiB, page_bytes) of the next so the words that cross its end are complete when its
+        // windows are inserted (a longer word cannot be stored anyway: SEPO_E_TOOLARGE)
         if (t->in_stage[0].grow(n_bytes + 16)) return fail(SEPO_E_NOMEM, "device staging for host text");
-        CK(t, cudaMemcpyAsync(t->in_stage[0].p, text, n_bytes, cudaMemcpyHostToDevice, t->stream));
-        CK(t, cudaStreamSynchronize(t->stream));
-        t->st.t_h2d_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
-        return sepo_run_text(t, (const uint8_t*)t->in_stage[0].p, n_bytes);
+        const char* pch = getenv("SEPO_H2D_TEXT_CHUNK");
+        uint64_t cb = pch ? strtoull(pch, nullptr, 10) : (1ull << 30);
+        cb = std::max<uint64_t>(512, cb & ~511ull);
+        const uint64_t nch = (n_bytes + cb - 1) / cb;
+        std::vector<cudaEvent_t> evs(nch);
+        for (auto& e : evs) cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+        cudaEvent_t h0, h1;
+        cudaEventCreate(&h0);
+        cudaEventCreate(&h1);
+        uint8_t* dst = (uint8_t*)t->in_stage[0].p;
+        CK(t, cudaEventRecord(h0, t->copy_stream));
+        uint64_t copied = 0;  // bytes [0, copied) are enqueued
+        for (uint64_t c = 0; c < nch; ++c) {
+            // the overlap covers any word that can be stored (an entry fits one page)
+            const uint64_t want = std::min<uint64_t>(n_bytes, (c + 1) * cb + std::max<uint64_t>(64ull << 10, t->page_bytes));
+            if (want > copied) {
+                CK(t, cudaMemcpyAsync(dst + copied, text + copied, want - copied, cudaMemcpyHostToDevice, t->copy_stream));
+                copied = want;
+            }
+            CK(t, cudaEventRecord(evs[c], t->copy_stream));
+        }
+        CK(t, cudaEventRecord(h1, t->copy_stream));
+        t->h2d_chunks = &evs;
+        t->h2d_chunk_records = cb;  // (bytes per chunk for text)
+        const int64_t r = sepo_run_text(t, dst, n_bytes);
+        t->h2d_chunks = nullptr;
+        cudaEventSynchronize(h1);
+        t->st.t_h2d_ms += elapsed_ms(h0, h1);
+        for (auto& e : evs) cudaEventDestroy(e);
+        cudaEventDestroy(h0);
+        cudaEventDestroy(h1);
+        return r;
     }
+    std::vector<cudaEvent_t>* chunks = t->h2d_chunks;  // pipelined host text: per-chunk copy events
+    t->h2d_chunks = nullptr;
     if ((uintptr_t)text & 15) return fail(SEPO_E_INVAL, "device text must be 16-byte aligned");
     const int64_t passes_start = (int64_t)t->st.passes;
     Batch cur{};
@@ -1345,8 +1378,21 @@ int64_t sepo_run_text(sepo_table* t, const uint8_t* text, uint64_t n_bytes) {
     CK(t, cudaMemsetAsync(&t->d.ctrl->text_words, 0, 8, t->stream));
     CK(t, cudaEventRecord(t->ev0, t->stream));
     if (t->hot.grow(sepo_hot_scratch_bytes())) return fail(SEPO_E_NOMEM, "hot-set scratch");
-    rc = sepo_launch_insert_text(t->d, cur, t->grid, t->stream, t->hot.p);
-    if (rc) return cuda_check(t, (cudaError_t)rc, "text insert kernel launch");
+    if (chunks) {  // each chunk's windows as soon as its copy landed; the hot set from the first
+        const uint64_t cb = t->h2d_chunk_records;
+        for (size_t k = 0; k < chunks->size(); ++k) {
+            CK(t, cudaStreamWaitEvent(t->stream, (*chunks)[k], 0));
+            Batch bc = cur;
+            bc.w_begin = (k * cb) / 512;
+            bc.w_end = std::min<uint64_t>((k + 1) * cb, n_bytes + 511) / 512;
+            if (k + 1 == chunks->size()) bc.w_end = ~0ull;
+            rc = sepo_launch_insert_text(t->d, bc, t->grid, t->stream, t->hot.p, k == 0 ? std::min<uint64_t>(cb, n_bytes) : 0);
+            if (rc) return cuda_check(t, (cudaError_t)rc, "text insert kernel launch");
+        }
+    } else {
+        rc = sepo_launch_insert_text(t->d, cur, t->grid, t->stream, t->hot.p, n_bytes);
+        if (rc) return cuda_check(t, (cudaError_t)rc, "text insert kernel launch");
+    }
     CK(t, cudaEventRecord(t->ev1, t->stream));
     t->st.kernel_launches += (n_bytes >= (64ull << 18)) ? 7 : 1;
     CK(t, cudaMemcpyAsync(&t->h_ko[0], cur.out_n, 8, cudaMemcpyDeviceToHost, t->stream));

@@ -2276,7 +2276,8 @@ __global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, B
     const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
     const uint8_t* T = b.keys;
     const uint64_t n = b.n;
-    const uint64_t nwin = (n + WB - 1) / WB;
+    const uint64_t nwin_all = (n + WB - 1) / WB;
+    const uint64_t wbeg = b.w_begin, nwin = b.w_end < nwin_all ? b.w_end : nwin_all;  // this launch's windows
     const bool big = n / 2 >= (1ull << 32);  // words < 2^32: a CTA-local count cannot wrap
     WarpText& W = S.w[wid];
     auto& Q = S.q[wid];
@@ -2286,7 +2287,7 @@ __global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, B
     unsigned long long words = 0;  // lane 0
     const uint8_t* ring = reinterpret_cast<const uint8_t*>(&W.t[0][0]);
     const uint64_t nwarps = (uint64_t)gridDim.x * WARPS;
-    for (uint64_t c0 = ((uint64_t)blockIdx.x * WARPS + wid) * CHW; c0 < nwin; c0 += nwarps * CHW) {
+    for (uint64_t c0 = wbeg + ((uint64_t)blockIdx.x * WARPS + wid) * CHW; c0 < nwin; c0 += nwarps * CHW) {
         const uint64_t c1 = (c0 + CHW < nwin) ? c0 + CHW : nwin;
         uint32_t prev = 1u;  // is the byte before the window a separator (text start: yes)
         if (c0 > 0) prev = is_sep(ld_in8(T + c0 * WB - 1)) ? 1u : 0u;
@@ -2535,11 +2536,20 @@ __global__ void __launch_bounds__(512) evict_copy_kernel(const uint8_t* __restri
 // ================================================================ launchers
 using namespace sepo;
 
-int sepo_launch_insert_text(const Dev& d, const Batch& b, int grid, cudaStream_t s, void* hot_scratch) {
+int sepo_launch_insert_text(const Dev& d, const Batch& b0, int grid, cudaStream_t s, void* hot_scratch,
+                            uint64_t sample_bytes) {
     const hot::Entry* hl = nullptr;
     const unsigned int* nh = nullptr;
     const uint64_t n_sample = 1ull << 18;
-    if (hot_scratch && b.n >= 64 * n_sample) {  // hot-set discovery on words at sampled byte offsets
+    const Batch& b = b0;
+    Batch bs = b0;  // bs.n: the prefix the sample positions come from (its words are read whole:
+    bs.n = sample_bytes < b0.n ? sample_bytes : b0.n;  // the caller has copied past the prefix)
+    if (hot_scratch && sample_bytes == 0) {  // reuse the previous launch's hot set
+        uint8_t* p = reinterpret_cast<uint8_t*>(hot_scratch);
+        hot::Entry* list = reinterpret_cast<hot::Entry*>(p + sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS);
+        hl = list;
+        nh = reinterpret_cast<unsigned int*>(list + hot::K);
+    } else if (hot_scratch && bs.n >= 64 * n_sample) {  // hot-set discovery on words at sampled byte offsets
         uint8_t* p = reinterpret_cast<uint8_t*>(hot_scratch);
         hot::SampleSlot* tab = reinterpret_cast<hot::SampleSlot*>(p);
         hot::Entry* list = reinterpret_cast<hot::Entry*>(p + sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS);
@@ -2547,7 +2557,7 @@ int sepo_launch_insert_text(const Dev& d, const Batch& b, int grid, cudaStream_t
         unsigned int* hist = n_out + 1;
         cudaMemsetAsync(tab, 0, sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS, s);
         cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
-        hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, b.n / n_sample, n_sample, tab);
+        hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, bs.n / n_sample, n_sample, tab);  // positions in the prefix
         hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
         hot_threshold_kernel<<<1, 1024, 0, s>>>(hist, 4u, (uint32_t)textk::TK);
         hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)textk::TK);

@@ -38,6 +38,7 @@ struct Batch {
     // words that do not fit the prepared list set bit (start) in tbm (u32 words over the text).
     uint32_t text = 0;
     uint32_t* tbm = nullptr;
+    uint64_t w_begin = 0, w_end = ~0ull;  // text: the 512-byte windows this launch tokenizes
 };
 }  // namespace sepo
 
@@ -62,7 +63,10 @@ int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec,
                               uint64_t total, cudaStream_t s);
 int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);
 int sepo_launch_evict_copy(const sepo::Dev& d, uint32_t n, uint8_t* dst, int grid, cudaStream_t s);
-int sepo_launch_insert_text(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s, void* hot_scratch);
+// sample_bytes: tokenize a hot-set sample from the first sample_bytes of the text (0: reuse the hot
+// set the previous launch selected, still in hot_scratch)
+int sepo_launch_insert_text(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s, void* hot_scratch,
+                            uint64_t sample_bytes);
 int sepo_launch_lookup_gen(const sepo::Dev& d, const sepo::Batch& b, const uint32_t* pages, uint32_t np,
                            unsigned long long* vals, uint32_t* found, cudaStream_t s);
 int sepo_launch_text_bits(const sepo::Dev& d, const sepo::Batch& b, unsigned long long* counter, cudaStream_t s);

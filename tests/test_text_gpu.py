@@ -93,3 +93,22 @@ def test_text_adversarial(cuda):
     assert got == {}
     got, passes, _ = run_text(_dev(b" \n \t"), 16)
     assert got == {}
+
+
+@pytest.mark.parametrize("chunk", [512, 4096, 1 << 20])
+def test_text_host_pipelined(cuda, monkeypatch, chunk):
+    """host text copied in chunks while earlier chunks are tokenized and inserted (the hot set from
+    the first chunk): same counts, including words across chunk ends and an over-budget run"""
+    monkeypatch.setenv("SEPO_H2D_TEXT_CHUNK", str(chunk))
+    s = gen.config("C1", scale=0.25)
+    text = s.text_host()
+    exp = s.expected_combine()
+    got, passes, _ = run_text(text, 4096)
+    assert got == exp and passes == 1
+    F = footprint_pages(s, 1 << 14, 4096)
+    got, passes, _ = run_text(text, max(8, F // 3))
+    assert got == exp and passes >= 2
+    t = b"".join([b"w%d " % i for i in range(3000)] + [b"L" * 1500, b" ", b"y" * 511, b"\n", b"z" * 513, b" end"])
+    exp2 = oracle.word_count_text(np.frombuffer(t, dtype=np.uint8))
+    got, _, _ = run_text(np.frombuffer(t, dtype=np.uint8).copy(), 256, pb=8192)
+    assert got == exp2
