@@ -1185,8 +1185,12 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
     // n/4 (SEPO_PREP_CAP overrides); on overflow the job continues on the index path.
     const char* no_prep = getenv("SEPO_NO_PREP");
     bool use_prep = t->opts.mode == SEPO_COMBINE_SUM_U64 && combine_exact && !(no_prep && no_prep[0] == '1') && n > 0;
-    const uint64_t prb = vals ? sizeof(PRec) : 32;  // prepared record bytes (implicit value 1: 32)
+    // prepared record bytes: 32 for implicit values, 32 for values with fixed keys of <= 8 bytes
+    // (the key is one word: {key, value, hash, offset | length}), else 48
+    const bool short_keys = !ko && kw > 0 && kw <= 8;
+    const uint64_t prb = (vals && !short_keys) ? sizeof(PRec) : 32;
     cur.prep_rb = (uint32_t)prb;
+    cur.prep_fmt = (vals && short_keys) ? 33u : 0u;
     if (use_prep) {
         uint64_t cap = std::max<uint64_t>(1ull << 16, n / 4);
         if (const char* pc = getenv("SEPO_PREP_CAP")) cap = strtoull(pc, nullptr, 10);

@@ -774,9 +774,10 @@ __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, strea
         if (act && res == R_POST && base >= b.out_cap && b.tbm)  // text: the list is full, mark the word
             atomicOr(b.tbm + (s >> 5), 1u << (s & 31));
         if (act && res == R_POST && base < b.out_cap) {
-            ulonglong2* o = reinterpret_cast<ulonglong2*>(reinterpret_cast<uint8_t*>(b.out) + base * RB);
-            o[0] = make_ulonglong2(w0, w1);
-            if (RB == 32) {  // implicit value 1: {key words, hash, offset | length << 48}
+            constexpr uint32_t RS = RB == 48 ? 48u : 32u;  // record bytes (RB 33: 32-byte records too)
+            ulonglong2* o = reinterpret_cast<ulonglong2*>(reinterpret_cast<uint8_t*>(b.out) + base * RS);
+            o[0] = make_ulonglong2(w0, RB == 33 ? v : w1);
+            if (RB == 32 || RB == 33) {  // {key words | key + value, hash, offset | length << 48}
                 o[1] = make_ulonglong2(h, s | ((unsigned long long)len << 48));
             } else {
                 o[1] = make_ulonglong2(h, s);
@@ -816,7 +817,9 @@ __device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, str
         const uint32_t ll = Q.ll[k];
         len = ll >> 5; gl = ll & 31u;
     }
-    resolve_core<VALS ? 48 : 32>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
+    if (!VALS) resolve_core<32>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
+    else if (b.prep_fmt == 33) resolve_core<33>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
+    else resolve_core<48>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
 }
 
 // Reinsert pass of sepo_run (a9 re-issue): the prepared records of the previous pass, 32 per warp
@@ -844,8 +847,8 @@ __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
     ulonglong2 n0 = make_ulonglong2(0, 0), n1 = make_ulonglong2(0, 0);
     {
         const uint64_t i0 = ((uint64_t)blockIdx.x * (blockDim.x / 32) + (tid >> 5)) * 32 + lane;
-        if (RB == 32 && i0 < b.n) {
-            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(reinterpret_cast<const uint8_t*>(b.prep) + i0 * RB);
+        if ((RB == 32 || RB == 33) && i0 < b.n) {
+            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(reinterpret_cast<const uint8_t*>(b.prep) + i0 * 32);
             n0 = __ldcs(p); n1 = __ldcs(p + 1);
         }
     }
@@ -854,32 +857,34 @@ __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
         const uint64_t i = base + lane;
         ulonglong2 r0 = make_ulonglong2(0, 0), r1 = make_ulonglong2(0, 0), r2 = make_ulonglong2(1, 0);
 #if SEPO_REINS_PF
-        if (RB == 32) {
+        if (RB == 32 || RB == 33) {
             r0 = n0; r1 = n1;
             const uint64_t inx = i + nw * 32;
             if (inx < b.n) {
-                const ulonglong2* p = reinterpret_cast<const ulonglong2*>(reinterpret_cast<const uint8_t*>(b.prep) + inx * RB);
+                const ulonglong2* p = reinterpret_cast<const ulonglong2*>(reinterpret_cast<const uint8_t*>(b.prep) + inx * 32);
                 n0 = __ldcs(p); n1 = __ldcs(p + 1);
             }
         } else
 #endif
         if (i < b.n) {
-            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(reinterpret_cast<const uint8_t*>(b.prep) + i * RB);
+            const ulonglong2* p = reinterpret_cast<const ulonglong2*>(reinterpret_cast<const uint8_t*>(b.prep) + i * (RB == 48 ? 48 : 32));
             r0 = __ldcs(p); r1 = __ldcs(p + 1);
             if (RB == 48) r2 = __ldcs(p + 2);
         }
         uint64_t s = r1.y, v = r2.x;
         uint32_t len = (uint32_t)r2.y;
         bool act;
-        if (RB == 32) {  // {w0, w1, h, s | len << 48}, value 1
+        uint64_t kw1 = r0.y;
+        if (RB == 32 || RB == 33) {  // {w0, w1 | value, h, s | len << 48}
             len = (uint32_t)(r1.y >> 48);
             s = r1.y & 0xffffffffffffull;
-            v = 1;
+            v = RB == 33 ? r0.y : 1ull;
+            if (RB == 33) kw1 = 0;  // keys of at most 8 bytes
             act = i < b.n && len != (uint32_t)PREP_HOLE32;
         } else {
             act = i < b.n && len != PREP_HOLE;
         }
-        resolve_core<RB>(d, b, S, act, r0.x, r0.y, r1.x, s, v, act ? len : 0u, (uint32_t)(i >> 5), (uint32_t)(i & 31), inj,
+        resolve_core<RB>(d, b, S, act, r0.x, kw1, r1.x, s, v, act ? len : 0u, (uint32_t)(i >> 5), (uint32_t)(i & 31), inj,
                      w_full, w_quiet, pc);
     }
     if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
@@ -2680,7 +2685,8 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
 }
 int sepo_launch_reinsert(const Dev& d, const Batch& b, int grid, cudaStream_t s) {
     if (b.n == 0) return cudaGetLastError();
-    if (b.prep_rb == 32) reinsert_kernel<32><<<grid, 1024, 0, s>>>(d, b);
+    if (b.prep_fmt == 33) reinsert_kernel<33><<<grid, 1024, 0, s>>>(d, b);
+    else if (b.prep_rb == 32) reinsert_kernel<32><<<grid, 1024, 0, s>>>(d, b);
     else reinsert_kernel<48><<<grid, 1024, 0, s>>>(d, b);
     return cudaGetLastError();
 }

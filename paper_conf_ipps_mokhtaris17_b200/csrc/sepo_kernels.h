@@ -33,6 +33,7 @@ struct Batch {
     const PRec* prep = nullptr;
     uint32_t prep_rb = 48;  // bytes per prepared record: 48 (PRec), or 32 when every value is 1:
                             // {w0, w1, h, s | len << 48} (a third less re-issue traffic)
+    uint32_t prep_fmt = 0;  // 33: 32-byte records {key, value, h, s | len << 48} (keys of <= 8 bytes)
     // raw-text input (sepo_run_text, NEXT-2): keys = text bytes, n = text bytes; records are the
     // words (maximal runs of non-separator bytes), identified by their start offset. Declined
     // words that do not fit the prepared list set bit (start) in tbm (u32 words over the text).
