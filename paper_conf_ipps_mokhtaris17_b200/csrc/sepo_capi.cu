@@ -471,7 +471,14 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
         CK(t, cudaStreamSynchronize(t->stream));
         key_end = t->h_ko[1];
     }
-    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p, halt_slots, key_end);
+    // in-budget tables larger than L2: the misses' directory lines are prefetched into L2 while
+    // they wait in the queue (measured: helps when the directory + entries live in HBM, hurts when
+    // a generation fits L2); SEPO_DIR_PF=0/1 forces it
+    static const int dpf_env = [] { const char* e = getenv("SEPO_DIR_PF"); return e ? atoi(e) : -1; }();
+    int l2 = 0;
+    cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device);
+    const bool dpf = dpf_env >= 0 ? dpf_env == 1 : (t->budget > (size_t)l2);
+    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p, halt_slots, key_end, dpf);
     if (rc) return cuda_check(t, (cudaError_t)rc, "insert kernel launch");
     CK(t, cudaEventRecord(t->ev1, t->stream));
     t->st.kernel_launches += (n >= (8ull << 18)) ? 7 : 1;

@@ -388,7 +388,9 @@ namespace stream {
 #define SEPO_IN_PREFETCH 0        // L2 prefetch of the input this many groups ahead (0: off)
 #endif
 #ifndef SEPO_DIR_PREFETCH
-#define SEPO_DIR_PREFETCH 0       // L2 prefetch of a queued miss's directory word (in budget -1.5 %, 4x +1.3 %)
+#define SEPO_DIR_PREFETCH 0       // 1: always L2-prefetch a queued miss's directory word (default: host
+                                  // decides per table, c.dirpf: on when the budget exceeds L2 — C5u 4x
+                                  // insert 67.3 -> 61.0 ms, C2 in budget 28.6 -> 28.1 ms, C2 4x off)
 #endif
 constexpr int THREADS = SEPO_STREAM_THREADS;
 constexpr uint64_t CH = SEPO_CHUNK_GROUPS;
@@ -540,6 +542,7 @@ struct InCtx {
     uint32_t ngroups, nw, tail;  // groups, warps in the grid, records in the last group (1..32)
     uint64_t kend;               // key bytes end of the batch (ko[n] or n*kw)
     bool kal;                    // key bytes 16-byte aligned (chunked loads allowed)
+    bool dirpf;                  // L2-prefetch a queued miss's directory word (the table exceeds L2)
 };
 // input forms of a batch (template parameter of the stream kernel): contiguous CSR keys, fixed-
 // width keys, or a re-issue index list into the caller's arrays
@@ -1224,11 +1227,10 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         const unsigned mm = __ballot_sync(FULLMASK, miss);
         if (lane == 0) b.bitmap[g] = 0u;
         if (miss) {
-#if SEPO_DIR_PREFETCH
-            // the directory word is read when the queue is resolved (a few groups later): start
-            // bringing its line into L2 now
-            asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(d.dir + bucket_of(h, d.n_buckets)));
-#endif
+            // the directory word is read when the queue is resolved (a few groups later): when the
+            // table does not fit L2 (host decision, c.dirpf) start bringing its line in now
+            if (SEPO_DIR_PREFETCH || c.dirpf)
+                asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(d.dir + bucket_of(h, d.n_buckets)));
             const uint32_t k = (qtail + __popc(mm & lanemask_lt())) & (stream::QCAP - 1);
             Q.w0[k] = w0; Q.w1[k] = w1; Q.h[k] = h; Q.s[k] = s;
             if (VALS) Q.v[k] = v;
@@ -2609,7 +2611,7 @@ int sepo_launch_evict_copy(const Dev& d, uint32_t n, uint8_t* dst, int grid, cud
 }
 
 int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
-                       uint32_t halt_slots, uint64_t key_end) {
+                       uint32_t halt_slots, uint64_t key_end, bool dir_prefetch) {
     if (mode == 2) {
         insert_basic_kernel<<<grid, 1024, 0, s>>>(d, b, halt_slots);
         return cudaGetLastError();
@@ -2656,6 +2658,7 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
         c.nw = (uint32_t)grid * (T / 32);
         c.kend = in == IN_IDX ? 0ull : (in == IN_CSR ? key_end : b.n * (uint64_t)b.kw);
         c.kal = !(reinterpret_cast<uintptr_t>(b.keys) & 15);
+        c.dirpf = dir_prefetch;
         if (b.vals) {
             if (in == IN_CSR) insert_stream_kernel<true, T, IN_CSR><<<grid, T, sm, s>>>(d, b, hl, nh, c);
             else if (in == IN_FIXED) insert_stream_kernel<true, T, IN_FIXED><<<grid, T, sm, s>>>(d, b, hl, nh, c);

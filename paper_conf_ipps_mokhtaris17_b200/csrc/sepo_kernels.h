@@ -45,7 +45,7 @@ struct Batch {
 
 // key_end: key_offsets[n] of a CSR batch (the end of its key bytes), read by the host
 int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
-                       uint32_t halt_slots = 0, uint64_t key_end = 0);
+                       uint32_t halt_slots = 0, uint64_t key_end = 0, bool dir_prefetch = false);
 int sepo_launch_reinsert(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s);
 size_t sepo_hot_scratch_bytes();
 int sepo_default_grid(int mode, int n_sms);
