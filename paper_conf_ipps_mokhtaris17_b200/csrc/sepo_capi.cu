@@ -1365,6 +1365,12 @@ int64_t sepo_run_text(sepo_table* t, const uint8_t* text, uint64_t n_bytes) {
     cur.n = n_bytes;
     cur.text = 1;
     cur.prep_rb = 32;
+    {
+        const char* e = getenv("SEPO_DIR_PF");
+        int l2 = 0;
+        cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device);
+        cur.dirpf = (e ? atoi(e) == 1 : t->budget > (size_t)l2) ? 1u : 0u;
+    }
     // prepared list for pass 1 (a word is >= 2 bytes with its separator; ~n/32 slots = a quarter of
     // 8-byte words), the overflow bitmap over the text bytes (zero between uses)
     uint64_t cap = std::max<uint64_t>(1ull << 16, n_bytes / 32);

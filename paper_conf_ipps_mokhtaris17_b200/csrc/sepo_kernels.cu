@@ -2401,6 +2401,8 @@ __global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, B
                 const bool miss = valid && pos < 0;
                 const unsigned mm = __ballot_sync(FULLMASK, miss);
                 if (miss) {
+                    if (b.dirpf)  // (tables larger than L2: see the CSR kernel)
+                        asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(d.dir + bucket_of(h, d.n_buckets)));
                     const uint32_t kq = (qtail + __popc(mm & lanemask_lt())) & (stream::QCAP - 1);
                     Q.w0[kq] = w0; Q.w1[kq] = w1; Q.h[kq] = h; Q.s[kq] = s;
                     Q.g[kq] = 0;

@@ -34,6 +34,7 @@ struct Batch {
     uint32_t prep_rb = 48;  // bytes per prepared record: 48 (PRec), or 32 when every value is 1:
                             // {w0, w1, h, s | len << 48} (a third less re-issue traffic)
     uint32_t prep_fmt = 0;  // 33: 32-byte records {key, value, h, s | len << 48} (keys of <= 8 bytes)
+    uint32_t dirpf = 0;     // text kernel: L2-prefetch queued misses' directory lines (table > L2)
     // raw-text input (sepo_run_text, NEXT-2): keys = text bytes, n = text bytes; records are the
     // words (maximal runs of non-separator bytes), identified by their start offset. Declined
     // words that do not fit the prepared list set bit (start) in tbm (u32 words over the text).
