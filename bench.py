@@ -8,10 +8,15 @@ postponed, and transfer the final generation to pinned host memory (P:L227 timin
 Default workload: C2 (word count, 8 GiB Zipf(1.0) text = 1.1e9 words, V = 2^22) with the device
 budget capped at F/4, i.e. the table is 4x the budget (BASELINE.json configs[1]).
 
-Prints ONE JSON line (rank 0). `value` is input GB/s (CSR bytes the job consumes: key bytes +
-8 B offsets [+ values]) over the device-timed steps; `e2e` is the same job through sepo_run with
-pinned HOST buffers (H2D of the input + job + result assembly on the host). The oracle
-(oracle/, test infrastructure) is run only by the cpu_baseline leg and by --impl reference.
+Prints ONE JSON line (rank 0). For word counts (C1/C2) the headline is SURVEY §8(d) M2 on the RAW
+text: `value` = GB/s of raw text (each word + one separator, 8.6 GB for C2) over the device-timed
+sepo_run_text jobs — the tokenizer is fused into the insert kernel, so it is inside the job;
+`e2e` = the same job from pinned HOST text through the public API (H2D + job + sepo_export).
+`csr_job` is the same workload from a pre-tokenised CSR (sepo_run). `roofline` is M1: the pass-1
+insert kernel of the IN-BUDGET job (C2 at 0.5x, one pass), CUDA events on the table's stream;
+`roofline_m1_c3` the same for C3 at P = 1; `roofline_headline_kernel` the headline step's own
+pass-1 kernel. The oracle (oracle/, test infrastructure) is run only by the cpu_baseline leg and
+by --impl reference.
 """
 import argparse
 import json
@@ -298,6 +303,114 @@ def timed_steps(job, t, steps, stream, route_fn=None):
                                      last=st)
 
 
+def cpu_info():
+    """host CPU model, nproc and the affinity mask size (SURVEY §8(d) timing protocol)"""
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except Exception:
+        pass
+    try:
+        aff = len(os.sched_getaffinity(0))
+    except Exception:
+        aff = None
+    return {"cpu_model": model, "nproc": os.cpu_count(), "affinity": aff}
+
+
+def time_text_jobs(t, text, steps, stream):
+    """`steps` raw-text jobs (sepo_run_text) back to back, CUDA events on the table's stream"""
+    import torch
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    p1, launches = 0.0, 0
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(steps):
+        t.reset()
+        t.run_text(text)
+        st = t.stats()
+        p1 += st["t_insert_ms_per_pass"][0]
+        launches += st["kernel_launches"]
+    e1.record(stream)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1), dict(p1_ms=p1, launches=launches, last=st)
+
+
+def roofline_of(alg_bytes, p1_ms_total, steps, pk, kernel, extra=None):
+    achieved = alg_bytes * steps / (p1_ms_total / 1e3) / 1e9
+    r = {"bound": "hbm", "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s", "frac": achieved / pk["hbm_gbs"],
+         "kernel": kernel, "alg_bytes_per_launch": alg_bytes, "launch_ms": p1_ms_total / steps,
+         "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy, burst)" if not pk.get("_fallback") else "fallback 6.65 TB/s"}
+    if extra:
+        r.update(extra)
+    return r
+
+
+def traffic_of(name):
+    """dram read+write bytes and warp instructions per launch from a committed ncu --set full capture"""
+    tj = os.path.join(ROOT, "profiles", name)
+    if not os.path.exists(tj):
+        return None
+    return json.load(open(tj))
+
+
+def issue_of(tr, n_records, launch_ms, clocks):
+    """instruction-issue roofline of a kernel (148 SMs x 4 schedulers x 1 warp instruction / cycle)"""
+    if not tr or "warp_instructions" not in tr:
+        return None
+    peak_wi = 148 * 4 * (clocks.get("sm_mhz") or 1965.0) * 1e6
+    wi_per_s = tr["warp_instructions"] / (launch_ms / 1e3)
+    return {"warp_instructions_per_launch": tr["warp_instructions"], "warp_instructions_per_record": tr["warp_instructions"] / n_records,
+            "achieved_warp_instr_per_s": wi_per_s, "peak_warp_instr_per_s": peak_wi, "frac": wi_per_s / peak_wi,
+            "ncu_issue_active": tr.get("issue_active_pct", 0) / 100.0, "source": tr.get("launch")}
+
+
+def e2e_text(t, text_dev, n_words, steps, world=1):
+    """the headline job end to end: pinned HOST text -> sepo_run_text (H2D pipelined with pass 1,
+    all passes, page D2H) -> sepo_export (host result assembly); wall clock, synchronized"""
+    import torch
+    tb = text_dev.numel()
+    ht = torch.empty(tb, dtype=torch.uint8, pin_memory=True)
+    ht.copy_(text_dev)
+    t.reset(); t.run_text(ht); t.export(copy=False)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    d2h = 0
+    for _ in range(steps):
+        t.reset()
+        t.run_text(ht)
+        t.export(copy=False)
+        d2h += t.stats()["bytes_evicted"]
+    el = (time.perf_counter() - t0) / steps
+    del ht
+    return {"value": world * tb / el / 1e9, "unit": "GB/s of raw text", "kv_inserts_per_s": world * n_words / el,
+            "h2d_bytes_per_step": tb, "d2h_bytes_per_step": d2h // steps,
+            "note": "sepo_run_text on pinned host text + sepo_export: H2D (pipelined with pass 1), all passes, page D2H, "
+                    "host result assembly"}
+
+
+def e2e_csr(t, k, o, v, csr, n, steps, world=1):
+    import torch
+    hk = torch.empty(k.numel(), dtype=torch.uint8, pin_memory=True); hk.copy_(k)
+    ho = torch.empty(o.numel(), dtype=torch.int64, pin_memory=True).copy_(o) if o is not None else None
+    hv = torch.empty(v.numel(), dtype=torch.uint8, pin_memory=True).copy_(v) if v is not None else None
+    t.reset(); t.run(hk, ho, hv); t.export(copy=False)
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    d2h = 0
+    for _ in range(steps):
+        t.reset()
+        t.run(hk, ho, hv)
+        t.export(copy=False)
+        d2h += t.stats()["bytes_evicted"]
+    el = (time.perf_counter() - t0) / steps
+    return {"value": world * csr / el / 1e9, "unit": "GB/s", "h2d_bytes_per_step": csr, "d2h_bytes_per_step": d2h // steps,
+            "kv_inserts_per_s": world * n / el,
+            "note": "sepo_run on pinned host CSR + sepo_export: H2D (pipelined), all passes, page D2H, host result assembly"}
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -307,101 +420,96 @@ def run_ours(args):
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    if args.route and world == 1 and not dist.is_initialized():
-        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        os.environ.setdefault("MASTER_PORT", "29511")
-        dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", local))
+    routed = world > 1 or args.route
+    if routed:
+        return run_routed(args, world, rank, local)
     job = Job(args.config, args.ratio, scale=args.scale)
     stream = torch.cuda.current_stream()
-    routed = world > 1 or args.route
-    fixed = job.stream.family == 2
-    route_fn = None
-    if routed:
-        # strong scaling: rank r holds records [r*n/W, (r+1)*n/W) of the SAME global stream; each
-        # step routes them by key hash (sepo_partition + NCCL all-to-all) and runs
-        # the SEPO job on the records this rank owns
-        from paper_conf_ipps_mokhtaris17_b200 import shard
-        if not dist.is_initialized():
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        n_all = job.stream.n
-        j0, j1 = rank * n_all // world, (rank + 1) * n_all // world
-        sk, so, sv = job.stream.device(j0, j1 - j0)
-        if fixed:
-            so = None
-
-        def route_fn():
-            return shard.route(sk, so, sv, route_seed=0x5eed, fixed_key_width=8 if fixed else 0,
-                               fixed_val_width=job.stream.val_width if sv is not None else 0)
-        job.distinct = max(1, job.distinct // world)  # keys per rank (sizes the directory)
-        job._inputs = route_fn()
-        job.slice_bytes = sk.numel() + (8 * (so.numel() - 1) if so is not None else 0) + (sv.numel() if sv is not None else 0)
-        job.slice_records = j1 - j0
-    job.inputs()
+    pk = peaks()
+    text_ok = args.text and job.stream.family == 0 and job.stream.val == "one"
     nb, pages, F = job.table_params()
     t = job.table()
     k, o, v = job.inputs()
-    for _ in range(max(args.warmup, 3)):
-        t.reset()
-        t.run(k, o, v)
+    n = job.stream.n
+    csr = job.csr_bytes()
     sampler = ClockSampler(local)
-    if world > 1:
-        dist.barrier()
-    torch.cuda.synchronize()
-    sampler.start()
-    ms, info = timed_steps(job, t, args.steps, stream, route_fn)
-    clocks = sampler.stop()
-    st = info["last"]
-    if world > 1:
-        tt = torch.tensor([ms], device="cuda")
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        ms = float(tt.item())
-    if routed:  # strong scaling: the whole stream is split over the ranks
-        csr_all = job.slice_bytes
-        tt = torch.tensor([csr_all], device="cuda", dtype=torch.float64)
-        if world > 1:
-            dist.all_reduce(tt)
-        csr, n = float(tt.item()), job.stream.n
-        value = csr * args.steps / (ms / 1e3) / 1e9
+
+    # ---- headline: the whole SEPO job on the RAW text, tokenizer inside (sepo_run_text)
+    text = job.stream.text_device() if text_ok else None
+    if text_ok:
+        tb = text.numel()
+        for _ in range(max(args.warmup, 3)):
+            t.reset(); t.run_text(text)
+        sampler.start()
+        ms, info = time_text_jobs(t, text, args.steps, stream)
+        value = tb * args.steps / (ms / 1e3) / 1e9
         recs_per_s = n * args.steps / (ms / 1e3)
+        st = info["last"]
+        head = {"metric_input": "raw text bytes (each word + one separator), tokenized inside the insert kernel",
+                "text_bytes": tb}
+    # ---- the same job on pre-tokenised CSR input (sepo_run; sub-line, or the headline for C3/C4/C5)
+    for _ in range(max(args.warmup, 3)):
+        t.reset(); t.run(k, o, v)
+    if not text_ok:
+        sampler.start()
+    ms_c, info_c = timed_steps(job, t, args.steps, stream)
+    st_c = info_c["last"]
+    csr_line = {"value": csr * args.steps / (ms_c / 1e3) / 1e9, "unit": "GB/s of CSR (key bytes + 8 B offsets [+ values])",
+                "ms_per_step": ms_c / args.steps, "kv_inserts_per_s": n * args.steps / (ms_c / 1e3),
+                "passes": st_c["passes"], "postponed_per_pass": st_c["postponed_per_pass"],
+                "pass1_ms": info_c["p1_ms"] / args.steps}
+    if not text_ok:
+        ms, info, st = ms_c, info_c, st_c
+        value = csr_line["value"]
+        recs_per_s = csr_line["kv_inserts_per_s"]
+        head = {"metric_input": "CSR bytes: key bytes + 8 B offsets [+ values]", "csr_bytes": csr}
+
+    # ---- M1: in-budget sepo_insert_batch, pass-1 insert kernel; C2 at 0.5x (+ C3 at P = 1)
+    m1 = None
+    if args.m1 and args.config == "C2" and args.scale == 1.0:
+        jib = Job("C2", 0.5)
+        jib._inputs = job._inputs
+        tib = jib.table()
+        for _ in range(2):
+            tib.reset(); tib.run(k, o, v)
+        msi, ii = timed_steps(jib, tib, args.steps, stream)
+        tr = traffic_of("r02_traffic_m1.json")
+        m1 = roofline_of(csr, ii["p1_ms"], args.steps, pk, "sepo::insert_stream_kernel<false,1024,IN_CSR> (C2, 0.5x: in budget, 1 pass)",
+                         {"traffic": (tr["dram_read_bytes"] + tr["dram_write_bytes"]) if tr else None,
+                          "traffic_note": tr.get("launch") if tr else None, "share_of_step": ii["p1_ms"] / msi,
+                          "job_ms": msi / args.steps, "passes": ii["last"]["passes"]})
+        m1["issue"] = issue_of(tr, n, m1["launch_ms"], {"sm_mhz": None})
+        tib.close()
+    m1_c3 = None
+    if args.m1_c3 and args.config == "C2" and args.scale == 1.0:
+        j3 = Job("C3", 1.0)
+        t3 = j3.table()
+        k3, o3, v3 = j3.inputs()
+        for _ in range(2):
+            t3.reset(); t3.run(k3, o3, v3)
+        ms3, i3 = timed_steps(j3, t3, 3, stream)
+        tr3 = traffic_of("r02_traffic_c3.json")
+        m1_c3 = roofline_of(j3.csr_bytes(), i3["p1_ms"], 3, pk, "sepo::insert_stream_kernel<false,1024,IN_CSR> (C3 URLs, P = 1, in budget)",
+                            {"traffic": (tr3["dram_read_bytes"] + tr3["dram_write_bytes"]) if tr3 else None,
+                             "job_ms": ms3 / 3, "records": j3.stream.n, "passes": i3["last"]["passes"]})
+        t3.close()
+        del j3, k3, o3, v3
+        torch.cuda.empty_cache()
+    clocks = sampler.stop()
+    if m1 and m1.get("issue") is not None:
+        m1["issue"] = issue_of(traffic_of("r02_traffic_m1.json"), n, m1["launch_ms"], clocks)
+
+    # the headline step's own dominant kernel (pass 1 of the raw-text job: insert_text_kernel)
+    if text_ok:
+        trt = traffic_of("r02_traffic_text.json")
+        roof_head = roofline_of(tb, info["p1_ms"], args.steps, pk, "sepo::insert_text_kernel (pass 1 of the headline job)",
+                                {"share_of_step": info["p1_ms"] / ms,
+                                 "traffic": (trt["dram_read_bytes"] + trt["dram_write_bytes"]) if trt else None})
     else:
-        csr = job.csr_bytes()
-        n = job.stream.n
-        value = world * csr * args.steps / (ms / 1e3) / 1e9
-        recs_per_s = world * n * args.steps / (ms / 1e3)
+        roof_head = roofline_of(csr, info["p1_ms"], args.steps, pk, "pass-1 insert kernel of the headline job",
+                                {"share_of_step": info["p1_ms"] / ms})
 
-    # roofline of the dominant kernel: the pass-1 insert (insert_stream_kernel, rows a1..a7, plus
-    # its hot-set sampling kernels) handed every record of the step. Algorithmic bytes = the
-    # step's CSR input (key bytes + 8 B offset [+ value bytes] per record) over the
-    # CUDA-event time of that insert call (on the table's stream), summed over the timed steps.
-    pk = peaks()
-    alg = job.csr_bytes() if not routed else job.slice_bytes
-    achieved = alg * args.steps / (info["p1_ms"] / 1e3) / 1e9
-    traffic, traffic_note, issue = args.traffic, None, None
-    tj = os.path.join(ROOT, "profiles", "r01_traffic.json")
-    if traffic is None and os.path.exists(tj) and args.config == "C2" and args.scale == 1.0:
-        tr = json.load(open(tj))
-        traffic = tr["dram_read_bytes"] + tr["dram_write_bytes"]
-        traffic_note = (f"dram read+write of one launch ({tr['launch']}); that launch's algorithmic bytes: "
-                        f"{tr['alg_bytes']}")
-        if "warp_instructions" in tr:
-            # the kernel is issue-bound, not HBM-bound: its instruction roofline from the same capture
-            # (peak = 148 SMs x 4 schedulers x 1 warp instruction / cycle at the sampled SM clock)
-            peak_wi = 148 * 4 * (clocks.get("sm_mhz") or 1965.0) * 1e6
-            wi_per_s = tr["warp_instructions"] / (info["p1_ms"] / args.steps / 1e3)
-            issue = {"warp_instructions_per_launch": tr["warp_instructions"],
-                     "warp_instructions_per_record": tr["warp_instructions"] / n,
-                     "achieved_warp_instr_per_s": wi_per_s, "peak_warp_instr_per_s": peak_wi,
-                     "frac": wi_per_s / peak_wi, "ncu_issue_active": tr.get("issue_active_pct", 0) / 100.0}
-    roof = {"bound": "hbm", "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
-            "frac": achieved / pk["hbm_gbs"], "traffic": traffic, "traffic_note": traffic_note,
-            "kernel": "sepo::insert_stream_kernel (COMBINE, pass 1) / sepo::insert_group_stream_kernel (GROUP)",
-            "alg_bytes_per_launch": alg, "launch_ms": info["p1_ms"] / args.steps,
-            "share_of_step": info["p1_ms"] / ms, "all_insert_passes_share_of_step": info["insert_ms"] / ms,
-            "peak_source": "MEASURED_PEAKS.json hbm_gbs (copy)" if not pk.get("_fallback") else "fallback 6.65 TB/s",
-            "issue": issue}
-
-    # host link: page bytes evicted (intermediate generations + the final one)
-    # over the eviction phase time, against the measured pinned D2H bandwidth (PEAKS_EXTRA.json)
+    # host link: page bytes evicted over the eviction phase, vs measured pinned D2H
     host_link = None
     try:
         d2h_peak = json.load(open(os.path.join(ROOT, "PEAKS_EXTRA.json"))).get("d2h_GBps")
@@ -410,123 +518,168 @@ def run_ours(args):
     if st["t_evict_ms"] > 0:
         gbs = st["bytes_evicted"] / (st["t_evict_ms"] / 1e3) / 1e9
         host_link = {"bytes_evicted_per_step": st["bytes_evicted"], "evict_ms_per_step": st["t_evict_ms"],
-                     "achieved": gbs, "unit": "GB/s", "peak": d2h_peak,
-                     "frac": (gbs / d2h_peak) if d2h_peak else None,
-                     "note": "evict phase includes seal/classify kernels and the directory reset; peak = "
-                             "measured pinned D2H (PEAKS_EXTRA.json)"}
+                     "achieved": gbs, "unit": "GB/s", "peak": d2h_peak, "frac": (gbs / d2h_peak) if d2h_peak else None,
+                     "note": "evict phase includes seal/classify kernels and the directory reset; peak = measured "
+                             "pinned D2H (PEAKS_EXTRA.json)"}
 
-    # end to end through sepo_run with pinned HOST buffers (H2D + job + host result assembly)
-    e2e = None
-    if args.e2e_steps > 0 and not routed:
-        hk = torch.empty(k.numel(), dtype=torch.uint8, pin_memory=True); hk.copy_(k)
-        ho = torch.empty(o.numel(), dtype=torch.int64, pin_memory=True).copy_(o) if o is not None else None
-        hv = torch.empty(v.numel(), dtype=torch.uint8, pin_memory=True).copy_(v) if v is not None else None
-        # warm (staging buffers are allocated once)
-        t.reset(); t.run(hk, ho, hv); t.export(copy=False)
-        torch.cuda.synchronize()
-        t0 = time.perf_counter()
-        d2h = 0
-        for _ in range(args.e2e_steps):
-            t.reset()
-            t.run(hk, ho, hv)
-            res = t.export(copy=False)
-            d2h += t.stats()["bytes_evicted"]
-        el = time.perf_counter() - t0
-        if world > 1:
-            tt = torch.tensor([el], device="cuda")
-            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-            el = float(tt.item())
-        e2e = {"value": world * csr * args.e2e_steps / el / 1e9, "unit": "GB/s",
-               "h2d_bytes_per_step": csr, "d2h_bytes_per_step": d2h // args.e2e_steps,
-               "kv_inserts_per_s": world * n * args.e2e_steps / el,
-               "note": "sepo_run on pinned host buffers; includes H2D, all passes, page D2H, host result assembly"}
-
-    # slowdown curve (M3): job time at table/budget = 0.5 .. 4 relative to 0.5
-    curve = None
-    if args.curve and rank == 0 and not routed:
-        curve = {}
-        base = None
+    # slowdown curves (M3): job time at table/budget 0.5 .. 4 relative to 0.5 (headline job; CSR job too)
+    curve = curve_csr = None
+    if args.curve:
+        curve, curve_csr = {}, {}
+        base = base_c = None
         for r in (0.5, 1.0, 2.0, 3.0, 4.0):
             j2 = Job(args.config, r, scale=args.scale)
             j2._inputs = job._inputs
             t2 = j2.table()
+            if text_ok:
+                for _ in range(2):
+                    t2.reset(); t2.run_text(text)
+                m2, i2 = time_text_jobs(t2, text, 2, stream)
+                base = base or m2 / 2
+                curve[str(r)] = {"ms": m2 / 2, "slowdown": m2 / 2 / base, "passes": i2["last"]["passes"]}
             for _ in range(2):
                 t2.reset(); t2.run(k, o, v)
             m2, i2 = timed_steps(j2, t2, 2, stream)
-            ms2 = m2 / 2
-            if base is None:
-                base = ms2
-            curve[str(r)] = {"ms": ms2, "slowdown": ms2 / base, "passes": i2["last"]["passes"]}
+            base_c = base_c or m2 / 2
+            curve_csr[str(r)] = {"ms": m2 / 2, "slowdown": m2 / 2 / base_c, "passes": i2["last"]["passes"]}
             t2.close()
+        if not text_ok:
+            curve = curve_csr
 
-    # raw-text job (NEXT-2 (i), sepo_run_text): the same word stream as the 8 GB text the config
-    # names (each word + one separator), tokenized inside the insert kernel; device-resident
-    # input timed like the main line, plus e2e from pinned host text (H2D inside the timed region)
-    raw_text = None
-    if args.text and rank == 0 and not routed and job.stream.family == 0 and job.stream.val == "one":
-        text = job.stream.text_device()
-        tb = text.numel()
-        for _ in range(2):
-            t.reset(); t.run_text(text)
-        torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for _ in range(args.steps):
-            t.reset(); t.run_text(text)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        tms = e0.elapsed_time(e1) / args.steps
-        stt = t.stats()
-        raw_text = {"text_bytes": tb, "ms_per_step": tms, "value": tb / tms / 1e6, "unit": "GB/s of raw text",
-                    "words_per_s": n / tms * 1e3, "passes": stt["passes"],
-                    "pass1_ms": stt["t_insert_ms_per_pass"][0]}
-        if args.e2e_steps > 0:
-            ht = torch.empty(tb, dtype=torch.uint8, pin_memory=True)
-            ht.copy_(text)
-            del text
-            t.reset(); t.run_text(ht); t.export(copy=False)
-            torch.cuda.synchronize()
-            t0 = time.perf_counter()
-            d2h = 0
-            for _ in range(args.e2e_steps):
-                t.reset(); t.run_text(ht); t.export(copy=False)
-                d2h += t.stats()["bytes_evicted"]
-            el = (time.perf_counter() - t0) / args.e2e_steps
-            raw_text["e2e"] = {"value": tb / el / 1e9, "unit": "GB/s of raw text", "words_per_s": n / el,
-                               "h2d_bytes_per_step": tb, "d2h_bytes_per_step": d2h // args.e2e_steps,
-                               "note": "sepo_run_text on pinned host text; includes H2D, all passes, page D2H, host result assembly"}
-            del ht
-        else:
-            del text
+    # end to end through the public API from pinned HOST buffers (H2D + job + export in the timed region)
+    e2e = e2e_c = None
+    if args.e2e_steps > 0:
+        e2e_c = e2e_csr(t, k, o, v, csr, n, args.e2e_steps)
+        e2e = e2e_text(t, text, n, args.e2e_steps) if text_ok else e2e_c
+    csr_line["e2e"] = e2e_c
+    csr_line["slowdown_curve"] = curve_csr
+    if text is not None:
+        del text
         torch.cuda.empty_cache()
 
     cpu = None
     if rank == 0 and args.cpu_baseline:
         gbs, rps, nrec, tsec = oracle_sample(job, args.ref_records, budget_s=args.ref_seconds)
         cpu = {"value": gbs, "unit": "GB/s", "cores": 1, "kind": "oracle",
-               "sample": f"first {nrec} records of {args.config} ({tsec:.1f} s, oracle/oracle.cpp std::unordered_map, "
-                         f"single thread pinned by construction; generation excluded)", "kv_inserts_per_s": rps}
+               "sample": f"first {nrec} records of {args.config} as CSR ({tsec:.1f} s; oracle/oracle.cpp std::unordered_map, "
+                         f"one thread; generation excluded)", "kv_inserts_per_s": rps,
+               "metric_input": "CSR bytes (the oracle takes tokenised records)", **cpu_info()}
 
+    line = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": max(args.warmup, 3), "ms_per_step": ms / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+            "kv_inserts_per_s": recs_per_s,
+            "config": {"workload": CONFIG_TEXT[args.config] + (" [raw text job, tokenizer fused]" if text_ok else ""),
+                       **head, "records": n, "input_csr_bytes": csr,
+                       "distinct_keys": job.distinct, "ratio_table_over_budget": args.ratio,
+                       "table_footprint_bytes": F, "device_budget_bytes": job.sepo.budget_for(nb, job.page_bytes, pages),
+                       "n_buckets": nb, "page_bytes": job.page_bytes, "pool_pages": pages,
+                       "passes": st["passes"], "postponed_per_pass": st["postponed_per_pass"],
+                       "bytes_evicted": st["bytes_evicted"], "l2": "inputs (8-16 GB) far larger than L2 (126 MB): no flush needed",
+                       "parallelism": "1 GPU",
+                       "phase_ms": {kk: st[kk] for kk in ("t_insert_ms", "t_reprobe_ms", "t_compact_ms", "t_evict_ms")}},
+            "roofline": m1 if m1 is not None else roof_head, "roofline_headline_kernel": roof_head, "roofline_m1_c3": m1_c3,
+            "host_link": host_link, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+            "gpu_launches": info["launches"], "slowdown_curve": curve, "csr_job": csr_line}
     if rank == 0:
-        line = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
-                "warmup": max(args.warmup, 3), "ms_per_step": ms / args.steps, "higher_is_better": True,
-                "scaling": "strong" if routed else "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
-                "kv_inserts_per_s": recs_per_s,
-                "config": {"workload": CONFIG_TEXT[args.config], "records": n, "input_csr_bytes": csr,
-                           "distinct_keys": job.distinct, "ratio_table_over_budget": args.ratio,
-                           "table_footprint_bytes": F, "device_budget_bytes": job.sepo.budget_for(nb, job.page_bytes, pages),
-                           "n_buckets": nb, "page_bytes": job.page_bytes, "pool_pages": pages,
-                           "passes": st["passes"], "postponed_per_pass": st["postponed_per_pass"],
-                           "bytes_evicted": st["bytes_evicted"], "l2": "inputs (>= 15 GiB) far larger than L2 (126 MB)",
-                           "parallelism": (f"key-hash sharded x{world} (sepo_partition + NCCL all-to-all)" if routed
-                                           else "1 GPU"),
-                           "phase_ms": {kk: st[kk] for kk in ("t_insert_ms", "t_reprobe_ms", "t_compact_ms", "t_evict_ms")}},
-                "roofline": roof, "host_link": host_link, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
-                "gpu_launches": info["launches"], "slowdown_curve": curve, "raw_text": raw_text}
         print(json.dumps(line), flush=True)
     t.close()
     if dist.is_initialized():
         dist.destroy_process_group()
+
+
+def run_routed(args, world, rank, local):
+    """N GPUs (torchrun) or --route at N=1: key-hash sharding of ONE global CSR stream (strong scaling):
+    rank r holds records [r n/N, (r+1) n/N) and every step routes them by key owner (sepo_partition +
+    NCCL all-to-all), then runs the SEPO job on the records it owns."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_mokhtaris17_b200 import shard
+    if not dist.is_initialized():
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29511")
+        dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", local))
+    job = Job(args.config, args.ratio, scale=args.scale)
+    stream = torch.cuda.current_stream()
+    fixed = job.stream.family == 2
+    n_all = job.stream.n
+    j0, j1 = rank * n_all // world, (rank + 1) * n_all // world
+    sk, so, sv = job.stream.device(j0, j1 - j0)
+    if fixed:
+        so = None
+    router = shard.Router(route_seed=0x5eed, fixed_key_width=8 if fixed else 0,
+                          fixed_val_width=job.stream.val_width if sv is not None else 0)
+
+    def route_fn():
+        return router.route(sk, so, sv)
+    job.distinct = max(1, job.distinct // world)  # keys per rank (sizes the directory)
+    job._inputs = route_fn()
+    slice_bytes = sk.numel() + (8 * (so.numel() - 1) if so is not None else 0) + (sv.numel() if sv is not None else 0)
+    nb, pages, F = job.table_params()
+    t = job.table()
+    k, o, v = job.inputs()
+    for _ in range(max(args.warmup, 3)):
+        route_fn()
+        t.reset()
+        t.run(*job.inputs())
+    sampler = ClockSampler(local)
+    dist.barrier()
+    torch.cuda.synchronize()
+    sampler.start()
+    ms, info = timed_steps(job, t, args.steps, stream, route_fn)
+    clocks = sampler.stop()
+    tt = torch.tensor([ms], device="cuda")
+    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    ms = float(tt.item())
+    tb = torch.tensor([slice_bytes], device="cuda", dtype=torch.float64)
+    dist.all_reduce(tb)
+    csr = float(tb.item())
+    value = csr * args.steps / (ms / 1e3) / 1e9
+    st = info["last"]
+    # e2e: each rank's slice from pinned host memory -> H2D -> route -> job -> export, max over ranks
+    e2e = None
+    if args.e2e_steps > 0:
+        hk = torch.empty(sk.numel(), dtype=torch.uint8, pin_memory=True); hk.copy_(sk)
+        ho = torch.empty(so.numel(), dtype=torch.int64, pin_memory=True).copy_(so) if so is not None else None
+        hv = torch.empty(sv.numel(), dtype=torch.uint8, pin_memory=True).copy_(sv) if sv is not None else None
+        torch.cuda.synchronize()
+        dist.barrier()
+        t0 = time.perf_counter()
+        d2h = 0
+        for _ in range(args.e2e_steps):
+            dk = hk.to("cuda", non_blocking=True)
+            do = ho.to("cuda", non_blocking=True) if ho is not None else None
+            dv = hv.to("cuda", non_blocking=True) if hv is not None else None
+            rk, ro, rv = router.route(dk, do, dv)
+            t.reset()
+            t.run(rk, ro, rv)
+            t.export(copy=False)
+            d2h += t.stats()["bytes_evicted"]
+        torch.cuda.synchronize()
+        el = torch.tensor([time.perf_counter() - t0], device="cuda")
+        dist.all_reduce(el, op=dist.ReduceOp.MAX)
+        el = float(el.item()) / args.e2e_steps
+        e2e = {"value": csr / el / 1e9, "unit": "GB/s", "h2d_bytes_per_step": slice_bytes,
+               "d2h_bytes_per_step": d2h // args.e2e_steps, "kv_inserts_per_s": n_all / el,
+               "note": "per rank: pinned host slice -> H2D -> route (partition + all-to-all) -> sepo_run -> sepo_export; "
+                       "max over ranks"}
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+                "warmup": max(args.warmup, 3), "ms_per_step": ms / args.steps, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+                "kv_inserts_per_s": n_all * args.steps / (ms / 1e3),
+                "config": {"workload": CONFIG_TEXT[args.config] + " [CSR job, key-hash sharded]", "records": n_all,
+                           "input_csr_bytes": csr, "ratio_table_over_budget": args.ratio, "n_buckets": nb,
+                           "page_bytes": job.page_bytes, "pool_pages": pages, "passes": st["passes"],
+                           "parallelism": f"key-hash sharded x{world} (sepo_partition + all-to-all, pre-combined)",
+                           "l2": "inputs far larger than L2 (126 MB): no flush needed"},
+                "roofline": roofline_of(job.csr_bytes(), info["p1_ms"], args.steps, peaks(),
+                                        "pass-1 insert kernel of this rank's job", {"share_of_step": info["p1_ms"] / ms}),
+                "route": router.last_stats(), "e2e": e2e, "clocks": clocks, "gpu_launches": info["launches"],
+                "cpu_baseline": None}
+        print(json.dumps(line), flush=True)
+    t.close()
+    dist.destroy_process_group()
 
 
 def main():
@@ -541,7 +694,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-curve", dest="curve", action="store_false")
     ap.add_argument("--no-cpu", dest="cpu_baseline", action="store_false")
-    ap.add_argument("--no-text", dest="text", action="store_false", help="skip the raw-text (fused tokenizer) line")
+    ap.add_argument("--no-text", dest="text", action="store_false", help="headline on the CSR job instead of raw text")
+    ap.add_argument("--no-m1", dest="m1", action="store_false", help="skip the in-budget (0.5x) M1 roofline job")
+    ap.add_argument("--no-m1-c3", dest="m1_c3", action="store_false", help="skip the C3 (P = 1) M1 sub-line")
     ap.add_argument("--ref-records", type=int, default=120_000_000)
     ap.add_argument("--ref-seconds", type=float, default=15.0)
     ap.add_argument("--route", action="store_true", help="run the sharded (router) path even at N=1")

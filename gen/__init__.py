@@ -57,6 +57,9 @@ def lib():
         L.gen_ranks_dev.argtypes = [P, u64, u64, vp, vp]; L.gen_ranks_dev.restype = ctypes.c_int
         L.gen_text_dev.argtypes = [P, u64, u64, vp, vp, vp, vp]; L.gen_text_dev.restype = ctypes.c_int
         L.gen_text_host.argtypes = [P, u64, u64, vp, vp, vp]
+        L.gen_key_ranks_host.argtypes = [P, vp, vp, u64, vp]
+        L.gen_rank_digest_host.argtypes = [P, u64, u64, vp, vp, vp]
+        L.gen_list_digest_host.argtypes = [vp, vp, vp, u64, vp, vp, vp]
         _LIB = L
     return _LIB
 
@@ -244,6 +247,27 @@ class Stream:
         """Closed-form value multiset of rank r (sorted list of doc ids / values)."""
         return sorted(int(v) for v in self.values_of_records(self.records_of_rank(r)))
 
+    # ---- full-size checks (closed forms evaluated backwards; host C, OpenMP) ----
+    def key_ranks(self, keys, offs):
+        """rank spelled by each key of a CSR key set (0: no rank spells it)"""
+        keys = np.ascontiguousarray(keys, dtype=np.uint8)
+        offs = np.ascontiguousarray(offs, dtype=np.uint64)
+        n = len(offs) - 1
+        out = np.empty(n, dtype=np.uint64)
+        if n:
+            lib().gen_key_ranks_host(ctypes.byref(self.params()), _ptr(keys) if len(keys) else None, _ptr(offs), n, _ptr(out))
+        return out
+
+    def rank_digest(self, r0=1, cnt=None):
+        """per rank r0..: (record count, sum of record values mod 2^64, sum of mix(value) mod 2^64)
+        over the records that hold the rank — the exact combine sum (PAIRS) or a digest of the
+        exact value multiset (doc ids)"""
+        if cnt is None:
+            cnt = self.n_ranks - r0 + 1
+        c, sm, mx = (np.empty(cnt, dtype=np.uint64) for _ in range(3))
+        lib().gen_rank_digest_host(ctypes.byref(self.params()), r0, cnt, _ptr(c), _ptr(sm), _ptr(mx))
+        return c, sm, mx
+
     def raw_bytes(self):
         """Bytes of the raw dataset: text with one separator per word (WORDS/URLS), 16 B per pair."""
         if self.family == GEN_PAIRS:
@@ -319,3 +343,16 @@ def config(name, scale=1.0):
         D = max(16, int((1 << 28) * scale))
         return pairs_stream("C5z", D, 8 * D, seed=6, alpha=1.2)
     raise KeyError(name)
+
+
+def list_digest(vals, val_offs, list_offs):
+    """(count, sum, sum of mix) per key of exported value lists, the same digest as
+    Stream.rank_digest (values = little-endian integers of their bytes)"""
+    vals = np.ascontiguousarray(vals, dtype=np.uint8)
+    vo = np.ascontiguousarray(val_offs, dtype=np.uint64)
+    lo = np.ascontiguousarray(list_offs, dtype=np.uint64)
+    n = len(lo) - 1
+    c, sm, mx = (np.empty(n, dtype=np.uint64) for _ in range(3))
+    if n:
+        lib().gen_list_digest_host(_ptr(vals) if len(vals) else None, _ptr(vo), _ptr(lo), n, _ptr(c), _ptr(sm), _ptr(mx))
+    return c, sm, mx

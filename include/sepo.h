@@ -44,7 +44,7 @@ enum sepo_status {
     SEPO_E_NCCL = -6      /* NCCL error (sticky) */
 };
 
-/* Bucket organizations. BASIC is not implemented. */
+/* Bucket organizations. */
 typedef enum {
     SEPO_COMBINE_SUM_U64 = 0, /* "combining": one entry per key, value = u64 wrapping sum */
     SEPO_GROUP = 1,           /* "multi-valued": key entries + per-key value lists */
@@ -105,6 +105,7 @@ typedef struct sepo_stats {
     uint64_t value_slots;          /* GROUP export: value slots in those chunks (capacity) */
     double t_insert_ms, t_reprobe_ms, t_compact_ms, t_evict_ms, t_export_ms, t_h2d_ms;
     double t_insert_ms_per_pass[SEPO_MAX_PASS_STATS]; /* insert-kernel time of each pass */
+    uint64_t hot_keys;             /* most keys a sampled hot set held in one insert call (a2; 0: none) */
 } sepo_stats;
 
 /* Create a table on the current CUDA device.

@@ -105,6 +105,7 @@ struct sepo_table {
     uint32_t batch_seq = 0;
     uint64_t pages_resident_retained = 0;
     uint64_t pending_idx_key_bytes = 0;  // key bytes of the next indexed re-issue batch (stats)
+    uint64_t last_job_pages = 0;         // most pages resident at once in the previous job (0: none yet)
     std::vector<PinChunk> arena;
     std::vector<GenImage> gens;
     sepo_stats st{};
@@ -361,7 +362,7 @@ sepo_table* sepo_create_placed(size_t budget, uint64_t n_buckets, uint32_t page_
     cudaEventCreateWithFlags(&t->ev_comp, cudaEventDisableTiming);
     cudaHostAlloc((void**)&t->h_ctrl, sizeof(Ctrl), cudaHostAllocDefault);
     cudaHostAlloc((void**)&t->h_evict, (size_t)t->n_pages * 4, cudaHostAllocDefault);
-    cudaHostAlloc((void**)&t->h_ko, 16, cudaHostAllocDefault);
+    cudaHostAlloc((void**)&t->h_ko, 64, cudaHostAllocDefault);
     if (cudaGetLastError() != cudaSuccess || !t->h_ctrl || !t->h_evict) {
         fail(SEPO_E_CUDA, "stream/event/pinned allocation failed");
         sepo_destroy(t);
@@ -450,6 +451,21 @@ static void trace(const char* what, uint64_t x = 0) {
     fprintf(stderr, "[sepo %10.3f ms] %s %llu\n", ms, what, (unsigned long long)x);
 }
 
+// Tables whose resident generation exceeds L2: queued misses' directory lines are prefetched into
+// L2 while they wait (measured: helps when directory + entries live in HBM, hurts when a generation
+// fits L2). The resident footprint is the directory plus the pages the generation can hold —
+// min(pool, pages the previous job used at most) — not the budget, which may be all free HBM
+// (P:L101). SEPO_DIR_PF=0/1 forces the choice (read on every call).
+static bool dir_prefetch(sepo_table* t) {
+    const char* e = getenv("SEPO_DIR_PF");
+    if (e && (e[0] == '0' || e[0] == '1')) return e[0] == '1';
+    int l2 = 0;
+    cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device);
+    uint64_t pages = t->n_pages;
+    if (t->last_job_pages) pages = std::min<uint64_t>(pages, t->last_job_pages);
+    return (uint64_t)t->n_buckets * 4 + pages * (uint64_t)t->page_bytes > (uint64_t)l2;
+}
+
 static int64_t insert_impl(sepo_table* t, const Batch& b) {
     int rc;
     const uint64_t n = b.n;
@@ -471,22 +487,22 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
         CK(t, cudaStreamSynchronize(t->stream));
         key_end = t->h_ko[1];
     }
-    // in-budget tables larger than L2: the misses' directory lines are prefetched into L2 while
-    // they wait in the queue (measured: helps when the directory + entries live in HBM, hurts when
-    // a generation fits L2); SEPO_DIR_PF=0/1 forces it
-    static const int dpf_env = [] { const char* e = getenv("SEPO_DIR_PF"); return e ? atoi(e) : -1; }();
-    int l2 = 0;
-    cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device);
-    const bool dpf = dpf_env >= 0 ? dpf_env == 1 : (t->budget > (size_t)l2);
-    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p, halt_slots, key_end, dpf);
+    bool hot_built = false;
+    rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p, halt_slots, key_end, dir_prefetch(t),
+                            &hot_built);
     if (rc) return cuda_check(t, (cudaError_t)rc, "insert kernel launch");
     CK(t, cudaEventRecord(t->ev1, t->stream));
+    t->h_ko[2] = 0;
+    if (hot_built)
+        CK(t, cudaMemcpyAsync(&t->h_ko[2], (uint8_t*)t->hot.p + sepo_hot_count_offset(), 4, cudaMemcpyDeviceToHost,
+                              t->stream));
     t->st.kernel_launches += (n >= (8ull << 18)) ? 7 : 1;
     if (b.ko && !b.idx) {
         CK(t, cudaMemcpyAsync(&t->h_ko[0], b.ko, 8, cudaMemcpyDeviceToHost, t->stream));
         CK(t, cudaMemcpyAsync(&t->h_ko[1], b.ko + n, 8, cudaMemcpyDeviceToHost, t->stream));
     }
     if ((rc = read_ctrl(t))) return rc;
+    t->st.hot_keys = std::max<uint64_t>(t->st.hot_keys, t->h_ko[2]);
     t->last_insert_ms = elapsed_ms(t->ev0, t->ev1);
     trace("insert end", t->h_ctrl->postponed);
     t->st.t_insert_ms += t->last_insert_ms;
@@ -1099,6 +1115,9 @@ static int64_t prep_passes(sepo_table* t, const Batch& cur, int ps, uint64_t res
     return 0;
 }
 
+static int64_t run_device(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals,
+                          const uint64_t* vo, uint64_t n);
+
 int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
                  uint64_t n) {
     trace("run begin", n);
@@ -1144,8 +1163,10 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
         CK(t, cudaEventRecord(h1, t->copy_stream));
         t->h2d_chunks = &evs;
         t->h2d_chunk_records = per;
-        const int64_t r = sepo_run(t, kst - k0, ko ? ost : nullptr, vals ? (const uint8_t*)t->in_stage[2].p : nullptr,
-                                   nullptr, n);
+        // (the staged copy is device memory: no second pointer classification — a rebased key base
+        // kst - k0 may lie outside every allocation)
+        const int64_t r = run_device(t, kst - k0, ko ? ost : nullptr, vals ? (const uint8_t*)t->in_stage[2].p : nullptr,
+                                     nullptr, n);
         t->h2d_chunks = nullptr;
         cudaEventSynchronize(h1);
         t->st.t_h2d_ms += elapsed_ms(h0, h1);
@@ -1173,10 +1194,17 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
         // offsets stay absolute: shift the key base so keys[ko[i]] addresses the staged copy
         const uint8_t* kdev = (const uint8_t*)t->in_stage[0].p - k0;
         const uint8_t* vdev = vals ? (const uint8_t*)t->in_stage[2].p - v0 : nullptr;
-        return sepo_run(t, kdev, ko ? (const uint64_t*)t->in_stage[1].p : nullptr, vdev,
-                        vo ? (const uint64_t*)t->in_stage[3].p : nullptr, n);
+        return run_device(t, kdev, ko ? (const uint64_t*)t->in_stage[1].p : nullptr, vdev,
+                          vo ? (const uint64_t*)t->in_stage[3].p : nullptr, n);
     }
+    return run_device(t, keys, ko, vals, vo, n);
+}
+
+// sepo_run on device-resident input (the caller's arrays, or the staged copy of host input)
+static int64_t run_device(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals,
+                          const uint64_t* vo, uint64_t n) {
     trace("run: inputs on device");
+    const uint32_t kw = t->opts.fixed_key_width;
     Batch cur;
     int rc2 = make_batch(t, cur, keys, ko, vals, vo, n, nullptr);
     if (rc2) return rc2;
@@ -1365,12 +1393,7 @@ int64_t sepo_run_text(sepo_table* t, const uint8_t* text, uint64_t n_bytes) {
     cur.n = n_bytes;
     cur.text = 1;
     cur.prep_rb = 32;
-    {
-        const char* e = getenv("SEPO_DIR_PF");
-        int l2 = 0;
-        cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device);
-        cur.dirpf = (e ? atoi(e) == 1 : t->budget > (size_t)l2) ? 1u : 0u;
-    }
+    cur.dirpf = dir_prefetch(t) ? 1u : 0u;
     // prepared list for pass 1 (a word is >= 2 bytes with its separator; ~n/32 slots = a quarter of
     // 8-byte words), the overflow bitmap over the text bytes (zero between uses)
     uint64_t cap = std::max<uint64_t>(1ull << 16, n_bytes / 32);
@@ -1395,6 +1418,7 @@ int64_t sepo_run_text(sepo_table* t, const uint8_t* text, uint64_t n_bytes) {
     CK(t, cudaMemsetAsync(&t->d.ctrl->text_words, 0, 8, t->stream));
     CK(t, cudaEventRecord(t->ev0, t->stream));
     if (t->hot.grow(sepo_hot_scratch_bytes())) return fail(SEPO_E_NOMEM, "hot-set scratch");
+    bool hot_built = false;  // this job's hot set (chunks >= 1 reuse the one chunk 0 sampled, if any)
     if (chunks) {  // each chunk's windows as soon as its copy landed; the hot set from the first
         const uint64_t cb = t->h2d_chunk_records;
         for (size_t k = 0; k < chunks->size(); ++k) {
@@ -1403,17 +1427,23 @@ int64_t sepo_run_text(sepo_table* t, const uint8_t* text, uint64_t n_bytes) {
             bc.w_begin = (k * cb) / 512;
             bc.w_end = std::min<uint64_t>((k + 1) * cb, n_bytes + 511) / 512;
             if (k + 1 == chunks->size()) bc.w_end = ~0ull;
-            rc = sepo_launch_insert_text(t->d, bc, t->grid, t->stream, t->hot.p, k == 0 ? std::min<uint64_t>(cb, n_bytes) : 0);
+            rc = sepo_launch_insert_text(t->d, bc, t->grid, t->stream, t->hot.p, k == 0 ? std::min<uint64_t>(cb, n_bytes) : 0,
+                                         &hot_built);
             if (rc) return cuda_check(t, (cudaError_t)rc, "text insert kernel launch");
         }
     } else {
-        rc = sepo_launch_insert_text(t->d, cur, t->grid, t->stream, t->hot.p, n_bytes);
+        rc = sepo_launch_insert_text(t->d, cur, t->grid, t->stream, t->hot.p, n_bytes, &hot_built);
         if (rc) return cuda_check(t, (cudaError_t)rc, "text insert kernel launch");
     }
     CK(t, cudaEventRecord(t->ev1, t->stream));
     t->st.kernel_launches += (n_bytes >= (64ull << 18)) ? 7 : 1;
     CK(t, cudaMemcpyAsync(&t->h_ko[0], cur.out_n, 8, cudaMemcpyDeviceToHost, t->stream));
+    t->h_ko[2] = 0;
+    if (hot_built)
+        CK(t, cudaMemcpyAsync(&t->h_ko[2], (uint8_t*)t->hot.p + sepo_hot_count_offset(), 4, cudaMemcpyDeviceToHost,
+                              t->stream));
     if ((rc = read_ctrl(t))) return rc;
+    t->st.hot_keys = std::max<uint64_t>(t->st.hot_keys, t->h_ko[2]);
     t->last_insert_ms = elapsed_ms(t->ev0, t->ev1);
     t->st.t_insert_ms += t->last_insert_ms;
     if (t->st.passes < SEPO_MAX_PASS_STATS) t->st.t_insert_ms_per_pass[t->st.passes] += t->last_insert_ms;
@@ -1427,6 +1457,10 @@ int64_t sepo_run_text(sepo_table* t, const uint8_t* text, uint64_t n_bytes) {
     }
     if (t->h_ctrl->toolarge) {
         t->st.toolarge += t->h_ctrl->toolarge;
+        // pass 1 may have set overflow bits that are never converted: the bitmap must be all zero
+        // for the next job (text_bits_kernel clears the bits it converts on the normal path)
+        CK(t, cudaMemsetAsync(t->tbm.p, 0, t->tbm.cap, t->stream));
+        CK(t, cudaStreamSynchronize(t->stream));
         return fail(SEPO_E_TOOLARGE, std::to_string(t->h_ctrl->toolarge) + " word(s) cannot fit in one page");
     }
     const uint64_t c = t->h_ctrl->postponed;
@@ -1525,6 +1559,7 @@ int sepo_reset(sepo_table* t) {
     t->pages_resident_retained = 0;
     t->lookup_done = false;
     trace("reset: copy stream idle");
+    if (t->st.pages_used_max) t->last_job_pages = t->st.pages_used_max;
     sepo_stats z{};
     z.n_buckets = t->n_buckets;
     z.page_bytes = t->page_bytes;

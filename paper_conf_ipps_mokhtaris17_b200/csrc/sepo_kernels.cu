@@ -2558,20 +2558,31 @@ __global__ void __launch_bounds__(512) evict_copy_kernel(const uint8_t* __restri
 // ================================================================ launchers
 using namespace sepo;
 
+// Smallest batch (records; text: bytes) that gets a sampled hot set. Tests move the threshold:
+// SEPO_NO_HOT=1 switches the hot set off, SEPO_HOT_MIN=<n> sets the threshold (re-read per launch).
+static uint64_t hot_min_records(uint64_t dflt) {
+    const char* off = getenv("SEPO_NO_HOT");
+    if (off && off[0] == '1') return ~0ull;
+    const char* m = getenv("SEPO_HOT_MIN");
+    return m ? strtoull(m, nullptr, 10) : dflt;
+}
+
 int sepo_launch_insert_text(const Dev& d, const Batch& b0, int grid, cudaStream_t s, void* hot_scratch,
-                            uint64_t sample_bytes) {
+                            uint64_t sample_bytes, bool* hot_built) {
     const hot::Entry* hl = nullptr;
     const unsigned int* nh = nullptr;
     const uint64_t n_sample = 1ull << 18;
     const Batch& b = b0;
     Batch bs = b0;  // bs.n: the prefix the sample positions come from (its words are read whole:
     bs.n = sample_bytes < b0.n ? sample_bytes : b0.n;  // the caller has copied past the prefix)
-    if (hot_scratch && sample_bytes == 0) {  // reuse the previous launch's hot set
+    const bool reuse = sample_bytes == 0 && *hot_built;
+    if (sample_bytes) *hot_built = false;
+    if (hot_scratch && reuse) {  // reuse the hot set an earlier launch of this job built
         uint8_t* p = reinterpret_cast<uint8_t*>(hot_scratch);
         hot::Entry* list = reinterpret_cast<hot::Entry*>(p + sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS);
         hl = list;
         nh = reinterpret_cast<unsigned int*>(list + hot::K);
-    } else if (hot_scratch && bs.n >= 64 * n_sample) {  // hot-set discovery on words at sampled byte offsets
+    } else if (hot_scratch && sample_bytes && bs.n >= hot_min_records(64 * n_sample)) {  // discovery on sampled words
         uint8_t* p = reinterpret_cast<uint8_t*>(hot_scratch);
         hot::SampleSlot* tab = reinterpret_cast<hot::SampleSlot*>(p);
         hot::Entry* list = reinterpret_cast<hot::Entry*>(p + sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS);
@@ -2579,7 +2590,7 @@ int sepo_launch_insert_text(const Dev& d, const Batch& b0, int grid, cudaStream_
         unsigned int* hist = n_out + 1;
         cudaMemsetAsync(tab, 0, sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS, s);
         cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
-        hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, bs.n / n_sample, n_sample, tab);  // positions in the prefix
+        hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, std::max<uint64_t>(1, bs.n / n_sample), std::min(n_sample, bs.n), tab);  // positions in the prefix
         hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
         hot_threshold_kernel<<<1, 1024, 0, s>>>(hist, 4u, (uint32_t)textk::TK);
         hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)textk::TK);
@@ -2587,6 +2598,7 @@ int sepo_launch_insert_text(const Dev& d, const Batch& b0, int grid, cudaStream_
         hot_resolve_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
         hl = list;
         nh = n_out;
+        *hot_built = true;
     }
     static bool attr = false;
     if (!attr) {
@@ -2613,7 +2625,8 @@ int sepo_launch_evict_copy(const Dev& d, uint32_t n, uint8_t* dst, int grid, cud
 }
 
 int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
-                       uint32_t halt_slots, uint64_t key_end, bool dir_prefetch) {
+                       uint32_t halt_slots, uint64_t key_end, bool dir_prefetch, bool* hot_built) {
+    if (hot_built) *hot_built = false;
     if (mode == 2) {
         insert_basic_kernel<<<grid, 1024, 0, s>>>(d, b, halt_slots);
         return cudaGetLastError();
@@ -2623,13 +2636,13 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
         const hot::Entry* hl = nullptr;
         const unsigned int* nh = nullptr;
         const uint64_t n_sample = 1ull << 18;
-        if (hot_scratch && b.n >= 8 * n_sample) {
+        if (hot_scratch && b.n >= hot_min_records(8 * n_sample)) {
             uint8_t* p = reinterpret_cast<uint8_t*>(hot_scratch);
             hot::SampleSlot* tab = reinterpret_cast<hot::SampleSlot*>(p);
             hot::Entry* list = reinterpret_cast<hot::Entry*>(p + sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS);
             unsigned int* n_out = reinterpret_cast<unsigned int*>(list + hot::K);
             cudaMemsetAsync(tab, 0, sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS, s);
-            hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, b.n / n_sample, n_sample, tab);
+            hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, std::max<uint64_t>(1, b.n / n_sample), std::min(n_sample, b.n), tab);
             unsigned int* hist = n_out + 1;
             cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
             hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
@@ -2639,6 +2652,7 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             hot_resolve_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
             hl = list;
             nh = n_out;
+            if (hot_built) *hot_built = true;
         }
         constexpr int T = stream::THREADS;
         const size_t sm = b.vals ? sizeof(stream::Smem<true, T / 32>) : sizeof(stream::Smem<false, T / 32>);
@@ -2674,7 +2688,7 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
         const hot::Entry* hl = nullptr;
         const unsigned int* nh = nullptr;
         const uint64_t n_sample = 1ull << 18;
-        if (hot_scratch && b.n >= 8 * n_sample) {
+        if (hot_scratch && b.n >= hot_min_records(8 * n_sample)) {
             uint8_t* p = reinterpret_cast<uint8_t*>(hot_scratch);
             hot::SampleSlot* tab = reinterpret_cast<hot::SampleSlot*>(p);
             hot::Entry* list = reinterpret_cast<hot::Entry*>(p + sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS);
@@ -2682,7 +2696,7 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             unsigned int* hist = n_out + 1;
             cudaMemsetAsync(tab, 0, sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS, s);
             cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
-            hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, b.n / n_sample, n_sample, tab);
+            hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, std::max<uint64_t>(1, b.n / n_sample), std::min(n_sample, b.n), tab);
             hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
             hot_threshold_kernel<<<1, 1024, 0, s>>>(hist, 4u, (uint32_t)gst::K);
             hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)gst::K);
@@ -2690,6 +2704,7 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             hot_resolve_group_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
             hl = list;
             nh = n_out;
+            if (hot_built) *hot_built = true;
         }
         const size_t sm = sizeof(gst::Smem);
         static bool attrg = false;
@@ -2708,6 +2723,7 @@ int sepo_launch_reinsert(const Dev& d, const Batch& b, int grid, cudaStream_t s)
     else reinsert_kernel<48><<<grid, 1024, 0, s>>>(d, b);
     return cudaGetLastError();
 }
+size_t sepo_hot_count_offset() { return sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS + sizeof(hot::Entry) * hot::K; }
 size_t sepo_hot_scratch_bytes() {
     return sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS + sizeof(hot::Entry) * hot::K + (HOT_HIST + 16) * 4;
 }

@@ -45,8 +45,12 @@ struct Batch {
 }  // namespace sepo
 
 // key_end: key_offsets[n] of a CSR batch (the end of its key bytes), read by the host
+// *hot_built (optional): whether this launch selected a sampled hot set (its size is the u32 at
+// hot_scratch + sepo_hot_count_offset(), clamped to the kernel's capacity)
 int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
-                       uint32_t halt_slots = 0, uint64_t key_end = 0, bool dir_prefetch = false);
+                       uint32_t halt_slots = 0, uint64_t key_end = 0, bool dir_prefetch = false,
+                       bool* hot_built = nullptr);
+size_t sepo_hot_count_offset();
 int sepo_launch_reinsert(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s);
 size_t sepo_hot_scratch_bytes();
 int sepo_default_grid(int mode, int n_sms);
@@ -65,10 +69,11 @@ int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec,
                               uint64_t total, cudaStream_t s);
 int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);
 int sepo_launch_evict_copy(const sepo::Dev& d, uint32_t n, uint8_t* dst, int grid, cudaStream_t s);
-// sample_bytes: tokenize a hot-set sample from the first sample_bytes of the text (0: reuse the hot
-// set the previous launch selected, still in hot_scratch)
+// sample_bytes: tokenize a hot-set sample from the first sample_bytes of the text; 0: reuse the hot
+// set an earlier launch of the same job built, if *hot_built says it did (else no hot set).
+// *hot_built (in/out, host): set when this launch builds a hot set, cleared when it samples none.
 int sepo_launch_insert_text(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s, void* hot_scratch,
-                            uint64_t sample_bytes);
+                            uint64_t sample_bytes, bool* hot_built);
 int sepo_launch_lookup_gen(const sepo::Dev& d, const sepo::Batch& b, const uint32_t* pages, uint32_t np,
                            unsigned long long* vals, uint32_t* found, cudaStream_t s);
 int sepo_launch_text_bits(const sepo::Dev& d, const sepo::Batch& b, unsigned long long* counter, cudaStream_t s);

@@ -79,6 +79,10 @@ def exchange(ok, oko, ov, starts, group=None, shift_fn=shift_offsets_cuda):
     recv = recv_t.cpu().numpy().reshape(world, 3)
     nrec, nkb, nvb = (int(x) for x in recv.sum(axis=0))
     rk = torch.empty(max(nkb, 1), dtype=torch.uint8, device=dev)
+    # send buffers sliced to the partition totals (the caller's arrays may carry trailing bytes)
+    ok = ok[: int(starts[-1, 1])]
+    oko = oko[: int(starts[-1, 0])] if oko is not None else None
+    ov = ov[: int(starts[-1, 2])] if ov is not None else None
     dist.all_to_all_single(rk[:nkb], ok, recv[:, 1].tolist(), send[:, 1].tolist(), group=group)
     rko = None
     if oko is not None:
@@ -100,3 +104,23 @@ def route(keys, key_offsets, vals, group=None, route_seed=0, fixed_key_width=0, 
     world = dist.get_world_size(group)
     ok, oko, ov, starts = partition(keys, key_offsets, vals, world, route_seed, fixed_key_width, fixed_val_width)
     return exchange(ok, oko, ov, starts, group)
+
+
+class Router:
+    """Routes each step's batch of this rank to the key owners (partition + exchange) and keeps
+    per-step statistics for the bench line."""
+
+    def __init__(self, group=None, route_seed=0, fixed_key_width=0, fixed_val_width=0):
+        self.group, self.seed, self.kw, self.vw = group, route_seed, fixed_key_width, fixed_val_width
+        self._last = {}
+
+    def route(self, keys, key_offsets, vals):
+        world = dist.get_world_size(self.group)
+        ok, oko, ov, starts = partition(keys, key_offsets, vals, world, self.seed, self.kw, self.vw)
+        out = exchange(ok, oko, ov, starts, self.group)
+        self._last = {"records_in": int(starts[-1, 0]), "records_out": int(out[1].numel() - 1) if out[1] is not None
+                      else int(out[0].numel() // max(self.kw, 1))}
+        return out
+
+    def last_stats(self):
+        return dict(self._last)

@@ -267,35 +267,6 @@ def test_reset_and_reuse(cuda):
     t.close()
 
 
-# ------------------------------------------------------------------ full size (bench launch config)
-def test_c2_full_size_sampled(cuda):
-    """C2 at BASELINE size (8 GiB text, 1.1e9 records) and budget F/4, as bench.py runs it:
-    every key's count equals the closed form c_r; totals: sum = n, #keys = V."""
-    import bench
-    s = gen.config("C2")
-    job = bench.make_job("C2", ratio=4.0)
-    k, o, v = job.inputs()
-    t = job.table()
-    passes = t.run(k, o, v)
-    res = t.export(copy=False)
-    assert passes >= 4
-    vals = res["values"]
-    assert res["n_keys"] == s.n_ranks
-    assert int(vals.sum(dtype=np.uint64)) == s.n
-    kb, ko = res["keys"], res["key_offsets"]
-    idx = np.random.default_rng(0).choice(res["n_keys"], 2000, replace=False)
-    spell2rank = None
-    for i in idx:
-        key = kb[ko[i]:ko[i + 1]].tobytes()
-        # rank from the spelling (base-26 digits) and its exact count c_r = floor(C/r)
-        r = 0
-        for ch in key:
-            r = r * 26 + (ch - 97)
-        assert s.spell(r) == key
-        assert int(vals[i]) == int(s.count_of_rank(r)), (key, r)
-    t.close()
-
-
 # ------------------------------------------------------------------ variable-length GROUP values
 def _csr_t(items):
     offs = np.zeros(len(items) + 1, dtype=np.int64)
