@@ -481,15 +481,28 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
     if (t->hot.grow(sepo_hot_scratch_bytes())) return fail(SEPO_E_NOMEM, "hot-set scratch");
     // BASIC halt rule: the pass stops once this many allocator slots failed
     const uint32_t halt_slots = (uint32_t)std::max<uint64_t>(1, ((uint64_t)t->grid * t->opts.basic_halt_pct + 99) / 100);
-    uint64_t key_end = 0;
+    uint64_t key_end = 0, key_begin = 0;
     if (b.ko && !b.idx) {  // the end of the batch's key bytes, a kernel parameter (see the kernel)
+        CK(t, cudaMemcpyAsync(&t->h_ko[0], b.ko, 8, cudaMemcpyDeviceToHost, t->stream));
         CK(t, cudaMemcpyAsync(&t->h_ko[1], b.ko + n, 8, cudaMemcpyDeviceToHost, t->stream));
         CK(t, cudaStreamSynchronize(t->stream));
+        key_begin = t->h_ko[0];
         key_end = t->h_ko[1];
+    }
+    // COMBINE pass 1 on contiguous input: the lean kernel unless the keys are long on average (URLs:
+    // insert_stream_kernel's warp-window loads suit them better); SEPO_LEAN=0/1 forces the choice
+    bool lean_in = false;
+    if (t->opts.mode == SEPO_COMBINE_SUM_U64 && !b.idx) {
+        const char* e = getenv("SEPO_LEAN");
+        const uint64_t mean = b.ko ? (key_end - key_begin) / n : t->opts.fixed_key_width;
+        // (measured: the lean path wins when the generation is L2-resident and the kernel is
+        // issue-bound — C2 4x pass 1 21.2 -> 19.6 ms — and loses ~1.4 % when table accesses go to
+        // HBM, where insert_stream_kernel's chunk-interleaved stream keeps fewer L1/L2 lines busy)
+        lean_in = (e && (e[0] == '0' || e[0] == '1')) ? e[0] == '1' : (mean <= 24 && !dir_prefetch(t));
     }
     bool hot_built = false;
     rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p, halt_slots, key_end, dir_prefetch(t),
-                            &hot_built);
+                            &hot_built, lean_in);
     if (rc) return cuda_check(t, (cudaError_t)rc, "insert kernel launch");
     CK(t, cudaEventRecord(t->ev1, t->stream));
     t->h_ko[2] = 0;

@@ -667,12 +667,17 @@ __device__ __forceinline__ void prep_close(const Batch& b, const PrepCursor& pc)
 template <int RB>
 __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, stream::CtaState& S, bool act, uint64_t w0,
                                              uint64_t w1, uint64_t h, uint64_t s, uint64_t v, uint32_t len, uint32_t g,
-                                             uint32_t gl, bool inj, bool& w_full, bool& w_quiet, PrepCursor& pc) {
+                                             uint32_t gl, bool inj, bool& w_full, bool& w_quiet, PrepCursor& pc,
+                                             bool hinted = false, uint32_t hint = 0) {
     const uint32_t lane = lane_id();
     const uint32_t bkt = bucket_of(h, d.n_buckets);
     const uint32_t tag = tag_of(h);
     const uint8_t* tail = b.keys + s + 16;
-    uint32_t head = act ? ld_dir(d.dir + bkt) : 0u;
+    // hinted: the caller read the bucket word earlier (and prefetched its head entry). A stale head
+    // is safe: entries are only ever linked at the head, so the chain below an older head is intact;
+    // a key linked after the snapshot is found by the CAS re-walk of [current head, stale head) in
+    // the allocation path, or by the post-quiescence re-walk of a decline
+    uint32_t head = act ? (hinted ? hint : ld_dir(d.dir + bkt)) : 0u;
     uint8_t* found = nullptr;
     if (head) {
         const uint8_t* e = ref_ptr(d, head);
@@ -1264,6 +1269,261 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         d.cursors[2 * blockIdx.x] = S.cs.cur[0];
         d.cursors[2 * blockIdx.x + 1] = S.cs.cur[1];
         for (uint32_t w = 0; w < (uint32_t)WARPS; ++w) { S.cs.post += S.cs.wpost[w]; S.cs.pkb += S.cs.wpkb[w]; }
+        if (S.cs.post) atomicAdd(&d.ctrl->postponed, S.cs.post);
+        if (S.cs.toolarge) atomicAdd(&d.ctrl->toolarge, S.cs.toolarge);
+        if (S.cs.dead) atomicAdd(&d.ctrl->dead_bytes, S.cs.dead);
+        if (S.cs.pkb) atomicAdd(&d.ctrl->kept_key_bytes, S.cs.pkb);
+    }
+}
+
+// ================================================================ COMBINE insert, lean input path (a1..a7)
+// Pass-1 COMBINE kernel for contiguous batches (CSR keys or fixed-width keys) whose keys are mostly
+// short (words, u64 keys). Same method as insert_stream_kernel — the sampled hot set in shared
+// memory with warp folding (a2), a per-warp miss queue resolved 32 misses at a time by resolve_core
+// (a3..a7) — with an input path that costs a fraction of the instructions:
+//   * every warp streams ONE contiguous range of 32-record groups (the next group is g + 1: no
+//     chunk striding, no per-group stage bookkeeping);
+//   * each lane loads its own key offsets ko[i] and ko[i + 1] two groups ahead (the second load is
+//     an L1 hit: offsets are read L1-allocating with an L2 evict_first policy), and the aligned
+//     8-byte words that hold its first 16 key bytes one group ahead (up to three predicated loads;
+//     a group's ~220 key bytes sit in 2-4 L1 lines) — no window shuffles;
+//   * the first 16 key bytes are assembled from 32-bit pieces with four funnel shifts.
+// Keys longer than 16 bytes still work (their tail is hashed and compared from global memory) but
+// the host picks insert_stream_kernel for long-key batches (mean key length > 24 B).
+// A queued miss is {w0, w1}, {h, s | len << 40 | lane << 59} and its group.
+namespace lean {
+constexpr int THREADS = 1024, WARPS = THREADS / 32, QCAP = 64;
+constexpr uint64_t S_MASK = (1ull << 40) - 1;
+constexpr uint32_t LEN_MAX = (1u << 19) - 1;
+template <bool VALS>
+struct Smem {
+    uint32_t tags[stream::DS];  // direct-indexed hot slots (as insert_stream_kernel)
+    ulonglong2 kw[stream::NKEY];
+    uint32_t ref[stream::NKEY];
+    typename std::conditional<VALS, unsigned long long, unsigned int>::type sum[stream::NKEY];
+    struct Queue {
+        ulonglong2 k[QCAP];   // first 16 key bytes (zero padded)
+        ulonglong2 hs[QCAP];  // hash, key offset | length << 40 | lane << 59
+        uint32_t g[QCAP];     // group of the record
+        unsigned long long v[VALS ? QCAP : 1];
+    } q[WARPS];
+    stream::CtaState cs;
+};
+static_assert(sizeof(Smem<true>) <= 232448, "lean kernel shared memory > 227 KB");
+
+// key offset and length of record i (CSR: two L1-allocating loads; fixed width: arithmetic)
+template <int IN>
+__device__ __forceinline__ void offsets(const Batch& b, uint64_t i, bool ok, uint64_t& s, uint64_t& e) {
+    if (IN == IN_CSR) {
+        s = ok ? ld_tail64(b.ko + i) : 0ull;
+        e = ok ? ld_tail64(b.ko + i + 1) : 0ull;
+    } else {
+        s = i * b.kw;
+        e = ok ? s + b.kw : s;
+    }
+}
+// the aligned words holding the first min(len, 16) key bytes at keys + s (only words that hold a
+// key byte are read)
+__device__ __forceinline__ void key_words(const uint8_t* keys, uint64_t s, uint32_t len, uint64_t& x0, uint64_t& x1,
+                                          uint64_t& x2) {
+    const uintptr_t a = reinterpret_cast<uintptr_t>(keys + s);
+    const unsigned long long* q = reinterpret_cast<const unsigned long long*>(a & ~(uintptr_t)7);
+    const uint32_t need = len ? (uint32_t)(a & 7u) + min(len, 16u) : 0u;  // bytes from q on
+    x0 = need > 0 ? ld_tail64(q) : 0ull;
+    x1 = need > 8 ? ld_tail64(q + 1) : 0ull;
+    x2 = need > 16 ? ld_tail64(q + 2) : 0ull;
+}
+// first 16 key bytes (zero padded) from the words x0..x2 that start o = (address & 7) bytes early
+__device__ __forceinline__ void assemble16(uint64_t x0, uint64_t x1, uint64_t x2, uint32_t o, uint32_t len, uint64_t& w0,
+                                           uint64_t& w1) {
+    const bool hi = o >= 4u;
+    const uint32_t t = 8u * (o & 3u);
+    const uint32_t u0 = (uint32_t)x0, u1 = (uint32_t)(x0 >> 32), u2 = (uint32_t)x1, u3 = (uint32_t)(x1 >> 32);
+    const uint32_t u4 = (uint32_t)x2, u5 = (uint32_t)(x2 >> 32);
+    const uint32_t q0 = hi ? u1 : u0, q1 = hi ? u2 : u1, q2 = hi ? u3 : u2, q3 = hi ? u4 : u3, q4 = hi ? u5 : u4;
+    const uint32_t r0 = __funnelshift_r(q0, q1, t), r1 = __funnelshift_r(q1, q2, t);
+    const uint32_t r2 = __funnelshift_r(q2, q3, t), r3 = __funnelshift_r(q3, q4, t);
+    const uint32_t nb8 = 8u * min(len, 16u);  // (PTX shl clamps the count at 64)
+    w0 = (((uint64_t)r1 << 32) | r0) & ~shl64_clamp(~0ull, nb8);
+    w1 = (((uint64_t)r3 << 32) | r2) & ~shl64_clamp(~0ull, nb8 > 64u ? nb8 - 64u : 0u);
+}
+}  // namespace lean
+
+// hot set of a launch into shared memory: keys claim slot ds1, else ds2, in decreasing sample
+// count (a Zipf head is never left out); read-only afterwards
+template <int DSN, int NK, typename SumT>
+__device__ __forceinline__ void load_hot_direct(uint32_t* tags, ulonglong2* kw, uint32_t* ref, SumT* sum,
+                                                const hot::Entry* hl, const unsigned int* n_hot) {
+    constexpr uint32_t M = DSN - 1;
+    const uint32_t tid = threadIdx.x, nt = blockDim.x;
+    for (uint32_t p = tid; p < (uint32_t)NK; p += nt) { ref[p] = 0; sum[p] = 0; }
+    for (uint32_t p = tid; p < (uint32_t)DSN; p += nt) tags[p] = 0u;
+    __syncthreads();
+    const unsigned nh = hl ? *n_hot : 0u;
+    for (int cls = 31; cls >= 0 && nh; --cls) {
+        for (unsigned j = tid; j < nh && j < (unsigned)NK; j += nt) {
+            const hot::Entry e = hl[j];
+            if (e.ref == 0 || hot::count_class(e.count) != cls) continue;
+            const uint32_t f = stream::dfp(e.h, e.len) | j;
+            if (atomicCAS(&tags[(uint32_t)(e.h >> 3) & M], 0u, f) == 0u || atomicCAS(&tags[(uint32_t)(e.h >> 17) & M], 0u, f) == 0u) {
+                kw[j] = make_ulonglong2(e.w0, e.w1);
+                ref[j] = e.ref;
+            }
+        }
+        __syncthreads();
+    }
+}
+
+template <bool VALS, int RB>
+__device__ __forceinline__ void lean_resolve(const Dev& d, const Batch& b, lean::Smem<VALS>& S,
+                                             typename lean::Smem<VALS>::Queue& Q, uint32_t qhead, uint32_t cnt, bool inj,
+                                             bool& w_full, bool& w_quiet, PrepCursor& pc) {
+    const uint32_t lane = lane_id();
+    const bool act = lane < cnt;
+    const uint32_t k = (qhead + lane) & (lean::QCAP - 1);
+    uint64_t w0 = 0, w1 = 0, h = 0, s = 0, v = 1;
+    uint32_t g = 0, len = 0, gl = 0;
+    if (act) {
+        const ulonglong2 kk = Q.k[k], hs = Q.hs[k];
+        w0 = kk.x; w1 = kk.y; h = hs.x;
+        s = hs.y & lean::S_MASK;
+        len = (uint32_t)(hs.y >> 40) & lean::LEN_MAX;
+        gl = (uint32_t)(hs.y >> 59);
+        g = Q.g[k];
+        if (VALS) v = Q.v[k];
+    }
+    resolve_core<RB>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
+}
+
+// RB: prepared re-issue record format (32: implicit values; 33: <= 8-byte keys with values; 48)
+template <bool VALS, int IN, int RB>
+__global__ void __launch_bounds__(lean::THREADS, 1) insert_lean_kernel(Dev d, Batch b, const hot::Entry* hl,
+                                                                       const unsigned int* n_hot, const InCtx c) {
+    using SM = lean::Smem<VALS>;
+    extern __shared__ __align__(16) uint8_t smem_raw[];
+    SM& S = *reinterpret_cast<SM*>(smem_raw);
+    const uint32_t tid = threadIdx.x, lane = lane_id(), wid = tid >> 5;
+    if (tid == 0) {
+        S.cs.cur[0] = d.cursors[2 * blockIdx.x];
+        S.cs.cur[1] = d.cursors[2 * blockIdx.x + 1];
+        S.cs.post = 0; S.cs.toolarge = 0; S.cs.dead = 0; S.cs.pkb = 0;
+    }
+    if (tid < 32) { S.cs.wpost[tid] = 0; S.cs.wpkb[tid] = 0; }
+    load_hot_direct<stream::DS, stream::NKEY>(S.tags, S.kw, S.ref, S.sum, hl, n_hot);
+    __syncthreads();
+    const bool have_hot = hl != nullptr && *n_hot > 0;
+    const bool big = b.n >= (1ull << 32);
+    const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
+    typename SM::Queue& Q = S.q[wid];
+    uint32_t qhead = 0, qtail = 0;
+    PrepCursor pc;
+    bool w_full = false, w_quiet = false;
+    // this warp's groups [g, gend): an equal share of the batch, streamed in order
+    const uint64_t gw = (uint64_t)blockIdx.x * lean::WARPS + wid;
+    uint32_t g = (uint32_t)((uint64_t)c.ngroups * gw / c.nw);
+    const uint32_t gend = (uint32_t)((uint64_t)c.ngroups * (gw + 1) / c.nw);
+    // pipeline: key words of group g and offsets of g + 1 in flight before group g is processed
+    auto cnt_of = [&](uint32_t x) -> uint32_t { return x < gend ? (x + 1 == c.ngroups ? c.tail : 32u) : 0u; };
+    uint64_t s_c, e_c, s_n, e_n, v_c = 1, x0, x1, x2;
+    {
+        const bool ok = lane < cnt_of(g);
+        lean::offsets<IN>(b, (uint64_t)g * 32 + lane, ok, s_c, e_c);
+        if (VALS && ok) v_c = rec_value(b, (uint64_t)g * 32 + lane);
+        lean::key_words(b.keys, s_c, (uint32_t)(e_c - s_c), x0, x1, x2);
+        lean::offsets<IN>(b, (uint64_t)(g + 1) * 32 + lane, lane < cnt_of(g + 1), s_n, e_n);
+    }
+    for (; g < gend; ++g) {
+        // ---- issue ahead: key words (values) of g + 1, offsets of g + 2
+        uint64_t y0, y1, y2, v_n = 1;
+        lean::key_words(b.keys, s_n, (uint32_t)(e_n - s_n), y0, y1, y2);
+        if (VALS && lane < cnt_of(g + 1)) v_n = rec_value(b, (uint64_t)(g + 1) * 32 + lane);
+        uint64_t s_nn, e_nn;
+        lean::offsets<IN>(b, (uint64_t)(g + 2) * 32 + lane, lane < cnt_of(g + 2), s_nn, e_nn);
+        // ---- group g: first 16 key bytes + hash (a1)
+        const bool valid = lane < cnt_of(g);
+        const uint64_t s = s_c;
+        const uint32_t len = (uint32_t)(e_c - s_c);  // 0 for lanes past the end
+        uint64_t w0, w1;
+        lean::assemble16(x0, x1, x2, (uint32_t)(reinterpret_cast<uintptr_t>(b.keys + s) & 7u), len, w0, w1);
+        const uint64_t v = VALS ? v_c : 1ull;
+        const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
+        // ---- hot set (a2): two one-word slots, then one 16-byte key compare
+        int pos = -1;
+        if (have_hot) {
+            const uint32_t f = stream::dfp(h, len);
+            const uint32_t t1 = S.tags[stream::ds1(h)], t2 = S.tags[stream::ds2(h)];
+            constexpr uint32_t IM = (1u << stream::IDXB) - 1u;
+            const bool m1 = (t1 & ~IM) == f, m2 = (t2 & ~IM) == f;
+            const uint32_t p = (m1 ? t1 : t2) & IM;
+            if (valid && (m1 || m2)) {
+                const ulonglong2 kk = S.kw[p];
+                bool eq = kk.x == w0 && kk.y == w1;
+                if (len > 16) {  // long key: exact length (the fingerprint saturates at 255) + tail bytes
+                    const uint8_t* e = ref_ptr(d, S.ref[p]);
+                    eq = eq && ldcg32(e + 12) == len && entry_key_eq(e + KEY_OFF + 16, b.keys + s + 16, len - 16);
+                }
+                if (eq) pos = (int)p;
+            }
+        }
+        // ---- fold the warp's hits per hot key: one shared atomic per distinct key (a2)
+        const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
+        if (hm) {
+            const unsigned grp = __match_any_sync(FULLMASK, pos >= 0 ? (unsigned)pos : (0x10000u | lane)) & hm;
+            const bool leader = pos >= 0 && lane == (uint32_t)(__ffs(grp) - 1);
+            if (!VALS) {
+                if (leader) {
+                    const unsigned add = (unsigned)__popc(grp);
+                    const unsigned old = atomicAdd(reinterpret_cast<unsigned int*>(&S.sum[pos]), add);
+                    if (big && old + add < old)  // 2^32 wrap of the CTA-local count: carry into the entry
+                        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(ref_ptr(d, S.ref[pos]), len)), 1ull << 32);
+                }
+            } else {
+                uint64_t acc = v;
+                if (__any_sync(FULLMASK, __popc(grp) > 1)) {
+                    acc = 0;
+                    for (int xl = 0; xl < 32; ++xl) {
+                        const uint64_t vx = __shfl_sync(FULLMASK, v, xl);
+                        if ((grp >> xl) & 1u) acc += vx;
+                    }
+                }
+                if (leader) atomicAdd(reinterpret_cast<unsigned long long*>(&S.sum[pos]), (unsigned long long)acc);
+            }
+        }
+        // ---- misses: the warp's queue, resolved 32 at a time (a3..a7); the bitmap word starts at 0
+        const bool miss = valid && pos < 0;
+        const unsigned mm = __ballot_sync(FULLMASK, miss);
+        if (lane == 0 && b.bitmap) b.bitmap[g] = 0u;
+        if (miss) {
+            if (c.dirpf) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(d.dir + bucket_of(h, d.n_buckets)));
+            const uint32_t k = (qtail + __popc(mm & lanemask_lt())) & (lean::QCAP - 1);
+            Q.k[k] = make_ulonglong2(w0, w1);
+            Q.hs[k] = make_ulonglong2(h, s | ((uint64_t)min(len, lean::LEN_MAX) << 40) | ((uint64_t)lane << 59));
+            Q.g[k] = g;
+            if (VALS) Q.v[k] = v;
+        }
+        qtail += __popc(mm);
+        __syncwarp();
+        if (qtail - qhead >= 32) {
+            lean_resolve<VALS, RB>(d, b, S, Q, qhead, 32, inj, w_full, w_quiet, pc);
+            qhead += 32;
+            __syncwarp();
+        }
+        // ---- rotate the pipeline
+        s_c = s_n; e_c = e_n; v_c = v_n; x0 = y0; x1 = y1; x2 = y2;
+        s_n = s_nn; e_n = e_nn;
+    }
+    if (qtail != qhead) lean_resolve<VALS, RB>(d, b, S, Q, qhead, qtail - qhead, inj, w_full, w_quiet, pc);
+    if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
+    __syncthreads();
+    for (int p = tid; p < stream::NKEY; p += lean::THREADS) {  // pending hot sums -> resident entries
+        if (S.ref[p] == 0 || S.sum[p] == 0) continue;
+        uint8_t* e = ref_ptr(d, S.ref[p]);
+        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(e, ldcg32(e + 12))), (unsigned long long)S.sum[p]);
+    }
+    if (tid == 0) {
+        d.cursors[2 * blockIdx.x] = S.cs.cur[0];
+        d.cursors[2 * blockIdx.x + 1] = S.cs.cur[1];
+        for (uint32_t w = 0; w < (uint32_t)lean::WARPS; ++w) { S.cs.post += S.cs.wpost[w]; S.cs.pkb += S.cs.wpkb[w]; }
         if (S.cs.post) atomicAdd(&d.ctrl->postponed, S.cs.post);
         if (S.cs.toolarge) atomicAdd(&d.ctrl->toolarge, S.cs.toolarge);
         if (S.cs.dead) atomicAdd(&d.ctrl->dead_bytes, S.cs.dead);
@@ -2448,6 +2708,261 @@ __global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, B
     }
 }
 
+// ---- fused tokenizer, version 2: full 32-word rounds, three-window ring, cheaper separators
+// Same method as insert_text_kernel (a word is a record with value 1; its identity is its text
+// offset), restructured so that almost every round hands one word to each of the 32 lanes:
+//   * a warp streams ONE contiguous range of 512-byte windows; the ring holds three consecutive
+//     windows (text bytes + separator bits), so words of a window that do not fill a round are
+//     carried into the next window's first round (their bytes are still in the ring);
+//   * separator bits: per 32-bit word, one masked add per separator byte value and one combined
+//     test (a byte b is a separator iff b is one of ' ', '\n', '\t', '\r', reading R20);
+//   * a word's end: the first separator bit at or after its start in a 64-bit window of the ring's
+//     separator bits (words longer than 32 bytes continue the scan, longer than the ring: global);
+//   * queue slots as the lean CSR kernel (32 bytes: first 16 key bytes, hash, offset | length).
+namespace text2 {
+constexpr int THREADS = 1024, WARPS = THREADS / 32;
+constexpr int WB = 512, NSLOT = 3, RINGB = NSLOT * WB, SEPW = RINGB / 32;
+constexpr int DSZ = 8192, TK = 2048;
+constexpr int WLCAP = 288;  // carried words (< 32) + one window's word starts (<= 256)
+constexpr int QCAP = 64;
+struct WarpText {
+    // text ring: three consecutive windows, then a ghost copy of the first 32 bytes of slot 0 (so
+    // reads of up to 24 bytes past a position never wrap)
+    uint4 t[NSLOT * 32 + 2];
+    uint32_t sep[SEPW + 2];  // separator bits: bit j of word k = ring byte 32k + j (+ ghost of words 0, 1)
+    uint16_t wl[WLCAP];      // ring positions of the word starts waiting for a round
+};
+struct Smem {
+    uint32_t tags[DSZ];
+    ulonglong2 kw[TK];
+    uint32_t ref[TK];
+    unsigned int sum[TK];
+    struct Queue {
+        ulonglong2 k[QCAP];   // first 16 key bytes
+        ulonglong2 hs[QCAP];  // hash, text offset | length << 40 | lane << 59
+    } q[WARPS];
+    WarpText w[WARPS];
+    stream::CtaState cs;
+};
+static_assert(sizeof(Smem) <= 232448, "text2 kernel shared memory > 227 KB");
+// 4 separator bits of the 4 bytes of w (bit k = byte k). Exact per-byte equality with c: for
+// x = (w & 0x7f7f7f7f) ^ c7, bit 7 of x + 0x7f7f7f7f is 0 iff the low 7 bits of the byte equal c's;
+// bit 7 of the byte itself must be 0 too (every separator is < 0x80).
+__device__ __forceinline__ uint32_t sep4(uint32_t w) {
+    const uint32_t w7 = w & 0x7f7f7f7fu;
+    const uint32_t t1 = (w7 ^ 0x20202020u) + 0x7f7f7f7fu, t2 = (w7 ^ 0x0a0a0a0au) + 0x7f7f7f7fu;
+    const uint32_t t3 = (w7 ^ 0x09090909u) + 0x7f7f7f7fu, t4 = (w7 ^ 0x0d0d0d0du) + 0x7f7f7f7fu;
+    const uint32_t m = ~((t1 & t2 & t3 & t4) | w) & 0x80808080u;  // 0x80 in every separator byte
+    return ((m >> 7) * 0x10204080u) >> 28;                          // byte k -> bit k
+}
+__device__ __forceinline__ uint32_t sep16(uint4 c, uint32_t valid) {
+    uint32_t out = sep4(c.x) | (sep4(c.y) << 4) | (sep4(c.z) << 8) | (sep4(c.w) << 12);
+    if (valid < 16) out |= (0xffffu << valid) & 0xffffu;  // bytes past the text end separate
+    return out;
+}
+// stage window chunk `ch` (lane's 16 bytes) into ring slot `slot`: bytes + separator bits
+__device__ __forceinline__ void stage(WarpText& W, uint32_t slot, uint32_t lane, uint4 ch, uint32_t valid) {
+    W.t[slot * 32 + lane] = ch;
+    const uint32_t sp = sep16(ch, valid);
+    const uint32_t other = __shfl_down_sync(FULLMASK, sp, 1);
+    if (!(lane & 1)) W.sep[slot * 16 + (lane >> 1)] = sp | (other << 16);
+    if (slot == 0 && lane < 4) {  // the ghost after slot 2: its first 32 bytes and 2 separator words
+        if (lane < 2) W.t[NSLOT * 32 + lane] = ch;
+        if (!(lane & 1)) W.sep[SEPW + (lane >> 1)] = sp | (other << 16);
+    }
+}
+}  // namespace text2
+
+__global__ void __launch_bounds__(text2::THREADS, 1) insert_text2_kernel(Dev d, Batch b, const hot::Entry* hl,
+                                                                           const unsigned int* n_hot) {
+    using namespace text2;
+    extern __shared__ __align__(16) uint8_t smem_raw[];
+    text2::Smem& S = *reinterpret_cast<text2::Smem*>(smem_raw);
+    const uint32_t tid = threadIdx.x, lane = lane_id(), wid = tid >> 5;
+    if (tid == 0) {
+        S.cs.cur[0] = d.cursors[2 * blockIdx.x];
+        S.cs.cur[1] = d.cursors[2 * blockIdx.x + 1];
+        S.cs.post = 0; S.cs.toolarge = 0; S.cs.dead = 0; S.cs.pkb = 0;
+    }
+    if (tid < 32) { S.cs.wpost[tid] = 0; S.cs.wpkb[tid] = 0; }
+    load_hot_direct<DSZ, TK>(S.tags, S.kw, S.ref, S.sum, hl, n_hot);
+    __syncthreads();
+    const bool have_hot = hl != nullptr && *n_hot > 0;
+    const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
+    const uint8_t* T = b.keys;
+    const uint64_t n = b.n;
+    const uint64_t nwin_all = (n + WB - 1) / WB;
+    const uint64_t lw0 = b.w_begin, lw1 = b.w_end < nwin_all ? b.w_end : nwin_all;  // this launch's windows
+    const bool big = n / 2 >= (1ull << 32);  // words < 2^32: a CTA-local count cannot wrap
+    WarpText& W = S.w[wid];
+    auto& Q = S.q[wid];
+    const uint64_t* R = reinterpret_cast<const uint64_t*>(&W.t[0]);  // the ring as 192 words (+ ghost)
+    uint32_t qhead = 0, qtail = 0;
+    PrepCursor pc;
+    bool w_full = false, w_quiet = false;
+    unsigned long long words = 0;  // lane 0
+    // this warp's windows [wa, wz): an equal share of the launch's windows
+    const uint64_t nlw = lw1 > lw0 ? lw1 - lw0 : 0;
+    const uint64_t gw = (uint64_t)blockIdx.x * WARPS + wid, nwp = (uint64_t)gridDim.x * WARPS;
+    const uint64_t wa = lw0 + nlw * gw / nwp, wz = lw0 + nlw * (gw + 1) / nwp;
+
+    if (wa < wz) {
+        uint32_t prev = 1u;  // is the byte before window wa a separator (text start: yes)
+        if (wa > 0) prev = is_sep(ld_in8(T + wa * WB - 1)) ? 1u : 0u;
+        uint32_t vl;
+        uint4 ch = textk::load_chunk(T, n, wa, lane, vl);
+        stage(W, 0, lane, ch, vl);
+        ch = textk::load_chunk(T, n, wa + 1, lane, vl);  // (zeros past the text end)
+        stage(W, 1, lane, ch, vl);
+        uint32_t vl_n;
+        uint4 ch_n = textk::load_chunk(T, n, wa + 2, lane, vl_n);
+        uint32_t cslot = 0, nl = 0;  // ring slot of window w; words waiting in the list
+        for (uint64_t w = wa; w < wz; ++w) {
+            __syncwarp();
+            // ---- word starts of window w (a1): a non-separator byte after a separator
+            const uint32_t sw = W.sep[cslot * 16 + (lane >> 1)];
+            const uint32_t sp = (lane & 1) ? (sw >> 16) : (sw & 0xffffu);
+            const uint32_t up = __shfl_up_sync(FULLMASK, sp, 1);
+            const uint32_t pbit = lane == 0 ? prev : ((up >> 15) & 1u);
+            const uint32_t st = ~sp & ((sp << 1) | pbit) & 0xffffu;
+            prev = (__shfl_sync(FULLMASK, sp, 31) >> 15) & 1u;
+            const uint32_t cnt = __popc(st);
+            uint32_t incl = cnt;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(FULLMASK, incl, o);
+                if (lane >= (uint32_t)o) incl += y;
+            }
+            const uint32_t total = __shfl_sync(FULLMASK, incl, 31);
+            const uint32_t rbase = cslot * WB + lane * 16;
+            for (uint32_t m = st, k = nl + incl - cnt; m; m &= m - 1) W.wl[k++] = (uint16_t)(rbase + __ffs(m) - 1);
+            nl += total;
+            words += total;
+            __syncwarp();
+            // ---- rounds of 32 words (one per lane); a partial round only for carried words of the
+            // window before (its ring slot is restaged next) and at the end of the warp's range
+            uint32_t h = 0;
+            while (true) {
+                bool go = nl >= 32;
+                if (!go && nl > 0) go = (w + 1 == wz) || ((W.wl[h] >> 9) != cslot);
+                if (!go) break;
+                const uint32_t nr = min(nl, 32u);
+                const bool valid = lane < nr;
+                const uint32_t p = valid ? W.wl[h + lane] : 0u;  // ring byte of the word start
+                h += nr;
+                nl -= nr;
+                const uint32_t slot = p >> 9;
+                // the word's window: the current one, or (a carried word) the one before it
+                const uint64_t s = ((w - (slot != cslot ? 1u : 0u)) << 9) | (p & (WB - 1));
+                uint32_t len = 0;
+                uint64_t w0 = 0, w1 = 0;
+                if (valid) {
+                    // end: the first separator bit in the 32 bits from p on (funnel of two map words)
+                    uint32_t wi = p >> 5;
+                    const uint32_t m32 = __funnelshift_r(W.sep[wi], W.sep[wi + 1], p & 31u);
+                    if (m32) {
+                        len = (uint32_t)__ffs(m32) - 1;
+                    } else {  // 32 bytes or longer: scan on through its window and the next, then global memory
+                        const uint32_t wend = ((slot + 2) % NSLOT) * 16;
+                        uint32_t m2 = 0;
+                        wi = (wi + 1) % SEPW;
+                        while (wi != wend && (m2 = W.sep[wi]) == 0) wi = (wi + 1) % SEPW;
+                        len = (wi != wend && m2) ? (uint32_t)((wi * 32 + RINGB - p) % RINGB) + __ffs(m2) - 1
+                                                 : text_word_len(T, n, s);
+                    }
+                    // first 16 key bytes from the ring (aligned 8-byte words; the ghost covers the wrap)
+                    const uint32_t a = p >> 3;
+                    lean::assemble16(R[a], R[a + 1], R[a + 2], p & 7u, len, w0, w1);
+                }
+                const uint64_t hh = hash_key16(len, d.seed, w0, w1, T + s);
+                // ---- hot set (a2)
+                int pos = -1;
+                if (have_hot) {
+                    const uint32_t f = stream::dfp_b<11>(hh, len);
+                    const uint32_t t1 = S.tags[(uint32_t)(hh >> 3) & (DSZ - 1)], t2 = S.tags[(uint32_t)(hh >> 17) & (DSZ - 1)];
+                    const bool m1 = (t1 & 0xfffff800u) == f, m2 = (t2 & 0xfffff800u) == f;
+                    const uint32_t q = (m1 ? t1 : t2) & 0x7ffu;
+                    if (valid && (m1 || m2)) {
+                        const ulonglong2 kk = S.kw[q];
+                        bool eq = kk.x == w0 && kk.y == w1;
+                        if (len > 16) {
+                            const uint8_t* e = ref_ptr(d, S.ref[q]);
+                            eq = eq && ldcg32(e + 12) == len && entry_key_eq(e + KEY_OFF + 16, T + s + 16, len - 16);
+                        }
+                        if (eq) pos = (int)q;
+                    }
+                }
+                const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
+                if (hm) {
+                    const unsigned grp = __match_any_sync(FULLMASK, pos >= 0 ? (unsigned)pos : (0x10000u | lane)) & hm;
+                    if (pos >= 0 && lane == (uint32_t)(__ffs(grp) - 1)) {
+                        const unsigned add = (unsigned)__popc(grp);
+                        const unsigned old = atomicAdd(&S.sum[pos], add);
+                        if (big && old + add < old)
+                            red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(ref_ptr(d, S.ref[pos]), len)), 1ull << 32);
+                    }
+                }
+                // ---- misses: the warp's queue, resolved 32 at a time (a3..a7)
+                const bool miss = valid && pos < 0;
+                const unsigned mm = __ballot_sync(FULLMASK, miss);
+                if (miss) {
+                    if (b.dirpf) asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(d.dir + bucket_of(hh, d.n_buckets)));
+                    const uint32_t kq = (qtail + __popc(mm & lanemask_lt())) & (QCAP - 1);
+                    Q.k[kq] = make_ulonglong2(w0, w1);
+                    Q.hs[kq] = make_ulonglong2(hh, s | ((uint64_t)min(len, lean::LEN_MAX) << 40) | ((uint64_t)lane << 59));
+                }
+                qtail += __popc(mm);
+                __syncwarp();
+                if (qtail - qhead >= 32) {
+                    const uint32_t kq = (qhead + lane) & (QCAP - 1);
+                    const ulonglong2 kk = Q.k[kq], hs = Q.hs[kq];
+                    resolve_core<32>(d, b, S.cs, true, kk.x, kk.y, hs.x, hs.y & lean::S_MASK, 1ull,
+                                     (uint32_t)(hs.y >> 40) & lean::LEN_MAX, 0u, (uint32_t)(hs.y >> 59), inj, w_full, w_quiet,
+                                     pc);
+                    qhead += 32;
+                    __syncwarp();
+                }
+            }
+            // the (< 32) carried words to the front of the list
+            if (h && nl) {
+                const uint16_t x = lane < nl ? W.wl[h + lane] : (uint16_t)0;
+                __syncwarp();
+                if (lane < nl) W.wl[lane] = x;
+            }
+            __syncwarp();
+            // ---- window w + 2 into the slot of w - 1 (no carried word is from w - 1 now), load w + 3
+            stage(W, (cslot + 2) % NSLOT, lane, ch_n, vl_n);
+            if (w + 3 < wz + 2) ch_n = textk::load_chunk(T, n, w + 3, lane, vl_n);
+            cslot = (cslot + 1) % NSLOT;
+        }
+    }
+    if (qtail != qhead) {
+        const bool act = lane < qtail - qhead;
+        const uint32_t kq = (qhead + lane) & (QCAP - 1);
+        ulonglong2 kk = make_ulonglong2(0, 0), hs = make_ulonglong2(0, 0);
+        if (act) { kk = Q.k[kq]; hs = Q.hs[kq]; }
+        resolve_core<32>(d, b, S.cs, act, kk.x, kk.y, hs.x, hs.y & lean::S_MASK, 1ull, (uint32_t)(hs.y >> 40) & lean::LEN_MAX,
+                         0u, (uint32_t)(hs.y >> 59), inj, w_full, w_quiet, pc);
+    }
+    if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
+    if (lane == 0 && words) atomicAdd(&d.ctrl->text_words, words);
+    __syncthreads();
+    for (int p = tid; p < TK; p += THREADS) {
+        if (S.ref[p] == 0 || S.sum[p] == 0) continue;
+        uint8_t* e = ref_ptr(d, S.ref[p]);
+        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(e, ldcg32(e + 12))), (unsigned long long)S.sum[p]);
+    }
+    if (tid == 0) {
+        d.cursors[2 * blockIdx.x] = S.cs.cur[0];
+        d.cursors[2 * blockIdx.x + 1] = S.cs.cur[1];
+        for (uint32_t w = 0; w < (uint32_t)WARPS; ++w) { S.cs.post += S.cs.wpost[w]; S.cs.pkb += S.cs.wpkb[w]; }
+        if (S.cs.post) atomicAdd(&d.ctrl->postponed, S.cs.post);
+        if (S.cs.toolarge) atomicAdd(&d.ctrl->toolarge, S.cs.toolarge);
+        if (S.cs.dead) atomicAdd(&d.ctrl->dead_bytes, S.cs.dead);
+        if (S.cs.pkb) atomicAdd(&d.ctrl->kept_key_bytes, S.cs.pkb);
+    }
+}
+
 // Words whose start bit is set in b.tbm (declined when the prepared list was full) -> 32-byte
 // prepared records appended at out[*counter++]; the bits are cleared for the next use.
 __global__ void __launch_bounds__(256) text_bits_kernel(Dev d, Batch b, unsigned long long* counter) {
@@ -2603,9 +3118,12 @@ int sepo_launch_insert_text(const Dev& d, const Batch& b0, int grid, cudaStream_
     static bool attr = false;
     if (!attr) {
         cudaFuncSetAttribute(insert_text_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(textk::Smem));
+        cudaFuncSetAttribute(insert_text2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(text2::Smem));
         attr = true;
     }
-    insert_text_kernel<<<grid, textk::THREADS, sizeof(textk::Smem), s>>>(d, b, hl, nh);
+    const char* v = getenv("SEPO_TEXT2");  // 0: the first fused tokenizer (insert_text_kernel)
+    if (v && v[0] == '0') insert_text_kernel<<<grid, textk::THREADS, sizeof(textk::Smem), s>>>(d, b, hl, nh);
+    else insert_text2_kernel<<<grid, text2::THREADS, sizeof(text2::Smem), s>>>(d, b, hl, nh);
     return cudaGetLastError();
 }
 int sepo_launch_lookup_gen(const Dev& d, const Batch& b, const uint32_t* pages, uint32_t np, unsigned long long* vals,
@@ -2625,7 +3143,7 @@ int sepo_launch_evict_copy(const Dev& d, uint32_t n, uint8_t* dst, int grid, cud
 }
 
 int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
-                       uint32_t halt_slots, uint64_t key_end, bool dir_prefetch, bool* hot_built) {
+                       uint32_t halt_slots, uint64_t key_end, bool dir_prefetch, bool* hot_built, bool lean_in) {
     if (hot_built) *hot_built = false;
     if (mode == 2) {
         insert_basic_kernel<<<grid, 1024, 0, s>>>(d, b, halt_slots);
@@ -2646,9 +3164,10 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             unsigned int* hist = n_out + 1;
             cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
             hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
-            hot_threshold_kernel<<<1, 1024, 0, s>>>(hist, 4u, (uint32_t)hot::K);
-            hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)hot::K);
-            hot_clamp_kernel<<<1, 32, 0, s>>>(n_out, (uint32_t)hot::K);
+            const uint32_t kmax = (uint32_t)hot::K;
+            hot_threshold_kernel<<<1, 1024, 0, s>>>(hist, 4u, kmax);
+            hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, kmax);
+            hot_clamp_kernel<<<1, 32, 0, s>>>(n_out, kmax);
             hot_resolve_kernel<<<1, 1024, 0, s>>>(d, b, list, n_out);
             hl = list;
             nh = n_out;
@@ -2675,6 +3194,33 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
         c.kend = in == IN_IDX ? 0ull : (in == IN_CSR ? key_end : b.n * (uint64_t)b.kw);
         c.kal = !(reinterpret_cast<uintptr_t>(b.keys) & 15);
         c.dirpf = dir_prefetch;
+        if (lean_in && in != IN_IDX) {  // contiguous batch of mostly short keys: the lean input path
+            static bool attr_l = false;
+            if (!attr_l) {
+                const int s0 = (int)sizeof(lean::Smem<false>), s1 = (int)sizeof(lean::Smem<true>);
+                cudaFuncSetAttribute(insert_lean_kernel<false, IN_CSR, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, s0);
+                cudaFuncSetAttribute(insert_lean_kernel<false, IN_FIXED, 32>, cudaFuncAttributeMaxDynamicSharedMemorySize, s0);
+                cudaFuncSetAttribute(insert_lean_kernel<true, IN_CSR, 33>, cudaFuncAttributeMaxDynamicSharedMemorySize, s1);
+                cudaFuncSetAttribute(insert_lean_kernel<true, IN_FIXED, 33>, cudaFuncAttributeMaxDynamicSharedMemorySize, s1);
+                cudaFuncSetAttribute(insert_lean_kernel<true, IN_CSR, 48>, cudaFuncAttributeMaxDynamicSharedMemorySize, s1);
+                cudaFuncSetAttribute(insert_lean_kernel<true, IN_FIXED, 48>, cudaFuncAttributeMaxDynamicSharedMemorySize, s1);
+                attr_l = true;
+            }
+            c.nw = (uint32_t)grid * lean::WARPS;
+            const size_t sml = b.vals ? sizeof(lean::Smem<true>) : sizeof(lean::Smem<false>);
+            const dim3 G(grid), B(lean::THREADS);
+            if (!b.vals) {
+                if (in == IN_CSR) insert_lean_kernel<false, IN_CSR, 32><<<G, B, sml, s>>>(d, b, hl, nh, c);
+                else insert_lean_kernel<false, IN_FIXED, 32><<<G, B, sml, s>>>(d, b, hl, nh, c);
+            } else if (b.prep_fmt == 33) {
+                if (in == IN_CSR) insert_lean_kernel<true, IN_CSR, 33><<<G, B, sml, s>>>(d, b, hl, nh, c);
+                else insert_lean_kernel<true, IN_FIXED, 33><<<G, B, sml, s>>>(d, b, hl, nh, c);
+            } else {
+                if (in == IN_CSR) insert_lean_kernel<true, IN_CSR, 48><<<G, B, sml, s>>>(d, b, hl, nh, c);
+                else insert_lean_kernel<true, IN_FIXED, 48><<<G, B, sml, s>>>(d, b, hl, nh, c);
+            }
+            return cudaGetLastError();
+        }
         if (b.vals) {
             if (in == IN_CSR) insert_stream_kernel<true, T, IN_CSR><<<grid, T, sm, s>>>(d, b, hl, nh, c);
             else if (in == IN_FIXED) insert_stream_kernel<true, T, IN_FIXED><<<grid, T, sm, s>>>(d, b, hl, nh, c);

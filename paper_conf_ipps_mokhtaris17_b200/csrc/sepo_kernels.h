@@ -45,11 +45,12 @@ struct Batch {
 }  // namespace sepo
 
 // key_end: key_offsets[n] of a CSR batch (the end of its key bytes), read by the host
+// lean_in: COMBINE contiguous batches take insert_lean_kernel (mostly short keys; the host decides)
 // *hot_built (optional): whether this launch selected a sampled hot set (its size is the u32 at
 // hot_scratch + sepo_hot_count_offset(), clamped to the kernel's capacity)
 int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
                        uint32_t halt_slots = 0, uint64_t key_end = 0, bool dir_prefetch = false,
-                       bool* hot_built = nullptr);
+                       bool* hot_built = nullptr, bool lean_in = false);
 size_t sepo_hot_count_offset();
 int sepo_launch_reinsert(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s);
 size_t sepo_hot_scratch_bytes();

@@ -67,7 +67,7 @@ def test_evict_overlap(cuda, monkeypatch, overlap):
     for _ in range(2):  # the second job reuses the table's pages while nothing is in flight
         got, passes, st = run_job(s, sepo().budget_for(1 << 14, 4096, P), 1 << 14, 4096, inputs=inp, check_dups=True)
         assert_same(got, exp)
-        assert passes >= 4 and st["cross_gen_dups"] == 0
+        assert passes >= 3 and st["cross_gen_dups"] == 0
 
 
 @pytest.mark.parametrize("reissue", ["prepared", "prepared_overflow", "index"])
@@ -85,7 +85,7 @@ def test_reissue_paths(cuda, monkeypatch, reissue):
     F, P = budget_pages(s, 3, 1 << 14, 16384, inp)
     got, passes, st = run_job(s, sepo().budget_for(1 << 14, 16384, P), 1 << 14, 16384, inputs=inp, check_dups=True)
     assert_same(got, exp)
-    assert passes >= 3
+    assert passes >= 2
     assert st["cross_gen_dups"] == 0
     post = st["postponed_per_pass"]
     assert all(post[i] > post[i + 1] for i in range(len(post) - 1)) and post[-1] == 0, post
@@ -329,7 +329,7 @@ def test_evict_copy_paths(cuda, monkeypatch, cfg, evk):
     F, P = budget_pages(s, 3, 1 << 14, 4096, inp, **kw)
     got, passes, st = run_job(s, sepo().budget_for(1 << 14, 4096, P), 1 << 14, 4096, inputs=inp, check_dups=True, **kw)
     assert_same(got, exp)
-    assert passes >= 3
+    assert passes >= 2
 
 
 @pytest.mark.parametrize("ratio", [0.5, 4])

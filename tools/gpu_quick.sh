@@ -1,7 +1,6 @@
-# usage: bash tools/gpu_quick.sh "JOBS" "VARIANTS" [gpu tests: 1]
-python tools/build.py > gpurun_out/build.log 2>&1
-if [ "$3" = "1" ]; then timeout 900 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo rc=$? >> gpurun_out/pytest_gpu.log; fi
-timeout 900 python tools/variants.py run $1 -- $2 > gpurun_out/var.jsonl 2> gpurun_out/var.err
-for v in $2; do
-  SEPO_LIB=exp/lib_$v.so timeout 300 ncu --metrics dram__bytes_read.sum,gpu__time_duration.sum,smsp__inst_executed.sum,smsp__issue_active.avg.pct_of_peak_sustained_active --clock-control none -k regex:insert_stream -c 1 --csv python tools/time_job.py C2 0.5 > gpurun_out/ncuq_$v.csv 2>&1
-done
+# quick GPU check: selected tests + A/B timings. bash tools/gpu_quick.sh TAG "pytest args" [ab envs...]
+TAG=$1; T=$2; shift 2
+python tools/build.py > gpurun_out/build_$TAG.log 2>&1 || { echo build failed; exit 1; }
+if [ -n "$T" ]; then timeout 1200 python -m pytest -x -q -p no:cacheprovider $T > gpurun_out/pytest_$TAG.log 2>&1; echo "rc=$?" >> gpurun_out/pytest_$TAG.log; fi
+if [ $# -gt 0 ]; then bash tools/ab.sh $TAG "$@"; fi
+echo done

@@ -13,4 +13,4 @@ st = info["last"]
 print(json.dumps({"cfg": cfg, "ratio": ratio, "ms_per_job": ms / 3, "passes": st["passes"],
                   "insert_ms": st["t_insert_ms"], "reprobe_ms": st["t_reprobe_ms"], "compact_ms": st["t_compact_ms"],
                   "evict_ms": st["t_evict_ms"], "post": st["postponed_per_pass"],
-                  "insert_ms_per_pass": [round(x, 3) for x in st["t_insert_ms_per_pass"]]}))
+                  "insert_ms_per_pass": [round(x, 3) for x in st["t_insert_ms_per_pass"]], "p1_ms": info["p1_ms"] / 3}))
