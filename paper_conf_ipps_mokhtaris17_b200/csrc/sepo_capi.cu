@@ -940,14 +940,16 @@ int export_group(sepo_table* t) {
                     memcpy(&birth, base + off + KEY_OFF + ((klen + 7) & ~7u) + 8, 4);
                     uint64_t poolo = ((uint64_t)pages[i].page << t->page_shift) + off;
                     tk[w].push_back({base + off + KEY_OFF, klen, ((uint64_t)birth << 40) | ((poolo >> 3) + 1)});
-                } else if (kind == K_VCHUNK) {
-                    uint32_t fill, cap, cvw;
+                } else if (kind == K_VCHUNK || kind == K_VCHUNKV) {
+                    // 16-byte header: size | kind, fill, owner; the capacity follows from the size
+                    // (fixed-width slots of the table's fixed_val_width, or bytes of variable items)
+                    uint32_t fill;
                     uint64_t owner;
                     memcpy(&fill, base + off + 4, 4);
                     memcpy(&owner, base + off + 8, 8);
-                    memcpy(&cap, base + off + 24, 4);
-                    memcpy(&cvw, base + off + 28, 4);
-                    cap &= ~CHUNK_PRIVATE;
+                    const uint32_t cvw = kind == K_VCHUNK ? t->opts.fixed_val_width : 0u;
+                    const uint32_t cap = (sz - CHUNK_HDR) / (cvw ? cvw : 1u);
+                    fill &= ~CHUNK_PRIVATE;
                     ChunkRec cr{base + off + CHUNK_HDR, std::min(fill, cap), owner, cvw, 0, 0};
                     if (cvw) {
                         cr.nitems = cr.units;

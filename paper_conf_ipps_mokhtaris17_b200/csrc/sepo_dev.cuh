@@ -21,7 +21,9 @@
 //   COMBINE entry       : hdr | next u32 | tag u32 | klen u32 | key[pad8] | value u64
 //   GROUP key entry     : hdr | next u32 | tag u32 | klen u32 | key[pad8] | list_head u64 |
 //                                      birth_gen u32 | pad u32
-//   GROUP value chunk: hdr | fill u32 | owner u64 | next u64 | cap u32 | vw u32 | values
+//   GROUP value chunk: hdr | fill u32 | owner u64 | values  (16-byte header; the
+//                                      capacity follows from the size, the value format from the kind:
+//                                      K_VCHUNK fixed-width slots, K_VCHUNKV {u32 length, bytes} items)
 //   filler                            : hdr (size of the gap)
 #pragma once
 #include <cstdint>
@@ -30,11 +32,13 @@
 namespace sepo {
 
 constexpr uint32_t FULLMASK = 0xffffffffu;
-enum : uint32_t { K_FREE = 0, K_COMBINE = 1, K_FILL = 2, K_DEAD = 3, K_GKEY = 4, K_VCHUNK = 5, K_BASIC = 6 };
+enum : uint32_t { K_FREE = 0, K_COMBINE = 1, K_FILL = 2, K_DEAD = 3, K_GKEY = 4, K_VCHUNK = 5, K_BASIC = 6,
+                  K_VCHUNKV = 7 };
 constexpr uint32_t KIND_MASK = 7u;
 constexpr uint32_t KEY_OFF = 16;     // key bytes start here in combine and group key entries
-constexpr uint32_t CHUNK_HDR = 32;   // value chunk header
-constexpr uint32_t CHUNK_PRIVATE = 0x80000000u;  // cap flag: slots handed out by one CTA (hot key)
+constexpr uint32_t CHUNK_HDR = 16;   // value chunk header: size | kind, fill, owner
+constexpr uint32_t CHUNK_PRIVATE = 0x80000000u;  // fill flag: slots handed out by one CTA (hot key) — a
+                                                 // reserving thread sees the chunk as full
 constexpr uint32_t NOPAGE = 0xfffffffeu, FULLPAGE = 0xffffffffu;
 constexpr uint32_t PAGE_ENTRY = 1, PAGE_VALUE = 2;
 

@@ -97,22 +97,16 @@ __device__ __forceinline__ uint32_t item_units(uint32_t vw, uint32_t vlen) { ret
 // Sized by the demand rather than grown from the previous chunk: many CTAs may find a key's head
 // chunk full at once and each installs a chunk, so large geometric chunks would mostly stay empty
 // (measured: 8x slot over-allocation on C4 with doubling).
-#ifndef SEPO_CHUNK_GROW
-#define SEPO_CHUNK_GROW 0   // > 0: a key's next shared chunk gets min(2 x the full one's capacity, this many slots)
-#endif
-__device__ __forceinline__ uint32_t chunk_cap(const Dev& d, uint32_t need, uint32_t prev, uint32_t vw) {
+__device__ __forceinline__ uint32_t chunk_cap(const Dev& d, uint32_t need, uint32_t vw) {
     const uint32_t unit = vw ? vw : 1u;
     const uint32_t maxcap = (d.page_bytes / 4 - CHUNK_HDR) / unit;
     uint32_t c = max(vw ? 8u : 64u, 2u * need);
-#if SEPO_CHUNK_GROW
-    if (vw) c = max(c, min(2u * (prev & ~CHUNK_PRIVATE), (uint32_t)SEPO_CHUNK_GROW));
-#else
-    (void)prev;
-#endif
     c = min(c, max(maxcap, need));
     return min(c, (d.page_bytes - CHUNK_HDR) / unit);
 }
 __device__ __forceinline__ uint32_t chunk_bytes(uint32_t cap, uint32_t vw) { return align16(CHUNK_HDR + cap * (vw ? vw : 1u)); }
+// capacity (units) of a chunk of `size` bytes: every unit the 16-byte aligned record holds
+__device__ __forceinline__ uint32_t chunk_capacity(uint32_t size, uint32_t vw) { return (size - CHUNK_HDR) / (vw ? vw : 1u); }
 __device__ __forceinline__ uint64_t vref_of(const Dev& d, uint64_t off) { return ((uint64_t)d.gen << 40) | (uint64_t)off_ref(off); }
 __device__ __forceinline__ bool vref_resident(const Dev& d, uint64_t vref) { return vref != 0 && (uint32_t)(vref >> 40) == d.gen; }
 __device__ __forceinline__ uint8_t* vref_ptr(const Dev& d, uint64_t vref) { return ref_ptr(d, (uint32_t)vref); }
@@ -124,44 +118,36 @@ __device__ __forceinline__ uint64_t owner_of(const Dev& d, uint8_t* e) {
 __device__ __forceinline__ unsigned long long* list_head(uint8_t* e) {
     return reinterpret_cast<unsigned long long*>(entry_val(e, ldcg32(e + 12)));
 }
-__device__ __forceinline__ void init_chunk(uint8_t* c, uint32_t cap, uint32_t vwslot, uint32_t fill, uint64_t owner,
-                                           uint64_t next) {
-    *reinterpret_cast<uint32_t*>(c) = chunk_bytes(cap, vwslot) | K_VCHUNK;
+// a chunk of `cap` units: fill (CHUNK_PRIVATE for a CTA's private chunk) and owner key identity
+__device__ __forceinline__ void init_chunk(uint8_t* c, uint32_t cap, uint32_t vwslot, uint32_t fill, uint64_t owner) {
+    *reinterpret_cast<uint32_t*>(c) = chunk_bytes(cap, vwslot) | (vwslot ? K_VCHUNK : K_VCHUNKV);
     *reinterpret_cast<uint32_t*>(c + 4) = fill;
     *reinterpret_cast<unsigned long long*>(c + 8) = owner;
-    *reinterpret_cast<unsigned long long*>(c + 16) = next;
-    *reinterpret_cast<uint32_t*>(c + 24) = cap;
-    *reinterpret_cast<uint32_t*>(c + 28) = vwslot;
 }
 // push chunk `cref` (header already written) onto the list head of key entry e: one release-
-// exchange, then the chunk's `next` takes the previous head. Device code never follows `next`
-// (only the host export does, after the kernel), so a CAS retry loop — which serialises badly when
-// many CTAs push onto a hot key at once — is not needed.
-__device__ __forceinline__ void push_chunk(uint8_t* e, uint8_t* c, uint64_t cref, uint64_t observed) {
-    (void)observed;
+// exchange. The list is never walked (device code only reserves in the head chunk; the host export
+// attaches chunks to keys by their owner identity), so chunks keep no `next` link and no CAS retry
+// loop serialises the CTAs that push onto a hot key at once.
+__device__ __forceinline__ void push_chunk(uint8_t* e, uint64_t cref) {
     unsigned long long* head = list_head(e);
     unsigned long long old;
     asm volatile("atom.release.gpu.global.exch.b64 %0, [%1], %2;" : "=l"(old) : "l"(head), "l"(cref) : "memory");
-    *reinterpret_cast<unsigned long long*>(c + 16) = old;
+    (void)old;
 }
-// Reserve `units` (1 slot, or an item's bytes) in the resident head chunk of key entry e.
-// Returns 1 and the first unit in *base if the whole reservation fits, else 0. A reservation that
-// crosses the end of a variable-value chunk closes the chunk's tail with ITEM_END.
-__device__ __forceinline__ uint32_t reserve_head(const Dev& d, uint8_t* e, uint32_t units, uint64_t* cref, uint32_t* base,
-                                                 uint64_t* head_out, uint32_t* prev_cap) {
-    uint64_t h = ld_relaxed_u64(list_head(e));
-    *head_out = h;
-    *prev_cap = 0;
+// Reserve `units` (1 slot, or an item's bytes) in the resident head chunk of key entry e (vw: the
+// batch's value format). Returns 1 and the first unit in *base if the whole reservation fits, else 0.
+// A reservation that crosses the end of a variable-value chunk closes the chunk's tail with ITEM_END.
+__device__ __forceinline__ uint32_t reserve_head(const Dev& d, uint8_t* e, uint32_t units, uint32_t vw, uint64_t* cref,
+                                                 uint32_t* base) {
+    const uint64_t h = ld_relaxed_u64(list_head(e));
     *cref = 0;
     if (!vref_resident(d, h)) return 0;
     uint8_t* c = vref_ptr(d, h);
-    uint32_t cap = ldcg32(c + 24);
-    if (cap & CHUNK_PRIVATE) return 0;  // a CTA's private chunk: its units are handed out in smem
-    *prev_cap = cap;
-    if (ldcg32(c + 4) >= cap) return 0;
-    uint32_t old = atomicAdd(reinterpret_cast<unsigned int*>(c + 4), units);
+    const uint32_t cap = chunk_capacity(ldcg32(c) & ~KIND_MASK, vw);
+    if (ldcg32(c + 4) >= cap) return 0;  // full (or private: the fill carries CHUNK_PRIVATE)
+    const uint32_t old = atomicAdd(reinterpret_cast<unsigned int*>(c + 4), units);
     if (old + units > cap) {
-        if (old + 4 <= cap && ldcg32(c + 28) == 0) *reinterpret_cast<uint32_t*>(c + CHUNK_HDR + old) = ITEM_END;
+        if (old + 4 <= cap && vw == 0) *reinterpret_cast<uint32_t*>(c + CHUNK_HDR + old) = ITEM_END;
         return 0;
     }
     *cref = h;
@@ -1317,6 +1303,15 @@ __device__ __forceinline__ void offsets(const Batch& b, uint64_t i, bool ok, uin
     if (IN == IN_CSR) {
         s = ok ? ld_tail64(b.ko + i) : 0ull;
         e = ok ? ld_tail64(b.ko + i + 1) : 0ull;
+    } else if (IN == IN_IDX) {  // re-issue by index: record i of the batch is record idx[i]
+        const uint64_t j = ok ? ld_in64(b.idx + i) : 0ull;
+        if (b.ko) {
+            s = ok ? ld_in64(b.ko + j) : 0ull;
+            e = ok ? ld_in64(b.ko + j + 1) : 0ull;
+        } else {
+            s = j * b.kw;
+            e = ok ? s + b.kw : s;
+        }
     } else {
         s = i * b.kw;
         e = ok ? s + b.kw : s;
@@ -1755,9 +1750,8 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
                     if (coff != ~0ull) {
                         uint8_t* c = d.pool + coff;
                         uint8_t* ke = ref_ptr(d, S.ref[pos]);
-                        init_chunk(c, PC_CAP, vw, 0, owner_of(d, ke), 0ull);
-                        *reinterpret_cast<uint32_t*>(c + 24) = PC_CAP | CHUNK_PRIVATE;
-                        push_chunk(ke, c, vref_of(d, coff), ld_relaxed_u64(list_head(ke)));
+                        init_chunk(c, PC_CAP, vw, CHUNK_PRIVATE, owner_of(d, ke));
+                        push_chunk(ke, vref_of(d, coff));
                         nref = off_ref(coff);
                         const uint32_t rest = vw ? f0 + tot - PC_CAP : 0u;  // fixed: the overflow goes here
                         atomicExch(&S.pw[pos], ((unsigned long long)nref << 32) | rest);
@@ -1782,20 +1776,18 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
         if (valid && !done && pos < 0) e = chain_find_w(d, head, 0, tag, len, w0, w1, tail);
         bool need_key = valid && !done && e == nullptr;
         bool need_chunk = valid && !done;
-        uint32_t prev_cap = 0;
         if (valid && !done && e) {
-            uint64_t cr = 0, lh = 0;
-            uint32_t base = 0, pc = 0;
-            if (reserve_head(d, e, units, &cr, &base, &lh, &pc)) {
+            uint64_t cr = 0;
+            uint32_t base = 0;
+            if (reserve_head(d, e, units, vw, &cr, &base)) {
                 put_value(b, i, vref_ptr(d, cr), base);
                 done = true;
                 need_chunk = false;
             }
-            prev_cap = pc;
         }
         uint32_t res = R_OK;
         const uint32_t ksize = gkey_size(len);
-        const uint32_t ccap = chunk_cap(d, units, prev_cap, vw);
+        const uint32_t ccap = chunk_cap(d, units, vw);
         const uint32_t csize = chunk_bytes(ccap, vw);
         if ((need_key && (len > 65535u - 64u || ksize > PB)) || (need_chunk && CHUNK_HDR + units * (vw ? vw : 1u) > PB)) {
             need_key = false; need_chunk = false; res = R_TOOLARGE;
@@ -1847,9 +1839,9 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
             }
             if (need_chunk && coff != ~0ull && e) {
                 uint8_t* c = d.pool + coff;
-                init_chunk(c, ccap, vw, units, owner_of(d, e), 0ull);
+                init_chunk(c, ccap, vw, units, owner_of(d, e));
                 put_value(b, i, c, 0);
-                push_chunk(e, c, vref_of(d, coff), ld_relaxed_u64(list_head(e)));
+                push_chunk(e, vref_of(d, coff));
                 done = true;
             }
             __syncwarp();
@@ -1870,9 +1862,9 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
             if (declined) {
                 res = R_POST;
                 if (e) {  // resident key: its value may still fit a shared head chunk
-                    uint64_t cr = 0, lh = 0;
-                    uint32_t base = 0, pc = 0;
-                    if (reserve_head(d, e, units, &cr, &base, &lh, &pc)) {
+                    uint64_t cr = 0;
+                    uint32_t base = 0;
+                    if (reserve_head(d, e, units, vw, &cr, &base)) {
                         put_value(b, i, vref_ptr(d, cr), base);
                         res = R_OK;
                     } else {
@@ -1908,6 +1900,335 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
         if (S.post) atomicAdd(&d.ctrl->postponed, S.post);
         if (S.toolarge) atomicAdd(&d.ctrl->toolarge, S.toolarge);
         if (S.dead) atomicAdd(&d.ctrl->dead_bytes, S.dead);
+    }
+}
+
+// ================================================================ GROUP insert, lean (a1..a7)
+// The multi-valued method for fixed-width values of 1, 2, 4 or 8 bytes (C4: u32 doc
+// ids), on the lean input path (per-warp contiguous group streams; CSR, fixed-width or index
+// batches). Hot keys append into CTA-private value chunks (one shared atomic per warp per key, as
+// insert_group_stream_kernel); every other record goes to a per-warp miss queue and is resolved 32
+// at a time with every lane busy: directory word, chain walk to the key entry, one reservation in
+// the key's head chunk and the value store; keys without an entry and full head chunks take the
+// allocation path (announcement protocol, R15); a resident key whose value cannot be stored marks
+// its key page retained (pending key).
+namespace grp2 {
+constexpr int THREADS = 1024, WARPS = THREADS / 32, QCAP = 64;
+constexpr int DS = 4096, NK = 1024;  // hot slots / hot keys
+constexpr uint32_t PC_CAP = 256;     // slots of a private chunk
+struct Smem {
+    uint32_t tags[DS];
+    ulonglong2 kw[NK];
+    uint32_t ref[NK];
+    unsigned long long pw[NK];  // private chunk word: chunk ref << 32 | fill (ref 0: none)
+    struct Queue {
+        ulonglong2 k[QCAP];          // first 16 key bytes
+        ulonglong2 hs[QCAP];         // hash, key offset | length << 40 | lane << 59
+        unsigned long long v[QCAP];  // value
+        uint32_t g[QCAP];            // group
+    } q[WARPS];
+    stream::CtaState cs;
+};
+static_assert(sizeof(Smem) <= 232448, "grp2 kernel shared memory > 227 KB");
+// value v (vw bytes LE) into slot `at` of chunk c
+__device__ __forceinline__ void store_slot(uint8_t* c, uint32_t at, uint32_t vw, uint64_t v) {
+    uint8_t* dst = c + CHUNK_HDR + (uint64_t)at * vw;
+    if (vw == 4) *reinterpret_cast<uint32_t*>(dst) = (uint32_t)v;
+    else if (vw == 8) *reinterpret_cast<unsigned long long*>(dst) = v;
+    else if (vw == 2) *reinterpret_cast<uint16_t*>(dst) = (uint16_t)v;
+    else *dst = (uint8_t)v;
+}
+}  // namespace grp2
+
+// Resolve up to 32 queued GROUP records, one per lane (a3..a7).
+__device__ __forceinline__ void grp2_resolve(const Dev& d, const Batch& b, grp2::Smem& S, grp2::Smem::Queue& Q, uint32_t qhead,
+                                             uint32_t cnt, bool inj, bool& w_full, bool& w_quiet) {
+    const uint32_t lane = lane_id();
+    const uint32_t PB = d.page_bytes, vw = b.vw;
+    const bool act = lane < cnt;
+    const uint32_t k = (qhead + lane) & (grp2::QCAP - 1);
+    uint64_t w0 = 0, w1 = 0, h = 0, s = 0, v = 0;
+    uint32_t g = 0, len = 0, gl = 0;
+    if (act) {
+        const ulonglong2 kk = Q.k[k], hs = Q.hs[k];
+        w0 = kk.x; w1 = kk.y; h = hs.x;
+        s = hs.y & lean::S_MASK;
+        len = (uint32_t)(hs.y >> 40) & lean::LEN_MAX;
+        gl = (uint32_t)(hs.y >> 59);
+        g = Q.g[k];
+        v = Q.v[k];
+    }
+    const uint8_t* tail = b.keys + s + 16;
+    const uint32_t bkt = bucket_of(h, d.n_buckets), tag = tag_of(h);
+    const uint32_t head = act ? ld_dir(d.dir + bkt) : 0u;
+    uint8_t* e = act ? chain_find_w(d, head, 0, tag, len, w0, w1, tail) : nullptr;
+    bool done = false;
+    if (e) {  // resident key: one reservation in its head chunk
+        uint64_t cr = 0;
+        uint32_t base = 0;
+        if (reserve_head(d, e, 1u, vw, &cr, &base)) {
+            grp2::store_slot(vref_ptr(d, cr), base, vw, v);
+            done = true;
+        }
+    }
+    uint32_t res = R_OK;
+    bool need_key = act && !e, need_chunk = act && !done;
+    const uint32_t ksize = gkey_size(len);
+    const uint32_t ccap = chunk_cap(d, 1u, vw), csize = chunk_bytes(ccap, vw);
+    if (need_key && (len > 65535u - 64u || ksize > PB)) { need_key = false; need_chunk = false; res = R_TOOLARGE; }
+    if (inj && need_key && inject_fail(d, h, (uint64_t)g * 32 + gl)) { need_key = false; need_chunk = false; res = R_POST; }
+    // ---- allocation (a5) + link (a6) under the announcement protocol (R15), as resolve_core
+    if (__any_sync(FULLMASK, need_chunk)) {
+        if (!w_full) {
+            unsigned long long f0 = 0;
+            if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
+            if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
+        }
+        if (!w_full) {
+            unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
+            unsigned long long a = 0;
+            if (lane == 0) a = atomicAdd(my_ann, 1ull);
+            a = __shfl_sync(FULLMASK, a, 0);
+            uint64_t koff = ~0ull, coff = ~0ull;
+            if (a & ANN_FULL) {
+                w_full = true;
+            } else {
+                koff = warp_alloc(d, &S.cs.cur[0], need_key, ksize, (uint8_t)PAGE_ENTRY);
+                const bool wc = need_chunk && (!need_key || koff != ~0ull);
+                coff = warp_alloc(d, &S.cs.cur[1], wc, csize, (uint8_t)PAGE_VALUE);
+            }
+            if (need_key && koff != ~0ull) {  // new key entry, linked even if its chunk failed (pending)
+                uint8_t* ne = d.pool + koff;
+                *reinterpret_cast<uint4*>(ne) = make_uint4(ksize | K_GKEY, head, tag, len);
+                if (len > 0) *reinterpret_cast<unsigned long long*>(ne + KEY_OFF) = w0;
+                if (len > 8) *reinterpret_cast<unsigned long long*>(ne + KEY_OFF + 8) = w1;
+                if (len > 16) store_key(ne + KEY_OFF + 16, tail, len - 16);
+                *reinterpret_cast<unsigned long long*>(entry_val(ne, len)) = 0ull;
+                *reinterpret_cast<uint32_t*>(entry_val(ne, len) + 8) = d.gen;
+                *reinterpret_cast<uint32_t*>(entry_val(ne, len) + 12) = 0u;
+                const uint32_t me = off_ref(koff);
+                e = ne;
+                uint32_t hd = head;
+                while (true) {  // lock-free head insertion
+                    const uint32_t old = cas_release(d.dir + bkt, hd, me);
+                    if (old == hd) break;
+                    uint8_t* w = chain_find_w(d, old, hd, tag, len, w0, w1, tail);
+                    if (w) {  // linked meanwhile: retire ours
+                        *reinterpret_cast<uint32_t*>(ne) = ksize | K_DEAD;
+                        atomicAdd(&S.cs.dead, (unsigned long long)ksize);
+                        e = w;
+                        break;
+                    }
+                    hd = old;
+                    *reinterpret_cast<uint32_t*>(ne + 4) = hd;
+                }
+            }
+            if (need_chunk && coff != ~0ull && e) {
+                uint8_t* c = d.pool + coff;
+                init_chunk(c, ccap, vw, 1u, owner_of(d, e));
+                grp2::store_slot(c, 0, vw, v);
+                push_chunk(e, vref_of(d, coff));
+                done = true;
+            }
+            __syncwarp();
+            if (lane == 0) add_release64(my_ann, ~0ull);  // withdraw, after every link above
+        }
+    }
+    // ---- declines (a7): certified for new keys; a resident key with its value left over is pending
+    const bool declined = act && !done && res == R_OK;
+    if (__any_sync(FULLMASK, declined)) {
+        w_full = true;
+        if (!w_quiet) {
+            if (lane == 0)
+                for (uint32_t c = 0; c < d.n_slots; ++c)
+                    while (ld_acquire_u64(d.ann + (uint64_t)c * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
+            __syncwarp();
+            w_quiet = true;
+            if (declined && !e) e = chain_find_w(d, ld_dir(d.dir + bkt), 0, tag, len, w0, w1, tail);
+        }
+        if (declined) {
+            res = R_POST;
+            if (e) {  // resident key: its value may still fit the head chunk
+                uint64_t cr = 0;
+                uint32_t base = 0;
+                if (reserve_head(d, e, 1u, vw, &cr, &base)) {
+                    grp2::store_slot(vref_ptr(d, cr), base, vw, v);
+                    res = R_OK;
+                } else {
+                    d.retain[(uint32_t)((uint64_t)(e - d.pool) >> d.page_shift)] = 1;  // pending key
+                }
+            }
+        }
+    }
+    const bool out = act && res != R_OK;
+    const unsigned pend = __ballot_sync(FULLMASK, out);
+    if (pend) {
+        const unsigned tl = __ballot_sync(FULLMASK, act && res == R_TOOLARGE);
+        const unsigned pkb = __reduce_add_sync(FULLMASK, out ? len : 0u);
+        if (lane == 0) {
+            const uint32_t w = (threadIdx.x >> 5) & 31u;
+            S.cs.wpost[w] += (unsigned long long)__popc(pend);
+            S.cs.wpkb[w] += (unsigned long long)pkb;
+            if (tl) atomicAdd(&S.cs.toolarge, (unsigned long long)__popc(tl));
+        }
+        if (out && b.bitmap) atomicOr(b.bitmap + g, 1u << gl);
+    }
+}
+
+template <int IN>
+__global__ void __launch_bounds__(grp2::THREADS, 1) insert_group2_kernel(Dev d, Batch b, const hot::Entry* hl,
+                                                                           const unsigned int* n_hot, const InCtx c) {
+    using namespace grp2;
+    extern __shared__ __align__(16) uint8_t smem_raw[];
+    grp2::Smem& S = *reinterpret_cast<grp2::Smem*>(smem_raw);
+    const uint32_t tid = threadIdx.x, lane = lane_id(), wid = tid >> 5;
+    const uint32_t vw = b.vw;
+    if (tid == 0) {
+        S.cs.cur[0] = d.cursors[2 * blockIdx.x];
+        S.cs.cur[1] = d.cursors[2 * blockIdx.x + 1];
+        S.cs.post = 0; S.cs.toolarge = 0; S.cs.dead = 0; S.cs.pkb = 0;
+    }
+    if (tid < 32) { S.cs.wpost[tid] = 0; S.cs.wpkb[tid] = 0; }
+    load_hot_direct<DS, NK>(S.tags, S.kw, S.ref, S.pw, hl, n_hot);
+    for (int p = tid; p < NK; p += THREADS) S.pw[p] = PC_CAP;  // no private chunk yet: the first hits install one
+    __syncthreads();
+    const bool have_hot = hl != nullptr && *n_hot > 0;
+    const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
+    const uint32_t pc_bytes = chunk_bytes(PC_CAP, vw);
+    Smem::Queue& Q = S.q[wid];
+    uint32_t qhead = 0, qtail = 0;
+    bool w_full = false, w_quiet = false;
+    const uint64_t gw = (uint64_t)blockIdx.x * WARPS + wid;
+    uint32_t g = (uint32_t)((uint64_t)c.ngroups * gw / c.nw);
+    const uint32_t gend = (uint32_t)((uint64_t)c.ngroups * (gw + 1) / c.nw);
+    auto cnt_of = [&](uint32_t x) -> uint32_t { return x < gend ? (x + 1 == c.ngroups ? c.tail : 32u) : 0u; };
+    uint64_t s_c, e_c, s_n, e_n, v_c = 0, x0, x1, x2;
+    {
+        const bool ok = lane < cnt_of(g);
+        lean::offsets<IN>(b, (uint64_t)g * 32 + lane, ok, s_c, e_c);
+        if (ok) v_c = rec_value(b, (uint64_t)g * 32 + lane);
+        lean::key_words(b.keys, s_c, (uint32_t)(e_c - s_c), x0, x1, x2);
+        lean::offsets<IN>(b, (uint64_t)(g + 1) * 32 + lane, lane < cnt_of(g + 1), s_n, e_n);
+    }
+    for (; g < gend; ++g) {
+        // ---- issue ahead: key words + value of g + 1, offsets of g + 2
+        uint64_t y0, y1, y2, v_n = 0;
+        lean::key_words(b.keys, s_n, (uint32_t)(e_n - s_n), y0, y1, y2);
+        if (lane < cnt_of(g + 1)) v_n = rec_value(b, (uint64_t)(g + 1) * 32 + lane);
+        uint64_t s_nn, e_nn;
+        lean::offsets<IN>(b, (uint64_t)(g + 2) * 32 + lane, lane < cnt_of(g + 2), s_nn, e_nn);
+        // ---- group g: first 16 key bytes + hash (a1)
+        const bool valid = lane < cnt_of(g);
+        const uint64_t s = s_c;
+        const uint32_t len = (uint32_t)(e_c - s_c);
+        uint64_t w0, w1;
+        lean::assemble16(x0, x1, x2, (uint32_t)(reinterpret_cast<uintptr_t>(b.keys + s) & 7u), len, w0, w1);
+        const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
+        const uint64_t v = v_c;
+        // ---- hot set probe (a2)
+        int pos = -1;
+        if (have_hot) {
+            const uint32_t f = stream::dfp(h, len);
+            const uint32_t t1 = S.tags[(uint32_t)(h >> 3) & (DS - 1)], t2 = S.tags[(uint32_t)(h >> 17) & (DS - 1)];
+            constexpr uint32_t IM = (1u << stream::IDXB) - 1u;
+            const bool m1 = (t1 & ~IM) == f, m2 = (t2 & ~IM) == f;
+            const uint32_t p = (m1 ? t1 : t2) & IM;
+            if (valid && (m1 || m2)) {
+                const ulonglong2 kk = S.kw[p];
+                bool eq = kk.x == w0 && kk.y == w1;
+                if (len > 16) {
+                    const uint8_t* e = ref_ptr(d, S.ref[p]);
+                    eq = eq && ldcg32(e + 12) == len && entry_key_eq(e + KEY_OFF + 16, b.keys + s + 16, len - 16);
+                }
+                if (eq) pos = (int)p;
+            }
+        }
+        // ---- hot keys: the warp's values of a key reserved in its private chunk (one shared atomic)
+        bool done = false;
+        const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
+        if (hm) {
+            const unsigned grp = __match_any_sync(FULLMASK, pos >= 0 ? (unsigned)pos : (0x10000u | lane)) & hm;
+            const uint32_t leader = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
+            const uint32_t excl = __popc(grp & lanemask_lt()), tot = __popc(grp);
+            unsigned long long old = 0;
+            if (pos >= 0 && lane == leader) old = atomicAdd(&S.pw[pos], (unsigned long long)tot);
+            old = __shfl_sync(FULLMASK, old, leader);
+            const uint32_t cref = (uint32_t)(old >> 32), f0 = (uint32_t)old;
+            const bool cross = pos >= 0 && f0 <= PC_CAP && f0 + tot > PC_CAP;  // the warp that installs the next chunk
+            const bool fits_old = pos >= 0 && cref && f0 + excl < PC_CAP;
+            const bool want = cross && lane == leader && !w_full;
+            uint32_t nref = 0;
+            if (__any_sync(FULLMASK, want)) {
+                unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
+                unsigned long long a = 0;
+                if (lane == 0) a = atomicAdd(my_ann, 1ull);
+                a = __shfl_sync(FULLMASK, a, 0);
+                uint64_t coff = ~0ull;
+                if (a & ANN_FULL) w_full = true;
+                else coff = warp_alloc(d, &S.cs.cur[1], want, pc_bytes, (uint8_t)PAGE_VALUE);
+                if (want) {
+                    if (cref) *reinterpret_cast<uint32_t*>(ref_ptr(d, cref) + 4) = PC_CAP;  // the old chunk is full
+                    if (coff != ~0ull) {
+                        uint8_t* ch = d.pool + coff;
+                        uint8_t* ke = ref_ptr(d, S.ref[pos]);
+                        init_chunk(ch, PC_CAP, vw, CHUNK_PRIVATE, owner_of(d, ke));
+                        push_chunk(ke, vref_of(d, coff));
+                        nref = off_ref(coff);
+                        atomicExch(&S.pw[pos], ((unsigned long long)nref << 32) | (f0 + tot - PC_CAP));
+                    } else {
+                        atomicExch(&S.pw[pos], (unsigned long long)PC_CAP << 1);  // no chunk: hits go global
+                    }
+                }
+                __syncwarp();
+                if (lane == 0) add_release64(my_ann, ~0ull);
+            } else if (cross && lane == leader) {  // (pool known full: no private chunk any more)
+                if (cref) *reinterpret_cast<uint32_t*>(ref_ptr(d, cref) + 4) = PC_CAP;
+                atomicExch(&S.pw[pos], (unsigned long long)PC_CAP << 1);
+            }
+            nref = __shfl_sync(FULLMASK, nref, leader);
+            if (pos >= 0) {
+                const uint32_t at = f0 + excl;
+                if (fits_old) { store_slot(ref_ptr(d, cref), at, vw, v); done = true; }
+                else if (cross && nref && at >= PC_CAP) { store_slot(ref_ptr(d, nref), at - PC_CAP, vw, v); done = true; }
+            }
+        }
+        // ---- everything else: the warp's miss queue, resolved 32 at a time (a3..a7)
+        const bool miss = valid && !done;
+        const unsigned mm = __ballot_sync(FULLMASK, miss);
+        if (lane == 0 && b.bitmap) b.bitmap[g] = 0u;
+        if (miss) {
+            const uint32_t k = (qtail + __popc(mm & lanemask_lt())) & (QCAP - 1);
+            Q.k[k] = make_ulonglong2(w0, w1);
+            Q.hs[k] = make_ulonglong2(h, s | ((uint64_t)min(len, lean::LEN_MAX) << 40) | ((uint64_t)lane << 59));
+            Q.g[k] = g;
+            Q.v[k] = v;
+        }
+        qtail += __popc(mm);
+        __syncwarp();
+        if (qtail - qhead >= 32) {
+            grp2_resolve(d, b, S, Q, qhead, 32, inj, w_full, w_quiet);
+            qhead += 32;
+            __syncwarp();
+        }
+        s_c = s_n; e_c = e_n; v_c = v_n; x0 = y0; x1 = y1; x2 = y2;
+        s_n = s_nn; e_n = e_nn;
+    }
+    if (qtail != qhead) grp2_resolve(d, b, S, Q, qhead, qtail - qhead, inj, w_full, w_quiet);
+    __syncthreads();
+    // final fill of every private chunk still open (clears CHUNK_PRIVATE)
+    for (int p = tid; p < NK; p += THREADS) {
+        const unsigned long long w = S.pw[p];
+        const uint32_t cref = (uint32_t)(w >> 32);
+        if (cref) *reinterpret_cast<uint32_t*>(ref_ptr(d, cref) + 4) = min((uint32_t)w, PC_CAP);
+    }
+    if (tid == 0) {
+        d.cursors[2 * blockIdx.x] = S.cs.cur[0];
+        d.cursors[2 * blockIdx.x + 1] = S.cs.cur[1];
+        for (uint32_t w = 0; w < (uint32_t)WARPS; ++w) { S.cs.post += S.cs.wpost[w]; S.cs.pkb += S.cs.wpkb[w]; }
+        if (S.cs.post) atomicAdd(&d.ctrl->postponed, S.cs.post);
+        if (S.cs.toolarge) atomicAdd(&d.ctrl->toolarge, S.cs.toolarge);
+        if (S.cs.dead) atomicAdd(&d.ctrl->dead_bytes, S.cs.dead);
+        if (S.cs.pkb) atomicAdd(&d.ctrl->kept_key_bytes, S.cs.pkb);
     }
 }
 
@@ -1961,13 +2282,13 @@ __global__ void __launch_bounds__(RP_THREADS) reprobe_kernel(Dev d, Batch b, uns
                         rec_val_span(b, i, vs, vl);
                         const uint32_t cvw = b.vo ? 0u : b.vw;
                         units = item_units(cvw, vl);
-                        uint64_t cref = 0, lhead = 0;
-                        uint32_t base = 0, pcap = 0;
-                        if (reserve_head(d, e, units, &cref, &base, &lhead, &pcap)) {
+                        uint64_t cref = 0;
+                        uint32_t base = 0;
+                        if (reserve_head(d, e, units, cvw, &cref, &base)) {
                             put_value(b, i, vref_ptr(d, cref), base);
                             still = false;
                         } else {
-                            want_cap = chunk_cap(d, units, pcap, cvw);
+                            want_cap = chunk_cap(d, units, cvw);
                         }
                     }
                 }
@@ -1979,9 +2300,9 @@ __global__ void __launch_bounds__(RP_THREADS) reprobe_kernel(Dev d, Batch b, uns
                     if (want) {
                         if (coff != ~0ull) {
                             uint8_t* c = d.pool + coff;
-                            init_chunk(c, want_cap, cvw, units, owner_of(d, e), 0ull);
+                            init_chunk(c, want_cap, cvw, units, owner_of(d, e));
                             put_value(b, i, c, 0);
-                            push_chunk(e, c, vref_of(d, coff), ld_relaxed_u64(list_head(e)));
+                            push_chunk(e, vref_of(d, coff));
                             still = false;
                         } else {
                             // resident key with values still pending: keep its key page
@@ -3251,6 +3572,27 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             hl = list;
             nh = n_out;
             if (hot_built) *hot_built = true;
+        }
+        const char* g2 = getenv("SEPO_GROUP2");  // 0: insert_group_stream_kernel for every GROUP batch
+        if (!(g2 && g2[0] == '0') && !b.vo && (b.vw == 1 || b.vw == 2 || b.vw == 4 || b.vw == 8)) {
+            static bool attr2 = false;
+            if (!attr2) {
+                const int s2 = (int)sizeof(grp2::Smem);
+                cudaFuncSetAttribute(insert_group2_kernel<IN_CSR>, cudaFuncAttributeMaxDynamicSharedMemorySize, s2);
+                cudaFuncSetAttribute(insert_group2_kernel<IN_FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, s2);
+                cudaFuncSetAttribute(insert_group2_kernel<IN_IDX>, cudaFuncAttributeMaxDynamicSharedMemorySize, s2);
+                attr2 = true;
+            }
+            InCtx c{};
+            c.ngroups = (uint32_t)((b.n + 31) / 32);
+            c.tail = (uint32_t)(b.n - (uint64_t)(c.ngroups ? c.ngroups - 1 : 0) * 32);
+            c.nw = (uint32_t)grid * grp2::WARPS;
+            const int in = b.idx ? IN_IDX : (b.ko ? IN_CSR : IN_FIXED);
+            const size_t sm2 = sizeof(grp2::Smem);
+            if (in == IN_CSR) insert_group2_kernel<IN_CSR><<<grid, grp2::THREADS, sm2, s>>>(d, b, hl, nh, c);
+            else if (in == IN_FIXED) insert_group2_kernel<IN_FIXED><<<grid, grp2::THREADS, sm2, s>>>(d, b, hl, nh, c);
+            else insert_group2_kernel<IN_IDX><<<grid, grp2::THREADS, sm2, s>>>(d, b, hl, nh, c);
+            return cudaGetLastError();
         }
         const size_t sm = sizeof(gst::Smem);
         static bool attrg = false;
