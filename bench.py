@@ -75,6 +75,7 @@ class Job:
         self.distinct = s.n_ranks
         self.nb_full = max(1 << 16, next_pow2(self.distinct))
         self._inputs = None
+        self.run_fn = None  # routed jobs: runs the SEPO job on this rank's routed records
         self.kw = {}
         import paper_conf_ipps_mokhtaris17_b200 as sepo
         self.sepo = sepo
@@ -93,6 +94,12 @@ class Job:
             self._inputs = (k, o, v)
         return self._inputs
 
+    def run_job(self, t):
+        if self.run_fn is not None:
+            return self.run_fn(t)
+        k, o, v = self.inputs()
+        return t.run(k, o, v)
+
     def csr_bytes(self):
         k, o, v = self.inputs()
         b = k.numel()
@@ -107,10 +114,10 @@ class Job:
         key = (self.cfg, self.scale, self.page_bytes)
         if key not in Job._footprint_cache:
             sepo = self.sepo
-            t = sepo.Table(sepo.budget_for(self.nb_full, self.page_bytes, max(64, (self.csr_bytes() * 2) // self.page_bytes + 64)),
+            nbytes = self.bytes_hint if self.run_fn is not None else self.csr_bytes()
+            t = sepo.Table(sepo.budget_for(self.nb_full, self.page_bytes, max(64, (nbytes * 2) // self.page_bytes + 64)),
                            self.nb_full, self.page_bytes, **self.kw)
-            k, o, v = self.inputs()
-            passes = t.run(k, o, v)
+            passes = self.run_job(t)
             assert passes == 1
             pages = t.stats()["pages_used_max"]
             t.close()
@@ -279,17 +286,20 @@ def run_reference(args):
 # ---------------------------------------------------------------- our arm
 def timed_steps(job, t, steps, stream, route_fn=None):
     import torch
-    k, o, v = job.inputs()
+    k, o, v = job.inputs() if route_fn is None else (None, None, None)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ins_ms, launches, recs_ins, kb_ins, vb_ins, p1_ms = 0.0, 0, 0, 0, 0, 0.0
     torch.cuda.synchronize()
     e0.record(stream)
     for _ in range(steps):
         if route_fn is not None:  # sharded: route this rank's slice by key owner every step
-            k, o, v = route_fn()
+            route_fn()
             launches += 2
         t.reset()
-        t.run(k, o, v)
+        if route_fn is not None:
+            job.run_fn(t)
+        else:
+            t.run(k, o, v)
         st = t.stats()
         ins_ms += st["t_insert_ms"]
         p1_ms += st["t_insert_ms_per_pass"][0]
@@ -608,20 +618,27 @@ def run_routed(args, world, rank, local):
     if fixed:
         so = None
     router = shard.Router(route_seed=0x5eed, fixed_key_width=8 if fixed else 0,
-                          fixed_val_width=job.stream.val_width if sv is not None else 0)
+                          fixed_val_width=job.stream.val_width if sv is not None else 0,
+                          # pre-combine for fixed-width pairs (C5: SURVEY §8(e) makes it mandatory for
+                          # Zipf load balance); words go as CSR (their tiles combine too little to pay
+                          # for 32-byte wire records: C2 N=1 route 91 ms CSR vs 142 ms combined)
+                          combine=job.stream.family == 2 and not args.no_combine)
+    routed = {}
 
     def route_fn():
-        return router.route(sk, so, sv)
+        routed["r"] = router.route(sk, so, sv)
+        return routed["r"]
+    job.run_fn = lambda t: shard.Router.run(t, routed["r"])
     job.distinct = max(1, job.distinct // world)  # keys per rank (sizes the directory)
-    job._inputs = route_fn()
+    route_fn()
     slice_bytes = sk.numel() + (8 * (so.numel() - 1) if so is not None else 0) + (sv.numel() if sv is not None else 0)
+    job.bytes_hint = slice_bytes
     nb, pages, F = job.table_params()
     t = job.table()
-    k, o, v = job.inputs()
     for _ in range(max(args.warmup, 3)):
         route_fn()
         t.reset()
-        t.run(*job.inputs())
+        job.run_fn(t)
     sampler = ClockSampler(local)
     dist.barrier()
     torch.cuda.synchronize()
@@ -650,9 +667,9 @@ def run_routed(args, world, rank, local):
             dk = hk.to("cuda", non_blocking=True)
             do = ho.to("cuda", non_blocking=True) if ho is not None else None
             dv = hv.to("cuda", non_blocking=True) if hv is not None else None
-            rk, ro, rv = router.route(dk, do, dv)
+            r = router.route(dk, do, dv)
             t.reset()
-            t.run(rk, ro, rv)
+            shard.Router.run(t, r)
             t.export(copy=False)
             d2h += t.stats()["bytes_evicted"]
         torch.cuda.synchronize()
@@ -673,7 +690,7 @@ def run_routed(args, world, rank, local):
                            "page_bytes": job.page_bytes, "pool_pages": pages, "passes": st["passes"],
                            "parallelism": f"key-hash sharded x{world} (sepo_partition + all-to-all, pre-combined)",
                            "l2": "inputs far larger than L2 (126 MB): no flush needed"},
-                "roofline": roofline_of(job.csr_bytes(), info["p1_ms"], args.steps, peaks(),
+                "roofline": roofline_of(slice_bytes, info["p1_ms"], args.steps, peaks(),
                                         "pass-1 insert kernel of this rank's job", {"share_of_step": info["p1_ms"] / ms}),
                 "route": router.last_stats(), "e2e": e2e, "clocks": clocks, "gpu_launches": info["launches"],
                 "cpu_baseline": None}
@@ -700,6 +717,7 @@ def main():
     ap.add_argument("--ref-records", type=int, default=120_000_000)
     ap.add_argument("--ref-seconds", type=float, default=15.0)
     ap.add_argument("--route", action="store_true", help="run the sharded (router) path even at N=1")
+    ap.add_argument("--no-combine", action="store_true", help="routed path: CSR partition without the pre-combine")
     ap.add_argument("--traffic", type=float, default=None, help="dram bytes/launch from an ncu --set full capture")
     args = ap.parse_args()
     if args.impl == "reference":

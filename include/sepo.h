@@ -258,6 +258,30 @@ int sepo_partition(const uint8_t* keys, const uint64_t* key_offsets, uint32_t fi
  * seg_rec_start[s+1]); device arrays of n_segs entries) and writes key_offsets[n] = total_bytes. */
 int sepo_shift_offsets(uint64_t* key_offsets, uint64_t n, const uint64_t* seg_rec_start, const uint64_t* seg_byte_base,
                        uint32_t n_segs, uint64_t total_bytes, void* stream);
+/* Router with pre-combine (COMBINE mode; "CTA-level pre-combine of duplicate keys
+ * into (key, partial sum)"). Partitions n records by owner like sepo_partition, but each CTA first
+ * combines the equal keys of its tile of records in shared memory (u64 wrapping sum of the values,
+ * implicit 1 when vals == NULL), and every output record is a 32-byte wire record
+ *     struct { uint64_t w0, w1;  // key bytes 0..15, little endian, zero padded
+ *              uint64_t value;   // the combined value
+ *              uint64_t len; }   // key length (0..16)
+ * Keys must be at most 16 bytes (words, u64 keys); a longer key fails the call with SEPO_E_TOOLARGE and
+ * nothing is written (route such batches with sepo_partition). Inputs (device) as sepo_partition.
+ * out_wire (device, caller-owned, out_cap records) receives part p's records at [part_counts[p],
+ * part_counts[p + 1]); part_counts (HOST, n_parts + 1) is the exclusive prefix of the per-part counts
+ * with the total last. out_wire == NULL is a sizing call (counts only). The order of records within a
+ * part is unspecified. scratch: device, sepo_route_scratch(n_parts) bytes. Synchronizes the stream.
+ * Returns the number of wire records, or < 0 (SEPO_E_NOMEM: out_cap too small; part_counts valid). */
+size_t sepo_route_scratch(uint32_t n_parts);
+int64_t sepo_route_combine(const uint8_t* keys, const uint64_t* key_offsets, uint32_t fixed_key_width, const uint8_t* vals,
+                           uint32_t fixed_val_width, uint64_t n, uint32_t n_parts, uint64_t route_seed, void* out_wire,
+                           uint64_t out_cap, uint64_t* part_counts, void* scratch, size_t scratch_bytes, void* stream);
+
+/* The whole SEPO job (as sepo_run) on n wire records (device; the records a rank received after
+ * sepo_route_combine + the exchange): key = the record's first len bytes, value = its u64. COMBINE
+ * mode only. Returns the number of passes or < 0. */
+int64_t sepo_run_wire(sepo_table* t, const void* wire, uint64_t n);
+
 const char* sepo_last_error(void);
 const char* sepo_version(void);
 

@@ -65,7 +65,7 @@ POOL_DEVICE, POOL_HOST_PINNED, POOL_MANAGED = 0, 1, 2  # sepo_create_placed (inc
 EXPORTS = ["sepo_create", "sepo_create_placed", "sepo_configure", "sepo_run_text", "sepo_lookup", "sepo_insert_batch", "sepo_reprobe", "sepo_compact", "sepo_evict",
            "sepo_export", "sepo_run", "sepo_reset", "sepo_stats_get", "sepo_last_insert_ms", "sepo_destroy",
            "sepo_last_error", "sepo_version", "sepo_budget_for", "sepo_partition_scratch", "sepo_partition",
-           "sepo_shift_offsets"]
+           "sepo_shift_offsets", "sepo_route_scratch", "sepo_route_combine", "sepo_run_wire"]
 
 
 def budget_for(n_buckets, page_bytes, pool_pages):
@@ -98,6 +98,7 @@ def lib():
         L.sepo_last_error.restype = ctypes.c_char_p
         L.sepo_version.restype = ctypes.c_char_p
         L.sepo_budget_for.argtypes = [u64, u32, u64]; L.sepo_budget_for.restype = ctypes.c_size_t
+        L.sepo_run_wire.argtypes = [vp, vp, u64]; L.sepo_run_wire.restype = i64
         _LIB = L
     return _LIB
 
@@ -217,6 +218,15 @@ class Table:
         """Word count on raw text (sepo_run_text): tokenizer fused into the insert kernel."""
         n = int(n) if n is not None else (text.numel() if hasattr(text, "numel") else len(text))
         rc = self._L.sepo_run_text(self.h, _ptr(text), n)
+        if rc < 0:
+            _err(rc)
+        return int(rc)
+
+    def run_wire(self, wire, n=None):
+        """The whole job on routed wire records (sepo_run_wire): a uint8 device tensor of 32-byte records
+        {key words, value, length} as sepo_route_combine writes them."""
+        n = int(n) if n is not None else wire.numel() // 32
+        rc = self._L.sepo_run_wire(self.h, _ptr(wire), n)
         if rc < 0:
             _err(rc)
         return int(rc)

@@ -124,7 +124,6 @@ struct sepo_table {
     DevBuf tbm;      // sepo_run_text: start bits of declined words that did not fit the prepared list
     // cuStreamWriteValue32 (driver entry point): the copy stream publishes eviction progress
     int (*write_value32)(cudaStream_t, unsigned long long, unsigned int, unsigned int) = nullptr;
-    bool no_overlap = true;  // SEPO_EVICT_OVERLAP=1: the next pass starts while the copy drains
 
     // export storage
     std::vector<uint8_t> x_keys, x_vals;
@@ -389,10 +388,6 @@ sepo_table* sepo_create_placed(size_t budget, uint64_t n_buckets, uint32_t page_
                 t->write_value32 = wv;
         }
         cudaGetLastError();
-        // measured on C2 at 4x: every re-issue pass allocates pages at once, so it waits for the
-        // copies anyway (42.1 vs 41.6 ms per job) — the overlap is opt-in
-        const char* ov = getenv("SEPO_EVICT_OVERLAP");
-        t->no_overlap = !(ov && ov[0] == '1');
     }
     return t;
 }
@@ -694,7 +689,21 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
     // reusing it ("pages are copied to CPU memory" — overlapped with the next pass).
     CK(t, cudaEventRecord(t->ev_comp, t->stream));
     CK(t, cudaStreamWaitEvent(t->copy_stream, t->ev_comp, 0));
-    const bool overlapped = t->write_value32 != nullptr && !t->no_overlap;
+    // eviction overlapped with the next pass (the allocator waits per evicted page): measured
+    // worth it when a generation is large (C5u 4x job 86 -> 78 ms with a 192 MB pool), not for a
+    // pool inside L2 (C2 4x: 30.5 -> 31.8 ms) nor for GROUP (fragmented evict lists leave through
+    // the gather kernel, which cannot publish progress in evict-list order). SEPO_EVICT_OVERLAP=0/1
+    // forces the choice.
+    bool want_overlap;
+    {
+        const char* ov = getenv("SEPO_EVICT_OVERLAP");
+        int l2 = 0;
+        cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device);
+        want_overlap = (ov && (ov[0] == '0' || ov[0] == '1'))
+                           ? ov[0] == '1'
+                           : t->opts.mode == SEPO_COMBINE_SUM_U64 && (uint64_t)t->n_pages * t->page_bytes > (uint64_t)l2;
+    }
+    const bool overlapped = t->write_value32 != nullptr && want_overlap;
     GenImage img;
     img.gen = t->d.gen;
     uint64_t bytes = 0, done = 0;
@@ -1107,6 +1116,7 @@ static int64_t prep_passes(sepo_table* t, const Batch& cur, int ps, uint64_t res
         pb.keys = cur.keys; pb.ko = nullptr; pb.vals = nullptr; pb.vo = nullptr; pb.idx = nullptr;
         pb.bitmap = nullptr;
         pb.text = 0; pb.tbm = nullptr;
+        pb.wire = nullptr;
         pb.prep = (const PRec*)t->prep[ps].p;
         pb.n = reserved;
         pb.out = (PRec*)t->prep[ps ^ 1].p;
@@ -1131,7 +1141,7 @@ static int64_t prep_passes(sepo_table* t, const Batch& cur, int ps, uint64_t res
 }
 
 static int64_t run_device(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals,
-                          const uint64_t* vo, uint64_t n);
+                          const uint64_t* vo, uint64_t n, const WireRec* wire = nullptr);
 
 int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals, const uint64_t* vo,
                  uint64_t n) {
@@ -1217,12 +1227,20 @@ int64_t sepo_run(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const u
 
 // sepo_run on device-resident input (the caller's arrays, or the staged copy of host input)
 static int64_t run_device(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals,
-                          const uint64_t* vo, uint64_t n) {
+                          const uint64_t* vo, uint64_t n, const WireRec* wire) {
     trace("run: inputs on device");
-    const uint32_t kw = t->opts.fixed_key_width;
+    const uint32_t kw = wire ? 0u : t->opts.fixed_key_width;
     Batch cur;
-    int rc2 = make_batch(t, cur, keys, ko, vals, vo, n, nullptr);
-    if (rc2) return rc2;
+    if (wire) {  // routed records (a12): keys <= 16 bytes with pre-combined u64 values
+        cur = Batch{};
+        cur.wire = wire;
+        cur.n = n;
+        cur.vw = 8;
+        cur.vals = reinterpret_cast<const uint8_t*>(wire);  // (values present: 48-byte prepared records)
+    } else {
+        int rc2 = make_batch(t, cur, keys, ko, vals, vo, n, nullptr);
+        if (rc2) return rc2;
+    }
     int side = 0;
     int64_t passes_start = (int64_t)t->st.passes;
     uint64_t prev = ~0ull;
@@ -1237,18 +1255,23 @@ static int64_t run_device(sepo_table* t, const uint8_t* keys, const uint64_t* ko
     bool use_prep = t->opts.mode == SEPO_COMBINE_SUM_U64 && combine_exact && !(no_prep && no_prep[0] == '1') && n > 0;
     // prepared record bytes: 32 for implicit values, 32 for values with fixed keys of <= 8 bytes
     // (the key is one word: {key, value, hash, offset | length}), else 48
-    const bool short_keys = !ko && kw > 0 && kw <= 8;
-    const uint64_t prb = (vals && !short_keys) ? sizeof(PRec) : 32;
+    // (routed wire records carry values: 48-byte records, the format the wire kernel writes)
+    const bool short_keys = !wire && !ko && kw > 0 && kw <= 8;
+    const bool has_vals = vals != nullptr || wire != nullptr;
+    const uint64_t prb = (has_vals && !short_keys) ? sizeof(PRec) : 32;
     cur.prep_rb = (uint32_t)prb;
-    cur.prep_fmt = (vals && short_keys) ? 33u : 0u;
+    cur.prep_fmt = (has_vals && short_keys) ? 33u : 0u;
+    if (wire && !use_prep) return fail(SEPO_E_INVAL, "routed records need the prepared re-issue path (COMBINE)");
     if (use_prep) {
         uint64_t cap = std::max<uint64_t>(1ull << 16, n / 4);
         if (const char* pc = getenv("SEPO_PREP_CAP")) cap = strtoull(pc, nullptr, 10);
+        if (wire) cap = std::max<uint64_t>(1ull << 16, n);  // (no index re-issue for routed records: never overflow)
         if ((uint64_t)t->prep[0].cap < cap * prb) {  // first use / larger input: bound by free memory
             size_t fr = 0, tot = 0;
             if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) cap = std::min<uint64_t>(cap, (fr + t->prep[0].cap) / 3 / prb);
         }
         if (t->prep_n.grow(64) || t->prep[0].grow(std::max<uint64_t>(cap, 1) * prb)) {
+            if (wire) return fail(SEPO_E_NOMEM, "prepared re-issue list for routed records");
             use_prep = false;
         } else {
             CK(t, cudaMemsetAsync(t->prep_n.p, 0, 16, t->stream));
@@ -1301,6 +1324,7 @@ static int64_t run_device(sepo_table* t, const uint8_t* keys, const uint64_t* ko
             if (r < 0) return r;
             break;
         }
+        if (wire) return fail(SEPO_E_STATE, "prepared re-issue list overflow (routed records)");
         cur.out = nullptr;  // index re-issue from here on
         if (combine_exact) {
             // the insert's count is exact (certified declines, R15): only the per-tile counts
@@ -1636,6 +1660,63 @@ void sepo_destroy(sepo_table* t) {
 }
 
 // ---------------------------------------------------------------- key-hash router (a12)
+int64_t sepo_run_wire(sepo_table* t, const void* wire, uint64_t n) {
+    trace("run_wire begin", n);
+    int rc = check_active(t);
+    if (rc) return rc;
+    if (t->opts.mode != SEPO_COMBINE_SUM_U64) return fail(SEPO_E_INVAL, "sepo_run_wire needs COMBINE mode");
+    if (n && !is_device_ptr(wire)) return fail(SEPO_E_INVAL, "wire records must be device memory");
+    if (n == 0) {
+        if (t->dirty) { int64_t e = evict_impl(t, 0); if (e < 0) return e; }
+        return 0;
+    }
+    return run_device(t, nullptr, nullptr, nullptr, nullptr, n, reinterpret_cast<const WireRec*>(wire));
+}
+
+size_t sepo_route_scratch(uint32_t n_parts) { return 8 * (3 * (size_t)n_parts + 8); }
+
+int64_t sepo_route_combine(const uint8_t* keys, const uint64_t* ko, uint32_t kw, const uint8_t* vals, uint32_t vw,
+                           uint64_t n, uint32_t n_parts, uint64_t route_seed, void* out_wire, uint64_t out_cap,
+                           uint64_t* part_counts, void* scratch, size_t scratch_bytes, void* stream) {
+    if (n_parts < 1 || n_parts > 32) return fail(SEPO_E_INVAL, "n_parts must be in 1..32");
+    if (!ko && kw == 0) return fail(SEPO_E_INVAL, "key_offsets is NULL and fixed_key_width is 0");
+    if (vals && !(vw == 1 || vw == 2 || vw == 4 || vw == 8)) return fail(SEPO_E_INVAL, "fixed_val_width must be 1, 2, 4 or 8");
+    if (!part_counts || !scratch || scratch_bytes < sepo_route_scratch(n_parts)) return fail(SEPO_E_INVAL, "scratch / part_counts");
+    cudaStream_t s = (cudaStream_t)stream;
+    Batch b{};
+    b.keys = keys; b.ko = ko; b.kw = kw; b.vals = vals; b.vw = vw; b.n = n;
+    unsigned long long* totals = (unsigned long long*)scratch;
+    unsigned long long* cursors = totals + n_parts;
+    unsigned long long* base = cursors + n_parts;
+    unsigned long long* longk = base + n_parts;
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (cudaMemsetAsync(scratch, 0, sepo_route_scratch(n_parts), s) != cudaSuccess) return fail(SEPO_E_CUDA, "memset");
+    // pass 0: output records per part (and keys longer than 16 bytes)
+    // the same route hash as sepo_partition (seed decorrelated from a table seed of equal value)
+    route_seed ^= 0x6a09e667f3bcc909ull;
+    int rc = sepo_launch_route_combine(b, n_parts, route_seed, 0, totals, longk, nullptr, nullptr, nullptr, nsm, s);
+    if (rc) return fail(SEPO_E_CUDA, std::string("route combine: ") + cudaGetErrorString((cudaError_t)rc));
+    std::vector<unsigned long long> h(n_parts + 1);
+    if (cudaMemcpyAsync(h.data(), totals, 8 * n_parts, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaMemcpyAsync(&h[n_parts], longk, 8, cudaMemcpyDeviceToHost, s) != cudaSuccess || cudaStreamSynchronize(s) != cudaSuccess)
+        return fail(SEPO_E_CUDA, "route combine counts");
+    if (h[n_parts]) return fail(SEPO_E_TOOLARGE, "route combine: keys longer than 16 bytes (route them as CSR)");
+    uint64_t tot = 0;
+    for (uint32_t p = 0; p < n_parts; ++p) { part_counts[p] = tot; tot += h[p]; }
+    part_counts[n_parts] = tot;
+    if (!out_wire) return (int64_t)tot;  // sizing call
+    if (out_cap < tot) return fail(SEPO_E_NOMEM, "route combine: out_cap < " + std::to_string(tot) + " records");
+    std::vector<unsigned long long> hb(part_counts, part_counts + n_parts);
+    if (cudaMemcpyAsync(base, hb.data(), 8 * n_parts, cudaMemcpyHostToDevice, s) != cudaSuccess)
+        return fail(SEPO_E_CUDA, "route combine bases");
+    rc = sepo_launch_route_combine(b, n_parts, route_seed, 1, totals, nullptr, base, cursors, (WireRec*)out_wire, nsm, s);
+    if (rc) return fail(SEPO_E_CUDA, std::string("route combine: ") + cudaGetErrorString((cudaError_t)rc));
+    if (cudaStreamSynchronize(s) != cudaSuccess) return fail(SEPO_E_CUDA, "route combine");
+    return (int64_t)tot;
+}
+
 size_t sepo_partition_scratch(uint64_t n, uint32_t n_parts) {
     return (size_t)sepo_partition_tiles(n) * n_parts * 3 * 8 + 256;
 }

@@ -39,6 +39,7 @@ __device__ __forceinline__ uint32_t lanemask_lt() { return (1u << lane_id()) - 1
 __device__ __forceinline__ uint64_t rec_index(const Batch& b, uint64_t i) { return b.idx ? ld_in64(b.idx + i) : i; }
 // value of record i for COMBINE (vw bytes LE, or 1 when vals == nullptr)
 __device__ __forceinline__ uint64_t rec_value(const Batch& b, uint64_t i) {
+    if (b.wire) return b.wire[i].v;
     if (b.vals == nullptr) return 1ull;
     i = rec_index(b, i);
     switch (b.vw) {
@@ -206,6 +207,12 @@ __device__ __forceinline__ void red_add_u64(unsigned long long* p, unsigned long
 // hash + first 16 key bytes of record i
 __device__ __forceinline__ void rec_hash16(const Dev& d, const Batch& b, uint64_t i, uint64_t& s, uint32_t& len,
                                            uint64_t& w0, uint64_t& w1, uint64_t& h) {
+    if (b.wire) {  // a routed record: key words and length in the record
+        const WireRec r = b.wire[i];
+        s = 0; w0 = r.w0; w1 = r.w1; len = (uint32_t)r.len;
+        h = hash_key16(len, d.seed, w0, w1, nullptr);
+        return;
+    }
     rec_key(b, i, s, len);
     const uint8_t* p = b.keys + s;
     load_key16(p, len, w0, w1);
@@ -532,7 +539,7 @@ struct InCtx {
 };
 // input forms of a batch (template parameter of the stream kernel): contiguous CSR keys, fixed-
 // width keys, or a re-issue index list into the caller's arrays
-enum { IN_CSR = 0, IN_FIXED = 1, IN_IDX = 2 };
+enum { IN_CSR = 0, IN_FIXED = 1, IN_IDX = 2, IN_WIRE = 3 };  // (IN_WIRE: lean kernel only)
 // records in group g (1..32); g < ngroups
 __device__ __forceinline__ uint32_t group_cnt(const InCtx& c, uint32_t g) { return g + 1 == c.ngroups ? c.tail : 32u; }
 // (CSR: at the last group of a warp's chunk, lane 31 also loads the end of its key — the start of the
@@ -1303,15 +1310,6 @@ __device__ __forceinline__ void offsets(const Batch& b, uint64_t i, bool ok, uin
     if (IN == IN_CSR) {
         s = ok ? ld_tail64(b.ko + i) : 0ull;
         e = ok ? ld_tail64(b.ko + i + 1) : 0ull;
-    } else if (IN == IN_IDX) {  // re-issue by index: record i of the batch is record idx[i]
-        const uint64_t j = ok ? ld_in64(b.idx + i) : 0ull;
-        if (b.ko) {
-            s = ok ? ld_in64(b.ko + j) : 0ull;
-            e = ok ? ld_in64(b.ko + j + 1) : 0ull;
-        } else {
-            s = j * b.kw;
-            e = ok ? s + b.kw : s;
-        }
     } else {
         s = i * b.kw;
         e = ok ? s + b.kw : s;
@@ -1419,8 +1417,19 @@ __global__ void __launch_bounds__(lean::THREADS, 1) insert_lean_kernel(Dev d, Ba
     const uint32_t gend = (uint32_t)((uint64_t)c.ngroups * (gw + 1) / c.nw);
     // pipeline: key words of group g and offsets of g + 1 in flight before group g is processed
     auto cnt_of = [&](uint32_t x) -> uint32_t { return x < gend ? (x + 1 == c.ngroups ? c.tail : 32u) : 0u; };
-    uint64_t s_c, e_c, s_n, e_n, v_c = 1, x0, x1, x2;
-    {
+    // (IN_WIRE: s = 0, e = the key length, x0 / x1 = the record's key words, v = its value)
+    auto wire_rec = [&](uint32_t x, uint64_t& s, uint64_t& e, uint64_t& k0, uint64_t& k1, uint64_t& v) {
+        s = 0; e = 0; k0 = 0; k1 = 0; v = 0;
+        if (lane < cnt_of(x)) {
+            const ulonglong2* r = reinterpret_cast<const ulonglong2*>(b.wire + (uint64_t)x * 32 + lane);
+            const ulonglong2 a = __ldcs(r), c2 = __ldcs(r + 1);
+            k0 = a.x; k1 = a.y; v = c2.x; e = c2.y;
+        }
+    };
+    uint64_t s_c, e_c, s_n = 0, e_n = 0, v_c = 1, x0, x1, x2 = 0;
+    if (IN == IN_WIRE) {
+        wire_rec(g, s_c, e_c, x0, x1, v_c);
+    } else {
         const bool ok = lane < cnt_of(g);
         lean::offsets<IN>(b, (uint64_t)g * 32 + lane, ok, s_c, e_c);
         if (VALS && ok) v_c = rec_value(b, (uint64_t)g * 32 + lane);
@@ -1429,17 +1438,21 @@ __global__ void __launch_bounds__(lean::THREADS, 1) insert_lean_kernel(Dev d, Ba
     }
     for (; g < gend; ++g) {
         // ---- issue ahead: key words (values) of g + 1, offsets of g + 2
-        uint64_t y0, y1, y2, v_n = 1;
-        lean::key_words(b.keys, s_n, (uint32_t)(e_n - s_n), y0, y1, y2);
-        if (VALS && lane < cnt_of(g + 1)) v_n = rec_value(b, (uint64_t)(g + 1) * 32 + lane);
-        uint64_t s_nn, e_nn;
-        lean::offsets<IN>(b, (uint64_t)(g + 2) * 32 + lane, lane < cnt_of(g + 2), s_nn, e_nn);
+        uint64_t y0, y1, y2 = 0, v_n = 1, s_nn = 0, e_nn = 0, s_w = 0, e_w = 0;
+        if (IN == IN_WIRE) {
+            wire_rec(g + 1, s_w, e_w, y0, y1, v_n);
+        } else {
+            lean::key_words(b.keys, s_n, (uint32_t)(e_n - s_n), y0, y1, y2);
+            if (VALS && lane < cnt_of(g + 1)) v_n = rec_value(b, (uint64_t)(g + 1) * 32 + lane);
+            lean::offsets<IN>(b, (uint64_t)(g + 2) * 32 + lane, lane < cnt_of(g + 2), s_nn, e_nn);
+        }
         // ---- group g: first 16 key bytes + hash (a1)
         const bool valid = lane < cnt_of(g);
         const uint64_t s = s_c;
         const uint32_t len = (uint32_t)(e_c - s_c);  // 0 for lanes past the end
         uint64_t w0, w1;
-        lean::assemble16(x0, x1, x2, (uint32_t)(reinterpret_cast<uintptr_t>(b.keys + s) & 7u), len, w0, w1);
+        if (IN == IN_WIRE) { w0 = x0; w1 = x1; }
+        else lean::assemble16(x0, x1, x2, (uint32_t)(reinterpret_cast<uintptr_t>(b.keys + s) & 7u), len, w0, w1);
         const uint64_t v = VALS ? v_c : 1ull;
         const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
         // ---- hot set (a2): two one-word slots, then one 16-byte key compare
@@ -1504,7 +1517,9 @@ __global__ void __launch_bounds__(lean::THREADS, 1) insert_lean_kernel(Dev d, Ba
             __syncwarp();
         }
         // ---- rotate the pipeline
-        s_c = s_n; e_c = e_n; v_c = v_n; x0 = y0; x1 = y1; x2 = y2;
+        if (IN == IN_WIRE) { s_c = s_w; e_c = e_w; }
+        else { s_c = s_n; e_c = e_n; }
+        v_c = v_n; x0 = y0; x1 = y1; x2 = y2;
         s_n = s_nn; e_n = e_nn;
     }
     if (qtail != qhead) lean_resolve<VALS, RB>(d, b, S, Q, qhead, qtail - qhead, inj, w_full, w_quiet, pc);
@@ -1900,335 +1915,6 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
         if (S.post) atomicAdd(&d.ctrl->postponed, S.post);
         if (S.toolarge) atomicAdd(&d.ctrl->toolarge, S.toolarge);
         if (S.dead) atomicAdd(&d.ctrl->dead_bytes, S.dead);
-    }
-}
-
-// ================================================================ GROUP insert, lean (a1..a7)
-// The multi-valued method for fixed-width values of 1, 2, 4 or 8 bytes (C4: u32 doc
-// ids), on the lean input path (per-warp contiguous group streams; CSR, fixed-width or index
-// batches). Hot keys append into CTA-private value chunks (one shared atomic per warp per key, as
-// insert_group_stream_kernel); every other record goes to a per-warp miss queue and is resolved 32
-// at a time with every lane busy: directory word, chain walk to the key entry, one reservation in
-// the key's head chunk and the value store; keys without an entry and full head chunks take the
-// allocation path (announcement protocol, R15); a resident key whose value cannot be stored marks
-// its key page retained (pending key).
-namespace grp2 {
-constexpr int THREADS = 1024, WARPS = THREADS / 32, QCAP = 64;
-constexpr int DS = 4096, NK = 1024;  // hot slots / hot keys
-constexpr uint32_t PC_CAP = 256;     // slots of a private chunk
-struct Smem {
-    uint32_t tags[DS];
-    ulonglong2 kw[NK];
-    uint32_t ref[NK];
-    unsigned long long pw[NK];  // private chunk word: chunk ref << 32 | fill (ref 0: none)
-    struct Queue {
-        ulonglong2 k[QCAP];          // first 16 key bytes
-        ulonglong2 hs[QCAP];         // hash, key offset | length << 40 | lane << 59
-        unsigned long long v[QCAP];  // value
-        uint32_t g[QCAP];            // group
-    } q[WARPS];
-    stream::CtaState cs;
-};
-static_assert(sizeof(Smem) <= 232448, "grp2 kernel shared memory > 227 KB");
-// value v (vw bytes LE) into slot `at` of chunk c
-__device__ __forceinline__ void store_slot(uint8_t* c, uint32_t at, uint32_t vw, uint64_t v) {
-    uint8_t* dst = c + CHUNK_HDR + (uint64_t)at * vw;
-    if (vw == 4) *reinterpret_cast<uint32_t*>(dst) = (uint32_t)v;
-    else if (vw == 8) *reinterpret_cast<unsigned long long*>(dst) = v;
-    else if (vw == 2) *reinterpret_cast<uint16_t*>(dst) = (uint16_t)v;
-    else *dst = (uint8_t)v;
-}
-}  // namespace grp2
-
-// Resolve up to 32 queued GROUP records, one per lane (a3..a7).
-__device__ __forceinline__ void grp2_resolve(const Dev& d, const Batch& b, grp2::Smem& S, grp2::Smem::Queue& Q, uint32_t qhead,
-                                             uint32_t cnt, bool inj, bool& w_full, bool& w_quiet) {
-    const uint32_t lane = lane_id();
-    const uint32_t PB = d.page_bytes, vw = b.vw;
-    const bool act = lane < cnt;
-    const uint32_t k = (qhead + lane) & (grp2::QCAP - 1);
-    uint64_t w0 = 0, w1 = 0, h = 0, s = 0, v = 0;
-    uint32_t g = 0, len = 0, gl = 0;
-    if (act) {
-        const ulonglong2 kk = Q.k[k], hs = Q.hs[k];
-        w0 = kk.x; w1 = kk.y; h = hs.x;
-        s = hs.y & lean::S_MASK;
-        len = (uint32_t)(hs.y >> 40) & lean::LEN_MAX;
-        gl = (uint32_t)(hs.y >> 59);
-        g = Q.g[k];
-        v = Q.v[k];
-    }
-    const uint8_t* tail = b.keys + s + 16;
-    const uint32_t bkt = bucket_of(h, d.n_buckets), tag = tag_of(h);
-    const uint32_t head = act ? ld_dir(d.dir + bkt) : 0u;
-    uint8_t* e = act ? chain_find_w(d, head, 0, tag, len, w0, w1, tail) : nullptr;
-    bool done = false;
-    if (e) {  // resident key: one reservation in its head chunk
-        uint64_t cr = 0;
-        uint32_t base = 0;
-        if (reserve_head(d, e, 1u, vw, &cr, &base)) {
-            grp2::store_slot(vref_ptr(d, cr), base, vw, v);
-            done = true;
-        }
-    }
-    uint32_t res = R_OK;
-    bool need_key = act && !e, need_chunk = act && !done;
-    const uint32_t ksize = gkey_size(len);
-    const uint32_t ccap = chunk_cap(d, 1u, vw), csize = chunk_bytes(ccap, vw);
-    if (need_key && (len > 65535u - 64u || ksize > PB)) { need_key = false; need_chunk = false; res = R_TOOLARGE; }
-    if (inj && need_key && inject_fail(d, h, (uint64_t)g * 32 + gl)) { need_key = false; need_chunk = false; res = R_POST; }
-    // ---- allocation (a5) + link (a6) under the announcement protocol (R15), as resolve_core
-    if (__any_sync(FULLMASK, need_chunk)) {
-        if (!w_full) {
-            unsigned long long f0 = 0;
-            if (lane == 0) f0 = ld_relaxed_u64(&d.ctrl->full);
-            if (__shfl_sync(FULLMASK, f0, 0)) w_full = true;
-        }
-        if (!w_full) {
-            unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
-            unsigned long long a = 0;
-            if (lane == 0) a = atomicAdd(my_ann, 1ull);
-            a = __shfl_sync(FULLMASK, a, 0);
-            uint64_t koff = ~0ull, coff = ~0ull;
-            if (a & ANN_FULL) {
-                w_full = true;
-            } else {
-                koff = warp_alloc(d, &S.cs.cur[0], need_key, ksize, (uint8_t)PAGE_ENTRY);
-                const bool wc = need_chunk && (!need_key || koff != ~0ull);
-                coff = warp_alloc(d, &S.cs.cur[1], wc, csize, (uint8_t)PAGE_VALUE);
-            }
-            if (need_key && koff != ~0ull) {  // new key entry, linked even if its chunk failed (pending)
-                uint8_t* ne = d.pool + koff;
-                *reinterpret_cast<uint4*>(ne) = make_uint4(ksize | K_GKEY, head, tag, len);
-                if (len > 0) *reinterpret_cast<unsigned long long*>(ne + KEY_OFF) = w0;
-                if (len > 8) *reinterpret_cast<unsigned long long*>(ne + KEY_OFF + 8) = w1;
-                if (len > 16) store_key(ne + KEY_OFF + 16, tail, len - 16);
-                *reinterpret_cast<unsigned long long*>(entry_val(ne, len)) = 0ull;
-                *reinterpret_cast<uint32_t*>(entry_val(ne, len) + 8) = d.gen;
-                *reinterpret_cast<uint32_t*>(entry_val(ne, len) + 12) = 0u;
-                const uint32_t me = off_ref(koff);
-                e = ne;
-                uint32_t hd = head;
-                while (true) {  // lock-free head insertion
-                    const uint32_t old = cas_release(d.dir + bkt, hd, me);
-                    if (old == hd) break;
-                    uint8_t* w = chain_find_w(d, old, hd, tag, len, w0, w1, tail);
-                    if (w) {  // linked meanwhile: retire ours
-                        *reinterpret_cast<uint32_t*>(ne) = ksize | K_DEAD;
-                        atomicAdd(&S.cs.dead, (unsigned long long)ksize);
-                        e = w;
-                        break;
-                    }
-                    hd = old;
-                    *reinterpret_cast<uint32_t*>(ne + 4) = hd;
-                }
-            }
-            if (need_chunk && coff != ~0ull && e) {
-                uint8_t* c = d.pool + coff;
-                init_chunk(c, ccap, vw, 1u, owner_of(d, e));
-                grp2::store_slot(c, 0, vw, v);
-                push_chunk(e, vref_of(d, coff));
-                done = true;
-            }
-            __syncwarp();
-            if (lane == 0) add_release64(my_ann, ~0ull);  // withdraw, after every link above
-        }
-    }
-    // ---- declines (a7): certified for new keys; a resident key with its value left over is pending
-    const bool declined = act && !done && res == R_OK;
-    if (__any_sync(FULLMASK, declined)) {
-        w_full = true;
-        if (!w_quiet) {
-            if (lane == 0)
-                for (uint32_t c = 0; c < d.n_slots; ++c)
-                    while (ld_acquire_u64(d.ann + (uint64_t)c * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
-            __syncwarp();
-            w_quiet = true;
-            if (declined && !e) e = chain_find_w(d, ld_dir(d.dir + bkt), 0, tag, len, w0, w1, tail);
-        }
-        if (declined) {
-            res = R_POST;
-            if (e) {  // resident key: its value may still fit the head chunk
-                uint64_t cr = 0;
-                uint32_t base = 0;
-                if (reserve_head(d, e, 1u, vw, &cr, &base)) {
-                    grp2::store_slot(vref_ptr(d, cr), base, vw, v);
-                    res = R_OK;
-                } else {
-                    d.retain[(uint32_t)((uint64_t)(e - d.pool) >> d.page_shift)] = 1;  // pending key
-                }
-            }
-        }
-    }
-    const bool out = act && res != R_OK;
-    const unsigned pend = __ballot_sync(FULLMASK, out);
-    if (pend) {
-        const unsigned tl = __ballot_sync(FULLMASK, act && res == R_TOOLARGE);
-        const unsigned pkb = __reduce_add_sync(FULLMASK, out ? len : 0u);
-        if (lane == 0) {
-            const uint32_t w = (threadIdx.x >> 5) & 31u;
-            S.cs.wpost[w] += (unsigned long long)__popc(pend);
-            S.cs.wpkb[w] += (unsigned long long)pkb;
-            if (tl) atomicAdd(&S.cs.toolarge, (unsigned long long)__popc(tl));
-        }
-        if (out && b.bitmap) atomicOr(b.bitmap + g, 1u << gl);
-    }
-}
-
-template <int IN>
-__global__ void __launch_bounds__(grp2::THREADS, 1) insert_group2_kernel(Dev d, Batch b, const hot::Entry* hl,
-                                                                           const unsigned int* n_hot, const InCtx c) {
-    using namespace grp2;
-    extern __shared__ __align__(16) uint8_t smem_raw[];
-    grp2::Smem& S = *reinterpret_cast<grp2::Smem*>(smem_raw);
-    const uint32_t tid = threadIdx.x, lane = lane_id(), wid = tid >> 5;
-    const uint32_t vw = b.vw;
-    if (tid == 0) {
-        S.cs.cur[0] = d.cursors[2 * blockIdx.x];
-        S.cs.cur[1] = d.cursors[2 * blockIdx.x + 1];
-        S.cs.post = 0; S.cs.toolarge = 0; S.cs.dead = 0; S.cs.pkb = 0;
-    }
-    if (tid < 32) { S.cs.wpost[tid] = 0; S.cs.wpkb[tid] = 0; }
-    load_hot_direct<DS, NK>(S.tags, S.kw, S.ref, S.pw, hl, n_hot);
-    for (int p = tid; p < NK; p += THREADS) S.pw[p] = PC_CAP;  // no private chunk yet: the first hits install one
-    __syncthreads();
-    const bool have_hot = hl != nullptr && *n_hot > 0;
-    const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
-    const uint32_t pc_bytes = chunk_bytes(PC_CAP, vw);
-    Smem::Queue& Q = S.q[wid];
-    uint32_t qhead = 0, qtail = 0;
-    bool w_full = false, w_quiet = false;
-    const uint64_t gw = (uint64_t)blockIdx.x * WARPS + wid;
-    uint32_t g = (uint32_t)((uint64_t)c.ngroups * gw / c.nw);
-    const uint32_t gend = (uint32_t)((uint64_t)c.ngroups * (gw + 1) / c.nw);
-    auto cnt_of = [&](uint32_t x) -> uint32_t { return x < gend ? (x + 1 == c.ngroups ? c.tail : 32u) : 0u; };
-    uint64_t s_c, e_c, s_n, e_n, v_c = 0, x0, x1, x2;
-    {
-        const bool ok = lane < cnt_of(g);
-        lean::offsets<IN>(b, (uint64_t)g * 32 + lane, ok, s_c, e_c);
-        if (ok) v_c = rec_value(b, (uint64_t)g * 32 + lane);
-        lean::key_words(b.keys, s_c, (uint32_t)(e_c - s_c), x0, x1, x2);
-        lean::offsets<IN>(b, (uint64_t)(g + 1) * 32 + lane, lane < cnt_of(g + 1), s_n, e_n);
-    }
-    for (; g < gend; ++g) {
-        // ---- issue ahead: key words + value of g + 1, offsets of g + 2
-        uint64_t y0, y1, y2, v_n = 0;
-        lean::key_words(b.keys, s_n, (uint32_t)(e_n - s_n), y0, y1, y2);
-        if (lane < cnt_of(g + 1)) v_n = rec_value(b, (uint64_t)(g + 1) * 32 + lane);
-        uint64_t s_nn, e_nn;
-        lean::offsets<IN>(b, (uint64_t)(g + 2) * 32 + lane, lane < cnt_of(g + 2), s_nn, e_nn);
-        // ---- group g: first 16 key bytes + hash (a1)
-        const bool valid = lane < cnt_of(g);
-        const uint64_t s = s_c;
-        const uint32_t len = (uint32_t)(e_c - s_c);
-        uint64_t w0, w1;
-        lean::assemble16(x0, x1, x2, (uint32_t)(reinterpret_cast<uintptr_t>(b.keys + s) & 7u), len, w0, w1);
-        const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
-        const uint64_t v = v_c;
-        // ---- hot set probe (a2)
-        int pos = -1;
-        if (have_hot) {
-            const uint32_t f = stream::dfp(h, len);
-            const uint32_t t1 = S.tags[(uint32_t)(h >> 3) & (DS - 1)], t2 = S.tags[(uint32_t)(h >> 17) & (DS - 1)];
-            constexpr uint32_t IM = (1u << stream::IDXB) - 1u;
-            const bool m1 = (t1 & ~IM) == f, m2 = (t2 & ~IM) == f;
-            const uint32_t p = (m1 ? t1 : t2) & IM;
-            if (valid && (m1 || m2)) {
-                const ulonglong2 kk = S.kw[p];
-                bool eq = kk.x == w0 && kk.y == w1;
-                if (len > 16) {
-                    const uint8_t* e = ref_ptr(d, S.ref[p]);
-                    eq = eq && ldcg32(e + 12) == len && entry_key_eq(e + KEY_OFF + 16, b.keys + s + 16, len - 16);
-                }
-                if (eq) pos = (int)p;
-            }
-        }
-        // ---- hot keys: the warp's values of a key reserved in its private chunk (one shared atomic)
-        bool done = false;
-        const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
-        if (hm) {
-            const unsigned grp = __match_any_sync(FULLMASK, pos >= 0 ? (unsigned)pos : (0x10000u | lane)) & hm;
-            const uint32_t leader = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
-            const uint32_t excl = __popc(grp & lanemask_lt()), tot = __popc(grp);
-            unsigned long long old = 0;
-            if (pos >= 0 && lane == leader) old = atomicAdd(&S.pw[pos], (unsigned long long)tot);
-            old = __shfl_sync(FULLMASK, old, leader);
-            const uint32_t cref = (uint32_t)(old >> 32), f0 = (uint32_t)old;
-            const bool cross = pos >= 0 && f0 <= PC_CAP && f0 + tot > PC_CAP;  // the warp that installs the next chunk
-            const bool fits_old = pos >= 0 && cref && f0 + excl < PC_CAP;
-            const bool want = cross && lane == leader && !w_full;
-            uint32_t nref = 0;
-            if (__any_sync(FULLMASK, want)) {
-                unsigned long long* my_ann = d.ann + (uint64_t)blockIdx.x * ANN_STRIDE;
-                unsigned long long a = 0;
-                if (lane == 0) a = atomicAdd(my_ann, 1ull);
-                a = __shfl_sync(FULLMASK, a, 0);
-                uint64_t coff = ~0ull;
-                if (a & ANN_FULL) w_full = true;
-                else coff = warp_alloc(d, &S.cs.cur[1], want, pc_bytes, (uint8_t)PAGE_VALUE);
-                if (want) {
-                    if (cref) *reinterpret_cast<uint32_t*>(ref_ptr(d, cref) + 4) = PC_CAP;  // the old chunk is full
-                    if (coff != ~0ull) {
-                        uint8_t* ch = d.pool + coff;
-                        uint8_t* ke = ref_ptr(d, S.ref[pos]);
-                        init_chunk(ch, PC_CAP, vw, CHUNK_PRIVATE, owner_of(d, ke));
-                        push_chunk(ke, vref_of(d, coff));
-                        nref = off_ref(coff);
-                        atomicExch(&S.pw[pos], ((unsigned long long)nref << 32) | (f0 + tot - PC_CAP));
-                    } else {
-                        atomicExch(&S.pw[pos], (unsigned long long)PC_CAP << 1);  // no chunk: hits go global
-                    }
-                }
-                __syncwarp();
-                if (lane == 0) add_release64(my_ann, ~0ull);
-            } else if (cross && lane == leader) {  // (pool known full: no private chunk any more)
-                if (cref) *reinterpret_cast<uint32_t*>(ref_ptr(d, cref) + 4) = PC_CAP;
-                atomicExch(&S.pw[pos], (unsigned long long)PC_CAP << 1);
-            }
-            nref = __shfl_sync(FULLMASK, nref, leader);
-            if (pos >= 0) {
-                const uint32_t at = f0 + excl;
-                if (fits_old) { store_slot(ref_ptr(d, cref), at, vw, v); done = true; }
-                else if (cross && nref && at >= PC_CAP) { store_slot(ref_ptr(d, nref), at - PC_CAP, vw, v); done = true; }
-            }
-        }
-        // ---- everything else: the warp's miss queue, resolved 32 at a time (a3..a7)
-        const bool miss = valid && !done;
-        const unsigned mm = __ballot_sync(FULLMASK, miss);
-        if (lane == 0 && b.bitmap) b.bitmap[g] = 0u;
-        if (miss) {
-            const uint32_t k = (qtail + __popc(mm & lanemask_lt())) & (QCAP - 1);
-            Q.k[k] = make_ulonglong2(w0, w1);
-            Q.hs[k] = make_ulonglong2(h, s | ((uint64_t)min(len, lean::LEN_MAX) << 40) | ((uint64_t)lane << 59));
-            Q.g[k] = g;
-            Q.v[k] = v;
-        }
-        qtail += __popc(mm);
-        __syncwarp();
-        if (qtail - qhead >= 32) {
-            grp2_resolve(d, b, S, Q, qhead, 32, inj, w_full, w_quiet);
-            qhead += 32;
-            __syncwarp();
-        }
-        s_c = s_n; e_c = e_n; v_c = v_n; x0 = y0; x1 = y1; x2 = y2;
-        s_n = s_nn; e_n = e_nn;
-    }
-    if (qtail != qhead) grp2_resolve(d, b, S, Q, qhead, qtail - qhead, inj, w_full, w_quiet);
-    __syncthreads();
-    // final fill of every private chunk still open (clears CHUNK_PRIVATE)
-    for (int p = tid; p < NK; p += THREADS) {
-        const unsigned long long w = S.pw[p];
-        const uint32_t cref = (uint32_t)(w >> 32);
-        if (cref) *reinterpret_cast<uint32_t*>(ref_ptr(d, cref) + 4) = min((uint32_t)w, PC_CAP);
-    }
-    if (tid == 0) {
-        d.cursors[2 * blockIdx.x] = S.cs.cur[0];
-        d.cursors[2 * blockIdx.x + 1] = S.cs.cur[1];
-        for (uint32_t w = 0; w < (uint32_t)WARPS; ++w) { S.cs.post += S.cs.wpost[w]; S.cs.pkb += S.cs.wpkb[w]; }
-        if (S.cs.post) atomicAdd(&d.ctrl->postponed, S.cs.post);
-        if (S.cs.toolarge) atomicAdd(&d.ctrl->toolarge, S.cs.toolarge);
-        if (S.cs.dead) atomicAdd(&d.ctrl->dead_bytes, S.cs.dead);
-        if (S.cs.pkb) atomicAdd(&d.ctrl->kept_key_bytes, S.cs.pkb);
     }
 }
 
@@ -2635,6 +2321,150 @@ __global__ void __launch_bounds__(PT_THREADS) part_scatter_kernel(Batch b, uint3
                 for (uint32_t x = 0; x < b.vw; ++x) ov[orec * b.vw + x] = __ldg(b.vals + vs + x);
             }
         }
+        __syncthreads();
+    }
+}
+
+// ---- router with CTA pre-combine (COMBINE mode, keys of at most 16 bytes)
+// Records of one rank go to their owners as 32-byte WireRecs {key words, value, length} after the
+// CTA has combined equal keys of its tile in shared memory (a hot Zipf key leaves a tile once, with
+// its partial sum: C5-Zipf's top key, 18 % of the records, would otherwise overload its owner).
+// Two passes over the batch, the same combine in both (the set of distinct keys of a tile does not
+// depend on thread timing): pass 0 counts each part's output, pass 1 writes it through per-part
+// cursors (the order of records within a part is immaterial: the method is order independent).
+namespace rc {
+constexpr int THREADS = 1024, TILE = 2048, NSLOT = 4096, R = TILE / THREADS, NCOL = 64;
+// meta: 0 empty, else the key's route hash (high 48 bits) | owner << 8 | (len + 2)
+struct Slot { unsigned long long w0, w1, v, meta; };
+struct Smem {
+    Slot t[NSLOT];
+    Slot col[NCOL];                   // records whose (hash, length) matched a different key's slot
+    unsigned int pc[PT_MAXP];         // records of the tile per part
+    unsigned long long pb[PT_MAXP];   // base of the tile's records in each part
+    unsigned int ncol;
+};
+static_assert(sizeof(Smem) <= 232448, "route-combine shared memory > 227 KB");
+}  // namespace rc
+
+// Per tile, in three barrier-separated phases (no thread ever waits for another's progress):
+//   A  every warp folds its equal keys; one lane per distinct key claims or finds the slot of its
+//      (hash, length) by CAS on the slot's meta word; a claimer writes its key words and partial sum;
+//   B  the other lanes of a slot add their sums after comparing key words (equal hash and length
+//      but different key bytes — a 48-bit hash collision — go to a small list emitted one by one);
+//   C  (pass 1) the tile's records are written to their owners' parts.
+__global__ void __launch_bounds__(rc::THREADS, 1) route_combine_kernel(Batch b, uint32_t P, uint64_t seed, int pass,
+                                                                      unsigned long long* part_totals,
+                                                                      unsigned long long* long_keys,
+                                                                      const unsigned long long* part_base,
+                                                                      unsigned long long* cursors, WireRec* out) {
+    using namespace rc;
+    extern __shared__ __align__(16) uint8_t smem_raw[];
+    rc::Smem& S = *reinterpret_cast<rc::Smem*>(smem_raw);
+    const uint32_t tid = threadIdx.x, lane = lane_id();
+    const uint64_t ntiles = (b.n + TILE - 1) / TILE;
+    for (uint32_t x = tid; x < NSLOT; x += THREADS) S.t[x].meta = 0ull;
+    if (tid < PT_MAXP) S.pc[tid] = 0u;
+    if (tid == 0) S.ncol = 0u;
+    __syncthreads();
+    for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+        uint64_t kw0[R], kw1[R], ksum[R], kmeta[R];
+        uint32_t kslot[R];
+        bool klead[R], kclaim[R];
+        // ---- A
+        for (int r = 0; r < R; ++r) {
+            const uint64_t i = tile * TILE + (uint64_t)r * THREADS + tid;
+            const bool valid = i < b.n;
+            uint64_t s = 0, w0 = 0, w1 = 0, v = 0;
+            uint32_t len = 0;
+            if (valid) {
+                rec_key(b, i, s, len);
+                load_key16(b.keys + s, len, w0, w1);
+                v = rec_value(b, i);
+            }
+            const bool ok = valid && len <= 16;
+            if (valid && !ok && long_keys) atomicAdd(long_keys, 1ull);  // the caller routes this batch as CSR
+            const uint64_t h = hash_key16(ok ? len : 0u, seed, w0, w1, b.keys + s);
+            // warp fold: one lane per distinct key carries the warp's sum (a lane joins the lowest lane
+            // of its hash group only with equal key bytes)
+            const unsigned vm = __ballot_sync(FULLMASK, ok);
+            const unsigned grp = __match_any_sync(FULLMASK, ok ? h : (~0ull ^ lane)) & vm;
+            const uint32_t first = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
+            const uint64_t fw0 = __shfl_sync(FULLMASK, w0, first), fw1 = __shfl_sync(FULLMASK, w1, first);
+            const uint32_t flen = __shfl_sync(FULLMASK, len, first);
+            const bool same = ok && fw0 == w0 && fw1 == w1 && flen == len;
+            const unsigned sm = __ballot_sync(FULLMASK, same) & grp;
+            const bool lead = ok && (!same || lane == first);
+            const unsigned mine = same ? sm : (ok ? (1u << lane) : 0u);
+            uint64_t sum = v;
+            if (b.vals == nullptr) {
+                sum = (uint64_t)__popc(mine);
+            } else if (__any_sync(FULLMASK, __popc(mine) > 1)) {
+                sum = 0;
+                for (int xl = 0; xl < 32; ++xl) {
+                    const uint64_t vx = __shfl_sync(FULLMASK, v, xl);
+                    if ((mine >> xl) & 1u) sum += vx;
+                }
+            }
+            const uint32_t owner = (uint32_t)(((h >> 32) * (uint64_t)P) >> 32);
+            const unsigned long long meta = (h & ~0xffffull) | ((unsigned long long)owner << 8) | (unsigned long long)(len + 2);
+            uint32_t x = (uint32_t)(h >> 7) & (NSLOT - 1);
+            bool claim = false;
+            if (lead) {
+                while (true) {
+                    const unsigned long long m = atomicCAS(&S.t[x].meta, 0ull, meta);
+                    if (m == 0ull) { claim = true; break; }
+                    if (m == meta) break;
+                    x = (x + 1) & (NSLOT - 1);
+                }
+                if (claim) {
+                    S.t[x].w0 = w0; S.t[x].w1 = w1; S.t[x].v = sum;
+                    atomicAdd(&S.pc[owner], 1u);
+                }
+            }
+            kw0[r] = w0; kw1[r] = w1; ksum[r] = sum; kmeta[r] = meta; kslot[r] = x; klead[r] = lead; kclaim[r] = claim;
+        }
+        __syncthreads();
+        // ---- B
+        for (int r = 0; r < R; ++r) {
+            if (!klead[r] || kclaim[r]) continue;
+            const uint32_t x = kslot[r];
+            if (S.t[x].w0 == kw0[r] && S.t[x].w1 == kw1[r]) {
+                atomicAdd(&S.t[x].v, ksum[r]);
+            } else {  // (hash collision: emitted on its own)
+                const uint32_t c = atomicAdd(&S.ncol, 1u);
+                if (c < NCOL) {
+                    S.col[c].w0 = kw0[r]; S.col[c].w1 = kw1[r]; S.col[c].v = ksum[r]; S.col[c].meta = kmeta[r];
+                    atomicAdd(&S.pc[(uint32_t)(kmeta[r] >> 8) & 0xffu], 1u);
+                } else if (long_keys) {
+                    atomicAdd(long_keys, 1ull);  // (never seen: the caller falls back to the CSR route)
+                }
+            }
+        }
+        __syncthreads();
+        // ---- C
+        if (pass == 0) {
+            if (tid < P && S.pc[tid]) atomicAdd(&part_totals[tid], (unsigned long long)S.pc[tid]);
+        } else {
+            if (tid < P) {
+                S.pb[tid] = part_base[tid] + atomicAdd(&cursors[tid], (unsigned long long)S.pc[tid]);
+                S.pc[tid] = 0u;
+            }
+            __syncthreads();
+            const uint32_t ncol = min(S.ncol, (uint32_t)NCOL);
+            for (uint32_t x = tid; x < NSLOT + ncol; x += THREADS) {
+                const Slot& sl = x < NSLOT ? S.t[x] : S.col[x - NSLOT];
+                const unsigned long long m = sl.meta;
+                if (m == 0ull) continue;
+                const uint32_t owner = (uint32_t)(m >> 8) & 0xffu;
+                const unsigned long long at = S.pb[owner] + atomicAdd(&S.pc[owner], 1u);
+                reinterpret_cast<ulonglong2*>(out + at)[0] = make_ulonglong2(sl.w0, sl.w1);
+                reinterpret_cast<ulonglong2*>(out + at)[1] = make_ulonglong2(sl.v, (m & 0xffull) - 2ull);
+            }
+        }
+        __syncthreads();
+        for (uint32_t x = tid; x < NSLOT; x += THREADS) S.t[x].meta = 0ull;
+        if (tid < PT_MAXP) S.pc[tid] = 0u;
+        if (tid == 0) S.ncol = 0u;
         __syncthreads();
     }
 }
@@ -3507,7 +3337,7 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             cudaFuncSetAttribute(insert_stream_kernel<true, T, IN_IDX>, cudaFuncAttributeMaxDynamicSharedMemorySize, s1);
             attr = true;
         }
-        const int in = b.idx ? IN_IDX : (b.ko ? IN_CSR : IN_FIXED);
+        const int in = b.wire ? IN_WIRE : (b.idx ? IN_IDX : (b.ko ? IN_CSR : IN_FIXED));
         InCtx c;
         c.ngroups = (uint32_t)((b.n + 31) / 32);
         c.tail = (uint32_t)(b.n - (uint64_t)(c.ngroups ? c.ngroups - 1 : 0) * 32);
@@ -3515,7 +3345,7 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
         c.kend = in == IN_IDX ? 0ull : (in == IN_CSR ? key_end : b.n * (uint64_t)b.kw);
         c.kal = !(reinterpret_cast<uintptr_t>(b.keys) & 15);
         c.dirpf = dir_prefetch;
-        if (lean_in && in != IN_IDX) {  // contiguous batch of mostly short keys: the lean input path
+        if ((lean_in && in != IN_IDX) || in == IN_WIRE) {  // contiguous batch of mostly short keys: the lean input path
             static bool attr_l = false;
             if (!attr_l) {
                 const int s0 = (int)sizeof(lean::Smem<false>), s1 = (int)sizeof(lean::Smem<true>);
@@ -3530,7 +3360,15 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             c.nw = (uint32_t)grid * lean::WARPS;
             const size_t sml = b.vals ? sizeof(lean::Smem<true>) : sizeof(lean::Smem<false>);
             const dim3 G(grid), B(lean::THREADS);
-            if (!b.vals) {
+            if (b.wire) {
+                static bool attr_w = false;
+                if (!attr_w) {
+                    cudaFuncSetAttribute(insert_lean_kernel<true, IN_WIRE, 48>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)sizeof(lean::Smem<true>));
+                    attr_w = true;
+                }
+                insert_lean_kernel<true, IN_WIRE, 48><<<G, B, sizeof(lean::Smem<true>), s>>>(d, b, hl, nh, c);
+            } else if (!b.vals) {
                 if (in == IN_CSR) insert_lean_kernel<false, IN_CSR, 32><<<G, B, sml, s>>>(d, b, hl, nh, c);
                 else insert_lean_kernel<false, IN_FIXED, 32><<<G, B, sml, s>>>(d, b, hl, nh, c);
             } else if (b.prep_fmt == 33) {
@@ -3572,27 +3410,6 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             hl = list;
             nh = n_out;
             if (hot_built) *hot_built = true;
-        }
-        const char* g2 = getenv("SEPO_GROUP2");  // 0: insert_group_stream_kernel for every GROUP batch
-        if (!(g2 && g2[0] == '0') && !b.vo && (b.vw == 1 || b.vw == 2 || b.vw == 4 || b.vw == 8)) {
-            static bool attr2 = false;
-            if (!attr2) {
-                const int s2 = (int)sizeof(grp2::Smem);
-                cudaFuncSetAttribute(insert_group2_kernel<IN_CSR>, cudaFuncAttributeMaxDynamicSharedMemorySize, s2);
-                cudaFuncSetAttribute(insert_group2_kernel<IN_FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, s2);
-                cudaFuncSetAttribute(insert_group2_kernel<IN_IDX>, cudaFuncAttributeMaxDynamicSharedMemorySize, s2);
-                attr2 = true;
-            }
-            InCtx c{};
-            c.ngroups = (uint32_t)((b.n + 31) / 32);
-            c.tail = (uint32_t)(b.n - (uint64_t)(c.ngroups ? c.ngroups - 1 : 0) * 32);
-            c.nw = (uint32_t)grid * grp2::WARPS;
-            const int in = b.idx ? IN_IDX : (b.ko ? IN_CSR : IN_FIXED);
-            const size_t sm2 = sizeof(grp2::Smem);
-            if (in == IN_CSR) insert_group2_kernel<IN_CSR><<<grid, grp2::THREADS, sm2, s>>>(d, b, hl, nh, c);
-            else if (in == IN_FIXED) insert_group2_kernel<IN_FIXED><<<grid, grp2::THREADS, sm2, s>>>(d, b, hl, nh, c);
-            else insert_group2_kernel<IN_IDX><<<grid, grp2::THREADS, sm2, s>>>(d, b, hl, nh, c);
-            return cudaGetLastError();
         }
         const size_t sm = sizeof(gst::Smem);
         static bool attrg = false;
@@ -3668,6 +3485,18 @@ int sepo_launch_partition(const Batch& b, uint32_t P, uint64_t seed, unsigned lo
     return cudaGetLastError();
 }
 uint64_t sepo_partition_tiles(uint64_t n) { return (n + PT_TILE - 1) / PT_TILE; }
+int sepo_launch_route_combine(const Batch& b, uint32_t P, uint64_t seed, int pass, unsigned long long* part_totals,
+                              unsigned long long* long_keys, const unsigned long long* part_base,
+                              unsigned long long* cursors, WireRec* out, int grid, cudaStream_t s) {
+    static bool attr = false;
+    if (!attr) {
+        cudaFuncSetAttribute(route_combine_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(rc::Smem));
+        attr = true;
+    }
+    if (b.n) route_combine_kernel<<<grid, rc::THREADS, sizeof(rc::Smem), s>>>(b, P, seed, pass, part_totals, long_keys,
+                                                                              part_base, cursors, out);
+    return cudaGetLastError();
+}
 int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const uint64_t* seg_base, uint32_t n_segs,
                               uint64_t total, cudaStream_t s) {
     shift_offsets_kernel<<<(unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n + 255) / 256, 4096)), 256, 0, s>>>(

@@ -5,6 +5,7 @@
 #include "sepo_dev.cuh"
 
 namespace sepo {
+struct WireRec;
 // A postponed COMBINE record, re-issued by sepo_run in "prepared" form (a9): its hash, first 16
 // key bytes (zero padded), key offset in the caller's key bytes (tail of keys longer than 16 B),
 // value and key length — the next pass needs neither the input gather nor the hash again.
@@ -41,7 +42,15 @@ struct Batch {
     uint32_t text = 0;
     uint32_t* tbm = nullptr;
     uint64_t w_begin = 0, w_end = ~0ull;  // text: the 512-byte windows this launch tokenizes
+    // wire input (a12, the routed path): record i is the 32-byte WireRec wire[i] (keys of at most
+    // 16 bytes, pre-combined values); keys / ko / vals are unused then
+    const struct WireRec* wire = nullptr;
 };
+// A routed record (a12): a key of at most 16 bytes (zero padded) and its pre-combined u64 value.
+struct WireRec {
+    uint64_t w0, w1, v, len;
+};
+static_assert(sizeof(WireRec) == 32, "WireRec layout");
 }  // namespace sepo
 
 // key_end: key_offsets[n] of a CSR batch (the end of its key bytes), read by the host
@@ -53,6 +62,13 @@ int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int g
                        bool* hot_built = nullptr, bool lean_in = false);
 size_t sepo_hot_count_offset();
 int sepo_launch_reinsert(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s);
+// Router with CTA pre-combine (a12): pass 0 counts per-part output records (part_totals[P], device,
+// zeroed by the caller) and flags keys longer than 16 bytes in *long_keys; pass 1 writes the
+// WireRecs of part p at out + part_base[p] (device, exclusive prefix of the totals) through the
+// per-part cursors cursors[P] (device, zeroed by the caller).
+int sepo_launch_route_combine(const sepo::Batch& b, uint32_t P, uint64_t seed, int pass, unsigned long long* part_totals,
+                              unsigned long long* long_keys, const unsigned long long* part_base,
+                              unsigned long long* cursors, sepo::WireRec* out, int grid, cudaStream_t s);
 size_t sepo_hot_scratch_bytes();
 int sepo_default_grid(int mode, int n_sms);
 int sepo_launch_reprobe(const sepo::Dev& d, const sepo::Batch& b, int mode, int probe, int grid,

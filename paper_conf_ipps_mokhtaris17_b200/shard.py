@@ -28,6 +28,10 @@ def _bind():
     L.sepo_partition.restype = ctypes.c_int
     L.sepo_shift_offsets.argtypes = [vp, u64, vp, vp, u32, u64, vp]
     L.sepo_shift_offsets.restype = ctypes.c_int
+    L.sepo_route_scratch.argtypes = [u32]
+    L.sepo_route_scratch.restype = ctypes.c_size_t
+    L.sepo_route_combine.argtypes = [vp, vp, u32, vp, u32, u64, u32, u64, vp, u64, vp, vp, ctypes.c_size_t, vp]
+    L.sepo_route_combine.restype = ctypes.c_int64
     _bound = True
 
 
@@ -50,6 +54,55 @@ def partition(keys, key_offsets, vals, n_parts, route_seed=0, fixed_key_width=0,
     if rc:
         _err(rc)
     return ok, (oko[:n] if oko is not None else None), ov, starts.reshape(n_parts + 1, 3)
+
+
+WIRE_BYTES = 32  # sepo_route_combine's record: key words w0, w1, value, length (u64 each)
+E_TOOLARGE = -3
+
+
+def route_combine(keys, key_offsets, vals, n_parts, route_seed=0, fixed_key_width=0, fixed_val_width=0, out=None):
+    """Partition with CTA pre-combine (COMBINE, keys <= 16 B; sepo_route_combine) -> (wire uint8 tensor,
+    part_counts numpy [n_parts + 1]): part p's 32-byte records are rows [counts[p], counts[p+1]).
+    Returns None if some key is longer than 16 bytes (route the batch with partition())."""
+    _bind()
+    L = lib()
+    n = (key_offsets.numel() - 1) if key_offsets is not None else keys.numel() // fixed_key_width
+    dev = keys.device
+    scratch = torch.empty(int(L.sepo_route_scratch(n_parts)), dtype=torch.uint8, device=dev)
+    counts = np.zeros(n_parts + 1, dtype=np.uint64)
+    stream = ctypes.c_void_p(torch.cuda.current_stream(dev).cuda_stream)
+    args = (_ptr(keys), _ptr(key_offsets), fixed_key_width, _ptr(vals), fixed_val_width, n, n_parts, route_seed)
+    E_NOMEM = -2
+    for _ in range(2):
+        cap = out.numel() // WIRE_BYTES if out is not None else 0
+        m = L.sepo_route_combine(*args, out.data_ptr() if cap else None, cap, counts.ctypes.data, scratch.data_ptr(),
+                                 scratch.numel(), stream)
+        if m == E_TOOLARGE:
+            return None
+        if m == E_NOMEM or (m >= 0 and not cap):  # (too small / sizing call): allocate and run again
+            out = torch.empty(max(int(counts[-1]), 1) * WIRE_BYTES, dtype=torch.uint8, device=dev)
+            continue
+        if m < 0:
+            _err(m)
+        return out[: int(m) * WIRE_BYTES], counts
+    raise RuntimeError("sepo_route_combine: output size changed between calls")
+
+
+def exchange_wire(wire, counts, group=None):
+    """All-to-all of routed wire records (part p -> rank p) -> the records this rank owns."""
+    world = dist.get_world_size(group)
+    send = np.diff(np.asarray(counts, dtype=np.int64))
+    if world == 1:
+        return wire
+    dev = wire.device
+    send_t = torch.as_tensor(send, dtype=torch.int64, device=dev)
+    recv_t = torch.empty_like(send_t)
+    dist.all_to_all_single(recv_t, send_t, group=group)
+    recv = recv_t.cpu().numpy()
+    out = torch.empty(max(int(recv.sum()), 1) * WIRE_BYTES, dtype=torch.uint8, device=dev)
+    dist.all_to_all_single(out[: int(recv.sum()) * WIRE_BYTES], wire[: int(send.sum()) * WIRE_BYTES],
+                           (recv * WIRE_BYTES).tolist(), (send * WIRE_BYTES).tolist(), group=group)
+    return out[: int(recv.sum()) * WIRE_BYTES]
 
 
 def shift_offsets_cuda(ko, seg_rec, seg_base, total):
@@ -107,20 +160,42 @@ def route(keys, key_offsets, vals, group=None, route_seed=0, fixed_key_width=0, 
 
 
 class Router:
-    """Routes each step's batch of this rank to the key owners (partition + exchange) and keeps
-    per-step statistics for the bench line."""
+    """Routes each step's batch of this rank to the key owners and keeps per-step statistics.
 
-    def __init__(self, group=None, route_seed=0, fixed_key_width=0, fixed_val_width=0):
-        self.group, self.seed, self.kw, self.vw = group, route_seed, fixed_key_width, fixed_val_width
+    combine=True (COMBINE tables, keys <= 16 B): sepo_route_combine pre-combines every CTA tile and
+    the exchange carries 32-byte wire records -> route() returns ("wire", tensor) for Table.run_wire;
+    batches with longer keys (and combine=False) are partitioned as CSR -> ("csr", (keys, offsets,
+    vals)) for Table.run."""
+
+    def __init__(self, group=None, route_seed=0, fixed_key_width=0, fixed_val_width=0, combine=True):
+        self.group, self.seed, self.kw, self.vw, self.combine = group, route_seed, fixed_key_width, fixed_val_width, combine
         self._last = {}
+        self._wire_buf = None
 
     def route(self, keys, key_offsets, vals):
         world = dist.get_world_size(self.group)
+        n_in = (key_offsets.numel() - 1) if key_offsets is not None else keys.numel() // max(self.kw, 1)
+        if self.combine:
+            r = route_combine(keys, key_offsets, vals, world, self.seed, self.kw, self.vw, out=self._wire_buf)
+            if r is not None:
+                wire, counts = r
+                if self._wire_buf is None or self._wire_buf.numel() < wire.numel():
+                    self._wire_buf = wire
+                out = exchange_wire(wire, counts, self.group)
+                self._last = {"records_in": n_in, "records_sent": int(counts[-1]), "records_out": out.numel() // WIRE_BYTES,
+                              "format": "wire (pre-combined)"}
+                return "wire", out
         ok, oko, ov, starts = partition(keys, key_offsets, vals, world, self.seed, self.kw, self.vw)
         out = exchange(ok, oko, ov, starts, self.group)
-        self._last = {"records_in": int(starts[-1, 0]), "records_out": int(out[1].numel() - 1) if out[1] is not None
-                      else int(out[0].numel() // max(self.kw, 1))}
-        return out
+        self._last = {"records_in": n_in, "records_out": int(out[1].numel() - 1) if out[1] is not None
+                      else int(out[0].numel() // max(self.kw, 1)), "format": "csr"}
+        return "csr", out
+
+    @staticmethod
+    def run(table, routed):
+        """the SEPO job on what route() returned"""
+        kind, data = routed
+        return table.run_wire(data) if kind == "wire" else table.run(*data)
 
     def last_stats(self):
         return dict(self._last)

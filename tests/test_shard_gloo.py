@@ -90,3 +90,52 @@ def test_exchange_world2():
     for rank, ok, n, closed in res:
         assert ok, f"rank {rank} received the wrong records"
         assert closed and n > 0
+
+
+def _wire_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_mokhtaris17_b200 import shard
+    rng = np.random.default_rng(10 + rank)
+    n_per = [int(x) for x in rng.integers(0, 40, size=world)]
+    recs, counts = [], [0]
+    for p in range(world):  # part p's records: key "r<rank>p<p>i<i>", value = rank*1000 + i
+        for i in range(n_per[p]):
+            key = b"r%dp%di%d" % (rank, p, i)
+            w = key.ljust(16, b"\0")
+            recs.append(np.frombuffer(w, dtype=np.uint64).tolist() + [rank * 1000 + i, len(key)])
+        counts.append(counts[-1] + n_per[p])
+    wire = torch.from_numpy(np.array(recs, dtype=np.uint64).reshape(-1).view(np.uint8).copy() if recs
+                            else np.zeros(0, dtype=np.uint8))
+    out = shard.exchange_wire(wire, np.array(counts, dtype=np.uint64))
+    q.put((rank, out.numpy().tobytes(), n_per))
+    dist.destroy_process_group()
+
+
+def test_exchange_wire_gloo():
+    """wire records (32 B each) of part p reach rank p, in sender-rank order, byte for byte"""
+    world = 2
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_wire_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in ps:
+        p.start()
+    res = {}
+    for _ in range(world):
+        r, b, n_per = q.get(timeout=120)
+        res[r] = (b, n_per)
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for dst in range(world):
+        got = np.frombuffer(res[dst][0], dtype=np.uint64).reshape(-1, 4)
+        exp = []
+        for src in range(world):
+            for i in range(res[src][1][dst]):
+                key = b"r%dp%di%d" % (src, dst, i)
+                exp.append(np.frombuffer(key.ljust(16, b"\0"), dtype=np.uint64).tolist() + [src * 1000 + i, len(key)])
+        assert got.tolist() == exp

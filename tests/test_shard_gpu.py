@@ -107,3 +107,86 @@ def test_sharded_job_loopback(cuda, name, P):
         assert not (set(part) & set(got))  # shards own disjoint keys
         got.update(part)
     assert got == exp
+
+
+# ---- router with CTA pre-combine (sepo_route_combine) + wire records
+def wire_dict(wire):
+    """32-byte wire records -> {key bytes: summed value} (test-side decode; records of one key may repeat)"""
+    a = wire.cpu().numpy().view(np.uint64).reshape(-1, 4)
+    out = {}
+    for w0, w1, v, ln in a:
+        key = (int(w0).to_bytes(8, "little") + int(w1).to_bytes(8, "little"))[: int(ln)]
+        out[key] = (out.get(key, 0) + int(v)) % (1 << 64)
+    return out
+
+
+@pytest.mark.parametrize("name,P", [("C2", 1), ("C2", 4), ("C5z", 3), ("C5u", 2)])
+def test_route_combine_parts(cuda, name, P):
+    """every part's pre-combined records sum to the oracle's values of exactly the keys it owns, the
+    parts own disjoint key sets, and equal keys were combined inside each CTA tile (fewer records)"""
+    from paper_conf_ipps_mokhtaris17_b200 import shard
+    scale = {"C2": 1 / 1024, "C5z": 2 ** -12, "C5u": 2 ** -14}[name]
+    s = gen.config(name, scale=scale)
+    exp = oracle_expected(s)
+    k, o, v = s.device()
+    fixed = s.family == gen.GEN_PAIRS
+    wire, counts = shard.route_combine(k, None if fixed else o, v, P, route_seed=5, fixed_key_width=8 if fixed else 0,
+                                       fixed_val_width=8 if v is not None else 0)
+    assert counts[0] == 0 and int(counts[-1]) == wire.numel() // 32
+    got, owners = {}, []
+    for p in range(P):
+        part = wire_dict(wire[int(counts[p]) * 32:int(counts[p + 1]) * 32])
+        owners.append(set(part))
+        for key, val in part.items():
+            got[key] = (got.get(key, 0) + val) % (1 << 64)
+    for a in range(P):
+        for b in range(a + 1, P):
+            assert not (owners[a] & owners[b])
+    assert got == exp
+    if name != "C5u":  # Zipf: the hot keys leave each tile once
+        assert int(counts[-1]) < 0.7 * s.n
+    # the owners agree with the CSR partition's (same route hash)
+    if P > 1 and not fixed:
+        ok, oko, _, starts = shard.partition(k, o, None, P, route_seed=5)
+        for p in range(P):
+            sk, so = segment(ok, oko, starts, p)
+            keys_p = set(oracle.combine(sk.cpu().numpy(), so.cpu().numpy().view(np.uint64)).as_dict())
+            assert keys_p == owners[p]
+
+
+def test_route_combine_rejects_long_keys(cuda):
+    from paper_conf_ipps_mokhtaris17_b200 import shard
+    s = gen.config("C3", scale=1 / 8000)  # URLs: longer than 16 bytes
+    k, o, _ = s.device()
+    assert shard.route_combine(k, o, None, 2, route_seed=1) is None
+
+
+@pytest.mark.parametrize("name,ratio", [("C5z", 4), ("C2", 4), ("C2", 0.5)])
+def test_run_wire_vs_oracle(cuda, name, ratio):
+    """the SEPO job on routed (pre-combined) wire records, one rank (loopback), in and over budget:
+    == the oracle on the original records (hot set active at these sizes)"""
+    from paper_conf_ipps_mokhtaris17_b200 import shard
+    scale = {"C2": 1 / 256, "C5z": 1 / 128}[name]
+    s = gen.config(name, scale=scale)
+    exp = oracle_expected(s)
+    k, o, v = s.device()
+    fixed = s.family == gen.GEN_PAIRS
+    wire, counts = shard.route_combine(k, None if fixed else o, v, 1, route_seed=9, fixed_key_width=8 if fixed else 0,
+                                       fixed_val_width=8 if v is not None else 0)
+    n = wire.numel() // 32
+    assert n >= 2_097_152 or name == "C2"
+    big = sepo().budget_for(1 << 18, 16384, 1 << 14)
+    t = sepo().Table(big, 1 << 18, 16384)
+    assert t.run_wire(wire) == 1
+    F = t.stats()["pages_used_max"]
+    t.close()
+    P = int(np.ceil(F / ratio)) + 2
+    t = sepo().Table(sepo().budget_for(1 << 18, 16384, P), 1 << 18, 16384, check_dups=True)
+    passes = t.run_wire(wire)
+    got = sepo().result_dict(t.export())
+    st = t.stats()
+    t.close()
+    assert got == exp
+    assert st["cross_gen_dups"] == 0
+    if ratio > 1:
+        assert passes >= 2
