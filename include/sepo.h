@@ -282,6 +282,45 @@ int64_t sepo_route_combine(const uint8_t* keys, const uint64_t* key_offsets, uin
  * mode only. Returns the number of passes or < 0. */
 int64_t sepo_run_wire(sepo_table* t, const void* wire, uint64_t n);
 
+/* ---- map runtime (the paper's MapReduce library): the map tasks of the
+ * paper's applications as built-in kernels that turn raw text into the records of one SEPO job (map
+ * callbacks cannot cross a C ABI as device code).
+ *   SEPO_MAP_WORDS     MAP_REDUCE, COMBINE table: every word -> (word, 1)   (Word Count)
+ *                      = sepo_run_text (tokenizer fused into the insert kernel)
+ *   SEPO_MAP_LINES     MAP_REDUCE, COMBINE table: every non-empty line (bytes other than '\n') -> (line, 1)
+ *                      (Page View Count on a log of URLs, one per line)
+ *   SEPO_MAP_WORD_DOCS MAP_GROUP, GROUP table with fixed_val_width 4: every word -> (word, u32 doc id),
+ *                      doc d = text bytes [doc_offsets[d], doc_offsets[d+1]) (Inverted Index)
+ * text, doc_offsets (n_docs entries, ascending, doc_offsets[0] = 0): device memory. Words follow reading
+ * R20. The mapped batch lives in table-owned scratch; the whole SEPO job runs as sepo_run (all passes, final
+ * eviction). Returns the number of passes or < 0. */
+enum { SEPO_MAP_WORDS = 0, SEPO_MAP_LINES = 1, SEPO_MAP_WORD_DOCS = 2 };
+int64_t sepo_map_run(sepo_table* t, int mapper, const uint8_t* text, uint64_t n_bytes, const uint64_t* doc_offsets,
+                     uint64_t n_docs);
+
+/* ---- the multi-GPU data plane inside the library (one process per GPU; NCCL over NVLink / NVSwitch)
+ * sepo_nccl_unique_id: 128 bytes for out_id (ncclGetUniqueId) — rank 0 creates it, the caller
+ *   broadcasts it (e.g. torch.distributed) to every rank.
+ * sepo_attach_nccl: joins the table to a communicator of nranks (1..32) ranks (ncclCommInitRank on the
+ *   table's device; collective). SEPO_E_NCCL on NCCL errors (sticky), SEPO_E_STATE if one is attached.
+ * sepo_insert_batch_sharded: COLLECTIVE over the attached ranks (every rank calls it, n may be 0).
+ *   The batch (device arrays as sepo_insert_batch; fixed-width values only) is routed by key owner
+ *   owner(k) = hi32(H(route seed, k)) * nranks >> 32 — COMBINE batches of keys <= 16 bytes as
+ *   pre-combined wire records (sepo_route_combine), others as a CSR partition (sepo_partition) —
+ *   the parts are exchanged with NCCL send/recv (counts, then payloads, each one NCCL group on the
+ *   table's stream), and the records this rank owns are appended to a table-owned buffer. A table
+ *   holds one format at a time (wire or CSR: SEPO_E_INVAL on a mix). Returns the records held.
+ * sepo_drain: the SEPO job on the records held (as sepo_run: insert, postpone, evict, re-issue until
+ *   nothing is postponed; the final generation goes to host memory), then the buffer is emptied.
+ *   No communication: postponed records are never re-routed, a key's records all live on its owner,
+ *   so each rank's sepo_export is final and the union over ranks is the result (no merge).
+ *   Returns the number of passes or < 0. */
+int sepo_nccl_unique_id(void* out_id);
+int sepo_attach_nccl(sepo_table* t, const void* nccl_unique_id, int nranks, int rank);
+int64_t sepo_insert_batch_sharded(sepo_table* t, const uint8_t* keys, const uint64_t* key_offsets, const uint8_t* vals,
+                                  const uint64_t* val_offsets, uint64_t n);
+int64_t sepo_drain(sepo_table* t);
+
 const char* sepo_last_error(void);
 const char* sepo_version(void);
 

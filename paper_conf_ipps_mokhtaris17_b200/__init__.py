@@ -60,12 +60,23 @@ class SepoError(RuntimeError):
 
 E_INVAL, E_NOMEM, E_TOOLARGE, E_CUDA, E_STATE, E_NCCL = -1, -2, -3, -4, -5, -6
 POOL_DEVICE, POOL_HOST_PINNED, POOL_MANAGED = 0, 1, 2  # sepo_create_placed (include/sepo.h)
+MAP_WORDS, MAP_LINES, MAP_WORD_DOCS = 0, 1, 2  # sepo_map_run mappers (include/sepo.h)
 
 # every entry point declared in include/sepo.h
 EXPORTS = ["sepo_create", "sepo_create_placed", "sepo_configure", "sepo_run_text", "sepo_lookup", "sepo_insert_batch", "sepo_reprobe", "sepo_compact", "sepo_evict",
            "sepo_export", "sepo_run", "sepo_reset", "sepo_stats_get", "sepo_last_insert_ms", "sepo_destroy",
            "sepo_last_error", "sepo_version", "sepo_budget_for", "sepo_partition_scratch", "sepo_partition",
-           "sepo_shift_offsets", "sepo_route_scratch", "sepo_route_combine", "sepo_run_wire"]
+           "sepo_shift_offsets", "sepo_route_scratch", "sepo_route_combine", "sepo_run_wire", "sepo_nccl_unique_id",
+           "sepo_attach_nccl", "sepo_insert_batch_sharded", "sepo_drain", "sepo_map_run"]
+
+
+def nccl_unique_id():
+    """128-byte NCCL unique id (rank 0 creates it; broadcast it to the other ranks)"""
+    buf = ctypes.create_string_buffer(128)
+    rc = lib().sepo_nccl_unique_id(buf)
+    if rc:
+        _err(rc)
+    return buf.raw
 
 
 def budget_for(n_buckets, page_bytes, pool_pages):
@@ -99,6 +110,11 @@ def lib():
         L.sepo_version.restype = ctypes.c_char_p
         L.sepo_budget_for.argtypes = [u64, u32, u64]; L.sepo_budget_for.restype = ctypes.c_size_t
         L.sepo_run_wire.argtypes = [vp, vp, u64]; L.sepo_run_wire.restype = i64
+        L.sepo_nccl_unique_id.argtypes = [vp]; L.sepo_nccl_unique_id.restype = ctypes.c_int
+        L.sepo_attach_nccl.argtypes = [vp, vp, ctypes.c_int, ctypes.c_int]; L.sepo_attach_nccl.restype = ctypes.c_int
+        L.sepo_insert_batch_sharded.argtypes = [vp, vp, vp, vp, vp, u64]; L.sepo_insert_batch_sharded.restype = i64
+        L.sepo_drain.argtypes = [vp]; L.sepo_drain.restype = i64
+        L.sepo_map_run.argtypes = [vp, ctypes.c_int, vp, u64, vp, u64]; L.sepo_map_run.restype = i64
         _LIB = L
     return _LIB
 
@@ -227,6 +243,36 @@ class Table:
         {key words, value, length} as sepo_route_combine writes them."""
         n = int(n) if n is not None else wire.numel() // 32
         rc = self._L.sepo_run_wire(self.h, _ptr(wire), n)
+        if rc < 0:
+            _err(rc)
+        return int(rc)
+
+    # ---- map runtime (NEXT-4): built-in mappers of the paper's applications on raw text
+    def map_run(self, mapper, text, doc_offsets=None):
+        """sepo_map_run: MAP_WORDS / MAP_LINES (COMBINE) or MAP_WORD_DOCS (GROUP, doc_offsets device int64)"""
+        nd = doc_offsets.numel() if doc_offsets is not None else 0
+        rc = self._L.sepo_map_run(self.h, int(mapper), _ptr(text), text.numel(), _ptr(doc_offsets), nd)
+        if rc < 0:
+            _err(rc)
+        return int(rc)
+
+    # ---- the multi-GPU data plane in the library (NCCL): attach, route + exchange, drain
+    def attach_nccl(self, unique_id, nranks, rank):
+        buf = ctypes.create_string_buffer(bytes(unique_id), 128)
+        rc = self._L.sepo_attach_nccl(self.h, buf, int(nranks), int(rank))
+        if rc:
+            _err(rc)
+
+    def insert_batch_sharded(self, keys, key_offsets, vals=None, n=None):
+        """collective: route by key owner + NCCL exchange; returns the records this rank holds"""
+        n = self._n(key_offsets, keys, n) if (keys is not None or key_offsets is not None) else 0
+        rc = self._L.sepo_insert_batch_sharded(self.h, _ptr(keys), _ptr(key_offsets), _ptr(vals), None, n)
+        if rc < 0:
+            _err(rc)
+        return int(rc)
+
+    def drain(self):
+        rc = self._L.sepo_drain(self.h)
         if rc < 0:
             _err(rc)
         return int(rc)

@@ -23,6 +23,9 @@
 #include "sepo.h"
 #include "sepo_dev.cuh"
 #include "sepo_kernels.h"
+#if SEPO_WITH_NCCL
+#include <nccl.h>
+#endif
 
 using namespace sepo;
 
@@ -118,6 +121,12 @@ struct sepo_table {
     DevBuf prep[2];  // sepo_run COMBINE: prepared re-issue records (ping-pong)
     DevBuf prep_n;   // their device counters
     DevBuf lk_pages; // sepo_lookup: page ids of the generation being probed
+    // multi-GPU data plane (sepo_attach_nccl / sepo_insert_batch_sharded / sepo_drain)
+    void* nccl = nullptr;     // ncclComm_t
+    int nranks = 1, rank = 0;
+    int shard_fmt = 0;        // records held: 0 none yet, 1 wire records, 2 CSR (keys, offsets[, values])
+    DevBuf sh_send[3], sh_held[3], sh_tmp[3], sh_cnt;  // route output; records held; exchange scratch; counts
+    uint64_t sh_n = 0, sh_kb = 0, sh_vb = 0;          // records / key bytes / value bytes held
     bool lookup_done = false;
     std::vector<cudaEvent_t>* h2d_chunks = nullptr;  // sepo_run on host input: copy events of pass-1 chunks
     uint64_t h2d_chunk_records = 0;  // sepo_lookup restored old generations into the pool: no inserts until reset
@@ -1636,6 +1645,11 @@ void sepo_destroy(sepo_table* t) {
     t->tbm.release();
     t->lk_pages.release();
     t->bm.release();
+    for (int i = 0; i < 3; ++i) { t->sh_send[i].release(); t->sh_held[i].release(); t->sh_tmp[i].release(); }
+    t->sh_cnt.release();
+#if SEPO_WITH_NCCL
+    if (t->nccl) ncclCommDestroy((ncclComm_t)t->nccl);
+#endif
     for (auto& s : t->buf)
         for (auto& b : s) b.release();
     for (auto& b : t->in_stage) b.release();
@@ -1761,4 +1775,275 @@ int sepo_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const 
     int rc = sepo_launch_shift_offsets(ko, n, seg_rec, seg_base, n_segs, total, (cudaStream_t)stream);
     if (rc) return fail(SEPO_E_CUDA, std::string("shift_offsets: ") + cudaGetErrorString((cudaError_t)rc));
     return 0;
+}
+
+// ---------------------------------------------------------------- map runtime (NEXT-4)
+int64_t sepo_map_run(sepo_table* t, int mapper, const uint8_t* text, uint64_t n_bytes, const uint64_t* doc_offsets,
+                     uint64_t n_docs) {
+    int rc = check_active(t);
+    if (rc) return rc;
+    if (mapper == SEPO_MAP_WORDS) return sepo_run_text(t, text, n_bytes);
+    if (mapper != SEPO_MAP_LINES && mapper != SEPO_MAP_WORD_DOCS) return fail(SEPO_E_INVAL, "unknown mapper");
+    if (mapper == SEPO_MAP_LINES && t->opts.mode != SEPO_COMBINE_SUM_U64) return fail(SEPO_E_INVAL, "MAP_LINES needs COMBINE");
+    if (mapper == SEPO_MAP_WORD_DOCS) {
+        if (t->opts.mode != SEPO_GROUP || t->opts.fixed_val_width != 4) return fail(SEPO_E_INVAL, "MAP_WORD_DOCS needs GROUP, fixed_val_width 4");
+        if (!doc_offsets || n_docs == 0 || n_docs > 0xffffffffull) return fail(SEPO_E_INVAL, "doc_offsets / n_docs");
+        if (!is_device_ptr(doc_offsets)) return fail(SEPO_E_INVAL, "doc_offsets must be device memory");
+    }
+    if (n_bytes && (!text || !is_device_ptr(text))) return fail(SEPO_E_INVAL, "text must be device memory");
+    if (t->opts.fixed_key_width) return fail(SEPO_E_INVAL, "map runs produce CSR keys (fixed_key_width must be 0)");
+    const int lines = mapper == SEPO_MAP_LINES;
+    const uint64_t nch = sepo_map_chunks(n_bytes);
+    if (t->tile_counts.grow((nch + 1) * 24)) return fail(SEPO_E_NOMEM, "map counts");
+    unsigned long long* tc = (unsigned long long*)t->tile_counts.p;
+    uint64_t tot[3] = {0, 0, 0};
+    if (nch) {
+        rc = sepo_launch_map(text, n_bytes, lines, 0, tc, nullptr, 0, nullptr, nullptr, nullptr, t->stream);
+        if (rc) return cuda_check(t, (cudaError_t)rc, "map count");
+        CK(t, cudaMemcpyAsync(tot, tc + 3 * nch, 24, cudaMemcpyDeviceToHost, t->stream));
+        CK(t, cudaStreamSynchronize(t->stream));
+    }
+    const uint64_t m = tot[0], kbytes = tot[1];
+    // the mapped batch (table-owned scratch): key bytes, offsets, doc ids
+    if (t->buf[0][0].grow(kbytes + 16) || t->buf[0][1].grow((m + 1) * 8) ||
+        (mapper == SEPO_MAP_WORD_DOCS && t->buf[0][2].grow(m * 4 + 16)))
+        return fail(SEPO_E_NOMEM, "mapped batch");
+    uint8_t* okeys = (uint8_t*)t->buf[0][0].p;
+    uint64_t* oko = (uint64_t*)t->buf[0][1].p;
+    uint32_t* odoc = mapper == SEPO_MAP_WORD_DOCS ? (uint32_t*)t->buf[0][2].p : nullptr;
+    if (m) {
+        rc = sepo_launch_map(text, n_bytes, lines, 1, tc, doc_offsets, n_docs, okeys, oko, odoc, t->stream);
+        if (rc) return cuda_check(t, (cudaError_t)rc, "map write");
+    }
+    t->h_ko[3] = kbytes;
+    CK(t, cudaMemcpyAsync(oko + m, &t->h_ko[3], 8, cudaMemcpyHostToDevice, t->stream));
+    CK(t, cudaStreamSynchronize(t->stream));
+    return run_device(t, okeys, oko, (const uint8_t*)odoc, nullptr, m);
+}
+
+// ---------------------------------------------------------------- multi-GPU data plane (a12)
+// One process per GPU. sepo_insert_batch_sharded routes a batch by key owner (pre-combined wire
+// records for COMBINE batches of keys <= 16 bytes, else a CSR partition), exchanges the parts with
+// NCCL point-to-point sends over NVLink (one ncclGroup: counts, then payloads), and appends what
+// this rank owns to a table-owned buffer; sepo_drain runs the SEPO job on it (insert, postpone,
+// evict, re-issue until nothing is postponed). Postponed records are never re-routed: a key's
+// records all live on its owner, so every rank's export is final (no merge).
+#if SEPO_WITH_NCCL
+namespace {
+const uint64_t kRouteSeed = 0x5eedull;  // owner hash seed (the library decorrelates it from table seeds)
+int nccl_check(sepo_table* t, ncclResult_t r, const char* what) {
+    if (r == ncclSuccess) return 0;
+    t->state = ST_BROKEN;
+    return fail(SEPO_E_NCCL, std::string(what) + ": " + ncclGetErrorString(r));
+}
+#define NK(t, expr)                                                  \
+    do {                                                             \
+        int _rc = nccl_check((t), (expr), #expr);                    \
+        if (_rc) return _rc;                                         \
+    } while (0)
+// append device bytes [src, src + bytes) to buffer b (holding `have` bytes)
+int append_dev(sepo_table* t, DevBuf& b, uint64_t have, const void* src, uint64_t bytes, DevBuf& tmp) {
+    if (!bytes) return 0;
+    if ((uint64_t)b.cap < have + bytes) {  // grow, keeping the contents
+        if (tmp.grow(have + bytes)) return fail(SEPO_E_NOMEM, "sharded buffer");
+        if (have) CK(t, cudaMemcpyAsync(tmp.p, b.p, have, cudaMemcpyDeviceToDevice, t->stream));
+        std::swap(b.p, tmp.p);
+        std::swap(b.cap, tmp.cap);
+    }
+    CK(t, cudaMemcpyAsync((uint8_t*)b.p + have, src, bytes, cudaMemcpyDeviceToDevice, t->stream));
+    return 0;
+}
+}  // namespace
+#endif
+
+int sepo_nccl_unique_id(void* out_id) {
+#if SEPO_WITH_NCCL
+    if (!out_id) return fail(SEPO_E_INVAL, "out_id is NULL");
+    ncclUniqueId id;
+    ncclResult_t r = ncclGetUniqueId(&id);
+    if (r != ncclSuccess) return fail(SEPO_E_NCCL, ncclGetErrorString(r));
+    memcpy(out_id, &id, sizeof(id));
+    return 0;
+#else
+    (void)out_id;
+    return fail(SEPO_E_NCCL, "built without NCCL");
+#endif
+}
+
+int sepo_attach_nccl(sepo_table* t, const void* nccl_unique_id, int nranks, int rank) {
+    int rc = check_active(t);
+    if (rc) return rc;
+    if (!nccl_unique_id || nranks < 1 || nranks > 32 || rank < 0 || rank >= nranks)
+        return fail(SEPO_E_INVAL, "attach: id / nranks in 1..32 / rank");
+#if SEPO_WITH_NCCL
+    if (t->nccl) return fail(SEPO_E_STATE, "a communicator is attached already");
+    CK(t, cudaSetDevice(t->device));
+    ncclUniqueId id;
+    memcpy(&id, nccl_unique_id, sizeof(id));
+    ncclComm_t comm;
+    NK(t, ncclCommInitRank(&comm, nranks, id, rank));
+    t->nccl = comm;
+    t->nranks = nranks;
+    t->rank = rank;
+    return 0;
+#else
+    return fail(SEPO_E_NCCL, "built without NCCL");
+#endif
+}
+
+int64_t sepo_insert_batch_sharded(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals,
+                                  const uint64_t* vo, uint64_t n) {
+    int rc = check_active(t);
+    if (rc) return rc;
+#if SEPO_WITH_NCCL
+    if (!t->nccl) return fail(SEPO_E_STATE, "no communicator (sepo_attach_nccl)");
+    if (vo) return fail(SEPO_E_INVAL, "sharded batches take fixed-width values");
+    if (n && !(is_device_ptr(keys) && is_device_ptr(ko) && is_device_ptr(vals))) return fail(SEPO_E_INVAL, "device inputs only");
+    const uint32_t P = (uint32_t)t->nranks;
+    const uint32_t kw = t->opts.fixed_key_width, vw = vals ? t->opts.fixed_val_width : 0u;
+    ncclComm_t comm = (ncclComm_t)t->nccl;
+    cudaStream_t s = t->stream;
+    if (t->sh_cnt.grow(8 * (6 * (size_t)P + 64))) return fail(SEPO_E_NOMEM, "count scratch");
+    uint64_t* dsend = (uint64_t*)t->sh_cnt.p;   // [P][3]: records, key bytes, value bytes per destination
+    uint64_t* drecv = dsend + 3 * P;             // [P][3] from each source
+    std::vector<uint64_t> send(3 * P, 0), recv(3 * P, 0);
+    // ---- route: pre-combined wire records (COMBINE, keys <= 16 bytes), else a CSR partition
+    int fmt = 0;
+    int64_t m = -1;
+    std::vector<uint64_t> pc(P + 1, 0);
+    if (t->opts.mode == SEPO_COMBINE_SUM_U64 && t->shard_fmt != 2 && n) {
+        void* scr = nullptr;
+        if (t->sh_tmp[2].grow(sepo_route_scratch(P))) return fail(SEPO_E_NOMEM, "route scratch");
+        scr = t->sh_tmp[2].p;
+        m = sepo_route_combine(keys, ko, kw, vals, vw, n, P, kRouteSeed, nullptr, 0, pc.data(), scr, sepo_route_scratch(P), s);
+        if (m >= 0) {
+            if (t->sh_send[0].grow((size_t)std::max<int64_t>(m, 1) * sizeof(WireRec))) return fail(SEPO_E_NOMEM, "wire send buffer");
+            m = sepo_route_combine(keys, ko, kw, vals, vw, n, P, kRouteSeed, t->sh_send[0].p, (uint64_t)m, pc.data(), scr,
+                                   sepo_route_scratch(P), s);
+            if (m < 0) return m;
+            fmt = 1;
+            for (uint32_t p = 0; p < P; ++p) send[3 * p] = pc[p + 1] - pc[p];
+        } else if (m != SEPO_E_TOOLARGE) {
+            return m;
+        }
+    }
+    if (!fmt && n) {
+        if (t->shard_fmt == 1) return fail(SEPO_E_INVAL, "a batch with keys longer than 16 bytes after wire batches");
+        const uint64_t kbytes = ko ? 0 : n * (uint64_t)kw;
+        uint64_t k0 = 0, kend = kbytes;
+        if (ko) {
+            CK(t, cudaMemcpy(&k0, ko, 8, cudaMemcpyDeviceToHost));
+            CK(t, cudaMemcpy(&kend, ko + n, 8, cudaMemcpyDeviceToHost));
+        }
+        if (t->sh_send[0].grow(kend - k0 + 16) || (ko && t->sh_send[1].grow((n + 1) * 8)) ||
+            (vals && t->sh_send[2].grow(n * (uint64_t)vw + 16)) || t->sh_tmp[2].grow(sepo_partition_scratch(n, P)))
+            return fail(SEPO_E_NOMEM, "partition buffers");
+        std::vector<uint64_t> st(3 * (P + 1));
+        rc = sepo_partition(keys, ko, kw, vals, vw, n, P, kRouteSeed, (uint8_t*)t->sh_send[0].p,
+                            ko ? (uint64_t*)t->sh_send[1].p : nullptr, vals ? (uint8_t*)t->sh_send[2].p : nullptr, st.data(),
+                            t->sh_tmp[2].p, sepo_partition_scratch(n, P), s);
+        if (rc) return rc;
+        fmt = 2;
+        for (uint32_t p = 0; p < P; ++p)
+            for (int c = 0; c < 3; ++c) send[3 * p + c] = st[3 * (p + 1) + c] - st[3 * p + c];
+        for (uint32_t p = 0; p < P; ++p) pc[p] = st[3 * p];
+    }
+    if (!fmt) fmt = t->shard_fmt ? t->shard_fmt : 1;  // (an empty batch: nothing to send, counts still exchanged)
+    // ---- counts (every rank takes part, also with n == 0)
+    CK(t, cudaMemcpyAsync(dsend, send.data(), 8 * 3 * P, cudaMemcpyHostToDevice, s));
+    NK(t, ncclGroupStart());
+    for (uint32_t p = 0; p < P; ++p) {
+        NK(t, ncclSend(dsend + 3 * p, 3, ncclUint64, (int)p, comm, s));
+        NK(t, ncclRecv(drecv + 3 * p, 3, ncclUint64, (int)p, comm, s));
+    }
+    NK(t, ncclGroupEnd());
+    CK(t, cudaMemcpyAsync(recv.data(), drecv, 8 * 3 * P, cudaMemcpyDeviceToHost, s));
+    CK(t, cudaStreamSynchronize(s));
+    // (a rank whose batch was empty learns the format from its peers' counts: wire batches send no key bytes)
+    uint64_t rn = 0, rk = 0, rv = 0;
+    for (uint32_t p = 0; p < P; ++p) { rn += recv[3 * p]; rk += recv[3 * p + 1]; rv += recv[3 * p + 2]; }
+    if (rk && fmt == 1 && !n) fmt = 2;
+    if (t->shard_fmt && t->shard_fmt != fmt && rn) return fail(SEPO_E_INVAL, "mixed wire / CSR sharded batches");
+    // ---- payloads into receive scratch, then appended to the records held
+    const uint64_t rb0 = fmt == 1 ? rn * sizeof(WireRec) : rk;
+    if (t->sh_tmp[0].grow(rb0 + 16) || (fmt == 2 && t->sh_tmp[1].grow((rn + 1) * 8)) || (fmt == 2 && t->sh_tmp[2].grow(rv + 16)))
+        return fail(SEPO_E_NOMEM, "receive buffers");
+    NK(t, ncclGroupStart());
+    uint64_t so = 0, ro = 0, sko = 0, rko = 0, svo = 0, rvo = 0;
+    for (uint32_t p = 0; p < P; ++p) {
+        if (fmt == 1) {
+            const uint64_t sb = send[3 * p] * sizeof(WireRec), rbb = recv[3 * p] * sizeof(WireRec);
+            if (sb) NK(t, ncclSend((uint8_t*)t->sh_send[0].p + pc[p] * sizeof(WireRec), sb, ncclUint8, (int)p, comm, s));
+            if (rbb) NK(t, ncclRecv((uint8_t*)t->sh_tmp[0].p + ro, rbb, ncclUint8, (int)p, comm, s));
+            ro += rbb;
+        } else {
+            if (send[3 * p + 1]) NK(t, ncclSend((uint8_t*)t->sh_send[0].p + so, send[3 * p + 1], ncclUint8, (int)p, comm, s));
+            if (recv[3 * p + 1]) NK(t, ncclRecv((uint8_t*)t->sh_tmp[0].p + ro, recv[3 * p + 1], ncclUint8, (int)p, comm, s));
+            if (ko && send[3 * p]) NK(t, ncclSend((uint64_t*)t->sh_send[1].p + sko, send[3 * p], ncclUint64, (int)p, comm, s));
+            if (recv[3 * p] && (ko || t->opts.fixed_key_width == 0))
+                NK(t, ncclRecv((uint64_t*)t->sh_tmp[1].p + rko, recv[3 * p], ncclUint64, (int)p, comm, s));
+            if (vals && send[3 * p + 2]) NK(t, ncclSend((uint8_t*)t->sh_send[2].p + svo, send[3 * p + 2], ncclUint8, (int)p, comm, s));
+            if (recv[3 * p + 2]) NK(t, ncclRecv((uint8_t*)t->sh_tmp[2].p + rvo, recv[3 * p + 2], ncclUint8, (int)p, comm, s));
+            so += send[3 * p + 1]; ro += recv[3 * p + 1]; sko += send[3 * p]; rko += recv[3 * p];
+            svo += send[3 * p + 2]; rvo += recv[3 * p + 2];
+        }
+    }
+    NK(t, ncclGroupEnd());
+    DevBuf scratch;
+    if (fmt == 1) {
+        rc = append_dev(t, t->sh_held[0], t->sh_n * sizeof(WireRec), t->sh_tmp[0].p, rn * sizeof(WireRec), scratch);
+        if (rc) { scratch.release(); return rc; }
+    } else if (rn) {
+        // received offsets are relative to each sender's segment: rebase them onto the key bytes held
+        const bool csr = ko || t->opts.fixed_key_width == 0;
+        if (csr) {
+            std::vector<uint64_t> seg_rec(P), seg_base(P);
+            uint64_t r = 0, kb = 0;
+            for (uint32_t p = 0; p < P; ++p) { seg_rec[p] = r; seg_base[p] = t->sh_kb + kb; r += recv[3 * p]; kb += recv[3 * p + 1]; }
+            uint64_t* dseg = drecv + 3 * P;  // (2P words after the counts)
+            CK(t, cudaMemcpyAsync(dseg, seg_rec.data(), 8 * P, cudaMemcpyHostToDevice, s));
+            CK(t, cudaMemcpyAsync(dseg + P, seg_base.data(), 8 * P, cudaMemcpyHostToDevice, s));
+            rc = sepo_launch_shift_offsets((uint64_t*)t->sh_tmp[1].p, rn, dseg, dseg + P, P, t->sh_kb + rk, s);
+            if (rc) { scratch.release(); return cuda_check(t, (cudaError_t)rc, "shift offsets"); }
+            // held offsets: n + 1 entries (the last one is rewritten by each append)
+            const uint64_t have = t->sh_n ? t->sh_n * 8 : 0;
+            rc = append_dev(t, t->sh_held[1], have, t->sh_tmp[1].p, (rn + 1) * 8, scratch);
+            if (rc) { scratch.release(); return rc; }
+        }
+        rc = append_dev(t, t->sh_held[0], t->sh_kb, t->sh_tmp[0].p, rk, scratch);
+        if (!rc) rc = append_dev(t, t->sh_held[2], t->sh_vb, t->sh_tmp[2].p, rv, scratch);
+        if (rc) { scratch.release(); return rc; }
+    }
+    CK(t, cudaStreamSynchronize(s));
+    scratch.release();
+    if (rn) t->shard_fmt = fmt;
+    t->sh_n += rn;
+    t->sh_kb += fmt == 2 ? rk : 0;
+    t->sh_vb += fmt == 2 ? rv : 0;
+    return (int64_t)t->sh_n;
+#else
+    (void)keys; (void)ko; (void)vals; (void)vo; (void)n;
+    return fail(SEPO_E_NCCL, "built without NCCL");
+#endif
+}
+
+int64_t sepo_drain(sepo_table* t) {
+    int rc = check_active(t);
+    if (rc) return rc;
+    int64_t r = 0;
+    const uint64_t n = t->sh_n;
+    if (t->shard_fmt == 1) {
+        r = run_device(t, nullptr, nullptr, nullptr, nullptr, n, (const WireRec*)t->sh_held[0].p);
+    } else if (t->shard_fmt == 2) {
+        const bool csr = t->opts.fixed_key_width == 0;
+        r = run_device(t, (const uint8_t*)t->sh_held[0].p, csr ? (const uint64_t*)t->sh_held[1].p : nullptr,
+                       t->sh_vb ? (const uint8_t*)t->sh_held[2].p : nullptr, nullptr, n);
+    } else if (t->dirty) {
+        int64_t e = evict_impl(t, 0);
+        if (e < 0) return e;
+    }
+    if (r < 0) return r;
+    t->sh_n = t->sh_kb = t->sh_vb = 0;
+    t->shard_fmt = 0;
+    return r;
 }

@@ -3136,6 +3136,82 @@ __global__ void __launch_bounds__(256) text_bits_kernel(Dev d, Batch b, unsigned
     }
 }
 
+// ================================================================ map runtime (NEXT-4): built-in mappers
+// The paper's MapReduce library runs map tasks that emit key/value pairs straight into
+// the table (MAP_REDUCE -> combining organization, MAP_GROUP -> multi-valued). Map callbacks cannot
+// cross a C ABI as device code, so the runtime ships the mappers of the paper's applications as
+// kernels: every record of a text chunk becomes a (key, value) pair in a compacted CSR batch that
+// the SEPO job then consumes.
+//   MAP_LINES     : key = a line (maximal run of bytes other than '\n'), value 1 (Page View Count)
+//   MAP_WORD_DOCS : key = a word (reading R20), value = u32 id of the document holding it (Inverted
+//                   Index; documents given as byte offsets)
+// (MAP_WORDS, Word Count, is the fused tokenizer: sepo_run_text.) Two passes over chunks of MC bytes:
+// count the records starting in each chunk and their key bytes, scan, write.
+constexpr uint32_t MC = 256;
+__device__ __forceinline__ bool map_sep(uint32_t c, int lines) { return lines ? c == 0x0au : is_sep(c); }
+// records starting in chunk ch: a non-separator byte at the chunk start preceded by a separator (or
+// the text start), or after a separator inside the chunk
+__global__ void __launch_bounds__(256) map_count_kernel(const uint8_t* T, uint64_t n, int lines, unsigned long long* tc) {
+    const uint64_t nch = (n + MC - 1) / MC;
+    for (uint64_t ch = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; ch < nch; ch += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t a = ch * MC, z = min(a + MC, n);
+        unsigned long long cnt = 0, bytes = 0;
+        bool prev_sep = a == 0 || map_sep(T[a - 1], lines);
+        uint64_t i = a;
+        while (i < z) {
+            const bool sp = map_sep(T[i], lines);
+            if (!sp && prev_sep) {  // a record starts at i: measure it (it may run past the chunk)
+                uint64_t e = i;
+                while (e < n && !map_sep(T[e], lines)) ++e;
+                ++cnt;
+                bytes += e - i;
+                i = e;
+                prev_sep = false;
+                continue;
+            }
+            prev_sep = sp;
+            ++i;
+        }
+        tc[3 * ch] = cnt;
+        tc[3 * ch + 1] = bytes;
+        tc[3 * ch + 2] = 0;
+    }
+}
+__global__ void __launch_bounds__(256) map_write_kernel(const uint8_t* T, uint64_t n, int lines, const unsigned long long* tc,
+                                                        const uint64_t* doc_offsets, uint64_t n_docs, uint8_t* okeys,
+                                                        uint64_t* oko, uint32_t* odoc) {
+    const uint64_t nch = (n + MC - 1) / MC;
+    for (uint64_t ch = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; ch < nch; ch += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t a = ch * MC, z = min(a + MC, n);
+        uint64_t r = tc[3 * ch], kb = tc[3 * ch + 1];
+        bool prev_sep = a == 0 || map_sep(T[a - 1], lines);
+        uint64_t i = a;
+        while (i < z) {
+            const bool sp = map_sep(T[i], lines);
+            if (!sp && prev_sep) {
+                uint64_t e = i;
+                while (e < n && !map_sep(T[e], lines)) { okeys[kb + (e - i)] = T[e]; ++e; }
+                oko[r] = kb;
+                if (odoc) {  // the document holding byte i: the last d with doc_offsets[d] <= i
+                    uint64_t lo = 0, hi = n_docs - 1;
+                    while (lo < hi) {
+                        const uint64_t mid = lo + ((hi - lo + 1) >> 1);
+                        if (doc_offsets[mid] <= i) lo = mid; else hi = mid - 1;
+                    }
+                    odoc[r] = (uint32_t)lo;
+                }
+                ++r;
+                kb += e - i;
+                i = e;
+                prev_sep = false;
+                continue;
+            }
+            prev_sep = sp;
+            ++i;
+        }
+    }
+}
+
 // ================================================================ SEPO lookups (NEXT-4)
 // Lookups on the larger-than-memory table ("The SEPO model can also be used for lookup
 // operations on larger-than-memory hash tables"): the host streams the evicted generations back
@@ -3485,6 +3561,21 @@ int sepo_launch_partition(const Batch& b, uint32_t P, uint64_t seed, unsigned lo
     return cudaGetLastError();
 }
 uint64_t sepo_partition_tiles(uint64_t n) { return (n + PT_TILE - 1) / PT_TILE; }
+uint64_t sepo_map_chunks(uint64_t n) { return (n + MC - 1) / MC; }
+int sepo_launch_map(const uint8_t* text, uint64_t n, int lines, int pass, unsigned long long* tc, const uint64_t* doc_offsets,
+                    uint64_t n_docs, uint8_t* okeys, uint64_t* oko, uint32_t* odoc, cudaStream_t s) {
+    const uint64_t nch = (n + MC - 1) / MC;
+    if (!nch) return 0;
+    const int grid = (int)std::min<uint64_t>((nch + 255) / 256, 8 * 148);
+    if (pass == 0) {  // (tc has nch + 1 entries: after the scan the last one holds the totals)
+        cudaMemsetAsync(tc + 3 * nch, 0, 24, s);
+        map_count_kernel<<<grid, 256, 0, s>>>(text, n, lines, tc);
+        scan_tiles_kernel<<<1, 1024, 0, s>>>(tc, nch + 1);
+    } else {
+        map_write_kernel<<<grid, 256, 0, s>>>(text, n, lines, tc, doc_offsets, n_docs, okeys, oko, odoc);
+    }
+    return cudaGetLastError();
+}
 int sepo_launch_route_combine(const Batch& b, uint32_t P, uint64_t seed, int pass, unsigned long long* part_totals,
                               unsigned long long* long_keys, const unsigned long long* part_base,
                               unsigned long long* cursors, WireRec* out, int grid, cudaStream_t s) {

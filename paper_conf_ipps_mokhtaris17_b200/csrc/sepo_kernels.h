@@ -82,6 +82,11 @@ int sepo_launch_compact_index(const sepo::Batch& b, unsigned long long* tile_cou
 int sepo_launch_partition(const sepo::Batch& b, uint32_t P, uint64_t seed, unsigned long long* counts, uint8_t* ok,
                           uint64_t* oko, uint8_t* ov, unsigned long long* h_counts, int grid, cudaStream_t s);
 uint64_t sepo_partition_tiles(uint64_t n);
+// map runtime (NEXT-4): pass 0 counts records / key bytes per chunk of text into tc (3 u64 per chunk)
+// and scans them; pass 1 writes the compacted CSR (okeys, oko) and, with doc_offsets, u32 doc ids
+uint64_t sepo_map_chunks(uint64_t n);
+int sepo_launch_map(const uint8_t* text, uint64_t n, int lines, int pass, unsigned long long* tc, const uint64_t* doc_offsets,
+                    uint64_t n_docs, uint8_t* okeys, uint64_t* oko, uint32_t* odoc, cudaStream_t s);
 int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const uint64_t* seg_base, uint32_t n_segs,
                               uint64_t total, cudaStream_t s);
 int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);

@@ -190,3 +190,34 @@ def test_run_wire_vs_oracle(cuda, name, ratio):
     assert st["cross_gen_dups"] == 0
     if ratio > 1:
         assert passes >= 2
+
+
+# ---- the in-library NCCL data plane (sepo_attach_nccl / sepo_insert_batch_sharded / sepo_drain)
+@pytest.mark.parametrize("name,ratio", [("C2", 4), ("C5z", 4), ("C3", 2)])
+def test_nccl_sharded_one_rank(cuda, name, ratio):
+    """a one-rank NCCL communicator (the box has one GPU): the batch, split in 3 sharded calls, is
+    routed (wire records for words / pairs, a CSR partition for URLs), exchanged through NCCL
+    send/recv to itself and drained: the export equals the oracle"""
+    scale = {"C2": 1 / 512, "C5z": 2 ** -12, "C3": 1 / 8000}[name]
+    s = gen.config(name, scale=scale)
+    exp = oracle_expected(s)
+    k, o, v = s.device()
+    fixed = s.family == gen.GEN_PAIRS
+    kw = dict(fixed_key_width=8, fixed_val_width=8) if fixed else {}
+    pb = 65536 if name == "C3" else 16384
+    t = sepo().Table(sepo().budget_for(1 << 16, pb, 1 << 12), 1 << 16, pb, **kw)
+    t.attach_nccl(sepo().nccl_unique_id(), 1, 0)
+    n = s.n
+    cuts = [0, n // 3, 2 * n // 3, n]
+    held = 0
+    for a, b in zip(cuts[:-1], cuts[1:]):
+        if fixed:
+            held = t.insert_batch_sharded(k[8 * a:8 * b], None, v[8 * a:8 * b], n=b - a)
+        else:
+            held = t.insert_batch_sharded(k, o[a:b + 1].contiguous(), None, n=b - a)
+    assert held > 0
+    passes = t.drain()
+    got = sepo().result_dict(t.export())
+    t.close()
+    assert passes >= 1
+    assert got == exp

@@ -120,3 +120,63 @@ def test_text_host_pipelined(cuda, monkeypatch, chunk):
     exp2 = oracle.word_count_text(np.frombuffer(t, dtype=np.uint8))
     got, _, _ = run_text(np.frombuffer(t, dtype=np.uint8).copy(), 256, pb=8192)
     assert got == exp2
+
+
+# ---- map runtime (NEXT-4): the paper's applications from raw text (sepo_map_run)
+def test_map_lines_page_view_count(cuda):
+    """MAP_LINES: one URL per line -> (URL, 1) combined == the oracle's count of the lines"""
+    s = gen.config("C3", scale=1 / 8000)
+    keys, offs, _ = s.host()
+    kb = keys.tobytes()
+    lines = [kb[offs[i]:offs[i + 1]] for i in range(s.n)]
+    text = b"\n".join(lines) + b"\n\n"
+    exp = {}
+    for ln in lines:
+        exp[ln] = exp.get(ln, 0) + 1
+    S = sepo()
+    t = S.Table(S.budget_for(1 << 14, 65536, 256), 1 << 14, 65536, check_dups=True)
+    d = torch.from_numpy(np.frombuffer(text, dtype=np.uint8).copy()).cuda()
+    passes = t.map_run(S.MAP_LINES, d)
+    got = S.result_dict(t.export())
+    t.close()
+    assert passes >= 1 and got == exp
+    assert exp == s.expected_combine()
+
+
+@pytest.mark.parametrize("budget_pages", [4096, 40])
+def test_map_word_docs_inverted_index(cuda, budget_pages):
+    """MAP_WORD_DOCS: documents of words -> (word, doc id) grouped == oracle.group over the same pairs,
+    in one pass and over budget"""
+    rng = np.random.default_rng(4)
+    s = gen.config("C1", scale=0.05)
+    text = s.text_host()
+    n = len(text)
+    cuts = np.sort(rng.choice(np.arange(1, n), size=40, replace=False))
+    doc_offsets = np.concatenate([[0], cuts]).astype(np.int64)
+    # oracle pairs: every word with the document holding its first byte
+    tb = text.tobytes()
+    words, docs = [], []
+    i = 0
+    seps = b" \n\t\r"
+    while i < n:
+        if tb[i] in seps:
+            i += 1
+            continue
+        j = i
+        while j < n and tb[j] not in seps:
+            j += 1
+        words.append(tb[i:j])
+        docs.append(int(np.searchsorted(doc_offsets, i, side="right") - 1))
+        i = j
+    ko = np.zeros(len(words) + 1, dtype=np.uint64)
+    ko[1:] = np.cumsum([len(w) for w in words])
+    vals = np.array(docs, dtype=np.uint32).view(np.uint8)
+    exp = oracle.group(np.frombuffer(b"".join(words), dtype=np.uint8), ko, vals, val_width=4).as_dict()
+    S = sepo()
+    t = S.Table(S.budget_for(1 << 14, 4096, budget_pages), 1 << 14, 4096, mode=S.GROUP, fixed_val_width=4, check_dups=True)
+    passes = t.map_run(S.MAP_WORD_DOCS, torch.from_numpy(text.copy()).cuda(), torch.from_numpy(doc_offsets).cuda())
+    got = S.result_dict(t.export(), S.GROUP)
+    t.close()
+    assert got == exp
+    if budget_pages < 100:
+        assert passes >= 2

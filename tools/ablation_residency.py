@@ -30,6 +30,7 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--ratios", default="1,2,4")
     ap.add_argument("--out", default=None)
+    ap.add_argument("--oversub", default="1,2,4", help="managed pool with HBM capped to F/k (k list; '' skips)")
     a = ap.parse_args()
     import torch
     import bench
@@ -83,8 +84,31 @@ def main():
         t0 = time.time()
         row(name, sepo.Table(sepo.budget_for(nb_full, base.page_bytes, fit_pages), nb_full, base.page_bytes,
                              host_arena_bytes=arena, placement=pl, **base.kw), {"ratio": 1.0, "wall_s": time.time() - t0})
+    # managed pool OVERSUBSCRIBED (NEXT-1 (ii), the Table III analogue): the same pool
+    # with device memory capped by a balloon so that only F/k of it fits in HBM at once — the driver
+    # demand-pages the table in and evicts pages back to host memory during the job
+    if a.oversub:
+        for kk in [float(x) for x in a.oversub.split(",")]:
+            t = sepo.Table(sepo.budget_for(nb_full, base.page_bytes, fit_pages), nb_full, base.page_bytes,
+                           host_arena_bytes=arena, placement=sepo.POOL_MANAGED, **base.kw)
+            t.reset(); t.run(k, o, v)  # every library buffer allocated before the balloon
+            torch.cuda.synchronize()
+            free, _ = torch.cuda.mem_get_info()
+            leave = int(F / kk) + (8 << 20)
+            balloon = torch.empty(max(free - leave, 0), dtype=torch.uint8, device="cuda") if free > leave else None
+            torch.cuda.synchronize()
+            t0 = time.time()
+            try:
+                row(f"managed_oversub_{kk:g}x", t, {"ratio": kk, "device_free_for_pool": leave, "wall_s": time.time() - t0})
+            except Exception as e:  # (an allocation inside the job failed under the cap)
+                out["rows"].append({"name": f"managed_oversub_{kk:g}x", "error": str(e)[:200]})
+                print(json.dumps(out["rows"][-1]), flush=True)
+            del balloon
+            torch.cuda.empty_cache()
     fit = out["rows"][0]["ms"]
     for r in out["rows"]:
+        if "ms" not in r:
+            continue
         r["slowdown_vs_device_fit"] = r["ms"] / fit
     print(json.dumps(out), flush=True)
     if a.out:
