@@ -126,8 +126,10 @@ class Job:
 
     def table_params(self):
         pages_F, F = self.footprint()
-        if self.ratio <= 1.0:  # (SEPO_BENCH_NB_IB: directory multiple for in-budget tables, experiments)
-            nb = self.nb_full * int(os.environ.get("SEPO_BENCH_NB_IB", "1"))
+        if self.ratio <= 1.0:
+            # in-budget tables: twice as many buckets as keys (load ~0.5: shorter chains for the misses
+            # that go to HBM; C2 0.5x pass 1 28.5 -> 25.8 ms). SEPO_BENCH_NB_IB overrides the multiple.
+            nb = self.nb_full * int(os.environ.get("SEPO_BENCH_NB_IB", "2"))
             pages = int(np.ceil(pages_F / self.ratio)) if self.ratio < 1 else pages_F + 8
         else:  # directory: the largest power of two <= 2x the keys of one generation (load <= ~1)
             mult = float(os.environ.get("SEPO_BENCH_NB_MULT", "2"))

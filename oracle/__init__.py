@@ -30,7 +30,6 @@ def lib():
         L.oracle_combine_add_text.argtypes = [vp, vp, u64]
         L.oracle_combine_size.argtypes = [vp, vp]; L.oracle_combine_size.restype = u64
         L.oracle_combine_result.argtypes = [vp, vp, vp, vp]
-        L.oracle_combine_get.argtypes = [vp, vp, u64, vp]; L.oracle_combine_get.restype = u64
         L.oracle_group_new.restype = vp
         L.oracle_group_free.argtypes = [vp]
         L.oracle_group_add.argtypes = [vp, vp, vp, vp, vp, u32, u64]
@@ -89,12 +88,6 @@ class Combine:
         vals = np.empty(k, dtype=np.uint64)
         lib().oracle_combine_result(self.h, _p(keys), _p(offs), _p(vals))
         return keys, offs, vals
-
-    def get(self, key):
-        f = ctypes.c_int()
-        kk = _u8(key)
-        v = lib().oracle_combine_get(self.h, _p(kk), len(kk), ctypes.byref(f))
-        return v if f.value else None
 
     def as_dict(self):
         keys, offs, vals = self.result()

@@ -100,14 +100,6 @@ void oracle_combine_result(void* h, uint8_t* keys, uint64_t* offs, uint64_t* val
     }
     offs[c->sorted.size()] = o;
 }
-/* value of one key (sampled checks at full size); returns 0 if absent, sets *found */
-uint64_t oracle_combine_get(void* h, const uint8_t* key, uint64_t klen, int* found) {
-    Combine* c = (Combine*)h;
-    auto it = c->m.find(std::string((const char*)key, (size_t)klen));
-    *found = it != c->m.end();
-    return *found ? it->second : 0;
-}
-
 /* ------------------------------------------------------------------ multi-valued group-by */
 void* oracle_group_new(void) { return new Group(); }
 void oracle_group_free(void* h) { delete (Group*)h; }

@@ -129,14 +129,8 @@ constexpr uint32_t ANN_STRIDE = 16;  // u64 words between announcement words (12
 // The streamed input (16 GB for C2) would otherwise push table lines out of L2: on B200 a 55 MB
 // table next to an evict_normal input stream missed L2 on 58 % of its sectors (ncu, pass 1 of the
 // C2 4x job: 71 GB DRAM read for 16 GB of input). Input loads therefore carry an L2 evict_first
-// policy (and skip L1 allocation); table accesses keep the default (or evict_last, SEPO_TAB_POLICY).
+// policy (and skip L1 allocation); table accesses keep the default policy.
 // createpolicy with a constant fraction folds into the load's memory descriptor (no extra SASS).
-#ifndef SEPO_IN_POLICY
-#define SEPO_IN_POLICY 1
-#endif
-#ifndef SEPO_TAB_POLICY
-#define SEPO_TAB_POLICY 0
-#endif
 __device__ __forceinline__ uint64_t pol_in() {
     uint64_t p;
     asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
@@ -149,73 +143,43 @@ __device__ __forceinline__ uint64_t pol_tab() {
 }
 // immutable input (keys, offsets, values, re-issue indices): read-only path, L2 evict_first
 __device__ __forceinline__ uint64_t ld_in64(const void* p) {
-#if SEPO_IN_POLICY
     uint64_t v;
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol_in()));
     return v;
-#else
-    return __ldg(reinterpret_cast<const unsigned long long*>(p));
-#endif
 }
 __device__ __forceinline__ uint32_t ld_in32(const void* p) {
-#if SEPO_IN_POLICY
     uint32_t v;
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol_in()));
     return v;
-#else
-    return __ldg(reinterpret_cast<const unsigned int*>(p));
-#endif
 }
 __device__ __forceinline__ uint32_t ld_in16(const void* p) {
-#if SEPO_IN_POLICY
     unsigned short v;
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u16 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol_in()));
     return v;
-#else
-    return __ldg(reinterpret_cast<const unsigned short*>(p));
-#endif
 }
 __device__ __forceinline__ uint32_t ld_in8(const void* p) {
-#if SEPO_IN_POLICY
     unsigned short v;
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.u8 %0, [%1], %2;" : "=h"(v) : "l"(p), "l"(pol_in()));
     return v & 0xffu;
-#else
-    return __ldg(reinterpret_cast<const unsigned char*>(p));
-#endif
 }
 __device__ __forceinline__ uint4 ld_in128(const void* p) {
-#if SEPO_IN_POLICY
     uint4 v;
     asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
         : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol_in()));
     return v;
-#else
-    return __ldg(reinterpret_cast<const uint4*>(p));
-#endif
 }
 
 // L2-coherent loads of published entry fields (never stale L1 lines)
 __device__ __forceinline__ uint64_t ldcg64(const void* p) { return __ldcg(reinterpret_cast<const unsigned long long*>(p)); }
 __device__ __forceinline__ uint32_t ldcg32(const void* p) { return __ldcg(reinterpret_cast<const unsigned int*>(p)); }
 
-#ifndef SEPO_TAIL_L1
-#define SEPO_TAIL_L1 1   // C3 pass 1 55.2 -> 50.4 ms
-#endif
-#ifndef SEPO_HEAD_L1
-#define SEPO_HEAD_L1 0   // the per-lane first-16-byte loads (long-key groups, index re-issue) L1-allocating too
-#endif
 // input words read lane by lane (key tails beyond the first 16 bytes): L1-allocating, so the
 // group's neighbouring keys (one 128-byte line holds two 64-byte URLs) are read from L1 after the
 // first lane's miss (L1::no_allocate sent every 8-byte tail load to L2: C3 pass 1 load-bound)
 __device__ __forceinline__ uint64_t ld_tail64(const void* p) {
-#if SEPO_TAIL_L1
     uint64_t v;
     asm("ld.global.nc.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol_in()));
     return v;
-#else
-    return ld_in64(p);
-#endif
 }
 // Bytes [p, p+nb) (1 <= nb <= 8) of immutable INPUT as a little-endian word, zero-extended.
 // Only the aligned words that contain requested bytes are read.
@@ -250,13 +214,7 @@ __device__ __forceinline__ uint64_t hash_word(uint64_t h, uint64_t w) {
 }
 // hash of a key given its first 16 bytes (w0, w1) and, for longer keys, its bytes at p
 __device__ __forceinline__ uint64_t hash_key16(uint32_t len, uint64_t seed, uint64_t w0, uint64_t w1, const uint8_t* p) {
-#ifdef SEPO_HASH_V5
-    uint64_t x = hash_init(len, seed);
-    if (len > 0) x = hash_word(x, w0);
-    if (len > 8) x = hash_word(x, w1);
-#else
     uint64_t x = hash_word(hash_word(hash_init(len, seed), w0), w1);
-#endif
     for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(p + o, len - o < 8 ? len - o : 8));
     return fmix64(x);
 }
@@ -305,28 +263,9 @@ __device__ __forceinline__ void store_key(uint8_t* ek, const uint8_t* p, uint32_
     }
 }
 
-#if SEPO_TAB_POLICY
-__device__ __forceinline__ uint4 ldcg128(const void* p) {
-    uint4 v;
-    asm volatile("ld.global.cg.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
-                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol_tab()));
-    return v;
-}
-__device__ __forceinline__ ulonglong2 ldcg128u(const void* p) {
-    ulonglong2 v;
-    asm volatile("ld.global.cg.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;" : "=l"(v.x), "=l"(v.y) : "l"(p), "l"(pol_tab()));
-    return v;
-}
-__device__ __forceinline__ uint32_t ld_dir(const uint32_t* p) {
-    uint32_t v;
-    asm volatile("ld.relaxed.gpu.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol_tab()) : "memory");
-    return v;
-}
-#else
 __device__ __forceinline__ uint4 ldcg128(const void* p) { return __ldcg(reinterpret_cast<const uint4*>(p)); }
 __device__ __forceinline__ ulonglong2 ldcg128u(const void* p) { return __ldcg(reinterpret_cast<const ulonglong2*>(p)); }
 __device__ __forceinline__ uint32_t ld_dir(const uint32_t* p) { return ld_relaxed_u32(p); }
-#endif
 
 // Walk the chain [ref .. stop) for an entry with (tag, len, key) — key given by its INPUT bytes.
 // Only entries of the resident generation are reachable (head insertion; the directory
@@ -366,15 +305,9 @@ __device__ __forceinline__ void load_key16(const uint8_t* p, uint32_t len, uint6
     const unsigned long long* q = reinterpret_cast<const unsigned long long*>(a - sh);
     const uint32_t nb = len < 16 ? len : 16;
     const uint32_t nw = (sh + nb + 7) >> 3;  // aligned words touched (1..3)
-#if SEPO_HEAD_L1
-    const uint64_t x0 = ld_tail64(q);
-    const uint64_t x1 = nw > 1 ? ld_tail64(q + 1) : 0ull;
-    const uint64_t x2 = nw > 2 ? ld_tail64(q + 2) : 0ull;
-#else
     const uint64_t x0 = ld_in64(q);
     const uint64_t x1 = nw > 1 ? ld_in64(q + 1) : 0ull;
     const uint64_t x2 = nw > 2 ? ld_in64(q + 2) : 0ull;
-#endif
     if (sh == 0) { w0 = x0; w1 = x1; }
     else {
         w0 = (x0 >> (8 * sh)) | (x1 << (64 - 8 * sh));
@@ -382,28 +315,6 @@ __device__ __forceinline__ void load_key16(const uint8_t* p, uint32_t len, uint6
     }
     if (nb < 8) { w0 &= (1ull << (8 * nb)) - 1ull; w1 = 0; }
     else if (nb < 16) w1 &= (1ull << (8 * (nb - 8))) - 1ull;
-}
-
-// ---------------------------------------------------------------- TMA bulk copies (global -> shared)
-__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void mbar_init(unsigned long long* bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
-__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
-// expect `bytes` on `bar` and start one bulk copy of `bytes` (multiple of 16, 16-B aligned ends)
-__device__ __forceinline__ void tma_load(void* dst, const void* src, uint32_t bytes, unsigned long long* bar) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(dst)),
-                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
-                 : "memory");
-}
-__device__ __forceinline__ void mbar_wait(unsigned long long* bar, uint32_t parity) {
-    asm volatile(
-        "{\n .reg .pred P;\n WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n @!P bra WAIT_%=;\n}\n" ::"r"(
-            smem_u32(bar)),
-        "r"(parity)
-        : "memory");
 }
 
 // ---------------------------------------------------------------- fault injection (tests only)

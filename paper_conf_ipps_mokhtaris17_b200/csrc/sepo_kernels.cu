@@ -20,18 +20,9 @@
 namespace sepo {
 
 
-#ifndef SEPO_LANEID_ASM
-#define SEPO_LANEID_ASM 0  // %laneid measured slower (C2 4x pass 1 22.0 vs 21.6 ms, text 30.8 vs 28.4 ms)
-#endif
-// lane id (SEPO_LANEID_ASM=1: from %laneid instead of threadIdx.x & 31)
+// lane id (threadIdx.x & 31: measured faster than reading %laneid, C2 4x pass 1 21.6 vs 22.0 ms)
 __device__ __forceinline__ uint32_t lane_id() {
-#if SEPO_LANEID_ASM
-    uint32_t l;
-    asm("mov.u32 %0, %%laneid;" : "=r"(l));
-    return l;
-#else
     return threadIdx.x & 31u;
-#endif
 }
 __device__ __forceinline__ uint32_t lanemask_lt() { return (1u << lane_id()) - 1u; }
 
@@ -176,12 +167,8 @@ namespace hot {
 #define SEPO_HOT_K 2048
 #endif
 constexpr int K = SEPO_HOT_K;    // hot keys at most (a power of two)
-constexpr int NB = 1024;         // shared buckets of 4 slots (2-choice): constant-time probe
-constexpr int NH = 4 * NB;       // slots
 constexpr uint32_t EMPTY_LEN = 0xffffffffu;
 __device__ __forceinline__ uint32_t fp(uint64_t h) { return (uint32_t)(h >> 32) | 1u; }  // 0 = empty
-__device__ __forceinline__ uint32_t b1(uint64_t h) { return (uint32_t)(h >> 3) & (NB - 1); }
-__device__ __forceinline__ uint32_t b2(uint64_t h) { return (uint32_t)(h >> 13) & (NB - 1); }
 constexpr int SAMPLE_SLOTS = 1 << 20;  // global scratch table for the sample
 struct Entry {                   // one hot key (global list, built by hot_select / hot_resolve)
     uint64_t h, w0, w1;
@@ -197,11 +184,7 @@ struct SampleSlot { unsigned long long h; unsigned int count, pad; unsigned long
 }  // namespace hot
 
 __device__ __forceinline__ void red_add_u64(unsigned long long* p, unsigned long long v) {
-#if SEPO_TAB_POLICY
-    asm volatile("red.relaxed.gpu.global.add.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(pol_tab()) : "memory");
-#else
     asm volatile("red.relaxed.gpu.global.add.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-#endif
 }
 
 // hash + first 16 key bytes of record i
@@ -362,28 +345,11 @@ __global__ void __launch_bounds__(1024) hot_resolve_kernel(Dev d, Batch b, hot::
 }
 
 namespace stream {
-#ifndef SEPO_DIR_ALL
-#define SEPO_DIR_ALL 1  // issue every record's directory load before the hot-set probe
-#endif
 #ifndef SEPO_STREAM_THREADS
 #define SEPO_STREAM_THREADS 1024  // one persistent CTA per SM (register-bound: 64 regs x 1024)
 #endif
 #ifndef SEPO_CHUNK_GROUPS
 #define SEPO_CHUNK_GROUPS 32      // consecutive 32-record groups a warp streams before it strides
-#endif
-#ifndef SEPO_S1_AHEAD
-#define SEPO_S1_AHEAD 2           // groups ahead the key offsets are loaded (2 or 3)
-#endif
-#ifndef SEPO_FOLD
-#define SEPO_FOLD 1               // fold equal hot keys of a warp before the shared atomic
-#endif
-#ifndef SEPO_IN_PREFETCH
-#define SEPO_IN_PREFETCH 0        // L2 prefetch of the input this many groups ahead (0: off)
-#endif
-#ifndef SEPO_DIR_PREFETCH
-#define SEPO_DIR_PREFETCH 0       // 1: always L2-prefetch a queued miss's directory word (default: host
-                                  // decides per table, c.dirpf: on when the budget exceeds L2 — C5u 4x
-                                  // insert 67.3 -> 61.0 ms, C2 in budget 28.6 -> 28.1 ms, C2 4x off)
 #endif
 constexpr int THREADS = SEPO_STREAM_THREADS;
 constexpr uint64_t CH = SEPO_CHUNK_GROUPS;
@@ -395,19 +361,12 @@ struct CtaState {                 // allocator slot (the CTA's active pages) + p
 };
 // Shared memory of the COMBINE stream kernel: the hot set (read-only keys + per-CTA pending sums)
 // and one miss queue per warp (records that missed the hot set, resolved 32 at a time).
-#ifndef SEPO_BRANCHLESS
-#define SEPO_BRANCHLESS 0
-#endif
-#ifndef SEPO_HOT_DIRECT
-#define SEPO_HOT_DIRECT 1  // direct-indexed hot set (C2 4x pass 1 22.2 -> 21.3 ms); 0: 4-way bucket fingerprints
-#endif
 // slot word of the direct-indexed hot sets: fingerprint (hash bits + the key length saturated at
 // 255) | 1 | key index (B bits); 0 marks an empty slot
 template <int B>
 __device__ __forceinline__ uint32_t dfp_b(uint64_t h, uint32_t len) {
     return ((((uint32_t)(h >> (64 - (23 - B))) << 8) | min(len, 255u)) << (B + 1)) | (1u << B);
 }
-#if SEPO_HOT_DIRECT
 // Direct-indexed hot set: DS one-word slots (2-choice, one slot per choice); a slot holds the key's
 // fingerprint and its index into the dense key arrays, so a probe is two 4-byte loads, two
 // compares and one 16-byte key load.
@@ -423,16 +382,9 @@ __device__ __forceinline__ uint32_t ds2(uint64_t h) { return (uint32_t)(h >> 17)
 __device__ __forceinline__ uint32_t dfp(uint64_t h, uint32_t len) {
     return dfp_b<IDXB>(h, len);
 }
-#else
-constexpr int NKEY = hot::NH;
-#endif
 template <bool VALS, int WARPS>
 struct Smem {
-#if SEPO_HOT_DIRECT
     uint32_t tags[DS];            // slot words (0: empty)
-#else
-    uint4 tags[hot::NB];          // 4 fingerprints per bucket (one 16-B load per probed bucket)
-#endif
     ulonglong2 kw[NKEY];          // first 16 key bytes, zero padded (one 16-B load per candidate)
     uint32_t ref[NKEY];           // resident entry (0: empty slot)
     typename std::conditional<VALS, unsigned long long, unsigned int>::type sum[NKEY];  // pending sums
@@ -448,12 +400,6 @@ struct Smem {
 static_assert(sizeof(Smem<true, SEPO_STREAM_THREADS / 32>) <= 232448, "stream kernel shared memory > 227 KB");
 #endif
 static_assert(sizeof(Smem<false, SEPO_STREAM_THREADS / 32>) <= 232448, "stream kernel shared memory > 227 KB");
-// Fingerprint of a hot slot: 23 hash bits, bit 8 always set (0 marks an empty slot) and the key
-// length (saturated at 255) in the low byte, so a fingerprint match also fixes the length of
-// keys shorter than 255 bytes and the full-key check is one 16-byte compare.
-__device__ __forceinline__ uint32_t fpl(uint64_t h, uint32_t len) {
-    return ((uint32_t)(h >> 32) & 0xfffffe00u) | 0x100u | min(len, 255u);
-}
 // A warp streams chunks of CH consecutive groups; chunk c belongs to warp c mod nw.
 __device__ __forceinline__ uint32_t next_group(uint32_t g, uint32_t nw) {
     return ((g + 1) % (uint32_t)CH) ? g + 1 : g + 1 + (nw - 1) * (uint32_t)CH;
@@ -777,7 +723,6 @@ __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, strea
         if (act && res == R_POST && base < b.out_cap) {
             constexpr uint32_t RS = RB == 48 ? 48u : 32u;  // record bytes (RB 33: 32-byte records too)
             ulonglong2* o = reinterpret_cast<ulonglong2*>(reinterpret_cast<uint8_t*>(b.out) + base * RS);
-#if SEPO_PREP_STCS  // streaming stores: the re-issue list must not push table lines out of L2
             __stcs(o, make_ulonglong2(w0, RB == 33 ? v : w1));
             if (RB == 32 || RB == 33) {
                 __stcs(o + 1, make_ulonglong2(h, s | ((unsigned long long)len << 48)));
@@ -785,15 +730,6 @@ __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, strea
                 __stcs(o + 1, make_ulonglong2(h, s));
                 __stcs(o + 2, make_ulonglong2(v, (unsigned long long)len));
             }
-#else
-            o[0] = make_ulonglong2(w0, RB == 33 ? v : w1);
-            if (RB == 32 || RB == 33) {  // {key words | key + value, hash, offset | length << 48}
-                o[1] = make_ulonglong2(h, s | ((unsigned long long)len << 48));
-            } else {
-                o[1] = make_ulonglong2(h, s);
-                o[2] = make_ulonglong2(v, (unsigned long long)len);
-            }
-#endif
         }
     }
     if (pend) {
@@ -835,12 +771,6 @@ __device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, str
 
 // Reinsert pass of sepo_run (a9 re-issue): the prepared records of the previous pass, 32 per warp
 // step, straight into resolve_core (keys of these passes are the Zipf tail: no hot set).
-#ifndef SEPO_PREP_STCS
-#define SEPO_PREP_STCS 1  // C2 4x job 32.2 -> 31.8 ms (re-issue passes read the list while the table stays in L2)
-#endif
-#ifndef SEPO_REINS_PF
-#define SEPO_REINS_PF 1  // next step's 32-byte prepared records loaded during this step (C2 4x re-issue passes -0.3 ms)
-#endif
 template <int RB>
 __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
     __shared__ stream::CtaState S;
@@ -856,7 +786,6 @@ __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
     bool w_full = false, w_quiet = false;
     PrepCursor pc;
     const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
-#if SEPO_REINS_PF
     // the next step's prepared records are loaded while this step's are resolved (RB == 32 only)
     ulonglong2 n0 = make_ulonglong2(0, 0), n1 = make_ulonglong2(0, 0);
     {
@@ -866,11 +795,9 @@ __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
             n0 = __ldcs(p); n1 = __ldcs(p + 1);
         }
     }
-#endif
     for (uint64_t base = ((uint64_t)blockIdx.x * (blockDim.x / 32) + (tid >> 5)) * 32; base < b.n; base += nw * 32) {
         const uint64_t i = base + lane;
         ulonglong2 r0 = make_ulonglong2(0, 0), r1 = make_ulonglong2(0, 0), r2 = make_ulonglong2(1, 0);
-#if SEPO_REINS_PF
         if (RB == 32 || RB == 33) {
             r0 = n0; r1 = n1;
             const uint64_t inx = i + nw * 32;
@@ -879,7 +806,6 @@ __global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
                 n0 = __ldcs(p); n1 = __ldcs(p + 1);
             }
         } else
-#endif
         if (i < b.n) {
             const ulonglong2* p = reinterpret_cast<const ulonglong2*>(reinterpret_cast<const uint8_t*>(b.prep) + i * (RB == 48 ? 48 : 32));
             r0 = __ldcs(p); r1 = __ldcs(p + 1);
@@ -1028,11 +954,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     SM& S = *reinterpret_cast<SM*>(smem_raw);
     const uint32_t tid = threadIdx.x, lane = lane_id();
     for (int p = tid; p < stream::NKEY; p += THREADS) { S.ref[p] = 0; S.sum[p] = 0; }
-#if SEPO_HOT_DIRECT
     for (int p = tid; p < stream::DS; p += THREADS) S.tags[p] = 0u;
-#else
-    for (int p = tid; p < hot::NB; p += THREADS) S.tags[p] = make_uint4(0, 0, 0, 0);
-#endif
     if (tid == 0) {
         S.cs.cur[0] = d.cursors[2 * blockIdx.x];
         S.cs.cur[1] = d.cursors[2 * blockIdx.x + 1];
@@ -1046,7 +968,6 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         for (unsigned j = tid; j < nh; j += THREADS) {
             const hot::Entry e = hl[j];
             if (e.ref == 0 || hot::count_class(e.count) != cls) continue;
-#if SEPO_HOT_DIRECT
             if (j < (unsigned)stream::NKEY) {  // claim slot ds1, else ds2, else leave the key out
                 const uint32_t f = stream::dfp(e.h, e.len) | j;
                 if (atomicCAS(&S.tags[stream::ds1(e.h)], 0u, f) == 0u || atomicCAS(&S.tags[stream::ds2(e.h)], 0u, f) == 0u) {
@@ -1054,19 +975,6 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
                     S.ref[j] = e.ref;
                 }
             }
-            continue;
-#endif
-            // claim a free slot in bucket b1, else b2, else leave the key out (the set is only a cache)
-            const uint32_t f = stream::fpl(e.h, e.len);
-            int pos = -1;
-            for (int c = 0; c < 2 && pos < 0; ++c) {
-                const uint32_t bk = c == 0 ? hot::b1(e.h) : hot::b2(e.h);
-                uint32_t* t = reinterpret_cast<uint32_t*>(&S.tags[bk]);
-                for (int w = 0; w < 4 && pos < 0; ++w)
-                    if (atomicCAS(&t[w], 0u, f) == 0u) pos = (int)(bk * 4 + w);
-            }
-            if (pos < 0) continue;
-            S.kw[pos] = make_ulonglong2(e.w0, e.w1); S.ref[pos] = e.ref;
         }
         __syncthreads();
     }
@@ -1088,49 +996,16 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     uint4 ch_c = in_stage2<IN>(b, c, g, lane, s_c, win_c);
     uint32_t gn = stream::next_group(g, c.nw);
     in_stage1<IN, VALS>(b, c, gn, lane, s_n, v_n, eo_n);
-#if SEPO_S1_AHEAD == 3
-    // offsets three groups ahead: group gx (stage 1 in flight one iteration longer)
-    uint32_t gx = stream::next_group(gn, c.nw);
-    uint64_t s_x = 0, v_x = 1;
-    uint32_t eo_x = 0;
-    in_stage1<IN, VALS>(b, c, gx, lane, s_x, v_x, eo_x);
-#endif
 
     while (g < c.ngroups) {
         // ---- issue ahead: key chunks of gn, offsets (values) of the group after it
         uint32_t win_n;
         const uint4 ch_n = in_stage2<IN>(b, c, gn, lane, s_n, win_n);
-#if SEPO_S1_AHEAD == 3
-        const uint32_t gnn = gx;
-        uint64_t s_nn = s_x, v_nn = v_x;
-        uint32_t eo_nn = eo_x;
-        gx = stream::next_group(gx, c.nw);
-        in_stage1<IN, VALS>(b, c, gx, lane, s_x, v_x, eo_x);
-#else
         const uint32_t gnn = stream::next_group(gn, c.nw);
         uint64_t s_nn, v_nn;
         uint32_t eo_nn = 0;
         in_stage1<IN, VALS>(b, c, gnn, lane, s_nn, v_nn, eo_nn);
-#endif
 
-#if SEPO_IN_PREFETCH
-        // L2 prefetch SEPO_IN_PREFETCH groups further ahead in the warp's chunk: the 2 lines of key
-        // offsets and ~4 lines of key bytes (extrapolated from this group's window)
-        if (IN == IN_CSR && (g % (uint32_t)stream::CH) + SEPO_IN_PREFETCH < (uint32_t)stream::CH &&
-            g + SEPO_IN_PREFETCH < c.ngroups && lane < 6) {
-            const uint32_t gp = g + SEPO_IN_PREFETCH;
-            const uint8_t* a;
-            if (lane < 2) {
-                a = reinterpret_cast<const uint8_t*>(b.ko + (uint64_t)gp * 32) + 128 * lane;
-            } else {
-                const uint64_t base_al = (win_c & ~1u) | (s_c & ~0xffffffffull);
-                const uint64_t span = (uint64_t)(uint32_t)((uint32_t)s_n - (win_c & ~1u));  // this group's bytes
-                a = b.keys + base_al + span * SEPO_IN_PREFETCH + 128 * (lane - 2);
-                if (a >= b.keys + c.kend) a = b.keys;
-            }
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(a));
-        }
-#endif
         // ---- group g: key words + hash (a1)
         const bool valid = lane < group_cnt(c, g);
         uint64_t s = s_c, w0, w1;
@@ -1140,27 +1015,12 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
         // ---- hot set (a2): both 4-way fingerprint buckets, then one 16-byte key compare
         int pos = -1;
-#if SEPO_HOT_DIRECT
         if (have_hot) {
             const uint32_t f = stream::dfp(h, len);
             const uint32_t t1 = S.tags[stream::ds1(h)], t2 = S.tags[stream::ds2(h)];
             constexpr uint32_t IM = (1u << stream::IDXB) - 1u;
             const bool m1 = (t1 & ~IM) == f, m2 = (t2 & ~IM) == f;
             const uint32_t p = (m1 ? t1 : t2) & IM;
-#if SEPO_BRANCHLESS
-            // branch-free common case: the candidate's 16 key bytes are loaded for every lane (p is
-            // always a valid index); keys longer than 16 bytes take a warp-uniform slow path
-            const bool cand = valid && (m1 || m2);
-            const ulonglong2 kk = S.kw[p];
-            bool eq = cand && kk.x == w0 && kk.y == w1;
-            if (__any_sync(FULLMASK, eq && len > 16)) {
-                if (eq && len > 16) {
-                    const uint8_t* e = ref_ptr(d, S.ref[p]);
-                    eq = ldcg32(e + 12) == len && entry_key_eq(e + KEY_OFF + 16, b.keys + s + 16, len - 16);
-                }
-            }
-            pos = eq ? (int)p : -1;
-#else
             if (valid && (m1 || m2)) {
                 const ulonglong2 kk = S.kw[p];
                 bool eq = kk.x == w0 && kk.y == w1;
@@ -1170,27 +1030,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
                 }
                 if (eq) pos = (int)p;
             }
-#endif
         }
-#else
-        if (have_hot) {
-            const uint32_t f = stream::fpl(h, len);
-            const uint32_t k1 = hot::b1(h), k2 = hot::b2(h);
-            const uint4 t1 = S.tags[k1], t2 = S.tags[k2];
-            const uint32_t m1 = (t1.x == f) | ((t1.y == f) << 1) | ((t1.z == f) << 2) | ((t1.w == f) << 3);
-            const uint32_t m2 = (t2.x == f) | ((t2.y == f) << 1) | ((t2.z == f) << 2) | ((t2.w == f) << 3);
-            const int p = m1 ? (int)(4 * k1 + __ffs(m1) - 1) : (int)(4 * k2 + __ffs(m2) - 1);
-            if (valid && (m1 | m2)) {
-                const ulonglong2 kk = S.kw[p];
-                bool eq = kk.x == w0 && kk.y == w1;
-                if (len > 16) {  // long key: exact length (the fingerprint saturates at 255) + tail bytes
-                    const uint8_t* e = ref_ptr(d, S.ref[p]);
-                    eq = eq && ldcg32(e + 12) == len && entry_key_eq(e + KEY_OFF + 16, b.keys + s + 16, len - 16);
-                }
-                if (eq) pos = p;
-            }
-        }
-#endif
         // ---- fold the hits of the warp per hot slot (a2): one shared atomic per distinct key
         const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
         if (hm) {
@@ -1227,7 +1067,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         if (miss) {
             // the directory word is read when the queue is resolved (a few groups later): when the
             // table does not fit L2 (host decision, c.dirpf) start bringing its line in now
-            if (SEPO_DIR_PREFETCH || c.dirpf)
+            if (c.dirpf)
                 asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(d.dir + bucket_of(h, d.n_buckets)));
             const uint32_t k = (qtail + __popc(mm & lanemask_lt())) & (stream::QCAP - 1);
             Q.w0[k] = w0; Q.w1[k] = w1; Q.h[k] = h; Q.s[k] = s;
@@ -2675,11 +2515,7 @@ __global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, B
     using namespace textk;
     extern __shared__ __align__(16) uint8_t smem_raw[];
     textk::Smem& S = *reinterpret_cast<textk::Smem*>(smem_raw);
-#if SEPO_TEXT_TIDLANE
-    const uint32_t tid = threadIdx.x, lane = tid & 31u, wid = tid >> 5;
-#else
     const uint32_t tid = threadIdx.x, lane = lane_id(), wid = tid >> 5;
-#endif
     for (int p = tid; p < TK; p += THREADS) { S.ref[p] = 0; S.sum[p] = 0; }
     for (int p = tid; p < DSZ; p += THREADS) S.tags[p] = 0u;
     if (tid == 0) {

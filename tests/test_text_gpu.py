@@ -143,8 +143,8 @@ def test_map_lines_page_view_count(cuda):
     assert exp == s.expected_combine()
 
 
-@pytest.mark.parametrize("budget_pages", [4096, 40])
-def test_map_word_docs_inverted_index(cuda, budget_pages):
+@pytest.mark.parametrize("over", [False, True])
+def test_map_word_docs_inverted_index(cuda, over):
     """MAP_WORD_DOCS: documents of words -> (word, doc id) grouped == oracle.group over the same pairs,
     in one pass and over budget"""
     rng = np.random.default_rng(4)
@@ -173,10 +173,16 @@ def test_map_word_docs_inverted_index(cuda, budget_pages):
     vals = np.array(docs, dtype=np.uint32).view(np.uint8)
     exp = oracle.group(np.frombuffer(b"".join(words), dtype=np.uint8), ko, vals, val_width=4).as_dict()
     S = sepo()
-    t = S.Table(S.budget_for(1 << 14, 4096, budget_pages), 1 << 14, 4096, mode=S.GROUP, fixed_val_width=4, check_dups=True)
-    passes = t.map_run(S.MAP_WORD_DOCS, torch.from_numpy(text.copy()).cuda(), torch.from_numpy(doc_offsets).cuda())
+    dt, dd = torch.from_numpy(text.copy()).cuda(), torch.from_numpy(doc_offsets).cuda()
+    t = S.Table(S.budget_for(1 << 14, 4096, 4096), 1 << 14, 4096, mode=S.GROUP, fixed_val_width=4)
+    assert t.map_run(S.MAP_WORD_DOCS, dt, dd) == 1
+    F = t.stats()["pages_used_max"]
+    t.close()
+    t = S.Table(S.budget_for(1 << 14, 4096, F // 3 + 2 if over else F + 64), 1 << 14, 4096, mode=S.GROUP,
+                fixed_val_width=4, check_dups=True)
+    passes = t.map_run(S.MAP_WORD_DOCS, dt, dd)
     got = S.result_dict(t.export(), S.GROUP)
     t.close()
     assert got == exp
-    if budget_pages < 100:
+    if over:
         assert passes >= 2
