@@ -246,8 +246,8 @@ size_t sepo_partition_scratch(uint64_t n, uint32_t n_parts);
  * each). Outputs (device, caller-owned, same sizes as the inputs): out_keys, out_key_offsets
  * (n entries: record j's offset relative to the first byte of ITS part; NULL for fixed-width
  * keys), out_vals. part_starts (HOST, 3 * (n_parts + 1) u64): for part p, (first record, first key
- * byte, first value byte) in the outputs; entry n_parts holds the totals. Records keep their input
- * order within a part. Synchronizes the stream. */
+ * byte, first value byte) in the outputs; entry n_parts holds the totals. The order of records within a
+ * part is unspecified (each record takes its slot with one shared-memory atomic). Synchronizes the stream. */
 int sepo_partition(const uint8_t* keys, const uint64_t* key_offsets, uint32_t fixed_key_width, const uint8_t* vals,
                    uint32_t fixed_val_width, uint64_t n, uint32_t n_parts, uint64_t route_seed, uint8_t* out_keys,
                    uint64_t* out_key_offsets, uint8_t* out_vals, uint64_t* part_starts, void* scratch,

@@ -2056,37 +2056,55 @@ __device__ __forceinline__ uint32_t route_owner(const Batch& b, uint64_t i, uint
     return (uint32_t)(((h >> 32) * (uint64_t)P) >> 32);
 }
 
+// Per tile of PT_TILE records, the lanes of a warp with the same owner (one __match_any_sync) reserve
+// their slots in their part with ONE shared-memory atomic on a packed per-part cursor {records << 32 |
+// key bytes} issued by the group's first lane; a lane's rank is the popcount of the group below it and
+// its byte offset the sum of the group's lengths below it, taken bit by bit (one ballot per bit of the
+// warp's longest key). Rank and byte offset come from the same atomic, so key bytes and offsets stay a
+// CSR. (The order of records within a part follows the atomics; the method is order independent.)
+// Pass count: the tile's per-part totals; pass scatter: base of (part, tile) from the scan + the rank.
+__device__ __forceinline__ void pt_reserve(unsigned long long* cur, bool valid, uint32_t p, uint32_t len, uint32_t& rank,
+                                           uint32_t& boff, unsigned long long& slot) {
+    const uint32_t lane = lane_id();
+    const unsigned gm = __match_any_sync(FULLMASK, valid ? p : (0x100u | lane));
+    const unsigned lt = lanemask_lt();
+    const uint32_t nbits = 32u - __clz(__reduce_max_sync(FULLMASK, valid ? len : 0u));
+    uint32_t pre = 0, tot = 0;
+    for (uint32_t bit = 0; bit < nbits; ++bit) {
+        const unsigned m = __ballot_sync(FULLMASK, valid && ((len >> bit) & 1u)) & gm;
+        pre += (uint32_t)__popc(m & lt) << bit;
+        tot += (uint32_t)__popc(m) << bit;
+    }
+    const uint32_t leader = (uint32_t)(__ffs(gm) - 1);
+    unsigned long long r = 0;
+    if (valid && lane == leader) r = atomicAdd(&cur[p], ((unsigned long long)__popc(gm) << 32) | (unsigned long long)tot);
+    slot = __shfl_sync(FULLMASK, r, leader);
+    rank = (uint32_t)__popc(gm & lt);
+    boff = pre;
+}
 __global__ void __launch_bounds__(PT_THREADS) part_count_kernel(Batch b, uint32_t P, uint64_t seed,
                                                                 unsigned long long* counts, uint64_t ntiles) {
-    __shared__ unsigned long long c[PT_MAXP][3];
+    __shared__ unsigned long long cur[PT_MAXP];
     for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        for (int x = threadIdx.x; x < PT_MAXP * 3; x += blockDim.x) (&c[0][0])[x] = 0;
+        if (threadIdx.x < PT_MAXP) cur[threadIdx.x] = 0ull;
         __syncthreads();
-        const uint32_t lane = threadIdx.x & 31u;
         for (int k = 0; k < PT_TILE / PT_THREADS; ++k) {
             const uint64_t i = tile * PT_TILE + k * PT_THREADS + threadIdx.x;
             const bool valid = i < b.n;
-            uint64_t s = 0, w0, w1; uint32_t len = 0, o = 0xffu;
+            uint64_t s = 0, w0, w1; uint32_t len = 0, o = 0;
             if (valid) o = route_owner(b, i, seed, P, s, len, w0, w1);
-            // warp-aggregated: one shared atomic per destination part present in the warp (per-record
-            // atomics on P counters serialised: 370 ms for 1.1e9 records at P = 1)
-            unsigned todo = __ballot_sync(FULLMASK, valid);
-            while (todo) {
-                const uint32_t p = __shfl_sync(FULLMASK, o, __ffs(todo) - 1);
-                const bool mem = valid && o == p;
-                const unsigned mm = __ballot_sync(FULLMASK, mem);
-                todo &= ~mm;
-                const unsigned bytes = __reduce_add_sync(FULLMASK, mem ? len : 0u);
-                if (lane == (uint32_t)(__ffs(mm) - 1)) {
-                    atomicAdd(&c[p][0], (unsigned long long)__popc(mm));
-                    atomicAdd(&c[p][1], (unsigned long long)bytes);
-                    if (b.vals) atomicAdd(&c[p][2], (unsigned long long)__popc(mm) * b.vw);
-                }
-            }
+            uint32_t rank, boff;
+            unsigned long long slot;
+            pt_reserve(cur, valid, o, len, rank, boff, slot);
         }
         __syncthreads();
-        for (uint32_t x = threadIdx.x; x < P * 3; x += blockDim.x)
-            counts[((uint64_t)(x / 3) * ntiles + tile) * 3 + (x % 3)] = c[x / 3][x % 3];
+        if (threadIdx.x < P) {
+            const unsigned long long c = cur[threadIdx.x];
+            unsigned long long* dst = counts + ((uint64_t)threadIdx.x * ntiles + tile) * 3;
+            dst[0] = c >> 32;
+            dst[1] = c & 0xffffffffull;
+            dst[2] = b.vals ? (c >> 32) * b.vw : 0ull;
+        }
         __syncthreads();
     }
 }
@@ -2094,75 +2112,50 @@ __global__ void __launch_bounds__(PT_THREADS) part_count_kernel(Batch b, uint32_
 __global__ void __launch_bounds__(PT_THREADS) part_scatter_kernel(Batch b, uint32_t P, uint64_t seed,
                                                                   const unsigned long long* base, uint64_t ntiles,
                                                                   uint8_t* ok, uint64_t* oko, uint8_t* ov) {
-    constexpr int R = PT_TILE / PT_THREADS, NW = PT_THREADS / 32;
-    __shared__ unsigned int wrec[R][NW][PT_MAXP];
-    __shared__ unsigned long long wbytes[R][NW][PT_MAXP];
-    const uint32_t lane = threadIdx.x & 31u, warp = threadIdx.x >> 5;
+    __shared__ unsigned long long cur[PT_MAXP];
     for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        uint32_t own[R], rank[R], len[R];
-        uint64_t src[R], boff[R], kw0[R], kw1[R];
-        for (int k = 0; k < R; ++k) {
+        if (threadIdx.x < PT_MAXP) cur[threadIdx.x] = 0ull;
+        __syncthreads();
+        for (int k = 0; k < PT_TILE / PT_THREADS; ++k) {
             const uint64_t i = tile * PT_TILE + k * PT_THREADS + threadIdx.x;
             const bool valid = i < b.n;
-            own[k] = 0xffu; len[k] = 0; src[k] = 0; kw0[k] = 0; kw1[k] = 0;
-            if (valid) own[k] = route_owner(b, i, seed, P, src[k], len[k], kw0[k], kw1[k]);
-            // per part present in the warp: exclusive rank and byte offset among its members
-            for (uint32_t p = lane; p < P; p += 32) { wrec[k][warp][p] = 0; wbytes[k][warp][p] = 0; }
-            __syncwarp();
-            unsigned todo = __ballot_sync(FULLMASK, valid);
-            rank[k] = 0; boff[k] = 0;
-            while (todo) {
-                const uint32_t p = __shfl_sync(FULLMASK, own[k], __ffs(todo) - 1);
-                const bool mem = valid && own[k] == p;
-                const unsigned mm = __ballot_sync(FULLMASK, mem);
-                todo &= ~mm;
-                const unsigned long long x = mem ? len[k] : 0ull;
-                unsigned long long incl = x;
-                for (int o = 1; o < 32; o <<= 1) {
-                    const unsigned long long y = __shfl_up_sync(FULLMASK, incl, o);
-                    if (lane >= (uint32_t)o) incl += y;
-                }
-                if (mem) { rank[k] = __popc(mm & ((1u << lane) - 1u)); boff[k] = incl - x; }
-                if (lane == 31) { wrec[k][warp][p] = __popc(mm); wbytes[k][warp][p] = incl; }
-                __syncwarp();
-            }
-        }
-        __syncthreads();
-        // exclusive prefix per part over the (k, warp) order, one thread per part
-        if (threadIdx.x < P) {
-            const uint32_t p = threadIdx.x;
-            unsigned int r = 0;
-            unsigned long long by = 0;
-            for (int k = 0; k < R; ++k)
-                for (int w = 0; w < NW; ++w) {
-                    const unsigned int r0 = wrec[k][w][p];
-                    const unsigned long long b0 = wbytes[k][w][p];
-                    wrec[k][w][p] = r; wbytes[k][w][p] = by;
-                    r += r0; by += b0;
-                }
-        }
-        __syncthreads();
-        for (int k = 0; k < R; ++k) {
-            const uint64_t i = tile * PT_TILE + k * PT_THREADS + threadIdx.x;
-            if (i >= b.n) continue;
-            const uint32_t p = own[k];
-            const unsigned long long rb = wrec[k][warp][p], bb = wbytes[k][warp][p];
+            uint64_t src = 0, kw0 = 0, kw1 = 0; uint32_t len = 0, p = 0;
+            if (valid) p = route_owner(b, i, seed, P, src, len, kw0, kw1);
+            uint32_t rank, boff;
+            unsigned long long r;
+            pt_reserve(cur, valid, p, len, rank, boff, r);
+            if (!valid) continue;
             const unsigned long long* bp = base + ((uint64_t)p * ntiles + tile) * 3;
             const unsigned long long* b0 = base + ((uint64_t)p * ntiles) * 3;  // start of part p
-            const uint64_t orec = bp[0] + rb + rank[k];
-            const uint64_t obyte = bp[1] + bb + boff[k];
+            const uint64_t orec = bp[0] + (r >> 32) + rank;
+            const uint64_t obyte = bp[1] + (r & 0xffffffffull) + boff;
             if (oko) oko[orec] = obyte - b0[1];  // rebased to the part's segment
             // the first 16 key bytes come from registers (loaded for the hash), the rest from input
-            for (uint32_t x = 0; x < len[k]; ++x)
-                ok[obyte + x] = x < 8 ? (uint8_t)(kw0[k] >> (8 * x)) : x < 16 ? (uint8_t)(kw1[k] >> (8 * (x - 8)))
-                                                                      : __ldg(b.keys + src[k] + x);
+            uint8_t* dst = ok + obyte;
+            const uint32_t head = min(len, 16u);
+            for (uint32_t x = 0; x < head; ++x) dst[x] = (uint8_t)((x < 8 ? kw0 >> (8 * x) : kw1 >> (8 * (x - 8))) & 0xffu);
+            for (uint32_t x = 16; x < len; ++x) dst[x] = (uint8_t)ld_in8(b.keys + src + x);
             if (b.vals) {
                 const uint64_t vs = rec_index(b, i) * (uint64_t)b.vw;
-                for (uint32_t x = 0; x < b.vw; ++x) ov[orec * b.vw + x] = __ldg(b.vals + vs + x);
+                uint8_t* vd = ov + orec * b.vw;
+                if (b.vw == 8) *reinterpret_cast<unsigned long long*>(vd) = ld_in64(b.vals + vs);
+                else for (uint32_t x = 0; x < b.vw; ++x) vd[x] = (uint8_t)ld_in8(b.vals + vs + x);
             }
         }
         __syncthreads();
     }
+}
+
+// received segments: offsets of segment s are relative to its own bytes; shift them by the bytes
+// of the segments before it and close the CSR with the total
+__global__ void shift_offsets_kernel(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const uint64_t* seg_base,
+                                     uint32_t n_segs, uint64_t total) {
+    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < n; j += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t sgi = 0;
+        while (sgi + 1 < n_segs && seg_rec[sgi + 1] <= j) ++sgi;
+        ko[j] += seg_base[sgi];
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) ko[n] = total;
 }
 
 // ---- router with CTA pre-combine (COMBINE mode, keys of at most 16 bytes)
@@ -2309,17 +2302,6 @@ __global__ void __launch_bounds__(rc::THREADS, 1) route_combine_kernel(Batch b, 
     }
 }
 
-// received segments: offsets of segment s are relative to its own bytes; shift them by the bytes
-// of the segments before it and close the CSR with the total
-__global__ void shift_offsets_kernel(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const uint64_t* seg_base,
-                                     uint32_t n_segs, uint64_t total) {
-    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < n; j += (uint64_t)gridDim.x * blockDim.x) {
-        uint32_t sgi = 0;
-        while (sgi + 1 < n_segs && seg_rec[sgi + 1] <= j) ++sgi;
-        ko[j] += seg_base[sgi];
-    }
-    if (blockIdx.x == 0 && threadIdx.x == 0) ko[n] = total;
-}
 
 // ================================================================ pass boundary (a10)
 // Seal every open page (filler over its unused tail) and reset the CTA cursors.
