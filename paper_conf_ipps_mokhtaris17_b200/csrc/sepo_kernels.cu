@@ -1125,7 +1125,10 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
 // the host picks insert_stream_kernel for long-key batches (mean key length > 24 B).
 // A queued miss is {w0, w1}, {h, s | len << 40 | lane << 59} and its group.
 namespace lean {
-constexpr int THREADS = 1024, WARPS = THREADS / 32, QCAP = 64;
+#ifndef SEPO_LEAN_THREADS
+#define SEPO_LEAN_THREADS 1024
+#endif
+constexpr int THREADS = SEPO_LEAN_THREADS, WARPS = THREADS / 32, QCAP = 64;
 constexpr uint64_t S_MASK = (1ull << 40) - 1;
 constexpr uint32_t LEN_MAX = (1u << 19) - 1;
 template <bool VALS>
@@ -2689,7 +2692,10 @@ __global__ void __launch_bounds__(textk::THREADS, 1) insert_text_kernel(Dev d, B
 //     separator bits (words longer than 32 bytes continue the scan, longer than the ring: global);
 //   * queue slots as the lean CSR kernel (32 bytes: first 16 key bytes, hash, offset | length).
 namespace text2 {
-constexpr int THREADS = 1024, WARPS = THREADS / 32;
+#ifndef SEPO_TEXT_THREADS
+#define SEPO_TEXT_THREADS 768  // 24 warps, 80 registers: C2 text 4x pass 1 26.1 -> 25.3 ms, in budget 45.0 -> 28.9 ms
+#endif                         // (896: 26.7 / 45.1, 640: 28.9 / 33.2, 512: 34.7 / 39.8; profiles/r02)
+constexpr int THREADS = SEPO_TEXT_THREADS, WARPS = THREADS / 32;
 constexpr int WB = 512, NSLOT = 3, RINGB = NSLOT * WB, SEPW = RINGB / 32;
 constexpr int DSZ = 8192, TK = 2048;
 constexpr int WLCAP = 288;  // carried words (< 32) + one window's word starts (<= 256)
