@@ -1395,7 +1395,10 @@ __global__ void __launch_bounds__(lean::THREADS, 1) insert_lean_kernel(Dev d, Ba
 // P:L165); new-key declines are certified as in the COMBINE kernel (R15), so a GROUP pass needs no
 // separate re-probe.
 namespace gst {
-constexpr int THREADS = 1024;
+#ifndef SEPO_GROUP_THREADS
+#define SEPO_GROUP_THREADS 1024
+#endif
+constexpr int THREADS = SEPO_GROUP_THREADS;
 constexpr int NB = 512, NH = 4 * NB;  // hot slots (2-choice 4-way buckets)
 constexpr int K = 1024;               // hot keys at most
 constexpr uint32_t PC_CAP = 256;      // slots of a private chunk
@@ -3280,7 +3283,24 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             }
             return cudaGetLastError();
         }
-        if (b.vals) {
+        if (b.vals && in != IN_CSR) {
+            // fixed-width keys with values (C5), and index re-issue batches with values: 24 warps per
+            // CTA, 80 registers — C5u 4x pass 1 20.6 -> 12.8 ms, index re-issue passes 18.9 / 15.3 ->
+            // 13.2 / 10.0 ms (CSR batches keep 32 warps: C2 in budget 25.5 vs 27.9 ms, C3 48.9 vs 55.7 ms at 24)
+            constexpr int T2 = 768;
+            static bool attr2 = false;
+            if (!attr2) {
+                cudaFuncSetAttribute(insert_stream_kernel<true, T2, IN_FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)sizeof(stream::Smem<true, T2 / 32>));
+                cudaFuncSetAttribute(insert_stream_kernel<true, T2, IN_IDX>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)sizeof(stream::Smem<true, T2 / 32>));
+                attr2 = true;
+            }
+            c.nw = (uint32_t)grid * (T2 / 32);
+            const size_t sm2 = sizeof(stream::Smem<true, T2 / 32>);
+            if (in == IN_FIXED) insert_stream_kernel<true, T2, IN_FIXED><<<grid, T2, sm2, s>>>(d, b, hl, nh, c);
+            else insert_stream_kernel<true, T2, IN_IDX><<<grid, T2, sm2, s>>>(d, b, hl, nh, c);
+        } else if (b.vals) {
             if (in == IN_CSR) insert_stream_kernel<true, T, IN_CSR><<<grid, T, sm, s>>>(d, b, hl, nh, c);
             else if (in == IN_FIXED) insert_stream_kernel<true, T, IN_FIXED><<<grid, T, sm, s>>>(d, b, hl, nh, c);
             else insert_stream_kernel<true, T, IN_IDX><<<grid, T, sm, s>>>(d, b, hl, nh, c);
