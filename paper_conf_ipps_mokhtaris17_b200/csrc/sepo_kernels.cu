@@ -771,8 +771,11 @@ __device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, str
 
 // Reinsert pass of sepo_run (a9 re-issue): the prepared records of the previous pass, 32 per warp
 // step, straight into resolve_core (keys of these passes are the Zipf tail: no hot set).
+#ifndef SEPO_REINS_THREADS
+#define SEPO_REINS_THREADS 1024
+#endif
 template <int RB>
-__global__ void __launch_bounds__(1024, 1) reinsert_kernel(Dev d, Batch b) {
+__global__ void __launch_bounds__(SEPO_REINS_THREADS, 1) reinsert_kernel(Dev d, Batch b) {
     __shared__ stream::CtaState S;
     const uint32_t tid = threadIdx.x, lane = lane_id();
     if (tid == 0) {
@@ -3343,9 +3346,9 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
 }
 int sepo_launch_reinsert(const Dev& d, const Batch& b, int grid, cudaStream_t s) {
     if (b.n == 0) return cudaGetLastError();
-    if (b.prep_fmt == 33) reinsert_kernel<33><<<grid, 1024, 0, s>>>(d, b);
-    else if (b.prep_rb == 32) reinsert_kernel<32><<<grid, 1024, 0, s>>>(d, b);
-    else reinsert_kernel<48><<<grid, 1024, 0, s>>>(d, b);
+    if (b.prep_fmt == 33) reinsert_kernel<33><<<grid, SEPO_REINS_THREADS, 0, s>>>(d, b);
+    else if (b.prep_rb == 32) reinsert_kernel<32><<<grid, SEPO_REINS_THREADS, 0, s>>>(d, b);
+    else reinsert_kernel<48><<<grid, SEPO_REINS_THREADS, 0, s>>>(d, b);
     return cudaGetLastError();
 }
 size_t sepo_hot_count_offset() { return sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS + sizeof(hot::Entry) * hot::K; }
