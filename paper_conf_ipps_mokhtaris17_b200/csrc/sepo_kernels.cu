@@ -371,9 +371,9 @@ __device__ __forceinline__ uint32_t dfp_b(uint64_t h, uint32_t len) {
 // fingerprint and its index into the dense key arrays, so a probe is two 4-byte loads, two
 // compares and one 16-byte key load.
 #ifndef SEPO_HOT_DS
-#define SEPO_HOT_DS 16384
-#endif
-constexpr int DS = SEPO_HOT_DS;           // slots (2048 hot keys in 16384: load <= 1/8)
+#define SEPO_HOT_DS 8192  // 16384 measured slower: the 32 KB it takes from L1 cost C2 0.5x pass 1
+#endif                       // 25.5 -> 22.7 ms, C2 4x 19.6 -> 19.3, C3 1x 48.4 -> 47.1 (4096: = 8192)
+constexpr int DS = SEPO_HOT_DS;           // slots (2048 hot keys in 8192: load <= 1/4)
 constexpr int NKEY = hot::K;
 constexpr int IDXB = NKEY <= 2048 ? 11 : (NKEY <= 4096 ? 12 : 13);  // key-index bits of a slot word
 __device__ __forceinline__ uint32_t ds1(uint64_t h) { return (uint32_t)(h >> 3) & (DS - 1); }
@@ -2703,7 +2703,10 @@ namespace text2 {
 #endif                         // (896: 26.7 / 45.1, 640: 28.9 / 33.2, 512: 34.7 / 39.8; profiles/r02)
 constexpr int THREADS = SEPO_TEXT_THREADS, WARPS = THREADS / 32;
 constexpr int WB = 512, NSLOT = 3, RINGB = NSLOT * WB, SEPW = RINGB / 32;
-constexpr int DSZ = 8192, TK = 2048;
+#ifndef SEPO_TEXT_DS
+#define SEPO_TEXT_DS 8192
+#endif
+constexpr int DSZ = SEPO_TEXT_DS, TK = 2048;
 constexpr int WLCAP = 288;  // carried words (< 32) + one window's word starts (<= 256)
 constexpr int QCAP = 64;
 struct WarpText {
