@@ -495,7 +495,7 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
     }
     // COMBINE pass 1 on contiguous input: the lean kernel unless the keys are long on average (URLs:
     // insert_stream_kernel's warp-window loads suit them better); SEPO_LEAN=0/1 forces the choice
-    bool lean_in = false;
+    bool lean_in = false, long_keys = false;
     if (t->opts.mode == SEPO_COMBINE_SUM_U64 && !b.idx) {
         const char* e = getenv("SEPO_LEAN");
         const uint64_t mean = b.ko ? (key_end - key_begin) / n : t->opts.fixed_key_width;
@@ -503,10 +503,12 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
         // issue-bound — C2 4x pass 1 21.2 -> 19.6 ms — and loses ~1.4 % when table accesses go to
         // HBM, where insert_stream_kernel's chunk-interleaved stream keeps fewer L1/L2 lines busy)
         lean_in = (e && (e[0] == '0' || e[0] == '1')) ? e[0] == '1' : (mean <= 24 && !dir_prefetch(t));
+        const char* el = getenv("SEPO_LONG");
+        long_keys = b.ko && ((el && (el[0] == '0' || el[0] == '1')) ? el[0] == '1' : mean > 24);
     }
     bool hot_built = false;
     rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p, halt_slots, key_end, dir_prefetch(t),
-                            &hot_built, lean_in);
+                            &hot_built, lean_in, long_keys);
     if (rc) return cuda_check(t, (cudaError_t)rc, "insert kernel launch");
     CK(t, cudaEventRecord(t->ev1, t->stream));
     t->h_ko[2] = 0;
@@ -550,7 +552,9 @@ static int64_t reinsert_impl(sepo_table* t, const Batch& b, uint64_t key_bytes, 
     sync_dev(t);
     if ((rc = zero_ctrl_counters(t))) return rc;
     CK(t, cudaEventRecord(t->ev0, t->stream));
-    rc = sepo_launch_reinsert(t->d, b, t->grid, t->stream);
+    const char* el = getenv("SEPO_LONG");
+    const bool long_keys = (el && (el[0] == '0' || el[0] == '1')) ? el[0] == '1' : key_bytes > 24 * records;
+    rc = sepo_launch_reinsert(t->d, b, t->grid, t->stream, long_keys);
     if (rc) return cuda_check(t, (cudaError_t)rc, "reinsert kernel launch");
     CK(t, cudaEventRecord(t->ev1, t->stream));
     t->st.kernel_launches += 1;

@@ -200,23 +200,143 @@ __device__ __forceinline__ uint64_t shl64_clamp(uint64_t x, uint32_t n) {
     return r;
 }
 
+// key word from the aligned words x (holding its first byte) and y (the next): 32-bit halves
+// selected by bit 2 of the key's address, then two funnel shifts by 8 x (address & 3)
+__device__ __forceinline__ uint64_t key_word(uint64_t x, uint64_t y, bool o, uint32_t s) {
+    const uint32_t xl = (uint32_t)x, xh = (uint32_t)(x >> 32), yl = (uint32_t)y, yh = (uint32_t)(y >> 32);
+    const uint32_t b0 = o ? xh : xl, b1 = o ? yl : xh, b2 = o ? yh : yl;
+    return ((uint64_t)__funnelshift_r(b1, b2, s) << 32) | __funnelshift_r(b0, b1, s);
+}
+// mask of the key's last word (bytes 1..8 of it are key bytes)
+__device__ __forceinline__ uint64_t last_word_mask(uint32_t n) {
+    return ~shl64_clamp(~0ull, 8u * (n - 8u * ((n - 1u) >> 3)));
+}
+// Input bytes [p, p+n) (n >= 1, immutable) as zero-padded 8-byte LE words, U words per round: a
+// round's aligned words are loaded together and shifted into key words, so a key tail costs
+// ceil(words / U) load round trips instead of one (two loads) per word — the per-word loop held
+// 48 % of C3 pass 1's stall samples (ncu source page, profiles/r02_summary.md). f(k, w) receives key
+// words k .. k + U - 1 (beyond the key: unspecified, callers test k + u < words) and returns false
+// to stop. Used by the long-key kernel instantiations (U > 1); U = 1 keeps the per-word loop.
+template <int U, typename F>
+__device__ __forceinline__ void tail_rounds(const uint8_t* p, uint32_t n, F&& f) {
+    const uintptr_t a = reinterpret_cast<uintptr_t>(p);
+    const bool o = (a >> 2) & 1u;
+    const uint32_t s = 8u * (uint32_t)(a & 3u);
+    const unsigned long long* q = reinterpret_cast<const unsigned long long*>(a & ~(uintptr_t)7);
+    const uint32_t naw = ((uint32_t)(a & 7u) + n + 7u) >> 3, nw = (n + 7u) >> 3;  // aligned words touched, key words
+    const uint64_t lm = last_word_mask(n);
+    uint64_t cur = ld_tail64(q);
+    for (uint32_t k = 0; k < nw; k += U) {
+        uint64_t x[U + 1];
+        x[0] = cur;
+#pragma unroll
+        for (int u = 1; u <= U; ++u) x[u] = k + u < naw ? ld_tail64(q + k + u) : 0ull;
+        uint64_t w[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            w[u] = key_word(x[u], x[u + 1], o, s);
+            if (k + u == nw - 1) w[u] &= lm;
+        }
+        if (!f(k, w)) return;
+        cur = x[U];
+    }
+}
+
 // ---------------------------------------------------------------- key hash (the paper leaves it open)
 __device__ __forceinline__ uint64_t fmix64(uint64_t k) {
     k ^= k >> 33; k *= 0xff51afd7ed558ccdull;
     k ^= k >> 33; k *= 0xc4ceb9fe1a85ec53ull;
     k ^= k >> 33; return k;
 }
-// h = fmix64(multiply-xor fold over the key's 8-byte LE words, zero padded, seeded with the length).
-// Every key folds at least two words (w0, w1), so keys of up to 16 bytes hash without branches.
+// h = fmix64(head + tail): head = a multiply-xor fold of the length, seed and the first 16 key bytes
+// (w0, w1: 8-byte LE words, zero padded); tail = the sum mod 2^64 of mix_word(word k, k) over the
+// key's remaining 8-byte words (zero padded). A sum, not a fold, so one key's tail can be hashed by
+// one lane or by a whole warp (lanes take words, the warp adds) with the same result (R32).
+// Keys of at most 16 bytes hash without branches.
 __device__ __forceinline__ uint64_t hash_init(uint32_t len, uint64_t seed) { return seed ^ ((uint64_t)len * 0x87c37b91114253d5ull); }
 __device__ __forceinline__ uint64_t hash_word(uint64_t h, uint64_t w) {
     return (h ^ w) * 0x9e3779b97f4a7c15ull;  // odd multiplier: a bijection per word
 }
+__device__ __forceinline__ uint64_t hash_head(uint32_t len, uint64_t seed, uint64_t w0, uint64_t w1) {
+    return hash_word(hash_word(hash_init(len, seed), w0), w1);
+}
+__device__ __forceinline__ uint64_t mix_word(uint64_t w, uint32_t k) {
+    uint64_t t = (w ^ ((uint64_t)(k + 1) * 0x9e3779b97f4a7c15ull)) * 0xbf58476d1ce4e5b9ull;
+    return t ^ (t >> 31);
+}
+// tail sum of the key bytes [p, p+n) (p = key + 16), by one lane
+template <int U = 1>
+__device__ __forceinline__ uint64_t tail_sum(const uint8_t* p, uint32_t n) {
+    uint64_t x = 0;
+    if (U == 1) {
+        for (uint32_t o = 0, k = 0; o < n; o += 8, ++k) x += mix_word(load_in_word(p + o, n - o < 8 ? n - o : 8), k);
+    } else if (n > 0) {
+        const uint32_t nw = (n + 7) >> 3;
+        tail_rounds<U>(p, n, [&](uint32_t k, const uint64_t (&w)[U]) {
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+                if (k + u < nw) x += mix_word(w[u], k + u);
+            return true;
+        });
+    }
+    return x;
+}
 // hash of a key given its first 16 bytes (w0, w1) and, for longer keys, its bytes at p
+template <int U = 1>
 __device__ __forceinline__ uint64_t hash_key16(uint32_t len, uint64_t seed, uint64_t w0, uint64_t w1, const uint8_t* p) {
-    uint64_t x = hash_word(hash_word(hash_init(len, seed), w0), w1);
-    for (uint32_t o = 16; o < len; o += 8) x = hash_word(x, load_in_word(p + o, len - o < 8 ? len - o : 8));
+    uint64_t x = hash_head(len, seed, w0, w1);
+    if (len > 16) x += tail_sum<U>(p + 16, len - 16);
     return fmix64(x);
+}
+// Warp-cooperative pieces for one long key (all 32 lanes call with the same p, n; n >= 1): lane l
+// takes the key words l, l + 32, ... of the input bytes [p, p+n) — one coalesced load per lane and
+// a shuffle for the neighbouring aligned word — instead of one lane walking the whole key.
+__device__ __forceinline__ uint64_t shfl_down64(uint64_t v, uint32_t d) {
+    const uint32_t lo = __shfl_down_sync(0xffffffffu, (uint32_t)v, d), hi = __shfl_down_sync(0xffffffffu, (uint32_t)(v >> 32), d);
+    return ((uint64_t)hi << 32) | lo;
+}
+__device__ __forceinline__ uint64_t shfl_xor64(uint64_t v, uint32_t m) {
+    const uint32_t lo = __shfl_xor_sync(0xffffffffu, (uint32_t)v, m), hi = __shfl_xor_sync(0xffffffffu, (uint32_t)(v >> 32), m);
+    return ((uint64_t)hi << 32) | lo;
+}
+template <typename F>
+__device__ __forceinline__ void warp_tail_words(const uint8_t* p, uint32_t n, F&& f) {
+    const uint32_t lane = threadIdx.x & 31u;
+    const uintptr_t a = reinterpret_cast<uintptr_t>(p);
+    const bool o = (a >> 2) & 1u;
+    const uint32_t s = 8u * (uint32_t)(a & 3u);
+    const unsigned long long* q = reinterpret_cast<const unsigned long long*>(a & ~(uintptr_t)7);
+    const uint32_t naw = ((uint32_t)(a & 7u) + n + 7u) >> 3, nw = (n + 7u) >> 3;
+    const uint64_t lm = last_word_mask(n);
+    for (uint32_t k0 = 0; k0 < nw; k0 += 32) {
+        const uint32_t k = k0 + lane;
+        const uint64_t x = k < naw ? ld_tail64(q + k) : 0ull;
+        uint64_t y = shfl_down64(x, 1);
+        if (lane == 31 && k + 1 < naw) y = ld_tail64(q + k + 1);
+        uint64_t w = key_word(x, y, o, s);
+        if (k == nw - 1) w &= lm;
+        if (!f(k, k < nw, w)) return;
+    }
+}
+// the tail sum of hash_key16 for the key bytes [p, p+n) (p = key + 16), in every lane
+__device__ __forceinline__ uint64_t warp_tail_sum(const uint8_t* p, uint32_t n) {
+    uint64_t acc = 0;
+    warp_tail_words(p, n, [&](uint32_t k, bool in, uint64_t w) {
+        if (in) acc += mix_word(w, k);
+        return true;
+    });
+#pragma unroll
+    for (uint32_t o = 16; o; o >>= 1) acc += shfl_xor64(acc, o);
+    return acc;
+}
+// input bytes [p, p+n) == the zero-padded entry words at ek (8-aligned), in every lane
+__device__ __forceinline__ bool warp_tail_eq(const uint8_t* ek, const uint8_t* p, uint32_t n) {
+    bool eq = true;
+    warp_tail_words(p, n, [&](uint32_t k, bool in, uint64_t w) {
+        eq = !__any_sync(0xffffffffu, in && ldcg64(ek + 8 * k) != w);
+        return eq;
+    });
+    return eq;
 }
 __device__ __forceinline__ void load_key16(const uint8_t* p, uint32_t len, uint64_t& w0, uint64_t& w1);
 __device__ __forceinline__ uint64_t hash_key(const uint8_t* p, uint32_t len, uint64_t seed) {
@@ -240,12 +360,26 @@ __device__ __forceinline__ uint8_t* ref_ptr(const Dev& d, uint32_t ref) { return
 __device__ __forceinline__ uint32_t off_ref(uint64_t off) { return (uint32_t)(off >> 3) + 1u; }
 
 // Key equality: entry key at e + koff (8-aligned, zero padded) vs input key [p, p+len).
+// U > 1: the entry words of a round are loaded with the input words (no dependency between them).
+template <int U = 1>
 __device__ __forceinline__ bool entry_key_eq(const uint8_t* ek, const uint8_t* p, uint32_t len) {
-    for (uint32_t o = 0; o < len; o += 8) {
-        uint32_t nb = len - o < 8 ? len - o : 8;
-        if (ldcg64(ek + o) != load_in_word(p + o, nb)) return false;
+    if (U == 1) {
+        for (uint32_t o = 0; o < len; o += 8) {
+            uint32_t nb = len - o < 8 ? len - o : 8;
+            if (ldcg64(ek + o) != load_in_word(p + o, nb)) return false;
+        }
+        return true;
     }
-    return true;
+    if (len == 0) return true;
+    const uint32_t nw = (len + 7) >> 3;
+    bool eq = true;
+    tail_rounds<U>(p, len, [&](uint32_t k, const uint64_t (&w)[U]) {
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+            if (k + u < nw) eq = eq && ldcg64(ek + 8 * (k + u)) == w[u];
+        return eq;
+    });
+    return eq;
 }
 // Input-vs-input key equality (both immutable input bytes)
 __device__ __forceinline__ bool in_key_eq(const uint8_t* a, const uint8_t* b, uint32_t len) {
@@ -256,11 +390,23 @@ __device__ __forceinline__ bool in_key_eq(const uint8_t* a, const uint8_t* b, ui
     return true;
 }
 // Copy an input key into an entry (8-aligned destination, zero padded tail)
+template <int U = 1>
 __device__ __forceinline__ void store_key(uint8_t* ek, const uint8_t* p, uint32_t len) {
-    for (uint32_t o = 0; o < len; o += 8) {
-        uint32_t nb = len - o < 8 ? len - o : 8;
-        *reinterpret_cast<unsigned long long*>(ek + o) = load_in_word(p + o, nb);
+    if (U == 1) {
+        for (uint32_t o = 0; o < len; o += 8) {
+            uint32_t nb = len - o < 8 ? len - o : 8;
+            *reinterpret_cast<unsigned long long*>(ek + o) = load_in_word(p + o, nb);
+        }
+        return;
     }
+    if (len == 0) return;
+    const uint32_t nw = (len + 7) >> 3;
+    tail_rounds<U>(p, len, [&](uint32_t k, const uint64_t (&w)[U]) {
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+            if (k + u < nw) *reinterpret_cast<unsigned long long*>(ek + 8 * (k + u)) = w[u];
+        return true;
+    });
 }
 
 __device__ __forceinline__ uint4 ldcg128(const void* p) { return __ldcg(reinterpret_cast<const uint4*>(p)); }
@@ -282,6 +428,7 @@ __device__ __forceinline__ uint8_t* chain_find(const Dev& d, uint32_t ref, uint3
 }
 // Same, with the key's first 16 bytes in registers (w0, w1 zero padded); bytes >= 16 of a long
 // key are compared against `tail` (the input key + 16).
+template <int U = 1>
 __device__ __forceinline__ uint8_t* chain_find_w(const Dev& d, uint32_t ref, uint32_t stop, uint32_t tag, uint32_t len,
                                                  uint64_t w0, uint64_t w1, const uint8_t* tail) {
     const uint64_t m0 = len ? ~0ull : 0ull, m1 = len > 8 ? ~0ull : 0ull;  // words that hold key bytes
@@ -290,7 +437,7 @@ __device__ __forceinline__ uint8_t* chain_find_w(const Dev& d, uint32_t ref, uin
         const uint4 hd = ldcg128(e);
         const ulonglong2 kw = ldcg128u(e + KEY_OFF);
         bool eq = hd.z == tag && hd.w == len && !((kw.x ^ w0) & m0) && !((kw.y ^ w1) & m1);
-        if (len > 16) eq = eq && entry_key_eq(e + KEY_OFF + 16, tail, len - 16);
+        if (len > 16) eq = eq && entry_key_eq<U>(e + KEY_OFF + 16, tail, len - 16);
         if (eq) return e;
         ref = hd.y;
     }

@@ -507,7 +507,7 @@ __device__ __forceinline__ void in_stage1(const Batch& b, const InCtx& c, uint32
 // Stage 2: the group's key-byte window [base & ~15, min(start of its last record + 16, kend)) —
 // the first 16 bytes of every key — as 16-B chunks, chunk `lane` per lane. `win` returns the low
 // 32 bits of the aligned window base with bit 0 = the window was loaded (fits 32 x 16 B).
-template <int IN>
+template <int IN, bool PF = false>
 __device__ __forceinline__ uint4 in_stage2(const Batch& b, const InCtx& c, uint32_t g, uint32_t lane, uint64_t s,
                                            uint32_t& win) {
     uint4 ch = make_uint4(0, 0, 0, 0);
@@ -524,6 +524,10 @@ __device__ __forceinline__ uint4 in_stage2(const Batch& b, const InCtx& c, uint3
     }
     const uint64_t base_al = base & ~15ull;
     const uint64_t wend = min(last + 16, c.kend);
+    if (PF) {  // long keys: bring the group's bytes (up to 4 KB from its first key) into L2 a group early
+        const uint64_t a = (base & ~127ull) + 128ull * lane;
+        if (a < min(last + 256, c.kend)) asm volatile("prefetch.global.L2 [%0];" ::"l"(b.keys + a));
+    }
     const bool fast = c.kal && wend - base_al <= 512;
     win = (uint32_t)base_al | (fast ? 1u : 0u);
     if (fast && base_al + 16ull * lane < wend) ch = ld_in128(b.keys + base_al + 16ull * lane);
@@ -602,8 +606,32 @@ __device__ __forceinline__ void prep_close(const Batch& b, const PrepCursor& pc)
     }
 }
 
+// Long-key kernels (TU > 1): keys longer than COOP_LEN bytes have their tails hashed and compared by
+// the whole warp, one key at a time (warp_tail_sum / warp_tail_eq); shorter tails stay per lane,
+// TU words per round trip. Per-lane loops run as long as the warp's longest key, so without the
+// split one URL of 200 B kept a warp at 7 of 32 active lanes (r02 C3 ncu source page: 10 of 32
+// average over the kernel).
+#ifndef SEPO_COOP_LEN
+#define SEPO_COOP_LEN 112  // C3 1x pass 1: 80 -> 40.3 ms (est.), 96 39.3, 112 39.1, 144 40.3, no warp path 48.5
+#endif
+constexpr uint32_t COOP_LEN = SEPO_COOP_LEN;
+// verify the tails of the lanes in `cm` (each against its own entry tail) with the whole warp
+__device__ __forceinline__ bool coop_verify(unsigned cm, bool eq, const uint8_t* ek, const uint8_t* tail, uint32_t tlen) {
+    const uint32_t lane = lane_id();
+    while (cm) {
+        const int j = __ffs(cm) - 1;
+        cm &= cm - 1;
+        const uint8_t* ej = reinterpret_cast<const uint8_t*>(__shfl_sync(FULLMASK, reinterpret_cast<uintptr_t>(ek), j));
+        const uint8_t* pj = reinterpret_cast<const uint8_t*>(__shfl_sync(FULLMASK, reinterpret_cast<uintptr_t>(tail), j));
+        const uint32_t nj = __shfl_sync(FULLMASK, tlen, j);
+        const bool r = warp_tail_eq(ej, pj, nj);
+        if (lane == (uint32_t)j) eq = r;
+    }
+    return eq;
+}
+
 // RB: bytes of a prepared re-issue record written for a declined record (32: implicit value 1)
-template <int RB>
+template <int RB, int TU = 1>
 __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, stream::CtaState& S, bool act, uint64_t w0,
                                              uint64_t w1, uint64_t h, uint64_t s, uint64_t v, uint32_t len, uint32_t g,
                                              uint32_t gl, bool inj, bool& w_full, bool& w_quiet, PrepCursor& pc,
@@ -618,16 +646,25 @@ __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, strea
     // the allocation path, or by the post-quiescence re-walk of a decline
     uint32_t head = act ? (hinted ? hint : ld_dir(d.dir + bkt)) : 0u;
     uint8_t* found = nullptr;
+    const uint8_t* e = ref_ptr(d, head);
+    bool eq = false;
+    uint32_t nxt = 0;
     if (head) {
-        const uint8_t* e = ref_ptr(d, head);
         const uint4 e_hd = ldcg128(e);
         const ulonglong2 e_kw = ldcg128u(e + KEY_OFF);
         // entry key words are zero padded to 8 bytes and followed by the value: a key of at most 8
         // bytes compares one word, an empty key none
         const uint64_t m0 = len ? ~0ull : 0ull, m1 = len > 8 ? ~0ull : 0ull;
-        bool eq = e_hd.z == tag && e_hd.w == len && !((e_kw.x ^ w0) & m0) && !((e_kw.y ^ w1) & m1);
-        if (len > 16) eq = eq && entry_key_eq(e + KEY_OFF + 16, tail, len - 16);
-        found = eq ? const_cast<uint8_t*>(e) : chain_find_w(d, e_hd.y, 0, tag, len, w0, w1, tail);
+        eq = e_hd.z == tag && e_hd.w == len && !((e_kw.x ^ w0) & m0) && !((e_kw.y ^ w1) & m1);
+        if (TU == 1 || len <= COOP_LEN) {
+            if (len > 16) eq = eq && entry_key_eq<TU>(e + KEY_OFF + 16, tail, len - 16);
+        }
+        nxt = e_hd.y;
+    }
+    // long keys (TU > 1): the head's tail compared by the whole warp (every lane takes part)
+    if (TU > 1) eq = coop_verify(__ballot_sync(FULLMASK, eq && len > COOP_LEN), eq, e + KEY_OFF + 16, tail, len - 16);
+    if (head) {
+        found = eq ? const_cast<uint8_t*>(e) : chain_find_w<TU>(d, nxt, 0, tag, len, w0, w1, tail);
         if (found) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(found, len)), v);
     }
     // ---- new keys: allocate + link (a5, a6), decline (a7)
@@ -665,13 +702,13 @@ __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, strea
             *reinterpret_cast<uint4*>(e) = make_uint4(esize | K_COMBINE, hd, tag, len);
             if (len > 0) *reinterpret_cast<unsigned long long*>(e + KEY_OFF) = w0;
             if (len > 8) *reinterpret_cast<unsigned long long*>(e + KEY_OFF + 8) = w1;
-            if (len > 16) store_key(e + KEY_OFF + 16, tail, len - 16);
+            if (len > 16) store_key<TU>(e + KEY_OFF + 16, tail, len - 16);
             *reinterpret_cast<unsigned long long*>(entry_val(e, len)) = v;
             const uint32_t me = off_ref(off);
             while (true) {  // lock-free head insertion
                 const uint32_t old = cas_release(d.dir + bkt, hd, me);
                 if (old == hd) break;
-                uint8_t* w = chain_find_w(d, old, hd, tag, len, w0, w1, tail);
+                uint8_t* w = chain_find_w<TU>(d, old, hd, tag, len, w0, w1, tail);
                 if (w) {  // linked meanwhile by another warp: combine there, retire ours
                     red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
                     *reinterpret_cast<uint32_t*>(e) = esize | K_DEAD;
@@ -694,7 +731,7 @@ __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, strea
                     while (ld_acquire_u64(d.ann + (uint64_t)cs * ANN_STRIDE) != ANN_FULL) __nanosleep(64);
             __syncwarp();
             if (declined) {
-                uint8_t* w = chain_find_w(d, ld_dir(d.dir + bkt), 0, tag, len, w0, w1, tail);
+                uint8_t* w = chain_find_w<TU>(d, ld_dir(d.dir + bkt), 0, tag, len, w0, w1, tail);
                 if (w) red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(w, len)), v);
                 else res = R_POST;
             }
@@ -748,7 +785,7 @@ __device__ __forceinline__ void resolve_core(const Dev& d, const Batch& b, strea
 }
 
 // Resolve up to 32 queued misses of the stream kernel, one per lane.
-template <bool VALS, int WARPS>
+template <bool VALS, int WARPS, int TU>
 __device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, stream::Smem<VALS, WARPS>& S,
                                                typename stream::Smem<VALS, WARPS>::Queue& Q, uint32_t qhead,
                                                uint32_t cnt, bool inj, bool& w_full, bool& w_quiet, PrepCursor& pc) {
@@ -764,9 +801,9 @@ __device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, str
         const uint32_t ll = Q.ll[k];
         len = ll >> 5; gl = ll & 31u;
     }
-    if (!VALS) resolve_core<32>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
-    else if (b.prep_fmt == 33) resolve_core<33>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
-    else resolve_core<48>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
+    if (!VALS) resolve_core<32, TU>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
+    else if (b.prep_fmt == 33) resolve_core<33, TU>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
+    else resolve_core<48, TU>(d, b, S.cs, act, w0, w1, h, s, v, len, g, gl, inj, w_full, w_quiet, pc);
 }
 
 // Reinsert pass of sepo_run (a9 re-issue): the prepared records of the previous pass, 32 per warp
@@ -774,7 +811,7 @@ __device__ __forceinline__ void resolve_misses(const Dev& d, const Batch& b, str
 #ifndef SEPO_REINS_THREADS
 #define SEPO_REINS_THREADS 1024
 #endif
-template <int RB>
+template <int RB, int TU = 1>
 __global__ void __launch_bounds__(SEPO_REINS_THREADS, 1) reinsert_kernel(Dev d, Batch b) {
     __shared__ stream::CtaState S;
     const uint32_t tid = threadIdx.x, lane = lane_id();
@@ -827,8 +864,8 @@ __global__ void __launch_bounds__(SEPO_REINS_THREADS, 1) reinsert_kernel(Dev d, 
         } else {
             act = i < b.n && len != PREP_HOLE;
         }
-        resolve_core<RB>(d, b, S, act, r0.x, kw1, r1.x, s, v, act ? len : 0u, (uint32_t)(i >> 5), (uint32_t)(i & 31), inj,
-                     w_full, w_quiet, pc);
+        resolve_core<RB, TU>(d, b, S, act, r0.x, kw1, r1.x, s, v, act ? len : 0u, (uint32_t)(i >> 5), (uint32_t)(i & 31),
+                             inj, w_full, w_quiet, pc);
     }
     if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
     __syncthreads();
@@ -948,7 +985,10 @@ __global__ void __launch_bounds__(1024, 1) insert_basic_kernel(Dev d, Batch b, u
 // host as a kernel parameter: in the constant bank a loop-invariant costs one load when the
 // register-bound loop (64 registers x 1024 threads) rematerialises it, not its whole computation
 // (measured ~30 warp instructions per group before).
-template <bool VALS, int THREADS, int IN>
+#ifndef SEPO_LONG_PF
+#define SEPO_LONG_PF 1
+#endif
+template <bool VALS, int THREADS, int IN, int TU = 1>
 __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch b, const hot::Entry* hl,
                                                                    const unsigned int* n_hot, const InCtx c) {
     constexpr int WARPS = THREADS / 32;
@@ -1003,7 +1043,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
     while (g < c.ngroups) {
         // ---- issue ahead: key chunks of gn, offsets (values) of the group after it
         uint32_t win_n;
-        const uint4 ch_n = in_stage2<IN>(b, c, gn, lane, s_n, win_n);
+        const uint4 ch_n = in_stage2<IN, (TU > 1 && SEPO_LONG_PF)>(b, c, gn, lane, s_n, win_n);
         const uint32_t gnn = stream::next_group(gn, c.nw);
         uint64_t s_nn, v_nn;
         uint32_t eo_nn = 0;
@@ -1015,7 +1055,23 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         uint32_t len;
         in_stage3<IN>(b, c, g, gn, lane, valid, s_n, eo_c, ch_c, win_c, s, len, w0, w1);
         const uint64_t v = VALS ? (IN == IN_IDX ? (valid ? rec_value(b, (uint64_t)g * 32 + lane) : 0ull) : v_c) : 1ull;
-        const uint64_t h = hash_key16(len, d.seed, w0, w1, b.keys + s);
+        uint64_t h;
+        if (TU == 1) {
+            h = hash_key16<TU>(len, d.seed, w0, w1, b.keys + s);
+        } else {  // long-key kernel: tails up to COOP_LEN per lane, longer ones by the whole warp
+            uint64_t x = hash_head(len, d.seed, w0, w1);
+            if (len > 16 && len <= COOP_LEN) x += tail_sum<TU>(b.keys + s + 16, len - 16);
+            unsigned cm = __ballot_sync(FULLMASK, len > COOP_LEN);
+            while (cm) {
+                const int j = __ffs(cm) - 1;
+                cm &= cm - 1;
+                const uint64_t sj = __shfl_sync(FULLMASK, s, j);
+                const uint32_t nj = __shfl_sync(FULLMASK, len, j) - 16u;
+                const uint64_t r = warp_tail_sum(b.keys + sj + 16, nj);
+                if (lane == (uint32_t)j) x += r;
+            }
+            h = fmix64(x);
+        }
         // ---- hot set (a2): both 4-way fingerprint buckets, then one 16-byte key compare
         int pos = -1;
         if (have_hot) {
@@ -1024,14 +1080,25 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
             constexpr uint32_t IM = (1u << stream::IDXB) - 1u;
             const bool m1 = (t1 & ~IM) == f, m2 = (t2 & ~IM) == f;
             const uint32_t p = (m1 ? t1 : t2) & IM;
+            const uint8_t* he = nullptr;
             if (valid && (m1 || m2)) {
                 const ulonglong2 kk = S.kw[p];
                 bool eq = kk.x == w0 && kk.y == w1;
                 if (len > 16) {  // long key: exact length (the fingerprint saturates at 255) + tail bytes
-                    const uint8_t* e = ref_ptr(d, S.ref[p]);
-                    eq = eq && ldcg32(e + 12) == len && entry_key_eq(e + KEY_OFF + 16, b.keys + s + 16, len - 16);
+                    he = ref_ptr(d, S.ref[p]);
+                    if (TU == 1) {
+                        eq = eq && ldcg32(he + 12) == len && entry_key_eq<TU>(he + KEY_OFF + 16, b.keys + s + 16, len - 16);
+                    } else {
+                        eq = eq && (len < 255u || ldcg32(he + 12) == len);
+                        if (len <= COOP_LEN) eq = eq && entry_key_eq<TU>(he + KEY_OFF + 16, b.keys + s + 16, len - 16);
+                    }
                 }
                 if (eq) pos = (int)p;
+            }
+            if (TU > 1) {
+                const bool ok = coop_verify(__ballot_sync(FULLMASK, pos >= 0 && len > COOP_LEN), pos >= 0, he + KEY_OFF + 16,
+                                            b.keys + s + 16, len - 16);
+                if (!ok) pos = -1;
             }
         }
         // ---- fold the hits of the warp per hot slot (a2): one shared atomic per distinct key
@@ -1081,7 +1148,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         qtail += __popc(mm);
         __syncwarp();
         if (qtail - qhead >= 32) {
-            resolve_misses<VALS, WARPS>(d, b, S, Q, qhead, 32, inj, w_full, w_quiet, pc);
+            resolve_misses<VALS, WARPS, TU>(d, b, S, Q, qhead, 32, inj, w_full, w_quiet, pc);
             qhead += 32;
             __syncwarp();
         }
@@ -1092,7 +1159,7 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         s_n = s_nn; v_n = v_nn;
         eo_c = eo_n; eo_n = eo_nn;
     }
-    if (qtail != qhead) resolve_misses<VALS, WARPS>(d, b, S, Q, qhead, qtail - qhead, inj, w_full, w_quiet, pc);
+    if (qtail != qhead) resolve_misses<VALS, WARPS, TU>(d, b, S, Q, qhead, qtail - qhead, inj, w_full, w_quiet, pc);
     if (b.out && pc.used < PREP_CHUNK) prep_close(b, pc);
     __syncthreads();
     // flush the hot keys' pending sums into their resident entries
@@ -1111,6 +1178,13 @@ __global__ void __launch_bounds__(THREADS, 1) insert_stream_kernel(Dev d, Batch 
         if (S.cs.pkb) atomicAdd(&d.ctrl->kept_key_bytes, S.cs.pkb);
     }
 }
+
+#ifndef SEPO_LONG_THREADS
+#define SEPO_LONG_THREADS 1024
+#endif
+#ifndef SEPO_LONG_U
+#define SEPO_LONG_U 2  // words per round trip: 2 -> C3 1x pass 1 39.1 ms; 3 40.8; 4 50.5 (spills at 64 registers)
+#endif
 
 // ================================================================ COMBINE insert, lean input path (a1..a7)
 // Pass-1 COMBINE kernel for contiguous batches (CSR keys or fixed-width keys) whose keys are mostly
@@ -3203,7 +3277,8 @@ int sepo_launch_evict_copy(const Dev& d, uint32_t n, uint8_t* dst, int grid, cud
 }
 
 int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
-                       uint32_t halt_slots, uint64_t key_end, bool dir_prefetch, bool* hot_built, bool lean_in) {
+                       uint32_t halt_slots, uint64_t key_end, bool dir_prefetch, bool* hot_built, bool lean_in,
+                       bool long_keys) {
     if (hot_built) *hot_built = false;
     if (mode == 2) {
         insert_basic_kernel<<<grid, 1024, 0, s>>>(d, b, halt_slots);
@@ -3310,6 +3385,18 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
             if (in == IN_CSR) insert_stream_kernel<true, T, IN_CSR><<<grid, T, sm, s>>>(d, b, hl, nh, c);
             else if (in == IN_FIXED) insert_stream_kernel<true, T, IN_FIXED><<<grid, T, sm, s>>>(d, b, hl, nh, c);
             else insert_stream_kernel<true, T, IN_IDX><<<grid, T, sm, s>>>(d, b, hl, nh, c);
+        } else if (in == IN_CSR && long_keys) {
+            // long keys: tails read SEPO_LONG_U words per round trip (tail_rounds)
+            constexpr int TL = SEPO_LONG_THREADS;
+            static bool attr3 = false;
+            if (!attr3) {
+                cudaFuncSetAttribute(insert_stream_kernel<false, TL, IN_CSR, SEPO_LONG_U>,
+                                     cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(stream::Smem<false, TL / 32>));
+                attr3 = true;
+            }
+            c.nw = (uint32_t)grid * (TL / 32);
+            insert_stream_kernel<false, TL, IN_CSR, SEPO_LONG_U>
+                <<<grid, TL, sizeof(stream::Smem<false, TL / 32>), s>>>(d, b, hl, nh, c);
         } else {
             if (in == IN_CSR) insert_stream_kernel<false, T, IN_CSR><<<grid, T, sm, s>>>(d, b, hl, nh, c);
             else if (in == IN_FIXED) insert_stream_kernel<false, T, IN_FIXED><<<grid, T, sm, s>>>(d, b, hl, nh, c);
@@ -3347,9 +3434,10 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
     }
     return cudaGetLastError();
 }
-int sepo_launch_reinsert(const Dev& d, const Batch& b, int grid, cudaStream_t s) {
+int sepo_launch_reinsert(const Dev& d, const Batch& b, int grid, cudaStream_t s, bool long_keys) {
     if (b.n == 0) return cudaGetLastError();
-    if (b.prep_fmt == 33) reinsert_kernel<33><<<grid, SEPO_REINS_THREADS, 0, s>>>(d, b);
+    if (long_keys && b.prep_rb == 32 && b.prep_fmt != 33) reinsert_kernel<32, SEPO_LONG_U><<<grid, SEPO_REINS_THREADS, 0, s>>>(d, b);
+    else if (b.prep_fmt == 33) reinsert_kernel<33><<<grid, SEPO_REINS_THREADS, 0, s>>>(d, b);
     else if (b.prep_rb == 32) reinsert_kernel<32><<<grid, SEPO_REINS_THREADS, 0, s>>>(d, b);
     else reinsert_kernel<48><<<grid, SEPO_REINS_THREADS, 0, s>>>(d, b);
     return cudaGetLastError();

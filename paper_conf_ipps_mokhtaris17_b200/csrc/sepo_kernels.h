@@ -55,13 +55,15 @@ static_assert(sizeof(WireRec) == 32, "WireRec layout");
 
 // key_end: key_offsets[n] of a CSR batch (the end of its key bytes), read by the host
 // lean_in: COMBINE contiguous batches take insert_lean_kernel (mostly short keys; the host decides)
+// long_keys: a CSR COMBINE batch of long keys (URLs): the stream kernel instantiation that reads key
+// tails several words per round trip
 // *hot_built (optional): whether this launch selected a sampled hot set (its size is the u32 at
 // hot_scratch + sepo_hot_count_offset(), clamped to the kernel's capacity)
 int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int grid, cudaStream_t s, void* hot_scratch,
                        uint32_t halt_slots = 0, uint64_t key_end = 0, bool dir_prefetch = false,
-                       bool* hot_built = nullptr, bool lean_in = false);
+                       bool* hot_built = nullptr, bool lean_in = false, bool long_keys = false);
 size_t sepo_hot_count_offset();
-int sepo_launch_reinsert(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s);
+int sepo_launch_reinsert(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s, bool long_keys = false);
 // Router with CTA pre-combine (a12): pass 0 counts per-part output records (part_totals[P], device,
 // zeroed by the caller) and flags keys longer than 16 bytes in *long_keys; pass 1 writes the
 // WireRecs of part p at out + part_base[p] (device, exclusive prefix of the totals) through the
