@@ -288,7 +288,6 @@ def run_reference(args):
 # ---------------------------------------------------------------- our arm
 def timed_steps(job, t, steps, stream, route_fn=None):
     import torch
-    k, o, v = job.inputs() if route_fn is None else (None, None, None)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ins_ms, launches, recs_ins, kb_ins, vb_ins, p1_ms = 0.0, 0, 0, 0, 0, 0.0
     torch.cuda.synchronize()
@@ -298,10 +297,7 @@ def timed_steps(job, t, steps, stream, route_fn=None):
             route_fn()
             launches += 2
         t.reset()
-        if route_fn is not None:
-            job.run_fn(t)
-        else:
-            t.run(k, o, v)
+        job.run_job(t)
         st = t.stats()
         ins_ms += st["t_insert_ms"]
         p1_ms += st["t_insert_ms_per_pass"][0]
@@ -619,6 +615,7 @@ def run_routed(args, world, rank, local):
     sk, so, sv = job.stream.device(j0, j1 - j0)
     if fixed:
         so = None
+    lib_plane = args.plane == "lib"
     router = shard.Router(route_seed=0x5eed, fixed_key_width=8 if fixed else 0,
                           fixed_val_width=job.stream.val_width if sv is not None else 0,
                           # pre-combine for fixed-width pairs (C5: SURVEY §8(e) makes it mandatory for
@@ -627,18 +624,35 @@ def run_routed(args, world, rank, local):
                           combine=job.stream.family == 2 and not args.no_combine)
     routed = {}
 
-    def route_fn():
-        routed["r"] = router.route(sk, so, sv)
-        return routed["r"]
-    job.run_fn = lambda t: shard.Router.run(t, routed["r"])
+    def attach(t):  # the library's own NCCL communicator (rank 0 makes the id, torch.distributed carries it)
+        if not getattr(t, "_attached", False):
+            uid = [job.sepo.nccl_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(uid, src=0)
+            t.attach_nccl(uid[0], world, rank)
+            t._attached = True
+
+    if lib_plane:
+        # sepo_run_sharded: route + NCCL exchange of chunk c+1 on a second stream beside chunk c's insert
+        route_fn = None
+
+        def run_lib(t, k=sk, o=so, v=sv):
+            attach(t)
+            return t.run_sharded(k, o, v)
+        job.run_fn = run_lib
+    else:
+        def route_fn():
+            routed["r"] = router.route(sk, so, sv)
+            return routed["r"]
+        job.run_fn = lambda t: shard.Router.run(t, routed["r"])
+        route_fn()
     job.distinct = max(1, job.distinct // world)  # keys per rank (sizes the directory)
-    route_fn()
     slice_bytes = sk.numel() + (8 * (so.numel() - 1) if so is not None else 0) + (sv.numel() if sv is not None else 0)
     job.bytes_hint = slice_bytes
     nb, pages, F = job.table_params()
     t = job.table()
     for _ in range(max(args.warmup, 3)):
-        route_fn()
+        if route_fn is not None:
+            route_fn()
         t.reset()
         job.run_fn(t)
     sampler = ClockSampler(local)
@@ -669,9 +683,12 @@ def run_routed(args, world, rank, local):
             dk = hk.to("cuda", non_blocking=True)
             do = ho.to("cuda", non_blocking=True) if ho is not None else None
             dv = hv.to("cuda", non_blocking=True) if hv is not None else None
-            r = router.route(dk, do, dv)
+            torch.cuda.current_stream().synchronize()  # (the table works on its own stream)
             t.reset()
-            shard.Router.run(t, r)
+            if lib_plane:
+                job.run_fn(t, dk, do, dv)
+            else:
+                shard.Router.run(t, router.route(dk, do, dv))
             t.export(copy=False)
             d2h += t.stats()["bytes_evicted"]
         torch.cuda.synchronize()
@@ -680,8 +697,9 @@ def run_routed(args, world, rank, local):
         el = float(el.item()) / args.e2e_steps
         e2e = {"value": csr / el / 1e9, "unit": "GB/s", "h2d_bytes_per_step": slice_bytes,
                "d2h_bytes_per_step": d2h // args.e2e_steps, "kv_inserts_per_s": n_all / el,
-               "note": "per rank: pinned host slice -> H2D -> route (partition + all-to-all) -> sepo_run -> sepo_export; "
-                       "max over ranks"}
+               "note": "per rank: pinned host slice -> H2D -> " + (
+                   "sepo_run_sharded (route + NCCL exchange pipelined with pass 1, re-issue passes)" if lib_plane else
+                   "route (partition + all-to-all) -> sepo_run") + " -> sepo_export; max over ranks"}
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
                 "warmup": max(args.warmup, 3), "ms_per_step": ms / args.steps, "higher_is_better": True,
@@ -690,11 +708,13 @@ def run_routed(args, world, rank, local):
                 "config": {"workload": CONFIG_TEXT[args.config] + " [CSR job, key-hash sharded]", "records": n_all,
                            "input_csr_bytes": csr, "ratio_table_over_budget": args.ratio, "n_buckets": nb,
                            "page_bytes": job.page_bytes, "pool_pages": pages, "passes": st["passes"],
-                           "parallelism": f"key-hash sharded x{world} (sepo_partition + all-to-all, pre-combined)",
+                           "parallelism": f"key-hash sharded x{world} " + (
+                               "(sepo_run_sharded: in-library NCCL send/recv, exchange pipelined with pass 1)" if lib_plane
+                               else "(sepo_partition / pre-combine + torch.distributed all-to-all)"),
                            "l2": "inputs far larger than L2 (126 MB): no flush needed"},
                 "roofline": roofline_of(slice_bytes, info["p1_ms"], args.steps, peaks(),
                                         "pass-1 insert kernel of this rank's job", {"share_of_step": info["p1_ms"] / ms}),
-                "route": router.last_stats(), "e2e": e2e, "clocks": clocks, "gpu_launches": info["launches"],
+                "route": {"plane": "libsepo NCCL (sepo_run_sharded)"} if lib_plane else router.last_stats(), "e2e": e2e, "clocks": clocks, "gpu_launches": info["launches"],
                 "cpu_baseline": None}
         print(json.dumps(line), flush=True)
     t.close()
@@ -720,6 +740,8 @@ def main():
     ap.add_argument("--ref-seconds", type=float, default=15.0)
     ap.add_argument("--route", action="store_true", help="run the sharded (router) path even at N=1")
     ap.add_argument("--no-combine", action="store_true", help="routed path: CSR partition without the pre-combine")
+    ap.add_argument("--plane", choices=["lib", "torch"], default="lib",
+                    help="routed path: the library's pipelined NCCL job (sepo_run_sharded) or torch.distributed all-to-all")
     ap.add_argument("--traffic", type=float, default=None, help="dram bytes/launch from an ncu --set full capture")
     args = ap.parse_args()
     if args.impl == "reference":

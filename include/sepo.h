@@ -320,6 +320,18 @@ int sepo_attach_nccl(sepo_table* t, const void* nccl_unique_id, int nranks, int 
 int64_t sepo_insert_batch_sharded(sepo_table* t, const uint8_t* keys, const uint64_t* key_offsets, const uint8_t* vals,
                                   const uint64_t* val_offsets, uint64_t n);
 int64_t sepo_drain(sepo_table* t);
+/* sepo_run_sharded: COLLECTIVE; the whole SEPO job over a batch sharded by key
+ *   owner, with the exchange pipelined against pass 1 (chunk c+1 is routed and exchanged
+ *   on a second stream while chunk c is inserted). COMBINE mode only; device inputs as sepo_insert_batch
+ *   (fixed-width values, val_offsets NULL; n may be 0 on some ranks). The ranks agree (one NCCL
+ *   all-reduce) on the number of chunks (SEPO_SHARD_CHUNK records each, default 2^26, a multiple of
+ *   2048) and on the format: pre-combined wire records when every rank's keys are <= 16 bytes, else a
+ *   CSR partition. Records declined in pass 1 become prepared re-issue records; the re-issue passes,
+ *   evictions and the final transfer to host run locally. Afterwards sepo_export gives this rank's
+ *   keys; the union over ranks is the result. Returns the number of passes or < 0 (SEPO_E_STATE if
+ *   records from sepo_insert_batch_sharded are held, SEPO_E_INVAL for GROUP / BASIC tables). */
+int64_t sepo_run_sharded(sepo_table* t, const uint8_t* keys, const uint64_t* key_offsets, const uint8_t* vals,
+                         const uint64_t* val_offsets, uint64_t n);
 
 const char* sepo_last_error(void);
 const char* sepo_version(void);

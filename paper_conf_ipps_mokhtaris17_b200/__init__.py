@@ -67,7 +67,8 @@ EXPORTS = ["sepo_create", "sepo_create_placed", "sepo_configure", "sepo_run_text
            "sepo_export", "sepo_run", "sepo_reset", "sepo_stats_get", "sepo_last_insert_ms", "sepo_destroy",
            "sepo_last_error", "sepo_version", "sepo_budget_for", "sepo_partition_scratch", "sepo_partition",
            "sepo_shift_offsets", "sepo_route_scratch", "sepo_route_combine", "sepo_run_wire", "sepo_nccl_unique_id",
-           "sepo_attach_nccl", "sepo_insert_batch_sharded", "sepo_drain", "sepo_map_run"]
+           "sepo_attach_nccl", "sepo_insert_batch_sharded", "sepo_drain", "sepo_map_run",
+           "sepo_run_sharded"]
 
 
 def nccl_unique_id():
@@ -114,6 +115,7 @@ def lib():
         L.sepo_attach_nccl.argtypes = [vp, vp, ctypes.c_int, ctypes.c_int]; L.sepo_attach_nccl.restype = ctypes.c_int
         L.sepo_insert_batch_sharded.argtypes = [vp, vp, vp, vp, vp, u64]; L.sepo_insert_batch_sharded.restype = i64
         L.sepo_drain.argtypes = [vp]; L.sepo_drain.restype = i64
+        L.sepo_run_sharded.argtypes = [vp, vp, vp, vp, vp, u64]; L.sepo_run_sharded.restype = i64
         L.sepo_map_run.argtypes = [vp, ctypes.c_int, vp, u64, vp, u64]; L.sepo_map_run.restype = i64
         _LIB = L
     return _LIB
@@ -273,6 +275,15 @@ class Table:
 
     def drain(self):
         rc = self._L.sepo_drain(self.h)
+        if rc < 0:
+            _err(rc)
+        return int(rc)
+
+    def run_sharded(self, keys, key_offsets, vals=None, n=None):
+        """collective: the whole SEPO job on a batch sharded by key owner, the exchange of chunk c+1
+        pipelined with the insert of chunk c (sepo_run_sharded); returns the number of passes"""
+        n = self._n(key_offsets, keys, n) if (keys is not None or key_offsets is not None) else 0
+        rc = self._L.sepo_run_sharded(self.h, _ptr(keys), _ptr(key_offsets), _ptr(vals), None, n)
         if rc < 0:
             _err(rc)
         return int(rc)

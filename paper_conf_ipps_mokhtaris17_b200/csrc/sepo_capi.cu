@@ -127,6 +127,8 @@ struct sepo_table {
     int shard_fmt = 0;        // records held: 0 none yet, 1 wire records, 2 CSR (keys, offsets[, values])
     DevBuf sh_send[3], sh_held[3], sh_tmp[3], sh_cnt;  // route output; records held; exchange scratch; counts
     uint64_t sh_n = 0, sh_kb = 0, sh_vb = 0;          // records / key bytes / value bytes held
+    cudaStream_t route_stream = nullptr;  // sepo_run_sharded: route + exchange of chunk c+1 beside chunk c's insert
+    DevBuf sh_recv[2];                    // sepo_run_sharded: wire records received (ping-pong per chunk)
     bool lookup_done = false;
     std::vector<cudaEvent_t>* h2d_chunks = nullptr;  // sepo_run on host input: copy events of pass-1 chunks
     uint64_t h2d_chunk_records = 0;  // sepo_lookup restored old generations into the pool: no inserts until reset
@@ -470,10 +472,35 @@ static bool dir_prefetch(sepo_table* t) {
     return (uint64_t)t->n_buckets * 4 + pages * (uint64_t)t->page_bytes > (uint64_t)l2;
 }
 
+// An insert pass over one batch, split so a caller can overlap other work with the kernel:
+// insert_begin enqueues it on t->stream without a host sync (key_begin / key_end = ko[0], ko[n]
+// for contiguous CSR batches, known to the caller), insert_end waits for it and reads the counters.
+struct InsertLaunch {
+    bool hot_built = false;
+    uint64_t key_bytes = 0;
+};
+static int insert_begin(sepo_table* t, const Batch& b, uint64_t key_begin, uint64_t key_end, InsertLaunch& L);
+static int64_t insert_end(sepo_table* t, const Batch& b, const InsertLaunch& L);
+
 static int64_t insert_impl(sepo_table* t, const Batch& b) {
+    if (b.n == 0) return 0;
+    uint64_t key_end = 0, key_begin = 0;
+    if (b.ko && !b.idx) {  // the end of the batch's key bytes, a kernel parameter (see the kernel)
+        CK(t, cudaMemcpyAsync(&t->h_ko[0], b.ko, 8, cudaMemcpyDeviceToHost, t->stream));
+        CK(t, cudaMemcpyAsync(&t->h_ko[1], b.ko + b.n, 8, cudaMemcpyDeviceToHost, t->stream));
+        CK(t, cudaStreamSynchronize(t->stream));
+        key_begin = t->h_ko[0];
+        key_end = t->h_ko[1];
+    }
+    InsertLaunch L;
+    int rc = insert_begin(t, b, key_begin, key_end, L);
+    if (rc) return rc;
+    return insert_end(t, b, L);
+}
+
+static int insert_begin(sepo_table* t, const Batch& b, uint64_t key_begin, uint64_t key_end, InsertLaunch& L) {
     int rc;
     const uint64_t n = b.n;
-    if (n == 0) return 0;
     trace("insert begin", n);
     if (!b.bitmap) return fail(SEPO_E_INVAL, "postponed_bitmap is NULL");
     t->inserted = true;
@@ -485,14 +512,8 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
     if (t->hot.grow(sepo_hot_scratch_bytes())) return fail(SEPO_E_NOMEM, "hot-set scratch");
     // BASIC halt rule: the pass stops once this many allocator slots failed
     const uint32_t halt_slots = (uint32_t)std::max<uint64_t>(1, ((uint64_t)t->grid * t->opts.basic_halt_pct + 99) / 100);
-    uint64_t key_end = 0, key_begin = 0;
-    if (b.ko && !b.idx) {  // the end of the batch's key bytes, a kernel parameter (see the kernel)
-        CK(t, cudaMemcpyAsync(&t->h_ko[0], b.ko, 8, cudaMemcpyDeviceToHost, t->stream));
-        CK(t, cudaMemcpyAsync(&t->h_ko[1], b.ko + n, 8, cudaMemcpyDeviceToHost, t->stream));
-        CK(t, cudaStreamSynchronize(t->stream));
-        key_begin = t->h_ko[0];
-        key_end = t->h_ko[1];
-    }
+    if (b.idx) L.key_bytes = t->pending_idx_key_bytes;
+    else L.key_bytes = b.ko ? key_end - key_begin : n * (uint64_t)t->opts.fixed_key_width;
     // COMBINE pass 1 on contiguous input: the lean kernel unless the keys are long on average (URLs:
     // insert_stream_kernel's warp-window loads suit them better); SEPO_LEAN=0/1 forces the choice
     bool lean_in = false, long_keys = false;
@@ -506,20 +527,21 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
         const char* el = getenv("SEPO_LONG");
         long_keys = b.ko && ((el && (el[0] == '0' || el[0] == '1')) ? el[0] == '1' : mean > 24);
     }
-    bool hot_built = false;
     rc = sepo_launch_insert(t->d, b, t->opts.mode, t->grid, t->stream, t->hot.p, halt_slots, key_end, dir_prefetch(t),
-                            &hot_built, lean_in, long_keys);
+                            &L.hot_built, lean_in, long_keys);
     if (rc) return cuda_check(t, (cudaError_t)rc, "insert kernel launch");
     CK(t, cudaEventRecord(t->ev1, t->stream));
     t->h_ko[2] = 0;
-    if (hot_built)
+    if (L.hot_built)
         CK(t, cudaMemcpyAsync(&t->h_ko[2], (uint8_t*)t->hot.p + sepo_hot_count_offset(), 4, cudaMemcpyDeviceToHost,
                               t->stream));
     t->st.kernel_launches += (n >= (8ull << 18)) ? 7 : 1;
-    if (b.ko && !b.idx) {
-        CK(t, cudaMemcpyAsync(&t->h_ko[0], b.ko, 8, cudaMemcpyDeviceToHost, t->stream));
-        CK(t, cudaMemcpyAsync(&t->h_ko[1], b.ko + n, 8, cudaMemcpyDeviceToHost, t->stream));
-    }
+    return 0;
+}
+
+static int64_t insert_end(sepo_table* t, const Batch& b, const InsertLaunch& L) {
+    int rc;
+    const uint64_t n = b.n;
     if ((rc = read_ctrl(t))) return rc;
     t->st.hot_keys = std::max<uint64_t>(t->st.hot_keys, t->h_ko[2]);
     t->last_insert_ms = elapsed_ms(t->ev0, t->ev1);
@@ -528,8 +550,7 @@ static int64_t insert_impl(sepo_table* t, const Batch& b) {
     if (t->st.passes < SEPO_MAX_PASS_STATS) t->st.t_insert_ms_per_pass[t->st.passes] += t->last_insert_ms;
     t->st.insert_calls++;
     t->st.records_inserted += n;
-    if (b.idx) t->st.key_bytes_inserted += t->pending_idx_key_bytes;
-    else t->st.key_bytes_inserted += b.ko ? (t->h_ko[1] - t->h_ko[0]) : n * (uint64_t)t->opts.fixed_key_width;
+    t->st.key_bytes_inserted += L.key_bytes;
     t->st.val_bytes_inserted += b.vals ? n * (uint64_t)t->opts.fixed_val_width : 0;
     t->st.dead_bytes += t->h_ctrl->dead_bytes;
     const uint64_t used = std::min<uint64_t>(t->h_ctrl->pool_taken, t->d.n_free) + t->pages_resident_retained;
@@ -1674,6 +1695,8 @@ void sepo_destroy(sepo_table* t) {
     if (t->ev_comp) cudaEventDestroy(t->ev_comp);
     if (t->own_stream && t->stream) cudaStreamDestroy(t->stream);
     if (t->copy_stream) cudaStreamDestroy(t->copy_stream);
+    if (t->route_stream) cudaStreamDestroy(t->route_stream);
+    for (auto& b : t->sh_recv) b.release();
     delete t;
 }
 
@@ -2050,4 +2073,293 @@ int64_t sepo_drain(sepo_table* t) {
     t->sh_n = t->sh_kb = t->sh_vb = 0;
     t->shard_fmt = 0;
     return r;
+}
+
+// ---------------------------------------------------------------- pipelined sharded job (a12)
+// sepo_run_sharded: the whole SEPO job over a batch sharded by key owner, with pass 1 pipelined
+// against the exchange. The batch is cut into chunks (SEPO_SHARD_CHUNK records, a multiple of the
+// router's 2048-record tile); for chunk c the route stream runs the router and the two NCCL groups
+// (counts, payload) while t->stream inserts chunk c-1 — each insert waits only for its own chunk's
+// receive event, and the host reads an insert's counters only after the next chunk's exchange is
+// enqueued. Declined records become prepared re-issue records (a9; the list is kept large enough for
+// every record received so far, so pass 1 never needs an index re-issue), then the ordinary re-issue
+// passes and evictions run locally (no communication: a key's records all live on its owner).
+//   wire format (every rank's keys <= 16 bytes): pre-combined 32-byte records, received into a
+//     ping-pong pair of buffers (the prepared records carry the whole key);
+//   CSR (some key > 16 bytes): partitioned key bytes / offsets [/ values] appended to the records
+//     held (prepared records of long keys point into them), offsets rebased on the device.
+#if SEPO_WITH_NCCL
+namespace {
+// grow b to hold `need` bytes keeping its first `have` bytes (stream s is synchronised)
+int grow_keep(sepo_table* t, DevBuf& b, size_t have, size_t need, cudaStream_t s) {
+    if (need <= b.cap) return 0;
+    DevBuf nb;
+    if (nb.grow(std::max(need, 2 * b.cap))) return fail(SEPO_E_NOMEM, "sharded job buffer");
+    if (have) CK(t, cudaMemcpyAsync(nb.p, b.p, have, cudaMemcpyDeviceToDevice, s));
+    CK(t, cudaStreamSynchronize(s));
+    b.release();
+    b = nb;
+    return 0;
+}
+}  // namespace
+#endif
+
+int64_t sepo_run_sharded(sepo_table* t, const uint8_t* keys, const uint64_t* ko, const uint8_t* vals,
+                         const uint64_t* vo, uint64_t n) {
+    trace("run_sharded begin", n);
+    int rc = check_active(t);
+    if (rc) return rc;
+#if SEPO_WITH_NCCL
+    if (!t->nccl) return fail(SEPO_E_STATE, "no communicator (sepo_attach_nccl)");
+    if (t->opts.mode != SEPO_COMBINE_SUM_U64) return fail(SEPO_E_INVAL, "sepo_run_sharded needs COMBINE mode");
+    if (t->opts.fail_alloc_ppm && t->opts.fail_mode == 1) return fail(SEPO_E_INVAL, "record-mode fault injection");
+    if (vo) return fail(SEPO_E_INVAL, "sharded batches take fixed-width values");
+    if (t->sh_n) return fail(SEPO_E_STATE, "records held by sepo_insert_batch_sharded (sepo_drain first)");
+    const uint32_t kw = t->opts.fixed_key_width, vw = vals ? t->opts.fixed_val_width : 0u;
+    if (n && (!keys || (!ko && kw == 0))) return fail(SEPO_E_INVAL, "keys / key_offsets");
+    if (n && !(is_device_ptr(keys) && is_device_ptr(ko) && is_device_ptr(vals))) return fail(SEPO_E_INVAL, "device inputs only");
+    if (vals && !(vw == 1 || vw == 2 || vw == 4 || vw == 8)) return fail(SEPO_E_INVAL, "fixed_val_width must be 1, 2, 4 or 8");
+    const uint32_t P = (uint32_t)t->nranks;
+    ncclComm_t comm = (ncclComm_t)t->nccl;
+    cudaStream_t s = t->stream;
+    if (!t->route_stream) CK(t, cudaStreamCreateWithFlags(&t->route_stream, cudaStreamNonBlocking));
+    cudaStream_t rs = t->route_stream;
+    // (the caller's inputs may have been written on t->stream or on the legacy default stream)
+    CK(t, cudaStreamSynchronize(s));
+    CK(t, cudaStreamSynchronize(cudaStreamLegacy));
+    if (t->sh_cnt.grow(8 * (6 * (size_t)P + 64))) return fail(SEPO_E_NOMEM, "count scratch");
+    uint64_t* dsend = (uint64_t*)t->sh_cnt.p;  // [P][3] records, key bytes, value bytes per destination
+    uint64_t* drecv = dsend + 3 * P;            // [P][3] from each source
+    uint64_t* dseg = drecv + 3 * P;             // [2P] segment starts / byte bases of a received chunk
+    uint64_t* dagree = dseg + 2 * P;            // [2] longest key, chunks
+    // ---- agree on the format and the number of chunks: one all-reduce (max)
+    uint64_t per = 64ull << 20;
+    if (const char* e = getenv("SEPO_SHARD_CHUNK")) per = strtoull(e, nullptr, 10);
+    per = std::max<uint64_t>(2048, per / 2048 * 2048);
+    // CSR keys travel as CSR (word tiles combine too little to pay for 32-byte wire records: C2 at
+    // N = 1, 146 ms per job as wire records vs 82 ms as CSR); SEPO_SHARD_WIRE=1 sends CSR batches whose
+    // keys are all <= 16 bytes as wire records
+    const char* ew = getenv("SEPO_SHARD_WIRE");
+    const bool wire_csr = ew && ew[0] == '1';
+    uint64_t agree[2] = {ko ? 0ull : (uint64_t)kw, (n + per - 1) / per};
+    if (ko && !wire_csr) agree[0] = 1ull << 20;  // (never wire)
+    if (ko && wire_csr) {
+        rc = sepo_launch_max_key_len(ko, n, (unsigned long long*)dagree, rs);
+        if (rc) return cuda_check(t, (cudaError_t)rc, "max key length");
+        t->st.kernel_launches += 1;
+    } else {
+        CK(t, cudaMemcpyAsync(dagree, &agree[0], 8, cudaMemcpyHostToDevice, rs));
+    }
+    CK(t, cudaMemcpyAsync(dagree + 1, &agree[1], 8, cudaMemcpyHostToDevice, rs));
+    CK(t, cudaStreamSynchronize(rs));  // (agree is pageable host memory)
+    NK(t, ncclAllReduce(dagree, dagree, 2, ncclUint64, ncclMax, comm, rs));
+    CK(t, cudaMemcpyAsync(agree, dagree, 16, cudaMemcpyDeviceToHost, rs));
+    CK(t, cudaStreamSynchronize(rs));
+    const bool wire = agree[0] <= 16;
+    const uint64_t nch = agree[1];
+    const bool csr_keys = !wire && (ko != nullptr || kw == 0);  // received keys carry offsets
+    // ---- job state (as run_device): prepared re-issue records sized for what was received
+    Batch cur{};
+    cur.kw = wire ? 0u : kw;
+    cur.vw = wire ? 8u : vw;
+    // (fixed-width keys of at most 8 bytes, routed as wire records or not: 32-byte prepared records)
+    const bool short_keys = !csr_keys && kw > 0 && kw <= 8;
+    const bool has_vals = wire || vals != nullptr;
+    const uint64_t prb = (has_vals && !short_keys) ? sizeof(PRec) : 32;
+    cur.prep_rb = (uint32_t)prb;
+    cur.prep_fmt = (has_vals && short_keys) ? 33u : 0u;
+    const uint64_t slack = (uint64_t)t->grid * 32 * kPrepChunk;
+    if (t->prep_n.grow(64)) return fail(SEPO_E_NOMEM, "prepared list counter");
+    {   // the prepared list, sized once for about as many records as this rank sends (hash routing
+        // balances the parts), bounded by half the free memory; it grows (one copy) if a rank receives more
+        size_t fr = 0, tot = 0;
+        uint64_t want = n + slack * std::max<uint64_t>(nch, 1);
+        if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) want = std::min<uint64_t>(want, (fr + t->prep[0].cap) / 2 / prb);
+        if ((uint64_t)t->prep[0].cap < want * prb) {
+            t->prep[0].release();
+            if (t->prep[0].grow(want * prb)) return fail(SEPO_E_NOMEM, "prepared re-issue list");
+        }
+    }
+    if (!wire && n) {  // CSR: room for about as many records / bytes as this rank sends (grown if needed)
+        uint64_t kb = n * (uint64_t)kw;
+        if (ko) {
+            CK(t, cudaMemcpyAsync(&t->h_ko[4], ko, 8, cudaMemcpyDeviceToHost, rs));
+            CK(t, cudaMemcpyAsync(&t->h_ko[5], ko + n, 8, cudaMemcpyDeviceToHost, rs));
+            CK(t, cudaStreamSynchronize(rs));
+            kb = t->h_ko[5] - t->h_ko[4];
+        }
+        const uint64_t m = n + n / 16;
+        if (t->sh_held[0].grow(kb + kb / 16 + 16) || (csr_keys && t->sh_held[1].grow((m + 1) * 8)) ||
+            (vals && t->sh_held[2].grow(m * (uint64_t)vw + 16)))
+            return fail(SEPO_E_NOMEM, "sharded job: records held");
+    }
+    CK(t, cudaMemsetAsync(t->prep_n.p, 0, 16, s));
+    int64_t passes_start = (int64_t)t->st.passes;
+    std::vector<cudaEvent_t> evs(std::max<uint64_t>(nch, 1));
+    for (auto& e : evs) cudaEventCreateWithFlags(&e, cudaEventDisableTiming);
+    struct Guard {
+        std::vector<cudaEvent_t>& e;
+        ~Guard() { for (auto& x : e) cudaEventDestroy(x); }
+    } guard{evs};
+    // records / key bytes / value bytes held (CSR) and the previous chunk's insert
+    uint64_t hn = 0, hkb = 0, hvb = 0;
+    uint64_t post = 0, kept_kb = 0, reserved = 0;
+    bool prev_live = false;
+    Batch prev{};
+    InsertLaunch prevL;
+    auto finish_prev = [&]() -> int {
+        if (!prev_live) return 0;
+        prev_live = false;
+        const int64_t c = insert_end(t, prev, prevL);
+        if (c < 0) return (int)c;
+        post += (uint64_t)c;
+        kept_kb += t->h_ctrl->kept_key_bytes;
+        CK(t, cudaMemcpyAsync(&t->h_ko[0], t->prep_n.p, 8, cudaMemcpyDeviceToHost, s));
+        CK(t, cudaStreamSynchronize(s));
+        reserved = t->h_ko[0];
+        return 0;
+    };
+    const uint64_t scr_bytes = wire ? sepo_route_scratch(P) : sepo_partition_scratch(std::min(n, per), P);
+    if (t->sh_tmp[2].grow(scr_bytes)) return fail(SEPO_E_NOMEM, "route scratch");
+    for (uint64_t c = 0; c < nch; ++c) {
+        const uint64_t r0 = std::min(n, c * per), r1 = std::min(n, r0 + per), cn = r1 - r0;
+        std::vector<uint64_t> send(3 * P, 0), recv(3 * P, 0), pc(P + 1, 0);
+        // ---- route chunk c (route stream; the router syncs it)
+        if (cn && wire) {
+            if (t->sh_send[0].grow(cn * sizeof(WireRec))) return fail(SEPO_E_NOMEM, "wire send buffer");
+            const int64_t m = sepo_route_combine(keys + (ko ? 0 : r0 * (uint64_t)kw), ko ? ko + r0 : nullptr, kw,
+                                                 vals ? vals + r0 * (uint64_t)vw : nullptr, vw, cn, P, kRouteSeed,
+                                                 t->sh_send[0].p, cn, pc.data(), t->sh_tmp[2].p, scr_bytes, rs);
+            if (m < 0) return m;
+            for (uint32_t p = 0; p < P; ++p) send[3 * p] = pc[p + 1] - pc[p];
+            t->st.kernel_launches += 2;
+        } else if (cn) {
+            uint64_t kb0 = r0 * (uint64_t)kw, kb1 = r1 * (uint64_t)kw;
+            if (ko) {
+                CK(t, cudaMemcpyAsync(&t->h_ko[4], ko + r0, 8, cudaMemcpyDeviceToHost, rs));
+                CK(t, cudaMemcpyAsync(&t->h_ko[5], ko + r1, 8, cudaMemcpyDeviceToHost, rs));
+                CK(t, cudaStreamSynchronize(rs));
+                kb0 = t->h_ko[4];
+                kb1 = t->h_ko[5];
+            }
+            if (t->sh_send[0].grow(kb1 - kb0 + 16) || (csr_keys && t->sh_send[1].grow((cn + 1) * 8)) ||
+                (vals && t->sh_send[2].grow(cn * (uint64_t)vw + 16)))
+                return fail(SEPO_E_NOMEM, "partition buffers");
+            std::vector<uint64_t> st(3 * (P + 1));
+            rc = sepo_partition(ko ? keys : keys + kb0, ko ? ko + r0 : nullptr, kw, vals ? vals + r0 * (uint64_t)vw : nullptr,
+                                vw, cn, P, kRouteSeed, (uint8_t*)t->sh_send[0].p, csr_keys ? (uint64_t*)t->sh_send[1].p : nullptr,
+                                vals ? (uint8_t*)t->sh_send[2].p : nullptr, st.data(), t->sh_tmp[2].p, scr_bytes, rs);
+            if (rc) return rc;
+            for (uint32_t p = 0; p < P; ++p)
+                for (int x = 0; x < 3; ++x) send[3 * p + x] = st[3 * (p + 1) + x] - st[3 * p + x];
+            t->st.kernel_launches += 3;
+        }
+        // ---- counts
+        CK(t, cudaMemcpyAsync(dsend, send.data(), 8 * 3 * P, cudaMemcpyHostToDevice, rs));
+        NK(t, ncclGroupStart());
+        for (uint32_t p = 0; p < P; ++p) {
+            NK(t, ncclSend(dsend + 3 * p, 3, ncclUint64, (int)p, comm, rs));
+            NK(t, ncclRecv(drecv + 3 * p, 3, ncclUint64, (int)p, comm, rs));
+        }
+        NK(t, ncclGroupEnd());
+        CK(t, cudaMemcpyAsync(recv.data(), drecv, 8 * 3 * P, cudaMemcpyDeviceToHost, rs));
+        CK(t, cudaStreamSynchronize(rs));
+        uint64_t rn = 0, rk = 0, rv = 0;
+        for (uint32_t p = 0; p < P; ++p) { rn += recv[3 * p]; rk += recv[3 * p + 1]; rv += recv[3 * p + 2]; }
+        // ---- receive space (wire: slot c & 1, last read by chunk c-2's insert, finished already;
+        // CSR: appended to the records held — growing them waits for the running insert)
+        if (wire) {
+            if (t->sh_recv[c & 1].grow(std::max<uint64_t>(rn, 1) * sizeof(WireRec))) return fail(SEPO_E_NOMEM, "wire receive buffer");
+        } else {
+            const bool fit = hkb + rk + 16 <= t->sh_held[0].cap && (!csr_keys || (hn + rn + 1) * 8 <= t->sh_held[1].cap) &&
+                             (!vals || hvb + rv + 16 <= t->sh_held[2].cap);
+            if (!fit) {
+                CK(t, cudaStreamSynchronize(s));
+                if ((rc = grow_keep(t, t->sh_held[0], hkb, hkb + rk + 16, rs))) return rc;
+                if (csr_keys && (rc = grow_keep(t, t->sh_held[1], hn * 8, (hn + rn + 1) * 8, rs))) return rc;
+                if (vals && (rc = grow_keep(t, t->sh_held[2], hvb, hvb + rv + 16, rs))) return rc;
+            }
+        }
+        // ---- payload (one NCCL group), then rebase the received offsets onto the bytes held
+        NK(t, ncclGroupStart());
+        uint64_t so = 0, ro = 0, sko = 0, rko = 0, svo = 0, rvo = 0;
+        for (uint32_t p = 0; p < P; ++p) {
+            if (wire) {
+                const uint64_t sb = send[3 * p] * sizeof(WireRec), rbb = recv[3 * p] * sizeof(WireRec);
+                if (sb) NK(t, ncclSend((uint8_t*)t->sh_send[0].p + pc[p] * sizeof(WireRec), sb, ncclUint8, (int)p, comm, rs));
+                if (rbb) NK(t, ncclRecv((uint8_t*)t->sh_recv[c & 1].p + ro, rbb, ncclUint8, (int)p, comm, rs));
+                ro += rbb;
+                continue;
+            }
+            uint8_t* hk = (uint8_t*)t->sh_held[0].p + hkb;
+            uint64_t* hko = (uint64_t*)t->sh_held[1].p + hn;
+            uint8_t* hv = (uint8_t*)t->sh_held[2].p + hvb;
+            if (send[3 * p + 1]) NK(t, ncclSend((uint8_t*)t->sh_send[0].p + so, send[3 * p + 1], ncclUint8, (int)p, comm, rs));
+            if (recv[3 * p + 1]) NK(t, ncclRecv(hk + ro, recv[3 * p + 1], ncclUint8, (int)p, comm, rs));
+            if (csr_keys && send[3 * p]) NK(t, ncclSend((uint64_t*)t->sh_send[1].p + sko, send[3 * p], ncclUint64, (int)p, comm, rs));
+            if (csr_keys && recv[3 * p]) NK(t, ncclRecv(hko + rko, recv[3 * p], ncclUint64, (int)p, comm, rs));
+            if (vals && send[3 * p + 2]) NK(t, ncclSend((uint8_t*)t->sh_send[2].p + svo, send[3 * p + 2], ncclUint8, (int)p, comm, rs));
+            if (vals && recv[3 * p + 2]) NK(t, ncclRecv(hv + rvo, recv[3 * p + 2], ncclUint8, (int)p, comm, rs));
+            so += send[3 * p + 1]; ro += recv[3 * p + 1]; sko += send[3 * p]; rko += recv[3 * p];
+            svo += send[3 * p + 2]; rvo += recv[3 * p + 2];
+        }
+        NK(t, ncclGroupEnd());
+        if (!wire && csr_keys && rn) {
+            std::vector<uint64_t> seg(2 * P);
+            uint64_t r = 0, kb = 0;
+            for (uint32_t p = 0; p < P; ++p) { seg[p] = r; seg[P + p] = hkb + kb; r += recv[3 * p]; kb += recv[3 * p + 1]; }
+            CK(t, cudaMemcpyAsync(dseg, seg.data(), 16 * P, cudaMemcpyHostToDevice, rs));
+            rc = sepo_launch_shift_offsets((uint64_t*)t->sh_held[1].p + hn, rn, dseg, dseg + P, P, hkb + rk, rs);
+            if (rc) return cuda_check(t, (cudaError_t)rc, "shift offsets");
+            t->st.kernel_launches += 1;
+            CK(t, cudaStreamSynchronize(rs));  // (seg is pageable host memory read by the copy above)
+        }
+        CK(t, cudaEventRecord(evs[c], rs));
+        // ---- the previous chunk's counters, room in the prepared list, then this chunk's insert
+        if ((rc = finish_prev())) return rc;
+        if (rn) {
+            const uint64_t need = (reserved + rn + slack) * prb;
+            if ((uint64_t)t->prep[0].cap < need && (rc = grow_keep(t, t->prep[0], reserved * prb, need + need / 2, s))) return rc;
+            if (t->bm.grow(((rn + 31) / 32) * 4)) return fail(SEPO_E_NOMEM, "bitmap scratch");
+            CK(t, cudaStreamWaitEvent(s, evs[c], 0));
+            Batch bc = cur;
+            if (wire) {
+                bc.wire = (const WireRec*)t->sh_recv[c & 1].p;
+                bc.vals = (const uint8_t*)bc.wire;
+            } else {
+                bc.keys = (const uint8_t*)t->sh_held[0].p + (csr_keys ? 0 : hkb);
+                bc.ko = csr_keys ? (const uint64_t*)t->sh_held[1].p + hn : nullptr;
+                bc.vals = vals ? (const uint8_t*)t->sh_held[2].p + hvb : nullptr;
+            }
+            bc.n = rn;
+            bc.bitmap = (uint32_t*)t->bm.p;
+            bc.out = (PRec*)t->prep[0].p;
+            bc.out_n = (unsigned long long*)t->prep_n.p;
+            bc.out_cap = t->prep[0].cap / prb;
+            rc = insert_begin(t, bc, csr_keys ? hkb : 0, csr_keys ? hkb + rk : 0, prevL);
+            if (rc) return rc;
+            prev = bc;
+            prev_live = true;
+        }
+        if (!wire) { hn += rn; hkb += rk; hvb += rv; }
+    }
+    if ((rc = finish_prev())) return rc;
+    if (reserved > t->prep[0].cap / prb) return fail(SEPO_E_STATE, "prepared re-issue list overflow (sharded job)");
+    trace("run_sharded pass 1 end", post);
+    if (post) {
+        cur.keys = wire ? nullptr : (const uint8_t*)t->sh_held[0].p;
+        const int64_t r = prep_passes(t, cur, 0, reserved, post, kept_kb, prb, passes_start);
+        if (r < 0) return r;
+    }
+    if (t->dirty) {
+        int64_t e = evict_impl(t, 0);
+        if (e < 0) return e;
+    }
+    CK(t, cudaStreamSynchronize(t->copy_stream));
+    trace("run_sharded end", t->st.passes - passes_start);
+    return (int64_t)t->st.passes - passes_start;
+#else
+    (void)keys; (void)ko; (void)vals; (void)vo; (void)n;
+    return fail(SEPO_E_NCCL, "built without NCCL");
+#endif
 }

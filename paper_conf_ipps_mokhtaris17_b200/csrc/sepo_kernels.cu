@@ -2241,6 +2241,16 @@ __global__ void shift_offsets_kernel(uint64_t* ko, uint64_t n, const uint64_t* s
     if (blockIdx.x == 0 && threadIdx.x == 0) ko[n] = total;
 }
 
+// longest key of a CSR batch (the pipelined sharded job picks wire records when every rank's keys
+// are at most 16 bytes): warp max, one atomicMax per warp
+__global__ void __launch_bounds__(256) max_key_len_kernel(const uint64_t* ko, uint64_t n, unsigned long long* out) {
+    unsigned long long m = 0;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        m = max(m, (unsigned long long)(ld_in64(ko + i + 1) - ld_in64(ko + i)));
+    m = __reduce_max_sync(FULLMASK, (unsigned)min(m, 0xffffffffull));
+    if (lane_id() == 0 && m) atomicMax(out, m);
+}
+
 // ---- router with CTA pre-combine (COMBINE mode, keys of at most 16 bytes)
 // Records of one rank go to their owners as 32-byte WireRecs {key words, value, length} after the
 // CTA has combined equal keys of its tile in shared memory (a hot Zipf key leaves a tile once, with
@@ -3349,9 +3359,14 @@ int sepo_launch_insert(const Dev& d, const Batch& b, int mode, int grid, cudaStr
                 if (!attr_w) {
                     cudaFuncSetAttribute(insert_lean_kernel<true, IN_WIRE, 48>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          (int)sizeof(lean::Smem<true>));
+                    cudaFuncSetAttribute(insert_lean_kernel<true, IN_WIRE, 33>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)sizeof(lean::Smem<true>));
                     attr_w = true;
                 }
-                insert_lean_kernel<true, IN_WIRE, 48><<<G, B, sizeof(lean::Smem<true>), s>>>(d, b, hl, nh, c);
+                // (33: every key of the batch is at most 8 bytes — routed fixed-width keys — so a
+                // declined record fits a 32-byte prepared record {key, value, hash, length})
+                if (b.prep_fmt == 33) insert_lean_kernel<true, IN_WIRE, 33><<<G, B, sizeof(lean::Smem<true>), s>>>(d, b, hl, nh, c);
+                else insert_lean_kernel<true, IN_WIRE, 48><<<G, B, sizeof(lean::Smem<true>), s>>>(d, b, hl, nh, c);
             } else if (!b.vals) {
                 if (in == IN_CSR) insert_lean_kernel<false, IN_CSR, 32><<<G, B, sml, s>>>(d, b, hl, nh, c);
                 else insert_lean_kernel<false, IN_FIXED, 32><<<G, B, sml, s>>>(d, b, hl, nh, c);
@@ -3524,6 +3539,11 @@ int sepo_launch_route_combine(const Batch& b, uint32_t P, uint64_t seed, int pas
     }
     if (b.n) route_combine_kernel<<<grid, rc::THREADS, sizeof(rc::Smem), s>>>(b, P, seed, pass, part_totals, long_keys,
                                                                               part_base, cursors, out);
+    return cudaGetLastError();
+}
+int sepo_launch_max_key_len(const uint64_t* ko, uint64_t n, unsigned long long* out, cudaStream_t s) {
+    cudaMemsetAsync(out, 0, 8, s);
+    if (n) max_key_len_kernel<<<(unsigned)std::min<uint64_t>((n + 255) / 256, 4 * 148), 256, 0, s>>>(ko, n, out);
     return cudaGetLastError();
 }
 int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const uint64_t* seg_base, uint32_t n_segs,

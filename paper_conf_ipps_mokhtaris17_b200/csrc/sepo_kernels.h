@@ -89,6 +89,7 @@ uint64_t sepo_partition_tiles(uint64_t n);
 uint64_t sepo_map_chunks(uint64_t n);
 int sepo_launch_map(const uint8_t* text, uint64_t n, int lines, int pass, unsigned long long* tc, const uint64_t* doc_offsets,
                     uint64_t n_docs, uint8_t* okeys, uint64_t* oko, uint32_t* odoc, cudaStream_t s);
+int sepo_launch_max_key_len(const uint64_t* ko, uint64_t n, unsigned long long* out, cudaStream_t s);
 int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec, const uint64_t* seg_base, uint32_t n_segs,
                               uint64_t total, cudaStream_t s);
 int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);

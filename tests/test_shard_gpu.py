@@ -213,3 +213,73 @@ def test_nccl_sharded_one_rank(cuda, name, ratio):
     t.close()
     assert passes >= 1
     assert got == exp
+
+
+# ---- the pipelined sharded job (sepo_run_sharded): chunk c+1 routed / exchanged beside chunk c's insert
+@pytest.mark.parametrize("name,ratio,chunk", [("C2", 4, 1 << 17), ("C5z", 4, 1 << 16), ("C5u", 2, 1 << 16),
+                                              ("C3", 2, 1 << 15), ("C1", 1, 10_000)])
+def test_nccl_run_sharded_one_rank(cuda, monkeypatch, name, ratio, chunk):
+    """sepo_run_sharded over a one-rank NCCL communicator, many chunks (SEPO_SHARD_CHUNK), the table
+    `ratio` times its budget so chunks decline records into the prepared list: the export equals the
+    oracle (wire records for words / pairs, a CSR partition for URLs — whose held buffers grow)"""
+    monkeypatch.setenv("SEPO_SHARD_CHUNK", str(chunk))
+    scale = {"C1": 0.25, "C2": 1 / 512, "C5z": 2 ** -12, "C5u": 2 ** -12, "C3": 1 / 2000}[name]
+    s = gen.config(name, scale=scale)
+    exp = oracle_expected(s)
+    k, o, v = s.device()
+    fixed = s.family == gen.GEN_PAIRS
+    kw = dict(fixed_key_width=8, fixed_val_width=8) if fixed else {}
+    pb = 65536 if name == "C3" else 16384
+    t = sepo().Table(sepo().budget_for(1 << 16, pb, 1 << 14), 1 << 16, pb, **kw)
+    if fixed:
+        t.run(k, None, v)
+    else:
+        t.run(k, o)
+    need = t.stats()["pages_used_max"]
+    t.close()
+    t = sepo().Table(sepo().budget_for(1 << 16, pb, max(8, need // (2 * ratio if name == "C3" else ratio))), 1 << 16, pb,
+                     check_dups=True, **kw)
+    t.attach_nccl(sepo().nccl_unique_id(), 1, 0)
+    passes = t.run_sharded(k, None, v) if fixed else t.run_sharded(k, o)
+    st = t.stats()
+    got = sepo().result_dict(t.export())
+    t.close()
+    assert got == exp
+    assert st["cross_gen_dups"] == 0
+    if ratio > 1:
+        assert passes >= 2
+    assert st["records_inserted"] >= s.n if name in ("C3", "C1") else True
+
+
+def test_nccl_run_sharded_wire_words(cuda, monkeypatch):
+    """SEPO_SHARD_WIRE=1: a CSR batch of words (all <= 16 bytes) goes as pre-combined wire records"""
+    monkeypatch.setenv("SEPO_SHARD_CHUNK", str(1 << 16))
+    monkeypatch.setenv("SEPO_SHARD_WIRE", "1")
+    s = gen.config("C2", scale=1 / 1024)
+    exp = oracle_expected(s)
+    k, o, _ = s.device()
+    t = sepo().Table(sepo().budget_for(1 << 16, 16384, 96), 1 << 16, 16384, check_dups=True)
+    t.attach_nccl(sepo().nccl_unique_id(), 1, 0)
+    assert t.run_sharded(k, o) >= 1
+    assert sepo().result_dict(t.export()) == exp
+    t.close()
+
+
+def test_nccl_run_sharded_hot_and_empty(cuda, monkeypatch):
+    """chunks large enough for the hot set (>= 2^21 records), a trailing short chunk, and a second job
+    with an empty batch on the same communicator (the rank still takes part in the agreement)"""
+    monkeypatch.setenv("SEPO_SHARD_CHUNK", str(3 << 20))
+    s = gen.config("C2", scale=1 / 200)
+    exp = oracle_expected(s)
+    k, o, _ = s.device()
+    t = sepo().Table(sepo().budget_for(1 << 20, 65536, 4096), 1 << 20, 65536, check_dups=True)
+    t.attach_nccl(sepo().nccl_unique_id(), 1, 0)
+    assert t.run_sharded(k, o) >= 1
+    st = t.stats()
+    got = sepo().result_dict(t.export())
+    assert got == exp
+    assert st["hot_keys"] > 0
+    t.reset()
+    assert t.run_sharded(None, None, n=0) >= 0
+    assert sepo().result_dict(t.export()) == {}
+    t.close()
