@@ -127,9 +127,11 @@ class Job:
     def table_params(self):
         pages_F, F = self.footprint()
         if self.ratio <= 1.0:
-            # in-budget tables: twice as many buckets as keys (load ~0.5: shorter chains for the misses
-            # that go to HBM; C2 0.5x pass 1 28.5 -> 25.8 ms). SEPO_BENCH_NB_IB overrides the multiple.
-            nb = self.nb_full * int(os.environ.get("SEPO_BENCH_NB_IB", "2"))
+            # in-budget tables: four times as many buckets as keys (load ~0.25: shorter chains for the
+            # misses that go to HBM — head insertion leaves a Zipf key's old entry behind the later ones;
+            # C2 0.5x pass 1: load 1 28.5, 0.5 25.8 -> 22.7, 0.25 21.9, 0.125 21.6 ms,
+            # profiles/r02/ab_directory_ib.jsonl, ab_nb_r3.jsonl). SEPO_BENCH_NB_IB overrides the multiple.
+            nb = self.nb_full * int(os.environ.get("SEPO_BENCH_NB_IB", "4"))
             pages = int(np.ceil(pages_F / self.ratio)) if self.ratio < 1 else pages_F + 8
         else:  # directory: the largest power of two <= 2x the keys of one generation (load <= ~1)
             mult = float(os.environ.get("SEPO_BENCH_NB_MULT", "2"))
@@ -482,7 +484,7 @@ def run_ours(args):
             tib.reset(); tib.run(k, o, v)
         msi, ii = timed_steps(jib, tib, args.steps, stream)
         tr = traffic_of("r02_traffic_m1.json")
-        m1 = roofline_of(csr, ii["p1_ms"], args.steps, pk, "sepo::insert_stream_kernel<false,1024,IN_CSR> (C2, 0.5x: in budget, 1 pass)",
+        m1 = roofline_of(csr, ii["p1_ms"], args.steps, pk, "sepo::insert_lean_kernel<false,IN_CSR,32> (C2, 0.5x: in budget, 1 pass)",
                          {"traffic": (tr["dram_read_bytes"] + tr["dram_write_bytes"]) if tr else None,
                           "traffic_note": tr.get("launch") if tr else None, "share_of_step": ii["p1_ms"] / msi,
                           "job_ms": msi / args.steps, "passes": ii["last"]["passes"]})
@@ -618,10 +620,9 @@ def run_routed(args, world, rank, local):
     lib_plane = args.plane == "lib"
     router = shard.Router(route_seed=0x5eed, fixed_key_width=8 if fixed else 0,
                           fixed_val_width=job.stream.val_width if sv is not None else 0,
-                          # pre-combine for fixed-width pairs (C5: SURVEY §8(e) makes it mandatory for
-                          # Zipf load balance); words go as CSR (their tiles combine too little to pay
-                          # for 32-byte wire records: C2 N=1 route 91 ms CSR vs 142 ms combined)
-                          combine=job.stream.family == 2 and not args.no_combine)
+                          # hot-key pre-combine + 32-byte wire records for keys <= 16 B (SURVEY §8(e) makes
+                          # it mandatory for Zipf load balance); longer keys (URLs) go as a CSR partition
+                          combine=not args.no_combine)
     routed = {}
 
     def attach(t):  # the library's own NCCL communicator (rank 0 makes the id, torch.distributed carries it)

@@ -106,6 +106,8 @@ typedef struct sepo_stats {
     double t_insert_ms, t_reprobe_ms, t_compact_ms, t_evict_ms, t_export_ms, t_h2d_ms;
     double t_insert_ms_per_pass[SEPO_MAX_PASS_STATS]; /* insert-kernel time of each pass */
     uint64_t hot_keys;             /* most keys a sampled hot set held in one insert call (a2; 0: none) */
+    uint64_t p2p_chunks;           /* sepo_run_sharded: chunks routed straight into the owners' windows
+                                      over peer memory (0: NCCL send/recv) */
 } sepo_stats;
 
 /* Create a table on the current CUDA device.
@@ -259,9 +261,11 @@ int sepo_partition(const uint8_t* keys, const uint64_t* key_offsets, uint32_t fi
 int sepo_shift_offsets(uint64_t* key_offsets, uint64_t n, const uint64_t* seg_rec_start, const uint64_t* seg_byte_base,
                        uint32_t n_segs, uint64_t total_bytes, void* stream);
 /* Router with pre-combine (COMBINE mode; "CTA-level pre-combine of duplicate keys
- * into (key, partial sum)"). Partitions n records by owner like sepo_partition, but each CTA first
- * combines the equal keys of its tile of records in shared memory (u64 wrapping sum of the values,
- * implicit 1 when vals == NULL), and every output record is a 32-byte wire record
+ * into (key, partial sum)"). Partitions n records by owner like sepo_partition, but the keys of the
+ * batch's sampled hot set (batches of >= 2^21 records; the insert kernels' discovery on the route hash)
+ * are combined over the whole batch first — each leaves as ONE record carrying its sum (u64 wrapping sum
+ * of the values, implicit 1 when vals == NULL); every other record leaves as its own record.
+ * Every output record is a 32-byte wire record
  *     struct { uint64_t w0, w1;  // key bytes 0..15, little endian, zero padded
  *              uint64_t value;   // the combined value
  *              uint64_t len; }   // key length (0..16)
@@ -270,7 +274,8 @@ int sepo_shift_offsets(uint64_t* key_offsets, uint64_t n, const uint64_t* seg_re
  * out_wire (device, caller-owned, out_cap records) receives part p's records at [part_counts[p],
  * part_counts[p + 1]); part_counts (HOST, n_parts + 1) is the exclusive prefix of the per-part counts
  * with the total last. out_wire == NULL is a sizing call (counts only). The order of records within a
- * part is unspecified. scratch: device, sepo_route_scratch(n_parts) bytes. Synchronizes the stream.
+ * part is unspecified. scratch: device, sepo_route_scratch(n_parts) bytes (for the current device).
+ * Synchronizes the stream.
  * Returns the number of wire records, or < 0 (SEPO_E_NOMEM: out_cap too small; part_counts valid). */
 size_t sepo_route_scratch(uint32_t n_parts);
 int64_t sepo_route_combine(const uint8_t* keys, const uint64_t* key_offsets, uint32_t fixed_key_width, const uint8_t* vals,
@@ -324,7 +329,7 @@ int64_t sepo_drain(sepo_table* t);
  *   owner, with the exchange pipelined against pass 1 (chunk c+1 is routed and exchanged
  *   on a second stream while chunk c is inserted). COMBINE mode only; device inputs as sepo_insert_batch
  *   (fixed-width values, val_offsets NULL; n may be 0 on some ranks). The ranks agree (one NCCL
- *   all-reduce) on the number of chunks (SEPO_SHARD_CHUNK records each, default 2^26, a multiple of
+ *   all-reduce) on the number of chunks (SEPO_SHARD_CHUNK records each, default 2^28, a multiple of
  *   2048) and on the format: pre-combined wire records when every rank's keys are <= 16 bytes, else a
  *   CSR partition. Records declined in pass 1 become prepared re-issue records; the re-issue passes,
  *   evictions and the final transfer to host run locally. Afterwards sepo_export gives this rank's

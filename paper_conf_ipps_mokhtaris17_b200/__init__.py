@@ -43,7 +43,8 @@ class Stats(ctypes.Structure):
                 ("key_bytes_inserted", u64), ("val_bytes_inserted", u64), ("kernel_launches", u64), ("value_chunks", u64), ("value_slots", u64), ("t_insert_ms", ctypes.c_double),
                 ("t_reprobe_ms", ctypes.c_double), ("t_compact_ms", ctypes.c_double), ("t_evict_ms", ctypes.c_double),
                 ("t_export_ms", ctypes.c_double), ("t_h2d_ms", ctypes.c_double),
-                ("t_insert_ms_per_pass", ctypes.c_double * MAXP), ("hot_keys", u64)]
+                ("t_insert_ms_per_pass", ctypes.c_double * MAXP), ("hot_keys", u64),
+                ("p2p_chunks", u64)]
 
     def as_dict(self):
         d = {k: getattr(self, k) for k, _ in self._fields_ if k not in ("postponed_per_pass", "t_insert_ms_per_pass")}

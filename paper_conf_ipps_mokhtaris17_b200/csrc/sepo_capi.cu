@@ -129,6 +129,11 @@ struct sepo_table {
     uint64_t sh_n = 0, sh_kb = 0, sh_vb = 0;          // records / key bytes / value bytes held
     cudaStream_t route_stream = nullptr;  // sepo_run_sharded: route + exchange of chunk c+1 beside chunk c's insert
     DevBuf sh_recv[2];                    // sepo_run_sharded: wire records received (ping-pong per chunk)
+    // sepo_run_sharded over peer memory: a symmetric NCCL window of 2 x win_cap wire records per rank
+    void* win_buf = nullptr;              // ncclMemAlloc
+    void* win = nullptr;                  // ncclWindow_t (device-side handle)
+    uint64_t win_cap = 0;                 // records per slot
+    bool win_failed = false;              // registration failed once: NCCL send/recv from then on
     bool lookup_done = false;
     std::vector<cudaEvent_t>* h2d_chunks = nullptr;  // sepo_run on host input: copy events of pass-1 chunks
     uint64_t h2d_chunk_records = 0;  // sepo_lookup restored old generations into the pool: no inserts until reset
@@ -523,7 +528,9 @@ static int insert_begin(sepo_table* t, const Batch& b, uint64_t key_begin, uint6
         // (measured: the lean path wins when the generation is L2-resident and the kernel is
         // issue-bound — C2 4x pass 1 21.2 -> 19.6 ms — and loses ~1.4 % when table accesses go to
         // HBM, where insert_stream_kernel's chunk-interleaved stream keeps fewer L1/L2 lines busy)
-        lean_in = (e && (e[0] == '0' || e[0] == '1')) ? e[0] == '1' : (mean <= 24 && !dir_prefetch(t));
+        // (in budget, CSR words: lean 21.5 vs stream 21.9 ms with the 4x directory; fixed-width pairs in
+        // HBM-resident tables keep the stream kernel: C5u 4x pass 1 147 vs 156 ms, profiles/r02/var_r5.jsonl)
+        lean_in = (e && (e[0] == '0' || e[0] == '1')) ? e[0] == '1' : (mean <= 24 && (b.ko || !dir_prefetch(t)));
         const char* el = getenv("SEPO_LONG");
         long_keys = b.ko && ((el && (el[0] == '0' || el[0] == '1')) ? el[0] == '1' : mean > 24);
     }
@@ -1673,6 +1680,9 @@ void sepo_destroy(sepo_table* t) {
     for (int i = 0; i < 3; ++i) { t->sh_send[i].release(); t->sh_held[i].release(); t->sh_tmp[i].release(); }
     t->sh_cnt.release();
 #if SEPO_WITH_NCCL
+    if (t->route_stream) cudaStreamSynchronize(t->route_stream);
+    if (t->nccl && t->win) ncclCommWindowDeregister((ncclComm_t)t->nccl, (ncclWindow_t)t->win);
+    if (t->win_buf) ncclMemFree(t->win_buf);
     if (t->nccl) ncclCommDestroy((ncclComm_t)t->nccl);
 #endif
     for (auto& s : t->buf)
@@ -1714,7 +1724,64 @@ int64_t sepo_run_wire(sepo_table* t, const void* wire, uint64_t n) {
     return run_device(t, nullptr, nullptr, nullptr, nullptr, n, reinterpret_cast<const WireRec*>(wire));
 }
 
-size_t sepo_route_scratch(uint32_t n_parts) { return 8 * (3 * (size_t)n_parts + 8); }
+static int cur_sms() {
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    return nsm;
+}
+size_t sepo_route_scratch(uint32_t n_parts) { return sepo_route_scratch_bytes(std::max<uint32_t>(n_parts, 1), cur_sms()); }
+
+namespace {
+// The router's two passes, split so sepo_run_sharded can place the parts itself (peer windows).
+// route_pass0: hot-set discovery + counts; hc = [P][G] non-hot records per (part, CTA), then per part
+// the hot keys it owns [32], (unused) [64], the long-key count. Synchronizes s.
+int route_pass0(const Batch& b, uint32_t P, uint64_t seed, void* scratch, int G, cudaStream_t s,
+                std::vector<unsigned long long>& hc) {
+    int rc = sepo_launch_route_hot(b, P, seed, 0, scratch, G, nullptr, s);
+    if (rc) return fail(SEPO_E_CUDA, std::string("route: ") + cudaGetErrorString((cudaError_t)rc));
+    size_t co = 0, ho = 0;
+    sepo_route_layout(P, G, &co, &ho);
+    hc.assign((size_t)P * G + 3 * 32 + 8, 0);
+    if (cudaMemcpyAsync(hc.data(), (uint8_t*)scratch + co, 8 * (size_t)P * G, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaMemcpyAsync(hc.data() + (size_t)P * G, (uint8_t*)scratch + ho, 8 * (3 * 32 + 8), cudaMemcpyDeviceToHost, s) != cudaSuccess ||
+        cudaStreamSynchronize(s) != cudaSuccess)
+        return fail(SEPO_E_CUDA, "route counts");
+    if (hc[(size_t)P * G + 3 * 32]) return fail(SEPO_E_TOOLARGE, "route combine: keys longer than 16 bytes (route them as CSR)");
+    return 0;
+}
+// records this rank sends to each part (non-hot + hot keys owned)
+void route_part_totals(const std::vector<unsigned long long>& hc, uint32_t P, int G, std::vector<uint64_t>& tot) {
+    tot.assign(P, 0);
+    for (uint32_t p = 0; p < P; ++p) {
+        for (int c = 0; c < G; ++c) tot[p] += hc[(size_t)p * G + c];
+        tot[p] += hc[(size_t)P * G + p];
+    }
+}
+// route_pass1: part p's records from record index start[p] of its destination (out, or dstp[p]):
+// CTA by CTA, then its hot keys. Enqueued on s (no sync).
+int route_pass1(const Batch& b, uint32_t P, uint64_t seed, void* scratch, int G, cudaStream_t s,
+                const std::vector<unsigned long long>& hc, const std::vector<uint64_t>& start, WireRec* out,
+                WireRec* const* dstp) {
+    std::vector<unsigned long long> hb((size_t)P * G + 32, 0);
+    for (uint32_t p = 0; p < P; ++p) {
+        uint64_t at = start[p];
+        for (int c = 0; c < G; ++c) { hb[(size_t)p * G + c] = at; at += hc[(size_t)p * G + c]; }
+        hb[(size_t)P * G + p] = at;  // hot base of part p
+    }
+    size_t co = 0, ho = 0;
+    sepo_route_layout(P, G, &co, &ho);
+    unsigned long long* bases = (unsigned long long*)((uint8_t*)scratch + co) + (size_t)P * G;
+    unsigned long long* hot_base = (unsigned long long*)((uint8_t*)scratch + ho) + 32;
+    // (hb is pageable host memory: these copies complete before cudaMemcpyAsync returns)
+    if (cudaMemcpyAsync(bases, hb.data(), 8 * (size_t)P * G, cudaMemcpyHostToDevice, s) != cudaSuccess ||
+        cudaMemcpyAsync(hot_base, hb.data() + (size_t)P * G, 8 * P, cudaMemcpyHostToDevice, s) != cudaSuccess)
+        return fail(SEPO_E_CUDA, "route bases");
+    int rc = sepo_launch_route_hot(b, P, seed, 1, scratch, G, out, s, dstp);
+    if (rc) return fail(SEPO_E_CUDA, std::string("route: ") + cudaGetErrorString((cudaError_t)rc));
+    return 0;
+}
+}  // namespace
 
 int64_t sepo_route_combine(const uint8_t* keys, const uint64_t* ko, uint32_t kw, const uint8_t* vals, uint32_t vw,
                            uint64_t n, uint32_t n_parts, uint64_t route_seed, void* out_wire, uint64_t out_cap,
@@ -1723,39 +1790,27 @@ int64_t sepo_route_combine(const uint8_t* keys, const uint64_t* ko, uint32_t kw,
     if (!ko && kw == 0) return fail(SEPO_E_INVAL, "key_offsets is NULL and fixed_key_width is 0");
     if (vals && !(vw == 1 || vw == 2 || vw == 4 || vw == 8)) return fail(SEPO_E_INVAL, "fixed_val_width must be 1, 2, 4 or 8");
     if (!part_counts || !scratch || scratch_bytes < sepo_route_scratch(n_parts)) return fail(SEPO_E_INVAL, "scratch / part_counts");
+    const uint32_t P = n_parts;
+    const int G = cur_sms();
     cudaStream_t s = (cudaStream_t)stream;
     Batch b{};
     b.keys = keys; b.ko = ko; b.kw = kw; b.vals = vals; b.vw = vw; b.n = n;
-    unsigned long long* totals = (unsigned long long*)scratch;
-    unsigned long long* cursors = totals + n_parts;
-    unsigned long long* base = cursors + n_parts;
-    unsigned long long* longk = base + n_parts;
-    int dev = 0, nsm = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    if (cudaMemsetAsync(scratch, 0, sepo_route_scratch(n_parts), s) != cudaSuccess) return fail(SEPO_E_CUDA, "memset");
-    // pass 0: output records per part (and keys longer than 16 bytes)
     // the same route hash as sepo_partition (seed decorrelated from a table seed of equal value)
     route_seed ^= 0x6a09e667f3bcc909ull;
-    int rc = sepo_launch_route_combine(b, n_parts, route_seed, 0, totals, longk, nullptr, nullptr, nullptr, nsm, s);
-    if (rc) return fail(SEPO_E_CUDA, std::string("route combine: ") + cudaGetErrorString((cudaError_t)rc));
-    std::vector<unsigned long long> h(n_parts + 1);
-    if (cudaMemcpyAsync(h.data(), totals, 8 * n_parts, cudaMemcpyDeviceToHost, s) != cudaSuccess ||
-        cudaMemcpyAsync(&h[n_parts], longk, 8, cudaMemcpyDeviceToHost, s) != cudaSuccess || cudaStreamSynchronize(s) != cudaSuccess)
-        return fail(SEPO_E_CUDA, "route combine counts");
-    if (h[n_parts]) return fail(SEPO_E_TOOLARGE, "route combine: keys longer than 16 bytes (route them as CSR)");
-    uint64_t tot = 0;
-    for (uint32_t p = 0; p < n_parts; ++p) { part_counts[p] = tot; tot += h[p]; }
-    part_counts[n_parts] = tot;
-    if (!out_wire) return (int64_t)tot;  // sizing call
-    if (out_cap < tot) return fail(SEPO_E_NOMEM, "route combine: out_cap < " + std::to_string(tot) + " records");
-    std::vector<unsigned long long> hb(part_counts, part_counts + n_parts);
-    if (cudaMemcpyAsync(base, hb.data(), 8 * n_parts, cudaMemcpyHostToDevice, s) != cudaSuccess)
-        return fail(SEPO_E_CUDA, "route combine bases");
-    rc = sepo_launch_route_combine(b, n_parts, route_seed, 1, totals, nullptr, base, cursors, (WireRec*)out_wire, nsm, s);
-    if (rc) return fail(SEPO_E_CUDA, std::string("route combine: ") + cudaGetErrorString((cudaError_t)rc));
-    if (cudaStreamSynchronize(s) != cudaSuccess) return fail(SEPO_E_CUDA, "route combine");
-    return (int64_t)tot;
+    std::vector<unsigned long long> hc;
+    int rc = route_pass0(b, P, route_seed, scratch, G, s, hc);
+    if (rc) return rc;
+    std::vector<uint64_t> tot, start(P, 0);
+    route_part_totals(hc, P, G, tot);
+    uint64_t all = 0;
+    for (uint32_t p = 0; p < P; ++p) { part_counts[p] = start[p] = all; all += tot[p]; }
+    part_counts[P] = all;
+    if (!out_wire) return (int64_t)all;  // sizing call
+    if (out_cap < all) return fail(SEPO_E_NOMEM, "route combine: out_cap < " + std::to_string(all) + " records");
+    rc = route_pass1(b, P, route_seed, scratch, G, s, hc, start, (WireRec*)out_wire, nullptr);
+    if (rc) return rc;
+    if (cudaStreamSynchronize(s) != cudaSuccess) return fail(SEPO_E_CUDA, "route");
+    return (int64_t)all;
 }
 
 size_t sepo_partition_scratch(uint64_t n, uint32_t n_parts) {
@@ -1856,7 +1911,13 @@ int64_t sepo_map_run(sepo_table* t, int mapper, const uint8_t* text, uint64_t n_
 // evict, re-issue until nothing is postponed). Postponed records are never re-routed: a key's
 // records all live on its owner, so every rank's export is final (no merge).
 #if SEPO_WITH_NCCL
+#include <nccl_device.h>
 namespace {
+// destination of part p in chunk slot `off` of the window: rank p's copy, through its LSA (NVLink) mapping
+__global__ void p2p_ptrs_kernel(ncclWindow_t w, size_t off, int P, sepo::WireRec** out) {
+    const int p = threadIdx.x;
+    if (p < P) out[p] = reinterpret_cast<sepo::WireRec*>(ncclGetPeerPointer(w, off, p));
+}
 const uint64_t kRouteSeed = 0x5eedull;  // owner hash seed (the library decorrelates it from table seeds)
 int nccl_check(sepo_table* t, ncclResult_t r, const char* what) {
     if (r == ncclSuccess) return 0;
@@ -1942,12 +2003,11 @@ int64_t sepo_insert_batch_sharded(sepo_table* t, const uint8_t* keys, const uint
         void* scr = nullptr;
         if (t->sh_tmp[2].grow(sepo_route_scratch(P))) return fail(SEPO_E_NOMEM, "route scratch");
         scr = t->sh_tmp[2].p;
-        m = sepo_route_combine(keys, ko, kw, vals, vw, n, P, kRouteSeed, nullptr, 0, pc.data(), scr, sepo_route_scratch(P), s);
+        // (one call: a batch leaves at most one wire record per record)
+        if (t->sh_send[0].grow((size_t)std::max<uint64_t>(n, 1) * sizeof(WireRec))) return fail(SEPO_E_NOMEM, "wire send buffer");
+        m = sepo_route_combine(keys, ko, kw, vals, vw, n, P, kRouteSeed, t->sh_send[0].p, n, pc.data(), scr,
+                               sepo_route_scratch(P), s);
         if (m >= 0) {
-            if (t->sh_send[0].grow((size_t)std::max<int64_t>(m, 1) * sizeof(WireRec))) return fail(SEPO_E_NOMEM, "wire send buffer");
-            m = sepo_route_combine(keys, ko, kw, vals, vw, n, P, kRouteSeed, t->sh_send[0].p, (uint64_t)m, pc.data(), scr,
-                                   sepo_route_scratch(P), s);
-            if (m < 0) return m;
             fmt = 1;
             for (uint32_t p = 0; p < P; ++p) send[3 * p] = pc[p + 1] - pc[p];
         } else if (m != SEPO_E_TOOLARGE) {
@@ -2094,11 +2154,41 @@ namespace {
 int grow_keep(sepo_table* t, DevBuf& b, size_t have, size_t need, cudaStream_t s) {
     if (need <= b.cap) return 0;
     DevBuf nb;
-    if (nb.grow(std::max(need, 2 * b.cap))) return fail(SEPO_E_NOMEM, "sharded job buffer");
+    if (nb.grow(std::max(need, b.cap + b.cap / 2))) return fail(SEPO_E_NOMEM, "sharded job buffer");
     if (have) CK(t, cudaMemcpyAsync(nb.p, b.p, have, cudaMemcpyDeviceToDevice, s));
     CK(t, cudaStreamSynchronize(s));
     b.release();
     b = nb;
+    return 0;
+}
+// The receive window of the peer-memory exchange: 2 slots of `need` (+25 %) wire records, symmetric
+// (ncclMemAlloc + ncclCommWindowRegister, COLLECTIVE — every rank calls this with the same `need`, which
+// comes from the all-gathered count matrix). Returns 0, or 1 if some rank could not register one (the
+// ranks agree through an all-reduce; the job then uses NCCL send/recv).
+int ensure_window(sepo_table* t, ncclComm_t comm, uint64_t need, uint64_t* dflag) {
+    if (need <= t->win_cap && t->win) return 0;
+    CK(t, cudaStreamSynchronize(t->stream));  // (an insert may still read the old window)
+    CK(t, cudaStreamSynchronize(t->route_stream));
+    if (t->win) ncclCommWindowDeregister(comm, (ncclWindow_t)t->win);
+    if (t->win_buf) ncclMemFree(t->win_buf);
+    t->win = nullptr; t->win_buf = nullptr; t->win_cap = 0;
+    const uint64_t cap = std::max<uint64_t>(need + need / 4, 1ull << 16);
+    const size_t bytes = ((2 * cap * sizeof(WireRec)) + (2u << 20) - 1) & ~(size_t)((2u << 20) - 1);
+    void* buf = nullptr;
+    ncclWindow_t w = nullptr;
+    uint64_t ok = ncclMemAlloc(&buf, bytes) == ncclSuccess && ncclCommWindowRegister(comm, buf, bytes, &w, NCCL_WIN_COLL_SYMMETRIC) == ncclSuccess;
+    CK(t, cudaMemcpyAsync(dflag, &ok, 8, cudaMemcpyHostToDevice, t->route_stream));
+    NK(t, ncclAllReduce(dflag, dflag, 1, ncclUint64, ncclMin, comm, t->route_stream));
+    CK(t, cudaMemcpyAsync(&ok, dflag, 8, cudaMemcpyDeviceToHost, t->route_stream));
+    CK(t, cudaStreamSynchronize(t->route_stream));
+    if (!ok) {
+        if (w) ncclCommWindowDeregister(comm, w);
+        if (buf) ncclMemFree(buf);
+        t->win_failed = true;
+        trace("run_sharded: peer window unavailable, NCCL send/recv");
+        return 1;
+    }
+    t->win = w; t->win_buf = buf; t->win_cap = cap;
     return 0;
 }
 }  // namespace
@@ -2127,20 +2217,23 @@ int64_t sepo_run_sharded(sepo_table* t, const uint8_t* keys, const uint64_t* ko,
     // (the caller's inputs may have been written on t->stream or on the legacy default stream)
     CK(t, cudaStreamSynchronize(s));
     CK(t, cudaStreamSynchronize(cudaStreamLegacy));
-    if (t->sh_cnt.grow(8 * (6 * (size_t)P + 64))) return fail(SEPO_E_NOMEM, "count scratch");
+    if (t->sh_cnt.grow(8 * ((size_t)P * P + 10 * (size_t)P + 64))) return fail(SEPO_E_NOMEM, "count scratch");
     uint64_t* dsend = (uint64_t*)t->sh_cnt.p;  // [P][3] records, key bytes, value bytes per destination
     uint64_t* drecv = dsend + 3 * P;            // [P][3] from each source
     uint64_t* dseg = drecv + 3 * P;             // [2P] segment starts / byte bases of a received chunk
     uint64_t* dagree = dseg + 2 * P;            // [2] longest key, chunks
+    uint64_t* dflag = dagree + 2;               // [2] window agreement / barrier word
+    uint64_t* dmat = dflag + 2;                 // [P][P] records rank s sends to rank d (peer-memory path)
+    WireRec** dptr = (WireRec**)(dmat + (size_t)P * P);  // [P] destination of each part
     // ---- agree on the format and the number of chunks: one all-reduce (max)
-    uint64_t per = 64ull << 20;
+    uint64_t per = 256ull << 20;  // (each chunk pays two hot-set discoveries and ~6 host syncs)
     if (const char* e = getenv("SEPO_SHARD_CHUNK")) per = strtoull(e, nullptr, 10);
     per = std::max<uint64_t>(2048, per / 2048 * 2048);
-    // CSR keys travel as CSR (word tiles combine too little to pay for 32-byte wire records: C2 at
-    // N = 1, 146 ms per job as wire records vs 82 ms as CSR); SEPO_SHARD_WIRE=1 sends CSR batches whose
-    // keys are all <= 16 bytes as wire records
+    // CSR batches whose keys are all <= 16 bytes (words) travel as wire records too: with the hot keys
+    // folded out, C2 at N = 1 takes 76.9 ms per routed job as wire records vs 116.5 ms as a CSR partition
+    // (profiles/r02/routed_n1.jsonl); SEPO_SHARD_WIRE=0 keeps CSR batches CSR
     const char* ew = getenv("SEPO_SHARD_WIRE");
-    const bool wire_csr = ew && ew[0] == '1';
+    const bool wire_csr = !(ew && ew[0] == '0');
     uint64_t agree[2] = {ko ? 0ull : (uint64_t)kw, (n + per - 1) / per};
     if (ko && !wire_csr) agree[0] = 1ull << 20;  // (never wire)
     if (ko && wire_csr) {
@@ -2158,6 +2251,11 @@ int64_t sepo_run_sharded(sepo_table* t, const uint8_t* keys, const uint64_t* ko,
     const bool wire = agree[0] <= 16;
     const uint64_t nch = agree[1];
     const bool csr_keys = !wire && (ko != nullptr || kw == 0);  // received keys carry offsets
+    // wire chunks go straight into the owners' receive windows over peer memory (the route kernel's
+    // stores are the exchange, NEXT-2 ii) unless SEPO_SHARD_P2P=0 or a window cannot be registered
+    const char* ep = getenv("SEPO_SHARD_P2P");
+    bool p2p = wire && !(ep && ep[0] == '0') && !t->win_failed;
+    const uint64_t seed_x = kRouteSeed ^ 0x6a09e667f3bcc909ull;  // (as sepo_route_combine)
     // ---- job state (as run_device): prepared re-issue records sized for what was received
     Batch cur{};
     cur.kw = wire ? 0u : kw;
@@ -2170,11 +2268,12 @@ int64_t sepo_run_sharded(sepo_table* t, const uint8_t* keys, const uint64_t* ko,
     cur.prep_fmt = (has_vals && short_keys) ? 33u : 0u;
     const uint64_t slack = (uint64_t)t->grid * 32 * kPrepChunk;
     if (t->prep_n.grow(64)) return fail(SEPO_E_NOMEM, "prepared list counter");
-    {   // the prepared list, sized once for about as many records as this rank sends (hash routing
-        // balances the parts), bounded by half the free memory; it grows (one copy) if a rank receives more
+    {   // the prepared list: room for a quarter of the records this rank sends (hash routing balances
+        // the parts), at most a quarter of the free memory; it grows by half (one copy) when a chunk
+        // could overflow it (a table far over budget declines most records)
         size_t fr = 0, tot = 0;
-        uint64_t want = n + slack * std::max<uint64_t>(nch, 1);
-        if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) want = std::min<uint64_t>(want, (fr + t->prep[0].cap) / 2 / prb);
+        uint64_t want = n / 4 + slack * std::max<uint64_t>(nch, 1);
+        if (cudaMemGetInfo(&fr, &tot) == cudaSuccess) want = std::min<uint64_t>(want, (fr + t->prep[0].cap) / 4 / prb);
         if ((uint64_t)t->prep[0].cap < want * prb) {
             t->prep[0].release();
             if (t->prep[0].grow(want * prb)) return fail(SEPO_E_NOMEM, "prepared re-issue list");
@@ -2224,8 +2323,54 @@ int64_t sepo_run_sharded(sepo_table* t, const uint8_t* keys, const uint64_t* ko,
     for (uint64_t c = 0; c < nch; ++c) {
         const uint64_t r0 = std::min(n, c * per), r1 = std::min(n, r0 + per), cn = r1 - r0;
         std::vector<uint64_t> send(3 * P, 0), recv(3 * P, 0), pc(P + 1, 0);
-        // ---- route chunk c (route stream; the router syncs it)
-        if (cn && wire) {
+        const WireRec* p2p_in = nullptr;  // this rank's window slot holding chunk c (peer-memory path)
+        uint64_t rn = 0, rk = 0, rv = 0;
+        if (p2p) {
+            // ---- route pass 0, all-gather of the count matrix, pass 1 storing into the owners' windows
+            Batch bc{};
+            bc.keys = keys + (ko ? 0 : r0 * (uint64_t)kw); bc.ko = ko ? ko + r0 : nullptr; bc.kw = kw;
+            bc.vals = vals ? vals + r0 * (uint64_t)vw : nullptr; bc.vw = vw; bc.n = cn;
+            std::vector<unsigned long long> hc;
+            std::vector<uint64_t> tot, mat((size_t)P * P), start(P, 0);
+            rc = route_pass0(bc, P, seed_x, t->sh_tmp[2].p, cur_sms(), rs, hc);
+            if (rc) return rc;
+            route_part_totals(hc, P, cur_sms(), tot);
+            CK(t, cudaMemcpyAsync(dsend, tot.data(), 8 * P, cudaMemcpyHostToDevice, rs));
+            NK(t, ncclAllGather(dsend, dmat, P, ncclUint64, comm, rs));
+            CK(t, cudaMemcpyAsync(mat.data(), dmat, 8 * (size_t)P * P, cudaMemcpyDeviceToHost, rs));
+            CK(t, cudaStreamSynchronize(rs));
+            uint64_t need = 0;
+            for (uint32_t d = 0; d < P; ++d) {
+                uint64_t in = 0;
+                for (uint32_t sr = 0; sr < P; ++sr) {
+                    in += mat[(size_t)sr * P + d];
+                    if (sr < (uint32_t)t->rank) start[d] += mat[(size_t)sr * P + d];
+                }
+                need = std::max(need, in);
+                if (d == (uint32_t)t->rank) rn = in;
+            }
+            t->st.kernel_launches += 2;
+            trace("run_sharded: counts gathered", rn);
+            rc = ensure_window(t, comm, need, dflag);
+            if (rc < 0) return rc;
+            if (rc == 0) {
+                const size_t off = (size_t)(c & 1) * t->win_cap * sizeof(WireRec);
+                p2p_ptrs_kernel<<<1, 32, 0, rs>>>((ncclWindow_t)t->win, off, (int)P, dptr);
+                rc = route_pass1(bc, P, seed_x, t->sh_tmp[2].p, cur_sms(), rs, hc, start, nullptr, dptr);
+                if (rc) return rc;
+                // every rank's stores into every window are done before any rank reads its own
+                NK(t, ncclAllReduce(dflag + 1, dflag + 1, 1, ncclUint64, ncclSum, comm, rs));
+                CK(t, cudaEventRecord(evs[c], rs));
+                p2p_in = reinterpret_cast<const WireRec*>((const uint8_t*)t->win_buf + off);
+                t->st.kernel_launches += 3;
+                t->st.p2p_chunks++;
+            } else {
+                p2p = false;  // (all ranks: the agreement above) — this chunk and the rest via send/recv
+            }
+        }
+        if (p2p_in) {
+            // (received already: skip the send/recv exchange)
+        } else if (cn && wire) {
             if (t->sh_send[0].grow(cn * sizeof(WireRec))) return fail(SEPO_E_NOMEM, "wire send buffer");
             const int64_t m = sepo_route_combine(keys + (ko ? 0 : r0 * (uint64_t)kw), ko ? ko + r0 : nullptr, kw,
                                                  vals ? vals + r0 * (uint64_t)vw : nullptr, vw, cn, P, kRouteSeed,
@@ -2254,77 +2399,80 @@ int64_t sepo_run_sharded(sepo_table* t, const uint8_t* keys, const uint64_t* ko,
                 for (int x = 0; x < 3; ++x) send[3 * p + x] = st[3 * (p + 1) + x] - st[3 * p + x];
             t->st.kernel_launches += 3;
         }
-        // ---- counts
-        CK(t, cudaMemcpyAsync(dsend, send.data(), 8 * 3 * P, cudaMemcpyHostToDevice, rs));
-        NK(t, ncclGroupStart());
-        for (uint32_t p = 0; p < P; ++p) {
-            NK(t, ncclSend(dsend + 3 * p, 3, ncclUint64, (int)p, comm, rs));
-            NK(t, ncclRecv(drecv + 3 * p, 3, ncclUint64, (int)p, comm, rs));
-        }
-        NK(t, ncclGroupEnd());
-        CK(t, cudaMemcpyAsync(recv.data(), drecv, 8 * 3 * P, cudaMemcpyDeviceToHost, rs));
-        CK(t, cudaStreamSynchronize(rs));
-        uint64_t rn = 0, rk = 0, rv = 0;
-        for (uint32_t p = 0; p < P; ++p) { rn += recv[3 * p]; rk += recv[3 * p + 1]; rv += recv[3 * p + 2]; }
-        // ---- receive space (wire: slot c & 1, last read by chunk c-2's insert, finished already;
-        // CSR: appended to the records held — growing them waits for the running insert)
-        if (wire) {
-            if (t->sh_recv[c & 1].grow(std::max<uint64_t>(rn, 1) * sizeof(WireRec))) return fail(SEPO_E_NOMEM, "wire receive buffer");
-        } else {
-            const bool fit = hkb + rk + 16 <= t->sh_held[0].cap && (!csr_keys || (hn + rn + 1) * 8 <= t->sh_held[1].cap) &&
-                             (!vals || hvb + rv + 16 <= t->sh_held[2].cap);
-            if (!fit) {
-                CK(t, cudaStreamSynchronize(s));
-                if ((rc = grow_keep(t, t->sh_held[0], hkb, hkb + rk + 16, rs))) return rc;
-                if (csr_keys && (rc = grow_keep(t, t->sh_held[1], hn * 8, (hn + rn + 1) * 8, rs))) return rc;
-                if (vals && (rc = grow_keep(t, t->sh_held[2], hvb, hvb + rv + 16, rs))) return rc;
+        if (!p2p_in) {
+            trace("run_sharded: chunk routed", c);
+            // ---- counts
+            CK(t, cudaMemcpyAsync(dsend, send.data(), 8 * 3 * P, cudaMemcpyHostToDevice, rs));
+            NK(t, ncclGroupStart());
+            for (uint32_t p = 0; p < P; ++p) {
+                NK(t, ncclSend(dsend + 3 * p, 3, ncclUint64, (int)p, comm, rs));
+                NK(t, ncclRecv(drecv + 3 * p, 3, ncclUint64, (int)p, comm, rs));
             }
-        }
-        // ---- payload (one NCCL group), then rebase the received offsets onto the bytes held
-        NK(t, ncclGroupStart());
-        uint64_t so = 0, ro = 0, sko = 0, rko = 0, svo = 0, rvo = 0;
-        for (uint32_t p = 0; p < P; ++p) {
+            NK(t, ncclGroupEnd());
+            CK(t, cudaMemcpyAsync(recv.data(), drecv, 8 * 3 * P, cudaMemcpyDeviceToHost, rs));
+            CK(t, cudaStreamSynchronize(rs));
+            for (uint32_t p = 0; p < P; ++p) { rn += recv[3 * p]; rk += recv[3 * p + 1]; rv += recv[3 * p + 2]; }
+            trace("run_sharded: counts exchanged", rn);
+            // ---- receive space (wire: slot c & 1, last read by chunk c-2's insert, finished already;
+            // CSR: appended to the records held — growing them waits for the running insert)
             if (wire) {
-                const uint64_t sb = send[3 * p] * sizeof(WireRec), rbb = recv[3 * p] * sizeof(WireRec);
-                if (sb) NK(t, ncclSend((uint8_t*)t->sh_send[0].p + pc[p] * sizeof(WireRec), sb, ncclUint8, (int)p, comm, rs));
-                if (rbb) NK(t, ncclRecv((uint8_t*)t->sh_recv[c & 1].p + ro, rbb, ncclUint8, (int)p, comm, rs));
-                ro += rbb;
-                continue;
+                if (t->sh_recv[c & 1].grow(std::max<uint64_t>(rn, 1) * sizeof(WireRec))) return fail(SEPO_E_NOMEM, "wire receive buffer");
+            } else {
+                const bool fit = hkb + rk + 16 <= t->sh_held[0].cap && (!csr_keys || (hn + rn + 1) * 8 <= t->sh_held[1].cap) &&
+                                 (!vals || hvb + rv + 16 <= t->sh_held[2].cap);
+                if (!fit) {
+                    CK(t, cudaStreamSynchronize(s));
+                    if ((rc = grow_keep(t, t->sh_held[0], hkb, hkb + rk + 16, rs))) return rc;
+                    if (csr_keys && (rc = grow_keep(t, t->sh_held[1], hn * 8, (hn + rn + 1) * 8, rs))) return rc;
+                    if (vals && (rc = grow_keep(t, t->sh_held[2], hvb, hvb + rv + 16, rs))) return rc;
+                }
             }
-            uint8_t* hk = (uint8_t*)t->sh_held[0].p + hkb;
-            uint64_t* hko = (uint64_t*)t->sh_held[1].p + hn;
-            uint8_t* hv = (uint8_t*)t->sh_held[2].p + hvb;
-            if (send[3 * p + 1]) NK(t, ncclSend((uint8_t*)t->sh_send[0].p + so, send[3 * p + 1], ncclUint8, (int)p, comm, rs));
-            if (recv[3 * p + 1]) NK(t, ncclRecv(hk + ro, recv[3 * p + 1], ncclUint8, (int)p, comm, rs));
-            if (csr_keys && send[3 * p]) NK(t, ncclSend((uint64_t*)t->sh_send[1].p + sko, send[3 * p], ncclUint64, (int)p, comm, rs));
-            if (csr_keys && recv[3 * p]) NK(t, ncclRecv(hko + rko, recv[3 * p], ncclUint64, (int)p, comm, rs));
-            if (vals && send[3 * p + 2]) NK(t, ncclSend((uint8_t*)t->sh_send[2].p + svo, send[3 * p + 2], ncclUint8, (int)p, comm, rs));
-            if (vals && recv[3 * p + 2]) NK(t, ncclRecv(hv + rvo, recv[3 * p + 2], ncclUint8, (int)p, comm, rs));
-            so += send[3 * p + 1]; ro += recv[3 * p + 1]; sko += send[3 * p]; rko += recv[3 * p];
-            svo += send[3 * p + 2]; rvo += recv[3 * p + 2];
+            // ---- payload (one NCCL group), then rebase the received offsets onto the bytes held
+            NK(t, ncclGroupStart());
+            uint64_t so = 0, ro = 0, sko = 0, rko = 0, svo = 0, rvo = 0;
+            for (uint32_t p = 0; p < P; ++p) {
+                if (wire) {
+                    const uint64_t sb = send[3 * p] * sizeof(WireRec), rbb = recv[3 * p] * sizeof(WireRec);
+                    if (sb) NK(t, ncclSend((uint8_t*)t->sh_send[0].p + pc[p] * sizeof(WireRec), sb, ncclUint8, (int)p, comm, rs));
+                    if (rbb) NK(t, ncclRecv((uint8_t*)t->sh_recv[c & 1].p + ro, rbb, ncclUint8, (int)p, comm, rs));
+                    ro += rbb;
+                    continue;
+                }
+                uint8_t* hk = (uint8_t*)t->sh_held[0].p + hkb;
+                uint64_t* hko = (uint64_t*)t->sh_held[1].p + hn;
+                uint8_t* hv = (uint8_t*)t->sh_held[2].p + hvb;
+                if (send[3 * p + 1]) NK(t, ncclSend((uint8_t*)t->sh_send[0].p + so, send[3 * p + 1], ncclUint8, (int)p, comm, rs));
+                if (recv[3 * p + 1]) NK(t, ncclRecv(hk + ro, recv[3 * p + 1], ncclUint8, (int)p, comm, rs));
+                if (csr_keys && send[3 * p]) NK(t, ncclSend((uint64_t*)t->sh_send[1].p + sko, send[3 * p], ncclUint64, (int)p, comm, rs));
+                if (csr_keys && recv[3 * p]) NK(t, ncclRecv(hko + rko, recv[3 * p], ncclUint64, (int)p, comm, rs));
+                if (vals && send[3 * p + 2]) NK(t, ncclSend((uint8_t*)t->sh_send[2].p + svo, send[3 * p + 2], ncclUint8, (int)p, comm, rs));
+                if (vals && recv[3 * p + 2]) NK(t, ncclRecv(hv + rvo, recv[3 * p + 2], ncclUint8, (int)p, comm, rs));
+                so += send[3 * p + 1]; ro += recv[3 * p + 1]; sko += send[3 * p]; rko += recv[3 * p];
+                svo += send[3 * p + 2]; rvo += recv[3 * p + 2];
+            }
+            NK(t, ncclGroupEnd());
+            if (!wire && csr_keys && rn) {
+                std::vector<uint64_t> seg(2 * P);
+                uint64_t r = 0, kb = 0;
+                for (uint32_t p = 0; p < P; ++p) { seg[p] = r; seg[P + p] = hkb + kb; r += recv[3 * p]; kb += recv[3 * p + 1]; }
+                CK(t, cudaMemcpyAsync(dseg, seg.data(), 16 * P, cudaMemcpyHostToDevice, rs));
+                rc = sepo_launch_shift_offsets((uint64_t*)t->sh_held[1].p + hn, rn, dseg, dseg + P, P, hkb + rk, rs);
+                if (rc) return cuda_check(t, (cudaError_t)rc, "shift offsets");
+                t->st.kernel_launches += 1;
+                CK(t, cudaStreamSynchronize(rs));  // (seg is pageable host memory read by the copy above)
+            }
+            CK(t, cudaEventRecord(evs[c], rs));
         }
-        NK(t, ncclGroupEnd());
-        if (!wire && csr_keys && rn) {
-            std::vector<uint64_t> seg(2 * P);
-            uint64_t r = 0, kb = 0;
-            for (uint32_t p = 0; p < P; ++p) { seg[p] = r; seg[P + p] = hkb + kb; r += recv[3 * p]; kb += recv[3 * p + 1]; }
-            CK(t, cudaMemcpyAsync(dseg, seg.data(), 16 * P, cudaMemcpyHostToDevice, rs));
-            rc = sepo_launch_shift_offsets((uint64_t*)t->sh_held[1].p + hn, rn, dseg, dseg + P, P, hkb + rk, rs);
-            if (rc) return cuda_check(t, (cudaError_t)rc, "shift offsets");
-            t->st.kernel_launches += 1;
-            CK(t, cudaStreamSynchronize(rs));  // (seg is pageable host memory read by the copy above)
-        }
-        CK(t, cudaEventRecord(evs[c], rs));
         // ---- the previous chunk's counters, room in the prepared list, then this chunk's insert
         if ((rc = finish_prev())) return rc;
         if (rn) {
             const uint64_t need = (reserved + rn + slack) * prb;
-            if ((uint64_t)t->prep[0].cap < need && (rc = grow_keep(t, t->prep[0], reserved * prb, need + need / 2, s))) return rc;
+            if ((uint64_t)t->prep[0].cap < need && (rc = grow_keep(t, t->prep[0], reserved * prb, need, s))) return rc;
             if (t->bm.grow(((rn + 31) / 32) * 4)) return fail(SEPO_E_NOMEM, "bitmap scratch");
             CK(t, cudaStreamWaitEvent(s, evs[c], 0));
             Batch bc = cur;
             if (wire) {
-                bc.wire = (const WireRec*)t->sh_recv[c & 1].p;
+                bc.wire = p2p_in ? p2p_in : (const WireRec*)t->sh_recv[c & 1].p;
                 bc.vals = (const uint8_t*)bc.wire;
             } else {
                 bc.keys = (const uint8_t*)t->sh_held[0].p + (csr_keys ? 0 : hkb);

@@ -2251,148 +2251,237 @@ __global__ void __launch_bounds__(256) max_key_len_kernel(const uint64_t* ko, ui
     if (lane_id() == 0 && m) atomicMax(out, m);
 }
 
-// ---- router with CTA pre-combine (COMBINE mode, keys of at most 16 bytes)
-// Records of one rank go to their owners as 32-byte WireRecs {key words, value, length} after the
-// CTA has combined equal keys of its tile in shared memory (a hot Zipf key leaves a tile once, with
-// its partial sum: C5-Zipf's top key, 18 % of the records, would otherwise overload its owner).
-// Two passes over the batch, the same combine in both (the set of distinct keys of a tile does not
-// depend on thread timing): pass 0 counts each part's output, pass 1 writes it through per-part
-// cursors (the order of records within a part is immaterial: the method is order independent).
-namespace rc {
-constexpr int THREADS = 1024, TILE = 2048, NSLOT = 4096, R = TILE / THREADS, NCOL = 64;
-// meta: 0 empty, else the key's route hash (high 48 bits) | owner << 8 | (len + 2)
-struct Slot { unsigned long long w0, w1, v, meta; };
+// ---- router with hot-key pre-combine (COMBINE mode, keys of at most 16 bytes)
+// Records of one rank go to their owners as 32-byte WireRecs {key words, value, length}. The keys of
+// the batch's sampled hot set (the same discovery as the insert kernels, on the route hash) never
+// leave as records: every CTA folds their records into pending sums in shared memory (warp
+// __match_any_sync fold + one shared atomic per distinct key), the CTAs' sums meet in a global array,
+// and each hot key leaves the rank ONCE, as one wire record carrying its total (C5-Zipf's top key,
+// 18 % of the records, would otherwise overload its owner and the links into it). Other records leave
+// one wire record each (a tile of uniform keys holds almost no duplicates to combine).
+// Two passes over the batch with the same static split of 32-record groups over the warps (the
+// hot / not-hot decision reads a fixed hot set): pass 0 counts each CTA's non-hot records per part,
+// the host scans them into per-(part, CTA) bases, pass 1 writes the records through per-CTA cursors
+// and flushes the hot sums; rh_emit_hot then appends each part's hot keys after its other records.
+// (The order of records within a part is immaterial: the method is order independent.)
+namespace rh {
+constexpr int THREADS = 1024, WARPS = THREADS / 32;
+constexpr int DS = stream::DS, NK = hot::K;  // hot slots (2-choice, direct indexed) / hot keys at most
+constexpr int IDXB = stream::IDXB;
 struct Smem {
-    Slot t[NSLOT];
-    Slot col[NCOL];                   // records whose (hash, length) matched a different key's slot
-    unsigned int pc[PT_MAXP];         // records of the tile per part
-    unsigned long long pb[PT_MAXP];   // base of the tile's records in each part
-    unsigned int ncol;
+    uint32_t tags[DS];               // slot words: fingerprint | key index
+    ulonglong2 kw[NK];               // hot keys' words (zero padded)
+    unsigned long long sum[NK];      // the CTA's pending sums
+    unsigned int cnt[PT_MAXP];       // pass 0: non-hot records per part; pass 1: cursors
+    unsigned long long base[PT_MAXP];
+    WireRec* dst[PT_MAXP];           // pass 1: where part p's records go
 };
-static_assert(sizeof(Smem) <= 232448, "route-combine shared memory > 227 KB");
-}  // namespace rc
+static_assert(sizeof(Smem) <= 232448, "route kernel shared memory > 227 KB");
+}  // namespace rh
 
-// Per tile, in three barrier-separated phases (no thread ever waits for another's progress):
-//   A  every warp folds its equal keys; one lane per distinct key claims or finds the slot of its
-//      (hash, length) by CAS on the slot's meta word; a claimer writes its key words and partial sum;
-//   B  the other lanes of a slot add their sums after comparing key words (equal hash and length
-//      but different key bytes — a 48-bit hash collision — go to a small list emitted one by one);
-//   C  (pass 1) the tile's records are written to their owners' parts.
-__global__ void __launch_bounds__(rc::THREADS, 1) route_combine_kernel(Batch b, uint32_t P, uint64_t seed, int pass,
-                                                                      unsigned long long* part_totals,
-                                                                      unsigned long long* long_keys,
-                                                                      const unsigned long long* part_base,
-                                                                      unsigned long long* cursors, WireRec* out) {
-    using namespace rc;
+// out: part p's records at out[bases...] — or, with dstp (the fused route + exchange over peer memory,
+// sepo_run_sharded), at dstp[p][bases...]: rank p's receive window, written through NVLink
+template <int PASS, int IN>
+__global__ void __launch_bounds__(rh::THREADS, 1) route_hot_kernel(Batch b, uint32_t P, uint64_t seed, const hot::Entry* hl,
+                                                                  const unsigned int* n_hot, unsigned long long* counts,
+                                                                  const unsigned long long* bases, unsigned long long* hot_sum,
+                                                                  unsigned long long* long_keys, WireRec* out,
+                                                                  WireRec* const* dstp) {
+    using namespace rh;
     extern __shared__ __align__(16) uint8_t smem_raw[];
-    rc::Smem& S = *reinterpret_cast<rc::Smem*>(smem_raw);
-    const uint32_t tid = threadIdx.x, lane = lane_id();
-    const uint64_t ntiles = (b.n + TILE - 1) / TILE;
-    for (uint32_t x = tid; x < NSLOT; x += THREADS) S.t[x].meta = 0ull;
-    if (tid < PT_MAXP) S.pc[tid] = 0u;
-    if (tid == 0) S.ncol = 0u;
+    Smem& S = *reinterpret_cast<Smem*>(smem_raw);
+    const uint32_t tid = threadIdx.x, lane = lane_id(), G = gridDim.x;
+    constexpr uint32_t IM = (1u << IDXB) - 1u;
+    for (uint32_t x = tid; x < (uint32_t)DS; x += THREADS) S.tags[x] = 0u;
+    for (uint32_t x = tid; x < (uint32_t)NK; x += THREADS) S.sum[x] = 0ull;
+    if (tid < PT_MAXP) {
+        S.cnt[tid] = 0u;
+        S.base[tid] = (PASS == 1 && tid < P) ? bases[(uint64_t)tid * G + blockIdx.x] : 0ull;
+        S.dst[tid] = (PASS == 1 && tid < P) ? (dstp ? dstp[tid] : out) : nullptr;
+    }
     __syncthreads();
-    for (uint64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
-        uint64_t kw0[R], kw1[R], ksum[R], kmeta[R];
-        uint32_t kslot[R];
-        bool klead[R], kclaim[R];
-        // ---- A
-        for (int r = 0; r < R; ++r) {
-            const uint64_t i = tile * TILE + (uint64_t)r * THREADS + tid;
-            const bool valid = i < b.n;
-            uint64_t s = 0, w0 = 0, w1 = 0, v = 0;
-            uint32_t len = 0;
-            if (valid) {
-                rec_key(b, i, s, len);
-                load_key16(b.keys + s, len, w0, w1);
-                v = rec_value(b, i);
-            }
-            const bool ok = valid && len <= 16;
-            if (valid && !ok && long_keys) atomicAdd(long_keys, 1ull);  // the caller routes this batch as CSR
-            const uint64_t h = hash_key16(ok ? len : 0u, seed, w0, w1, b.keys + s);
-            // warp fold: one lane per distinct key carries the warp's sum (a lane joins the lowest lane
-            // of its hash group only with equal key bytes)
-            const unsigned vm = __ballot_sync(FULLMASK, ok);
-            const unsigned grp = __match_any_sync(FULLMASK, ok ? h : (~0ull ^ lane)) & vm;
-            const uint32_t first = grp ? (uint32_t)(__ffs(grp) - 1) : lane;
-            const uint64_t fw0 = __shfl_sync(FULLMASK, w0, first), fw1 = __shfl_sync(FULLMASK, w1, first);
-            const uint32_t flen = __shfl_sync(FULLMASK, len, first);
-            const bool same = ok && fw0 == w0 && fw1 == w1 && flen == len;
-            const unsigned sm = __ballot_sync(FULLMASK, same) & grp;
-            const bool lead = ok && (!same || lane == first);
-            const unsigned mine = same ? sm : (ok ? (1u << lane) : 0u);
-            uint64_t sum = v;
-            if (b.vals == nullptr) {
-                sum = (uint64_t)__popc(mine);
-            } else if (__any_sync(FULLMASK, __popc(mine) > 1)) {
-                sum = 0;
-                for (int xl = 0; xl < 32; ++xl) {
-                    const uint64_t vx = __shfl_sync(FULLMASK, v, xl);
-                    if ((mine >> xl) & 1u) sum += vx;
-                }
-            }
-            const uint32_t owner = (uint32_t)(((h >> 32) * (uint64_t)P) >> 32);
-            const unsigned long long meta = (h & ~0xffffull) | ((unsigned long long)owner << 8) | (unsigned long long)(len + 2);
-            uint32_t x = (uint32_t)(h >> 7) & (NSLOT - 1);
-            bool claim = false;
-            if (lead) {
-                while (true) {
-                    const unsigned long long m = atomicCAS(&S.t[x].meta, 0ull, meta);
-                    if (m == 0ull) { claim = true; break; }
-                    if (m == meta) break;
-                    x = (x + 1) & (NSLOT - 1);
-                }
-                if (claim) {
-                    S.t[x].w0 = w0; S.t[x].w1 = w1; S.t[x].v = sum;
-                    atomicAdd(&S.pc[owner], 1u);
-                }
-            }
-            kw0[r] = w0; kw1[r] = w1; ksum[r] = sum; kmeta[r] = meta; kslot[r] = x; klead[r] = lead; kclaim[r] = claim;
-        }
-        __syncthreads();
-        // ---- B
-        for (int r = 0; r < R; ++r) {
-            if (!klead[r] || kclaim[r]) continue;
-            const uint32_t x = kslot[r];
-            if (S.t[x].w0 == kw0[r] && S.t[x].w1 == kw1[r]) {
-                atomicAdd(&S.t[x].v, ksum[r]);
-            } else {  // (hash collision: emitted on its own)
-                const uint32_t c = atomicAdd(&S.ncol, 1u);
-                if (c < NCOL) {
-                    S.col[c].w0 = kw0[r]; S.col[c].w1 = kw1[r]; S.col[c].v = ksum[r]; S.col[c].meta = kmeta[r];
-                    atomicAdd(&S.pc[(uint32_t)(kmeta[r] >> 8) & 0xffu], 1u);
-                } else if (long_keys) {
-                    atomicAdd(long_keys, 1ull);  // (never seen: the caller falls back to the CSR route)
+    // Slot placement must be the same in both passes and every CTA (pass 0 counts what pass 1 writes),
+    // so it is decided by priorities, not by the order of atomics: a key's priority is its sample-count
+    // class, then its index in the (hash-sorted, rh_sort_hot) list; round 1 gives slot ds1 to its
+    // highest-priority claimant, round 2 gives each slot still empty to the best key that lost round 1.
+    const unsigned nh = hl ? min(*n_hot, (unsigned)NK) : 0u;
+    if (nh) {
+        constexpr uint32_t JB = 12;  // index bits of a priority (NK <= 4096)
+        static_assert(NK <= (1 << JB), "hot keys");
+        uint32_t prio[(NK + THREADS - 1) / THREADS], d1[(NK + THREADS - 1) / THREADS], d2[(NK + THREADS - 1) / THREADS];
+        bool won[(NK + THREADS - 1) / THREADS], try2[(NK + THREADS - 1) / THREADS];
+#pragma unroll
+        for (int r = 0; r < (NK + THREADS - 1) / THREADS; ++r) {
+            const unsigned j = tid + r * THREADS;
+            prio[r] = 0; won[r] = false; try2[r] = false; d1[r] = 0; d2[r] = 0;
+            if (j < nh) {
+                const hot::Entry e = hl[j];
+                if (e.len <= 16u) {
+                    prio[r] = ((uint32_t)(hot::count_class(e.count) + 1) << JB) | ((1u << JB) - 1u - j);
+                    d1[r] = stream::ds1(e.h); d2[r] = stream::ds2(e.h);
+                    atomicMax(&S.tags[d1[r]], prio[r]);
                 }
             }
         }
         __syncthreads();
-        // ---- C
-        if (pass == 0) {
-            if (tid < P && S.pc[tid]) atomicAdd(&part_totals[tid], (unsigned long long)S.pc[tid]);
-        } else {
-            if (tid < P) {
-                S.pb[tid] = part_base[tid] + atomicAdd(&cursors[tid], (unsigned long long)S.pc[tid]);
-                S.pc[tid] = 0u;
-            }
-            __syncthreads();
-            const uint32_t ncol = min(S.ncol, (uint32_t)NCOL);
-            for (uint32_t x = tid; x < NSLOT + ncol; x += THREADS) {
-                const Slot& sl = x < NSLOT ? S.t[x] : S.col[x - NSLOT];
-                const unsigned long long m = sl.meta;
-                if (m == 0ull) continue;
-                const uint32_t owner = (uint32_t)(m >> 8) & 0xffu;
-                const unsigned long long at = S.pb[owner] + atomicAdd(&S.pc[owner], 1u);
-                reinterpret_cast<ulonglong2*>(out + at)[0] = make_ulonglong2(sl.w0, sl.w1);
-                reinterpret_cast<ulonglong2*>(out + at)[1] = make_ulonglong2(sl.v, (m & 0xffull) - 2ull);
-            }
+#pragma unroll
+        for (int r = 0; r < (NK + THREADS - 1) / THREADS; ++r) {
+            won[r] = prio[r] && S.tags[d1[r]] == prio[r];
+            try2[r] = prio[r] && !won[r] && S.tags[d2[r]] == 0u;  // (read before any round-2 write)
         }
         __syncthreads();
-        for (uint32_t x = tid; x < NSLOT; x += THREADS) S.t[x].meta = 0ull;
-        if (tid < PT_MAXP) S.pc[tid] = 0u;
-        if (tid == 0) S.ncol = 0u;
+#pragma unroll
+        for (int r = 0; r < (NK + THREADS - 1) / THREADS; ++r)
+            if (try2[r]) atomicMax(&S.tags[d2[r]], prio[r]);
+        __syncthreads();
+        uint32_t slot[(NK + THREADS - 1) / THREADS];
+#pragma unroll
+        for (int r = 0; r < (NK + THREADS - 1) / THREADS; ++r) {
+            slot[r] = won[r] ? d1[r] : ((try2[r] && S.tags[d2[r]] == prio[r]) ? d2[r] : ~0u);
+        }
+        __syncthreads();
+        for (uint32_t x = tid; x < (uint32_t)DS; x += THREADS) S.tags[x] = 0u;  // (slots nobody won stay empty)
+        __syncthreads();
+#pragma unroll
+        for (int r = 0; r < (NK + THREADS - 1) / THREADS; ++r) {
+            const unsigned j = tid + r * THREADS;
+            if (slot[r] != ~0u) {
+                const hot::Entry e = hl[j];
+                S.tags[slot[r]] = stream::dfp(e.h, e.len) | j;
+                S.kw[j] = make_ulonglong2(e.w0, e.w1);
+            }
+        }
         __syncthreads();
     }
+    const uint64_t ngroups = (b.n + 31) / 32, nw = (uint64_t)G * WARPS, gw = (uint64_t)blockIdx.x * WARPS + (tid >> 5);
+    unsigned long long nlong = 0;
+    for (uint64_t g = ngroups * gw / nw, gend = ngroups * (gw + 1) / nw; g < gend; ++g) {
+        const uint64_t i = g * 32 + lane;
+        const bool valid = i < b.n;
+        uint64_t s = 0, e = 0, w0 = 0, w1 = 0;
+        lean::offsets<IN>(b, i, valid, s, e);
+        const uint32_t len = (uint32_t)(e - s);
+        const bool ok = valid && len <= 16u;
+        if (valid && !ok) ++nlong;
+        if (ok) {
+            uint64_t x0, x1, x2;
+            lean::key_words(b.keys, s, len, x0, x1, x2);
+            lean::assemble16(x0, x1, x2, (uint32_t)(reinterpret_cast<uintptr_t>(b.keys + s) & 7u), len, w0, w1);
+        }
+        const uint64_t h = hash_key16(ok ? len : 0u, seed, w0, w1, nullptr);
+        int pos = -1;
+        if (nh) {
+            const uint32_t f = stream::dfp(h, len);
+            const uint32_t t1 = S.tags[stream::ds1(h)], t2 = S.tags[stream::ds2(h)];
+            const bool m1 = (t1 & ~IM) == f, m2 = (t2 & ~IM) == f;
+            const uint32_t p = (m1 ? t1 : t2) & IM;
+            if (ok && (m1 || m2)) {
+                const ulonglong2 kk = S.kw[p];
+                if (kk.x == w0 && kk.y == w1) pos = (int)p;
+            }
+        }
+        if (PASS == 1) {  // hot records: one shared atomic per distinct key of the warp
+            const uint64_t v = ok ? rec_value(b, i) : 0ull;
+            const unsigned hm = __ballot_sync(FULLMASK, pos >= 0);
+            if (hm) {
+                const unsigned grp = __match_any_sync(FULLMASK, pos >= 0 ? (unsigned)pos : (0x10000u | lane)) & hm;
+                uint64_t acc = v;
+                if (__any_sync(FULLMASK, __popc(grp) > 1)) {
+                    acc = 0;
+                    for (int xl = 0; xl < 32; ++xl) {
+                        const uint64_t vx = __shfl_sync(FULLMASK, v, xl);
+                        if ((grp >> xl) & 1u) acc += vx;
+                    }
+                }
+                if (pos >= 0 && lane == (uint32_t)(__ffs(grp) - 1)) atomicAdd(&S.sum[pos], (unsigned long long)acc);
+            }
+            // other records: one wire record each, slots reserved per owner group of the warp
+            const bool cold = ok && pos < 0;
+            const uint32_t owner = (uint32_t)(((h >> 32) * (uint64_t)P) >> 32);
+            const unsigned cm = __ballot_sync(FULLMASK, cold);
+            if (cm) {
+                const unsigned gm = __match_any_sync(FULLMASK, cold ? owner : (0x100u | lane)) & cm;
+                const uint32_t leader = (uint32_t)(__ffs(gm | (1u << lane)) - 1);
+                unsigned r = 0;
+                if (cold && lane == leader) r = atomicAdd(&S.cnt[owner], (unsigned)__popc(gm));
+                r = __shfl_sync(FULLMASK, r, leader);
+                if (cold) {
+                    const uint64_t at = S.base[owner] + r + __popc(gm & lanemask_lt());
+                    ulonglong2* o = reinterpret_cast<ulonglong2*>(S.dst[owner] + at);
+                    __stcs(o, make_ulonglong2(w0, w1));
+                    __stcs(o + 1, make_ulonglong2(v, (unsigned long long)len));
+                }
+            }
+        } else {
+            const bool cold = ok && pos < 0;
+            const uint32_t owner = (uint32_t)(((h >> 32) * (uint64_t)P) >> 32);
+            const unsigned cm = __ballot_sync(FULLMASK, cold);
+            if (cm) {
+                const unsigned gm = __match_any_sync(FULLMASK, cold ? owner : (0x100u | lane)) & cm;
+                if (cold && lane == (uint32_t)(__ffs(gm) - 1)) atomicAdd(&S.cnt[owner], (unsigned)__popc(gm));
+            }
+        }
+    }
+    if (nlong && long_keys) atomicAdd(long_keys, nlong);
+    __syncthreads();
+    if (PASS == 0) {
+        if (tid < P) counts[(uint64_t)tid * G + blockIdx.x] = S.cnt[tid];
+    } else {
+        for (uint32_t j = tid; j < nh; j += THREADS)
+            if (S.sum[j]) red_add_u64(&hot_sum[j], S.sum[j]);
+        if (dstp) __threadfence_system();  // (peer stores performed before the exchange's barrier)
+    }
+}
+// the emitted hot list in hash order (the emit kernel's order follows its atomics): one CTA, bitonic
+// sort of (hash, index) in shared memory, then the entries permuted into `out`
+__global__ void __launch_bounds__(1024) rh_sort_hot(const hot::Entry* in, const unsigned int* n_hot, hot::Entry* out) {
+    __shared__ unsigned long long kh[hot::K];
+    __shared__ uint32_t ki[hot::K];
+    const unsigned nh = min(*n_hot, (unsigned)hot::K);
+    for (unsigned j = threadIdx.x; j < (unsigned)hot::K; j += blockDim.x) {
+        kh[j] = j < nh ? in[j].h : ~0ull;
+        ki[j] = j;
+    }
+    __syncthreads();
+    for (unsigned k = 2; k <= (unsigned)hot::K; k <<= 1) {
+        for (unsigned jj = k >> 1; jj > 0; jj >>= 1) {
+            for (unsigned i = threadIdx.x; i < (unsigned)hot::K; i += blockDim.x) {
+                const unsigned l = i ^ jj;
+                if (l > i) {
+                    const bool up = (i & k) == 0;
+                    const bool gt = kh[i] > kh[l] || (kh[i] == kh[l] && ki[i] > ki[l]);
+                    if (gt == up) {
+                        const unsigned long long th = kh[i]; kh[i] = kh[l]; kh[l] = th;
+                        const uint32_t ti = ki[i]; ki[i] = ki[l]; ki[l] = ti;
+                    }
+                }
+            }
+            __syncthreads();
+        }
+    }
+    for (unsigned j = threadIdx.x; j < nh; j += blockDim.x) out[j] = in[ki[j]];
+}
+
+// per part: hot keys owned (pass 0), then each hot key's wire record after the part's other records
+__global__ void rh_count_hot(const hot::Entry* hl, const unsigned int* n_hot, uint32_t P, unsigned long long* hot_pp) {
+    const unsigned nh = hl ? min(*n_hot, (unsigned)rh::NK) : 0u;
+    for (unsigned j = blockIdx.x * blockDim.x + threadIdx.x; j < nh; j += gridDim.x * blockDim.x)
+        if (hl[j].len <= 16u) atomicAdd(&hot_pp[(uint32_t)(((hl[j].h >> 32) * (uint64_t)P) >> 32)], 1ull);
+}
+__global__ void rh_emit_hot(const hot::Entry* hl, const unsigned int* n_hot, uint32_t P, const unsigned long long* hot_sum,
+                            const unsigned long long* hot_base, unsigned long long* hot_cur, WireRec* out,
+                            WireRec* const* dstp) {
+    const unsigned nh = hl ? min(*n_hot, (unsigned)rh::NK) : 0u;
+    for (unsigned j = blockIdx.x * blockDim.x + threadIdx.x; j < nh; j += gridDim.x * blockDim.x) {
+        const hot::Entry e = hl[j];
+        if (e.len > 16u) continue;
+        const uint32_t p = (uint32_t)(((e.h >> 32) * (uint64_t)P) >> 32);
+        const unsigned long long at = hot_base[p] + atomicAdd(&hot_cur[p], 1ull);
+        WireRec r;
+        r.w0 = e.w0; r.w1 = e.w1; r.v = hot_sum[j]; r.len = e.len;
+        (dstp ? dstp[p] : out)[at] = r;
+    }
+    if (dstp) __threadfence_system();
 }
 
 
@@ -3529,16 +3618,75 @@ int sepo_launch_map(const uint8_t* text, uint64_t n, int lines, int pass, unsign
     }
     return cudaGetLastError();
 }
-int sepo_launch_route_combine(const Batch& b, uint32_t P, uint64_t seed, int pass, unsigned long long* part_totals,
-                              unsigned long long* long_keys, const unsigned long long* part_base,
-                              unsigned long long* cursors, WireRec* out, int grid, cudaStream_t s) {
+// Router scratch (device): hot-set discovery scratch, then counts [P][grid], bases [P][grid], the hot
+// keys' sums [K], per-part hot counts / bases / cursors [3][32] and the long-key counter.
+static size_t rh_off_counts() { return (sepo_hot_scratch_bytes() + 255) & ~(size_t)255; }
+size_t sepo_route_scratch_bytes(uint32_t P, int grid) {
+    return rh_off_counts() + 8 * (2 * (size_t)P * grid + hot::K + 3 * 32 + 8);
+}
+void sepo_route_layout(uint32_t P, int grid, size_t* counts_off, size_t* hot_pp_off) {
+    *counts_off = rh_off_counts();
+    *hot_pp_off = rh_off_counts() + 8 * (2 * (size_t)P * grid + hot::K);
+}
+int sepo_launch_route_hot(const Batch& b, uint32_t P, uint64_t seed, int pass, void* scratch, int grid, WireRec* out,
+                          cudaStream_t s, WireRec* const* dstp) {
     static bool attr = false;
     if (!attr) {
-        cudaFuncSetAttribute(route_combine_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(rc::Smem));
+        const int sm = (int)sizeof(rh::Smem);
+        cudaFuncSetAttribute(route_hot_kernel<0, IN_CSR>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+        cudaFuncSetAttribute(route_hot_kernel<0, IN_FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+        cudaFuncSetAttribute(route_hot_kernel<1, IN_CSR>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+        cudaFuncSetAttribute(route_hot_kernel<1, IN_FIXED>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
         attr = true;
     }
-    if (b.n) route_combine_kernel<<<grid, rc::THREADS, sizeof(rc::Smem), s>>>(b, P, seed, pass, part_totals, long_keys,
-                                                                              part_base, cursors, out);
+    uint8_t* p = reinterpret_cast<uint8_t*>(scratch);
+    hot::SampleSlot* tab = reinterpret_cast<hot::SampleSlot*>(p);
+    hot::Entry* list = reinterpret_cast<hot::Entry*>(p + sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS);
+    unsigned int* n_out = reinterpret_cast<unsigned int*>(list + hot::K);
+    unsigned long long* counts = reinterpret_cast<unsigned long long*>(p + rh_off_counts());
+    unsigned long long* bases = counts + (size_t)P * grid;
+    unsigned long long* hot_sum = bases + (size_t)P * grid;
+    unsigned long long* hot_pp = hot_sum + hot::K;   // [32] hot keys per part
+    unsigned long long* hot_base = hot_pp + 32;      // [32]
+    unsigned long long* hot_cur = hot_base + 32;     // [32]
+    unsigned long long* longk = hot_cur + 32;
+    const bool have = b.n >= hot_min_records(8ull << 18);
+    // the sorted hot list lives in the sample table's space (free once the list is emitted)
+    hot::Entry* sorted = reinterpret_cast<hot::Entry*>(p + sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS -
+                                                       sizeof(hot::Entry) * hot::K);
+    const hot::Entry* hl = have ? sorted : nullptr;
+    const size_t sm = sizeof(rh::Smem);
+    if (pass == 0) {
+        cudaMemsetAsync(hot_pp, 0, 8 * (3 * 32 + 8), s);
+        cudaMemsetAsync(n_out, 0, (HOT_HIST + 2) * sizeof(unsigned int), s);
+        if (have) {  // hot-set discovery on the route hash (no table entries: nothing to resolve)
+            Dev d{};
+            d.seed = seed;
+            const uint64_t n_sample = 1ull << 18;
+            unsigned int* hist = n_out + 1;
+            cudaMemsetAsync(tab, 0, sizeof(hot::SampleSlot) * hot::SAMPLE_SLOTS, s);
+            hot_sample_kernel<<<4 * 148, 256, 0, s>>>(d, b, std::max<uint64_t>(1, b.n / n_sample), std::min(n_sample, b.n), tab);
+            hot_hist_kernel<<<2 * 148, 256, 0, s>>>(tab, hist, 4u);
+            hot_threshold_kernel<<<1, 1024, 0, s>>>(hist, 4u, (uint32_t)hot::K);
+            hot_emit_kernel<<<2 * 148, 256, 0, s>>>(d, b, tab, hist, list, n_out, (uint32_t)hot::K);
+            hot_clamp_kernel<<<1, 32, 0, s>>>(n_out, (uint32_t)hot::K);
+            rh_sort_hot<<<1, 1024, 0, s>>>(list, n_out, sorted);
+            rh_count_hot<<<8, 256, 0, s>>>(hl, n_out, P, hot_pp);
+        }
+        if (b.n) {
+            if (b.ko) route_hot_kernel<0, IN_CSR><<<grid, rh::THREADS, sm, s>>>(b, P, seed, hl, n_out, counts, nullptr, nullptr, longk, nullptr, nullptr);
+            else route_hot_kernel<0, IN_FIXED><<<grid, rh::THREADS, sm, s>>>(b, P, seed, hl, n_out, counts, nullptr, nullptr, longk, nullptr, nullptr);
+        } else {
+            cudaMemsetAsync(counts, 0, 8 * (size_t)P * grid, s);
+        }
+    } else {
+        cudaMemsetAsync(hot_sum, 0, 8 * hot::K, s);
+        if (b.n) {
+            if (b.ko) route_hot_kernel<1, IN_CSR><<<grid, rh::THREADS, sm, s>>>(b, P, seed, hl, n_out, nullptr, bases, hot_sum, nullptr, out, dstp);
+            else route_hot_kernel<1, IN_FIXED><<<grid, rh::THREADS, sm, s>>>(b, P, seed, hl, n_out, nullptr, bases, hot_sum, nullptr, out, dstp);
+        }
+        if (have) rh_emit_hot<<<8, 256, 0, s>>>(hl, n_out, P, hot_sum, hot_base, hot_cur, out, dstp);
+    }
     return cudaGetLastError();
 }
 int sepo_launch_max_key_len(const uint64_t* ko, uint64_t n, unsigned long long* out, cudaStream_t s) {

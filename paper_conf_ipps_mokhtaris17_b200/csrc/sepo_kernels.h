@@ -64,13 +64,14 @@ int sepo_launch_insert(const sepo::Dev& d, const sepo::Batch& b, int mode, int g
                        bool* hot_built = nullptr, bool lean_in = false, bool long_keys = false);
 size_t sepo_hot_count_offset();
 int sepo_launch_reinsert(const sepo::Dev& d, const sepo::Batch& b, int grid, cudaStream_t s, bool long_keys = false);
-// Router with CTA pre-combine (a12): pass 0 counts per-part output records (part_totals[P], device,
-// zeroed by the caller) and flags keys longer than 16 bytes in *long_keys; pass 1 writes the
-// WireRecs of part p at out + part_base[p] (device, exclusive prefix of the totals) through the
-// per-part cursors cursors[P] (device, zeroed by the caller).
-int sepo_launch_route_combine(const sepo::Batch& b, uint32_t P, uint64_t seed, int pass, unsigned long long* part_totals,
-                              unsigned long long* long_keys, const unsigned long long* part_base,
-                              unsigned long long* cursors, sepo::WireRec* out, int grid, cudaStream_t s);
+// Router with hot-key pre-combine (a12). Scratch (device, sepo_route_scratch_bytes): hot-set
+// discovery scratch, counts [P][grid] at counts_off, bases [P][grid], hot sums [K], then at
+// hot_pp_off: hot keys per part [32], hot bases [32], hot cursors [32], long-key counter.
+// Pass 0 (discovery + counts; the host scans counts / hot_pp into bases / hot bases), pass 1 (write).
+size_t sepo_route_scratch_bytes(uint32_t P, int grid);
+void sepo_route_layout(uint32_t P, int grid, size_t* counts_off, size_t* hot_pp_off);
+int sepo_launch_route_hot(const sepo::Batch& b, uint32_t P, uint64_t seed, int pass, void* scratch, int grid,
+                          sepo::WireRec* out, cudaStream_t s, sepo::WireRec* const* dstp = nullptr);
 size_t sepo_hot_scratch_bytes();
 int sepo_default_grid(int mode, int n_sms);
 int sepo_launch_reprobe(const sepo::Dev& d, const sepo::Batch& b, int mode, int probe, int grid,

@@ -73,6 +73,8 @@ def route_combine(keys, key_offsets, vals, n_parts, route_seed=0, fixed_key_widt
     stream = ctypes.c_void_p(torch.cuda.current_stream(dev).cuda_stream)
     args = (_ptr(keys), _ptr(key_offsets), fixed_key_width, _ptr(vals), fixed_val_width, n, n_parts, route_seed)
     E_NOMEM = -2
+    if out is None or out.numel() < max(n, 1) * WIRE_BYTES:  # (at most one record per input record)
+        out = torch.empty(max(n, 1) * WIRE_BYTES, dtype=torch.uint8, device=dev)
     for _ in range(2):
         cap = out.numel() // WIRE_BYTES if out is not None else 0
         m = L.sepo_route_combine(*args, out.data_ptr() if cap else None, cap, counts.ctypes.data, scratch.data_ptr(),
@@ -162,8 +164,8 @@ def route(keys, key_offsets, vals, group=None, route_seed=0, fixed_key_width=0, 
 class Router:
     """Routes each step's batch of this rank to the key owners and keeps per-step statistics.
 
-    combine=True (COMBINE tables, keys <= 16 B): sepo_route_combine pre-combines every CTA tile and
-    the exchange carries 32-byte wire records -> route() returns ("wire", tensor) for Table.run_wire;
+    combine=True (COMBINE tables, keys <= 16 B): sepo_route_combine folds the batch's hot keys into one
+    record each and the exchange carries 32-byte wire records -> route() returns ("wire", tensor) for Table.run_wire;
     batches with longer keys (and combine=False) are partitioned as CSR -> ("csr", (keys, offsets,
     vals)) for Table.run."""
 
@@ -176,11 +178,12 @@ class Router:
         world = dist.get_world_size(self.group)
         n_in = (key_offsets.numel() - 1) if key_offsets is not None else keys.numel() // max(self.kw, 1)
         if self.combine:
+            if self._wire_buf is None or self._wire_buf.numel() < max(n_in, 1) * WIRE_BYTES:  # (reused step to step)
+                self._wire_buf = None
+                self._wire_buf = torch.empty(max(n_in, 1) * WIRE_BYTES, dtype=torch.uint8, device=keys.device)
             r = route_combine(keys, key_offsets, vals, world, self.seed, self.kw, self.vw, out=self._wire_buf)
             if r is not None:
                 wire, counts = r
-                if self._wire_buf is None or self._wire_buf.numel() < wire.numel():
-                    self._wire_buf = wire
                 out = exchange_wire(wire, counts, self.group)
                 self._last = {"records_in": n_in, "records_sent": int(counts[-1]), "records_out": out.numel() // WIRE_BYTES,
                               "format": "wire (pre-combined)"}

@@ -127,3 +127,23 @@ def test_hot_min_small_batches(cuda, monkeypatch):
             assert (st["hot_keys"] > 0) == (hm == "1000")
             assert_same(got, exp)
             assert st["cross_gen_dups"] == 0
+
+
+@pytest.mark.parametrize("name,scale,ratio", [("C2", 1 / 256, 0.5), ("C2", 1 / 256, 4), ("C3", 1 / 2000, 2),
+                                              ("C5z", 1 / 128, 4), ("C1", 1.0, 4)])
+def test_dir_prefetch_path(cuda, monkeypatch, name, scale, ratio):
+    """SEPO_DIR_PF=1 + SEPO_LEAN=0 force the path of tables larger than L2 (insert_stream_kernel with
+    queued misses' bucket lines L2-prefetched) on small tables — every config equals the oracle, in
+    budget and over (C3: long keys; C5z: values, 8 keys per bucket; C1: below the hot-set threshold)"""
+    monkeypatch.setenv("SEPO_DIR_PF", "1")
+    monkeypatch.setenv("SEPO_LEAN", "0")
+    s = gen.config(name, scale)
+    inp = device_inputs(s)
+    pb = 65536 if name == "C3" else 16384
+    F = footprint_pages(s, 1 << 18, pb, inputs=inp)
+    P = max(8, int(np.ceil(F / ratio))) + (2 if ratio >= 1 else 0)
+    got, passes, st = run_job(s, sepo().budget_for(1 << 18, pb, P), 1 << 18, pb, inputs=inp, check_dups=True)
+    assert_same(got, oracle_expected(s))
+    assert st["cross_gen_dups"] == 0
+    if ratio > 1:
+        assert passes >= 2

@@ -101,7 +101,24 @@ def test_sharded_job_loopback(cuda, name, P):
     assert got == exp
 
 
-# ---- router with CTA pre-combine (sepo_route_combine) + wire records
+# ---- router with hot-key pre-combine (sepo_route_combine) + wire records
+def top_key(s, exp):
+    """the most frequent key of a stream (pairs: by record count; words: the counts are the values)"""
+    if s.family != gen.GEN_PAIRS:
+        return max(exp, key=lambda x: exp[x])
+    keys, _, _ = s.host()
+    u, c = np.unique(np.asarray(keys).view(np.uint64), return_counts=True)
+    return int(u[np.argmax(c)]).to_bytes(8, "little")
+
+
+def wire_count(wire, key):
+    """records of `key` among 32-byte wire records"""
+    a = wire.cpu().numpy().view(np.uint64).reshape(-1, 4)
+    kb = key + bytes(16 - len(key))
+    w0, w1 = int.from_bytes(kb[:8], "little"), int.from_bytes(kb[8:], "little")
+    return int(((a[:, 0] == w0) & (a[:, 1] == w1) & (a[:, 3] == len(key))).sum())
+
+
 def wire_dict(wire):
     """32-byte wire records -> {key bytes: summed value} (test-side decode; records of one key may repeat)"""
     a = wire.cpu().numpy().view(np.uint64).reshape(-1, 4)
@@ -112,11 +129,15 @@ def wire_dict(wire):
     return out
 
 
-@pytest.mark.parametrize("name,P", [("C2", 1), ("C2", 4), ("C5z", 3), ("C5u", 2)])
-def test_route_combine_parts(cuda, name, P):
+@pytest.mark.parametrize("name,P,hot_min", [("C2", 1, None), ("C2", 4, None), ("C5z", 3, None), ("C5u", 2, None),
+                                             ("C2", 4, 1 << 16), ("C5z", 8, 1 << 16)])
+def test_route_combine_parts(cuda, monkeypatch, name, P, hot_min):
     """every part's pre-combined records sum to the oracle's values of exactly the keys it owns, the
-    parts own disjoint key sets, and equal keys were combined inside each CTA tile (fewer records)"""
+    parts own disjoint key sets, and each hot key left the batch as ONE record (Zipf: far fewer records
+    than the batch; the hot set runs from SEPO_HOT_MIN records, 2^21 by default)"""
     from paper_conf_ipps_mokhtaris17_b200 import shard
+    if hot_min:
+        monkeypatch.setenv("SEPO_HOT_MIN", str(hot_min))
     scale = {"C2": 1 / 1024, "C5z": 2 ** -12, "C5u": 2 ** -14}[name]
     s = gen.config(name, scale=scale)
     exp = oracle_expected(s)
@@ -135,8 +156,10 @@ def test_route_combine_parts(cuda, name, P):
         for b in range(a + 1, P):
             assert not (owners[a] & owners[b])
     assert got == exp
-    if name != "C5u":  # Zipf: the hot keys leave each tile once
+    if hot_min:  # Zipf: the hot keys leave the batch once
         assert int(counts[-1]) < 0.7 * s.n
+        top = top_key(s, exp)  # the batch's most frequent key is hot: exactly one record
+        assert wire_count(wire[:int(counts[-1]) * 32], top) == 1
     # the owners agree with the CSR partition's (same route hash)
     if P > 1 and not fixed:
         ok, oko, _, starts = shard.partition(k, o, None, P, route_seed=5)
@@ -144,6 +167,25 @@ def test_route_combine_parts(cuda, name, P):
             sk, so = segment(ok, oko, starts, p)
             keys_p = set(oracle.combine(sk.cpu().numpy(), so.cpu().numpy().view(np.uint64)).as_dict())
             assert keys_p == owners[p]
+
+
+def test_route_hot_set_active_large(cuda):
+    """a C5z batch above the hot-set threshold (2^21 records): the top keys leave once, the parts still sum
+    to the oracle"""
+    from paper_conf_ipps_mokhtaris17_b200 import shard
+    s = gen.config("C5z", scale=2 ** -9)
+    assert s.n >= (1 << 21)
+    exp = oracle_expected(s)
+    k, _, v = s.device()
+    wire, counts = shard.route_combine(k, None, v, 4, route_seed=9, fixed_key_width=8, fixed_val_width=8)
+    got = {}
+    for p in range(4):
+        for key, val in wire_dict(wire[int(counts[p]) * 32:int(counts[p + 1]) * 32]).items():
+            got[key] = (got.get(key, 0) + val) % (1 << 64)
+    assert got == exp
+    assert int(counts[-1]) < 0.5 * s.n
+    top = top_key(s, exp)
+    assert wire_count(wire[:int(counts[-1]) * 32], top) == 1
 
 
 def test_route_combine_rejects_long_keys(cuda):
@@ -216,13 +258,16 @@ def test_nccl_sharded_one_rank(cuda, name, ratio):
 
 
 # ---- the pipelined sharded job (sepo_run_sharded): chunk c+1 routed / exchanged beside chunk c's insert
-@pytest.mark.parametrize("name,ratio,chunk", [("C2", 4, 1 << 17), ("C5z", 4, 1 << 16), ("C5u", 2, 1 << 16),
-                                              ("C3", 2, 1 << 15), ("C1", 1, 10_000)])
-def test_nccl_run_sharded_one_rank(cuda, monkeypatch, name, ratio, chunk):
+@pytest.mark.parametrize("name,ratio,chunk,p2p", [("C2", 4, 1 << 17, "1"), ("C5z", 4, 1 << 16, "1"), ("C5u", 2, 1 << 16, "1"),
+                                                  ("C3", 2, 1 << 15, "1"), ("C1", 1, 10_000, "1"),
+                                                  ("C2", 4, 1 << 17, "0"), ("C5z", 4, 1 << 16, "0")])
+def test_nccl_run_sharded_one_rank(cuda, monkeypatch, name, ratio, chunk, p2p):
     """sepo_run_sharded over a one-rank NCCL communicator, many chunks (SEPO_SHARD_CHUNK), the table
     `ratio` times its budget so chunks decline records into the prepared list: the export equals the
-    oracle (wire records for words / pairs, a CSR partition for URLs — whose held buffers grow)"""
+    oracle (wire records for words / pairs — stored by the route kernel into the owner's symmetric
+    window, or sent with NCCL send/recv — and a CSR partition for URLs, whose held buffers grow)"""
     monkeypatch.setenv("SEPO_SHARD_CHUNK", str(chunk))
+    monkeypatch.setenv("SEPO_SHARD_P2P", p2p)  # 0: NCCL send/recv of the routed parts
     scale = {"C1": 0.25, "C2": 1 / 512, "C5z": 2 ** -12, "C5u": 2 ** -12, "C3": 1 / 2000}[name]
     s = gen.config(name, scale=scale)
     exp = oracle_expected(s)
@@ -248,13 +293,15 @@ def test_nccl_run_sharded_one_rank(cuda, monkeypatch, name, ratio, chunk):
     assert st["cross_gen_dups"] == 0
     if ratio > 1:
         assert passes >= 2
-    assert st["records_inserted"] >= s.n if name in ("C3", "C1") else True
+    # keys <= 16 bytes go as wire records, routed straight into the owner's window over peer memory
+    assert (st["p2p_chunks"] > 0) == (name != "C3" and p2p == "1")
 
 
-def test_nccl_run_sharded_wire_words(cuda, monkeypatch):
-    """SEPO_SHARD_WIRE=1: a CSR batch of words (all <= 16 bytes) goes as pre-combined wire records"""
+def test_nccl_run_sharded_csr_words(cuda, monkeypatch):
+    """SEPO_SHARD_WIRE=0: a CSR batch of words (all <= 16 bytes, wire records by default) goes as a CSR
+    partition appended to the records held"""
     monkeypatch.setenv("SEPO_SHARD_CHUNK", str(1 << 16))
-    monkeypatch.setenv("SEPO_SHARD_WIRE", "1")
+    monkeypatch.setenv("SEPO_SHARD_WIRE", "0")
     s = gen.config("C2", scale=1 / 1024)
     exp = oracle_expected(s)
     k, o, _ = s.device()
@@ -265,10 +312,13 @@ def test_nccl_run_sharded_wire_words(cuda, monkeypatch):
     t.close()
 
 
-def test_nccl_run_sharded_hot_and_empty(cuda, monkeypatch):
-    """chunks large enough for the hot set (>= 2^21 records), a trailing short chunk, and a second job
+@pytest.mark.parametrize("wire", ["1", "0"], ids=["wire", "csr"])
+def test_nccl_run_sharded_hot_and_empty(cuda, monkeypatch, wire):
+    """chunks large enough for the hot set (>= 2^21 records: the router folds the hot words out of
+    wire chunks, the insert kernel folds them in CSR chunks), a trailing short chunk, and a second job
     with an empty batch on the same communicator (the rank still takes part in the agreement)"""
     monkeypatch.setenv("SEPO_SHARD_CHUNK", str(3 << 20))
+    monkeypatch.setenv("SEPO_SHARD_WIRE", wire)
     s = gen.config("C2", scale=1 / 200)
     exp = oracle_expected(s)
     k, o, _ = s.device()
@@ -278,7 +328,8 @@ def test_nccl_run_sharded_hot_and_empty(cuda, monkeypatch):
     st = t.stats()
     got = sepo().result_dict(t.export())
     assert got == exp
-    assert st["hot_keys"] > 0
+    if wire == "0":
+        assert st["hot_keys"] > 0
     t.reset()
     assert t.run_sharded(None, None, n=0) >= 0
     assert sepo().result_dict(t.export()) == {}
