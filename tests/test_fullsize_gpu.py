@@ -106,3 +106,22 @@ def test_c4_full(cuda):
     assert (c == ec[r]).all(), "list lengths differ from the record counts"
     assert (sm == es[r]).all() and (mx == em[r]).all(), "a value multiset differs"
     t.close()
+
+
+@pytest.mark.parametrize("cfg,scale", [("C2", 1.0), ("C5z", 0.125), ("C3", 1.0)])
+def test_sharded_full(cuda, cfg, scale):
+    """the routed job at full size through sepo_run_sharded on a one-rank communicator (hot-key route
+    into the rank's symmetric window for words / pairs, CSR send/recv for URLs; 2^28-record chunks;
+    table 4x over budget) equals the closed forms key by key"""
+    import paper_conf_ipps_mokhtaris17_b200 as sepo
+    job = _job(cfg, 4.0, scale=scale)
+    k, o, v = job.inputs()
+    t = job.table()
+    t.attach_nccl(sepo.nccl_unique_id(), 1, 0)
+    passes = t.run_sharded(k, o, v)
+    st = t.stats()
+    res = t.export(copy=False)
+    check_combine(job.stream, res)
+    assert passes >= 2 and st["cross_gen_dups"] == 0
+    assert (st["p2p_chunks"] > 0) == (cfg != "C3")
+    t.close()
