@@ -1401,9 +1401,13 @@ __global__ void __launch_bounds__(lean::THREADS, 1) insert_lean_kernel(Dev d, Ba
             if (!VALS) {
                 if (leader) {
                     const unsigned add = (unsigned)__popc(grp);
-                    const unsigned old = atomicAdd(reinterpret_cast<unsigned int*>(&S.sum[pos]), add);
-                    if (big && old + add < old)  // 2^32 wrap of the CTA-local count: carry into the entry
-                        red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(ref_ptr(d, S.ref[pos]), len)), 1ull << 32);
+                    if (!big) {  // fewer than 2^32 records: a CTA-local count cannot wrap (no returned value to wait for)
+                        atomicAdd(reinterpret_cast<unsigned int*>(&S.sum[pos]), add);
+                    } else {
+                        const unsigned old = atomicAdd(reinterpret_cast<unsigned int*>(&S.sum[pos]), add);
+                        if (old + add < old)  // 2^32 wrap of the CTA-local count: carry into the entry
+                            red_add_u64(reinterpret_cast<unsigned long long*>(entry_val(ref_ptr(d, S.ref[pos]), len)), 1ull << 32);
+                    }
                 }
             } else {
                 uint64_t acc = v;

@@ -147,3 +147,20 @@ def test_dir_prefetch_path(cuda, monkeypatch, name, scale, ratio):
     assert st["cross_gen_dups"] == 0
     if ratio > 1:
         assert passes >= 2
+
+
+@pytest.mark.parametrize("name,scale,ratio", [("C4", 1 / 256, 3), ("C4", 1 / 1000, 2), ("C2", 1 / 256, 4), ("C5u", 2 ** -12, 4)])
+def test_evict_overlap_forced(cuda, monkeypatch, name, scale, ratio):
+    """SEPO_EVICT_OVERLAP=1 on tables small enough to skip it by default: every eviction's copies (batched
+    copy-engine copies, progress published per step) overlap the next pass, whose allocator waits per
+    evicted page before reusing it — GROUP (retained key pages between evicted ones) and COMBINE equal
+    the oracle"""
+    monkeypatch.setenv("SEPO_EVICT_OVERLAP", "1")
+    s = gen.config(name, scale)
+    inp = device_inputs(s)
+    kw = dict(mode=sepo().GROUP, fixed_val_width=4) if name == "C4" else {}
+    F = footprint_pages(s, 1 << 18, 16384, inputs=inp, **kw)
+    P = max(8, int(np.ceil(F / ratio))) + 2
+    got, passes, st = run_job(s, sepo().budget_for(1 << 18, 16384, P), 1 << 18, 16384, inputs=inp, check_dups=True, **kw)
+    assert_same(got, oracle_expected(s))
+    assert passes >= 2 and st["cross_gen_dups"] == 0
