@@ -732,10 +732,9 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
     CK(t, cudaStreamWaitEvent(t->copy_stream, t->ev_comp, 0));
     // eviction overlapped with the next pass (the allocator waits per evicted page): measured
     // worth it when a generation is large (C5u 4x job 86 -> 78 ms with a 192 MB pool), not for a
-    // pool inside L2 (C2 4x: 30.5 -> 31.8 ms). GROUP generations (fragmented evict lists: retained
-    // key pages between the evicted ones) overlap through batched copy-engine copies
-    // (cudaMemcpyBatchAsync, one batch per progress step) — one cudaMemcpyAsync per run cost
-    // C4 3x 491 -> 712 ms. SEPO_EVICT_OVERLAP=0/1 forces the choice.
+    // pool inside L2 (C2 4x: 30.5 -> 31.8 ms) nor for GROUP (fragmented evict lists leave through
+    // the gather kernel, which cannot publish progress in evict-list order). SEPO_EVICT_OVERLAP=0/1
+    // forces the choice.
     bool want_overlap;
     {
         const char* ov = getenv("SEPO_EVICT_OVERLAP");
@@ -743,8 +742,7 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
         cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device);
         want_overlap = (ov && (ov[0] == '0' || ov[0] == '1'))
                            ? ov[0] == '1'
-                           : (t->opts.mode == SEPO_COMBINE_SUM_U64 || t->opts.mode == SEPO_GROUP) &&
-                                 (uint64_t)t->n_pages * t->page_bytes > (uint64_t)l2;
+                           : t->opts.mode == SEPO_COMBINE_SUM_U64 && (uint64_t)t->n_pages * t->page_bytes > (uint64_t)l2;
     }
     const bool overlapped = t->write_value32 != nullptr && want_overlap;
     GenImage img;
@@ -778,32 +776,6 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
         bytes = nbytes;
         done = ne;
     }
-    // Copies in evict-list order. Overlapped, the list is cut into progress steps of chunk_pages
-    // positions; the pieces of the runs inside one step go out as ONE batch of copy-engine copies
-    // (cudaMemcpyBatchAsync), then the copy stream publishes the step in ctrl->copied.
-    std::vector<void*> b_dst, b_src;
-    std::vector<size_t> b_size;
-    uint64_t next_step = chunk_pages;
-    auto flush = [&]() -> int {
-        if (b_dst.empty()) return 0;
-        if (b_dst.size() == 1) {
-            CK(t, cudaMemcpyAsync(b_dst[0], b_src[0], b_size[0], cudaMemcpyDefault, t->copy_stream));
-        } else {
-            cudaMemcpyAttributes at{};
-            at.srcAccessOrder = cudaMemcpySrcAccessOrderStream;
-            at.flags = cudaMemcpyFlagPreferOverlapWithCompute;
-            size_t ai = 0, fidx = 0;
-            CK(t, cudaMemcpyBatchAsync(b_dst.data(), b_src.data(), b_size.data(), b_dst.size(), &at, &ai, 1, &fidx,
-                                       t->copy_stream));
-        }
-        b_dst.clear(); b_src.clear(); b_size.clear();
-        if (overlapped) {
-            const int wr = t->write_value32(t->copy_stream, (unsigned long long)(uintptr_t)&t->d.ctrl->copied,
-                                            (unsigned int)done, 0);
-            if (wr) return fail(SEPO_E_CUDA, "cuStreamWriteValue32 failed");
-        }
-        return 0;
-    };
     for (uint64_t i = use_kernel ? ne : 0; i < ne;) {
         uint64_t j = i + 1;
         while (j < ne && t->h_evict[j] == t->h_evict[j - 1] + 1) ++j;
@@ -811,23 +783,21 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
         const size_t nbytes = (size_t)cnt * t->page_bytes;
         uint8_t* hp = arena_alloc(t, nbytes);
         if (!hp) return fail(SEPO_E_NOMEM, "pinned host arena exhausted");
-        for (uint64_t c0 = 0; c0 < cnt;) {
-            const uint64_t cc = std::min<uint64_t>(cnt - c0, next_step - done);  // up to the step boundary
-            b_dst.push_back(hp + (c0 << t->page_shift));
-            b_src.push_back(t->d.pool + ((size_t)(first + c0) << t->page_shift));
-            b_size.push_back((size_t)cc << t->page_shift);
+        for (uint64_t c0 = 0; c0 < cnt; c0 += chunk_pages) {
+            const uint64_t cc = std::min<uint64_t>(chunk_pages, cnt - c0);
+            CK(t, cudaMemcpyAsync(hp + (c0 << t->page_shift), t->d.pool + ((size_t)(first + c0) << t->page_shift),
+                                  (size_t)cc << t->page_shift, cudaMemcpyDefault, t->copy_stream));
             done += cc;
-            c0 += cc;
-            if (done == next_step) {
-                if ((rc = flush())) return rc;
-                next_step += chunk_pages;
+            if (overlapped) {
+                const int wr = t->write_value32(t->copy_stream, (unsigned long long)(uintptr_t)&t->d.ctrl->copied,
+                                                (unsigned int)done, 0);
+                if (wr) return fail(SEPO_E_CUDA, "cuStreamWriteValue32 failed");
             }
         }
         img.runs.push_back({first, cnt, hp});
         bytes += nbytes;
         i = j;
     }
-    if ((rc = flush())) return rc;
     CK(t, cudaEventRecord(t->ev_copy, t->copy_stream));
     if (overlap) {
         int orc = overlap();

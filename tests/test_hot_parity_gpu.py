@@ -151,10 +151,9 @@ def test_dir_prefetch_path(cuda, monkeypatch, name, scale, ratio):
 
 @pytest.mark.parametrize("name,scale,ratio", [("C4", 1 / 256, 3), ("C4", 1 / 1000, 2), ("C2", 1 / 256, 4), ("C5u", 2 ** -12, 4)])
 def test_evict_overlap_forced(cuda, monkeypatch, name, scale, ratio):
-    """SEPO_EVICT_OVERLAP=1 on tables small enough to skip it by default: every eviction's copies (batched
-    copy-engine copies, progress published per step) overlap the next pass, whose allocator waits per
-    evicted page before reusing it — GROUP (retained key pages between evicted ones) and COMBINE equal
-    the oracle"""
+    """SEPO_EVICT_OVERLAP=1 (off by default for GROUP and for pools inside L2): every eviction's copies
+    overlap the next pass, whose allocator waits per evicted page (progress published by the copy stream)
+    before reusing it — GROUP (retained key pages between evicted ones) and COMBINE equal the oracle"""
     monkeypatch.setenv("SEPO_EVICT_OVERLAP", "1")
     s = gen.config(name, scale)
     inp = device_inputs(s)
