@@ -138,6 +138,7 @@ struct sepo_table {
     std::vector<cudaEvent_t>* h2d_chunks = nullptr;  // sepo_run on host input: copy events of pass-1 chunks
     uint64_t h2d_chunk_records = 0;  // sepo_lookup restored old generations into the pool: no inserts until reset
     DevBuf tbm;      // sepo_run_text: start bits of declined words that did not fit the prepared list
+    DevBuf eprog;    // overlapped gather eviction: per-warp progress of evict_copy_prog_kernel
     // cuStreamWriteValue32 (driver entry point): the copy stream publishes eviction progress
     int (*write_value32)(cudaStream_t, unsigned long long, unsigned int, unsigned int) = nullptr;
 
@@ -224,6 +225,7 @@ int read_ctrl(sepo_table* t) {
 int zero_ctrl_counters(sepo_table* t) {
     // postponed, toolarge, dead_bytes, kept_key_bytes, kept_val_bytes (fields 1..5)
     CK(t, cudaMemsetAsync(&t->d.ctrl->postponed, 0, 5 * sizeof(unsigned long long), t->stream));
+    CK(t, cudaMemsetAsync(&t->d.ctrl->next_group, 0, sizeof(unsigned long long), t->stream));  // (GROUP schedule)
     return 0;
 }
 
@@ -241,6 +243,7 @@ int init_device_state(sepo_table* t) {
     t->st.kernel_launches += 1;
     t->d.n_free = t->n_pages;
     t->d.n_safe = t->n_pages;
+    t->d.eprog = nullptr;
     t->d.gen = 0;
     CK(t, cudaStreamSynchronize(t->stream));
     return 0;
@@ -717,6 +720,11 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
     // the previous eviction's copies (and its writes of ctrl->copied) are done before the reset
     CK(t, cudaStreamWaitEvent(t->stream, t->ev_copy, 0));
     CK(t, cudaMemsetAsync(&t->d.ctrl->copied, 0, sizeof(unsigned int), t->stream));
+    constexpr int kGatherCtas = 16;  // overlapped gather: a few SMs saturate the host link
+    const uint32_t gather_warps = kGatherCtas * 512 / 32;
+    if (t->eprog.grow(gather_warps * 4)) return fail(SEPO_E_NOMEM, "eviction progress");
+    CK(t, cudaMemsetAsync(t->eprog.p, 0, gather_warps * 4, t->stream));
+    t->d.eprog = nullptr;
     if ((rc = read_ctrl(t))) return rc;
     const uint64_t ne = t->h_ctrl->n_evict;
     if (ne) {
@@ -732,9 +740,10 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
     CK(t, cudaStreamWaitEvent(t->copy_stream, t->ev_comp, 0));
     // eviction overlapped with the next pass (the allocator waits per evicted page): measured
     // worth it when a generation is large (C5u 4x job 86 -> 78 ms with a 192 MB pool), not for a
-    // pool inside L2 (C2 4x: 30.5 -> 31.8 ms) nor for GROUP (fragmented evict lists leave through
-    // the gather kernel, which cannot publish progress in evict-list order). SEPO_EVICT_OVERLAP=0/1
-    // forces the choice.
+    // pool inside L2 (C2 4x: 30.5 -> 31.8 ms). Fragmented evict lists (GROUP generations with
+    // retained key pages between the evicted ones) overlap through the gather kernel on a few SMs,
+    // which publishes per-warp progress (one cudaMemcpyAsync per run with progress: C4 3x 496 ->
+    // 708 ms). SEPO_EVICT_OVERLAP=0/1 forces the choice.
     bool want_overlap;
     {
         const char* ov = getenv("SEPO_EVICT_OVERLAP");
@@ -742,29 +751,37 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
         cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, t->device);
         want_overlap = (ov && (ov[0] == '0' || ov[0] == '1'))
                            ? ov[0] == '1'
-                           : t->opts.mode == SEPO_COMBINE_SUM_U64 && (uint64_t)t->n_pages * t->page_bytes > (uint64_t)l2;
+                           : (t->opts.mode == SEPO_COMBINE_SUM_U64 || t->opts.mode == SEPO_GROUP) &&
+                                 (uint64_t)t->n_pages * t->page_bytes > (uint64_t)l2;
     }
-    const bool overlapped = t->write_value32 != nullptr && want_overlap;
+    // Fragmented evict lists (many short runs of consecutive pages) go through one gather-copy
+    // kernel into a contiguous host region; long runs through cudaMemcpyAsync (copy engine).
+    // SEPO_EVICT_KERNEL=0/1 forces either.
+    uint64_t n_runs = 0;
+    for (uint64_t i = 0; i < ne; ++i) n_runs += (i == 0 || t->h_evict[i] != t->h_evict[i - 1] + 1);
+    const char* eks = getenv("SEPO_EVICT_KERNEL");
+    const int ek = eks ? atoi(eks) : -1;
+    const bool use_kernel = ne > 0 && (ek == 1 || (ek < 0 && n_runs * 64 > ne));
+    const bool gather_ov = use_kernel && want_overlap;
+    const bool overlapped = gather_ov || (!use_kernel && t->write_value32 != nullptr && want_overlap);
     GenImage img;
     img.gen = t->d.gen;
     uint64_t bytes = 0, done = 0;
     const uint64_t chunk_pages = overlapped ? std::max<uint64_t>(std::max<uint64_t>(1, (1u << 20) >> t->page_shift), ne / 48)
                                             : ~0ull;  // progress granularity (overlap only)
-    // Fragmented evict lists (many short runs of consecutive pages, e.g. GROUP generations with
-    // retained key pages) go through one gather-copy kernel into a contiguous host region; long
-    // runs through cudaMemcpyAsync (copy engine). SEPO_EVICT_KERNEL=0/1 forces either.
-    uint64_t n_runs = 0;
-    for (uint64_t i = 0; i < ne; ++i) n_runs += (i == 0 || t->h_evict[i] != t->h_evict[i - 1] + 1);
-    const char* eks = getenv("SEPO_EVICT_KERNEL");
-    const int ek = eks ? atoi(eks) : -1;
-    const bool use_kernel = !overlapped && ne > 0 && (ek == 1 || (ek < 0 && n_runs * 64 > ne));
     if (use_kernel) {
         const size_t nbytes = (size_t)ne << t->page_shift;
         uint8_t* hp = arena_alloc(t, nbytes);
         if (!hp) return fail(SEPO_E_NOMEM, "pinned host arena exhausted");
         uint8_t* dp = nullptr;
         CK(t, cudaHostGetDevicePointer((void**)&dp, hp, 0));
-        rc = sepo_launch_evict_copy(t->d, (uint32_t)ne, dp, 2 * t->n_sms, t->copy_stream);
+        if (gather_ov) {
+            rc = sepo_launch_evict_copy_prog(t->d, (uint32_t)ne, dp, kGatherCtas, (unsigned int*)t->eprog.p, t->copy_stream);
+            t->d.eprog = (unsigned int*)t->eprog.p;  // (the next pass's allocator waits on it)
+            t->d.eprog_n = gather_warps;
+        } else {
+            rc = sepo_launch_evict_copy(t->d, (uint32_t)ne, dp, 2 * t->n_sms, t->copy_stream);
+        }
         if (rc) return cuda_check(t, (cudaError_t)rc, "evict copy kernel");
         t->st.kernel_launches += 1;
         for (uint64_t i = 0; i < ne;) {

@@ -60,7 +60,8 @@ struct Ctrl {
     unsigned int copied;               // evicted pages whose D2H copy finished (written by the copy stream)
     unsigned int failed_slots;         // BASIC: allocator slots whose allocation failed this generation
     unsigned long long text_words;     // sepo_run_text: words tokenized by the last insert call
-    unsigned long long pad[3];
+    unsigned long long next_group;     // GROUP insert: next 32-record group to hand out (dynamic schedule)
+    unsigned long long pad[2];
 };
 
 struct Dev {
@@ -88,6 +89,11 @@ struct Dev {
     uint32_t gen;             // generation (= pass index) of resident data
     uint32_t fail_ppm, fail_mode, fail_until;
     uint32_t batch_seq;
+    // Overlapped eviction through the gather kernel (GROUP): warp w of the kernel copies evict-list
+    // positions w, w + eprog_n, ... in order and publishes how many it finished in eprog[w], so
+    // position j is copied once eprog[j % eprog_n] > j / eprog_n. nullptr: progress is ctrl->copied.
+    unsigned int* eprog;
+    uint32_t eprog_n;
 };
 
 // ---------------------------------------------------------------- memory access helpers
@@ -525,10 +531,12 @@ __device__ __forceinline__ uint64_t warp_alloc(const Dev& d, unsigned long long*
                     unsigned long long nw;
                     if (q < d.n_free) {
                         if (q >= d.n_safe) {  // an evicted page: wait until its copy to the host is done
-                            const unsigned int need_copied = (unsigned int)(q - d.n_safe) + 1u;
+                            const uint32_t jpos = (uint32_t)(q - d.n_safe);
+                            const unsigned int* pw = d.eprog ? d.eprog + jpos % d.eprog_n : &d.ctrl->copied;
+                            const unsigned int need_copied = d.eprog ? jpos / d.eprog_n + 1u : jpos + 1u;
                             while (true) {
                                 unsigned int cp;
-                                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(cp) : "l"(&d.ctrl->copied) : "memory");
+                                asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(cp) : "l"(pw) : "memory");
                                 if (cp >= need_copied) break;
                                 __nanosleep(256);
                             }

@@ -1604,12 +1604,22 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
     const bool inj = d.fail_ppm != 0 && d.gen < d.fail_until;
     const uint32_t pc_bytes = chunk_bytes(PC_CAP, vw);
 
+    // groups are handed out GS at a time from a global counter (zeroed by the host before the launch):
+    // a CTA that starts late — its SM still busy with an overlapped eviction's gather — takes less work
     const uint64_t ngroups = (b.n + 31) / 32;
-    const uint64_t gw = (uint64_t)blockIdx.x * (THREADS / 32) + (tid >> 5);
-    const uint64_t nw = (uint64_t)gridDim.x * (THREADS / 32);
+    constexpr uint64_t GS = 16;
     unsigned long long c_post = 0, c_tl = 0, c_dead = 0, c_pkb = 0;
     bool w_full = false, w_quiet = false;
-    for (uint64_t g = gw; g < ngroups; g += nw) {
+    uint64_t g_lim = 0;
+    auto next_g = [&](uint64_t cur) -> uint64_t {
+        if (cur + 1 < g_lim) return cur + 1;
+        unsigned long long x = 0;
+        if (lane == 0) x = atomicAdd(&d.ctrl->next_group, (unsigned long long)GS);
+        x = __shfl_sync(FULLMASK, x, 0);
+        g_lim = min((uint64_t)x + GS, ngroups);
+        return x;
+    };
+    for (uint64_t g = next_g(~0ull); g < ngroups; g = next_g(g)) {
         const uint64_t i = g * 32 + lane;
         const bool valid = i < b.n;
         uint64_t s, w0, w1;
@@ -3305,6 +3315,31 @@ __global__ void __launch_bounds__(512) evict_copy_kernel(const uint8_t* __restri
     }
 }
 
+// The same gather, overlapped with the next pass (GROUP): warp w copies positions w, w + W, ... in
+// order and after each page publishes its count in eprog[w] (release, after __syncwarp: every lane's
+// loads of the page are done), so the allocator can reuse a page as soon as its own warp copied it.
+__global__ void __launch_bounds__(512) evict_copy_prog_kernel(const uint8_t* __restrict__ pool, const uint32_t* __restrict__ list,
+                                                           uint32_t n, uint8_t* __restrict__ dst, uint32_t page_shift,
+                                                           unsigned int* eprog) {
+    const uint32_t lane = lane_id();
+    const uint32_t W = gridDim.x * (blockDim.x / 32), w = blockIdx.x * (blockDim.x / 32) + (threadIdx.x >> 5);
+    const uint32_t per_page = (1u << page_shift) / 16;
+    unsigned int done = 0;
+    for (uint64_t k = w; k < n; k += W) {
+        const uint4* src = reinterpret_cast<const uint4*>(pool + ((uint64_t)list[k] << page_shift));
+        uint4* out = reinterpret_cast<uint4*>(dst + (k << page_shift));
+        uint32_t u = lane;
+        for (; u + 96 < per_page; u += 128) {
+            const uint4 a = __ldcg(src + u), b = __ldcg(src + u + 32), c = __ldcg(src + u + 64), e = __ldcg(src + u + 96);
+            __stcs(out + u, a); __stcs(out + u + 32, b); __stcs(out + u + 64, c); __stcs(out + u + 96, e);
+        }
+        for (; u < per_page; u += 32) __stcs(out + u, __ldcg(src + u));
+        __syncwarp();
+        ++done;
+        if (lane == 0) asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(eprog + w), "r"(done) : "memory");
+    }
+}
+
 }  // namespace sepo
 
 // ================================================================ launchers
@@ -3374,6 +3409,10 @@ int sepo_launch_text_bits(const Dev& d, const Batch& b, unsigned long long* coun
     return cudaGetLastError();
 }
 
+int sepo_launch_evict_copy_prog(const Dev& d, uint32_t n, uint8_t* dst, int grid, unsigned int* eprog, cudaStream_t s) {
+    if (n) evict_copy_prog_kernel<<<grid, 512, 0, s>>>(d.pool, d.evict_list, n, dst, d.page_shift, eprog);
+    return cudaGetLastError();
+}
 int sepo_launch_evict_copy(const Dev& d, uint32_t n, uint8_t* dst, int grid, cudaStream_t s) {
     if (n) evict_copy_kernel<<<grid, 512, 0, s>>>(d.pool, d.evict_list, n, dst, d.page_shift);
     return cudaGetLastError();
