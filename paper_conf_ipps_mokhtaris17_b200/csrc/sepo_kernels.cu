@@ -2179,6 +2179,35 @@ __device__ __forceinline__ void pt_reserve(unsigned long long* cur, bool valid, 
     rank = (uint32_t)__popc(gm & lt);
     boff = pre;
 }
+// Key bytes [src, src + len) -> [dst, dst + len) at any alignment: byte stores up to dst's first 8-byte
+// boundary, then aligned 8-byte stores each assembled from the two aligned source words that hold it
+// (funnel shift), then the last bytes. A lane only writes bytes of its own record, so neighbouring
+// records (adjacent within a part) never overlap a wide store. (URLs of ~74 bytes: ~17 stores instead
+// of 74 byte stores.)
+__device__ __forceinline__ void copy_key_bytes(uint8_t* dst, const uint8_t* src, uint32_t len) {
+    uint32_t x = min(len, (uint32_t)((8u - (reinterpret_cast<uintptr_t>(dst) & 7u)) & 7u));
+    for (uint32_t y = 0; y < x; ++y) dst[y] = (uint8_t)ld_in8(src + y);
+    const uint32_t nfull = (len - x) / 8;  // whole 8-byte words of dst from dst + x (8-aligned)
+    if (nfull) {
+        const uintptr_t sa = reinterpret_cast<uintptr_t>(src + x);
+        const uint32_t sh = (uint32_t)(sa & 7u) * 8u;
+        const uint64_t* sw = reinterpret_cast<const uint64_t*>(sa & ~(uintptr_t)7);
+        uint64_t* dw = reinterpret_cast<uint64_t*>(dst + x);
+        if (sh == 0) {
+            for (uint32_t k = 0; k < nfull; ++k) dw[k] = ld_in64(sw + k);
+        } else {  // (every aligned source word read holds a key byte)
+            uint64_t lo = ld_in64(sw);
+            for (uint32_t k = 0; k < nfull; ++k) {
+                const uint64_t hi = ld_in64(sw + k + 1);
+                dw[k] = (lo >> sh) | (hi << (64u - sh));
+                lo = hi;
+            }
+        }
+        x += 8 * nfull;
+    }
+    for (; x < len; ++x) dst[x] = (uint8_t)ld_in8(src + x);
+}
+
 __global__ void __launch_bounds__(PT_THREADS) part_count_kernel(Batch b, uint32_t P, uint64_t seed,
                                                                 unsigned long long* counts, uint64_t ntiles) {
     __shared__ unsigned long long cur[PT_MAXP];
@@ -2227,11 +2256,7 @@ __global__ void __launch_bounds__(PT_THREADS) part_scatter_kernel(Batch b, uint3
             const uint64_t orec = bp[0] + (r >> 32) + rank;
             const uint64_t obyte = bp[1] + (r & 0xffffffffull) + boff;
             if (oko) oko[orec] = obyte - b0[1];  // rebased to the part's segment
-            // the first 16 key bytes come from registers (loaded for the hash), the rest from input
-            uint8_t* dst = ok + obyte;
-            const uint32_t head = min(len, 16u);
-            for (uint32_t x = 0; x < head; ++x) dst[x] = (uint8_t)((x < 8 ? kw0 >> (8 * x) : kw1 >> (8 * (x - 8))) & 0xffu);
-            for (uint32_t x = 16; x < len; ++x) dst[x] = (uint8_t)ld_in8(b.keys + src + x);
+            copy_key_bytes(ok + obyte, b.keys + src, len);
             if (b.vals) {
                 const uint64_t vs = rec_index(b, i) * (uint64_t)b.vw;
                 uint8_t* vd = ov + orec * b.vw;
