@@ -2015,6 +2015,35 @@ __global__ void __launch_bounds__(1024) scan_tiles_kernel(unsigned long long* tc
     }
 }
 
+// Key bytes [src, src + len) -> [dst, dst + len) at any alignment: byte stores up to dst's first 8-byte
+// boundary, then aligned 8-byte stores each assembled from the two aligned source words that hold it
+// (funnel shift), then the last bytes. A lane only writes bytes of its own record, so neighbouring
+// records (adjacent within a part) never overlap a wide store. (URLs of ~74 bytes: ~17 stores instead
+// of 74 byte stores.)
+__device__ __forceinline__ void copy_key_bytes(uint8_t* dst, const uint8_t* src, uint32_t len) {
+    uint32_t x = min(len, (uint32_t)((8u - (reinterpret_cast<uintptr_t>(dst) & 7u)) & 7u));
+    for (uint32_t y = 0; y < x; ++y) dst[y] = (uint8_t)ld_in8(src + y);
+    const uint32_t nfull = (len - x) / 8;  // whole 8-byte words of dst from dst + x (8-aligned)
+    if (nfull) {
+        const uintptr_t sa = reinterpret_cast<uintptr_t>(src + x);
+        const uint32_t sh = (uint32_t)(sa & 7u) * 8u;
+        const uint64_t* sw = reinterpret_cast<const uint64_t*>(sa & ~(uintptr_t)7);
+        uint64_t* dw = reinterpret_cast<uint64_t*>(dst + x);
+        if (sh == 0) {
+            for (uint32_t k = 0; k < nfull; ++k) dw[k] = ld_in64(sw + k);
+        } else {  // (every aligned source word read holds a key byte)
+            uint64_t lo = ld_in64(sw);
+            for (uint32_t k = 0; k < nfull; ++k) {
+                const uint64_t hi = ld_in64(sw + k + 1);
+                dw[k] = (lo >> sh) | (hi << (64u - sh));
+                lo = hi;
+            }
+        }
+        x += 8 * nfull;
+    }
+    for (; x < len; ++x) dst[x] = (uint8_t)ld_in8(src + x);
+}
+
 // gather: per tile, block scan of (kept, key bytes, value bytes) then copy
 constexpr int CP_THREADS = 256;
 __global__ void __launch_bounds__(CP_THREADS) compact_kernel(Batch b, const unsigned long long* tile_base, uint8_t* ok,
@@ -2062,7 +2091,7 @@ __global__ void __launch_bounds__(CP_THREADS) compact_kernel(Batch b, const unsi
             uint64_t s; uint32_t len;
             rec_key(b, i, s, len);
             if (b.ko) oko[pos[0]] = pos[1];
-            for (uint32_t x = 0; x < len; ++x) ok[pos[1] + x] = __ldg(b.keys + s + x);
+            copy_key_bytes(ok + pos[1], b.keys + s, len);
             if (b.vals) {
                 uint64_t vs; uint32_t vl;
                 if (b.vo) { rec_val_span(b, i, vs, vl); ovo[pos[0]] = pos[2]; }
@@ -2179,35 +2208,6 @@ __device__ __forceinline__ void pt_reserve(unsigned long long* cur, bool valid, 
     rank = (uint32_t)__popc(gm & lt);
     boff = pre;
 }
-// Key bytes [src, src + len) -> [dst, dst + len) at any alignment: byte stores up to dst's first 8-byte
-// boundary, then aligned 8-byte stores each assembled from the two aligned source words that hold it
-// (funnel shift), then the last bytes. A lane only writes bytes of its own record, so neighbouring
-// records (adjacent within a part) never overlap a wide store. (URLs of ~74 bytes: ~17 stores instead
-// of 74 byte stores.)
-__device__ __forceinline__ void copy_key_bytes(uint8_t* dst, const uint8_t* src, uint32_t len) {
-    uint32_t x = min(len, (uint32_t)((8u - (reinterpret_cast<uintptr_t>(dst) & 7u)) & 7u));
-    for (uint32_t y = 0; y < x; ++y) dst[y] = (uint8_t)ld_in8(src + y);
-    const uint32_t nfull = (len - x) / 8;  // whole 8-byte words of dst from dst + x (8-aligned)
-    if (nfull) {
-        const uintptr_t sa = reinterpret_cast<uintptr_t>(src + x);
-        const uint32_t sh = (uint32_t)(sa & 7u) * 8u;
-        const uint64_t* sw = reinterpret_cast<const uint64_t*>(sa & ~(uintptr_t)7);
-        uint64_t* dw = reinterpret_cast<uint64_t*>(dst + x);
-        if (sh == 0) {
-            for (uint32_t k = 0; k < nfull; ++k) dw[k] = ld_in64(sw + k);
-        } else {  // (every aligned source word read holds a key byte)
-            uint64_t lo = ld_in64(sw);
-            for (uint32_t k = 0; k < nfull; ++k) {
-                const uint64_t hi = ld_in64(sw + k + 1);
-                dw[k] = (lo >> sh) | (hi << (64u - sh));
-                lo = hi;
-            }
-        }
-        x += 8 * nfull;
-    }
-    for (; x < len; ++x) dst[x] = (uint8_t)ld_in8(src + x);
-}
-
 __global__ void __launch_bounds__(PT_THREADS) part_count_kernel(Batch b, uint32_t P, uint64_t seed,
                                                                 unsigned long long* counts, uint64_t ntiles) {
     __shared__ unsigned long long cur[PT_MAXP];

@@ -352,3 +352,22 @@ def test_host_input_pipelined(cuda, monkeypatch, ratio):
     assert_same(got, exp)
     assert st["records_inserted"] >= s.n and st["cross_gen_dups"] == 0
     assert (passes == 1) if ratio < 1 else (passes >= 2)
+
+
+def test_compact_long_keys(cuda):
+    """sepo_compact on URL keys (28-256 bytes: the copy's aligned 8-byte middle, byte head and tail at
+    every alignment) equals the oracle's compaction byte for byte"""
+    s = gen.config("C3", scale=1 / 8000)
+    hk, ho, _ = s.host()
+    k, o, _ = s.device()
+    n = s.n
+    t = sepo().Table(sepo().budget_for(1 << 12, 65536, 6), 1 << 12, 65536)
+    c, bm = t.insert_batch(k, o, n=n)
+    rem, kbytes, _ = t.reprobe(k, o, None, bm, n=n)
+    assert rem > 0
+    ok, oko, _, m = t.compact(k, o, None, bm, n=n)
+    ek, eo, _, _, em = oracle.compact(hk, np.asarray(ho).view(np.uint64), bm.cpu().numpy().view(np.uint32))
+    assert m == em == rem and int(oko[-1]) == kbytes
+    assert ok.cpu().numpy().tobytes() == ek.tobytes()
+    assert (oko.cpu().numpy().view(np.uint64) == eo).all()
+    t.close()
