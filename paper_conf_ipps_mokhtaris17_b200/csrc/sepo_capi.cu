@@ -139,6 +139,8 @@ struct sepo_table {
     uint64_t h2d_chunk_records = 0;  // sepo_lookup restored old generations into the pool: no inserts until reset
     DevBuf tbm;      // sepo_run_text: start bits of declined words that did not fit the prepared list
     DevBuf eprog;    // overlapped gather eviction: per-warp progress of evict_copy_prog_kernel
+    DevBuf evl;      // overlapped gather eviction: its own copy of the evict list (the next eviction's
+                     // classify rewrites d.evict_list while the gather may still be reading it)
     // cuStreamWriteValue32 (driver entry point): the copy stream publishes eviction progress
     int (*write_value32)(cudaStream_t, unsigned long long, unsigned int, unsigned int) = nullptr;
 
@@ -736,6 +738,11 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
     // evict-list order) in ctrl->copied after every chunk and the next pass starts at once: its
     // allocator takes the never-used pages first and waits for an evicted page's copy before
     // reusing it ("pages are copied to CPU memory" — overlapped with the next pass).
+    if (ne) {  // the gather kernel's own copy of the list, taken in stream order before the next
+               // eviction's classify can rewrite d.evict_list (an overlapped gather may outlive a short pass)
+        if (t->evl.grow(ne * 4)) return fail(SEPO_E_NOMEM, "evict list copy");
+        CK(t, cudaMemcpyAsync(t->evl.p, t->d.evict_list, ne * 4, cudaMemcpyDeviceToDevice, t->stream));
+    }
     CK(t, cudaEventRecord(t->ev_comp, t->stream));
     CK(t, cudaStreamWaitEvent(t->copy_stream, t->ev_comp, 0));
     // eviction overlapped with the next pass (the allocator waits per evicted page): measured
@@ -776,7 +783,8 @@ static int64_t evict_impl(sepo_table* t, int honor_retain, const std::function<i
         uint8_t* dp = nullptr;
         CK(t, cudaHostGetDevicePointer((void**)&dp, hp, 0));
         if (gather_ov) {
-            rc = sepo_launch_evict_copy_prog(t->d, (uint32_t)ne, dp, kGatherCtas, (unsigned int*)t->eprog.p, t->copy_stream);
+            rc = sepo_launch_evict_copy_prog(t->d, (uint32_t)ne, dp, kGatherCtas, (unsigned int*)t->eprog.p,
+                                             (const uint32_t*)t->evl.p, t->copy_stream);
             t->d.eprog = (unsigned int*)t->eprog.p;  // (the next pass's allocator waits on it)
             t->d.eprog_n = gather_warps;
         } else {
@@ -1692,6 +1700,8 @@ void sepo_destroy(sepo_table* t) {
     t->prep[1].release();
     t->prep_n.release();
     t->tbm.release();
+    t->eprog.release();
+    t->evl.release();
     t->lk_pages.release();
     t->bm.release();
     for (int i = 0; i < 3; ++i) { t->sh_send[i].release(); t->sh_held[i].release(); t->sh_tmp[i].release(); }

@@ -3434,8 +3434,9 @@ int sepo_launch_text_bits(const Dev& d, const Batch& b, unsigned long long* coun
     return cudaGetLastError();
 }
 
-int sepo_launch_evict_copy_prog(const Dev& d, uint32_t n, uint8_t* dst, int grid, unsigned int* eprog, cudaStream_t s) {
-    if (n) evict_copy_prog_kernel<<<grid, 512, 0, s>>>(d.pool, d.evict_list, n, dst, d.page_shift, eprog);
+int sepo_launch_evict_copy_prog(const Dev& d, uint32_t n, uint8_t* dst, int grid, unsigned int* eprog,
+                                const uint32_t* list, cudaStream_t s) {
+    if (n) evict_copy_prog_kernel<<<grid, 512, 0, s>>>(d.pool, list, n, dst, d.page_shift, eprog);
     return cudaGetLastError();
 }
 int sepo_launch_evict_copy(const Dev& d, uint32_t n, uint8_t* dst, int grid, cudaStream_t s) {

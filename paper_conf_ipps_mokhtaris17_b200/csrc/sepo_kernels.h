@@ -95,7 +95,10 @@ int sepo_launch_shift_offsets(uint64_t* ko, uint64_t n, const uint64_t* seg_rec,
                               uint64_t total, cudaStream_t s);
 int sepo_launch_seal(const sepo::Dev& d, uint32_t n_slots, cudaStream_t s);
 int sepo_launch_evict_copy(const sepo::Dev& d, uint32_t n, uint8_t* dst, int grid, cudaStream_t s);
-int sepo_launch_evict_copy_prog(const sepo::Dev& d, uint32_t n, uint8_t* dst, int grid, unsigned int* eprog, cudaStream_t s);
+// (list: a snapshot of the evict list — the overlapped gather may still run when the next eviction's
+// classify rewrites d.evict_list)
+int sepo_launch_evict_copy_prog(const sepo::Dev& d, uint32_t n, uint8_t* dst, int grid, unsigned int* eprog,
+                                const uint32_t* list, cudaStream_t s);
 // sample_bytes: tokenize a hot-set sample from the first sample_bytes of the text; 0: reuse the hot
 // set an earlier launch of the same job built, if *hot_built says it did (else no hot set).
 // *hot_built (in/out, host): set when this launch builds a hot set, cleared when it samples none.

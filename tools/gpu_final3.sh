@@ -6,7 +6,5 @@ timeout 1800 python -m pytest -x -q -p no:cacheprovider tests -m gpu > gpurun_ou
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke_$TAG.log 2>&1
 timeout 900 python bench.py > gpurun_out/bench_$TAG.log 2>&1
 tail -1 gpurun_out/bench_$TAG.log > gpurun_out/bench_$TAG.json
-timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/ref_$TAG.log 2>&1
-tail -1 gpurun_out/ref_$TAG.log > gpurun_out/ref_$TAG.json
-for c in C4 C5u C3; do timeout 600 python tools/time_job.py $c $( [ $c = C4 ] && echo 3 || echo 4 ) $( [ $c = C5u ] && echo 0.125 ) > gpurun_out/cfg_${TAG}_$c.json 2>&1; done
+echo skip-configs
 echo done
