@@ -1607,7 +1607,10 @@ __global__ void __launch_bounds__(gst::THREADS, 1) insert_group_stream_kernel(De
     // groups are handed out GS at a time from a global counter (zeroed by the host before the launch):
     // a CTA that starts late — its SM still busy with an overlapped eviction's gather — takes less work
     const uint64_t ngroups = (b.n + 31) / 32;
-    constexpr uint64_t GS = 16;
+#ifndef SEPO_GROUP_GS
+#define SEPO_GROUP_GS 16
+#endif
+    constexpr uint64_t GS = SEPO_GROUP_GS;  // groups per grab
     unsigned long long c_post = 0, c_tl = 0, c_dead = 0, c_pkb = 0;
     bool w_full = false, w_quiet = false;
     uint64_t g_lim = 0;
