@@ -1,6 +1,7 @@
 """Round-2 paths at small sizes with forced options (compute-sanitizer is closed on this GPU pool, so this
 runs them plainly and checks parity): the hot-key router (hot set forced on a small batch), the CSR
-gather eviction, and sepo_run_sharded on a one-rank NCCL communicator (peer-memory window and CSR).
+partition's aligned key copy, sepo_compact on URL keys, GROUP with the overlapped gather eviction, and
+sepo_run_sharded on a one-rank NCCL communicator (peer-memory window and CSR).
 Exits non-zero on a parity failure."""
 import os
 import sys
